@@ -1,0 +1,211 @@
+"""Seeded synthetic inputs shared by the tests, the bench and the oracle tests.
+
+This module holds NONE of the method's arithmetic: it generates graphs,
+labels, update streams and query patterns shaped like the paper's workloads
+(Table I, stream protocol P:331, query sizes P:331) and the
+concrete configurations of SURVEY.md §8d / BASELINE.json ``configs``.
+Neither the product (``paper_conf_ipps_wei024_b200``) nor ``oracle`` is
+imported here, and both may import this module.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, field
+
+import numpy as np
+
+from ._build import build as _build_lib, LIB_PATH
+
+_lib = None
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            _build_lib()
+        lib = ctypes.CDLL(LIB_PATH)
+        P = ctypes.c_void_p
+        lib.gi_rmat_edges.restype = ctypes.c_int64
+        lib.gi_rmat_edges.argtypes = [ctypes.c_int32, ctypes.c_int64, ctypes.c_double, ctypes.c_double,
+                                      ctypes.c_double, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int32, P]
+        lib.gi_build_csr.restype = ctypes.c_int32
+        lib.gi_build_csr.argtypes = [ctypes.c_int32, ctypes.c_int64, P, ctypes.c_int32, P, P]
+        lib.gi_labels.restype = None
+        lib.gi_labels.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_uint64, P]
+        lib.gi_stream.restype = ctypes.c_int64
+        lib.gi_stream.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_uint64, P, P]
+        _lib = lib
+    return _lib
+
+
+def _p(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _threads() -> int:
+    return int(os.environ.get("GCSM_GEN_THREADS", "0"))
+
+
+# ---------------------------------------------------------------- graphs
+
+def rmat_edges(scale: int, n_edges: int, a: float, b: float, c: float, seed: int,
+               id_limit: int = 0) -> np.ndarray:
+    """Exactly ``n_edges`` unique undirected R-MAT edges as an int32 [m,2] array (u<v)."""
+    out = np.empty((n_edges, 2), dtype=np.int32)
+    r = _load().gi_rmat_edges(scale, n_edges, a, b, c, seed & (2**64 - 1), id_limit, _threads(), _p(out))
+    if r != n_edges:
+        raise ValueError("R-MAT id space too small for the requested edge count")
+    return out
+
+
+def csr_from_edges(n: int, uv: np.ndarray):
+    """Symmetric CSR (row_ptr int64[n+1], col int32[2m]) with sorted rows."""
+    uv = np.ascontiguousarray(uv, dtype=np.int32).reshape(-1, 2)
+    rp = np.empty(n + 1, dtype=np.int64)
+    col = np.empty(2 * len(uv), dtype=np.int32)
+    if _load().gi_build_csr(n, len(uv), _p(uv), _threads(), _p(rp), _p(col)) != 0:
+        raise ValueError("bad edge list (out of range or self loop)")
+    return rp, col
+
+
+def labels(n: int, L: int, seed: int) -> np.ndarray:
+    out = np.empty(n, dtype=np.int32)
+    _load().gi_labels(n, L, seed & (2**64 - 1), _p(out))
+    return out
+
+
+def stream(m: int, n_sample: int, seed: int):
+    """indices of n_sample distinct edges in random order and their signs (+1 ins / -1 del)."""
+    sel = np.empty(n_sample, dtype=np.int64)
+    sign = np.empty(n_sample, dtype=np.int8)
+    if _load().gi_stream(m, n_sample, seed & (2**64 - 1), _p(sel), _p(sign)) != n_sample:
+        raise ValueError("sample larger than the edge set")
+    return sel, sign
+
+
+def random_graph(n: int, p: float, seed: int) -> np.ndarray:
+    """Small Erdos-Renyi G(n,p) edge list (u<v) for fuzz tests (numpy RNG, seeded)."""
+    rng = np.random.default_rng(seed)
+    iu, ju = np.triu_indices(n, 1)
+    keep = rng.random(len(iu)) < p
+    return np.stack([iu[keep], ju[keep]], axis=1).astype(np.int32)
+
+
+# ---------------------------------------------------------------- queries
+# Query patterns: (k, edge list over [0,k), labels or None). Sizes follow the
+# paper's 3..7-vertex patterns; the exact Fig. 7 shapes are lost
+# (image), so this catalogue is SURVEY §8d's.
+QUERIES = {
+    "edge": (2, [(0, 1)], None),
+    "wedge": (3, [(0, 1), (0, 2)], None),
+    "triangle": (3, [(0, 1), (0, 2), (1, 2)], None),
+    "star3": (4, [(0, 1), (0, 2), (0, 3)], None),
+    "path4": (4, [(0, 1), (1, 2), (2, 3)], None),
+    "c4": (4, [(0, 1), (1, 2), (2, 3), (0, 3)], None),
+    "diamond": (4, [(0, 1), (0, 2), (1, 2), (1, 3), (2, 3)], None),  # Fig. 1 Q
+    "k4": (4, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)], None),
+    "house5": (5, [(0, 1), (1, 2), (2, 3), (0, 3), (0, 4), (1, 4)], [0, 0, 1, 1, 2]),
+    "bowtie5": (5, [(0, 1), (0, 2), (1, 2), (0, 3), (0, 4), (3, 4)], [0, 1, 1, 2, 2]),
+    "k5e": (5, [(i, j) for i in range(5) for j in range(i + 1, 5) if (i, j) != (3, 4)], [0, 1, 2, 3, 3]),
+    "house5u": (5, [(0, 1), (1, 2), (2, 3), (0, 3), (0, 4), (1, 4)], None),
+    "k5": (5, [(i, j) for i in range(5) for j in range(i + 1, 5)], None),
+    "prism6": (6, [(0, 1), (0, 2), (1, 2), (3, 4), (3, 5), (4, 5), (0, 3), (1, 4), (2, 5)], None),
+    "k4tri6": (6, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3), (0, 4), (1, 4), (2, 5), (3, 5)], None),
+    "k6": (6, [(i, j) for i in range(6) for j in range(i + 1, 6)], None),
+}
+
+
+def query(name: str):
+    k, edges, lab = QUERIES[name]
+    qe = np.asarray(edges, dtype=np.int32).reshape(-1, 2)
+    ql = None if lab is None else np.asarray(lab, dtype=np.int32)
+    return k, qe, ql
+
+
+# ---------------------------------------------------------------- workloads
+
+@dataclass
+class Workload:
+    name: str
+    n: int
+    row_ptr: np.ndarray            # G_0 CSR
+    col: np.ndarray
+    labels: np.ndarray | None
+    queries: list
+    batches: list                  # [(ins int32[k,2], dele int32[k,2])]
+    budget_frac: float
+    meta: dict = field(default_factory=dict)
+
+    @property
+    def adj_bytes(self) -> int:
+        return 4 * int(self.row_ptr[-1])
+
+
+# SURVEY §8d configs. seed = 0x6C53 + config index.
+CONFIGS = {
+    "C1": dict(scale=10, n_edges=8192, abc=(0.57, 0.19, 0.19), id_limit=0, L=0,
+               queries=["triangle"], stream=256, batch=256, inserts_only=True, budget=1.0),
+    "C2": dict(scale=22, n_edges=70_000_000, abc=(0.50, 0.166, 0.166), id_limit=0, L=0,
+               queries=["k4", "c4"], stream=12 * 8192, batch=4096, inserts_only=False, budget=0.10),
+    "C3": dict(scale=22, n_edges=120_000_000, abc=(0.502, 0.166, 0.166), id_limit=3_000_000, L=8,
+               queries=["house5", "bowtie5", "k5e"], stream=12 * 8192, batch=4096, inserts_only=False,
+               budget=0.10),
+}
+
+
+def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = None,
+                  batch: int | None = None, n_batches: int | None = None) -> Workload:
+    """Build G_0 and the batch stream of a config (optionally scaled down for tests)."""
+    cfg = dict(CONFIGS[name])
+    idx = int(name[1:])
+    seed = 0x6C53 + idx
+    if scale is not None:
+        cfg["scale"] = scale
+        if cfg["id_limit"]:
+            cfg["id_limit"] = min(cfg["id_limit"], (1 << scale) * 3 // 4)
+    if n_edges is not None:
+        cfg["n_edges"] = n_edges
+    if batch is not None:
+        cfg["batch"] = batch
+    a, b, c = cfg["abc"]
+    uv = rmat_edges(cfg["scale"], cfg["n_edges"], a, b, c, seed, cfg["id_limit"])
+    n = cfg["id_limit"] if cfg["id_limit"] else (1 << cfg["scale"])
+    n_stream = min(cfg["stream"], len(uv) // 2)
+    sel, sign = stream(len(uv), n_stream, seed + 1000)
+    if cfg["inserts_only"]:
+        sign[:] = 1
+    ins_mask = np.zeros(len(uv), dtype=bool)
+    ins_mask[sel[sign > 0]] = True
+    g0 = uv[~ins_mask]
+    rp, col = csr_from_edges(n, g0)
+    lab = labels(n, cfg["L"], seed + 2000) if cfg["L"] else None
+    B = cfg["batch"]
+    nb = n_stream // B
+    if n_batches is not None:
+        nb = min(nb, n_batches)
+    batches = []
+    for t in range(nb):
+        s = sel[t * B:(t + 1) * B]
+        g = sign[t * B:(t + 1) * B]
+        batches.append((np.ascontiguousarray(uv[s[g > 0]]), np.ascontiguousarray(uv[s[g < 0]])))
+    return Workload(name=name, n=n, row_ptr=rp, col=col, labels=lab, queries=list(cfg["queries"]),
+                    batches=batches, budget_frac=cfg["budget"],
+                    meta=dict(seed=seed, scale=cfg["scale"], n_edges=cfg["n_edges"], abc=cfg["abc"],
+                              id_limit=cfg["id_limit"], L=cfg["L"], batch=B))
+
+
+def small_random_case(seed: int, n: int = 9, p: float = 0.45, n_ins: int = 4, n_del: int = 4):
+    """Tiny random graph + one mixed batch (valid by construction) for brute-force fuzzing."""
+    rng = np.random.default_rng(seed)
+    full = random_graph(n, p, seed)
+    if len(full) == 0:
+        full = np.array([[0, 1]], dtype=np.int32)
+    perm = rng.permutation(len(full))
+    ni = min(n_ins, len(full) // 2)
+    nd = min(n_del, len(full) - ni)
+    ins = full[perm[:ni]]
+    dele = full[perm[ni:ni + nd]]
+    g0 = full[np.sort(perm[ni:])]
+    return n, g0, ins, dele

@@ -1,0 +1,189 @@
+// gcsm_inputs/gen.cpp — seeded synthetic input generators.
+//
+// Shared by the product tests/bench AND the oracle tests: this module holds
+// none of the method's arithmetic (no matching, no estimator, no caching).
+// It only produces inputs shaped like the paper's workloads:
+//   * R-MAT graphs (recursive-matrix edge sampler), symmetrised, loop-free,
+//     deduplicated, vertex ids permuted with a seeded permutation
+//     (SURVEY §8d "Configs as concrete synthetic inputs");
+//   * vertex labels uniform over L values;
+//   * the update-stream protocol of PAPER.md P:331 (sample edges uniformly
+//     without replacement, mark each + or - with p = 1/2; G_0 drops the
+//     insertion-marked edges).
+// Every random draw is a pure function of (seed, counter) through splitmix64,
+// so the output is identical for any thread count and on any host.
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <numeric>
+#include <unordered_map>
+#include <vector>
+#include <parallel/algorithm>
+#include <omp.h>
+
+namespace {
+
+inline uint64_t sm64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ULL;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+inline uint64_t h2(uint64_t a, uint64_t b) { return sm64(a ^ sm64(b)); }
+inline double u01(uint64_t x) { return (double)(x >> 11) * (1.0 / 9007199254740992.0); }
+
+struct Cand {
+  uint64_t key;  // (u << 32) | v with u < v
+  int64_t idx;   // generation index (earlier wins)
+};
+
+// One R-MAT draw for candidate index j. Returns false for self loops / rejected ids.
+inline bool rmat_one(int scale, double a, double b, double c, uint64_t seed, int64_t j,
+                     int64_t id_limit, uint64_t* key) {
+  uint64_t u = 0, v = 0;
+  const uint64_t base = h2(seed, (uint64_t)j);
+  for (int l = 0; l < scale; ++l) {
+    const double r = u01(h2(base, (uint64_t)l + 1));
+    u <<= 1;
+    v <<= 1;
+    if (r < a) {
+    } else if (r < a + b) {
+      v |= 1;
+    } else if (r < a + b + c) {
+      u |= 1;
+    } else {
+      u |= 1;
+      v |= 1;
+    }
+  }
+  if (u == v) return false;
+  if (id_limit > 0 && ((int64_t)u >= id_limit || (int64_t)v >= id_limit)) return false;
+  if (u > v) std::swap(u, v);
+  *key = (u << 32) | v;
+  return true;
+}
+
+}  // namespace
+
+extern "C" {
+
+// Exactly n_edges unique undirected edges of an R-MAT(scale; a,b,c,d=1-a-b-c)
+// graph: candidates are drawn in index order, the first n_edges distinct
+// non-loop pairs (by generation index) are kept, then the vertex ids are
+// relabelled with a seeded uniform permutation of [0, n_ids) where
+// n_ids = id_limit > 0 ? id_limit : 2^scale. Output pairs (u<v) in generation
+// order. Returns n_edges, or -1 if the id space cannot hold that many edges.
+int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double c,
+                      uint64_t seed, int64_t id_limit, int32_t threads, int32_t* out_uv) {
+  if (threads > 0) omp_set_num_threads(threads);
+  const int64_t n_ids = id_limit > 0 ? id_limit : (int64_t(1) << scale);
+  if ((double)n_edges > 0.5 * (double)n_ids * (double)(n_ids - 1)) return -1;
+  std::vector<Cand> cands;
+  int64_t next_j = 0;
+  int64_t uniq = 0;
+  while (uniq < n_edges) {
+    const int64_t want = (int64_t)((double)(n_edges - uniq) * 1.25) + 1024;
+    const size_t old = cands.size();
+    cands.resize(old + (size_t)want);
+    std::vector<uint8_t> ok((size_t)want);
+#pragma omp parallel for schedule(static)
+    for (int64_t t = 0; t < want; ++t) {
+      uint64_t key = 0;
+      ok[t] = rmat_one(scale, a, b, c, seed, next_j + t, id_limit, &key);
+      cands[old + t] = Cand{key, next_j + t};
+    }
+    size_t w = old;
+    for (int64_t t = 0; t < want; ++t)
+      if (ok[t]) cands[w++] = cands[old + t];
+    cands.resize(w);
+    next_j += want;
+    __gnu_parallel::sort(cands.begin(), cands.end(), [](const Cand& x, const Cand& y) {
+      return x.key < y.key || (x.key == y.key && x.idx < y.idx);
+    });
+    size_t o = 0;
+    for (size_t i = 0; i < cands.size(); ++i)
+      if (o == 0 || cands[i].key != cands[o - 1].key) cands[o++] = cands[i];
+    cands.resize(o);
+    uniq = (int64_t)o;
+  }
+  // keep the n_edges earliest by generation index, in generation order
+  __gnu_parallel::sort(cands.begin(), cands.end(),
+                       [](const Cand& x, const Cand& y) { return x.idx < y.idx; });
+  cands.resize((size_t)n_edges);
+  // seeded permutation of vertex ids (Fisher-Yates, counter-based draws)
+  std::vector<int32_t> perm((size_t)n_ids);
+  std::iota(perm.begin(), perm.end(), 0);
+  const uint64_t pseed = h2(seed, 0x5045524DULL);
+  for (int64_t i = n_ids - 1; i > 0; --i) {
+    const uint64_t r = h2(pseed, (uint64_t)i);
+    const int64_t j = (int64_t)(r % (uint64_t)(i + 1));
+    std::swap(perm[i], perm[j]);
+  }
+#pragma omp parallel for schedule(static)
+  for (int64_t e = 0; e < n_edges; ++e) {
+    int32_t u = perm[(size_t)(cands[e].key >> 32)];
+    int32_t v = perm[(size_t)(cands[e].key & 0xFFFFFFFFULL)];
+    if (u > v) std::swap(u, v);
+    out_uv[2 * e] = u;
+    out_uv[2 * e + 1] = v;
+  }
+  return n_edges;
+}
+
+// Symmetric CSR of an undirected simple edge list (u != v, no duplicates):
+// row_ptr[n+1], col[2m], each row sorted ascending.
+int32_t gi_build_csr(int32_t n, int64_t m, const int32_t* uv, int32_t threads, int64_t* row_ptr,
+                     int32_t* col) {
+  if (threads > 0) omp_set_num_threads(threads);
+  std::vector<int64_t> deg((size_t)n + 1, 0);
+  for (int64_t e = 0; e < m; ++e) {
+    const int32_t u = uv[2 * e], v = uv[2 * e + 1];
+    if (u < 0 || v < 0 || u >= n || v >= n || u == v) return -1;
+    deg[u]++;
+    deg[v]++;
+  }
+  row_ptr[0] = 0;
+  for (int32_t i = 0; i < n; ++i) row_ptr[i + 1] = row_ptr[i] + deg[i];
+  std::vector<int64_t> pos(row_ptr, row_ptr + n);
+  for (int64_t e = 0; e < m; ++e) {
+    const int32_t u = uv[2 * e], v = uv[2 * e + 1];
+    col[pos[u]++] = v;
+    col[pos[v]++] = u;
+  }
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int32_t i = 0; i < n; ++i) std::sort(col + row_ptr[i], col + row_ptr[i + 1]);
+  return 0;
+}
+
+// Labels uniform over [0, L).
+void gi_labels(int32_t n, int32_t L, uint64_t seed, int32_t* labels) {
+  const uint64_t s = h2(seed, 0x4C4142454CULL);
+#pragma omp parallel for schedule(static)
+  for (int32_t i = 0; i < n; ++i) labels[i] = (int32_t)(h2(s, (uint64_t)i) % (uint64_t)L);
+}
+
+// P:331 stream protocol: n_sample edge indices drawn uniformly without
+// replacement from [0, m) in random order (sparse partial Fisher-Yates), each
+// marked insertion (sign=+1) or deletion (sign=-1) with p = 1/2.
+int64_t gi_stream(int64_t m, int64_t n_sample, uint64_t seed, int64_t* sel, int8_t* sign) {
+  if (n_sample > m) return -1;
+  std::unordered_map<int64_t, int64_t> swapped;
+  swapped.reserve((size_t)n_sample * 2);
+  const uint64_t s = h2(seed, 0x53545245414DULL);
+  auto at = [&](int64_t i) {
+    auto it = swapped.find(i);
+    return it == swapped.end() ? i : it->second;
+  };
+  for (int64_t t = 0; t < n_sample; ++t) {
+    const uint64_t r = h2(s, (uint64_t)t);
+    const int64_t j = t + (int64_t)(r % (uint64_t)(m - t));
+    const int64_t vj = at(j), vt = at(t);
+    swapped[j] = vt;
+    swapped[t] = vj;
+    sel[t] = vj;
+    sign[t] = (h2(s ^ 0xABCDEFULL, (uint64_t)t) & 1) ? (int8_t)1 : (int8_t)-1;
+  }
+  return n_sample;
+}
+
+}  // extern "C"
