@@ -1,0 +1,211 @@
+/*
+ * gcsm.h — C ABI of the B200-native GCSM incremental-matching hot path.
+ *
+ * Paper: "GCSM: GPU-Accelerated Continuous Subgraph Matching for Large
+ * Graphs" (Wei & Jiang, IPDPS). Citations "P:<line>" point into PAPER.md;
+ * "R<n>" are the readings listed in DESIGN.md §3 (where the paper is silent or
+ * garbled). Plain C types only: host pointers unless stated, sizes in
+ * elements, no ownership transfer (every input is caller-owned and only read
+ * during the call; every output is caller-allocated).
+ *
+ * Problem: a vertex-labelled undirected simple data graph
+ * G_t = (V, E_t, L) on the fixed id universe [0, n) (R9) receives batches of
+ * edge insertions I and deletions D; G_{t+1} = (E_t \ D) ∪ I (R8). For a
+ * connected query Q (2 <= k <= 8 vertices, R10) the library returns
+ *   added   = |Emb(Q, G_{t+1}) \ Emb(Q, G_t)|,
+ *   removed = |Emb(Q, G_t) \ Emb(Q, G_{t+1})|,
+ * where Emb is the set of injective, label- and edge-preserving maps
+ * V(Q) -> V(G) (non-induced, R1-R3). Subgraph counts are embeddings divided
+ * by gcsm_query_automorphisms().
+ *
+ * Pipeline of one gcsm_apply_batch (Fig. 3):
+ *   (1) append / mark the batch on the host store
+ *   (2) random-walk access-frequency estimation          P:183-260, eq. (3)
+ *   (3) pack the top vertices' lists, one DMA to HBM
+ *   (4) incremental matching on the GPU (eq. (1) terms)
+ *       cached lists from HBM, the rest zero-copy from the pinned host store
+ *   (4b) world > 1: one NCCL allreduce of the counters  (BASELINE north_star)
+ *   (5) reorganise the updated host lists (merge)
+ *
+ * Status conventions:
+ *   GCSM_EINVAL  bad argument, detected before any mutation (state unchanged);
+ *   GCSM_ENOMEM  host / device allocation failure;
+ *   GCSM_EDEVICE CUDA error: the context is poisoned;
+ *   GCSM_ENCCL   NCCL error: the context is poisoned;
+ *   GCSM_ESTATE  poisoned context, or apply_batch before set_query;
+ *   GCSM_ETRUNC  list mode only: a tuple buffer was too small; the counts are
+ *                still exact and the batch has been applied.
+ * Threading: one context per host thread. With world > 1 the calls
+ * set_query, set_cache_budget and apply_batch* are collective (every rank
+ * calls them in the same order with identical arguments, like NCCL).
+ */
+#ifndef GCSM_H_
+#define GCSM_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct gcsm_ctx gcsm_ctx; /* opaque, library-owned */
+
+typedef enum {
+  GCSM_OK = 0,
+  GCSM_EINVAL = 1,
+  GCSM_ENOMEM = 2,
+  GCSM_EDEVICE = 3,
+  GCSM_ENCCL = 4,
+  GCSM_ESTATE = 5,
+  GCSM_ETRUNC = 6
+} gcsm_status;
+
+/* Cache policies (step 3). ESTIMATOR is the paper's; the others are
+ * the paper's comparison points run on the same kernels. */
+enum {
+  GCSM_CACHE_ESTIMATOR = 0, /* random-walk estimates, highest first */
+  GCSM_CACHE_DEGREE = 1,    /* "Naive": degree as the frequency estimate */
+  GCSM_CACHE_NONE = 2       /* "ZP": pure zero-copy regardless of the budget */
+};
+
+/* Option flags */
+enum {
+  GCSM_FLAG_LOCAL_COUNTS = 1u /* world > 1 without NCCL: return this rank's shard counts
+                                 (single-GPU "emulated world" used by the parity tests) */
+};
+
+typedef struct {
+  int32_t device;          /* CUDA ordinal; -1 = the current device */
+  int32_t rank, world;     /* world = 1: single GPU */
+  const void *nccl_id;     /* 128-byte ncclUniqueId when world > 1 (gcsm_nccl_unique_id on rank 0,
+                              broadcast by the caller, e.g. through torch.distributed); NULL with
+                              GCSM_FLAG_LOCAL_COUNTS */
+  uint64_t seed;           /* estimator RNG seed (R22) */
+  int32_t host_threads;    /* 0 = all cores */
+  int32_t cache_policy;    /* GCSM_CACHE_* */
+  uint64_t walks_override; /* 0 = M = |ΔE| D^(k-2) / 32^k (R21) */
+  uint32_t flags;          /* GCSM_FLAG_* */
+  uint32_t reserved;
+} gcsm_options;
+
+/* Per-batch statistics (Table II-style breakdown; hit rate §8d). */
+typedef struct {
+  uint64_t batches;         /* batches applied so far */
+  uint64_t n_ins, n_del;    /* normalised insertions / deletions of the last batch */
+  uint64_t dropped;         /* no-op updates dropped by normalisation (R8) */
+  uint64_t units;           /* level-1 units (term, oriented seed) processed on this rank */
+  uint64_t n1;              /* |ΔE| of eq. (3): units of this rank (R15) */
+  uint64_t walks;           /* M */
+  uint64_t max_degree;      /* D (R19) */
+  uint64_t cached_vertices; /* K */
+  uint64_t cache_bytes;     /* bytes of cached lists (<= budget) */
+  uint64_t hit_bytes;       /* list bytes the kernels read from the HBM cache (algorithmic, §8d) */
+  uint64_t miss_bytes;      /* list bytes the kernels read zero-copy from host memory */
+  uint64_t frontier;        /* level-2 partial matches materialised */
+  uint64_t kernel_launches; /* this library's kernels launched in the last batch */
+  uint64_t added, removed;  /* last batch's global counts */
+  double ms_normalize;      /* (1) normalise + overlay + units */
+  double ms_estimate;       /* (2) */
+  double ms_pack;           /* (3) host packing */
+  double ms_copy;           /* (3) H2D: cache DMA + descriptors + deltas */
+  double ms_match;          /* (4) kernels (CUDA events) */
+  double ms_allreduce;      /* (4b) */
+  double ms_merge;          /* (5) */
+  double ms_total;          /* whole gcsm_apply_batch, host wall clock */
+} gcsm_stats;
+
+/* Fills *opt with the defaults (device -1, world 1, seed 0x6C53, all cores,
+ * estimator cache policy, M from P:339). */
+void gcsm_default_options(gcsm_options *opt);
+
+/* Creates a context from the symmetric CSR of G_0: row_ptr[n+1]
+ * (int64, because adjacency can exceed 2^31 entries), col[row_ptr[n]]; every
+ * row sorted ascending, no duplicates, no self loops, symmetric, ids in
+ * [0, n). labels: n values in [0, 65535], or NULL (unlabelled, R5).
+ * The graph is copied into the library's pinned, GPU-mapped host store with
+ * 2x capacity per list. opt may be NULL (defaults). EINVAL on any
+ * violation (nothing allocated). With world > 1 this is collective (NCCL
+ * communicator creation). */
+gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels,
+                        const gcsm_options *opt, gcsm_ctx **out);
+
+/* Sets the query pattern: k vertices (2..8), m edges qedges[2m] over [0,k)
+ * (undirected, simple, connected), qlabels[k] or NULL (any label), and the
+ * user matching order order[k] (a permutation of [0,k)) or NULL (identity).
+ * Builds the m IVM terms of eq. (1) as in Fig. 2b-f with the
+ * stable-split views (R7, R11, R12). EINVAL leaves the previous query. */
+gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                           const int32_t *order);
+
+/* Per-GPU byte budget of the HBM list cache ("GPU buffer"); it counts
+ * cached list payload (16-byte aligned lists). 0 = pure zero-copy. Applies
+ * from the next batch. ENOMEM if the device buffer cannot be allocated. */
+gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes);
+
+/* Applies one batch: ins[2*n_ins], del[2*n_del] (pairs of vertex ids, any
+ * orientation; duplicates collapse; inserting an existing edge or deleting an
+ * absent one is a counted no-op, R8). EINVAL (no mutation) on a self loop, an
+ * id outside [0,n), or an edge in both lists. On success *added / *removed
+ * are the global embedding counts (every rank gets the same values). */
+gcsm_status gcsm_apply_batch(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                             uint64_t *added, uint64_t *removed);
+
+/* Like gcsm_apply_batch, also listing the changed embeddings as k-tuples in
+ * query-vertex order (tuple[u] = f(u)): up to added_cap / removed_cap tuples
+ * (k int32 each) into added_tuples / removed_tuples. Single-GPU (world == 1 or
+ * GCSM_FLAG_LOCAL_COUNTS). Tuple order is unspecified. ETRUNC if a buffer was
+ * too small (counts exact, batch applied). */
+gcsm_status gcsm_apply_batch_list(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                                  int32_t *added_tuples, uint64_t added_cap, int32_t *removed_tuples,
+                                  uint64_t removed_cap, uint64_t *added, uint64_t *removed);
+
+/* Last batch's statistics. */
+gcsm_status gcsm_get_stats(const gcsm_ctx *ctx, gcsm_stats *out);
+
+/* |Aut_L(Q)| (label-preserving automorphisms) of the current query, 0 if none. */
+uint64_t gcsm_query_automorphisms(const gcsm_ctx *ctx);
+
+/* Static-lifetime (per ctx) message for the last error; "" if none. */
+const char *gcsm_last_error(const gcsm_ctx *ctx);
+
+/* Frees everything (pinned store, device buffers, stream, communicator). NULL-safe. */
+void gcsm_destroy(gcsm_ctx *ctx);
+
+/* ---------------------------------------------------------------- evidence helpers */
+
+/* 128-byte ncclUniqueId for rank 0 to broadcast (world > 1). */
+gcsm_status gcsm_nccl_unique_id(void *out128);
+
+/* CUDA stream (cudaStream_t) the library launches on, so a caller can time it. */
+gcsm_status gcsm_get_stream(const gcsm_ctx *ctx, void **stream);
+
+/* Current graph as symmetric CSR: row_ptr[n+1] always written; col written
+ * if col_cap >= row_ptr[n], else ETRUNC. */
+gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col, uint64_t col_cap);
+
+/* Last batch's estimator output (step 2): the vertices with a non-zero count,
+ * ascending, and per vertex the per-level sums of walk multiplicities B for
+ * tree levels 1..k-2 (eq. (3)): levcnt[i*8 + (l-1)]. *n_out = the number of
+ * such vertices (ETRUNC if > cap; the first cap are written). */
+gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levcnt, uint64_t cap, uint64_t *n_out);
+
+/* Last batch's cached vertex set (step 3), ascending. */
+gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out);
+
+/* Pure host, no device: the per-term plan the library would build for a query
+ * (for the Fig. 2 structural test). Arrays as in gcsm_set_query; outputs:
+ * out_seed[2m] (numbered query edges R_1..R_m), out_order[m*k],
+ * out_nb[m*k] (backward edges per term position), out_bq[m*k*8] (backward
+ * positions), out_view[2*m*k*8] (view per backward edge for + / - terms:
+ * 0 stable, 1 old N, 2 new N'). */
+gcsm_status gcsm_plan_inspect(int32_t k, int32_t m, const int32_t *qedges, const int32_t *order, int32_t *out_seed,
+                              int32_t *out_order, int32_t *out_nb, int32_t *out_bq, int32_t *out_view);
+
+/* Pure host, no device: the shard of each unit for world ranks (LPT on the
+ * cost proxy cost[i], ties by index): out_rank[n_units]. */
+gcsm_status gcsm_shard(int64_t n_units, const uint64_t *cost, int32_t world, int32_t *out_rank);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GCSM_H_ */

@@ -1,0 +1,716 @@
+// gcsm.cpp — the C ABI (include/gcsm.h) and the per-batch pipeline (Fig. 3).
+#include "gcsm.h"
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "estimator.h"
+#include "internal.h"
+#include "kernels.cuh"
+#include "store.h"
+
+using namespace gcsm;
+
+namespace {
+
+constexpr int64_t kF2CapLimit = 64ll << 20;  // level-2 frontier entries per chunk
+
+template <typename T>
+bool dev_ensure(T *&p, size_t &cap, size_t need) {
+  if (need <= cap && p) return true;
+  if (p) cudaFree(p);
+  p = nullptr;
+  cap = 0;
+  size_t n = std::max<size_t>(need, 1);
+  n = n + n / 4;
+  if (cudaMalloc((void **)&p, n * sizeof(T)) != cudaSuccess) return false;
+  cap = n;
+  return true;
+}
+
+template <typename T>
+bool host_ensure(T *&p, size_t &cap, size_t need) {
+  if (need <= cap && p) return true;
+  if (p) cudaFreeHost(p);
+  p = nullptr;
+  cap = 0;
+  size_t n = std::max<size_t>(need, 1);
+  n = n + n / 4;
+  if (cudaHostAlloc((void **)&p, n * sizeof(T), cudaHostAllocDefault) != cudaSuccess) return false;
+  cap = n;
+  return true;
+}
+
+}  // namespace
+
+struct gcsm_ctx {
+  gcsm_options opt{};
+  int device = 0;
+  std::string err;
+  bool poisoned = false;
+  HostStore store;
+  QueryPlan qp;
+  bool has_query = false;
+  uint64_t budget = 0;
+  cudaStream_t stream = nullptr;
+  cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr, ev_a0 = nullptr, ev_a1 = nullptr;
+  ncclComm_t comm = nullptr;
+  int grid = 0, warps_total = 0;
+
+  // device buffers
+  VDesc *d_vdesc = nullptr;
+  uint16_t *d_lab = nullptr;
+  DRec *d_drec = nullptr; size_t drec_cap = 0;
+  int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
+  Unit *d_units = nullptr; size_t units_cap = 0;
+  int2 *d_useg = nullptr; size_t useg_cap = 0;
+  int32_t *d_f2 = nullptr; size_t f2_cap = 0;  // 2 * f2 entries ints
+  int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
+  unsigned long long *d_cnt = nullptr;
+  char *d_cache = nullptr; size_t cache_cap = 0;
+  int64_t *d_pidx = nullptr; size_t pidx_cap = 0;
+  VDesc *d_pval = nullptr; size_t pval_cap = 0;
+  int32_t *d_tup = nullptr; size_t tup_cap = 0;
+
+  // pinned host staging
+  char *h_cache = nullptr; size_t h_cache_cap = 0;
+  int64_t *h_pidx = nullptr; size_t h_pidx_cap = 0;
+  VDesc *h_pval = nullptr; size_t h_pval_cap = 0;
+  DRec *h_drec = nullptr; size_t h_drec_cap = 0;
+  int32_t *h_dlist = nullptr; size_t h_dlist_cap = 0;
+  Unit *h_units = nullptr; size_t h_units_cap = 0;
+  unsigned long long *h_cnt = nullptr;
+
+  // cache / batch state
+  std::vector<VDesc> vd;             // host mirror of d_vdesc
+  std::vector<int32_t> cached;       // ascending
+  std::vector<int32_t> prev_cached, prev_U;
+  std::vector<uint8_t> mark;         // scratch (n)
+  EstimatorOutput est;
+  gcsm_stats stats{};
+  uint64_t batch_seq = 0;
+  std::vector<int32_t> degree_order;  // GCSM_CACHE_DEGREE ranking
+
+  gcsm_status fail(gcsm_status s, const std::string &m) {
+    err = m;
+    if (s == GCSM_EDEVICE || s == GCSM_ENCCL) poisoned = true;
+    return s;
+  }
+  gcsm_status cuda_fail(cudaError_t e, const char *where) {
+    return fail(GCSM_EDEVICE, std::string(where) + ": " + cudaGetErrorString(e));
+  }
+  ~gcsm_ctx();
+};
+
+#define CK(call)                                     \
+  do {                                               \
+    cudaError_t e_ = (call);                         \
+    if (e_ != cudaSuccess) return ctx->cuda_fail(e_, #call); \
+  } while (0)
+
+gcsm_ctx::~gcsm_ctx() {
+  if (stream) cudaStreamSynchronize(stream);
+  if (comm) ncclCommDestroy(comm);
+  void *dev[] = {d_vdesc, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cache, d_pidx, d_pval,
+                 d_tup};
+  for (void *p : dev)
+    if (p) cudaFree(p);
+  void *host[] = {h_cache, h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt};
+  for (void *p : host)
+    if (p) cudaFreeHost(p);
+  for (cudaEvent_t e : {ev_m0, ev_m1, ev_a0, ev_a1})
+    if (e) cudaEventDestroy(e);
+  if (stream) cudaStreamDestroy(stream);
+}
+
+extern "C" {
+
+void gcsm_default_options(gcsm_options *o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof *o);
+  o->device = -1;
+  o->rank = 0;
+  o->world = 1;
+  o->seed = 0x6C53;
+  o->host_threads = 0;
+  o->cache_policy = GCSM_CACHE_ESTIMATOR;
+}
+
+gcsm_status gcsm_nccl_unique_id(void *out128) {
+  if (!out128) return GCSM_EINVAL;
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return GCSM_ENCCL;
+  std::memcpy(out128, &id, sizeof id);
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels,
+                        const gcsm_options *opt, gcsm_ctx **out) {
+  if (!out) return GCSM_EINVAL;
+  *out = nullptr;
+  gcsm_options o;
+  gcsm_default_options(&o);
+  if (opt) o = *opt;
+  if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return GCSM_EINVAL;
+  if (o.world > 1 && !o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) return GCSM_EINVAL;
+  if (o.cache_policy < 0 || o.cache_policy > 2) return GCSM_EINVAL;
+  if (n < 1 || !row_ptr) return GCSM_EINVAL;
+  gcsm_ctx *ctx = new (std::nothrow) gcsm_ctx();
+  if (!ctx) return GCSM_ENOMEM;
+  ctx->opt = o;
+  int threads = o.host_threads > 0 ? o.host_threads : (int)std::max(1u, std::thread::hardware_concurrency());
+  ctx->opt.host_threads = threads;
+  // device
+  int dev = o.device;
+  if (dev < 0 && cudaGetDevice(&dev) != cudaSuccess) {
+    delete ctx;
+    return GCSM_EDEVICE;
+  }
+  if (cudaSetDevice(dev) != cudaSuccess) {
+    delete ctx;
+    return GCSM_EDEVICE;
+  }
+  ctx->device = dev;
+  bool cuda_err = false;
+  std::string e = ctx->store.init(n, row_ptr, col, labels, threads, &cuda_err);
+  if (!e.empty()) {
+    delete ctx;
+    return cuda_err ? GCSM_EDEVICE : GCSM_EINVAL;
+  }
+  auto bail = [&](gcsm_status s) {
+    delete ctx;
+    return s;
+  };
+  if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
+  for (cudaEvent_t *ev : {&ctx->ev_m0, &ctx->ev_m1, &ctx->ev_a0, &ctx->ev_a1})
+    if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
+  if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaHostAlloc(&ctx->h_cnt, sizeof(unsigned long long) * CNT_N, cudaHostAllocDefault) != cudaSuccess)
+    return bail(GCSM_ENOMEM);
+  ctx->vd.resize(n);
+  for (int32_t v = 0; v < n; ++v)
+    ctx->vd[v] = VDesc{ctx->store.dev_ptr(ctx->store.lst[v]), ctx->store.len[v], 0};
+  if (cudaMemcpy(ctx->d_vdesc, ctx->vd.data(), sizeof(VDesc) * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
+    return bail(GCSM_EDEVICE);
+  if (labels) {
+    if (cudaMalloc(&ctx->d_lab, 2 * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
+    if (cudaMemcpy(ctx->d_lab, ctx->store.lab.data(), 2 * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
+      return bail(GCSM_EDEVICE);
+  }
+  ctx->mark.assign(n, 0);
+  ctx->grid = match_grid(dev, &ctx->warps_total);
+  if (o.world > 1 && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
+    ncclUniqueId id;
+    std::memcpy(&id, o.nccl_id, sizeof id);
+    if (ncclCommInitRank(&ctx->comm, o.world, id, o.rank) != ncclSuccess) return bail(GCSM_ENCCL);
+  }
+  *out = ctx;
+  return GCSM_OK;
+}
+
+void gcsm_destroy(gcsm_ctx *ctx) { delete ctx; }
+
+const char *gcsm_last_error(const gcsm_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+gcsm_status gcsm_get_stream(const gcsm_ctx *ctx, void **stream) {
+  if (!ctx || !stream) return GCSM_EINVAL;
+  *stream = (void *)ctx->stream;
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                           const int32_t *order) {
+  if (!ctx) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  QueryPlan qp;
+  std::string e = build_plan(k, m, qedges, qlabels, order, qp);
+  if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
+  if (qp.labelled && !ctx->d_lab) {  // unlabelled graph: every data label is 0 (R5)
+    CK(cudaMalloc(&ctx->d_lab, 2 * (size_t)ctx->store.n));
+    CK(cudaMemset(ctx->d_lab, 0, 2 * (size_t)ctx->store.n));
+  }
+  CK(upload_plans(qp.plans.data(), (int)qp.plans.size(), ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  ctx->qp = qp;
+  ctx->has_query = true;
+  ctx->err.clear();
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
+  if (!ctx) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  bytes &= ~uint64_t(15);
+  if (bytes > ctx->cache_cap) {
+    if (ctx->d_cache) cudaFree(ctx->d_cache);
+    if (ctx->h_cache) cudaFreeHost(ctx->h_cache);
+    ctx->d_cache = nullptr;
+    ctx->h_cache = nullptr;
+    ctx->cache_cap = ctx->h_cache_cap = 0;
+    if (cudaMalloc(&ctx->d_cache, bytes) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "device cache allocation failed");
+    if (cudaHostAlloc(&ctx->h_cache, bytes, cudaHostAllocDefault) != cudaSuccess)
+      return ctx->fail(GCSM_ENOMEM, "pinned cache staging allocation failed");
+    ctx->cache_cap = ctx->h_cache_cap = bytes;
+  }
+  ctx->budget = bytes;
+  return GCSM_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------ pipeline
+
+static uint16_t host_label(const HostStore &s, int32_t v) { return s.lab.empty() ? 0 : s.lab[v]; }
+
+static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                              int32_t *tup_add, uint64_t add_cap, int32_t *tup_rem, uint64_t rem_cap,
+                              uint64_t *added, uint64_t *removed) {
+  if (!ctx) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  if (!ctx->has_query) return ctx->fail(GCSM_ESTATE, "apply_batch before set_query");
+  const bool listing = tup_add || tup_rem;
+  if (listing && ctx->opt.world > 1 && !(ctx->opt.flags & GCSM_FLAG_LOCAL_COUNTS))
+    return ctx->fail(GCSM_EINVAL, "list mode is single-GPU");
+  Timer total;
+  HostStore &S = ctx->store;
+  const QueryPlan &Q = ctx->qp;
+  const int k = Q.k;
+  const int T = ctx->opt.host_threads;
+  gcsm_stats st{};
+  st.batches = ctx->batch_seq + 1;
+
+  // ---- (1) normalise + overlay + units -------------------------------------------------
+  Timer t1;
+  std::string e = S.normalize(n_ins, ins, n_del, del);
+  if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
+  bool cuda_err = false;
+  if (!S.build_overlay(&cuda_err)) return ctx->fail(GCSM_EDEVICE, "pinned overlay allocation failed");
+  st.n_ins = S.I.size();
+  st.n_del = S.D.size();
+  st.dropped = S.dropped;
+  std::vector<Unit> units;
+  std::vector<uint64_t> cost;
+  units.reserve((S.I.size() + S.D.size()) * 2 * Q.m);
+  for (int term = 0; term < Q.m; ++term)
+    for (int kind = 0; kind < 2; ++kind) {
+      const DevPlan &P = Q.plans[2 * term + kind];
+      const std::vector<uint64_t> &E = kind ? S.D : S.I;
+      for (uint64_t key : E) {
+        const int32_t x = (int32_t)(key >> 32), y = (int32_t)(key & 0xffffffffu);
+        for (int o = 0; o < 2; ++o) {
+          const int32_t a = o ? y : x, b = o ? x : y;
+          if (P.label0 >= 0 && host_label(S, a) != P.label0) continue;
+          if (P.label1 >= 0 && host_label(S, b) != P.label1) continue;
+          units.push_back(Unit{a, b, 2 * term + kind, 0});
+        }
+      }
+    }
+  // cost proxy of a unit: the list lengths its first level reads
+  cost.resize(units.size());
+  for (size_t i = 0; i < units.size(); ++i) {
+    const DevPlan &P = Q.plans[units[i].plan];
+    uint64_t c = 1;
+    if (k > 2) {
+      const LevelPlan &L2 = P.lv[2];
+      const int32_t f[2] = {units[i].a, units[i].b};
+      for (int b = 0; b < L2.nb; ++b) c += S.view_len(f[L2.bpos[b]], L2.bview[b]);
+    }
+    cost[i] = c;
+  }
+  if (ctx->opt.world > 1) {
+    std::vector<int32_t> rk(units.size());
+    shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data());
+    size_t w = 0;
+    for (size_t i = 0; i < units.size(); ++i)
+      if (rk[i] == ctx->opt.rank) {
+        units[w] = units[i];
+        cost[w] = cost[i];
+        ++w;
+      }
+    units.resize(w);
+    cost.resize(w);
+  }
+  {  // heaviest units first (dynamic scheduling tail)
+    std::vector<size_t> idx(units.size());
+    std::iota(idx.begin(), idx.end(), 0);
+    std::stable_sort(idx.begin(), idx.end(), [&](size_t x, size_t y) { return cost[x] > cost[y]; });
+    std::vector<Unit> u2(units.size());
+    std::vector<uint64_t> c2(units.size());
+    for (size_t i = 0; i < idx.size(); ++i) {
+      u2[i] = units[idx[i]];
+      c2[i] = cost[idx[i]];
+    }
+    units.swap(u2);
+    cost.swap(c2);
+  }
+  const int64_t nu = (int64_t)units.size();
+  st.units = st.n1 = (uint64_t)nu;
+  const uint64_t D = std::max<uint64_t>(1, std::max<uint64_t>(S.maxdeg, S.maxdeg_new));
+  st.max_degree = D;
+  st.ms_normalize = t1.ms();
+
+  // ---- (2) estimator ---------------------------------------------------------------------
+  Timer t2;
+  ctx->est.ids.clear();
+  ctx->est.levcnt.clear();
+  std::vector<std::pair<double, int32_t>> ranked;  // (score, id)
+  const bool use_cache = ctx->budget > 0 && ctx->opt.cache_policy != GCSM_CACHE_NONE && k > 2;
+  uint64_t M = 0;
+  if (k > 2 && nu > 0) {
+    M = ctx->opt.walks_override ? ctx->opt.walks_override : walk_budget((uint64_t)nu, D, k);
+    st.walks = M;
+    if (ctx->opt.cache_policy == GCSM_CACHE_ESTIMATOR && ctx->budget > 0) {
+      EstimatorInput in;
+      in.plans = Q.plans.data();
+      in.units = units.data();
+      in.n_units = nu;
+      in.N1 = (uint64_t)nu;
+      in.D = D;
+      in.M = M;
+      in.seed = ctx->opt.seed;
+      in.batch_seq = ctx->batch_seq;
+      in.labels = S.lab.empty() ? nullptr : S.lab.data();
+      in.threads = T;
+      in.view = [&S](int32_t v, int vw) { return S.view(v, vw); };
+      run_estimator(in, ctx->est);
+      if (use_cache) {
+        ranked.reserve(ctx->est.ids.size());
+        for (size_t i = 0; i < ctx->est.ids.size(); ++i)
+          ranked.emplace_back(estimate_value(&ctx->est.levcnt[8 * i], k, (uint64_t)nu, D, M), ctx->est.ids[i]);
+      }
+    }
+  }
+  if (use_cache && ctx->opt.cache_policy == GCSM_CACHE_DEGREE) {
+    ranked.reserve(S.n);
+    for (int32_t v = 0; v < S.n; ++v) {
+      const uint32_t d = S.view_len(v, VIEW_S);
+      if (d) ranked.emplace_back((double)d, v);
+    }
+  }
+  st.ms_estimate = t2.ms();
+
+  // ---- (3) pack the cache + descriptors --------------------------------------------------
+  Timer t3;
+  std::vector<int32_t> sel;
+  std::vector<uint64_t> sel_off;
+  uint64_t used = 0;
+  if (use_cache && !ranked.empty()) {
+    std::sort(ranked.begin(), ranked.end(), [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {
+      return x.first > y.first || (x.first == y.first && x.second < y.second);
+    });
+    for (const auto &r : ranked) {
+      if (!(r.first > 0)) break;
+      const uint64_t bytes = (uint64_t)((S.view_len(r.second, VIEW_S) + 3u) & ~3u) * 4;
+      if (used + bytes > ctx->budget) break;  // longest prefix that fits (R23)
+      sel.push_back(r.second);
+      sel_off.push_back(used);
+      used += bytes;
+    }
+    parallel_for(T, (int64_t)sel.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i) {
+        const HList h = S.view(sel[i], VIEW_S);
+        std::memcpy(ctx->h_cache + sel_off[i], h.a, (size_t)h.na * 4);
+      }
+    });
+  }
+  st.cached_vertices = sel.size();
+  st.cache_bytes = used;
+  // descriptors to patch: previous cache / updated sets and the new ones
+  std::vector<int32_t> dirty;
+  dirty.reserve(ctx->prev_cached.size() + ctx->prev_U.size() + S.U.size() + sel.size());
+  auto add_dirty = [&](int32_t v) {
+    if (!ctx->mark[v]) {
+      ctx->mark[v] = 1;
+      dirty.push_back(v);
+    }
+  };
+  for (int32_t v : ctx->prev_cached) add_dirty(v);
+  for (int32_t v : ctx->prev_U) add_dirty(v);
+  for (int32_t v : S.U) add_dirty(v);
+  for (int32_t v : sel) add_dirty(v);
+  for (int32_t v : dirty) ctx->mark[v] = 0;
+  std::vector<int64_t> cache_slot;  // per dirty vertex: offset or -1
+  {
+    // map selected -> offset via a temporary mark pass
+    for (size_t i = 0; i < sel.size(); ++i) ctx->mark[sel[i]] = 1;
+  }
+  if (!host_ensure(ctx->h_pidx, ctx->h_pidx_cap, dirty.size()) ||
+      !host_ensure(ctx->h_pval, ctx->h_pval_cap, dirty.size()))
+    return ctx->fail(GCSM_ENOMEM, "pinned staging");
+  {
+    std::vector<int64_t> off_of;  // only for selected; find by binary search over a sorted copy
+    std::vector<std::pair<int32_t, uint64_t>> so(sel.size());
+    for (size_t i = 0; i < sel.size(); ++i) so[i] = {sel[i], sel_off[i]};
+    std::sort(so.begin(), so.end());
+    for (size_t i = 0; i < dirty.size(); ++i) {
+      const int32_t v = dirty[i];
+      const int32_t ui = S.uidx[v];
+      VDesc d;
+      d.upd = ui >= 0 ? (uint32_t)ui + 1 : 0;
+      d.len = ui >= 0 ? S.s_len[ui] : S.len[v];
+      if (ctx->mark[v]) {
+        auto it = std::lower_bound(so.begin(), so.end(), std::make_pair(v, (uint64_t)0));
+        d.ptr = (const int32_t *)(ctx->d_cache + it->second);
+      } else {
+        d.ptr = S.dev_ptr(ui >= 0 ? S.s_ptr[ui] : S.lst[v]);
+      }
+      ctx->h_pidx[i] = v;
+      ctx->h_pval[i] = d;
+      ctx->vd[v] = d;
+    }
+  }
+  for (int32_t v : sel) ctx->mark[v] = 0;
+  // delta lists of U
+  const size_t nU = S.U.size();
+  const size_t nd = S.ins_val.size() + S.del_val.size();
+  if (!host_ensure(ctx->h_drec, ctx->h_drec_cap, nU) || !host_ensure(ctx->h_dlist, ctx->h_dlist_cap, nd) ||
+      !host_ensure(ctx->h_units, ctx->h_units_cap, (size_t)nu))
+    return ctx->fail(GCSM_ENOMEM, "pinned staging");
+  for (size_t i = 0; i < nU; ++i)
+    ctx->h_drec[i] = DRec{S.ins_off[i], S.ins_off[i + 1] - S.ins_off[i], (uint32_t)S.ins_val.size() + S.del_off[i],
+                          S.del_off[i + 1] - S.del_off[i]};
+  std::memcpy(ctx->h_dlist, S.ins_val.data(), S.ins_val.size() * 4);
+  std::memcpy(ctx->h_dlist + S.ins_val.size(), S.del_val.data(), S.del_val.size() * 4);
+  std::memcpy(ctx->h_units, units.data(), sizeof(Unit) * (size_t)nu);
+  st.ms_pack = t3.ms();
+
+  Timer t4;
+  cudaStream_t s = ctx->stream;
+  if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
+      !dev_ensure(ctx->d_drec, ctx->drec_cap, nU) || !dev_ensure(ctx->d_dlist, ctx->dlist_cap, nd) ||
+      !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)nu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)nu))
+    return ctx->fail(GCSM_ENOMEM, "device buffers");
+  if (used) CK(cudaMemcpyAsync(ctx->d_cache, ctx->h_cache, used, cudaMemcpyHostToDevice, s));  // the one DMA
+  CK(cudaMemcpyAsync(ctx->d_pidx, ctx->h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(ctx->d_pval, ctx->h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
+  CK(launch_patch_vdesc(ctx->d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
+  uint64_t launches = dirty.empty() ? 0 : 1;
+  if (nU) CK(cudaMemcpyAsync(ctx->d_drec, ctx->h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
+  if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, ctx->h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
+  if (nu) CK(cudaMemcpyAsync(ctx->d_units, ctx->h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
+  st.ms_copy = t4.ms();
+
+  // ---- (4) matching kernels --------------------------------------------------------------
+  const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
+  const int nbuf = std::max(1, std::max(k - 4, 0) + (listing ? 1 : 0));
+  const size_t stride = (size_t)nbuf * (size_t)dcap;
+  if (!dev_ensure(ctx->d_scratch, ctx->scratch_cap, stride * (size_t)ctx->warps_total))
+    return ctx->fail(GCSM_ENOMEM, "scratch");
+  // level-2 frontier chunks: per unit an upper bound on its candidates
+  std::vector<std::pair<int64_t, int64_t>> chunks;
+  int64_t f2_need = 0;
+  if (k >= 4) {
+    int64_t start = 0, acc = 0;
+    for (int64_t i = 0; i < nu; ++i) {
+      const DevPlan &P = Q.plans[units[i].plan];
+      const LevelPlan &L2 = P.lv[2];
+      const int32_t f[2] = {units[i].a, units[i].b};
+      int64_t b = INT64_MAX;
+      for (int j = 0; j < L2.nb; ++j) b = std::min<int64_t>(b, S.view_len(f[L2.bpos[j]], L2.bview[j]));
+      if (acc + b > kF2CapLimit && i > start) {
+        chunks.push_back({start, i});
+        f2_need = std::max(f2_need, acc);
+        start = i;
+        acc = 0;
+      }
+      acc += b;
+    }
+    chunks.push_back({start, nu});
+    f2_need = std::max(f2_need, acc);
+    if (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)))
+      return ctx->fail(GCSM_ENOMEM, "frontier");
+  } else {
+    chunks.push_back({0, nu});
+  }
+  // list mode buffers
+  int32_t *d_tadd = nullptr, *d_trem = nullptr;
+  if (listing) {
+    const size_t need = (size_t)k * (add_cap + rem_cap);
+    if (!dev_ensure(ctx->d_tup, ctx->tup_cap, std::max<size_t>(need, 1))) return ctx->fail(GCSM_ENOMEM, "tuples");
+    d_tadd = ctx->d_tup;
+    d_trem = ctx->d_tup + (size_t)k * add_cap;
+  }
+  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N, s));
+  MatchArgs A{};
+  A.vdesc = ctx->d_vdesc;
+  A.lab = ctx->d_lab;
+  A.drec = ctx->d_drec;
+  A.dlist = ctx->d_dlist;
+  A.useg = ctx->d_useg;
+  A.f2 = reinterpret_cast<int2 *>(ctx->d_f2);
+  A.f2_cap = f2_need;
+  A.scratch = ctx->d_scratch;
+  A.scratch_stride = (int64_t)stride;
+  A.dcap = dcap;
+  A.cnt = ctx->d_cnt;
+  A.cache_lo = ctx->d_cache;
+  A.cache_hi = ctx->d_cache ? ctx->d_cache + ctx->cache_cap : nullptr;
+  A.tup_add = d_tadd;
+  A.tup_add_cap = add_cap;
+  A.tup_rem = d_trem;
+  A.tup_rem_cap = rem_cap;
+  A.k = k;
+  A.listing = listing ? 1 : 0;
+  CK(cudaEventRecord(ctx->ev_m0, s));
+  for (const auto &ch : chunks) {
+    if (ch.second <= ch.first) continue;
+    A.units = ctx->d_units + ch.first;
+    A.n_units = ch.second - ch.first;
+    // reset the work cursors and the frontier size of this chunk
+    CK(cudaMemsetAsync(ctx->d_cnt + CNT_F2, 0, sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(ctx->d_cnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), s));
+    CK(launch_level2(A, ctx->grid, s));
+    ++launches;
+    if (k >= 4) {
+      CK(launch_extend(A, ctx->grid, s));
+      ++launches;
+    }
+  }
+  CK(cudaEventRecord(ctx->ev_m1, s));
+  // ---- (4b) count allreduce over NVLink (world > 1) -------------------------------------
+  CK(cudaEventRecord(ctx->ev_a0, s));
+  if (ctx->comm) {
+    if (ncclAllReduce(ctx->d_cnt, ctx->d_cnt, 2, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
+      return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
+  }
+  CK(cudaEventRecord(ctx->ev_a1, s));
+  CK(cudaMemcpyAsync(ctx->h_cnt, ctx->d_cnt, sizeof(unsigned long long) * CNT_N, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (ctx->h_cnt[CNT_OVERFLOW]) return ctx->fail(GCSM_EDEVICE, "internal: level-2 frontier overflow");
+  float ms_m = 0, ms_a = 0;
+  cudaEventElapsedTime(&ms_m, ctx->ev_m0, ctx->ev_m1);
+  cudaEventElapsedTime(&ms_a, ctx->ev_a0, ctx->ev_a1);
+  st.ms_match = ms_m;
+  st.ms_allreduce = ms_a;
+  st.added = ctx->h_cnt[CNT_ADDED];
+  st.removed = ctx->h_cnt[CNT_REMOVED];
+  st.hit_bytes = ctx->h_cnt[CNT_HIT];
+  st.miss_bytes = ctx->h_cnt[CNT_MISS];
+  st.frontier = ctx->h_cnt[CNT_F2];
+  st.kernel_launches = launches;
+  bool trunc = false;
+  if (listing) {
+    const uint64_t na = std::min<uint64_t>(ctx->h_cnt[CNT_TUP_ADD], add_cap);
+    const uint64_t nr = std::min<uint64_t>(ctx->h_cnt[CNT_TUP_REM], rem_cap);
+    if (na) CK(cudaMemcpy(tup_add, d_tadd, sizeof(int32_t) * k * na, cudaMemcpyDeviceToHost));
+    if (nr) CK(cudaMemcpy(tup_rem, d_trem, sizeof(int32_t) * k * nr, cudaMemcpyDeviceToHost));
+    trunc = ctx->h_cnt[CNT_TUP_ADD] > add_cap || ctx->h_cnt[CNT_TUP_REM] > rem_cap;
+  }
+
+  // ---- (5) reorganise the host lists (after matching) -----------------------------
+  Timer t5;
+  S.merge();
+  ctx->prev_cached = sel;
+  std::sort(ctx->prev_cached.begin(), ctx->prev_cached.end());
+  ctx->cached = ctx->prev_cached;
+  ctx->prev_U = S.U;
+  S.clear_batch();
+  st.ms_merge = t5.ms();
+  ++ctx->batch_seq;
+  st.ms_total = total.ms();
+  ctx->stats = st;
+  if (added) *added = st.added;
+  if (removed) *removed = st.removed;
+  if (trunc) return ctx->fail(GCSM_ETRUNC, "tuple buffer too small");
+  ctx->err.clear();
+  return GCSM_OK;
+}
+
+extern "C" {
+
+gcsm_status gcsm_apply_batch(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                             uint64_t *added, uint64_t *removed) {
+  return apply_impl(ctx, n_ins, ins, n_del, del, nullptr, 0, nullptr, 0, added, removed);
+}
+
+gcsm_status gcsm_apply_batch_list(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                                  int32_t *added_tuples, uint64_t added_cap, int32_t *removed_tuples,
+                                  uint64_t removed_cap, uint64_t *added, uint64_t *removed) {
+  if (!added_tuples || !removed_tuples) return GCSM_EINVAL;
+  return apply_impl(ctx, n_ins, ins, n_del, del, added_tuples, added_cap, removed_tuples, removed_cap, added,
+                    removed);
+}
+
+gcsm_status gcsm_get_stats(const gcsm_ctx *ctx, gcsm_stats *out) {
+  if (!ctx || !out) return GCSM_EINVAL;
+  *out = ctx->stats;
+  return GCSM_OK;
+}
+
+uint64_t gcsm_query_automorphisms(const gcsm_ctx *ctx) {
+  return ctx && ctx->has_query ? ctx->qp.automorphisms : 0;
+}
+
+gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col, uint64_t col_cap) {
+  if (!ctx || !row_ptr) return GCSM_EINVAL;
+  const HostStore &S = ctx->store;
+  row_ptr[0] = 0;
+  for (int32_t v = 0; v < S.n; ++v) row_ptr[v + 1] = row_ptr[v] + S.len[v];
+  if (!col || col_cap < (uint64_t)row_ptr[S.n]) return GCSM_ETRUNC;
+  for (int32_t v = 0; v < S.n; ++v)
+    if (S.len[v]) std::memcpy(col + row_ptr[v], S.lst[v], (size_t)S.len[v] * 4);
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levcnt, uint64_t cap, uint64_t *n_out) {
+  if (!ctx || !n_out) return GCSM_EINVAL;
+  const uint64_t n = ctx->est.ids.size();
+  *n_out = n;
+  const uint64_t w = std::min(n, cap);
+  if (ids && w) std::memcpy(ids, ctx->est.ids.data(), 4 * w);
+  if (levcnt && w) std::memcpy(levcnt, ctx->est.levcnt.data(), 8 * 8 * w);
+  return n > cap ? GCSM_ETRUNC : GCSM_OK;
+}
+
+gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out) {
+  if (!ctx || !n_out) return GCSM_EINVAL;
+  const uint64_t n = ctx->cached.size();
+  *n_out = n;
+  const uint64_t w = std::min(n, cap);
+  if (ids && w) std::memcpy(ids, ctx->cached.data(), 4 * w);
+  return n > cap ? GCSM_ETRUNC : GCSM_OK;
+}
+
+gcsm_status gcsm_plan_inspect(int32_t k, int32_t m, const int32_t *qedges, const int32_t *order, int32_t *out_seed,
+                              int32_t *out_order, int32_t *out_nb, int32_t *out_bq, int32_t *out_view) {
+  QueryPlan qp;
+  if (!build_plan(k, m, qedges, nullptr, order, qp).empty()) return GCSM_EINVAL;
+  for (int t = 0; t < m; ++t) {
+    if (out_seed) {
+      out_seed[2 * t] = qp.qe[t][0];
+      out_seed[2 * t + 1] = qp.qe[t][1];
+    }
+    for (int kind = 0; kind < 2; ++kind) {
+      const DevPlan &P = qp.plans[2 * t + kind];
+      for (int p = 0; p < k; ++p) {
+        if (kind == 0 && out_order) out_order[t * k + p] = P.order[p];
+        const int nb = p >= 2 ? P.lv[p].nb : 0;
+        if (kind == 0 && out_nb) out_nb[t * k + p] = nb;
+        for (int b = 0; b < nb; ++b) {
+          if (kind == 0 && out_bq) out_bq[(t * k + p) * 8 + b] = P.lv[p].bpos[b];
+          if (out_view) out_view[((kind * m + t) * k + p) * 8 + b] = P.lv[p].bview[b];
+        }
+      }
+    }
+  }
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_shard(int64_t n_units, const uint64_t *cost, int32_t world, int32_t *out_rank) {
+  if (n_units < 0 || world < 1 || (n_units && (!cost || !out_rank))) return GCSM_EINVAL;
+  shard_lpt(n_units, cost, world, out_rank);
+  return GCSM_OK;
+}
+
+}  // extern "C"

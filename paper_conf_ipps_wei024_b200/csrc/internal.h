@@ -1,0 +1,137 @@
+// internal.h — shared declarations of libgcsm (product side).
+// Device/host data layout:
+//   VDesc  per vertex, 16 B, in HBM: where the vertex's *main* list lives
+//          (HBM cache slot or mapped pinned host memory — one generic
+//          pointer, UVA), its length, and its delta record (updated vertices).
+//   DRec   per updated vertex x ∈ U: offsets of ins(x) / del(x) in the
+//          device delta list. For x ∈ U the main list is the stable part
+//          N_S(x) = N(x) \ del(x); views: S = main, OLD (N) = main ∪ del,
+//          NEW (N') = main ∪ ins (SURVEY §8 notation; "N' = N ∪ ΔN").
+//   Unit   one level-1 node: term i, kind ±, oriented seed (a, b).
+#pragma once
+#include <cstdint>
+#include <cstddef>
+#include <atomic>
+#include <chrono>
+#include <functional>
+#include <string>
+#include <thread>
+#include <vector>
+
+#define GCSM_MAXK 8
+#define GCSM_MAXM 28
+#define GCSM_MAXPLANS (2 * GCSM_MAXM)
+
+namespace gcsm {
+
+enum View : int8_t { VIEW_S = 0, VIEW_OLD = 1, VIEW_NEW = 2 };
+
+struct alignas(16) VDesc {
+  const int32_t *ptr;  // main list (device-visible address: HBM cache or mapped host)
+  uint32_t len;        // main list length
+  uint32_t upd;        // 0, or 1 + index of the vertex's DRec (x ∈ U)
+};
+static_assert(sizeof(VDesc) == 16, "VDesc must be 16 bytes");
+
+struct alignas(16) DRec {
+  uint32_t ins_off, ins_len, del_off, del_len;  // into the device delta list
+};
+
+struct alignas(16) Unit {
+  int32_t a, b;   // f(order[0]) = a, f(order[1]) = b
+  int32_t plan;   // 2 * term + kind (kind 0 = insertion "+", 1 = deletion "-")
+  int32_t pad;
+};
+
+// One term position (a "loop level" of Fig. 2): candidates for order[p] are
+// the intersection of the views of the backward neighbours' lists.
+struct LevelPlan {
+  int8_t nb;           // number of backward lists
+  int8_t bpos[7];      // their term positions
+  int8_t bview[7];     // their views (View)
+  int8_t reuse;        // -1, or an earlier position p' >= 2 whose candidate set
+                       // (same label, lists ⊆ these lists) is the driver (code motion)
+  int8_t nrest;        // lists not covered by the reused set
+  int8_t rest[7];      // indices into bpos/bview
+  int8_t ninj;         // matched positions to exclude (not backward neighbours)
+  int8_t inj[7];
+  int32_t label;       // required data label of order[p], -1 = any
+};
+
+struct DevPlan {
+  int32_t k;
+  int32_t kind;              // 0 "+", 1 "-"
+  int8_t order[GCSM_MAXK];   // query vertex at each term position
+  int32_t label0, label1;    // labels of the seed endpoints (-1 = any)
+  LevelPlan lv[GCSM_MAXK];   // valid for positions 2..k-1
+};
+
+// ------------------------------------------------------------ host utilities
+struct Timer {
+  std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
+  double ms() const {
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  }
+};
+
+// Static-partitioned parallel for over [0, n) with `threads` workers.
+inline void parallel_for(int threads, int64_t n, const std::function<void(int, int64_t, int64_t)> &fn) {
+  if (n <= 0) return;
+  if (threads <= 1 || n < 2) {
+    fn(0, 0, n);
+    return;
+  }
+  int t = (int)std::min<int64_t>(threads, n);
+  std::vector<std::thread> th;
+  th.reserve(t);
+  for (int i = 0; i < t; ++i) {
+    int64_t lo = n * i / t, hi = n * (i + 1) / t;
+    th.emplace_back([&fn, i, lo, hi] { fn(i, lo, hi); });
+  }
+  for (auto &x : th) x.join();
+}
+
+// Dynamic (atomic cursor) parallel for, chunked.
+inline void parallel_dyn(int threads, int64_t n, int64_t chunk, const std::function<void(int, int64_t)> &fn) {
+  if (n <= 0) return;
+  std::atomic<int64_t> next{0};
+  auto work = [&](int tid) {
+    for (;;) {
+      int64_t s = next.fetch_add(chunk);
+      if (s >= n) break;
+      int64_t e = std::min(n, s + chunk);
+      for (int64_t i = s; i < e; ++i) fn(tid, i);
+    }
+  };
+  if (threads <= 1) {
+    work(0);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (int i = 0; i < threads; ++i) th.emplace_back(work, i);
+  for (auto &x : th) x.join();
+}
+
+// ------------------------------------------------------------ plan (plan.cpp)
+struct QueryPlan {
+  int k = 0, m = 0;
+  int qe[GCSM_MAXM][2];         // numbered query edges R_1..R_m (R12), (pos-min, pos-max) endpoints
+  int qlab[GCSM_MAXK];          // -1 = any
+  bool labelled = false;
+  uint64_t automorphisms = 0;
+  std::vector<DevPlan> plans;   // 2*m: index 2*term + kind
+};
+
+// Returns "" on success, else the EINVAL reason.
+std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabels, const int32_t *order,
+                       QueryPlan &out);
+
+// ------------------------------------------------------------ RNG (estimator.cpp)
+uint64_t rng_mix(uint64_t z);
+uint64_t rng_chain(uint64_t h, uint64_t x);
+int64_t binomial(uint64_t key, int64_t n, double p);
+
+// ------------------------------------------------------------ sharding
+void shard_lpt(int64_t n, const uint64_t *cost, int world, int32_t *rank_out);
+
+}  // namespace gcsm

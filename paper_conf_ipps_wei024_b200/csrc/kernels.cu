@@ -1,0 +1,370 @@
+// kernels.cu — sm_100a incremental-matching kernels (step ④ of Fig. 3).
+//
+// What runs: for every level-1 unit (term i of eq. (1), kind ±, oriented seed
+// edge (a, b)) the nested loops of Fig. 2b-f extend the
+// partial match one query vertex per level; the candidates of a level are the
+// intersection of the backward neighbours' lists under their views (DESIGN.md
+// R7: S / N / N'), filtered by label and injectivity; the last level only
+// counts ("output" -> count).
+//
+// B200 mapping:
+//   * k_level2: warp per unit (dynamic atomic cursor, persistent grid sized to
+//     the SM count x occupancy). It computes level 2 (position 2) and either
+//     counts (k = 3) or writes the unit's candidate set as one contiguous
+//     segment of the level-2 frontier (BFS for the first level).
+//   * k_extend: warp per frontier entry (unit, x2): DFS over the remaining
+//     levels with per-warp stacks in HBM (180 GB makes D ints per level per
+//     warp affordable), code motion (a later level starts from an earlier
+//     level's candidate set, STMatch [9] / P:298).
+//   * intersections: the 32 lanes take 32 consecutive driver elements
+//     (coalesced), each lane probes the other lists by binary search; the
+//     warp compacts survivors with ballot/popc. Lists are read through one
+//     16-byte descriptor per vertex whose pointer is either the HBM cache
+//     slot or the mapped pinned host list (zero-copy): one
+//     generic load path, UVA decides the route.
+//   * counts: per-warp registers, one 64-bit atomic per warp and counter at
+//     the end of the persistent loop.
+#include <cstdio>
+
+#include "kernels.cuh"
+
+namespace gcsm {
+
+__constant__ DevPlan c_plans[GCSM_MAXPLANS];
+
+namespace {
+
+constexpr int kWarps = 8;
+constexpr int kBlock = 32 * kWarps;
+constexpr unsigned kFull = 0xffffffffu;
+
+struct LRef {
+  const int32_t *m;  // main list
+  uint32_t ml;
+  const int32_t *x;  // delta segment (ins or del), device memory
+  uint32_t xl;
+};
+
+struct Acc {
+  unsigned long long add = 0, rem = 0, hit = 0, miss = 0;
+};
+
+__device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc) {
+  const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
+  LRef r;
+  r.m = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
+                                          ((unsigned long long)(unsigned)raw.y << 32));
+  r.ml = (uint32_t)raw.z;
+  r.x = nullptr;
+  r.xl = 0;
+  const uint32_t upd = (uint32_t)raw.w;
+  if (upd != 0 && view != VIEW_S) {
+    const int4 e = __ldg(reinterpret_cast<const int4 *>(A.drec + (upd - 1)));
+    if (view == VIEW_NEW) {
+      r.x = A.dlist + e.x;
+      r.xl = (uint32_t)e.y;
+    } else {
+      r.x = A.dlist + e.z;
+      r.xl = (uint32_t)e.w;
+    }
+  }
+  const char *p = reinterpret_cast<const char *>(r.m);
+  if (p >= A.cache_lo && p < A.cache_hi) acc.hit += 4ull * r.ml;
+  else acc.miss += 4ull * r.ml;
+  acc.hit += 4ull * r.xl;
+  return r;
+}
+
+__device__ __forceinline__ bool bsearch_has(const int32_t *a, uint32_t n, int32_t v) {
+  uint32_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (a[mid] < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo < n && a[lo] == v;
+}
+
+__device__ __forceinline__ bool contains(const LRef &L, int32_t v) {
+  return bsearch_has(L.m, L.ml, v) || (L.xl != 0 && bsearch_has(L.x, L.xl, v));
+}
+
+// Warp-cooperative intersection. Driver: the device set dset[0..dn) if dset
+// != nullptr (code motion; then every L[] is a probe), else L[drv] (main then
+// delta segment; L[drv] is not probed). A driver element v survives if it is
+// not any excl[], has the required label, and belongs to every probe list.
+// MATERIALIZE: survivors are compacted into out[]. Returns the survivor count
+// (warp-uniform).
+template <bool MATERIALIZE>
+__device__ __forceinline__ uint32_t warp_isect(const MatchArgs &A, const int32_t *dset, uint32_t dn, const LRef *L,
+                                               int nl, int drv, const int32_t *excl, int nexcl, int label,
+                                               int32_t *out, int lane) {
+  const int32_t *s0, *s1;
+  uint32_t n0, n1;
+  if (dset) {
+    s0 = dset; n0 = dn; s1 = nullptr; n1 = 0;
+  } else {
+    s0 = L[drv].m; n0 = L[drv].ml; s1 = L[drv].x; n1 = L[drv].xl;
+  }
+  const uint32_t total = n0 + n1;
+  uint32_t found = 0;
+  for (uint32_t base = 0; base < total; base += 32) {
+    const uint32_t i = base + lane;
+    bool ok = i < total;
+    int32_t v = 0;
+    if (ok) v = i < n0 ? s0[i] : s1[i - n0];
+    for (int e = 0; e < nexcl; ++e) ok = ok && v != excl[e];
+    if (ok && label >= 0) ok = A.lab[v] == (uint16_t)label;
+    for (int p = 0; p < nl; ++p)
+      if (ok && (dset || p != drv)) ok = contains(L[p], v);
+    const unsigned mask = __ballot_sync(kFull, ok);
+    if (MATERIALIZE && ok) out[found + __popc(mask & ((1u << lane) - 1u))] = v;
+    found += __popc(mask);
+  }
+  return found;
+}
+
+// Lists of position p for the current partial match f (positions 0..p-1).
+// Returns the number of probe lists written to L and sets *drv (index of the
+// smallest list) or uses the reused set.
+__device__ __forceinline__ int gather_lists(const MatchArgs &A, const LevelPlan &Lp, const int32_t *f, LRef *L,
+                                            int *drv, Acc &acc) {
+  int nl = 0;
+  uint32_t best = 0xffffffffu;
+  *drv = 0;
+  if (Lp.reuse >= 0) {
+    for (int r = 0; r < Lp.nrest; ++r) {
+      const int b = Lp.rest[r];
+      L[nl++] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc);
+    }
+    return nl;
+  }
+  for (int b = 0; b < Lp.nb; ++b) {
+    L[nl] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc);
+    const uint32_t sz = L[nl].ml + L[nl].xl;
+    if (sz < best) {
+      best = sz;
+      *drv = nl;
+    }
+    ++nl;
+  }
+  return nl;
+}
+
+__device__ __forceinline__ void emit_tuples(const MatchArgs &A, const DevPlan &P, const int32_t *f, int kind,
+                                            const int32_t *cand, uint32_t c, int lane) {
+  unsigned long long base = 0;
+  if (lane == 0) base = atomicAdd(&A.cnt[kind ? CNT_TUP_REM : CNT_TUP_ADD], (unsigned long long)c);
+  base = __shfl_sync(kFull, base, 0);
+  int32_t *T = kind ? A.tup_rem : A.tup_add;
+  const uint64_t cap = kind ? A.tup_rem_cap : A.tup_add_cap;
+  const int k = A.k;
+  for (uint32_t i = lane; i < c; i += 32) {
+    if (base + i >= cap) break;
+    int32_t *t = T + (base + i) * (uint64_t)k;
+    for (int p = 0; p < k - 1; ++p) t[P.order[p]] = f[p];
+    t[P.order[k - 1]] = cand[i];
+  }
+}
+
+__device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int lane) {
+  if (lane == 0) {
+    if (acc.add) atomicAdd(&A.cnt[CNT_ADDED], acc.add);
+    if (acc.rem) atomicAdd(&A.cnt[CNT_REMOVED], acc.rem);
+    if (acc.hit) atomicAdd(&A.cnt[CNT_HIT], acc.hit);
+    if (acc.miss) atomicAdd(&A.cnt[CNT_MISS], acc.miss);
+  }
+}
+
+// Level 2 (BFS step): warp per unit.
+template <bool LIST>
+__global__ void __launch_bounds__(kBlock) k_level2(const MatchArgs A) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int32_t *buf = A.scratch + gw * A.scratch_stride;
+  Acc acc;
+  for (;;) {
+    unsigned long long u = 0;
+    if (lane == 0) u = atomicAdd(&A.cnt[CNT_CURSOR0], 1ull);
+    u = __shfl_sync(kFull, u, 0);
+    if ((int64_t)u >= A.n_units) break;
+    const Unit U = A.units[u];
+    const DevPlan &P = c_plans[U.plan];
+    const int32_t f[2] = {U.a, U.b};
+    if (A.k == 2) {  // single-edge query: the seed itself is the embedding
+      if (P.kind) acc.rem += 1;
+      else acc.add += 1;
+      if (LIST) {
+        if (lane == 0) {
+          const unsigned long long base = atomicAdd(&A.cnt[P.kind ? CNT_TUP_REM : CNT_TUP_ADD], 1ull);
+          int32_t *T = P.kind ? A.tup_rem : A.tup_add;
+          if (base < (P.kind ? A.tup_rem_cap : A.tup_add_cap)) {
+            T[base * 2 + P.order[0]] = U.a;
+            T[base * 2 + P.order[1]] = U.b;
+          }
+        }
+      }
+      continue;
+    }
+    const LevelPlan &L2 = P.lv[2];
+    LRef L[7];
+    int drv;
+    const int nl = gather_lists(A, L2, f, L, &drv, acc);
+    int32_t excl[2];
+    int nex = 0;
+    for (int i = 0; i < L2.ninj; ++i) excl[nex++] = f[L2.inj[i]];
+    if (A.k == 3 && !LIST) {
+      const uint32_t c = warp_isect<false>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, nullptr, lane);
+      if (P.kind) acc.rem += c;
+      else acc.add += c;
+      continue;
+    }
+    const uint32_t c = warp_isect<true>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, buf, lane);
+    __syncwarp();
+    if (A.k == 3) {  // LIST
+      if (P.kind) acc.rem += c;
+      else acc.add += c;
+      emit_tuples(A, P, f, P.kind, buf, c, lane);
+      __syncwarp();
+      continue;
+    }
+    unsigned long long off = 0;
+    if (lane == 0 && c) off = atomicAdd(&A.cnt[CNT_F2], (unsigned long long)c);
+    off = __shfl_sync(kFull, off, 0);
+    if (off + c > (unsigned long long)A.f2_cap) {
+      if (lane == 0) atomicOr(&A.cnt[CNT_OVERFLOW], 1ull);
+      continue;
+    }
+    int32_t *f2c = reinterpret_cast<int32_t *>(A.f2);
+    int32_t *f2u = f2c + A.f2_cap;
+    for (uint32_t i = lane; i < c; i += 32) {
+      f2c[off + i] = buf[i];
+      f2u[off + i] = (int32_t)u;
+    }
+    if (lane == 0) A.useg[u] = make_int2((int)off, (int)c);
+    __syncwarp();
+  }
+  flush(A, acc, lane);
+}
+
+// Levels 3..k-1 (DFS): warp per level-2 frontier entry.
+template <bool LIST>
+__global__ void __launch_bounds__(kBlock) k_extend(const MatchArgs A) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int32_t *stack = A.scratch + gw * A.scratch_stride;  // buffer for position p: stack + (p - 3) * dcap
+  const int k = A.k;
+  int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
+  const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
+  const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
+  const int32_t *f2u = f2c + A.f2_cap;
+  Acc acc;
+  for (;;) {
+    unsigned long long e = 0;
+    if (lane == 0) e = atomicAdd(&A.cnt[CNT_CURSOR1], 1ull);
+    e = __shfl_sync(kFull, e, 0);
+    if ((int64_t)e >= n_f2) break;
+    const int32_t ui = f2u[e];
+    const Unit U = A.units[ui];
+    const DevPlan &P = c_plans[U.plan];
+    const int2 seg = A.useg[ui];
+    int32_t f[GCSM_MAXK];
+    f[0] = U.a;
+    f[1] = U.b;
+    f[2] = f2c[e];
+    const int32_t *set[GCSM_MAXK];
+    uint32_t sz[GCSM_MAXK], it[GCSM_MAXK];
+    set[2] = f2c + seg.x;
+    sz[2] = (uint32_t)seg.y;
+    int lvl = 2;   // deepest position with a chosen element
+    bool descend = true;
+    for (;;) {
+      if (descend) {
+        const int p = lvl + 1;  // compute candidates of position p
+        const LevelPlan &Lp = P.lv[p];
+        LRef L[7];
+        int drv;
+        const int nl = gather_lists(A, Lp, f, L, &drv, acc);
+        int32_t excl[GCSM_MAXK];
+        int nex = 0;
+        for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
+        const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
+        const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
+        if (p == k - 1) {
+          uint32_t c;
+          if (LIST) {
+            c = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, lastbuf, lane);
+            __syncwarp();
+            emit_tuples(A, P, f, P.kind, lastbuf, c, lane);
+            __syncwarp();
+          } else {
+            c = warp_isect<false>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, nullptr, lane);
+          }
+          if (P.kind) acc.rem += c;
+          else acc.add += c;
+          descend = false;
+        } else {
+          int32_t *out = stack + (int64_t)(p - 3) * A.dcap;
+          sz[p] = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, out, lane);
+          __syncwarp();
+          set[p] = out;
+          it[p] = 0;
+          lvl = p;
+          descend = false;
+        }
+      }
+      // choose the next element at the deepest open position (>= 3)
+      while (lvl >= 3 && it[lvl] == sz[lvl]) --lvl;
+      if (lvl < 3) break;
+      f[lvl] = set[lvl][it[lvl]++];
+      descend = true;
+    }
+    (void)lvl;
+  }
+  flush(A, acc, lane);
+}
+
+__global__ void k_patch(VDesc *vdesc, const int64_t *idx, const VDesc *val, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    vdesc[idx[i]] = val[i];
+}
+
+}  // namespace
+
+cudaError_t upload_plans(const DevPlan *plans, int n, cudaStream_t s) {
+  return cudaMemcpyToSymbolAsync(c_plans, plans, sizeof(DevPlan) * (size_t)n, 0, cudaMemcpyHostToDevice, s);
+}
+
+int match_grid(int device, int *warps_total) {
+  int sms = 0, occ = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false>, kBlock, 0);
+  int occ2 = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_level2<false>, kBlock, 0);
+  if (occ2 < occ) occ = occ2;
+  if (occ < 1) occ = 1;
+  const int grid = sms * occ;
+  if (warps_total) *warps_total = grid * kWarps;
+  return grid;
+}
+
+cudaError_t launch_level2(const MatchArgs &a, int grid, cudaStream_t s) {
+  if (a.listing) k_level2<true><<<grid, kBlock, 0, s>>>(a);
+  else k_level2<false><<<grid, kBlock, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_extend(const MatchArgs &a, int grid, cudaStream_t s) {
+  if (a.listing) k_extend<true><<<grid, kBlock, 0, s>>>(a);
+  else k_extend<false><<<grid, kBlock, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_patch_vdesc(VDesc *vdesc, const int64_t *idx, const VDesc *val, int64_t n, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  int grid = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  k_patch<<<grid, 256, 0, s>>>(vdesc, idx, val, n);
+  return cudaGetLastError();
+}
+
+}  // namespace gcsm

@@ -1,0 +1,336 @@
+// store.cpp — host dynamic-graph store (§V-A; see store.h).
+#include "store.h"
+
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstring>
+
+namespace gcsm {
+
+static inline uint32_t round4(uint64_t x) { return (uint32_t)((x + 3) & ~uint64_t(3)); }
+
+HostStore::~HostStore() {
+  for (auto &c : chunks_)
+    if (c.host) cudaFreeHost(c.host);
+  if (overlay_.host) cudaFreeHost(overlay_.host);
+}
+
+bool HostStore::new_chunk(size_t bytes, Chunk &c) {
+  void *h = nullptr;
+  if (cudaHostAlloc(&h, bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) return false;
+  void *d = nullptr;
+  if (cudaHostGetDevicePointer(&d, h, 0) != cudaSuccess) {
+    cudaFreeHost(h);
+    return false;
+  }
+  c.host = (char *)h;
+  c.dev = (char *)d;
+  c.size = bytes;
+  c.used = 0;
+  return true;
+}
+
+const int32_t *HostStore::dev_ptr(const int32_t *host) const {
+  if (!host) return nullptr;
+  const char *p = (const char *)host;
+  for (const auto &c : chunks_)
+    if (p >= c.host && p < c.host + c.size) return (const int32_t *)(c.dev + (p - c.host));
+  if (overlay_.host && p >= overlay_.host && p < overlay_.host + overlay_.size)
+    return (const int32_t *)(overlay_.dev + (p - overlay_.host));
+  return nullptr;
+}
+
+int32_t *HostStore::alloc_list(uint32_t capacity, bool *cuda_err) {
+  const size_t bytes = (size_t)capacity * 4;
+  if (chunks_.empty() || chunks_.back().used + bytes > chunks_.back().size) {
+    Chunk c;
+    size_t sz = std::max<size_t>((size_t)256 << 20, 4 * bytes);
+    if (!new_chunk(sz, c)) {
+      *cuda_err = true;
+      return nullptr;
+    }
+    chunks_.push_back(c);
+  }
+  Chunk &c = chunks_.back();
+  int32_t *p = (int32_t *)(c.host + c.used);
+  c.used += bytes;  // capacities are multiples of 4 ints: 16-byte alignment kept
+  return p;
+}
+
+std::string HostStore::init(int32_t n_, const int64_t *rp, const int32_t *col, const int32_t *labels, int threads_,
+                            bool *cuda_err) {
+  *cuda_err = false;
+  n = n_;
+  threads = std::max(1, threads_);
+  if (n < 1) return "n must be >= 1";
+  if (!rp || (rp[n] > 0 && !col)) return "row_ptr/col is NULL";
+  if (rp[0] != 0) return "row_ptr[0] must be 0";
+  for (int32_t v = 0; v < n; ++v)
+    if (rp[v + 1] < rp[v]) return "row_ptr is not monotone";
+  if (labels)
+    for (int32_t v = 0; v < n; ++v)
+      if (labels[v] < 0 || labels[v] > 65535) return "label out of [0, 65535]";
+  // rows: in range, strictly ascending (no duplicates), no self loops; symmetric
+  std::atomic<int> bad{0};
+  parallel_for(threads, n, [&](int, int64_t lo, int64_t hi) {
+    for (int64_t v = lo; v < hi && !bad.load(std::memory_order_relaxed); ++v) {
+      for (int64_t e = rp[v]; e < rp[v + 1]; ++e) {
+        const int32_t w = col[e];
+        if (w < 0 || w >= n) { bad = 1; break; }
+        if (w == v) { bad = 2; break; }
+        if (e > rp[v] && col[e - 1] >= w) { bad = 3; break; }
+        if (!std::binary_search(col + rp[w], col + rp[w + 1], (int32_t)v)) { bad = 4; break; }
+      }
+    }
+  });
+  switch (bad.load()) {
+    case 1: return "column id out of range";
+    case 2: return "self loop in the graph";
+    case 3: return "row not strictly ascending (unsorted or duplicate)";
+    case 4: return "graph is not symmetric";
+    default: break;
+  }
+  lst.assign(n, nullptr);
+  len.assign(n, 0);
+  cap.assign(n, 0);
+  uidx.assign(n, -1);
+  if (labels) {
+    lab.resize(n);
+    for (int32_t v = 0; v < n; ++v) lab[v] = (uint16_t)labels[v];
+  }
+  uint64_t total = 0;
+  maxdeg = 0;
+  for (int32_t v = 0; v < n; ++v) {
+    const uint64_t d = (uint64_t)(rp[v + 1] - rp[v]);
+    len[v] = (uint32_t)d;
+    cap[v] = d ? round4(std::max<uint64_t>(4, 2 * d)) : 0;  // double the initial size
+    total += cap[v];
+    maxdeg = std::max<uint32_t>(maxdeg, (uint32_t)d);
+  }
+  edges2 = (uint64_t)rp[n];
+  deg_hist.assign((size_t)maxdeg + 1, 0);
+  for (int32_t v = 0; v < n; ++v) deg_hist[len[v]]++;
+  Chunk c;
+  if (!new_chunk(total * 4 + ((size_t)64 << 20), c)) {
+    *cuda_err = true;
+    return "cudaHostAlloc of the pinned store failed";
+  }
+  chunks_.push_back(c);
+  size_t off = 0;
+  for (int32_t v = 0; v < n; ++v) {
+    if (cap[v]) {
+      lst[v] = (int32_t *)(chunks_[0].host + off);
+      off += (size_t)cap[v] * 4;
+    }
+  }
+  chunks_[0].used = off;
+  parallel_for(threads, n, [&](int, int64_t lo, int64_t hi) {
+    for (int64_t v = lo; v < hi; ++v)
+      if (len[v]) std::memcpy(lst[v], col + rp[v], (size_t)len[v] * 4);
+  });
+  return "";
+}
+
+bool HostStore::has_edge(int32_t u, int32_t v) const {
+  if (len[u] > len[v]) std::swap(u, v);
+  return std::binary_search(lst[u], lst[u] + len[u], v);
+}
+
+std::string HostStore::normalize(int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del) {
+  if (n_ins < 0 || n_del < 0) return "negative batch size";
+  if ((n_ins && !ins) || (n_del && !del)) return "batch pointer is NULL";
+  auto keys = [&](int64_t m, const int32_t *e, std::vector<uint64_t> &out) -> std::string {
+    out.resize(m);
+    for (int64_t i = 0; i < m; ++i) {
+      int32_t u = e[2 * i], v = e[2 * i + 1];
+      if (u < 0 || v < 0 || u >= n || v >= n) return "vertex id out of range";
+      if (u == v) return "self loop in batch";
+      if (u > v) std::swap(u, v);
+      out[i] = ((uint64_t)(uint32_t)u << 32) | (uint32_t)v;
+    }
+    std::sort(out.begin(), out.end());
+    out.erase(std::unique(out.begin(), out.end()), out.end());
+    return "";
+  };
+  std::vector<uint64_t> ki, kd;
+  std::string err = keys(n_ins, ins, ki);
+  if (!err.empty()) return err;
+  err = keys(n_del, del, kd);
+  if (!err.empty()) return err;
+  for (size_t i = 0, j = 0; i < ki.size() && j < kd.size();) {
+    if (ki[i] == kd[j]) return "edge both inserted and deleted";
+    if (ki[i] < kd[j]) ++i;
+    else ++j;
+  }
+  // --- no mutation before this point ---
+  I.clear();
+  D.clear();
+  dropped = 0;
+  for (uint64_t key : ki) {
+    if (has_edge((int32_t)(key >> 32), (int32_t)(key & 0xffffffffu))) ++dropped;
+    else I.push_back(key);
+  }
+  for (uint64_t key : kd) {
+    if (has_edge((int32_t)(key >> 32), (int32_t)(key & 0xffffffffu))) D.push_back(key);
+    else ++dropped;
+  }
+  // directed pairs grouped by source
+  auto directed = [](const std::vector<uint64_t> &E) {
+    std::vector<uint64_t> d;
+    d.reserve(2 * E.size());
+    for (uint64_t key : E) {
+      d.push_back(key);
+      d.push_back(((key & 0xffffffffu) << 32) | (key >> 32));
+    }
+    std::sort(d.begin(), d.end());
+    return d;
+  };
+  const std::vector<uint64_t> di = directed(I), dd = directed(D);
+  U.clear();
+  for (uint64_t x : di) U.push_back((int32_t)(x >> 32));
+  for (uint64_t x : dd) U.push_back((int32_t)(x >> 32));
+  std::sort(U.begin(), U.end());
+  U.erase(std::unique(U.begin(), U.end()), U.end());
+  for (size_t i = 0; i < U.size(); ++i) uidx[U[i]] = (int32_t)i;
+  ins_off.assign(U.size() + 1, 0);
+  del_off.assign(U.size() + 1, 0);
+  ins_val.resize(di.size());
+  del_val.resize(dd.size());
+  for (size_t i = 0; i < di.size(); ++i) {
+    ins_off[uidx[(int32_t)(di[i] >> 32)] + 1]++;
+    ins_val[i] = (int32_t)(di[i] & 0xffffffffu);
+  }
+  for (size_t i = 0; i < dd.size(); ++i) {
+    del_off[uidx[(int32_t)(dd[i] >> 32)] + 1]++;
+    del_val[i] = (int32_t)(dd[i] & 0xffffffffu);
+  }
+  for (size_t i = 0; i < U.size(); ++i) {
+    ins_off[i + 1] += ins_off[i];
+    del_off[i + 1] += del_off[i];
+  }
+  return "";
+}
+
+bool HostStore::build_overlay(bool *cuda_err) {
+  *cuda_err = false;
+  const size_t nu = U.size();
+  s_ptr.assign(nu, nullptr);
+  s_len.assign(nu, 0);
+  std::vector<size_t> off(nu + 1, 0);
+  for (size_t i = 0; i < nu; ++i) {
+    const bool has_del = del_off[i + 1] > del_off[i];
+    off[i + 1] = off[i] + (has_del ? round4(len[U[i]]) : 0);
+  }
+  const size_t bytes = off[nu] * 4 + 64;
+  if (overlay_.size < bytes) {
+    if (overlay_.host) cudaFreeHost(overlay_.host);
+    overlay_ = Chunk();
+    if (!new_chunk(std::max<size_t>(bytes * 2, (size_t)16 << 20), overlay_)) {
+      *cuda_err = true;
+      return false;
+    }
+  }
+  maxdeg_new = 0;
+  std::vector<uint32_t> newdeg(nu);
+  parallel_for(threads, (int64_t)nu, [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      const int32_t x = U[i];
+      const int32_t *dl = del_val.data() + del_off[i];
+      const uint32_t nd = del_off[i + 1] - del_off[i];
+      if (nd == 0) {
+        s_ptr[i] = lst[x];
+        s_len[i] = len[x];
+      } else {
+        int32_t *out = (int32_t *)(overlay_.host) + off[i];
+        const int32_t *e = std::set_difference(lst[x], lst[x] + len[x], dl, dl + nd, out);
+        s_ptr[i] = out;
+        s_len[i] = (uint32_t)(e - out);
+      }
+      newdeg[i] = s_len[i] + (ins_off[i + 1] - ins_off[i]);
+    }
+  });
+  for (size_t i = 0; i < nu; ++i) maxdeg_new = std::max(maxdeg_new, newdeg[i]);
+  return true;
+}
+
+HList HostStore::view(int32_t v, int vw) const {
+  const int32_t i = uidx[v];
+  if (i < 0) return HList{lst[v], len[v], nullptr, 0};
+  HList h{s_ptr[i], s_len[i], nullptr, 0};
+  if (vw == VIEW_NEW) {
+    h.b = ins_val.data() + ins_off[i];
+    h.nb = ins_off[i + 1] - ins_off[i];
+  } else if (vw == VIEW_OLD) {
+    h.b = del_val.data() + del_off[i];
+    h.nb = del_off[i + 1] - del_off[i];
+  }
+  return h;
+}
+
+uint32_t HostStore::view_len(int32_t v, int vw) const {
+  const int32_t i = uidx[v];
+  if (i < 0) return len[v];
+  if (vw == VIEW_NEW) return s_len[i] + ins_off[i + 1] - ins_off[i];
+  if (vw == VIEW_OLD) return s_len[i] + del_off[i + 1] - del_off[i];
+  return s_len[i];
+}
+
+void HostStore::merge() {
+  const size_t nu = U.size();
+  std::vector<int32_t *> target(nu, nullptr);
+  std::vector<uint32_t> newlen(nu), newcap(nu);
+  bool err = false;
+  for (size_t i = 0; i < nu; ++i) {
+    const int32_t x = U[i];
+    newlen[i] = s_len[i] + (ins_off[i + 1] - ins_off[i]);
+    newcap[i] = cap[x];
+    target[i] = lst[x];
+    if (newlen[i] > cap[x]) {  // a new array with double capacity
+      newcap[i] = round4(std::max<uint64_t>(4, 2ull * newlen[i]));
+      target[i] = alloc_list(newcap[i], &err);
+    }
+  }
+  parallel_for(threads, (int64_t)nu, [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      const int32_t x = U[i];
+      const int32_t *in = ins_val.data() + ins_off[i];
+      const uint32_t ni = ins_off[i + 1] - ins_off[i];
+      int32_t *t = target[i];
+      if (!t) continue;
+      if (t == lst[x] && s_ptr[i] == lst[x]) {
+        // in place, insertions only: merge from the back
+        int64_t a = (int64_t)s_len[i] - 1, b = (int64_t)ni - 1, w = (int64_t)newlen[i] - 1;
+        while (b >= 0) {
+          if (a >= 0 && t[a] > in[b]) t[w--] = t[a--];
+          else t[w--] = in[b--];
+        }
+      } else {
+        std::merge(s_ptr[i], s_ptr[i] + s_len[i], in, in + ni, t);
+      }
+    }
+  });
+  for (size_t i = 0; i < nu; ++i) {
+    const int32_t x = U[i];
+    deg_hist[len[x]]--;
+    if (newlen[i] >= deg_hist.size()) deg_hist.resize((size_t)newlen[i] + 1, 0);
+    deg_hist[newlen[i]]++;
+    edges2 += newlen[i];
+    edges2 -= len[x];
+    len[x] = newlen[i];
+    cap[x] = newcap[i];
+    lst[x] = target[i];
+  }
+  maxdeg = (uint32_t)deg_hist.size() - 1;
+  while (maxdeg > 0 && deg_hist[maxdeg] == 0) --maxdeg;
+}
+
+void HostStore::clear_batch() {
+  for (int32_t x : U) uidx[x] = -1;
+  U.clear();
+  I.clear();
+  D.clear();
+}
+
+}  // namespace gcsm

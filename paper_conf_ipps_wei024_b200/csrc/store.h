@@ -1,0 +1,76 @@
+// store.h — host dynamic-graph store (§V-A).
+//
+// The paper allocates one pinned, GPU-mapped array per vertex (cudaHostAlloc +
+// cudaHostGetDevicePointer), appends insertions, marks deletions as -v
+// and merges after matching. Here: one pinned mapped
+// arena (a few large cudaHostAlloc chunks, 16-byte aligned lists, 2x capacity
+// per list as P:270), and the batch is applied *out of place* as an overlay
+// for the updated vertices U: stable list S(x) = N(x) \ del(x) (written to a
+// pinned overlay area only when x has deletions), plus sorted ins(x) / del(x)
+// — so every view (S, N = S ∪ del, N' = S ∪ ins) is a pair of sorted arrays
+// (reading R13: no -v marks, vertex 0 is not ambiguous). Step ⑤ merges
+// S(x) ∪ ins(x) into x's array (in place when the capacity allows, else a
+// doubled relocation).
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "estimator.h"
+#include "internal.h"
+
+namespace gcsm {
+
+struct Chunk {
+  char *host = nullptr;
+  char *dev = nullptr;
+  size_t size = 0, used = 0;
+};
+
+class HostStore {
+ public:
+  ~HostStore();
+  // returns "" or an error message; *cuda_err set if the failure is a CUDA error
+  std::string init(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels, int threads,
+                   bool *cuda_err);
+
+  int32_t n = 0;
+  int threads = 1;
+  std::vector<int32_t *> lst;   // host address of each list (pinned, mapped)
+  std::vector<uint32_t> len, cap;
+  std::vector<uint16_t> lab;    // empty if unlabelled
+  uint32_t maxdeg = 0;
+  uint64_t edges2 = 0;          // Σ len
+
+  const int32_t *dev_ptr(const int32_t *host) const;  // device-visible address of a pinned host address
+
+  // ---- batch (steps ① / a0-a1) ----
+  // Validates and normalises; on EINVAL returns the message and mutates nothing.
+  std::string normalize(int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del);
+  bool build_overlay(bool *cuda_err);   // S(x) for x ∈ U with deletions
+  HList view(int32_t v, int view) const;
+  uint32_t view_len(int32_t v, int view) const;
+  void merge();                         // step ⑤
+  void clear_batch();
+
+  // batch state
+  std::vector<uint64_t> I, D;    // canonical keys (u << 32 | v), u < v, sorted
+  uint64_t dropped = 0;
+  std::vector<int32_t> U;        // updated vertices, ascending
+  std::vector<int32_t> uidx;     // vertex -> index in U, or -1 (size n)
+  std::vector<uint32_t> ins_off, del_off;  // size |U|+1, into ins_val / del_val
+  std::vector<int32_t> ins_val, del_val;
+  std::vector<const int32_t *> s_ptr;      // host address of S(x)
+  std::vector<uint32_t> s_len;
+  uint32_t maxdeg_new = 0;                 // max |N'(x)| over U
+  std::vector<uint64_t> deg_hist;          // vertices per degree (exact max degree)
+
+ private:
+  std::vector<Chunk> chunks_;
+  Chunk overlay_;
+  int32_t *alloc_list(uint32_t capacity, bool *cuda_err);
+  bool new_chunk(size_t bytes, Chunk &c);
+  bool has_edge(int32_t u, int32_t v) const;
+};
+
+}  // namespace gcsm

@@ -1,0 +1,98 @@
+"""CPU tests of the boundary: libgcsm.so loads, exports every symbol include/gcsm.h declares, and its pure-host
+logic (plan builder vs Fig. 2, LPT sharding) is right. No compute call needs a GPU here."""
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+import gcsm_inputs as gi
+import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def pkg():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_wei024_b200 as p
+    return p
+
+
+def header_symbols():
+    src = open(os.path.join(ROOT, "include", "gcsm.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(gcsm_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_exports_every_header_symbol(pkg):
+    lib = pkg._lib.load()
+    syms = header_symbols()
+    assert len(syms) >= 17
+    out = subprocess.run(["nm", "-D", "--defined-only", pkg._lib.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (gcsm_\w+)", out))
+    for s in syms:
+        assert s in exported, s
+        assert hasattr(lib, s)
+    assert sorted(pkg._lib.SYMBOLS) == syms
+
+
+def test_library_is_sm100a(pkg):
+    out = subprocess.run(["cuobjdump", "--list-elf", pkg._lib.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_plan_matches_fig2_and_oracle(pkg):
+    for name in ["diamond", "triangle", "c4", "k4", "house5u", "prism6", "k6", "star3"]:
+        k, qe, _ = gi.query(name)
+        a = pkg.plan_inspect(k, qe)
+        b = oracle.plan(k, qe)
+        assert np.array_equal(a["seed"], b["seed"])
+        assert np.array_equal(a["order"], b["order"])
+        assert np.array_equal(a["nb"], b["nb"])
+        for t in range(len(qe)):
+            for p in range(k):
+                nb = a["nb"][t, p]
+                ga = {int(a["order"][t, q]): (int(a["view"][0, t, p, i]), int(a["view"][1, t, p, i]))
+                      for i, q in enumerate(a["bq"][t, p, :nb])}
+                gb = {int(b["order"][t, q]): (int(b["view"][0, t, p, i]), int(b["view"][1, t, p, i]))
+                      for i, q in enumerate(b["bq"][t, p, :nb])}
+                assert ga == gb, (name, t, p)
+    # Fig. 2e: ΔM_4 of the diamond: order u1,u3,u0,u2; x2 ∈ S(x0) ∩ S(x1) ∩ N'(x3)
+    k, qe, _ = gi.query("diamond")
+    a = pkg.plan_inspect(k, qe)
+    assert a["order"][3].tolist() == [1, 3, 0, 2]
+    views = {int(a["order"][3, q]): int(a["view"][0, 3, 3, i]) for i, q in enumerate(a["bq"][3, 3, :3])}
+    assert views == {1: 0, 3: 2, 0: 0}
+
+
+def test_plan_rejects_bad_queries(pkg):
+    with pytest.raises(pkg.GcsmError):
+        pkg.plan_inspect(4, [(0, 1), (2, 3)])        # disconnected
+    with pytest.raises(pkg.GcsmError):
+        pkg.plan_inspect(3, [(0, 0), (1, 2)])        # self loop
+    with pytest.raises(pkg.GcsmError):
+        pkg.plan_inspect(9, [(i, i + 1) for i in range(8)])  # k > 8
+
+
+def test_shard_disjoint_cover_and_balance(pkg):
+    rng = np.random.default_rng(0)
+    cost = rng.integers(1, 10000, size=5000).astype(np.uint64)
+    for world in (1, 2, 4, 8):
+        r = pkg.shard(cost, world)
+        assert r.min() >= 0 and r.max() < world
+        loads = np.bincount(r, weights=cost.astype(float) + 1, minlength=world)
+        assert loads.max() <= loads.mean() + cost.max() + 1  # LPT bound
+        assert np.array_equal(r, pkg.shard(cost, world))      # deterministic
+
+
+def test_no_cpu_fallback(pkg):
+    torch = pytest.importorskip("torch")
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    w = gi.make_workload("C1", scale=6, n_edges=100, batch=8)
+    with pytest.raises(pkg.GcsmError) as ei:
+        pkg.Gcsm(w.n, w.row_ptr, w.col)
+    assert ei.value.name in ("GCSM_EDEVICE", "GCSM_ENOMEM")

@@ -1,0 +1,298 @@
+"""GPU parity: the CUDA path through the C ABI vs the oracle, bit-exact (integer counts, tuples, estimator sums).
+
+Sizes: small enough for the oracle to finish in seconds, large enough to span many warps/units, ragged tails,
+multi-segment lists (updated vertices), hub lists and the level-2 frontier; plus degenerate cases.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import gcsm_inputs as gi
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def G():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_wei024_b200 as pkg
+    return pkg
+
+
+def tuples_set(t):
+    return sorted(map(tuple, np.asarray(t).tolist()))
+
+
+def lib_run(G, n, rp, col, labels, name_or_q, batches, budget_frac=0.1, listing=False, **kw):
+    k, qe, ql = gi.query(name_or_q) if isinstance(name_or_q, str) else name_or_q
+    g = G.Gcsm(n, rp, col, labels, device=0, **kw)
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(int(4 * rp[-1] * budget_frac))
+    out = []
+    for ins, dele in batches:
+        if listing:
+            a, r, ta, tr = g.apply_batch_list(ins, dele, 1 << 18, 1 << 18)
+            out.append((a, r, tuples_set(ta), tuples_set(tr)))
+        else:
+            out.append(g.apply_batch(ins, dele))
+    st = g.stats()
+    rp2, col2 = g.export_csr()
+    g.close()
+    return out, st, (rp2, col2)
+
+
+def oracle_run(n, rp, col, labels, name_or_q, batches, listing=False):
+    k, qe, ql = gi.query(name_or_q) if isinstance(name_or_q, str) else name_or_q
+    out = []
+    for ins, dele in batches:
+        if listing:
+            (a, ta), (r, tr) = oracle.delta(n, rp, col, labels, k, qe, ql, ins, dele, listing=True, tuple_cap=1 << 18)
+            out.append((a, r, tuples_set(ta), tuples_set(tr)))
+        else:
+            out.append(oracle.delta(n, rp, col, labels, k, qe, ql, ins, dele))
+        I, D, _ = oracle.normalize_batch(n, rp, col, ins, dele)
+        rp, col = oracle.apply_batch(n, rp, col, I, D)
+    return out, (rp, col)
+
+
+# ------------------------------------------------------------------ C1 (BASELINE configs[0])
+
+@pytest.mark.parametrize("budget", [0.0, 0.1, 1.0])
+def test_c1_triangle_budgets(G, budget):
+    w = gi.make_workload("C1")
+    want, (rp1, col1) = oracle_run(w.n, w.row_ptr, w.col, None, "triangle", w.batches, listing=True)
+    got, st, (rp2, col2) = lib_run(G, w.n, w.row_ptr, w.col, None, "triangle", w.batches, budget, listing=True)
+    assert got == want
+    assert want[0][0] > 0
+    assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
+    if budget == 0:
+        assert st["hit_bytes"] == 0 and st["miss_bytes"] > 0
+    if budget == 1.0:
+        assert st["cached_vertices"] > 0
+
+
+# ------------------------------------------------------------------ fuzz
+
+FUZZ = ["edge", "wedge", "triangle", "path4", "c4", "diamond", "k4", "star3", "house5u", "k5", "prism6", "k4tri6"]
+
+
+@pytest.mark.parametrize("seed", range(36))
+def test_fuzz_small_graphs(G, seed):
+    rng = np.random.default_rng(1000 + seed)
+    n = int(rng.integers(8, 14))
+    n_, g0, ins, dele = gi.small_random_case(1000 + seed, n=n, p=float(rng.uniform(0.25, 0.7)),
+                                             n_ins=int(rng.integers(0, 7)), n_del=int(rng.integers(0, 7)))
+    name = FUZZ[seed % len(FUZZ)]
+    k, qe, _ = gi.query(name)
+    labels = ql = None
+    if seed % 3 == 1:
+        labels = rng.integers(0, 2, n).astype(np.int32)
+        ql = rng.integers(0, 2, k).astype(np.int32)
+    order = rng.permutation(k).astype(np.int32) if seed % 4 == 2 else None
+    rp, col = oracle.csr(n, g0)
+    want, _ = oracle_run(n, rp, col, labels, (k, qe, ql), [(ins, dele)], listing=True)
+    g = G.Gcsm(n, rp, col, labels, device=0)
+    g.set_query(k, qe, ql, order)
+    g.set_cache_budget([0, 64, 1 << 20][seed % 3])
+    a, r, ta, tr = g.apply_batch_list(ins, dele, 1 << 16, 1 << 16)
+    g.close()
+    assert (a, r, tuples_set(ta), tuples_set(tr)) == want[0]
+
+
+def test_degenerate_cases(G):
+    k, qe, _ = gi.query("triangle")
+    # empty batch; empty graph; complete graph built in one batch; all edges deleted
+    n = 7
+    E = [(i, j) for i in range(n) for j in range(i + 1, n)]
+    rp0, col0 = oracle.csr(n, np.zeros((0, 2), np.int32))
+    g = G.Gcsm(n, rp0, col0, device=0)
+    g.set_query(k, qe)
+    g.set_cache_budget(1 << 20)
+    assert g.apply_batch(np.zeros((0, 2)), np.zeros((0, 2))) == (0, 0)
+    assert g.apply_batch(E, []) == (n * (n - 1) * (n - 2), 0)
+    assert g.apply_batch([], E) == (0, n * (n - 1) * (n - 2))
+    # no-ops are dropped and counted (R8)
+    g.apply_batch([(0, 1)], [])
+    assert g.apply_batch([(0, 1), (1, 0)], [(2, 3)]) == (0, 0)
+    assert g.stats()["dropped"] == 2
+    # EINVAL leaves the graph unchanged
+    before = g.export_csr()
+    for ins, dele in [([(1, 1)], []), ([(0, 99)], []), ([(2, 4)], [(4, 2)])]:
+        with pytest.raises(G.GcsmError) as ei:
+            g.apply_batch(ins, dele)
+        assert ei.value.name == "GCSM_EINVAL"
+        after = g.export_csr()
+        assert all(np.array_equal(x, y) for x, y in zip(before, after))
+    g.close()
+    # apply before set_query -> ESTATE
+    g = G.Gcsm(n, rp0, col0, device=0)
+    with pytest.raises(G.GcsmError) as ei:
+        g.apply_batch([(0, 1)], [])
+    assert ei.value.name == "GCSM_ESTATE"
+    g.close()
+
+
+def test_bad_graph_rejected(G):
+    rp = np.array([0, 1, 1], np.int64)
+    col = np.array([1], np.int32)  # not symmetric
+    with pytest.raises(G.GcsmError) as ei:
+        G.Gcsm(2, rp, col, device=0)
+    assert ei.value.name == "GCSM_EINVAL"
+
+
+def test_list_truncation(G):
+    n = 6
+    E = [(i, j) for i in range(n) for j in range(i + 1, n)]
+    rp0, col0 = oracle.csr(n, np.zeros((0, 2), np.int32))
+    g = G.Gcsm(n, rp0, col0, device=0)
+    g.set_query(*gi.query("triangle")[:2])
+    with pytest.raises(G.GcsmError) as ei:
+        g.apply_batch_list(E, [], 5, 5)
+    assert ei.value.name == "GCSM_ETRUNC"
+    assert g.stats()["added"] == 120
+    g.close()
+
+
+# ------------------------------------------------------------------ streams (multi-batch state, store ① / ⑤)
+
+@pytest.mark.parametrize("name", ["diamond", "k4", "c4", "house5u"])
+def test_stream_of_mixed_batches(G, name):
+    w = gi.make_workload("C2", scale=11, n_edges=12000, batch=200)
+    batches = w.batches[:5]
+    want, (rp1, col1) = oracle_run(w.n, w.row_ptr, w.col, None, name, batches)
+    got, st, (rp2, col2) = lib_run(G, w.n, w.row_ptr, w.col, None, name, batches, 0.1)
+    assert got == want
+    assert any(a + r > 0 for a, r in want)
+    assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
+
+
+@pytest.mark.parametrize("order", [None, [3, 2, 1, 0], [2, 0, 3, 1]])
+def test_matching_order_invariance(G, order):
+    w = gi.make_workload("C2", scale=11, n_edges=12000, batch=300)
+    k, qe, _ = gi.query("diamond")
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, "diamond", w.batches[:2])
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    g.set_query(k, qe, None, order)
+    g.set_cache_budget(w.adj_bytes // 20)
+    assert [g.apply_batch(*b) for b in w.batches[:2]] == want
+    g.close()
+
+
+# ------------------------------------------------------------------ scaled configs C2 / C3
+
+@pytest.mark.parametrize("name", ["k4", "c4"])
+@pytest.mark.parametrize("budget", [0.0, 0.1, 1.0])
+def test_c2_shaped(G, name, budget):
+    w = gi.make_workload("C2", scale=16, n_edges=600_000, batch=1024, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    got, st, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, budget)
+    assert got == want
+
+
+@pytest.mark.parametrize("name", ["house5", "bowtie5", "k5e"])
+def test_c3_shaped_labelled(G, name):
+    w = gi.make_workload("C3", scale=14, n_edges=200_000, batch=1024, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, w.labels, name, w.batches)
+    got, st, _ = lib_run(G, w.n, w.row_ptr, w.col, w.labels, name, w.batches, 0.1)
+    assert got == want
+
+
+@pytest.mark.parametrize("name", ["prism6", "k4tri6", "k6"])
+def test_six_vertex_queries(G, name):
+    w = gi.make_workload("C2", scale=12, n_edges=40_000, batch=256, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    got, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.05)
+    assert got == want
+
+
+@pytest.mark.parametrize("r", [1, 2, 3])
+def test_star_closed_form_at_scale(G, r):
+    """SURVEY §8c degree closed form for K_{1,r}: added = Σ_U P(d',r) - P(s,r), removed = Σ_U P(d,r) - P(s,r)."""
+    w = gi.make_workload("C2", scale=18, n_edges=3_000_000, batch=4096, n_batches=2)
+    k = r + 1
+    qe = np.array([(0, i) for i in range(1, k)], np.int32)
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    g.set_query(k, qe)
+    g.set_cache_budget(w.adj_bytes // 10)
+    rp, col = w.row_ptr, w.col
+
+    def P(x):
+        out = np.ones_like(x, dtype=object)
+        for i in range(r):
+            out = out * (x - i)
+        return out
+
+    for ins, dele in w.batches:
+        I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+        rp1, col1 = oracle.apply_batch(w.n, rp, col, I, D)
+        rps, _ = oracle.stable_graph(w.n, rp, col, D)
+        U = np.unique(np.concatenate([I.ravel(), D.ravel()]))
+        d, d1, s = (np.diff(x)[U].astype(object) for x in (rp, rp1, rps))
+        want = (int((P(d1) - P(s)).sum()), int((P(d) - P(s)).sum()))
+        assert g.apply_batch(ins, dele) == want
+        rp, col = rp1, col1
+    g.close()
+
+
+# ------------------------------------------------------------------ estimator ② and packer ③ parity
+
+@pytest.mark.parametrize("name,labelled", [("diamond", False), ("k4", False), ("house5u", False), ("house5", True)])
+def test_estimator_and_cache_parity(G, name, labelled):
+    w = gi.make_workload("C3" if labelled else "C2", scale=12, n_edges=30_000, batch=256, n_batches=2)
+    labels = w.labels if labelled else None
+    k, qe, ql = gi.query(name)
+    seed = 0xBEEF
+    budget = w.adj_bytes // 25
+    g = G.Gcsm(w.n, w.row_ptr, w.col, labels, device=0, seed=seed)
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(budget)
+    rp, col = w.row_ptr, w.col
+    for t, (ins, dele) in enumerate(w.batches):
+        g.apply_batch(ins, dele)
+        st = g.stats()
+        e = oracle.estimate(w.n, rp, col, labels, k, qe, ql, ins, dele, seed=seed, batch_seq=t)
+        assert (st["n1"], st["max_degree"], st["walks"]) == (e["N1"], e["D"], e["M"])
+        ids, lev = g.estimates()
+        want_ids = np.nonzero(e["levcnt"].sum(1))[0]
+        assert np.array_equal(ids, want_ids)
+        assert np.array_equal(lev[:, :k - 2], e["levcnt"][want_ids])
+        # the cache: longest prefix of (estimate desc, id asc) whose 16-byte-aligned stable lists fit (R23)
+        I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+        rps, _ = oracle.stable_graph(w.n, rp, col, D)
+        sz = 16 * ((np.diff(rps) + 3) // 4)
+        assert np.array_equal(g.cached(), oracle.select_cache(e["est"], sz, budget & ~15))
+        rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+    g.close()
+
+
+# ------------------------------------------------------------------ multi-GPU sharding, emulated world on one GPU
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_emulated_world_sums(G, world):
+    w = gi.make_workload("C2", scale=13, n_edges=60_000, batch=512, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, "k4", w.batches)
+    tot = [[0, 0] for _ in w.batches]
+    units = 0
+    for rank in range(world):
+        got, st, _ = lib_run(G, w.n, w.row_ptr, w.col, None, "k4", w.batches, 0.1, rank=rank, world=world,
+                             local_counts=True)
+        for i, (a, r) in enumerate(got):
+            tot[i][0] += a
+            tot[i][1] += r
+    assert [tuple(x) for x in tot] == want
+
+
+def test_cache_policies_same_counts(G):
+    w = gi.make_workload("C2", scale=14, n_edges=150_000, batch=512, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, "k4", w.batches)
+    for pol in ("estimator", "degree", "none"):
+        got, st, _ = lib_run(G, w.n, w.row_ptr, w.col, None, "k4", w.batches, 0.05, cache_policy=pol)
+        assert got == want, pol
+        if pol == "none":
+            assert st["hit_bytes"] == 0 or st["cached_vertices"] == 0
