@@ -101,6 +101,7 @@ typedef struct {
   uint64_t cache_bytes;     /* bytes of cached lists (<= budget) */
   uint64_t hit_bytes;       /* list bytes the kernels read from the HBM cache (algorithmic, §8d) */
   uint64_t miss_bytes;      /* list bytes the kernels read zero-copy from host memory */
+  uint64_t delta_bytes;     /* list bytes read from the device-resident ins/del segments of updated vertices */
   uint64_t frontier;        /* level-2 partial matches materialised */
   uint64_t kernel_launches; /* this library's kernels launched in the last batch */
   uint64_t added, removed;  /* last batch's global counts */

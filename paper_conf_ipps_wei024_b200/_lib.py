@@ -31,7 +31,7 @@ class Options(ctypes.Structure):
 class Stats(ctypes.Structure):
     _fields_ = [(name, ctypes.c_uint64) for name in
                 ["batches", "n_ins", "n_del", "dropped", "units", "n1", "walks", "max_degree", "cached_vertices",
-                 "cache_bytes", "hit_bytes", "miss_bytes", "frontier", "kernel_launches", "added", "removed"]] + \
+                 "cache_bytes", "hit_bytes", "miss_bytes", "delta_bytes", "frontier", "kernel_launches", "added", "removed"]] + \
               [(name, ctypes.c_double) for name in
                ["ms_normalize", "ms_estimate", "ms_pack", "ms_copy", "ms_match", "ms_allreduce", "ms_merge",
                 "ms_total"]]

@@ -597,6 +597,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   st.removed = ctx->h_cnt[CNT_REMOVED];
   st.hit_bytes = ctx->h_cnt[CNT_HIT];
   st.miss_bytes = ctx->h_cnt[CNT_MISS];
+  st.delta_bytes = ctx->h_cnt[CNT_DELTA];
   st.frontier = ctx->h_cnt[CNT_F2];
   st.kernel_launches = launches;
   bool trunc = false;

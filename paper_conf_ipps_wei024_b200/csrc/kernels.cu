@@ -46,7 +46,7 @@ struct LRef {
 };
 
 struct Acc {
-  unsigned long long add = 0, rem = 0, hit = 0, miss = 0;
+  unsigned long long add = 0, rem = 0, hit = 0, miss = 0, delta = 0;
 };
 
 __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc) {
@@ -71,7 +71,7 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
   const char *p = reinterpret_cast<const char *>(r.m);
   if (p >= A.cache_lo && p < A.cache_hi) acc.hit += 4ull * r.ml;
   else acc.miss += 4ull * r.ml;
-  acc.hit += 4ull * r.xl;
+  acc.delta += 4ull * r.xl;
   return r;
 }
 
@@ -173,6 +173,7 @@ __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int la
     if (acc.rem) atomicAdd(&A.cnt[CNT_REMOVED], acc.rem);
     if (acc.hit) atomicAdd(&A.cnt[CNT_HIT], acc.hit);
     if (acc.miss) atomicAdd(&A.cnt[CNT_MISS], acc.miss);
+    if (acc.delta) atomicAdd(&A.cnt[CNT_DELTA], acc.delta);
   }
 }
 

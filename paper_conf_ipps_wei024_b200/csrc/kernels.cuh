@@ -18,6 +18,7 @@ enum Counter {
   CNT_TUP_REM = 7,
   CNT_CURSOR0 = 8,  // work cursors (reset per launch)
   CNT_CURSOR1 = 9,
+  CNT_DELTA = 10,   // list bytes served from the device delta segments (ins/del of U)
   CNT_N = 16
 };
 
