@@ -156,7 +156,7 @@ CONFIGS = {
 
 
 def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = None,
-                  batch: int | None = None, n_batches: int | None = None) -> Workload:
+                  batch: int | None = None, n_batches: int | None = None, n_stream: int | None = None) -> Workload:
     """Build G_0 and the batch stream of a config (optionally scaled down for tests)."""
     cfg = dict(CONFIGS[name])
     idx = int(name[1:])
@@ -169,6 +169,8 @@ def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = 
         cfg["n_edges"] = n_edges
     if batch is not None:
         cfg["batch"] = batch
+    if n_stream is not None:
+        cfg["stream"] = n_stream
     a, b, c = cfg["abc"]
     uv = rmat_edges(cfg["scale"], cfg["n_edges"], a, b, c, seed, cfg["id_limit"])
     n = cfg["id_limit"] if cfg["id_limit"] else (1 << cfg["scale"])

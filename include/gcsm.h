@@ -102,14 +102,19 @@ typedef struct {
   uint64_t hit_bytes;       /* list bytes the kernels read from the HBM cache (algorithmic, §8d) */
   uint64_t miss_bytes;      /* list bytes the kernels read zero-copy from host memory */
   uint64_t delta_bytes;     /* list bytes read from the device-resident ins/del segments of updated vertices */
+  uint64_t hit_bytes_ext, miss_bytes_ext, delta_bytes_ext; /* the same, k_extend only (levels >= 3) */
   uint64_t frontier;        /* level-2 partial matches materialised */
   uint64_t kernel_launches; /* this library's kernels launched in the last batch */
+  uint64_t h2d_bytes;       /* bytes copied host -> device in the batch (cache DMA, descriptors, deltas, units) */
+  uint64_t d2h_bytes;       /* bytes copied device -> host (counters, tuples) */
   uint64_t added, removed;  /* last batch's global counts */
   double ms_normalize;      /* (1) normalise + overlay + units */
   double ms_estimate;       /* (2) */
   double ms_pack;           /* (3) host packing */
   double ms_copy;           /* (3) H2D: cache DMA + descriptors + deltas */
   double ms_match;          /* (4) kernels (CUDA events) */
+  double ms_level2;         /* (4) k_level2 launches only (CUDA events) */
+  double ms_extend;         /* (4) k_extend launches only (CUDA events) */
   double ms_allreduce;      /* (4b) */
   double ms_merge;          /* (5) */
   double ms_total;          /* whole gcsm_apply_batch, host wall clock */
@@ -192,6 +197,13 @@ gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levc
 
 /* Last batch's cached vertex set (step 3), ascending. */
 gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out);
+
+/* Roofline denominators the hot path needs and MEASURED_PEAKS.json lacks
+ * (SURVEY §8d): best-of-5 GB/s of (i) a zero-copy streaming-read kernel over a
+ * mapped pinned buffer of `bytes`, (ii) one cudaMemcpyAsync H2D of it, and
+ * (iii) an HBM device copy (read + write bytes). device -1 = current. */
+gcsm_status gcsm_measure_host_link(int32_t device, uint64_t bytes, double *zero_copy_gbps, double *dma_h2d_gbps,
+                                   double *hbm_copy_gbps);
 
 /* Pure host, no device: the per-term plan the library would build for a query
  * (for the Fig. 2 structural test). Arrays as in gcsm_set_query; outputs:

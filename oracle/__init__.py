@@ -61,6 +61,8 @@ def _load():
         lib.ivm_run.restype = ctypes.c_int
         lib.ivm_run.argtypes = [I32, I32, P, P, P, P, P, P, P, I32, I32, P, P, P, I64, P, I32, U64, U64, I64, I64,
                                 P, P, P]
+        lib.o_apply.restype = ctypes.c_int
+        lib.o_apply.argtypes = [I32, P, P, I64, P, I64, P, P, P]
         lib.o_binom_many.restype = None
         lib.o_binom_many.argtypes = [U64, I64, ctypes.c_double, I64, P]
         _lib = lib
@@ -97,9 +99,8 @@ def csr(n, uv):
     dst = np.concatenate([uv[:, 1], uv[:, 0]])
     order = np.lexsort((dst, src))
     src, dst = src[order], dst[order]
-    rp = np.zeros(n + 1, dtype=np.int64)
-    np.add.at(rp, src + 1, 1)
-    return np.cumsum(rp).astype(np.int64), dst.astype(np.int32)
+    rp = np.concatenate([[0], np.cumsum(np.bincount(src, minlength=n))]).astype(np.int64)
+    return rp, dst.astype(np.int32)
 
 
 def _keys(uv):
@@ -110,6 +111,17 @@ def _keys(uv):
 def _unkey(keys):
     keys = np.asarray(keys, dtype=np.int64)
     return np.stack([keys >> 32, keys & 0xFFFFFFFF], axis=1).astype(np.int32)
+
+
+def has_edges(rp, col, uv):
+    """Membership of each pair (u, v) in the graph (binary search of row u)."""
+    uv = np.asarray(uv, dtype=np.int64).reshape(-1, 2)
+    out = np.zeros(len(uv), dtype=bool)
+    for i, (u, v) in enumerate(uv.tolist()):
+        row = col[rp[u]:rp[u + 1]]
+        j = np.searchsorted(row, v)
+        out[i] = j < len(row) and row[j] == v
+    return out
 
 
 def normalize_batch(n, rp, col, ins, dele):
@@ -130,15 +142,25 @@ def normalize_batch(n, rp, col, ins, dele):
     ki, kd = np.unique(_keys(ins)), np.unique(_keys(dele))
     if len(np.intersect1d(ki, kd)):
         raise ValueError("edge both inserted and deleted")
-    existing = _keys(edges_of(rp, col))
-    ki_new = np.setdiff1d(ki, existing)
-    kd_real = np.intersect1d(kd, existing)
+    ei, ed = has_edges(rp, col, _unkey(ki)), has_edges(rp, col, _unkey(kd))
+    ki_new, kd_real = ki[~ei], kd[ed]
     dropped = (len(ki) - len(ki_new)) + (len(kd) - len(kd_real))
     return _unkey(ki_new), _unkey(kd_real), int(dropped)
 
 
 def apply_batch(n, rp, col, I, D):
-    """a7: CSR of G_{t+1} = (E \\ D) ∪ I."""
+    """a7: CSR of G_{t+1} = (E \\ D) ∪ I for a normalised batch (row-by-row, oracle.c)."""
+    I = _i32(np.asarray(I).reshape(-1, 2))
+    D = _i32(np.asarray(D).reshape(-1, 2))
+    rp2 = np.zeros(n + 1, np.int64)
+    col2 = np.zeros(int(rp[-1]) + 2 * len(I) - 2 * len(D), np.int32)
+    _load().o_apply(n, _p(np.ascontiguousarray(rp, dtype=np.int64)), _p(np.ascontiguousarray(col, dtype=np.int32)),
+                    len(I), _p(I), len(D), _p(D), _p(rp2), _p(col2))
+    return rp2, col2
+
+
+def apply_batch_setalgebra(n, rp, col, I, D):
+    """The same as apply_batch by plain numpy set algebra on edge keys (small graphs; pins apply_batch)."""
     e = _keys(edges_of(rp, col))
     e = np.union1d(np.setdiff1d(e, _keys(D)), _keys(I))
     return csr(n, _unkey(e))
@@ -146,8 +168,7 @@ def apply_batch(n, rp, col, I, D):
 
 def stable_graph(n, rp, col, D):
     """CSR of the stable edge set S = E ∩ E' = E \\ D (§8 notation)."""
-    e = np.setdiff1d(_keys(edges_of(rp, col)), _keys(D))
-    return csr(n, _unkey(e))
+    return apply_batch(n, rp, col, np.zeros((0, 2), np.int32), D)
 
 
 # ------------------------------------------------------------------ counts

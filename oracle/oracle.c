@@ -119,6 +119,50 @@ static void run_threads(int threads, void *(*fn)(void *), void **args) {
   for (int t = 0; t < threads; ++t) pthread_join(th[t], NULL);
 }
 
+/* ================================================================== graph update */
+/*
+ * G_{t+1} = (E \ D) ∪ I row by row (reading R8): for every vertex,
+ * its list minus the deleted neighbours plus the inserted ones, sorted.
+ * ins/del: canonical pairs already normalised (I ∩ E = ∅, D ⊆ E). The caller
+ * sizes out_col as rp[n] + 2|I| - 2|D|.
+ */
+static int cmp_i32(const void *a, const void *b) {
+  int32_t x = *(const int32_t *)a, y = *(const int32_t *)b;
+  return x < y ? -1 : x > y;
+}
+
+int o_apply(int32_t n, const int64_t *rp, const int32_t *col, int64_t n_ins, const int32_t *ins, int64_t n_del,
+            const int32_t *del, int64_t *out_rp, int32_t *out_col) {
+  /* per-vertex change lists */
+  int64_t *ci = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+  int64_t *cd = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+  for (int64_t e = 0; e < n_ins; ++e) { ci[ins[2 * e] + 1]++; ci[ins[2 * e + 1] + 1]++; }
+  for (int64_t e = 0; e < n_del; ++e) { cd[del[2 * e] + 1]++; cd[del[2 * e + 1] + 1]++; }
+  for (int32_t v = 0; v < n; ++v) { ci[v + 1] += ci[v]; cd[v + 1] += cd[v]; }
+  int32_t *vi = (int32_t *)malloc(sizeof(int32_t) * (size_t)(2 * n_ins + 1));
+  int32_t *vd = (int32_t *)malloc(sizeof(int32_t) * (size_t)(2 * n_del + 1));
+  int64_t *pi = (int64_t *)malloc(sizeof(int64_t) * ((size_t)n + 1));
+  int64_t *pd = (int64_t *)malloc(sizeof(int64_t) * ((size_t)n + 1));
+  memcpy(pi, ci, sizeof(int64_t) * ((size_t)n + 1));
+  memcpy(pd, cd, sizeof(int64_t) * ((size_t)n + 1));
+  for (int64_t e = 0; e < n_ins; ++e) { vi[pi[ins[2 * e]]++] = ins[2 * e + 1]; vi[pi[ins[2 * e + 1]]++] = ins[2 * e]; }
+  for (int64_t e = 0; e < n_del; ++e) { vd[pd[del[2 * e]]++] = del[2 * e + 1]; vd[pd[del[2 * e + 1]]++] = del[2 * e]; }
+  out_rp[0] = 0;
+  for (int32_t v = 0; v < n; ++v) {
+    int64_t w = out_rp[v];
+    for (int64_t e = rp[v]; e < rp[v + 1]; ++e) {
+      int gone = 0;
+      for (int64_t j = cd[v]; j < cd[v + 1]; ++j) if (vd[j] == col[e]) gone = 1;
+      if (!gone) out_col[w++] = col[e];
+    }
+    for (int64_t j = ci[v]; j < ci[v + 1]; ++j) out_col[w++] = vi[j];
+    qsort(out_col + out_rp[v], (size_t)(w - out_rp[v]), sizeof(int32_t), cmp_i32);
+    out_rp[v + 1] = w;
+  }
+  free(ci); free(cd); free(vi); free(vd); free(pi); free(pd);
+  return 0;
+}
+
 /* ================================================================== O3 / O2 */
 /*
  * Plain backtracking: positions `ord[0..k-1]` (a BFS order of Q from the seed

@@ -20,7 +20,7 @@ import numpy as np
 from . import _lib
 from ._lib import Options, Stats, STATUS
 
-__all__ = ["Gcsm", "GcsmError", "plan_inspect", "shard", "nccl_unique_id", "CACHE_POLICIES"]
+__all__ = ["Gcsm", "GcsmError", "plan_inspect", "shard", "nccl_unique_id", "measure_host_link", "CACHE_POLICIES"]
 
 CACHE_POLICIES = {"estimator": 0, "degree": 1, "none": 2}
 FLAG_LOCAL_COUNTS = 1
@@ -191,6 +191,15 @@ def shard(cost, world):
     if s:
         raise GcsmError(s, "bad shard arguments")
     return out
+
+
+def measure_host_link(device=-1, nbytes=1 << 30):
+    """(zero-copy read GB/s, H2D DMA GB/s, HBM copy GB/s) measured by the library's micro-benchmarks."""
+    z, d, h = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+    s = _lib.load().gcsm_measure_host_link(device, nbytes, ctypes.byref(z), ctypes.byref(d), ctypes.byref(h))
+    if s:
+        raise GcsmError(s, "gcsm_measure_host_link failed")
+    return z.value, d.value, h.value
 
 
 def distributed_nccl_id():

@@ -18,7 +18,7 @@ STATUS = {0: "GCSM_OK", 1: "GCSM_EINVAL", 2: "GCSM_ENOMEM", 3: "GCSM_EDEVICE", 4
 SYMBOLS = ["gcsm_default_options", "gcsm_create", "gcsm_set_query", "gcsm_set_cache_budget", "gcsm_apply_batch",
            "gcsm_apply_batch_list", "gcsm_get_stats", "gcsm_query_automorphisms", "gcsm_last_error", "gcsm_destroy",
            "gcsm_nccl_unique_id", "gcsm_get_stream", "gcsm_export_csr", "gcsm_get_estimates", "gcsm_get_cached",
-           "gcsm_plan_inspect", "gcsm_shard"]
+           "gcsm_plan_inspect", "gcsm_shard", "gcsm_measure_host_link"]
 
 
 class Options(ctypes.Structure):
@@ -31,10 +31,11 @@ class Options(ctypes.Structure):
 class Stats(ctypes.Structure):
     _fields_ = [(name, ctypes.c_uint64) for name in
                 ["batches", "n_ins", "n_del", "dropped", "units", "n1", "walks", "max_degree", "cached_vertices",
-                 "cache_bytes", "hit_bytes", "miss_bytes", "delta_bytes", "frontier", "kernel_launches", "added", "removed"]] + \
+                 "cache_bytes", "hit_bytes", "miss_bytes", "delta_bytes", "hit_bytes_ext", "miss_bytes_ext",
+                 "delta_bytes_ext", "frontier", "kernel_launches", "h2d_bytes", "d2h_bytes", "added", "removed"]] + \
               [(name, ctypes.c_double) for name in
-               ["ms_normalize", "ms_estimate", "ms_pack", "ms_copy", "ms_match", "ms_allreduce", "ms_merge",
-                "ms_total"]]
+               ["ms_normalize", "ms_estimate", "ms_pack", "ms_copy", "ms_match", "ms_level2", "ms_extend",
+                "ms_allreduce", "ms_merge", "ms_total"]]
 
 
 _lib = None
@@ -68,6 +69,8 @@ def load():
         "gcsm_get_cached": (st, [P, P, U64, ctypes.POINTER(U64)]),
         "gcsm_plan_inspect": (st, [I32, I32, P, P, P, P, P, P, P]),
         "gcsm_shard": (st, [I64, P, I32, P]),
+        "gcsm_measure_host_link": (st, [I32, U64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double),
+                                        ctypes.POINTER(ctypes.c_double)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)

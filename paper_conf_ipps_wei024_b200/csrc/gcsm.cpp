@@ -63,12 +63,14 @@ struct gcsm_ctx {
   bool has_query = false;
   uint64_t budget = 0;
   cudaStream_t stream = nullptr;
-  cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr, ev_a0 = nullptr, ev_a1 = nullptr;
+  cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr, ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr, ev_c1 = nullptr;
+  std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
   ncclComm_t comm = nullptr;
   int grid = 0, warps_total = 0;
 
   // device buffers
   VDesc *d_vdesc = nullptr;
+  DevPlan *d_plans = nullptr;
   uint16_t *d_lab = nullptr;
   DRec *d_drec = nullptr; size_t drec_cap = 0;
   int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
@@ -121,15 +123,16 @@ struct gcsm_ctx {
 gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
-  void *dev[] = {d_vdesc, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cache, d_pidx, d_pval,
+  void *dev[] = {d_vdesc, d_plans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cache, d_pidx, d_pval,
                  d_tup};
   for (void *p : dev)
     if (p) cudaFree(p);
   void *host[] = {h_cache, h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt};
   for (void *p : host)
     if (p) cudaFreeHost(p);
-  for (cudaEvent_t e : {ev_m0, ev_m1, ev_a0, ev_a1})
+  for (cudaEvent_t e : {ev_m0, ev_m1, ev_a0, ev_a1, ev_c0, ev_c1})
     if (e) cudaEventDestroy(e);
+  for (cudaEvent_t e : kev) cudaEventDestroy(e);
   if (stream) cudaStreamDestroy(stream);
 }
 
@@ -192,10 +195,11 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
     return s;
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
-  for (cudaEvent_t *ev : {&ctx->ev_m0, &ctx->ev_m1, &ctx->ev_a0, &ctx->ev_a1})
+  for (cudaEvent_t *ev : {&ctx->ev_m0, &ctx->ev_m1, &ctx->ev_a0, &ctx->ev_a1, &ctx->ev_c0, &ctx->ev_c1})
     if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
   if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_plans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaHostAlloc(&ctx->h_cnt, sizeof(unsigned long long) * CNT_N, cudaHostAllocDefault) != cudaSuccess)
     return bail(GCSM_ENOMEM);
   ctx->vd.resize(n);
@@ -240,7 +244,7 @@ gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *q
     CK(cudaMalloc(&ctx->d_lab, 2 * (size_t)ctx->store.n));
     CK(cudaMemset(ctx->d_lab, 0, 2 * (size_t)ctx->store.n));
   }
-  CK(upload_plans(qp.plans.data(), (int)qp.plans.size(), ctx->stream));
+  CK(upload_plans(ctx->d_plans, qp.plans.data(), (int)qp.plans.size(), ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
   ctx->qp = qp;
   ctx->has_query = true;
@@ -485,12 +489,12 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   std::memcpy(ctx->h_units, units.data(), sizeof(Unit) * (size_t)nu);
   st.ms_pack = t3.ms();
 
-  Timer t4;
   cudaStream_t s = ctx->stream;
   if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
       !dev_ensure(ctx->d_drec, ctx->drec_cap, nU) || !dev_ensure(ctx->d_dlist, ctx->dlist_cap, nd) ||
       !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)nu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)nu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
+  CK(cudaEventRecord(ctx->ev_c0, s));
   if (used) CK(cudaMemcpyAsync(ctx->d_cache, ctx->h_cache, used, cudaMemcpyHostToDevice, s));  // the one DMA
   CK(cudaMemcpyAsync(ctx->d_pidx, ctx->h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(ctx->d_pval, ctx->h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
@@ -499,7 +503,9 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   if (nU) CK(cudaMemcpyAsync(ctx->d_drec, ctx->h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
   if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, ctx->h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
   if (nu) CK(cudaMemcpyAsync(ctx->d_units, ctx->h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
-  st.ms_copy = t4.ms();
+  CK(cudaEventRecord(ctx->ev_c1, s));
+  st.h2d_bytes = used + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU + 4 * nd +
+                 sizeof(Unit) * (size_t)nu;
 
   // ---- (4) matching kernels --------------------------------------------------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
@@ -543,6 +549,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   }
   CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N, s));
   MatchArgs A{};
+  A.plans = ctx->d_plans;
   A.vdesc = ctx->d_vdesc;
   A.lab = ctx->d_lab;
   A.drec = ctx->d_drec;
@@ -563,19 +570,29 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   A.k = k;
   A.listing = listing ? 1 : 0;
   CK(cudaEventRecord(ctx->ev_m0, s));
+  size_t nev = 0;
   for (const auto &ch : chunks) {
     if (ch.second <= ch.first) continue;
     A.units = ctx->d_units + ch.first;
     A.n_units = ch.second - ch.first;
+    while (ctx->kev.size() < nev + 3) {
+      cudaEvent_t ev;
+      CK(cudaEventCreate(&ev));
+      ctx->kev.push_back(ev);
+    }
     // reset the work cursors and the frontier size of this chunk
     CK(cudaMemsetAsync(ctx->d_cnt + CNT_F2, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(ctx->d_cnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), s));
+    CK(cudaEventRecord(ctx->kev[nev], s));
     CK(launch_level2(A, ctx->grid, s));
+    CK(cudaEventRecord(ctx->kev[nev + 1], s));
     ++launches;
     if (k >= 4) {
       CK(launch_extend(A, ctx->grid, s));
       ++launches;
     }
+    CK(cudaEventRecord(ctx->kev[nev + 2], s));
+    nev += 3;
   }
   CK(cudaEventRecord(ctx->ev_m1, s));
   // ---- (4b) count allreduce over NVLink (world > 1) -------------------------------------
@@ -593,11 +610,27 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   cudaEventElapsedTime(&ms_a, ctx->ev_a0, ctx->ev_a1);
   st.ms_match = ms_m;
   st.ms_allreduce = ms_a;
+  {
+    float ms_c = 0;
+    cudaEventElapsedTime(&ms_c, ctx->ev_c0, ctx->ev_c1);
+    st.ms_copy = ms_c;
+    for (size_t i = 0; i < nev; i += 3) {
+      float a = 0, b = 0;
+      cudaEventElapsedTime(&a, ctx->kev[i], ctx->kev[i + 1]);
+      cudaEventElapsedTime(&b, ctx->kev[i + 1], ctx->kev[i + 2]);
+      st.ms_level2 += a;
+      st.ms_extend += b;
+    }
+  }
   st.added = ctx->h_cnt[CNT_ADDED];
   st.removed = ctx->h_cnt[CNT_REMOVED];
-  st.hit_bytes = ctx->h_cnt[CNT_HIT];
-  st.miss_bytes = ctx->h_cnt[CNT_MISS];
-  st.delta_bytes = ctx->h_cnt[CNT_DELTA];
+  st.hit_bytes_ext = ctx->h_cnt[CNT_ACC_EXT + 0];
+  st.miss_bytes_ext = ctx->h_cnt[CNT_ACC_EXT + 1];
+  st.delta_bytes_ext = ctx->h_cnt[CNT_ACC_EXT + 2];
+  st.hit_bytes = ctx->h_cnt[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
+  st.miss_bytes = ctx->h_cnt[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
+  st.delta_bytes = ctx->h_cnt[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
+  st.d2h_bytes = sizeof(unsigned long long) * CNT_N;
   st.frontier = ctx->h_cnt[CNT_F2];
   st.kernel_launches = launches;
   bool trunc = false;
@@ -606,6 +639,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     const uint64_t nr = std::min<uint64_t>(ctx->h_cnt[CNT_TUP_REM], rem_cap);
     if (na) CK(cudaMemcpy(tup_add, d_tadd, sizeof(int32_t) * k * na, cudaMemcpyDeviceToHost));
     if (nr) CK(cudaMemcpy(tup_rem, d_trem, sizeof(int32_t) * k * nr, cudaMemcpyDeviceToHost));
+    st.d2h_bytes += sizeof(int32_t) * k * (na + nr);
     trunc = ctx->h_cnt[CNT_TUP_ADD] > add_cap || ctx->h_cnt[CNT_TUP_REM] > rem_cap;
   }
 

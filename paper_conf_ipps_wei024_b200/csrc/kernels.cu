@@ -30,8 +30,6 @@
 
 namespace gcsm {
 
-__constant__ DevPlan c_plans[GCSM_MAXPLANS];
-
 namespace {
 
 constexpr int kWarps = 8;
@@ -171,9 +169,9 @@ __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int la
   if (lane == 0) {
     if (acc.add) atomicAdd(&A.cnt[CNT_ADDED], acc.add);
     if (acc.rem) atomicAdd(&A.cnt[CNT_REMOVED], acc.rem);
-    if (acc.hit) atomicAdd(&A.cnt[CNT_HIT], acc.hit);
-    if (acc.miss) atomicAdd(&A.cnt[CNT_MISS], acc.miss);
-    if (acc.delta) atomicAdd(&A.cnt[CNT_DELTA], acc.delta);
+    if (acc.hit) atomicAdd(&A.cnt[A.acc_base + 0], acc.hit);
+    if (acc.miss) atomicAdd(&A.cnt[A.acc_base + 1], acc.miss);
+    if (acc.delta) atomicAdd(&A.cnt[A.acc_base + 2], acc.delta);
   }
 }
 
@@ -190,7 +188,7 @@ __global__ void __launch_bounds__(kBlock) k_level2(const MatchArgs A) {
     u = __shfl_sync(kFull, u, 0);
     if ((int64_t)u >= A.n_units) break;
     const Unit U = A.units[u];
-    const DevPlan &P = c_plans[U.plan];
+    const DevPlan &P = A.plans[U.plan];
     const int32_t f[2] = {U.a, U.b};
     if (A.k == 2) {  // single-edge query: the seed itself is the embedding
       if (P.kind) acc.rem += 1;
@@ -267,7 +265,7 @@ __global__ void __launch_bounds__(kBlock) k_extend(const MatchArgs A) {
     if ((int64_t)e >= n_f2) break;
     const int32_t ui = f2u[e];
     const Unit U = A.units[ui];
-    const DevPlan &P = c_plans[U.plan];
+    const DevPlan &P = A.plans[U.plan];
     const int2 seg = A.useg[ui];
     int32_t f[GCSM_MAXK];
     f[0] = U.a;
@@ -332,8 +330,8 @@ __global__ void k_patch(VDesc *vdesc, const int64_t *idx, const VDesc *val, int6
 
 }  // namespace
 
-cudaError_t upload_plans(const DevPlan *plans, int n, cudaStream_t s) {
-  return cudaMemcpyToSymbolAsync(c_plans, plans, sizeof(DevPlan) * (size_t)n, 0, cudaMemcpyHostToDevice, s);
+cudaError_t upload_plans(DevPlan *dst, const DevPlan *plans, int n, cudaStream_t s) {
+  return cudaMemcpyAsync(dst, plans, sizeof(DevPlan) * (size_t)n, cudaMemcpyHostToDevice, s);
 }
 
 int match_grid(int device, int *warps_total) {
@@ -349,13 +347,17 @@ int match_grid(int device, int *warps_total) {
   return grid;
 }
 
-cudaError_t launch_level2(const MatchArgs &a, int grid, cudaStream_t s) {
+cudaError_t launch_level2(const MatchArgs &a0, int grid, cudaStream_t s) {
+  MatchArgs a = a0;
+  a.acc_base = CNT_ACC_L2;
   if (a.listing) k_level2<true><<<grid, kBlock, 0, s>>>(a);
   else k_level2<false><<<grid, kBlock, 0, s>>>(a);
   return cudaGetLastError();
 }
 
-cudaError_t launch_extend(const MatchArgs &a, int grid, cudaStream_t s) {
+cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
+  MatchArgs a = a0;
+  a.acc_base = CNT_ACC_EXT;
   if (a.listing) k_extend<true><<<grid, kBlock, 0, s>>>(a);
   else k_extend<false><<<grid, kBlock, 0, s>>>(a);
   return cudaGetLastError();

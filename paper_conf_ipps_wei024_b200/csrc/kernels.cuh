@@ -10,19 +10,21 @@ namespace gcsm {
 enum Counter {
   CNT_ADDED = 0,    // embeddings found by + units
   CNT_REMOVED = 1,  // embeddings found by - units
-  CNT_HIT = 2,      // list bytes served from the HBM cache (algorithmic: 4 B x list length per use)
-  CNT_MISS = 3,     // list bytes served zero-copy from pinned host memory
   CNT_F2 = 4,       // level-2 frontier entries written
   CNT_OVERFLOW = 5, // frontier overflow guard (must stay 0)
   CNT_TUP_ADD = 6,  // tuples found (list mode)
   CNT_TUP_REM = 7,
   CNT_CURSOR0 = 8,  // work cursors (reset per launch)
   CNT_CURSOR1 = 9,
-  CNT_DELTA = 10,   // list bytes served from the device delta segments (ins/del of U)
+  // per kernel, 3 consecutive slots: list bytes (algorithmic: 4 B x list length per use) served from
+  // the HBM cache, zero-copy from pinned host memory, and from the device delta segments (ins/del of U)
+  CNT_ACC_L2 = 10,
+  CNT_ACC_EXT = 13,
   CNT_N = 16
 };
 
 struct MatchArgs {
+  const DevPlan *plans;     // per-context query plans (2 per term)
   const VDesc *vdesc;
   const uint16_t *lab;      // nullptr if unlabelled
   const DRec *drec;
@@ -43,9 +45,11 @@ struct MatchArgs {
   uint64_t tup_rem_cap;
   int32_t k;
   int32_t listing;
+  int32_t acc_base;         // CNT_ACC_L2 or CNT_ACC_EXT (set by the launchers)
 };
 
-cudaError_t upload_plans(const DevPlan *plans, int n, cudaStream_t s);
+// plans live in a per-context device buffer (contexts may run concurrently)
+cudaError_t upload_plans(DevPlan *dst, const DevPlan *plans, int n, cudaStream_t s);
 // grid sizes: persistent CTAs (multiple of the SM count)
 int match_grid(int device, int *warps_total);
 cudaError_t launch_level2(const MatchArgs &a, int grid, cudaStream_t s);

@@ -288,6 +288,25 @@ def test_emulated_world_sums(G, world):
     assert [tuple(x) for x in tot] == want
 
 
+def test_interleaved_contexts(G):
+    """Two live contexts with different queries (per-context plans and caches) applied alternately."""
+    w = gi.make_workload("C2", scale=12, n_edges=30_000, batch=256, n_batches=3)
+    want = {q: oracle_run(w.n, w.row_ptr, w.col, None, q, w.batches)[0] for q in ("k4", "c4", "house5u")}
+    ctx = {}
+    for q in want:
+        k, qe, ql = gi.query(q)
+        ctx[q] = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+        ctx[q].set_query(k, qe, ql)
+        ctx[q].set_cache_budget(w.adj_bytes // 10)
+    got = {q: [] for q in want}
+    for b in w.batches:
+        for q in want:
+            got[q].append(ctx[q].apply_batch(*b))
+    for g in ctx.values():
+        g.close()
+    assert got == want
+
+
 def test_cache_policies_same_counts(G):
     w = gi.make_workload("C2", scale=14, n_edges=150_000, batch=512, n_batches=2)
     want, _ = oracle_run(w.n, w.row_ptr, w.col, None, "k4", w.batches)

@@ -292,3 +292,17 @@ def test_normalize_batch_r8():
     for bad in [([(1, 1)], []), ([(0, 5)], []), ([(0, 2)], [(2, 0)]), ([], [(-1, 2)])]:
         with pytest.raises(ValueError):
             oracle.normalize_batch(5, rp, col, *bad)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_apply_batch_vs_set_algebra(seed):
+    """The row-by-row graph update (oracle.c o_apply) equals plain numpy set algebra on edge keys."""
+    n, g0, ins, dele = gi.small_random_case(500 + seed, n=30, p=0.2, n_ins=12, n_del=12)
+    rp, col = _csr(n, g0)
+    I, D, _ = oracle.normalize_batch(n, rp, col, ins, dele)
+    a = oracle.apply_batch(n, rp, col, I, D)
+    b = oracle.apply_batch_setalgebra(n, rp, col, I, D)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    s = oracle.stable_graph(n, rp, col, D)
+    e = {tuple(x) for x in oracle.edges_of(*s).tolist()}
+    assert e == {tuple(x) for x in g0.tolist()} - {tuple(x) for x in D.tolist()}
