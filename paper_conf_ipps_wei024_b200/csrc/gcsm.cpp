@@ -510,7 +510,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   // ---- (4) matching kernels --------------------------------------------------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
   const int nbuf = std::max(1, std::max(k - 4, 0) + (listing ? 1 : 0));
-  const size_t stride = (size_t)nbuf * (size_t)dcap;
+  const size_t stride = (size_t)(nbuf + 2) * (size_t)dcap;  // stacks + 2 HBM staging buffers
   if (!dev_ensure(ctx->d_scratch, ctx->scratch_cap, stride * (size_t)ctx->warps_total))
     return ctx->fail(GCSM_ENOMEM, "scratch");
   // level-2 frontier chunks: per unit an upper bound on its candidates

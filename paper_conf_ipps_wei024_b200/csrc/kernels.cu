@@ -35,6 +35,8 @@ namespace {
 constexpr int kWarps = 8;
 constexpr int kBlock = 32 * kWarps;
 constexpr unsigned kFull = 0xffffffffu;
+constexpr uint32_t kSmemInts = 1536;  // per-warp shared staging slice (6 KB)
+constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 
 struct LRef {
   const int32_t *m;  // main list
@@ -122,6 +124,72 @@ __device__ __forceinline__ uint32_t warp_isect(const MatchArgs &A, const int32_t
   return found;
 }
 
+__device__ __forceinline__ bool is_hit(const MatchArgs &A, const int32_t *p) {
+  return reinterpret_cast<const char *>(p) >= A.cache_lo && reinterpret_cast<const char *>(p) < A.cache_hi;
+}
+
+// Warp-cooperative bulk copy of a list (16-byte aligned source; lists are
+// allocated in 16-byte granules so reading up to round4(n) ints stays inside
+// the allocation). 4 x 16 B loads per lane are issued before any store, so a
+// warp keeps 2 KB in flight: a zero-copy list crosses PCIe at link speed
+// instead of one dependent 32 B sector per binary-search step.
+__device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
+  const uint32_t n4 = (n + 3) >> 2;
+  const int4 *s4 = reinterpret_cast<const int4 *>(src);
+  int4 *d4 = reinterpret_cast<int4 *>(dst);
+  for (uint32_t base = 0; base < n4; base += 128) {
+    const uint32_t i0 = base + lane, i1 = i0 + 32, i2 = i0 + 64, i3 = i0 + 96;
+    int4 v0, v1, v2, v3;
+    if (i0 < n4) v0 = s4[i0];
+    if (i1 < n4) v1 = s4[i1];
+    if (i2 < n4) v2 = s4[i2];
+    if (i3 < n4) v3 = s4[i3];
+    if (i0 < n4) d4[i0] = v0;
+    if (i1 < n4) d4[i1] = v1;
+    if (i2 < n4) d4[i2] = v2;
+    if (i3 < n4) d4[i3] = v3;
+  }
+}
+
+// Staging policy: a zero-copy driver list is bulk-copied once
+// (full MLP); a probe list is bulk-copied when reading it whole costs no more
+// bytes than the probes would (4 L <= 32 B x d x (log2 L - 3): one sector per
+// binary-search step below the first 8-int sector), into the warp's shared
+// memory slice if it fits, else (zero-copy lists only) into its HBM scratch.
+__device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl, int drv, bool has_set, uint32_t dn,
+                                            int32_t *sm, int32_t *gbuf, int lane) {
+  const uint32_t d = has_set ? dn : L[drv].ml + L[drv].xl;
+  uint32_t sm_used = 0, g_used = 0;
+  bool any = false;
+  for (int p = 0; p < nl; ++p) {
+    const uint32_t n = L[p].ml;
+    if (n < 32) continue;
+    const bool hit = is_hit(A, L[p].m);
+    const bool driver = !has_set && p == drv;
+    bool stage;
+    if (driver) {
+      stage = !hit;
+    } else {
+      const uint32_t lg = 32u - __clz(n);
+      stage = 4ull * n <= 32ull * d * (lg > 4 ? lg - 3 : 1);
+    }
+    if (!stage) continue;
+    const uint32_t n4 = (n + 3) & ~3u;
+    if (sm_used + n4 <= kSmemInts) {
+      warp_copy(sm + sm_used, L[p].m, n, lane);
+      L[p].m = sm + sm_used;
+      sm_used += n4;
+      any = true;
+    } else if (!hit && g_used + n4 <= 2u * (uint32_t)A.dcap) {
+      warp_copy(gbuf + g_used, L[p].m, n, lane);
+      L[p].m = gbuf + g_used;
+      g_used += n4;
+      any = true;
+    }
+  }
+  if (any) __syncwarp();
+}
+
 // Lists of position p for the current partial match f (positions 0..p-1).
 // Returns the number of probe lists written to L and sets *drv (index of the
 // smallest list) or uses the reused set.
@@ -177,10 +245,13 @@ __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int la
 
 // Level 2 (BFS step): warp per unit.
 template <bool LIST>
-__global__ void __launch_bounds__(kBlock) k_level2(const MatchArgs A) {
+__global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int32_t *buf = A.scratch + gw * A.scratch_stride;
+  int32_t *gstage = buf + A.scratch_stride - 2 * (int64_t)A.dcap;
+  extern __shared__ int4 smem_raw[];
+  int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
   Acc acc;
   for (;;) {
     unsigned long long u = 0;
@@ -209,6 +280,7 @@ __global__ void __launch_bounds__(kBlock) k_level2(const MatchArgs A) {
     LRef L[7];
     int drv;
     const int nl = gather_lists(A, L2, f, L, &drv, acc);
+    stage_lists(A, L, nl, drv, false, 0, sm, gstage, lane);
     int32_t excl[2];
     int nex = 0;
     for (int i = 0; i < L2.ninj; ++i) excl[nex++] = f[L2.inj[i]];
@@ -248,10 +320,13 @@ __global__ void __launch_bounds__(kBlock) k_level2(const MatchArgs A) {
 
 // Levels 3..k-1 (DFS): warp per level-2 frontier entry.
 template <bool LIST>
-__global__ void __launch_bounds__(kBlock) k_extend(const MatchArgs A) {
+__global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int32_t *stack = A.scratch + gw * A.scratch_stride;  // buffer for position p: stack + (p - 3) * dcap
+  int32_t *gstage = stack + A.scratch_stride - 2 * (int64_t)A.dcap;
+  extern __shared__ int4 smem_raw[];
+  int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
   const int k = A.k;
   int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
   const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
@@ -289,6 +364,7 @@ __global__ void __launch_bounds__(kBlock) k_extend(const MatchArgs A) {
         for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
         const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
+        stage_lists(A, L, nl, drv, dset != nullptr, dn, sm, gstage, lane);
         if (p == k - 1) {
           uint32_t c;
           if (LIST) {
@@ -337,9 +413,13 @@ cudaError_t upload_plans(DevPlan *dst, const DevPlan *plans, int n, cudaStream_t
 int match_grid(int device, int *warps_total) {
   int sms = 0, occ = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false>, kBlock, 0);
+  cudaFuncSetAttribute(k_extend<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_extend<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_level2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_level2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false>, kBlock, kSmemBytes);
   int occ2 = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_level2<false>, kBlock, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_level2<false>, kBlock, kSmemBytes);
   if (occ2 < occ) occ = occ2;
   if (occ < 1) occ = 1;
   const int grid = sms * occ;
@@ -350,16 +430,16 @@ int match_grid(int device, int *warps_total) {
 cudaError_t launch_level2(const MatchArgs &a0, int grid, cudaStream_t s) {
   MatchArgs a = a0;
   a.acc_base = CNT_ACC_L2;
-  if (a.listing) k_level2<true><<<grid, kBlock, 0, s>>>(a);
-  else k_level2<false><<<grid, kBlock, 0, s>>>(a);
+  if (a.listing) k_level2<true><<<grid, kBlock, kSmemBytes, s>>>(a);
+  else k_level2<false><<<grid, kBlock, kSmemBytes, s>>>(a);
   return cudaGetLastError();
 }
 
 cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
   MatchArgs a = a0;
   a.acc_base = CNT_ACC_EXT;
-  if (a.listing) k_extend<true><<<grid, kBlock, 0, s>>>(a);
-  else k_extend<false><<<grid, kBlock, 0, s>>>(a);
+  if (a.listing) k_extend<true><<<grid, kBlock, kSmemBytes, s>>>(a);
+  else k_extend<false><<<grid, kBlock, kSmemBytes, s>>>(a);
   return cudaGetLastError();
 }
 
