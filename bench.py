@@ -294,7 +294,7 @@ def main():
                                      "ms_extend": 0.0, "ms_normalize": 0.0, "ms_estimate": 0.0, "ms_pack": 0.0,
                                      "ms_copy": 0.0, "ms_allreduce": 0.0, "ms_merge": 0.0, "hit_bytes": 0,
                                      "miss_bytes": 0, "delta_bytes": 0, "hit_bytes_ext": 0, "miss_bytes_ext": 0,
-                                     "delta_bytes_ext": 0, "cache_bytes": 0, "cached_vertices": 0, "units": 0,
+                                     "delta_bytes_ext": 0, "host_copied_bytes": 0, "cache_bytes": 0, "cached_vertices": 0, "units": 0,
                                      "frontier": 0, "h2d_bytes": 0, "d2h_bytes": 0, "kernel_launches": 0})
             d["added"] += a
             d["removed"] += r
@@ -368,6 +368,7 @@ def main():
                           "hit_rate": (d["hit_bytes"] + d["delta_bytes"]) /
                           max(1, d["hit_bytes"] + d["delta_bytes"] + d["miss_bytes"]),
                           "cache_mb": d["cache_bytes"] / K / 2**20, "units": d["units"] / K,
+                          "miss_gb": d["miss_bytes"] / K / 1e9, "host_copied_gb": d["host_copied_bytes"] / K / 1e9,
                           "frontier": d["frontier"] / K} for q, d in per_q.items()},
         "gen_seconds": gen_s,
     }

@@ -103,6 +103,7 @@ typedef struct {
   uint64_t miss_bytes;      /* list bytes the kernels read zero-copy from host memory */
   uint64_t delta_bytes;     /* list bytes read from the device-resident ins/del segments of updated vertices */
   uint64_t hit_bytes_ext, miss_bytes_ext, delta_bytes_ext; /* the same, k_extend only (levels >= 3) */
+  uint64_t host_copied_bytes; /* bytes the kernels bulk-copied from host memory (staging; real zero-copy reads) */
   uint64_t frontier;        /* level-2 partial matches materialised */
   uint64_t kernel_launches; /* this library's kernels launched in the last batch */
   uint64_t h2d_bytes;       /* bytes copied host -> device in the batch (cache DMA, descriptors, deltas, units) */

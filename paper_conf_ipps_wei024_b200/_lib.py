@@ -32,7 +32,7 @@ class Stats(ctypes.Structure):
     _fields_ = [(name, ctypes.c_uint64) for name in
                 ["batches", "n_ins", "n_del", "dropped", "units", "n1", "walks", "max_degree", "cached_vertices",
                  "cache_bytes", "hit_bytes", "miss_bytes", "delta_bytes", "hit_bytes_ext", "miss_bytes_ext",
-                 "delta_bytes_ext", "frontier", "kernel_launches", "h2d_bytes", "d2h_bytes", "added", "removed"]] + \
+                 "delta_bytes_ext", "host_copied_bytes", "frontier", "kernel_launches", "h2d_bytes", "d2h_bytes", "added", "removed"]] + \
               [(name, ctypes.c_double) for name in
                ["ms_normalize", "ms_estimate", "ms_pack", "ms_copy", "ms_match", "ms_level2", "ms_extend",
                 "ms_allreduce", "ms_merge", "ms_total"]]

@@ -143,14 +143,11 @@ int64_t binomial(uint64_t key, int64_t n, double p) {
 }
 
 // Exact B' = 0 decision of the inversion branch before the draw completes:
-// Bin(n, p) with n p < 10 and p <= 1/2 is 0 iff the first uniform <= (1-p)^n.
-static inline bool binom_is_zero_fast(uint64_t key, int64_t n, double p, bool *decided) {
-  if (n <= 0 || p <= 0.0) { *decided = true; return true; }
-  if (p >= 1.0 || p > 0.5 || (double)n * p >= 10.0) { *decided = false; return false; }
+// Bin(n, p) with n p < 10 and 0 < p <= 1/2 is 0 iff the first uniform <= (1-p)^n
+// (binv's r0, computed once per parent: every child of a node shares n and p).
+static inline bool first_uniform_le(uint64_t key, double r0) {
   Uniforms U{key};
-  const double u = U.next();
-  *decided = true;
-  return !(u > std::pow(1.0 - p, (double)n));
+  return !(U.next() > r0);
 }
 
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k) {
@@ -183,9 +180,7 @@ struct Walker {
   std::vector<Rec> &out;
   const DevPlan *P = nullptr;
   int32_t f[GCSM_MAXK];
-  std::vector<std::vector<int32_t>> cand;  // per position
-
-  Walker(const EstimatorInput &i, std::vector<Rec> &o) : in(i), out(o), cand(GCSM_MAXK) {}
+  Walker(const EstimatorInput &i, std::vector<Rec> &o) : in(i), out(o) {}
 
   bool member(const HList &L, int32_t v) const {
     return std::binary_search(L.a, L.a + L.na, v) || (L.nb && std::binary_search(L.b, L.b + L.nb, v));
@@ -208,13 +203,14 @@ struct Walker {
     for (int b = 1; b < Lp.nb; ++b)
       if (L[b].na + L[b].nb < L[drv].na + L[drv].nb) drv = b;
     const double pD = 1.0 / (double)in.D;
+    const bool fast = B > 0 && pD > 0.0 && pD <= 0.5 && (double)B * pD < 10.0;
+    const double r0 = fast ? std::pow(1.0 - pD, (double)B) : 0.0;
     auto consider = [&](int32_t v) {
       for (int s = 0; s < p; ++s)
         if (f[s] == v) return;
       if (Lp.label >= 0 && (in.labels ? (int32_t)in.labels[v] : 0) != Lp.label) return;
       const uint64_t ck = rng_chain(key, (uint64_t)(uint32_t)v);
-      bool decided;
-      if (binom_is_zero_fast(ck, B, pD, &decided) && decided) return;
+      if (fast && first_uniform_le(ck, r0)) return;  // B' = 0: skip the probes
       for (int b = 0; b < Lp.nb; ++b)
         if (b != drv && !member(L[b], v)) return;
       const int64_t Bc = binomial(ck, B, pD);

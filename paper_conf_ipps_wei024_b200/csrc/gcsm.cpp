@@ -77,9 +77,18 @@ struct gcsm_ctx {
   Unit *d_units = nullptr; size_t units_cap = 0;
   int2 *d_useg = nullptr; size_t useg_cap = 0;
   int32_t *d_f2 = nullptr; size_t f2_cap = 0;  // 2 * f2 entries ints
+  int32_t *d_group = nullptr; size_t group_cap = 0;  // frontier entries grouped by candidate
+  uint32_t *d_hist = nullptr;                         // n counters + scan
+  uint32_t *d_bsum = nullptr;
   int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
   unsigned long long *d_cnt = nullptr;
-  char *d_cache = nullptr; size_t cache_cap = 0;
+  char *d_cache = nullptr; size_t cache_cap = 0;   // the buffer this batch's kernels read
+  char *d_cachebuf[2] = {nullptr, nullptr};        // double buffer: last batch's cache stays readable
+  int cache_cur = 0;                               // buffer holding the previous batch's cache
+  bool cache_valid = false;                        // prev_slot describes d_cachebuf[cache_cur]
+  std::vector<std::pair<int32_t, uint64_t>> prev_slot;  // (vertex, offset) of the previous cache, by vertex
+  uint64_t *d_gather = nullptr; size_t gather_cap = 0;  // retained lists: (src, dst, n16) triples
+  uint64_t *h_gather = nullptr; size_t h_gather_cap = 0;
   int64_t *d_pidx = nullptr; size_t pidx_cap = 0;
   VDesc *d_pval = nullptr; size_t pval_cap = 0;
   int32_t *d_tup = nullptr; size_t tup_cap = 0;
@@ -123,11 +132,11 @@ struct gcsm_ctx {
 gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
-  void *dev[] = {d_vdesc, d_plans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cache, d_pidx, d_pval,
-                 d_tup};
+  void *dev[] = {d_vdesc, d_plans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
+                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum};
   for (void *p : dev)
     if (p) cudaFree(p);
-  void *host[] = {h_cache, h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt};
+  void *host[] = {h_cache, h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt, h_gather};
   for (void *p : host)
     if (p) cudaFreeHost(p);
   for (cudaEvent_t e : {ev_m0, ev_m1, ev_a0, ev_a1, ev_c0, ev_c1})
@@ -200,6 +209,9 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_plans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)n + 2047) / 2048 + 1)) != cudaSuccess)
+    return bail(GCSM_ENOMEM);
   if (cudaHostAlloc(&ctx->h_cnt, sizeof(unsigned long long) * CNT_N, cudaHostAllocDefault) != cudaSuccess)
     return bail(GCSM_ENOMEM);
   ctx->vd.resize(n);
@@ -257,17 +269,22 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
   if (ctx->poisoned) return GCSM_ESTATE;
   bytes &= ~uint64_t(15);
   if (bytes > ctx->cache_cap) {
-    if (ctx->d_cache) cudaFree(ctx->d_cache);
+    for (char *&b : ctx->d_cachebuf) {
+      if (b) cudaFree(b);
+      b = nullptr;
+    }
     if (ctx->h_cache) cudaFreeHost(ctx->h_cache);
-    ctx->d_cache = nullptr;
     ctx->h_cache = nullptr;
     ctx->cache_cap = ctx->h_cache_cap = 0;
-    if (cudaMalloc(&ctx->d_cache, bytes) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "device cache allocation failed");
+    for (char *&b : ctx->d_cachebuf)
+      if (cudaMalloc(&b, bytes) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "device cache allocation failed");
     if (cudaHostAlloc(&ctx->h_cache, bytes, cudaHostAllocDefault) != cudaSuccess)
       return ctx->fail(GCSM_ENOMEM, "pinned cache staging allocation failed");
     ctx->cache_cap = ctx->h_cache_cap = bytes;
   }
   ctx->budget = bytes;
+  ctx->cache_valid = false;  // the next batch repacks everything
+  ctx->prev_slot.clear();
   return GCSM_OK;
 }
 
@@ -409,22 +426,61 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   std::vector<int32_t> sel;
   std::vector<uint64_t> sel_off;
   uint64_t used = 0;
+  // incremental cache (double buffered): a selected vertex whose list is unchanged since it was cached in the
+  // previous batch (not updated then, not updated now) is copied HBM -> HBM; only the other lists go through
+  // pinned staging and the one H2D DMA.
+  std::vector<uint64_t> gather;  // (src offset, dst offset, 16-byte units) per retained list
+  uint64_t new_bytes = 0;
+  const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
+  ctx->d_cache = ctx->d_cachebuf[tgt];
   if (use_cache && !ranked.empty()) {
     std::sort(ranked.begin(), ranked.end(), [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {
       return x.first > y.first || (x.first == y.first && x.second < y.second);
     });
+    std::vector<uint64_t> bytes_of;
     for (const auto &r : ranked) {
       if (!(r.first > 0)) break;
       const uint64_t bytes = (uint64_t)((S.view_len(r.second, VIEW_S) + 3u) & ~3u) * 4;
       if (used + bytes > ctx->budget) break;  // longest prefix that fits (R23)
       sel.push_back(r.second);
-      sel_off.push_back(used);
+      bytes_of.push_back(bytes);
       used += bytes;
     }
-    parallel_for(T, (int64_t)sel.size(), [&](int, int64_t lo, int64_t hi) {
-      for (int64_t i = lo; i < hi; ++i) {
+    // retained lists first, then the new ones
+    for (int32_t v : ctx->prev_U) ctx->mark[v] = 2;
+    std::vector<int64_t> old_off(sel.size(), -1);
+    if (ctx->cache_valid)
+      for (size_t i = 0; i < sel.size(); ++i) {
+        const int32_t v = sel[i];
+        if (ctx->mark[v] == 2 || S.uidx[v] >= 0) continue;
+        auto it = std::lower_bound(ctx->prev_slot.begin(), ctx->prev_slot.end(), std::make_pair(v, (uint64_t)0));
+        if (it != ctx->prev_slot.end() && it->first == v) old_off[i] = (int64_t)it->second;
+      }
+    for (int32_t v : ctx->prev_U) ctx->mark[v] = 0;
+    sel_off.assign(sel.size(), 0);
+    uint64_t o = 0;
+    for (size_t i = 0; i < sel.size(); ++i)
+      if (old_off[i] >= 0) {
+        sel_off[i] = o;
+        gather.push_back((uint64_t)old_off[i]);
+        gather.push_back(o);
+        gather.push_back(bytes_of[i] / 16);
+        o += bytes_of[i];
+      }
+    const uint64_t retained = o;
+    std::vector<size_t> fresh;
+    for (size_t i = 0; i < sel.size(); ++i)
+      if (old_off[i] < 0) {
+        sel_off[i] = o;
+        o += bytes_of[i];
+        fresh.push_back(i);
+      }
+    new_bytes = o - retained;
+    parallel_for(T, (int64_t)fresh.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t j = lo; j < hi; ++j) {
+        const size_t i = fresh[j];
         const HList h = S.view(sel[i], VIEW_S);
-        std::memcpy(ctx->h_cache + sel_off[i], h.a, (size_t)h.na * 4);
+        std::memcpy(ctx->h_cache + (sel_off[i] - retained), h.a, (size_t)h.na * 4);
       }
     });
   }
@@ -495,7 +551,17 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
       !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)nu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)nu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
   CK(cudaEventRecord(ctx->ev_c0, s));
-  if (used) CK(cudaMemcpyAsync(ctx->d_cache, ctx->h_cache, used, cudaMemcpyHostToDevice, s));  // the one DMA
+  const uint64_t retained_bytes = used - new_bytes;
+  if (!gather.empty()) {  // HBM -> HBM copy of the retained lists from the previous buffer
+    if (!host_ensure(ctx->h_gather, ctx->h_gather_cap, gather.size()) ||
+        !dev_ensure(ctx->d_gather, ctx->gather_cap, gather.size()))
+      return ctx->fail(GCSM_ENOMEM, "gather staging");
+    std::memcpy(ctx->h_gather, gather.data(), 8 * gather.size());
+    CK(cudaMemcpyAsync(ctx->d_gather, ctx->h_gather, 8 * gather.size(), cudaMemcpyHostToDevice, s));
+    CK(launch_gather_lists(ctx->d_cache, ctx->d_cachebuf[ctx->cache_cur], ctx->d_gather, (int64_t)gather.size() / 3, s));
+  }
+  if (new_bytes)  // the one DMA of the newly selected lists
+    CK(cudaMemcpyAsync(ctx->d_cache + retained_bytes, ctx->h_cache, new_bytes, cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(ctx->d_pidx, ctx->h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(ctx->d_pval, ctx->h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(launch_patch_vdesc(ctx->d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
@@ -504,13 +570,13 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, ctx->h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
   if (nu) CK(cudaMemcpyAsync(ctx->d_units, ctx->h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(ctx->ev_c1, s));
-  st.h2d_bytes = used + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU + 4 * nd +
-                 sizeof(Unit) * (size_t)nu;
+  st.h2d_bytes = new_bytes + 8 * gather.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
+                 4 * nd + sizeof(Unit) * (size_t)nu;
 
   // ---- (4) matching kernels --------------------------------------------------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
   const int nbuf = std::max(1, std::max(k - 4, 0) + (listing ? 1 : 0));
-  const size_t stride = (size_t)(nbuf + 2) * (size_t)dcap;  // stacks + 2 HBM staging buffers
+  const size_t stride = (size_t)(nbuf + 3) * (size_t)dcap;  // stacks + pinned-x2 + 2 HBM staging buffers
   if (!dev_ensure(ctx->d_scratch, ctx->scratch_cap, stride * (size_t)ctx->warps_total))
     return ctx->fail(GCSM_ENOMEM, "scratch");
   // level-2 frontier chunks: per unit an upper bound on its candidates
@@ -534,7 +600,8 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     }
     chunks.push_back({start, nu});
     f2_need = std::max(f2_need, acc);
-    if (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)))
+    if (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)) ||
+        !dev_ensure(ctx->d_group, ctx->group_cap, (size_t)std::max<int64_t>(f2_need, 1)))
       return ctx->fail(GCSM_ENOMEM, "frontier");
   } else {
     chunks.push_back({0, nu});
@@ -558,6 +625,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   A.f2 = reinterpret_cast<int2 *>(ctx->d_f2);
   A.f2_cap = f2_need;
   A.scratch = ctx->d_scratch;
+  A.scratch_end = ctx->d_scratch + stride * (size_t)ctx->warps_total;
   A.scratch_stride = (int64_t)stride;
   A.dcap = dcap;
   A.cnt = ctx->d_cnt;
@@ -588,6 +656,9 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     CK(cudaEventRecord(ctx->kev[nev + 1], s));
     ++launches;
     if (k >= 4) {
+      CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_group, s));
+      launches += 6;
+      A.group = ctx->d_group;
       CK(launch_extend(A, ctx->grid, s));
       ++launches;
     }
@@ -630,6 +701,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   st.hit_bytes = ctx->h_cnt[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
   st.miss_bytes = ctx->h_cnt[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
   st.delta_bytes = ctx->h_cnt[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
+  st.host_copied_bytes = ctx->h_cnt[CNT_COPIED];
   st.d2h_bytes = sizeof(unsigned long long) * CNT_N;
   st.frontier = ctx->h_cnt[CNT_F2];
   st.kernel_launches = launches;
@@ -648,6 +720,13 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   S.merge();
   ctx->prev_cached = sel;
   std::sort(ctx->prev_cached.begin(), ctx->prev_cached.end());
+  ctx->prev_slot.resize(sel.size());
+  for (size_t i = 0; i < sel.size(); ++i) ctx->prev_slot[i] = {sel[i], sel_off[i]};
+  std::sort(ctx->prev_slot.begin(), ctx->prev_slot.end());
+  if (ctx->budget > 0) {
+    ctx->cache_cur = tgt;
+    ctx->cache_valid = true;
+  }
   ctx->cached = ctx->prev_cached;
   ctx->prev_U = S.U;
   S.clear_batch();

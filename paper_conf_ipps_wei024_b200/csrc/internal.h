@@ -11,6 +11,7 @@
 #pragma once
 #include <cstdint>
 #include <cstddef>
+#include <algorithm>
 #include <atomic>
 #include <chrono>
 #include <functional>
@@ -74,42 +75,37 @@ struct Timer {
   }
 };
 
-// Static-partitioned parallel for over [0, n) with `threads` workers.
+// Persistent host worker pool (one per process): spawning std::threads per
+// call cost ~1 ms per parallel region on the 16-core box; the pool wakes
+// parked workers instead. run() executes fn(tid) for tid in [0, nthreads),
+// the caller being tid 0; calls from different host threads are serialised.
+void pool_run(int nthreads, const std::function<void(int)> &fn);
+int pool_size();
+
+// Static-partitioned parallel for over [0, n).
 inline void parallel_for(int threads, int64_t n, const std::function<void(int, int64_t, int64_t)> &fn) {
   if (n <= 0) return;
-  if (threads <= 1 || n < 2) {
+  const int t = (int)std::min<int64_t>(std::min(threads, pool_size()), n);
+  if (t <= 1) {
     fn(0, 0, n);
     return;
   }
-  int t = (int)std::min<int64_t>(threads, n);
-  std::vector<std::thread> th;
-  th.reserve(t);
-  for (int i = 0; i < t; ++i) {
-    int64_t lo = n * i / t, hi = n * (i + 1) / t;
-    th.emplace_back([&fn, i, lo, hi] { fn(i, lo, hi); });
-  }
-  for (auto &x : th) x.join();
+  pool_run(t, [&](int i) { fn(i, n * i / t, n * (i + 1) / t); });
 }
 
 // Dynamic (atomic cursor) parallel for, chunked.
 inline void parallel_dyn(int threads, int64_t n, int64_t chunk, const std::function<void(int, int64_t)> &fn) {
   if (n <= 0) return;
   std::atomic<int64_t> next{0};
-  auto work = [&](int tid) {
+  const int t = (int)std::max<int64_t>(1, std::min<int64_t>(std::min(threads, pool_size()), (n + chunk - 1) / chunk));
+  pool_run(t, [&](int tid) {
     for (;;) {
-      int64_t s = next.fetch_add(chunk);
+      const int64_t s = next.fetch_add(chunk);
       if (s >= n) break;
-      int64_t e = std::min(n, s + chunk);
+      const int64_t e = std::min(n, s + chunk);
       for (int64_t i = s; i < e; ++i) fn(tid, i);
     }
-  };
-  if (threads <= 1) {
-    work(0);
-    return;
-  }
-  std::vector<std::thread> th;
-  for (int i = 0; i < threads; ++i) th.emplace_back(work, i);
-  for (auto &x : th) x.join();
+  });
 }
 
 // ------------------------------------------------------------ plan (plan.cpp)

@@ -37,6 +37,7 @@ constexpr int kBlock = 32 * kWarps;
 constexpr unsigned kFull = 0xffffffffu;
 constexpr uint32_t kSmemInts = 1536;  // per-warp shared staging slice (6 KB)
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
+constexpr int kChunk = 32;  // frontier entries per k_extend work grab
 
 struct LRef {
   const int32_t *m;  // main list
@@ -46,10 +47,18 @@ struct LRef {
 };
 
 struct Acc {
-  unsigned long long add = 0, rem = 0, hit = 0, miss = 0, delta = 0;
+  unsigned long long add = 0, rem = 0, hit = 0, miss = 0, delta = 0, copied = 0;
 };
 
-__device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc) {
+// Persistent per-warp copy of one vertex's main list (the position-2 vertex x2 of a run of frontier entries
+// grouped by x2): `v` = -1 when empty.
+struct Pinned {
+  int32_t v = -1;
+  const int32_t *p = nullptr;
+};
+
+__device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc,
+                                        const Pinned &pin = Pinned()) {
   const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
   LRef r;
   r.m = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
@@ -72,6 +81,7 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
   if (p >= A.cache_lo && p < A.cache_hi) acc.hit += 4ull * r.ml;
   else acc.miss += 4ull * r.ml;
   acc.delta += 4ull * r.xl;
+  if (v == pin.v) r.m = pin.p;  // served from this warp's staged copy
   return r;
 }
 
@@ -128,6 +138,11 @@ __device__ __forceinline__ bool is_hit(const MatchArgs &A, const int32_t *p) {
   return reinterpret_cast<const char *>(p) >= A.cache_lo && reinterpret_cast<const char *>(p) < A.cache_hi;
 }
 
+// A list already in device memory outside the cache (a warp's staged copy in its HBM scratch).
+__device__ __forceinline__ bool is_device(const MatchArgs &A, const int32_t *p) {
+  return p >= A.scratch && p < A.scratch_end;
+}
+
 // Warp-cooperative bulk copy of a list (16-byte aligned source; lists are
 // allocated in 16-byte granules so reading up to round4(n) ints stays inside
 // the allocation). 4 x 16 B loads per lane are issued before any store, so a
@@ -157,14 +172,14 @@ __device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint
 // binary-search step below the first 8-int sector), into the warp's shared
 // memory slice if it fits, else (zero-copy lists only) into its HBM scratch.
 __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl, int drv, bool has_set, uint32_t dn,
-                                            int32_t *sm, int32_t *gbuf, int lane) {
+                                            int32_t *sm, int32_t *gbuf, int lane, Acc &acc) {
   const uint32_t d = has_set ? dn : L[drv].ml + L[drv].xl;
   uint32_t sm_used = 0, g_used = 0;
   bool any = false;
   for (int p = 0; p < nl; ++p) {
     const uint32_t n = L[p].ml;
     if (n < 32) continue;
-    const bool hit = is_hit(A, L[p].m);
+    const bool hit = is_hit(A, L[p].m) || is_device(A, L[p].m);
     const bool driver = !has_set && p == drv;
     bool stage;
     if (driver) {
@@ -175,6 +190,7 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
     }
     if (!stage) continue;
     const uint32_t n4 = (n + 3) & ~3u;
+    if (!hit && !is_device(A, L[p].m)) acc.copied += 4ull * n;
     if (sm_used + n4 <= kSmemInts) {
       warp_copy(sm + sm_used, L[p].m, n, lane);
       L[p].m = sm + sm_used;
@@ -194,19 +210,19 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
 // Returns the number of probe lists written to L and sets *drv (index of the
 // smallest list) or uses the reused set.
 __device__ __forceinline__ int gather_lists(const MatchArgs &A, const LevelPlan &Lp, const int32_t *f, LRef *L,
-                                            int *drv, Acc &acc) {
+                                            int *drv, Acc &acc, const Pinned &pin = Pinned()) {
   int nl = 0;
   uint32_t best = 0xffffffffu;
   *drv = 0;
   if (Lp.reuse >= 0) {
     for (int r = 0; r < Lp.nrest; ++r) {
       const int b = Lp.rest[r];
-      L[nl++] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc);
+      L[nl++] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, pin);
     }
     return nl;
   }
   for (int b = 0; b < Lp.nb; ++b) {
-    L[nl] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc);
+    L[nl] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, pin);
     const uint32_t sz = L[nl].ml + L[nl].xl;
     if (sz < best) {
       best = sz;
@@ -240,6 +256,7 @@ __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int la
     if (acc.hit) atomicAdd(&A.cnt[A.acc_base + 0], acc.hit);
     if (acc.miss) atomicAdd(&A.cnt[A.acc_base + 1], acc.miss);
     if (acc.delta) atomicAdd(&A.cnt[A.acc_base + 2], acc.delta);
+    if (acc.copied) atomicAdd(&A.cnt[CNT_COPIED], acc.copied);
   }
 }
 
@@ -280,7 +297,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
     LRef L[7];
     int drv;
     const int nl = gather_lists(A, L2, f, L, &drv, acc);
-    stage_lists(A, L, nl, drv, false, 0, sm, gstage, lane);
+    stage_lists(A, L, nl, drv, false, 0, sm, gstage, lane, acc);
     int32_t excl[2];
     int nex = 0;
     for (int i = 0; i < L2.ninj; ++i) excl[nex++] = f[L2.inj[i]];
@@ -325,6 +342,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int32_t *stack = A.scratch + gw * A.scratch_stride;  // buffer for position p: stack + (p - 3) * dcap
   int32_t *gstage = stack + A.scratch_stride - 2 * (int64_t)A.dcap;
+  int32_t *pstage = gstage - (int64_t)A.dcap;  // persistent copy of the current x2's main list
   extern __shared__ int4 smem_raw[];
   int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
   const int k = A.k;
@@ -333,11 +351,40 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
   const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
   const int32_t *f2u = f2c + A.f2_cap;
   Acc acc;
+  Pinned pin;
+  int64_t ci = 0, c_end = 0;
   for (;;) {
-    unsigned long long e = 0;
-    if (lane == 0) e = atomicAdd(&A.cnt[CNT_CURSOR1], 1ull);
-    e = __shfl_sync(kFull, e, 0);
-    if ((int64_t)e >= n_f2) break;
+    if (ci >= c_end) {  // grab the next chunk of the (x2-grouped) frontier order
+      unsigned long long c0 = 0;
+      if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)kChunk);
+      c0 = __shfl_sync(kFull, c0, 0);
+      if ((int64_t)c0 >= n_f2) break;
+      ci = (int64_t)c0;
+      c_end = min((int64_t)c0 + kChunk, n_f2);
+      pin.v = -1;
+    }
+    const int64_t e = A.group ? A.group[ci] : ci;
+    const int32_t x2 = f2c[e];
+    if (x2 != pin.v) {
+      // run of entries sharing x2 in this chunk: stage x2's zero-copy main list once for all of them
+      int64_t j = ci + 1 + lane;
+      const bool same = j < c_end && f2c[A.group ? A.group[j] : j] == x2;
+      const unsigned run_mask = __ballot_sync(kFull, same);
+      const int run = 1 + (run_mask == kFull ? 32 : __ffs(~run_mask) - 1);  // entries of this run (capped at 33)
+      pin.v = -1;
+      const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + x2));
+      const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
+                                                              ((unsigned long long)(unsigned)raw.y << 32));
+      const uint32_t ml = (uint32_t)raw.z;
+      if (run >= 2 && ml >= 32 && !is_hit(A, mp) && ml <= (uint32_t)A.dcap) {
+        warp_copy(pstage, mp, ml, lane);
+        acc.copied += 4ull * ml;
+        __syncwarp();
+        pin.v = x2;
+        pin.p = pstage;
+      }
+    }
+    ++ci;
     const int32_t ui = f2u[e];
     const Unit U = A.units[ui];
     const DevPlan &P = A.plans[U.plan];
@@ -358,13 +405,13 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
         const LevelPlan &Lp = P.lv[p];
         LRef L[7];
         int drv;
-        const int nl = gather_lists(A, Lp, f, L, &drv, acc);
+        const int nl = gather_lists(A, Lp, f, L, &drv, acc, pin);
         int32_t excl[GCSM_MAXK];
         int nex = 0;
         for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
         const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
-        stage_lists(A, L, nl, drv, dset != nullptr, dn, sm, gstage, lane);
+        stage_lists(A, L, nl, drv, dset != nullptr, dn, sm, gstage, lane, acc);
         if (p == k - 1) {
           uint32_t c;
           if (LIST) {
@@ -397,6 +444,110 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
     (void)lvl;
   }
   flush(A, acc, lane);
+}
+
+// ---- counting sort of the level-2 frontier by its candidate vertex x2 (entries sharing x2 are
+// processed back to back by one warp, which stages x2's zero-copy list once per run).
+__global__ void k_group_hist(const int32_t *f2c, const unsigned long long *cnt, uint32_t *hist) {
+  const int64_t n = (int64_t)cnt[CNT_F2];
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&hist[f2c[e]], 1u);
+}
+
+constexpr int kScanItems = 8;  // per thread, 256 threads: 2048 per block
+
+// in-place exclusive scan of a[0..n) per 2048-block; block totals to bsum
+__global__ void k_scan_local(uint32_t *a, int64_t n, uint32_t *bsum) {
+  __shared__ uint32_t ws[8];
+  const int64_t base = (int64_t)blockIdx.x * 2048 + threadIdx.x * kScanItems;
+  uint32_t v[kScanItems], run = 0;
+  for (int i = 0; i < kScanItems; ++i) {
+    v[i] = base + i < n ? a[base + i] : 0u;
+    const uint32_t t = v[i];
+    v[i] = run;
+    run += t;
+  }
+  // exclusive scan of the per-thread totals across the block
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = run;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) ws[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t t = lane < 8 ? ws[lane] : 0u;
+    for (int o = 1; o < 8; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFull, t, o);
+      if (lane >= o) t += y;
+    }
+    if (lane < 8) ws[lane] = t;
+  }
+  __syncthreads();
+  const uint32_t excl = x - run + (w ? ws[w - 1] : 0u);
+  for (int i = 0; i < kScanItems; ++i)
+    if (base + i < n) a[base + i] = v[i] + excl;
+  if (threadIdx.x == 255) bsum[blockIdx.x] = excl + run;
+}
+
+// single block: exclusive scan of the block totals (loops for any count)
+__global__ void k_scan_bsum(uint32_t *bsum, int64_t nb) {
+  __shared__ uint32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (int64_t s0 = 0; s0 < nb; s0 += 1024) {
+    const int64_t i = s0 + threadIdx.x;
+    const uint32_t v = i < nb ? bsum[i] : 0u;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    uint32_t x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFull, x, o);
+      if (lane >= o) x += y;
+    }
+    __shared__ uint32_t ws[32];
+    if (lane == 31) ws[w] = x;
+    __syncthreads();
+    if (w == 0) {
+      uint32_t t = ws[lane];
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, t, o);
+        if (lane >= o) t += y;
+      }
+      ws[lane] = t;
+    }
+    __syncthreads();
+    const uint32_t incl = x + (w ? ws[w - 1] : 0u);
+    if (i < nb) bsum[i] = carry + incl - v;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry += incl;
+    __syncthreads();
+  }
+}
+
+__global__ void k_scan_add(uint32_t *a, int64_t n, const uint32_t *bsum) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    a[i] += bsum[i / 2048];
+}
+
+__global__ void k_group_scatter(const int32_t *f2c, const unsigned long long *cnt, uint32_t *cursor,
+                                int32_t *group) {
+  const int64_t n = (int64_t)cnt[CNT_F2];
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+    group[atomicAdd(&cursor[f2c[e]], 1u)] = (int32_t)e;
+}
+
+// Warp per retained cache list: copy n16 16-byte granules from the previous cache buffer.
+__global__ void k_gather(char *dst, const char *src, const uint64_t *tri, int64_t n) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = w; i < n; i += nw) {
+    const int4 *s4 = reinterpret_cast<const int4 *>(src + tri[3 * i]);
+    int4 *d4 = reinterpret_cast<int4 *>(dst + tri[3 * i + 1]);
+    const uint64_t n16 = tri[3 * i + 2];
+    for (uint64_t j = lane; j < n16; j += 32) d4[j] = s4[j];
+  }
 }
 
 __global__ void k_patch(VDesc *vdesc, const int64_t *idx, const VDesc *val, int64_t n) {
@@ -440,6 +591,27 @@ cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
   a.acc_base = CNT_ACC_EXT;
   if (a.listing) k_extend<true><<<grid, kBlock, kSmemBytes, s>>>(a);
   else k_extend<false><<<grid, kBlock, kSmemBytes, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_group_frontier(const MatchArgs &a, int32_t n_vertices, uint32_t *hist, uint32_t *bsum,
+                                  int32_t *group, cudaStream_t s) {
+  const int32_t *f2c = reinterpret_cast<const int32_t *>(a.f2);
+  cudaError_t e = cudaMemsetAsync(hist, 0, sizeof(uint32_t) * (size_t)n_vertices, s);
+  if (e != cudaSuccess) return e;
+  k_group_hist<<<148 * 8, 256, 0, s>>>(f2c, a.cnt, hist);
+  const int64_t nb = ((int64_t)n_vertices + 2047) / 2048;
+  k_scan_local<<<(unsigned)nb, 256, 0, s>>>(hist, n_vertices, bsum);
+  k_scan_bsum<<<1, 1024, 0, s>>>(bsum, nb);
+  k_scan_add<<<148 * 8, 256, 0, s>>>(hist, n_vertices, bsum);
+  k_group_scatter<<<148 * 8, 256, 0, s>>>(f2c, a.cnt, hist, group);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_gather_lists(char *dst, const char *src, const uint64_t *tri, int64_t n, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((n + 7) / 8, 148 * 16);
+  k_gather<<<grid, 256, 0, s>>>(dst, src, tri, n);
   return cudaGetLastError();
 }
 
