@@ -169,21 +169,22 @@ uint64_t walk_budget(uint64_t N1, uint64_t D, int k) {
 
 namespace {
 
-struct Rec {
-  int32_t v;
-  int32_t level;  // 1..k-2
-  uint64_t B;
-};
-
 struct Walker {
   const EstimatorInput &in;
-  std::vector<Rec> &out;
+  EstimatorScratch &scr;
   const DevPlan *P = nullptr;
   int32_t f[GCSM_MAXK];
-  Walker(const EstimatorInput &i, std::vector<Rec> &o) : in(i), out(o) {}
+  Walker(const EstimatorInput &i, EstimatorScratch &s) : in(i), scr(s) {}
 
   bool member(const HList &L, int32_t v) const {
     return std::binary_search(L.a, L.a + L.na, v) || (L.nb && std::binary_search(L.b, L.b + L.nb, v));
+  }
+
+  void record(int32_t v, int level, uint64_t B) {
+    __atomic_fetch_add(&scr.sums[(size_t)(level - 1) * (size_t)scr.n + (size_t)v], B, __ATOMIC_RELAXED);
+    uint64_t *w = &scr.touched[(uint32_t)v >> 6];
+    const uint64_t bit = 1ull << (v & 63);
+    if (!(__atomic_load_n(w, __ATOMIC_RELAXED) & bit)) __atomic_fetch_or(w, bit, __ATOMIC_RELAXED);
   }
 
   // node at `level` (positions 0..level matched), multiplicity B, key
@@ -195,7 +196,7 @@ struct Walker {
     HList L[7];
     for (int b = 0; b < Lp.nb; ++b) {
       L[b] = in.view(f[Lp.bpos[b]], Lp.bview[b]);
-      out.push_back(Rec{f[Lp.bpos[b]], level, (uint64_t)B});
+      record(f[Lp.bpos[b]], level, (uint64_t)B);
     }
     if (level == k - 2) return;  // children are leaves: they read nothing
     // candidates of position p, each child drawn B' ~ Bin(B, 1/D)
@@ -225,16 +226,22 @@ struct Walker {
 
 }  // namespace
 
-void run_estimator(const EstimatorInput &in, EstimatorOutput &out) {
+void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOutput &out) {
   out.ids.clear();
   out.levcnt.clear();
   const int k = in.plans[0].k;
   if (k <= 2 || in.n_units == 0) return;
+  const int levels = k - 2;
+  if (scr.n != in.n || scr.levels < levels) {
+    scr.n = in.n;
+    scr.levels = levels;
+    scr.sums.assign((size_t)levels * (size_t)in.n, 0);
+    scr.touched.assign(((size_t)in.n + 63) / 64, 0);
+  }
   const int T = std::max(1, in.threads);
-  std::vector<std::vector<Rec>> recs(T);
   const uint64_t root = rng_mix(in.seed);
   const double p1 = 1.0 / (double)in.N1;
-  parallel_dyn(T, in.n_units, 64, [&](int tid, int64_t ui) {
+  parallel_dyn(T, in.n_units, 64, [&](int, int64_t ui) {
     const Unit &u = in.units[ui];
     const int term = u.plan >> 1, kind = u.plan & 1;
     const uint64_t key = rng_chain(rng_chain(rng_chain(rng_chain(rng_chain(root, in.batch_seq), (uint64_t)term),
@@ -242,29 +249,43 @@ void run_estimator(const EstimatorInput &in, EstimatorOutput &out) {
                                    (uint64_t)(uint32_t)u.b);
     const int64_t B = binomial(key, (int64_t)in.M, p1);
     if (B <= 0) return;
-    Walker w(in, recs[tid]);
+    Walker w(in, scr);
     w.P = &in.plans[u.plan];
     w.f[0] = u.a;
     w.f[1] = u.b;
     w.visit(1, B, key);
   });
-  size_t total = 0;
-  for (auto &r : recs) total += r.size();
-  std::vector<Rec> all;
-  all.reserve(total);
-  for (auto &r : recs) all.insert(all.end(), r.begin(), r.end());
-  std::sort(all.begin(), all.end(), [](const Rec &x, const Rec &y) { return x.v < y.v; });
-  for (size_t i = 0; i < all.size();) {
-    size_t j = i;
-    uint64_t lv[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    while (j < all.size() && all[j].v == all[i].v) {
-      lv[all[j].level - 1] += all[j].B;
-      ++j;
+  // touched vertices in ascending order (bitmap scan), their sums, then a sparse reset
+  const int64_t nw = (int64_t)scr.touched.size();
+  const int chunks = std::min<int64_t>(T, nw);
+  std::vector<int64_t> cnt(chunks + 1, 0);
+  parallel_for(chunks, nw, [&](int c, int64_t lo, int64_t hi) {
+    int64_t x = 0;
+    for (int64_t i = lo; i < hi; ++i) x += __builtin_popcountll(scr.touched[i]);
+    cnt[c + 1] = x;
+  });
+  for (int c = 0; c < chunks; ++c) cnt[c + 1] += cnt[c];
+  out.ids.resize(cnt[chunks]);
+  out.levcnt.assign(8 * (size_t)cnt[chunks], 0);
+  parallel_for(chunks, nw, [&](int c, int64_t lo, int64_t hi) {
+    int64_t o = cnt[c];
+    for (int64_t i = lo; i < hi; ++i) {
+      uint64_t w = scr.touched[i];
+      while (w) {
+        const int b = __builtin_ctzll(w);
+        w &= w - 1;
+        const int32_t v = (int32_t)(i * 64 + b);
+        out.ids[o] = v;
+        for (int l = 0; l < levels; ++l) {
+          uint64_t &x = scr.sums[(size_t)l * (size_t)scr.n + (size_t)v];
+          out.levcnt[8 * (size_t)o + l] = x;
+          x = 0;
+        }
+        ++o;
+      }
+      scr.touched[i] = 0;
     }
-    out.ids.push_back(all[i].v);
-    for (int l = 0; l < 8; ++l) out.levcnt.push_back(lv[l]);
-    i = j;
-  }
+  });
 }
 
 // est_v = (1/M) Σ_l N1 D^(l-1) levcnt[v][l]  (eq. (3) averaged over M walks)

@@ -21,8 +21,18 @@ struct EstimatorInput {
   uint64_t N1, D, M;
   uint64_t seed, batch_seq;
   const uint16_t *labels;  // nullptr = all 0
+  int32_t n;               // vertex universe
   int threads;
   std::function<HList(int32_t, int)> view;  // (vertex, View) -> host list view
+};
+
+// Persistent dense accumulators (n x (k-2) sums + a touched bitmap), reset
+// sparsely after each batch: O(records) accumulation, ids come out sorted.
+struct EstimatorScratch {
+  int32_t n = 0;
+  int levels = 0;
+  std::vector<uint64_t> sums;     // [levels][n]
+  std::vector<uint64_t> touched;  // n bits
 };
 
 struct EstimatorOutput {
@@ -31,7 +41,7 @@ struct EstimatorOutput {
 };
 
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k);
-void run_estimator(const EstimatorInput &in, EstimatorOutput &out);
+void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOutput &out);
 double estimate_value(const uint64_t *lev, int k, uint64_t N1, uint64_t D, uint64_t M);
 
 }  // namespace gcsm

@@ -5,8 +5,10 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <parallel/algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -89,12 +91,14 @@ struct gcsm_ctx {
   std::vector<std::pair<int32_t, uint64_t>> prev_slot;  // (vertex, offset) of the previous cache, by vertex
   uint64_t *d_gather = nullptr; size_t gather_cap = 0;  // retained lists: (src, dst, n16) triples
   uint64_t *h_gather = nullptr; size_t h_gather_cap = 0;
+  uint64_t *d_fresh = nullptr; size_t fresh_cap = 0;    // newly cached lists: (host src, dst, n16) triples
+  uint64_t *h_fresh = nullptr; size_t h_fresh_cap = 0;
+  std::vector<int32_t> sel_index;                       // vertex -> index in this batch's selection, or -1
   int64_t *d_pidx = nullptr; size_t pidx_cap = 0;
   VDesc *d_pval = nullptr; size_t pval_cap = 0;
   int32_t *d_tup = nullptr; size_t tup_cap = 0;
 
   // pinned host staging
-  char *h_cache = nullptr; size_t h_cache_cap = 0;
   int64_t *h_pidx = nullptr; size_t h_pidx_cap = 0;
   VDesc *h_pval = nullptr; size_t h_pval_cap = 0;
   DRec *h_drec = nullptr; size_t h_drec_cap = 0;
@@ -108,6 +112,7 @@ struct gcsm_ctx {
   std::vector<int32_t> prev_cached, prev_U;
   std::vector<uint8_t> mark;         // scratch (n)
   EstimatorOutput est;
+  EstimatorScratch est_scratch;
   gcsm_stats stats{};
   uint64_t batch_seq = 0;
   std::vector<int32_t> degree_order;  // GCSM_CACHE_DEGREE ranking
@@ -133,10 +138,10 @@ gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
   void *dev[] = {d_vdesc, d_plans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
-                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum};
+                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh};
   for (void *p : dev)
     if (p) cudaFree(p);
-  void *host[] = {h_cache, h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt, h_gather};
+  void *host[] = {h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt, h_gather, h_fresh};
   for (void *p : host)
     if (p) cudaFreeHost(p);
   for (cudaEvent_t e : {ev_m0, ev_m1, ev_a0, ev_a1, ev_c0, ev_c1})
@@ -273,14 +278,10 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
       if (b) cudaFree(b);
       b = nullptr;
     }
-    if (ctx->h_cache) cudaFreeHost(ctx->h_cache);
-    ctx->h_cache = nullptr;
-    ctx->cache_cap = ctx->h_cache_cap = 0;
+    ctx->cache_cap = 0;
     for (char *&b : ctx->d_cachebuf)
       if (cudaMalloc(&b, bytes) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "device cache allocation failed");
-    if (cudaHostAlloc(&ctx->h_cache, bytes, cudaHostAllocDefault) != cudaSuccess)
-      return ctx->fail(GCSM_ENOMEM, "pinned cache staging allocation failed");
-    ctx->cache_cap = ctx->h_cache_cap = bytes;
+    ctx->cache_cap = bytes;
   }
   ctx->budget = bytes;
   ctx->cache_valid = false;  // the next batch repacks everything
@@ -294,6 +295,25 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
 
 static uint16_t host_label(const HostStore &s, int32_t v) { return s.lab.empty() ? 0 : s.lab[v]; }
 
+// GCSM_TRACE=1: per-batch host sub-step timings on stderr (development aid).
+struct Trace {
+  bool on = std::getenv("GCSM_TRACE") != nullptr;
+  Timer t;
+  double last = 0;
+  std::string line;
+  void mark(const char *name) {
+    if (!on) return;
+    const double now = t.ms();
+    char buf[64];
+    std::snprintf(buf, sizeof buf, " %s=%.2f", name, now - last);
+    line += buf;
+    last = now;
+  }
+  ~Trace() {
+    if (on) std::fprintf(stderr, "[gcsm trace]%s\n", line.c_str());
+  }
+};
+
 static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
                               int32_t *tup_add, uint64_t add_cap, int32_t *tup_rem, uint64_t rem_cap,
                               uint64_t *added, uint64_t *removed) {
@@ -304,6 +324,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   if (listing && ctx->opt.world > 1 && !(ctx->opt.flags & GCSM_FLAG_LOCAL_COUNTS))
     return ctx->fail(GCSM_EINVAL, "list mode is single-GPU");
   Timer total;
+  Trace tr;
   HostStore &S = ctx->store;
   const QueryPlan &Q = ctx->qp;
   const int k = Q.k;
@@ -315,8 +336,10 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   Timer t1;
   std::string e = S.normalize(n_ins, ins, n_del, del);
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
+  tr.mark("normalize");
   bool cuda_err = false;
   if (!S.build_overlay(&cuda_err)) return ctx->fail(GCSM_EDEVICE, "pinned overlay allocation failed");
+  tr.mark("overlay");
   st.n_ins = S.I.size();
   st.n_del = S.D.size();
   st.dropped = S.dropped;
@@ -365,7 +388,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   {  // heaviest units first (dynamic scheduling tail)
     std::vector<size_t> idx(units.size());
     std::iota(idx.begin(), idx.end(), 0);
-    std::stable_sort(idx.begin(), idx.end(), [&](size_t x, size_t y) { return cost[x] > cost[y]; });
+    __gnu_parallel::stable_sort(idx.begin(), idx.end(), [&](size_t x, size_t y) { return cost[x] > cost[y]; });
     std::vector<Unit> u2(units.size());
     std::vector<uint64_t> c2(units.size());
     for (size_t i = 0; i < idx.size(); ++i) {
@@ -376,6 +399,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     cost.swap(c2);
   }
   const int64_t nu = (int64_t)units.size();
+  tr.mark("units");
   st.units = st.n1 = (uint64_t)nu;
   const uint64_t D = std::max<uint64_t>(1, std::max<uint64_t>(S.maxdeg, S.maxdeg_new));
   st.max_degree = D;
@@ -404,7 +428,9 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
       in.labels = S.lab.empty() ? nullptr : S.lab.data();
       in.threads = T;
       in.view = [&S](int32_t v, int vw) { return S.view(v, vw); };
-      run_estimator(in, ctx->est);
+      in.n = S.n;
+      run_estimator(in, ctx->est_scratch, ctx->est);
+      tr.mark("walks");
       if (use_cache) {
         ranked.reserve(ctx->est.ids.size());
         for (size_t i = 0; i < ctx->est.ids.size(); ++i)
@@ -420,6 +446,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     }
   }
   st.ms_estimate = t2.ms();
+  tr.mark("score");
 
   // ---- (3) pack the cache + descriptors --------------------------------------------------
   Timer t3;
@@ -430,13 +457,16 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   // previous batch (not updated then, not updated now) is copied HBM -> HBM; only the other lists go through
   // pinned staging and the one H2D DMA.
   std::vector<uint64_t> gather;  // (src offset, dst offset, 16-byte units) per retained list
+  std::vector<uint64_t> fresh;   // (src host address, dst offset, 16-byte units) per newly cached list
   uint64_t new_bytes = 0;
   const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
   ctx->d_cache = ctx->d_cachebuf[tgt];
   if (use_cache && !ranked.empty()) {
-    std::sort(ranked.begin(), ranked.end(), [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {
-      return x.first > y.first || (x.first == y.first && x.second < y.second);
-    });
+    __gnu_parallel::sort(ranked.begin(), ranked.end(),
+                         [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {
+                           return x.first > y.first || (x.first == y.first && x.second < y.second);
+                         });
+    tr.mark("rank_sort");
     std::vector<uint64_t> bytes_of;
     for (const auto &r : ranked) {
       if (!(r.first > 0)) break;
@@ -468,22 +498,21 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
         o += bytes_of[i];
       }
     const uint64_t retained = o;
-    std::vector<size_t> fresh;
+    // the newly selected lists are pulled by the GPU straight from the pinned host store (zero-copy bulk reads,
+    // warp per list): the same bytes as the paper's packed DMA without a host-side packing copy
     for (size_t i = 0; i < sel.size(); ++i)
       if (old_off[i] < 0) {
         sel_off[i] = o;
+        const HList h = S.view(sel[i], VIEW_S);
+        fresh.push_back((uint64_t)(uintptr_t)S.dev_ptr(h.a));
+        fresh.push_back(o);
+        fresh.push_back(bytes_of[i] / 16);
         o += bytes_of[i];
-        fresh.push_back(i);
       }
     new_bytes = o - retained;
-    parallel_for(T, (int64_t)fresh.size(), [&](int, int64_t lo, int64_t hi) {
-      for (int64_t j = lo; j < hi; ++j) {
-        const size_t i = fresh[j];
-        const HList h = S.view(sel[i], VIEW_S);
-        std::memcpy(ctx->h_cache + (sel_off[i] - retained), h.a, (size_t)h.na * 4);
-      }
-    });
+    tr.mark("layout");
   }
+  tr.mark("stage_copy");
   st.cached_vertices = sel.size();
   st.cache_bytes = used;
   // descriptors to patch: previous cache / updated sets and the new ones
@@ -500,37 +529,26 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   for (int32_t v : S.U) add_dirty(v);
   for (int32_t v : sel) add_dirty(v);
   for (int32_t v : dirty) ctx->mark[v] = 0;
-  std::vector<int64_t> cache_slot;  // per dirty vertex: offset or -1
-  {
-    // map selected -> offset via a temporary mark pass
-    for (size_t i = 0; i < sel.size(); ++i) ctx->mark[sel[i]] = 1;
-  }
+  if (ctx->sel_index.size() != (size_t)S.n) ctx->sel_index.assign(S.n, -1);
+  for (size_t i = 0; i < sel.size(); ++i) ctx->sel_index[sel[i]] = (int32_t)i;
   if (!host_ensure(ctx->h_pidx, ctx->h_pidx_cap, dirty.size()) ||
       !host_ensure(ctx->h_pval, ctx->h_pval_cap, dirty.size()))
     return ctx->fail(GCSM_ENOMEM, "pinned staging");
-  {
-    std::vector<int64_t> off_of;  // only for selected; find by binary search over a sorted copy
-    std::vector<std::pair<int32_t, uint64_t>> so(sel.size());
-    for (size_t i = 0; i < sel.size(); ++i) so[i] = {sel[i], sel_off[i]};
-    std::sort(so.begin(), so.end());
-    for (size_t i = 0; i < dirty.size(); ++i) {
+  parallel_for(T, (int64_t)dirty.size(), [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
       const int32_t v = dirty[i];
       const int32_t ui = S.uidx[v];
       VDesc d;
       d.upd = ui >= 0 ? (uint32_t)ui + 1 : 0;
       d.len = ui >= 0 ? S.s_len[ui] : S.len[v];
-      if (ctx->mark[v]) {
-        auto it = std::lower_bound(so.begin(), so.end(), std::make_pair(v, (uint64_t)0));
-        d.ptr = (const int32_t *)(ctx->d_cache + it->second);
-      } else {
-        d.ptr = S.dev_ptr(ui >= 0 ? S.s_ptr[ui] : S.lst[v]);
-      }
+      const int32_t si = ctx->sel_index[v];
+      d.ptr = si >= 0 ? (const int32_t *)(ctx->d_cache + sel_off[si]) : S.dev_ptr(ui >= 0 ? S.s_ptr[ui] : S.lst[v]);
       ctx->h_pidx[i] = v;
       ctx->h_pval[i] = d;
-      ctx->vd[v] = d;
     }
-  }
-  for (int32_t v : sel) ctx->mark[v] = 0;
+  });
+  for (int32_t v : sel) ctx->sel_index[v] = -1;
+  tr.mark("descriptors");
   // delta lists of U
   const size_t nU = S.U.size();
   const size_t nd = S.ins_val.size() + S.del_val.size();
@@ -544,6 +562,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   std::memcpy(ctx->h_dlist + S.ins_val.size(), S.del_val.data(), S.del_val.size() * 4);
   std::memcpy(ctx->h_units, units.data(), sizeof(Unit) * (size_t)nu);
   st.ms_pack = t3.ms();
+  tr.mark("staging");
 
   cudaStream_t s = ctx->stream;
   if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
@@ -560,8 +579,15 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     CK(cudaMemcpyAsync(ctx->d_gather, ctx->h_gather, 8 * gather.size(), cudaMemcpyHostToDevice, s));
     CK(launch_gather_lists(ctx->d_cache, ctx->d_cachebuf[ctx->cache_cur], ctx->d_gather, (int64_t)gather.size() / 3, s));
   }
-  if (new_bytes)  // the one DMA of the newly selected lists
-    CK(cudaMemcpyAsync(ctx->d_cache + retained_bytes, ctx->h_cache, new_bytes, cudaMemcpyHostToDevice, s));
+  if (!fresh.empty()) {  // newly selected lists: GPU gather over PCIe from the mapped host store
+    if (!host_ensure(ctx->h_fresh, ctx->h_fresh_cap, fresh.size()) ||
+        !dev_ensure(ctx->d_fresh, ctx->fresh_cap, fresh.size()))
+      return ctx->fail(GCSM_ENOMEM, "gather staging");
+    std::memcpy(ctx->h_fresh, fresh.data(), 8 * fresh.size());
+    CK(cudaMemcpyAsync(ctx->d_fresh, ctx->h_fresh, 8 * fresh.size(), cudaMemcpyHostToDevice, s));
+    CK(launch_gather_lists(ctx->d_cache, nullptr, ctx->d_fresh, (int64_t)fresh.size() / 3, s));
+  }
+  (void)retained_bytes;
   CK(cudaMemcpyAsync(ctx->d_pidx, ctx->h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(ctx->d_pval, ctx->h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(launch_patch_vdesc(ctx->d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
@@ -570,7 +596,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, ctx->h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
   if (nu) CK(cudaMemcpyAsync(ctx->d_units, ctx->h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(ctx->ev_c1, s));
-  st.h2d_bytes = new_bytes + 8 * gather.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
+  st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
                  4 * nd + sizeof(Unit) * (size_t)nu;
 
   // ---- (4) matching kernels --------------------------------------------------------------
@@ -716,8 +742,10 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   }
 
   // ---- (5) reorganise the host lists (after matching) -----------------------------
+  tr.mark("gpu");
   Timer t5;
   S.merge();
+  tr.mark("merge");
   ctx->prev_cached = sel;
   std::sort(ctx->prev_cached.begin(), ctx->prev_cached.end());
   ctx->prev_slot.resize(sel.size());

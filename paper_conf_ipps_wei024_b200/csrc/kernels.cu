@@ -537,16 +537,25 @@ __global__ void k_group_scatter(const int32_t *f2c, const unsigned long long *cn
     group[atomicAdd(&cursor[f2c[e]], 1u)] = (int32_t)e;
 }
 
-// Warp per retained cache list: copy n16 16-byte granules from the previous cache buffer.
+// Warp per cache list: copy n16 16-byte granules to dst + tri[3i+1] from src + tri[3i] (src == nullptr: tri[3i] is
+// an absolute address — a mapped pinned host list pulled over PCIe; else an offset into the previous cache buffer).
 __global__ void k_gather(char *dst, const char *src, const uint64_t *tri, int64_t n) {
   const int lane = threadIdx.x & 31;
   const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t i = w; i < n; i += nw) {
-    const int4 *s4 = reinterpret_cast<const int4 *>(src + tri[3 * i]);
+    const int4 *s4 = reinterpret_cast<const int4 *>(src ? src + tri[3 * i] : reinterpret_cast<const char *>(tri[3 * i]));
     int4 *d4 = reinterpret_cast<int4 *>(dst + tri[3 * i + 1]);
     const uint64_t n16 = tri[3 * i + 2];
-    for (uint64_t j = lane; j < n16; j += 32) d4[j] = s4[j];
+    for (uint64_t base = 0; base < n16; base += 128) {  // 4 x 16 B per lane in flight
+      int4 v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (base + lane + 32 * u < n16) v[u] = s4[base + lane + 32 * u];
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (base + lane + 32 * u < n16) d4[base + lane + 32 * u] = v[u];
+    }
   }
 }
 
