@@ -24,6 +24,7 @@
 //     generic load path, UVA decides the route.
 //   * counts: per-warp registers, one 64-bit atomic per warp and counter at
 //     the end of the persistent loop.
+#include <climits>
 #include <cstdio>
 
 #include "kernels.cuh"
@@ -206,6 +207,81 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
   if (any) __syncwarp();
 }
 
+// ---- merge-path intersection count (two sorted runs) ------------------------------
+// The warp splits the merged sequence a ∪ b into 32 equal diagonal ranges; each lane finds its start by a
+// co-rank binary search and merges its range sequentially, counting a[i] == b[j] when it consumes a[i] (ties
+// take A first, so an equal pair is counted exactly once even across lane boundaries). O((na+nb)/32 + log)
+// instructions per lane instead of ceil(d/32) * log2(L) dependent probes.
+__device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, const int32_t *b, uint32_t nb,
+                                                int label, const uint16_t *lab, int lane) {
+  const uint32_t T = na + nb;
+  const uint32_t d0 = (uint32_t)(((uint64_t)T * (uint32_t)lane) >> 5);
+  const uint32_t d1 = (uint32_t)(((uint64_t)T * (uint32_t)(lane + 1)) >> 5);
+  uint32_t lo = d0 > nb ? d0 - nb : 0, hi = d0 < na ? d0 : na;
+  while (lo < hi) {
+    const uint32_t i = (lo + hi) >> 1;
+    if (a[i] <= b[d0 - i - 1]) lo = i + 1;
+    else hi = i;
+  }
+  uint32_t i = lo, j = d0 - lo, cnt = 0;
+  int32_t ai = i < na ? a[i] : INT_MAX, bj = j < nb ? b[j] : INT_MAX;
+  for (uint32_t st = d0; st < d1; ++st) {
+    if (ai <= bj) {
+      if (ai == bj && (label < 0 || lab[ai] == (uint16_t)label)) ++cnt;
+      ++i;
+      ai = i < na ? a[i] : INT_MAX;
+    } else {
+      ++j;
+      bj = j < nb ? b[j] : INT_MAX;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
+  return cnt;
+}
+
+// lane-parallel count of x[0..nx) present in the sorted list y (label-filtered)
+__device__ __forceinline__ uint32_t probe_count(const int32_t *x, uint32_t nx, const int32_t *y, uint32_t ny, int label,
+                                                const uint16_t *lab, int lane) {
+  uint32_t cnt = 0;
+  for (uint32_t i = lane; i < nx; i += 32) {
+    const int32_t v = x[i];
+    if (bsearch_has(y, ny, v) && (label < 0 || lab[v] == (uint16_t)label)) ++cnt;
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
+  return cnt;
+}
+
+__device__ __forceinline__ bool is_host(const MatchArgs &A, const int32_t *p) {
+  return !(is_hit(A, p) || is_device(A, p) || __isShared(p));
+}
+
+__device__ __forceinline__ uint32_t ilog2(uint32_t x) { return 31u - __clz(x | 1u); }
+
+// Count of the last level for two lists without a reused set: merge path when both main runs are in device
+// memory and it is cheaper than per-lane binary search; the tiny delta runs are probed; excluded (matched,
+// non-adjacent) vertices that lie in the intersection are subtracted. Returns false if not applicable.
+__device__ __forceinline__ bool count2(const MatchArgs &A, const LRef *L, int drv, const int32_t *excl, int nexcl,
+                                       int label, int lane, uint32_t *out) {
+  const LRef &X = L[drv], &Y = L[1 - drv];
+  if (X.ml < 8 || Y.ml < 8 || is_host(A, X.m) || is_host(A, Y.m)) return false;
+  const uint32_t d = X.ml + X.xl, big = Y.ml + Y.xl;
+  const uint32_t bs_cost = ((d + 31) >> 5) * (7 * ilog2(big) + 12);
+  const uint32_t mg_cost = 10 * ilog2(min(X.ml, Y.ml)) + 7 * ((X.ml + Y.ml + 31) >> 5) + 30;
+  if (mg_cost >= bs_cost) return false;
+  uint32_t c = merge_count(X.m, X.ml, Y.m, Y.ml, label, A.lab, lane);
+  if (X.xl) c += probe_count(X.x, X.xl, Y.m, Y.ml, label, A.lab, lane);
+  if (Y.xl) c += probe_count(Y.x, Y.xl, X.m, X.ml, label, A.lab, lane);
+  if (X.xl && Y.xl) c += probe_count(X.x, X.xl, Y.x, Y.xl, label, A.lab, lane);
+  for (int e = 0; e < nexcl; ++e) {
+    const int32_t v = excl[e];
+    if ((label < 0 || A.lab[v] == (uint16_t)label) && contains(X, v) && contains(Y, v)) --c;
+  }
+  *out = c;
+  return true;
+}
+
 // Lists of position p for the current partial match f (positions 0..p-1).
 // Returns the number of probe lists written to L and sets *drv (index of the
 // smallest list) or uses the reused set.
@@ -302,7 +378,9 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
     int nex = 0;
     for (int i = 0; i < L2.ninj; ++i) excl[nex++] = f[L2.inj[i]];
     if (A.k == 3 && !LIST) {
-      const uint32_t c = warp_isect<false>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, nullptr, lane);
+      uint32_t c;
+      if (nl != 2 || !count2(A, L, drv, excl, nex, L2.label, lane, &c))
+        c = warp_isect<false>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, nullptr, lane);
       if (P.kind) acc.rem += c;
       else acc.add += c;
       continue;
@@ -419,7 +497,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
             __syncwarp();
             emit_tuples(A, P, f, P.kind, lastbuf, c, lane);
             __syncwarp();
-          } else {
+          } else if (dset || nl != 2 || !count2(A, L, drv, excl, nex, Lp.label, lane, &c)) {
             c = warp_isect<false>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, nullptr, lane);
           }
           if (P.kind) acc.rem += c;

@@ -1,0 +1,7 @@
+#!/bin/bash
+# full ncu capture of k_extend for c4 and k4 (second batch), tag in $1
+T=${1:-dev}
+ncu --set full --clock-control none --import-source on -k regex:k_extend -s 1 -c 1 -o gpurun_out/prof_ext_c4_$T -f \
+    python bench.py --steps 1 --warmup 1 --quick --queries c4 > gpurun_out/ncu_c4_$T.txt 2>&1
+ncu --set full --clock-control none --import-source on -k regex:k_extend -s 1 -c 1 -o gpurun_out/prof_ext_k4_$T -f \
+    python bench.py --steps 1 --warmup 1 --quick --queries k4 > gpurun_out/ncu_k4_$T.txt 2>&1
