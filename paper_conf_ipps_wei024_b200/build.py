@@ -37,9 +37,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB_PATH
     inc, lib = _nccl_dirs()
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    cmd = [nvcc, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v", "-Xcompiler", "-fPIC,-O3,-fopenmp",
+    cmd = [nvcc, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v", "-Xcompiler", "-fPIC,-O3",
            "-shared", "-cudart", "static", f"-I{os.path.join(ROOT, 'include')}", f"-I{inc}", *srcs,
-           "-o", LIB_PATH + ".tmp", f"-L{lib}", "-l:libnccl.so.2", "-Xlinker", f"-rpath,{lib}", "-lpthread", "-lgomp"]
+           "-o", LIB_PATH + ".tmp", f"-L{lib}", "-l:libnccl.so.2", "-Xlinker", f"-rpath,{lib}", "-lpthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)

@@ -18,9 +18,12 @@
 //  * the binomial B' of a child only depends on the child's key, so a child
 //    whose draw is 0 is discarded before its (costly) membership probes when
 //    the inversion branch is used (B/D < 10): the first uniform decides B' = 0.
+#include <immintrin.h>
+
 #include <algorithm>
 #include <cmath>
 #include <cstring>
+#include <memory>
 
 #include "estimator.h"
 
@@ -150,6 +153,60 @@ static inline bool first_uniform_le(uint64_t key, double r0) {
   return !(U.next() > r0);
 }
 
+// Children of one node whose draw B' ~ Bin(B, p) is non-zero under the inversion branch: the first uniform of
+// the child's stream exceeds r0 = (1-p)^B. With u = m * 2^-53 (m = mix(key' + C) >> 11, exact) the test
+// u > r0 is the integer test m > floor(r0 * 2^53) — the same decision, evaluated 8 children at a time.
+static inline uint64_t mix_s(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+
+static void coin_filter_scalar(const int32_t *v, uint32_t n, uint64_t key, uint64_t T, std::vector<uint32_t> &out) {
+  for (uint32_t i = 0; i < n; ++i) {
+    const uint64_t ck = mix_s(key + 0x9E3779B97F4A7C15ULL * ((uint64_t)(uint32_t)v[i] + 1));
+    if ((mix_s(ck + 0xD1B54A32D192ED03ULL) >> 11) > T) out.push_back(i);
+  }
+}
+
+__attribute__((target("avx512f,avx512dq"))) static inline __m512i mix_v(__m512i z, __m512i C1, __m512i C2) {
+  z = _mm512_mullo_epi64(_mm512_xor_si512(z, _mm512_srli_epi64(z, 30)), C1);
+  z = _mm512_mullo_epi64(_mm512_xor_si512(z, _mm512_srli_epi64(z, 27)), C2);
+  return _mm512_xor_si512(z, _mm512_srli_epi64(z, 31));
+}
+
+__attribute__((target("avx512f,avx512dq"))) static void coin_filter_avx512(const int32_t *v, uint32_t n, uint64_t key,
+                                                                           uint64_t T, std::vector<uint32_t> &out) {
+  const __m512i G = _mm512_set1_epi64((long long)0x9E3779B97F4A7C15ULL);
+  const __m512i K = _mm512_set1_epi64((long long)key);
+  const __m512i C1 = _mm512_set1_epi64((long long)0xBF58476D1CE4E5B9ULL);
+  const __m512i C2 = _mm512_set1_epi64((long long)0x94D049BB133111EBULL);
+  const __m512i D1 = _mm512_set1_epi64((long long)0xD1B54A32D192ED03ULL);
+  const __m512i one = _mm512_set1_epi64(1);
+  const __m512i TT = _mm512_set1_epi64((long long)T);
+  uint32_t i = 0;
+  for (; i + 8 <= n; i += 8) {
+    const __m512i x = _mm512_add_epi64(_mm512_cvtepu32_epi64(_mm256_loadu_si256((const __m256i *)(v + i))), one);
+    const __m512i ck = mix_v(_mm512_add_epi64(K, _mm512_mullo_epi64(G, x)), C1, C2);
+    const __m512i m = _mm512_srli_epi64(mix_v(_mm512_add_epi64(ck, D1), C1, C2), 11);
+    __mmask8 k = _mm512_cmpgt_epu64_mask(m, TT);
+    while (k) {
+      out.push_back(i + (uint32_t)__builtin_ctz(k));
+      k &= (__mmask8)(k - 1);
+    }
+  }
+  for (; i < n; ++i) {
+    const uint64_t ck = mix_s(key + 0x9E3779B97F4A7C15ULL * ((uint64_t)(uint32_t)v[i] + 1));
+    if ((mix_s(ck + 0xD1B54A32D192ED03ULL) >> 11) > T) out.push_back(i);
+  }
+}
+
+static void coin_filter(const int32_t *v, uint32_t n, uint64_t key, uint64_t T, std::vector<uint32_t> &out) {
+  static const bool avx512 = __builtin_cpu_supports("avx512f") && __builtin_cpu_supports("avx512dq");
+  if (avx512) coin_filter_avx512(v, n, key, T, out);
+  else coin_filter_scalar(v, n, key, T, out);
+}
+
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k) {
   // M = floor(N1 * D^(k-2) / 32^k), clamped to [1, 2^62] (R21), exact integer arithmetic.
   if (N1 == 0) return 1;
@@ -174,6 +231,7 @@ struct Walker {
   EstimatorScratch &scr;
   const DevPlan *P = nullptr;
   int32_t f[GCSM_MAXK];
+  std::vector<uint32_t> keep_[GCSM_MAXK];
   Walker(const EstimatorInput &i, EstimatorScratch &s) : in(i), scr(s) {}
 
   bool member(const HList &L, int32_t v) const {
@@ -219,8 +277,19 @@ struct Walker {
       f[p] = v;
       visit(level + 1, Bc, ck);
     };
-    for (uint32_t i = 0; i < L[drv].na; ++i) consider(L[drv].a[i]);
-    for (uint32_t i = 0; i < L[drv].nb; ++i) consider(L[drv].b[i]);
+    if (fast) {  // vectorised B' = 0 pre-filter (same decision as first_uniform_le)
+      const uint64_t T = (uint64_t)std::floor(r0 * 9007199254740992.0);
+      std::vector<uint32_t> &keep = keep_[level];  // reused per depth (no per-node allocation)
+      keep.clear();
+      coin_filter(L[drv].a, L[drv].na, key, T, keep);
+      for (uint32_t i : keep) consider(L[drv].a[i]);
+      keep.clear();
+      if (L[drv].nb) coin_filter(L[drv].b, L[drv].nb, key, T, keep);
+      for (uint32_t i : keep) consider(L[drv].b[i]);
+    } else {
+      for (uint32_t i = 0; i < L[drv].na; ++i) consider(L[drv].a[i]);
+      for (uint32_t i = 0; i < L[drv].nb; ++i) consider(L[drv].b[i]);
+    }
   }
 };
 
@@ -241,7 +310,9 @@ void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOut
   const int T = std::max(1, in.threads);
   const uint64_t root = rng_mix(in.seed);
   const double p1 = 1.0 / (double)in.N1;
-  parallel_dyn(T, in.n_units, 64, [&](int, int64_t ui) {
+  std::vector<std::unique_ptr<Walker>> walkers(T);
+  for (auto &w : walkers) w.reset(new Walker(in, scr));
+  parallel_dyn(T, in.n_units, 64, [&](int tid, int64_t ui) {
     const Unit &u = in.units[ui];
     const int term = u.plan >> 1, kind = u.plan & 1;
     const uint64_t key = rng_chain(rng_chain(rng_chain(rng_chain(rng_chain(root, in.batch_seq), (uint64_t)term),
@@ -249,7 +320,7 @@ void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOut
                                    (uint64_t)(uint32_t)u.b);
     const int64_t B = binomial(key, (int64_t)in.M, p1);
     if (B <= 0) return;
-    Walker w(in, scr);
+    Walker &w = *walkers[tid];
     w.P = &in.plans[u.plan];
     w.f[0] = u.a;
     w.f[1] = u.b;

@@ -5,7 +5,6 @@
 #include <nccl.h>
 
 #include <algorithm>
-#include <parallel/algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -34,7 +33,7 @@ bool dev_ensure(T *&p, size_t &cap, size_t need) {
   p = nullptr;
   cap = 0;
   size_t n = std::max<size_t>(need, 1);
-  n = n + n / 4;
+  n = 2 * n;
   if (cudaMalloc((void **)&p, n * sizeof(T)) != cudaSuccess) return false;
   cap = n;
   return true;
@@ -47,7 +46,7 @@ bool host_ensure(T *&p, size_t &cap, size_t need) {
   p = nullptr;
   cap = 0;
   size_t n = std::max<size_t>(need, 1);
-  n = n + n / 4;
+  n = 2 * n;
   if (cudaHostAlloc((void **)&p, n * sizeof(T), cudaHostAllocDefault) != cudaSuccess) return false;
   cap = n;
   return true;
@@ -362,16 +361,18 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     }
   // cost proxy of a unit: the list lengths its first level reads
   cost.resize(units.size());
-  for (size_t i = 0; i < units.size(); ++i) {
-    const DevPlan &P = Q.plans[units[i].plan];
-    uint64_t c = 1;
-    if (k > 2) {
-      const LevelPlan &L2 = P.lv[2];
-      const int32_t f[2] = {units[i].a, units[i].b};
-      for (int b = 0; b < L2.nb; ++b) c += S.view_len(f[L2.bpos[b]], L2.bview[b]);
+  parallel_for(T, (int64_t)units.size(), [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      const DevPlan &P = Q.plans[units[i].plan];
+      uint64_t c = 1;
+      if (k > 2) {
+        const LevelPlan &L2 = P.lv[2];
+        const int32_t f[2] = {units[i].a, units[i].b};
+        for (int b = 0; b < L2.nb; ++b) c += S.view_len(f[L2.bpos[b]], L2.bview[b]);
+      }
+      cost[i] = c;
     }
-    cost[i] = c;
-  }
+  });
   if (ctx->opt.world > 1) {
     std::vector<int32_t> rk(units.size());
     shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data());
@@ -388,7 +389,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   {  // heaviest units first (dynamic scheduling tail)
     std::vector<size_t> idx(units.size());
     std::iota(idx.begin(), idx.end(), 0);
-    __gnu_parallel::stable_sort(idx.begin(), idx.end(), [&](size_t x, size_t y) { return cost[x] > cost[y]; });
+    parallel_sort(idx, [&](size_t x, size_t y) { return cost[x] > cost[y]; }, T, /*stable=*/true);
     std::vector<Unit> u2(units.size());
     std::vector<uint64_t> c2(units.size());
     for (size_t i = 0; i < idx.size(); ++i) {
@@ -432,9 +433,11 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
       run_estimator(in, ctx->est_scratch, ctx->est);
       tr.mark("walks");
       if (use_cache) {
-        ranked.reserve(ctx->est.ids.size());
-        for (size_t i = 0; i < ctx->est.ids.size(); ++i)
-          ranked.emplace_back(estimate_value(&ctx->est.levcnt[8 * i], k, (uint64_t)nu, D, M), ctx->est.ids[i]);
+        ranked.resize(ctx->est.ids.size());
+        parallel_for(T, (int64_t)ranked.size(), [&](int, int64_t lo, int64_t hi) {
+          for (int64_t i = lo; i < hi; ++i)
+            ranked[i] = {estimate_value(&ctx->est.levcnt[8 * i], k, (uint64_t)nu, D, M), ctx->est.ids[i]};
+        });
       }
     }
   }
@@ -462,30 +465,40 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
   ctx->d_cache = ctx->d_cachebuf[tgt];
   if (use_cache && !ranked.empty()) {
-    __gnu_parallel::sort(ranked.begin(), ranked.end(),
-                         [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {
-                           return x.first > y.first || (x.first == y.first && x.second < y.second);
-                         });
+    parallel_sort(
+        ranked,
+        [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {
+          return x.first > y.first || (x.first == y.first && x.second < y.second);
+        },
+        T);
     tr.mark("rank_sort");
+    // list bytes of every ranked vertex (random accesses: in parallel), then the sequential prefix (R23)
+    std::vector<uint64_t> rbytes(ranked.size());
+    parallel_for(T, (int64_t)ranked.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i) rbytes[i] = (uint64_t)((S.view_len(ranked[i].second, VIEW_S) + 3u) & ~3u) * 4;
+    });
     std::vector<uint64_t> bytes_of;
-    for (const auto &r : ranked) {
-      if (!(r.first > 0)) break;
-      const uint64_t bytes = (uint64_t)((S.view_len(r.second, VIEW_S) + 3u) & ~3u) * 4;
-      if (used + bytes > ctx->budget) break;  // longest prefix that fits (R23)
-      sel.push_back(r.second);
-      bytes_of.push_back(bytes);
-      used += bytes;
+    for (size_t i = 0; i < ranked.size(); ++i) {
+      if (!(ranked[i].first > 0)) break;
+      if (used + rbytes[i] > ctx->budget) break;  // longest prefix that fits (R23)
+      sel.push_back(ranked[i].second);
+      bytes_of.push_back(rbytes[i]);
+      used += rbytes[i];
     }
     // retained lists first, then the new ones
     for (int32_t v : ctx->prev_U) ctx->mark[v] = 2;
     std::vector<int64_t> old_off(sel.size(), -1);
-    if (ctx->cache_valid)
-      for (size_t i = 0; i < sel.size(); ++i) {
+    std::vector<uint64_t> src(sel.size(), 0);
+    parallel_for(T, (int64_t)sel.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i) {
         const int32_t v = sel[i];
-        if (ctx->mark[v] == 2 || S.uidx[v] >= 0) continue;
-        auto it = std::lower_bound(ctx->prev_slot.begin(), ctx->prev_slot.end(), std::make_pair(v, (uint64_t)0));
-        if (it != ctx->prev_slot.end() && it->first == v) old_off[i] = (int64_t)it->second;
+        if (ctx->cache_valid && ctx->mark[v] != 2 && S.uidx[v] < 0) {
+          auto it = std::lower_bound(ctx->prev_slot.begin(), ctx->prev_slot.end(), std::make_pair(v, (uint64_t)0));
+          if (it != ctx->prev_slot.end() && it->first == v) old_off[i] = (int64_t)it->second;
+        }
+        if (old_off[i] < 0) src[i] = (uint64_t)(uintptr_t)S.dev_ptr(S.view(v, VIEW_S).a);
       }
+    });
     for (int32_t v : ctx->prev_U) ctx->mark[v] = 0;
     sel_off.assign(sel.size(), 0);
     uint64_t o = 0;
@@ -503,8 +516,7 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
     for (size_t i = 0; i < sel.size(); ++i)
       if (old_off[i] < 0) {
         sel_off[i] = o;
-        const HList h = S.view(sel[i], VIEW_S);
-        fresh.push_back((uint64_t)(uintptr_t)S.dev_ptr(h.a));
+        fresh.push_back(src[i]);
         fresh.push_back(o);
         fresh.push_back(bytes_of[i] / 16);
         o += bytes_of[i];
@@ -517,18 +529,25 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   st.cache_bytes = used;
   // descriptors to patch: previous cache / updated sets and the new ones
   std::vector<int32_t> dirty;
-  dirty.reserve(ctx->prev_cached.size() + ctx->prev_U.size() + S.U.size() + sel.size());
-  auto add_dirty = [&](int32_t v) {
-    if (!ctx->mark[v]) {
-      ctx->mark[v] = 1;
-      dirty.push_back(v);
-    }
-  };
-  for (int32_t v : ctx->prev_cached) add_dirty(v);
-  for (int32_t v : ctx->prev_U) add_dirty(v);
-  for (int32_t v : S.U) add_dirty(v);
-  for (int32_t v : sel) add_dirty(v);
-  for (int32_t v : dirty) ctx->mark[v] = 0;
+  {
+    const std::vector<int32_t> *srcs[4] = {&ctx->prev_cached, &ctx->prev_U, &S.U, &sel};
+    std::vector<int64_t> base(5, 0);
+    for (int i = 0; i < 4; ++i) base[i + 1] = base[i] + (int64_t)srcs[i]->size();
+    const int nt = std::max(1, std::min(T, pool_size()));
+    std::vector<std::vector<int32_t>> part(nt);
+    parallel_for(nt, base[4], [&](int tid, int64_t lo, int64_t hi) {
+      for (int64_t g = lo; g < hi; ++g) {
+        int l = 0;
+        while (g >= base[l + 1]) ++l;
+        const int32_t v = (*srcs[l])[g - base[l]];
+        if (__atomic_exchange_n(&ctx->mark[v], (uint8_t)1, __ATOMIC_RELAXED) == 0) part[tid].push_back(v);
+      }
+    });
+    for (auto &p : part) dirty.insert(dirty.end(), p.begin(), p.end());
+    parallel_for(T, (int64_t)dirty.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i) ctx->mark[dirty[i]] = 0;
+    });
+  }
   if (ctx->sel_index.size() != (size_t)S.n) ctx->sel_index.assign(S.n, -1);
   for (size_t i = 0; i < sel.size(); ++i) ctx->sel_index[sel[i]] = (int32_t)i;
   if (!host_ensure(ctx->h_pidx, ctx->h_pidx_cap, dirty.size()) ||

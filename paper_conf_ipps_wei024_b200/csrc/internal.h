@@ -108,6 +108,41 @@ inline void parallel_dyn(int threads, int64_t n, int64_t chunk, const std::funct
   });
 }
 
+// Parallel merge sort on the worker pool (no OpenMP: its spinning team would
+// compete with the pool for the cores). Stable if `stable`.
+template <typename T, typename Cmp>
+void parallel_sort(std::vector<T> &v, Cmp cmp, int threads, bool stable = false) {
+  const int64_t n = (int64_t)v.size();
+  int t = 1;
+  while (t * 2 <= threads && n / (t * 2) >= 4096) t *= 2;
+  if (t == 1) {
+    if (stable) std::stable_sort(v.begin(), v.end(), cmp);
+    else std::sort(v.begin(), v.end(), cmp);
+    return;
+  }
+  std::vector<int64_t> cut(t + 1);
+  for (int i = 0; i <= t; ++i) cut[i] = n * i / t;
+  parallel_for(t, t, [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      if (stable) std::stable_sort(v.begin() + cut[i], v.begin() + cut[i + 1], cmp);
+      else std::sort(v.begin() + cut[i], v.begin() + cut[i + 1], cmp);
+    }
+  });
+  std::vector<T> tmp(v.size());
+  std::vector<T> *src = &v, *dst = &tmp;
+  for (int w = 1; w < t; w *= 2) {
+    const int pairs = t / (2 * w);
+    parallel_for(pairs, pairs, [&](int, int64_t lo, int64_t hi) {
+      for (int64_t p = lo; p < hi; ++p) {
+        const int64_t a = cut[2 * w * p], b = cut[2 * w * p + w], c = cut[2 * w * (p + 1)];
+        std::merge(src->begin() + a, src->begin() + b, src->begin() + b, src->begin() + c, dst->begin() + a, cmp);
+      }
+    });
+    std::swap(src, dst);
+  }
+  if (src != &v) v.swap(tmp);
+}
+
 // ------------------------------------------------------------ plan (plan.cpp)
 struct QueryPlan {
   int k = 0, m = 0;
