@@ -9,7 +9,8 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libgcsm.so")
+# GCSM_LIB selects a tuning variant built by build.build(out=..., defines=...) (development only)
+LIB_PATH = os.environ.get("GCSM_LIB") or os.path.join(HERE, "libgcsm.so")
 
 STATUS = {0: "GCSM_OK", 1: "GCSM_EINVAL", 2: "GCSM_ENOMEM", 3: "GCSM_EDEVICE", 4: "GCSM_ENCCL", 5: "GCSM_ESTATE",
           6: "GCSM_ETRUNC"}

@@ -29,27 +29,30 @@ def sources():
     return sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu")) + glob.glob(os.path.join(HERE, "csrc", "*.cpp")))
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    """Compile libgcsm.so (or a variant to `out` with extra -D defines, for tuning experiments)."""
     srcs = sources()
+    target = out or LIB_PATH
     deps = srcs + glob.glob(os.path.join(HERE, "csrc", "*.h")) + glob.glob(os.path.join(HERE, "csrc", "*.cuh")) + \
         [os.path.join(ROOT, "include", "gcsm.h")]
-    if not force and os.path.exists(LIB_PATH) and os.path.getmtime(LIB_PATH) >= max(os.path.getmtime(d) for d in deps):
-        return LIB_PATH
+    if not force and os.path.exists(target) and os.path.getmtime(target) >= max(os.path.getmtime(d) for d in deps):
+        return target
     inc, lib = _nccl_dirs()
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
     cmd = [nvcc, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v", "-Xcompiler", "-fPIC,-O3",
            "-shared", "-cudart", "static", f"-I{os.path.join(ROOT, 'include')}", f"-I{inc}", *srcs,
-           "-o", LIB_PATH + ".tmp", f"-L{lib}", "-l:libnccl.so.2", "-Xlinker", f"-rpath,{lib}", "-lpthread"]
+           *[f"-D{d}" for d in defines], "-o", target + ".tmp", f"-L{lib}", "-l:libnccl.so.2", "-Xlinker", f"-rpath,{lib}", "-lpthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc build of libgcsm.so failed")
-    with open(os.path.join(HERE, "build_ptxas.log"), "w") as f:
-        f.write(r.stderr)
+    if out is None:
+        with open(os.path.join(HERE, "build_ptxas.log"), "w") as f:
+            f.write(r.stderr)
     if verbose:
         sys.stderr.write(r.stderr)
-    os.replace(LIB_PATH + ".tmp", LIB_PATH)
-    return LIB_PATH
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

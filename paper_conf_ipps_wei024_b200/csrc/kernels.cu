@@ -36,7 +36,16 @@ namespace {
 constexpr int kWarps = 8;
 constexpr int kBlock = 32 * kWarps;
 constexpr unsigned kFull = 0xffffffffu;
-constexpr uint32_t kSmemInts = 1536;  // per-warp shared staging slice (6 KB)
+#ifndef GCSM_SMEM_INTS
+#define GCSM_SMEM_INTS 1536
+#endif
+#ifndef GCSM_PRESTAGE_MERGE
+#define GCSM_PRESTAGE_MERGE 0
+#endif
+#ifndef GCSM_MERGE_INT4
+#define GCSM_MERGE_INT4 0
+#endif
+constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 constexpr int kChunk = 32;  // frontier entries per k_extend work grab
 
@@ -45,6 +54,7 @@ struct LRef {
   uint32_t ml;
   const int32_t *x;  // delta segment (ins or del), device memory
   uint32_t xl;
+  bool dev;          // main list is in device memory (HBM cache, a staged copy, or shared memory)
 };
 
 struct Acc {
@@ -79,10 +89,14 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
     }
   }
   const char *p = reinterpret_cast<const char *>(r.m);
-  if (p >= A.cache_lo && p < A.cache_hi) acc.hit += 4ull * r.ml;
+  r.dev = p >= A.cache_lo && p < A.cache_hi;
+  if (r.dev) acc.hit += 4ull * r.ml;
   else acc.miss += 4ull * r.ml;
   acc.delta += 4ull * r.xl;
-  if (v == pin.v) r.m = pin.p;  // served from this warp's staged copy
+  if (v == pin.v) {  // served from this warp's staged copy
+    r.m = pin.p;
+    r.dev = true;
+  }
   return r;
 }
 
@@ -180,7 +194,7 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
   for (int p = 0; p < nl; ++p) {
     const uint32_t n = L[p].ml;
     if (n < 32) continue;
-    const bool hit = is_hit(A, L[p].m) || is_device(A, L[p].m);
+    const bool hit = L[p].dev;
     const bool driver = !has_set && p == drv;
     bool stage;
     if (driver) {
@@ -191,15 +205,17 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
     }
     if (!stage) continue;
     const uint32_t n4 = (n + 3) & ~3u;
-    if (!hit && !is_device(A, L[p].m)) acc.copied += 4ull * n;
+    if (!hit) acc.copied += 4ull * n;
     if (sm_used + n4 <= kSmemInts) {
       warp_copy(sm + sm_used, L[p].m, n, lane);
       L[p].m = sm + sm_used;
+      L[p].dev = true;
       sm_used += n4;
       any = true;
     } else if (!hit && g_used + n4 <= 2u * (uint32_t)A.dcap) {
       warp_copy(gbuf + g_used, L[p].m, n, lane);
       L[p].m = gbuf + g_used;
+      L[p].dev = true;
       g_used += n4;
       any = true;
     }
@@ -212,6 +228,12 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
 // co-rank binary search and merges its range sequentially, counting a[i] == b[j] when it consumes a[i] (ties
 // take A first, so an equal pair is counted exactly once even across lane boundaries). O((na+nb)/32 + log)
 // instructions per lane instead of ceil(d/32) * log2(L) dependent probes.
+__device__ __forceinline__ int32_t pick4(const int4 &w, uint32_t k) {
+  return k == 0 ? w.x : (k == 1 ? w.y : (k == 2 ? w.z : w.w));
+}
+
+// Both runs are 16-byte aligned and allocated in 16-byte granules, so each lane reads its segment as int4
+// windows (one load per 4 elements, L1-friendly).
 __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, const int32_t *b, uint32_t nb,
                                                 int label, const uint16_t *lab, int lane) {
   const uint32_t T = na + nb;
@@ -224,17 +246,45 @@ __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, c
     else hi = i;
   }
   uint32_t i = lo, j = d0 - lo, cnt = 0;
-  int32_t ai = i < na ? a[i] : INT_MAX, bj = j < nb ? b[j] : INT_MAX;
+#if !GCSM_MERGE_INT4
+  // branch-free steps; an equal pair advances both runs (still counted once: the co-rank split puts a[i]
+  // before an equal b[j], so the lane owning a[i] counts it and the next lane starts past it)
+  while (i + j < d1) {
+    const int32_t ai = i < na ? a[i] : INT_MAX;
+    const int32_t bj = j < nb ? b[j] : INT_MAX;
+    const bool le = ai <= bj, ge = ai >= bj;
+    if (le && ge && (label < 0 || lab[ai] == (uint16_t)label)) ++cnt;
+    i += le;
+    j += ge;
+  }
+#else
+  const int4 *a4 = reinterpret_cast<const int4 *>(a);
+  const int4 *b4 = reinterpret_cast<const int4 *>(b);
+  int4 wa = make_int4(0, 0, 0, 0), wb = make_int4(0, 0, 0, 0);
+  if (i < na) wa = a4[i >> 2];
+  if (j < nb) wb = b4[j >> 2];
+  int32_t ai = i < na ? pick4(wa, i & 3) : INT_MAX, bj = j < nb ? pick4(wb, j & 3) : INT_MAX;
   for (uint32_t st = d0; st < d1; ++st) {
     if (ai <= bj) {
       if (ai == bj && (label < 0 || lab[ai] == (uint16_t)label)) ++cnt;
       ++i;
-      ai = i < na ? a[i] : INT_MAX;
+      if (i < na) {
+        if ((i & 3) == 0) wa = a4[i >> 2];
+        ai = pick4(wa, i & 3);
+      } else {
+        ai = INT_MAX;
+      }
     } else {
       ++j;
-      bj = j < nb ? b[j] : INT_MAX;
+      if (j < nb) {
+        if ((j & 3) == 0) wb = b4[j >> 2];
+        bj = pick4(wb, j & 3);
+      } else {
+        bj = INT_MAX;
+      }
     }
   }
+#endif
 #pragma unroll
   for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
   return cnt;
@@ -265,7 +315,7 @@ __device__ __forceinline__ uint32_t ilog2(uint32_t x) { return 31u - __clz(x | 1
 __device__ __forceinline__ bool count2(const MatchArgs &A, const LRef *L, int drv, const int32_t *excl, int nexcl,
                                        int label, int lane, uint32_t *out) {
   const LRef &X = L[drv], &Y = L[1 - drv];
-  if (X.ml < 8 || Y.ml < 8 || is_host(A, X.m) || is_host(A, Y.m)) return false;
+  if (X.ml < 8 || Y.ml < 8 || !X.dev || !Y.dev) return false;
   const uint32_t d = X.ml + X.xl, big = Y.ml + Y.xl;
   const uint32_t bs_cost = ((d + 31) >> 5) * (7 * ilog2(big) + 12);
   const uint32_t mg_cost = 10 * ilog2(min(X.ml, Y.ml)) + 7 * ((X.ml + Y.ml + 31) >> 5) + 30;
@@ -489,9 +539,16 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
         for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
         const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
-        stage_lists(A, L, nl, drv, dset != nullptr, dn, sm, gstage, lane, acc);
-        if (p == k - 1) {
-          uint32_t c;
+        uint32_t c = 0;
+        // last level, two lists already in device memory: merge without staging
+        const bool merged = GCSM_PRESTAGE_MERGE && !LIST && p == k - 1 && !dset && nl == 2 &&
+                            count2(A, L, drv, excl, nex, Lp.label, lane, &c);
+        if (!merged) stage_lists(A, L, nl, drv, dset != nullptr, dn, sm, gstage, lane, acc);
+        if (merged) {
+          if (P.kind) acc.rem += c;
+          else acc.add += c;
+          descend = false;
+        } else if (p == k - 1) {
           if (LIST) {
             c = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, lastbuf, lane);
             __syncwarp();
