@@ -49,6 +49,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=20.0)
     ap.add_argument("--quick", action="store_true", help="profiling mode: no clocks sampler / cpu baseline")
+    ap.add_argument("--serial", action="store_true",
+                    help="apply the batch to the query contexts one after the other (default: one host thread per "
+                         "query context, so one query's host steps overlap another's kernels)")
     return ap.parse_args()
 
 
@@ -254,11 +257,24 @@ def main():
     batches = [(np.ascontiguousarray(a, dtype=np.int32), np.ascontiguousarray(b, dtype=np.int32))
                for a, b in w.batches[:steps]]
 
+    def run_one(q, g, i, out, slot):
+        a, r = g.apply_batch(*batches[i])
+        out[slot] = (q, a, r, g.stats())
+
     def do_step(i):
-        recs = []
-        for q, g in ctxs:
-            a, r = g.apply_batch(*batches[i])
-            recs.append((q, a, r, g.stats()))
+        recs = [None] * len(ctxs)
+        # world > 1: serial, so every rank issues its contexts' NCCL allreduces in the same order
+        if args.serial or len(ctxs) == 1 or world > 1:
+            for slot, (q, g) in enumerate(ctxs):
+                run_one(q, g, i, recs, slot)
+        else:  # independent standing queries: one host thread each (ctypes releases the GIL)
+            ths = [threading.Thread(target=run_one, args=(q, g, i, recs, slot)) for slot, (q, g) in enumerate(ctxs)]
+            for t in ths:
+                t.start()
+            for t in ths:
+                t.join()
+        if any(r is None for r in recs):
+            raise RuntimeError("a query context failed")
         return recs
 
     for i in range(args.warmup):
@@ -351,7 +367,9 @@ def main():
                                f"{'+'.join(queries)}, {args.batch} mixed updates per GPU per step, cache budget "
                                f"{frac:.0%} of adjacency", "queries": queries, "global_batch": args.batch * world,
                    "graph_vertices": w.n, "graph_edges": int(w.row_ptr[-1] // 2), "budget_bytes": budget,
-                   "cache_policy": args.cache_policy, "parallelism": f"units LPT-sharded over {world} GPU(s)",
+                   "cache_policy": args.cache_policy,
+                   "parallelism": f"units LPT-sharded over {world} GPU(s); "
+                                  f"{'serial' if (args.serial or world > 1) else 'concurrent'} query contexts",
                    "l2": "inputs larger than L2 (560 MB pinned host graph; cache repacked every batch)"},
         "roofline": roofline,
         "cpu_baseline": cpu,

@@ -1,0 +1,96 @@
+"""N > 1 host plumbing on CPU with torch.distributed gloo, world_size 2 (no GPU needed).
+
+Covers what every rank of a multi-GPU run does before the count allreduce:
+* the ncclUniqueId created by rank 0 reaches every rank through torch.distributed (distributed_nccl_id);
+* every rank derives the same unit sharding from the same batch (gcsm_shard, LPT) and the shards are a disjoint
+  cover of the level-1 units;
+* the per-rank counts of the units a rank owns sum to the whole batch's counts (oracle IVM per unit shard),
+  i.e. a sum-allreduce of the rank counters is exact.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+import torch.distributed as dist  # noqa: E402
+import torch.multiprocessing as mp  # noqa: E402
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _worker(rank, world, port, out_q):
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import gcsm_inputs as gi
+        import oracle
+        import paper_conf_ipps_wei024_b200 as G
+        nid = G.distributed_nccl_id()
+        ids = [None] * world
+        dist.all_gather_object(ids, nid)
+        # the same batch on every rank -> the same units and costs -> the same shard map
+        w = gi.make_workload("C2", scale=10, n_edges=6000, batch=128, n_batches=1)
+        ins, dele = w.batches[0]
+        k, qe, ql = gi.query("diamond")
+        I, D, _ = oracle.normalize_batch(w.n, w.row_ptr, w.col, ins, dele)
+        U = oracle.units(k, qe, ql, None, I, D)
+        deg = np.diff(w.row_ptr)
+        cost = (1 + deg[U[:, 2]] + deg[U[:, 3]]).astype(np.uint64)
+        ranks = G.shard(cost, world)
+        maps = [None] * world
+        dist.all_gather_object(maps, ranks.tolist())
+        mine = set(np.nonzero(ranks == rank)[0].tolist())
+        # this rank's counts: the oracle's IVM loops over its own units only
+        keep = np.zeros(len(U), bool)
+        keep[sorted(mine)] = True
+        U_all = U
+
+        def unit_filter(Ux):
+            assert np.array_equal(Ux, U_all)
+            return keep
+
+        r = oracle._ivm(0, w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele, unit_filter=unit_filter)
+        t = torch.tensor([r["added"], r["removed"]], dtype=torch.int64)
+        dist.all_reduce(t)  # the count allreduce (gloo here, NCCL on the GPUs)
+        full = oracle.delta(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele)
+        out_q.put((rank, nid, ids, maps, sorted(mine), tuple(t.tolist()), full, len(U)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_shard_and_allreduce():
+    import __graft_entry__
+    __graft_entry__.build()
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    res.sort()
+    nid0 = res[0][1]
+    assert len(nid0) == 128
+    for rank, nid, ids, maps, mine, tot, full, n_units in res:
+        assert all(x == nid0 for x in ids)            # rank 0's id reached everyone
+        assert maps[0] == maps[1]                      # identical shard maps on every rank
+        assert tot == full                             # allreduce of shard counts == whole-batch counts
+    a, b = set(res[0][4]), set(res[1][4])
+    assert not (a & b) and len(a | b) == res[0][7]     # disjoint cover of the units
+    assert a and b                                     # both ranks got work
