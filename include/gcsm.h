@@ -166,6 +166,18 @@ gcsm_status gcsm_apply_batch_list(gcsm_ctx *ctx, int64_t n_ins, const int32_t *i
                                   int32_t *added_tuples, uint64_t added_cap, int32_t *removed_tuples,
                                   uint64_t removed_cap, uint64_t *added, uint64_t *removed);
 
+/* Pipelined form of gcsm_apply_batch (overlap batch t+1's host steps (1)-(3) with batch
+ * t's kernels). gcsm_submit_batch validates and normalises the batch (EINVAL without mutation as above), runs
+ * its host steps, enqueues its GPU work and its count allreduce on the library's stream, and merges it into
+ * the host store (G_{t+1} is the store's state on return) without waiting for the kernels: the merge writes
+ * fresh arrays, and the arrays an in-flight batch may read are recycled only after it completes (P:302's
+ * consistency). At most two batches may be outstanding (ESTATE otherwise). gcsm_wait_batch waits for the
+ * oldest outstanding batch and returns its counts (ESTATE if none); gcsm_get_stats then describes it.
+ * gcsm_apply_batch(_list) = submit + wait (draining older submissions first). set_query and set_cache_budget
+ * return ESTATE while a batch is outstanding. With world > 1 both calls are collective. */
+gcsm_status gcsm_submit_batch(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del);
+gcsm_status gcsm_wait_batch(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed);
+
 /* Last batch's statistics. */
 gcsm_status gcsm_get_stats(const gcsm_ctx *ctx, gcsm_stats *out);
 

@@ -105,6 +105,17 @@ class Gcsm:
                                                ctypes.byref(r)), "apply_batch")
         return a.value, r.value
 
+    def submit_batch(self, ins, dele):
+        """Pipelined: host steps + enqueue + merge; the counts come from wait_batch (at most 2 outstanding)."""
+        ins = _i32(ins).reshape(-1, 2)
+        dele = _i32(dele).reshape(-1, 2)
+        self._check(self._lib.gcsm_submit_batch(self._h, len(ins), _ptr(ins), len(dele), _ptr(dele)), "submit_batch")
+
+    def wait_batch(self):
+        a, r = ctypes.c_uint64(), ctypes.c_uint64()
+        self._check(self._lib.gcsm_wait_batch(self._h, ctypes.byref(a), ctypes.byref(r)), "wait_batch")
+        return a.value, r.value
+
     def apply_batch_list(self, ins, dele, added_cap=1 << 16, removed_cap=1 << 16):
         """Returns (added, removed, added_tuples[k], removed_tuples[k]); raises GcsmError(ETRUNC) if truncated."""
         ins = _i32(ins).reshape(-1, 2)

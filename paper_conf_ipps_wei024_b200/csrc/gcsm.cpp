@@ -64,8 +64,31 @@ struct gcsm_ctx {
   bool has_query = false;
   uint64_t budget = 0;
   cudaStream_t stream = nullptr;
-  cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr, ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr, ev_c1 = nullptr;
-  std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
+  // Per in-flight batch state (double buffered: batch t's async copies read its pinned staging while batch
+  // t+1's host steps fill the other slot; pipelined submit/wait).
+  struct Slot {
+    int64_t *h_pidx = nullptr; size_t h_pidx_cap = 0;
+    VDesc *h_pval = nullptr; size_t h_pval_cap = 0;
+    DRec *h_drec = nullptr; size_t h_drec_cap = 0;
+    int32_t *h_dlist = nullptr; size_t h_dlist_cap = 0;
+    Unit *h_units = nullptr; size_t h_units_cap = 0;
+    uint64_t *h_gather = nullptr; size_t h_gather_cap = 0;
+    uint64_t *h_fresh = nullptr; size_t h_fresh_cap = 0;
+    unsigned long long *h_cnt = nullptr;
+    cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr, ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr,
+                ev_c1 = nullptr, ev_done = nullptr;
+    std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
+    size_t nev = 0;
+    bool inflight = false;
+    gcsm_stats st{};
+    double host_ms = 0;
+    // list mode
+    int32_t *tup_add = nullptr, *tup_rem = nullptr, *d_tadd = nullptr, *d_trem = nullptr;
+    uint64_t add_cap = 0, rem_cap = 0;
+    std::vector<std::pair<int32_t *, uint32_t>> retired;  // host arrays replaced by this batch's merge
+  };
+  Slot slots[2];
+  uint64_t waited = 0;  // batches whose results have been collected
   ncclComm_t comm = nullptr;
   int grid = 0, warps_total = 0;
 
@@ -89,24 +112,14 @@ struct gcsm_ctx {
   bool cache_valid = false;                        // prev_slot describes d_cachebuf[cache_cur]
   std::vector<std::pair<int32_t, uint64_t>> prev_slot;  // (vertex, offset) of the previous cache, by vertex
   uint64_t *d_gather = nullptr; size_t gather_cap = 0;  // retained lists: (src, dst, n16) triples
-  uint64_t *h_gather = nullptr; size_t h_gather_cap = 0;
   uint64_t *d_fresh = nullptr; size_t fresh_cap = 0;    // newly cached lists: (host src, dst, n16) triples
-  uint64_t *h_fresh = nullptr; size_t h_fresh_cap = 0;
   std::vector<int32_t> sel_index;                       // vertex -> index in this batch's selection, or -1
   int64_t *d_pidx = nullptr; size_t pidx_cap = 0;
   VDesc *d_pval = nullptr; size_t pval_cap = 0;
   int32_t *d_tup = nullptr; size_t tup_cap = 0;
 
-  // pinned host staging
-  int64_t *h_pidx = nullptr; size_t h_pidx_cap = 0;
-  VDesc *h_pval = nullptr; size_t h_pval_cap = 0;
-  DRec *h_drec = nullptr; size_t h_drec_cap = 0;
-  int32_t *h_dlist = nullptr; size_t h_dlist_cap = 0;
-  Unit *h_units = nullptr; size_t h_units_cap = 0;
-  unsigned long long *h_cnt = nullptr;
 
   // cache / batch state
-  std::vector<VDesc> vd;             // host mirror of d_vdesc
   std::vector<int32_t> cached;       // ascending
   std::vector<int32_t> prev_cached, prev_U;
   std::vector<uint8_t> mark;         // scratch (n)
@@ -116,9 +129,10 @@ struct gcsm_ctx {
   uint64_t batch_seq = 0;
   std::vector<int32_t> degree_order;  // GCSM_CACHE_DEGREE ranking
 
+  bool in_batch = false;  // between a successful normalise and the end of submit: failures poison the ctx
   gcsm_status fail(gcsm_status s, const std::string &m) {
     err = m;
-    if (s == GCSM_EDEVICE || s == GCSM_ENCCL) poisoned = true;
+    if (s == GCSM_EDEVICE || s == GCSM_ENCCL || (in_batch && s != GCSM_EINVAL)) poisoned = true;
     return s;
   }
   gcsm_status cuda_fail(cudaError_t e, const char *where) {
@@ -140,12 +154,14 @@ gcsm_ctx::~gcsm_ctx() {
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh};
   for (void *p : dev)
     if (p) cudaFree(p);
-  void *host[] = {h_pidx, h_pval, h_drec, h_dlist, h_units, h_cnt, h_gather, h_fresh};
-  for (void *p : host)
-    if (p) cudaFreeHost(p);
-  for (cudaEvent_t e : {ev_m0, ev_m1, ev_a0, ev_a1, ev_c0, ev_c1})
-    if (e) cudaEventDestroy(e);
-  for (cudaEvent_t e : kev) cudaEventDestroy(e);
+  for (Slot &sl : slots) {
+    void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt};
+    for (void *p : host)
+      if (p) cudaFreeHost(p);
+    for (cudaEvent_t e : {sl.ev_m0, sl.ev_m1, sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done})
+      if (e) cudaEventDestroy(e);
+    for (cudaEvent_t e : sl.kev) cudaEventDestroy(e);
+  }
   if (stream) cudaStreamDestroy(stream);
 }
 
@@ -208,21 +224,24 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
     return s;
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
-  for (cudaEvent_t *ev : {&ctx->ev_m0, &ctx->ev_m1, &ctx->ev_a0, &ctx->ev_a1, &ctx->ev_c0, &ctx->ev_c1})
-    if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
+  for (auto &sl : ctx->slots) {
+    for (cudaEvent_t *ev : {&sl.ev_m0, &sl.ev_m1, &sl.ev_a0, &sl.ev_a1, &sl.ev_c0, &sl.ev_c1, &sl.ev_done})
+      if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
+    if (cudaHostAlloc(&sl.h_cnt, sizeof(unsigned long long) * CNT_N, cudaHostAllocDefault) != cudaSuccess)
+      return bail(GCSM_ENOMEM);
+  }
   if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_plans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)n + 2047) / 2048 + 1)) != cudaSuccess)
     return bail(GCSM_ENOMEM);
-  if (cudaHostAlloc(&ctx->h_cnt, sizeof(unsigned long long) * CNT_N, cudaHostAllocDefault) != cudaSuccess)
-    return bail(GCSM_ENOMEM);
-  ctx->vd.resize(n);
-  for (int32_t v = 0; v < n; ++v)
-    ctx->vd[v] = VDesc{ctx->store.dev_ptr(ctx->store.lst[v]), ctx->store.len[v], 0};
-  if (cudaMemcpy(ctx->d_vdesc, ctx->vd.data(), sizeof(VDesc) * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
-    return bail(GCSM_EDEVICE);
+  {
+    std::vector<VDesc> vd(n);
+    for (int32_t v = 0; v < n; ++v) vd[v] = VDesc{ctx->store.dev_ptr(ctx->store.lst[v]), ctx->store.len[v], 0};
+    if (cudaMemcpy(ctx->d_vdesc, vd.data(), sizeof(VDesc) * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
+      return bail(GCSM_EDEVICE);
+  }
   if (labels) {
     if (cudaMalloc(&ctx->d_lab, 2 * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
     if (cudaMemcpy(ctx->d_lab, ctx->store.lab.data(), 2 * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
@@ -253,6 +272,7 @@ gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *q
                            const int32_t *order) {
   if (!ctx) return GCSM_EINVAL;
   if (ctx->poisoned) return GCSM_ESTATE;
+  if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "set_query with a batch in flight");
   QueryPlan qp;
   std::string e = build_plan(k, m, qedges, qlabels, order, qp);
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
@@ -271,6 +291,7 @@ gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *q
 gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
   if (!ctx) return GCSM_EINVAL;
   if (ctx->poisoned) return GCSM_ESTATE;
+  if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "set_cache_budget with a batch in flight");
   bytes &= ~uint64_t(15);
   if (bytes > ctx->cache_cap) {
     for (char *&b : ctx->d_cachebuf) {
@@ -313,12 +334,16 @@ struct Trace {
   }
 };
 
-static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
-                              int32_t *tup_add, uint64_t add_cap, int32_t *tup_rem, uint64_t rem_cap,
-                              uint64_t *added, uint64_t *removed) {
+// Host steps (1)-(3) of one batch, its GPU work (3)-(4b) enqueued on the stream, and its host merge (5) into
+// fresh arrays; returns without waiting for the kernels (gcsm_wait_batch collects the counts).
+static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                               int32_t *tup_add, uint64_t add_cap, int32_t *tup_rem, uint64_t rem_cap) {
   if (!ctx) return GCSM_EINVAL;
   if (ctx->poisoned) return GCSM_ESTATE;
   if (!ctx->has_query) return ctx->fail(GCSM_ESTATE, "apply_batch before set_query");
+  if (ctx->batch_seq - ctx->waited >= 2)
+    return ctx->fail(GCSM_ESTATE, "two batches already in flight: gcsm_wait_batch first");
+  auto &sl = ctx->slots[ctx->batch_seq & 1];
   const bool listing = tup_add || tup_rem;
   if (listing && ctx->opt.world > 1 && !(ctx->opt.flags & GCSM_FLAG_LOCAL_COUNTS))
     return ctx->fail(GCSM_EINVAL, "list mode is single-GPU");
@@ -335,9 +360,11 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   Timer t1;
   std::string e = S.normalize(n_ins, ins, n_del, del);
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
+  ctx->in_batch = true;
   tr.mark("normalize");
   bool cuda_err = false;
-  if (!S.build_overlay(&cuda_err)) return ctx->fail(GCSM_EDEVICE, "pinned overlay allocation failed");
+  if (!S.build_overlay((int)(ctx->batch_seq & 1), &cuda_err))
+    return ctx->fail(GCSM_EDEVICE, "pinned overlay allocation failed");
   tr.mark("overlay");
   st.n_ins = S.I.size();
   st.n_del = S.D.size();
@@ -550,8 +577,8 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   }
   if (ctx->sel_index.size() != (size_t)S.n) ctx->sel_index.assign(S.n, -1);
   for (size_t i = 0; i < sel.size(); ++i) ctx->sel_index[sel[i]] = (int32_t)i;
-  if (!host_ensure(ctx->h_pidx, ctx->h_pidx_cap, dirty.size()) ||
-      !host_ensure(ctx->h_pval, ctx->h_pval_cap, dirty.size()))
+  if (!host_ensure(sl.h_pidx, sl.h_pidx_cap, dirty.size()) ||
+      !host_ensure(sl.h_pval, sl.h_pval_cap, dirty.size()))
     return ctx->fail(GCSM_ENOMEM, "pinned staging");
   parallel_for(T, (int64_t)dirty.size(), [&](int, int64_t lo, int64_t hi) {
     for (int64_t i = lo; i < hi; ++i) {
@@ -562,8 +589,8 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
       d.len = ui >= 0 ? S.s_len[ui] : S.len[v];
       const int32_t si = ctx->sel_index[v];
       d.ptr = si >= 0 ? (const int32_t *)(ctx->d_cache + sel_off[si]) : S.dev_ptr(ui >= 0 ? S.s_ptr[ui] : S.lst[v]);
-      ctx->h_pidx[i] = v;
-      ctx->h_pval[i] = d;
+      sl.h_pidx[i] = v;
+      sl.h_pval[i] = d;
     }
   });
   for (int32_t v : sel) ctx->sel_index[v] = -1;
@@ -571,15 +598,15 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   // delta lists of U
   const size_t nU = S.U.size();
   const size_t nd = S.ins_val.size() + S.del_val.size();
-  if (!host_ensure(ctx->h_drec, ctx->h_drec_cap, nU) || !host_ensure(ctx->h_dlist, ctx->h_dlist_cap, nd) ||
-      !host_ensure(ctx->h_units, ctx->h_units_cap, (size_t)nu))
+  if (!host_ensure(sl.h_drec, sl.h_drec_cap, nU) || !host_ensure(sl.h_dlist, sl.h_dlist_cap, nd) ||
+      !host_ensure(sl.h_units, sl.h_units_cap, (size_t)nu))
     return ctx->fail(GCSM_ENOMEM, "pinned staging");
   for (size_t i = 0; i < nU; ++i)
-    ctx->h_drec[i] = DRec{S.ins_off[i], S.ins_off[i + 1] - S.ins_off[i], (uint32_t)S.ins_val.size() + S.del_off[i],
+    sl.h_drec[i] = DRec{S.ins_off[i], S.ins_off[i + 1] - S.ins_off[i], (uint32_t)S.ins_val.size() + S.del_off[i],
                           S.del_off[i + 1] - S.del_off[i]};
-  std::memcpy(ctx->h_dlist, S.ins_val.data(), S.ins_val.size() * 4);
-  std::memcpy(ctx->h_dlist + S.ins_val.size(), S.del_val.data(), S.del_val.size() * 4);
-  std::memcpy(ctx->h_units, units.data(), sizeof(Unit) * (size_t)nu);
+  std::memcpy(sl.h_dlist, S.ins_val.data(), S.ins_val.size() * 4);
+  std::memcpy(sl.h_dlist + S.ins_val.size(), S.del_val.data(), S.del_val.size() * 4);
+  std::memcpy(sl.h_units, units.data(), sizeof(Unit) * (size_t)nu);
   st.ms_pack = t3.ms();
   tr.mark("staging");
 
@@ -588,33 +615,33 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
       !dev_ensure(ctx->d_drec, ctx->drec_cap, nU) || !dev_ensure(ctx->d_dlist, ctx->dlist_cap, nd) ||
       !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)nu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)nu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
-  CK(cudaEventRecord(ctx->ev_c0, s));
+  CK(cudaEventRecord(sl.ev_c0, s));
   const uint64_t retained_bytes = used - new_bytes;
   if (!gather.empty()) {  // HBM -> HBM copy of the retained lists from the previous buffer
-    if (!host_ensure(ctx->h_gather, ctx->h_gather_cap, gather.size()) ||
+    if (!host_ensure(sl.h_gather, sl.h_gather_cap, gather.size()) ||
         !dev_ensure(ctx->d_gather, ctx->gather_cap, gather.size()))
       return ctx->fail(GCSM_ENOMEM, "gather staging");
-    std::memcpy(ctx->h_gather, gather.data(), 8 * gather.size());
-    CK(cudaMemcpyAsync(ctx->d_gather, ctx->h_gather, 8 * gather.size(), cudaMemcpyHostToDevice, s));
+    std::memcpy(sl.h_gather, gather.data(), 8 * gather.size());
+    CK(cudaMemcpyAsync(ctx->d_gather, sl.h_gather, 8 * gather.size(), cudaMemcpyHostToDevice, s));
     CK(launch_gather_lists(ctx->d_cache, ctx->d_cachebuf[ctx->cache_cur], ctx->d_gather, (int64_t)gather.size() / 3, s));
   }
   if (!fresh.empty()) {  // newly selected lists: GPU gather over PCIe from the mapped host store
-    if (!host_ensure(ctx->h_fresh, ctx->h_fresh_cap, fresh.size()) ||
+    if (!host_ensure(sl.h_fresh, sl.h_fresh_cap, fresh.size()) ||
         !dev_ensure(ctx->d_fresh, ctx->fresh_cap, fresh.size()))
       return ctx->fail(GCSM_ENOMEM, "gather staging");
-    std::memcpy(ctx->h_fresh, fresh.data(), 8 * fresh.size());
-    CK(cudaMemcpyAsync(ctx->d_fresh, ctx->h_fresh, 8 * fresh.size(), cudaMemcpyHostToDevice, s));
+    std::memcpy(sl.h_fresh, fresh.data(), 8 * fresh.size());
+    CK(cudaMemcpyAsync(ctx->d_fresh, sl.h_fresh, 8 * fresh.size(), cudaMemcpyHostToDevice, s));
     CK(launch_gather_lists(ctx->d_cache, nullptr, ctx->d_fresh, (int64_t)fresh.size() / 3, s));
   }
   (void)retained_bytes;
-  CK(cudaMemcpyAsync(ctx->d_pidx, ctx->h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
-  CK(cudaMemcpyAsync(ctx->d_pval, ctx->h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(launch_patch_vdesc(ctx->d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
   uint64_t launches = dirty.empty() ? 0 : 1;
-  if (nU) CK(cudaMemcpyAsync(ctx->d_drec, ctx->h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
-  if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, ctx->h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
-  if (nu) CK(cudaMemcpyAsync(ctx->d_units, ctx->h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
-  CK(cudaEventRecord(ctx->ev_c1, s));
+  if (nU) CK(cudaMemcpyAsync(ctx->d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
+  if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
+  if (nu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
+  CK(cudaEventRecord(sl.ev_c1, s));
   st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
                  4 * nd + sizeof(Unit) * (size_t)nu;
 
@@ -682,23 +709,23 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   A.tup_rem_cap = rem_cap;
   A.k = k;
   A.listing = listing ? 1 : 0;
-  CK(cudaEventRecord(ctx->ev_m0, s));
+  CK(cudaEventRecord(sl.ev_m0, s));
   size_t nev = 0;
   for (const auto &ch : chunks) {
     if (ch.second <= ch.first) continue;
     A.units = ctx->d_units + ch.first;
     A.n_units = ch.second - ch.first;
-    while (ctx->kev.size() < nev + 3) {
+    while (sl.kev.size() < nev + 3) {
       cudaEvent_t ev;
       CK(cudaEventCreate(&ev));
-      ctx->kev.push_back(ev);
+      sl.kev.push_back(ev);
     }
     // reset the work cursors and the frontier size of this chunk
     CK(cudaMemsetAsync(ctx->d_cnt + CNT_F2, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(ctx->d_cnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), s));
-    CK(cudaEventRecord(ctx->kev[nev], s));
+    CK(cudaEventRecord(sl.kev[nev], s));
     CK(launch_level2(A, ctx->grid, s));
-    CK(cudaEventRecord(ctx->kev[nev + 1], s));
+    CK(cudaEventRecord(sl.kev[nev + 1], s));
     ++launches;
     if (k >= 4) {
       CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_group, s));
@@ -707,63 +734,34 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
       CK(launch_extend(A, ctx->grid, s));
       ++launches;
     }
-    CK(cudaEventRecord(ctx->kev[nev + 2], s));
+    CK(cudaEventRecord(sl.kev[nev + 2], s));
     nev += 3;
   }
-  CK(cudaEventRecord(ctx->ev_m1, s));
+  CK(cudaEventRecord(sl.ev_m1, s));
   // ---- (4b) count allreduce over NVLink (world > 1) -------------------------------------
-  CK(cudaEventRecord(ctx->ev_a0, s));
+  CK(cudaEventRecord(sl.ev_a0, s));
   if (ctx->comm) {
     if (ncclAllReduce(ctx->d_cnt, ctx->d_cnt, 2, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
       return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
   }
-  CK(cudaEventRecord(ctx->ev_a1, s));
-  CK(cudaMemcpyAsync(ctx->h_cnt, ctx->d_cnt, sizeof(unsigned long long) * CNT_N, cudaMemcpyDeviceToHost, s));
-  CK(cudaStreamSynchronize(s));
-  if (ctx->h_cnt[CNT_OVERFLOW]) return ctx->fail(GCSM_EDEVICE, "internal: level-2 frontier overflow");
-  float ms_m = 0, ms_a = 0;
-  cudaEventElapsedTime(&ms_m, ctx->ev_m0, ctx->ev_m1);
-  cudaEventElapsedTime(&ms_a, ctx->ev_a0, ctx->ev_a1);
-  st.ms_match = ms_m;
-  st.ms_allreduce = ms_a;
-  {
-    float ms_c = 0;
-    cudaEventElapsedTime(&ms_c, ctx->ev_c0, ctx->ev_c1);
-    st.ms_copy = ms_c;
-    for (size_t i = 0; i < nev; i += 3) {
-      float a = 0, b = 0;
-      cudaEventElapsedTime(&a, ctx->kev[i], ctx->kev[i + 1]);
-      cudaEventElapsedTime(&b, ctx->kev[i + 1], ctx->kev[i + 2]);
-      st.ms_level2 += a;
-      st.ms_extend += b;
-    }
-  }
-  st.added = ctx->h_cnt[CNT_ADDED];
-  st.removed = ctx->h_cnt[CNT_REMOVED];
-  st.hit_bytes_ext = ctx->h_cnt[CNT_ACC_EXT + 0];
-  st.miss_bytes_ext = ctx->h_cnt[CNT_ACC_EXT + 1];
-  st.delta_bytes_ext = ctx->h_cnt[CNT_ACC_EXT + 2];
-  st.hit_bytes = ctx->h_cnt[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
-  st.miss_bytes = ctx->h_cnt[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
-  st.delta_bytes = ctx->h_cnt[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
-  st.host_copied_bytes = ctx->h_cnt[CNT_COPIED];
-  st.d2h_bytes = sizeof(unsigned long long) * CNT_N;
-  st.frontier = ctx->h_cnt[CNT_F2];
-  st.kernel_launches = launches;
-  bool trunc = false;
-  if (listing) {
-    const uint64_t na = std::min<uint64_t>(ctx->h_cnt[CNT_TUP_ADD], add_cap);
-    const uint64_t nr = std::min<uint64_t>(ctx->h_cnt[CNT_TUP_REM], rem_cap);
-    if (na) CK(cudaMemcpy(tup_add, d_tadd, sizeof(int32_t) * k * na, cudaMemcpyDeviceToHost));
-    if (nr) CK(cudaMemcpy(tup_rem, d_trem, sizeof(int32_t) * k * nr, cudaMemcpyDeviceToHost));
-    st.d2h_bytes += sizeof(int32_t) * k * (na + nr);
-    trunc = ctx->h_cnt[CNT_TUP_ADD] > add_cap || ctx->h_cnt[CNT_TUP_REM] > rem_cap;
-  }
+  CK(cudaEventRecord(sl.ev_a1, s));
+  CK(cudaMemcpyAsync(sl.h_cnt, ctx->d_cnt, sizeof(unsigned long long) * CNT_N, cudaMemcpyDeviceToHost, s));
+  CK(cudaEventRecord(sl.ev_done, s));
+  sl.nev = nev;
+  sl.st = st;
+  sl.st.kernel_launches = launches;
+  sl.tup_add = tup_add;
+  sl.tup_rem = tup_rem;
+  sl.d_tadd = d_tadd;
+  sl.d_trem = d_trem;
+  sl.add_cap = add_cap;
+  sl.rem_cap = rem_cap;
+  tr.mark("enqueue");
 
-  // ---- (5) reorganise the host lists (after matching) -----------------------------
-  tr.mark("gpu");
+  // ---- (5) reorganise the host lists. P:302 runs it after matching so the kernel reads consistent data: here
+  // the merge writes fresh arrays and the ones the in-flight kernels may read are retired, not overwritten.
   Timer t5;
-  S.merge();
+  S.merge(sl.retired);
   tr.mark("merge");
   ctx->prev_cached = sel;
   std::sort(ctx->prev_cached.begin(), ctx->prev_cached.end());
@@ -777,15 +775,85 @@ static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, 
   ctx->cached = ctx->prev_cached;
   ctx->prev_U = S.U;
   S.clear_batch();
-  st.ms_merge = t5.ms();
+  sl.st.ms_merge = t5.ms();
   ++ctx->batch_seq;
-  st.ms_total = total.ms();
+  sl.inflight = true;
+  sl.host_ms = total.ms();
+  ctx->in_batch = false;
+  ctx->err.clear();
+  return GCSM_OK;
+}
+
+// Waits for the oldest in-flight batch and collects its counts and statistics.
+static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) {
+  if (!ctx) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  if (ctx->waited >= ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "no batch in flight");
+  Timer tw;
+  auto &sl = ctx->slots[ctx->waited & 1];
+  CK(cudaEventSynchronize(sl.ev_done));
+  gcsm_stats st = sl.st;
+  const int k = ctx->qp.k;
+  if (sl.h_cnt[CNT_OVERFLOW]) return ctx->fail(GCSM_EDEVICE, "internal: level-2 frontier overflow");
+  float ms_m = 0, ms_a = 0, ms_c = 0;
+  cudaEventElapsedTime(&ms_m, sl.ev_m0, sl.ev_m1);
+  cudaEventElapsedTime(&ms_a, sl.ev_a0, sl.ev_a1);
+  cudaEventElapsedTime(&ms_c, sl.ev_c0, sl.ev_c1);
+  st.ms_match = ms_m;
+  st.ms_allreduce = ms_a;
+  st.ms_copy = ms_c;
+  for (size_t i = 0; i < sl.nev; i += 3) {
+    float a = 0, b = 0;
+    cudaEventElapsedTime(&a, sl.kev[i], sl.kev[i + 1]);
+    cudaEventElapsedTime(&b, sl.kev[i + 1], sl.kev[i + 2]);
+    st.ms_level2 += a;
+    st.ms_extend += b;
+  }
+  const unsigned long long *h = sl.h_cnt;
+  st.added = h[CNT_ADDED];
+  st.removed = h[CNT_REMOVED];
+  st.hit_bytes_ext = h[CNT_ACC_EXT + 0];
+  st.miss_bytes_ext = h[CNT_ACC_EXT + 1];
+  st.delta_bytes_ext = h[CNT_ACC_EXT + 2];
+  st.hit_bytes = h[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
+  st.miss_bytes = h[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
+  st.delta_bytes = h[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
+  st.host_copied_bytes = h[CNT_COPIED];
+  st.d2h_bytes = sizeof(unsigned long long) * CNT_N;
+  st.frontier = h[CNT_F2];
+  bool trunc = false;
+  if (sl.tup_add || sl.tup_rem) {
+    const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);
+    const uint64_t nr = std::min<uint64_t>(h[CNT_TUP_REM], sl.rem_cap);
+    if (na) CK(cudaMemcpy(sl.tup_add, sl.d_tadd, sizeof(int32_t) * k * na, cudaMemcpyDeviceToHost));
+    if (nr) CK(cudaMemcpy(sl.tup_rem, sl.d_trem, sizeof(int32_t) * k * nr, cudaMemcpyDeviceToHost));
+    st.d2h_bytes += sizeof(int32_t) * k * (na + nr);
+    trunc = h[CNT_TUP_ADD] > sl.add_cap || h[CNT_TUP_REM] > sl.rem_cap;
+    sl.tup_add = sl.tup_rem = nullptr;
+  }
+  ctx->store.recycle(sl.retired);  // arrays the batch's kernels could read are free again
+  sl.inflight = false;
+  ++ctx->waited;
+  st.ms_total = sl.host_ms + tw.ms();
   ctx->stats = st;
   if (added) *added = st.added;
   if (removed) *removed = st.removed;
   if (trunc) return ctx->fail(GCSM_ETRUNC, "tuple buffer too small");
   ctx->err.clear();
   return GCSM_OK;
+}
+
+static gcsm_status apply_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
+                              int32_t *tup_add, uint64_t add_cap, int32_t *tup_rem, uint64_t rem_cap,
+                              uint64_t *added, uint64_t *removed) {
+  if (!ctx) return GCSM_EINVAL;
+  while (ctx->waited < ctx->batch_seq) {  // drain batches submitted asynchronously
+    gcsm_status w = wait_impl(ctx, nullptr, nullptr);
+    if (w != GCSM_OK && w != GCSM_ETRUNC) return w;
+  }
+  gcsm_status e = submit_impl(ctx, n_ins, ins, n_del, del, tup_add, add_cap, tup_rem, rem_cap);
+  if (e != GCSM_OK) return e;
+  return wait_impl(ctx, added, removed);
 }
 
 extern "C" {
@@ -801,6 +869,14 @@ gcsm_status gcsm_apply_batch_list(gcsm_ctx *ctx, int64_t n_ins, const int32_t *i
   if (!added_tuples || !removed_tuples) return GCSM_EINVAL;
   return apply_impl(ctx, n_ins, ins, n_del, del, added_tuples, added_cap, removed_tuples, removed_cap, added,
                     removed);
+}
+
+gcsm_status gcsm_submit_batch(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del) {
+  return submit_impl(ctx, n_ins, ins, n_del, del, nullptr, 0, nullptr, 0);
+}
+
+gcsm_status gcsm_wait_batch(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) {
+  return wait_impl(ctx, added, removed);
 }
 
 gcsm_status gcsm_get_stats(const gcsm_ctx *ctx, gcsm_stats *out) {

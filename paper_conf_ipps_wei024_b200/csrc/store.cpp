@@ -14,7 +14,8 @@ static inline uint32_t round4(uint64_t x) { return (uint32_t)((x + 3) & ~uint64_
 HostStore::~HostStore() {
   for (auto &c : chunks_)
     if (c.host) cudaFreeHost(c.host);
-  if (overlay_.host) cudaFreeHost(overlay_.host);
+  for (auto &o : overlay_)
+    if (o.host) cudaFreeHost(o.host);
 }
 
 bool HostStore::new_chunk(size_t bytes, Chunk &c) {
@@ -37,12 +38,18 @@ const int32_t *HostStore::dev_ptr(const int32_t *host) const {
   const char *p = (const char *)host;
   for (const auto &c : chunks_)
     if (p >= c.host && p < c.host + c.size) return (const int32_t *)(c.dev + (p - c.host));
-  if (overlay_.host && p >= overlay_.host && p < overlay_.host + overlay_.size)
-    return (const int32_t *)(overlay_.dev + (p - overlay_.host));
+  for (const auto &o : overlay_)
+    if (o.host && p >= o.host && p < o.host + o.size) return (const int32_t *)(o.dev + (p - o.host));
   return nullptr;
 }
 
 int32_t *HostStore::alloc_list(uint32_t capacity, bool *cuda_err) {
+  auto fit = free_.find(capacity);
+  if (fit != free_.end() && !fit->second.empty()) {
+    int32_t *p = fit->second.back();
+    fit->second.pop_back();
+    return p;
+  }
   const size_t bytes = (size_t)capacity * 4;
   if (chunks_.empty() || chunks_.back().used + bytes > chunks_.back().size) {
     Chunk c;
@@ -213,8 +220,9 @@ std::string HostStore::normalize(int64_t n_ins, const int32_t *ins, int64_t n_de
   return "";
 }
 
-bool HostStore::build_overlay(bool *cuda_err) {
+bool HostStore::build_overlay(int slot, bool *cuda_err) {
   *cuda_err = false;
+  Chunk &overlay_ = this->overlay_[slot & 1];
   const size_t nu = U.size();
   s_ptr.assign(nu, nullptr);
   s_len.assign(nu, 0);
@@ -277,7 +285,7 @@ uint32_t HostStore::view_len(int32_t v, int vw) const {
   return s_len[i];
 }
 
-void HostStore::merge() {
+void HostStore::merge(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
   const size_t nu = U.size();
   std::vector<int32_t *> target(nu, nullptr);
   std::vector<uint32_t> newlen(nu), newcap(nu);
@@ -286,33 +294,19 @@ void HostStore::merge() {
     const int32_t x = U[i];
     newlen[i] = s_len[i] + (ins_off[i + 1] - ins_off[i]);
     newcap[i] = cap[x];
-    target[i] = lst[x];
-    if (newlen[i] > cap[x]) {  // a new array with double capacity
-      newcap[i] = round4(std::max<uint64_t>(4, 2ull * newlen[i]));
-      target[i] = alloc_list(newcap[i], &err);
-    }
+    if (newlen[i] > cap[x]) newcap[i] = round4(std::max<uint64_t>(4, 2ull * newlen[i]));  // double
+    target[i] = newcap[i] ? alloc_list(newcap[i], &err) : nullptr;
   }
   parallel_for(threads, (int64_t)nu, [&](int, int64_t lo, int64_t hi) {
     for (int64_t i = lo; i < hi; ++i) {
-      const int32_t x = U[i];
       const int32_t *in = ins_val.data() + ins_off[i];
       const uint32_t ni = ins_off[i + 1] - ins_off[i];
-      int32_t *t = target[i];
-      if (!t) continue;
-      if (t == lst[x] && s_ptr[i] == lst[x]) {
-        // in place, insertions only: merge from the back
-        int64_t a = (int64_t)s_len[i] - 1, b = (int64_t)ni - 1, w = (int64_t)newlen[i] - 1;
-        while (b >= 0) {
-          if (a >= 0 && t[a] > in[b]) t[w--] = t[a--];
-          else t[w--] = in[b--];
-        }
-      } else {
-        std::merge(s_ptr[i], s_ptr[i] + s_len[i], in, in + ni, t);
-      }
+      if (target[i]) std::merge(s_ptr[i], s_ptr[i] + s_len[i], in, in + ni, target[i]);
     }
   });
   for (size_t i = 0; i < nu; ++i) {
     const int32_t x = U[i];
+    if (lst[x]) retired.push_back({lst[x], cap[x]});
     deg_hist[len[x]]--;
     if (newlen[i] >= deg_hist.size()) deg_hist.resize((size_t)newlen[i] + 1, 0);
     deg_hist[newlen[i]]++;
@@ -324,6 +318,11 @@ void HostStore::merge() {
   }
   maxdeg = (uint32_t)deg_hist.size() - 1;
   while (maxdeg > 0 && deg_hist[maxdeg] == 0) --maxdeg;
+}
+
+void HostStore::recycle(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
+  for (auto &r : retired) free_[r.second].push_back(r.first);
+  retired.clear();
 }
 
 void HostStore::clear_batch() {

@@ -14,6 +14,7 @@
 #pragma once
 #include <cstdint>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "estimator.h"
@@ -47,10 +48,14 @@ class HostStore {
   // ---- batch (steps ① / a0-a1) ----
   // Validates and normalises; on EINVAL returns the message and mutates nothing.
   std::string normalize(int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del);
-  bool build_overlay(bool *cuda_err);   // S(x) for x ∈ U with deletions
+  bool build_overlay(int slot, bool *cuda_err);  // S(x) for x ∈ U with deletions (per in-flight slot)
   HList view(int32_t v, int view) const;
   uint32_t view_len(int32_t v, int view) const;
-  void merge();                         // step ⑤
+  // step ⑤: base(x) <- S(x) ∪ ins(x) for x ∈ U, always into a *fresh* array (a recycled one of the same
+  // capacity class, or a doubled one when full) so that a batch whose kernels are still reading
+  // the old arrays (pipelined submit) is not disturbed; the old arrays are appended to `retired`.
+  void merge(std::vector<std::pair<int32_t *, uint32_t>> &retired);
+  void recycle(std::vector<std::pair<int32_t *, uint32_t>> &retired);  // once their batch has completed
   void clear_batch();
 
   // batch state
@@ -67,7 +72,8 @@ class HostStore {
 
  private:
   std::vector<Chunk> chunks_;
-  Chunk overlay_;
+  Chunk overlay_[2];
+  std::unordered_map<uint32_t, std::vector<int32_t *>> free_;  // recycled arrays by capacity
   int32_t *alloc_list(uint32_t capacity, bool *cuda_err);
   bool new_chunk(size_t bytes, Chunk &c);
   bool has_edge(int32_t u, int32_t v) const;

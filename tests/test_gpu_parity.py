@@ -315,3 +315,41 @@ def test_cache_policies_same_counts(G):
         assert got == want, pol
         if pol == "none":
             assert st["hit_bytes"] == 0 or st["cached_vertices"] == 0
+
+
+# ------------------------------------------------------------------ pipelined submit / wait (NEXT-2)
+
+@pytest.mark.parametrize("name", ["k4", "c4", "house5u"])
+def test_pipelined_submit_wait(G, name):
+    """Batch t+1's host steps overlap batch t's kernels; counts, final graph and state rules are unchanged."""
+    w = gi.make_workload("C2", scale=12, n_edges=40_000, batch=256, n_batches=6)
+    want, (rp1, col1) = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    k, qe, ql = gi.query(name)
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(w.adj_bytes // 10)
+    got = []
+    g.submit_batch(*w.batches[0])
+    for b in w.batches[1:]:
+        g.submit_batch(*b)
+        got.append(g.wait_batch())
+    got.append(g.wait_batch())
+    assert got == want
+    rp2, col2 = g.export_csr()
+    assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
+    # state rules
+    with pytest.raises(G.GcsmError) as ei:
+        g.wait_batch()
+    assert ei.value.name == "GCSM_ESTATE"
+    g.submit_batch(np.zeros((0, 2)), np.zeros((0, 2)))
+    g.submit_batch(np.zeros((0, 2)), np.zeros((0, 2)))
+    for call in (lambda: g.submit_batch(np.zeros((0, 2)), np.zeros((0, 2))), lambda: g.set_query(k, qe, ql),
+                 lambda: g.set_cache_budget(1 << 20)):
+        with pytest.raises(G.GcsmError) as ei:
+            call()
+        assert ei.value.name == "GCSM_ESTATE"
+    assert g.wait_batch() == (0, 0) and g.wait_batch() == (0, 0)
+    # apply_batch drains outstanding submissions first
+    g.submit_batch(np.zeros((0, 2)), np.zeros((0, 2)))
+    assert g.apply_batch(np.zeros((0, 2)), np.zeros((0, 2))) == (0, 0)
+    g.close()
