@@ -478,17 +478,20 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
   const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
   const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
   const int32_t *f2u = f2c + A.f2_cap;
+  // work grab size: runs of up to kChunk entries, smaller when the frontier would leave warps idle
+  const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t chunk = max((int64_t)1, min((int64_t)kChunk, n_f2 / (4 * warps)));
   Acc acc;
   Pinned pin;
   int64_t ci = 0, c_end = 0;
   for (;;) {
     if (ci >= c_end) {  // grab the next chunk of the (x2-grouped) frontier order
       unsigned long long c0 = 0;
-      if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)kChunk);
+      if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)chunk);
       c0 = __shfl_sync(kFull, c0, 0);
       if ((int64_t)c0 >= n_f2) break;
       ci = (int64_t)c0;
-      c_end = min((int64_t)c0 + kChunk, n_f2);
+      c_end = min((int64_t)c0 + chunk, n_f2);
       pin.v = -1;
     }
     const int64_t e = A.group ? A.group[ci] : ci;
