@@ -37,10 +37,16 @@ constexpr int kWarps = 8;
 constexpr int kBlock = 32 * kWarps;
 constexpr unsigned kFull = 0xffffffffu;
 #ifndef GCSM_SMEM_INTS
-#define GCSM_SMEM_INTS 1536
+#define GCSM_SMEM_INTS 1024
 #endif
 #ifndef GCSM_PRESTAGE_MERGE
 #define GCSM_PRESTAGE_MERGE 0
+#endif
+#ifndef GCSM_PIN_SMEM_MAX
+#define GCSM_PIN_SMEM_MAX 768  // largest x2 list (ints) pinned in the shared slice; larger ones go to HBM scratch
+#endif
+#ifndef GCSM_MINBLOCKS
+#define GCSM_MINBLOCKS 4  // resident 256-thread blocks per SM requested from ptxas for k_extend
 #endif
 #ifndef GCSM_MERGE_INT4
 #define GCSM_MERGE_INT4 0
@@ -187,7 +193,7 @@ __device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint
 // binary-search step below the first 8-int sector), into the warp's shared
 // memory slice if it fits, else (zero-copy lists only) into its HBM scratch.
 __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl, int drv, bool has_set, uint32_t dn,
-                                            int32_t *sm, int32_t *gbuf, int lane, Acc &acc) {
+                                            int32_t *sm, uint32_t sm_cap, int32_t *gbuf, int lane, Acc &acc) {
   const uint32_t d = has_set ? dn : L[drv].ml + L[drv].xl;
   uint32_t sm_used = 0, g_used = 0;
   bool any = false;
@@ -206,7 +212,7 @@ __device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl,
     if (!stage) continue;
     const uint32_t n4 = (n + 3) & ~3u;
     if (!hit) acc.copied += 4ull * n;
-    if (sm_used + n4 <= kSmemInts) {
+    if (sm_used + n4 <= sm_cap) {
       warp_copy(sm + sm_used, L[p].m, n, lane);
       L[p].m = sm + sm_used;
       L[p].dev = true;
@@ -423,7 +429,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
     LRef L[7];
     int drv;
     const int nl = gather_lists(A, L2, f, L, &drv, acc);
-    stage_lists(A, L, nl, drv, false, 0, sm, gstage, lane, acc);
+    stage_lists(A, L, nl, drv, false, 0, sm, kSmemInts, gstage, lane, acc);
     int32_t excl[2];
     int nex = 0;
     for (int i = 0; i < L2.ninj; ++i) excl[nex++] = f[L2.inj[i]];
@@ -464,8 +470,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
 }
 
 // Levels 3..k-1 (DFS): warp per level-2 frontier entry.
-template <bool LIST>
-__global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
+template <bool LIST, int KK>  // KK: compile-time query size (4: the level-3 count only), 0 = any
+__global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int32_t *stack = A.scratch + gw * A.scratch_stride;  // buffer for position p: stack + (p - 3) * dcap
@@ -473,7 +479,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
   int32_t *pstage = gstage - (int64_t)A.dcap;  // persistent copy of the current x2's main list
   extern __shared__ int4 smem_raw[];
   int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
-  const int k = A.k;
+  const int k = KK ? KK : A.k;
   int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
   const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
   const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
@@ -483,6 +489,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
   const int64_t chunk = max((int64_t)1, min((int64_t)kChunk, n_f2 / (4 * warps)));
   Acc acc;
   Pinned pin;
+  uint32_t pin_sm = 0;  // ints of the shared slice held by the pinned x2 list
   int64_t ci = 0, c_end = 0;
   for (;;) {
     if (ci >= c_end) {  // grab the next chunk of the (x2-grouped) frontier order
@@ -493,6 +500,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
       ci = (int64_t)c0;
       c_end = min((int64_t)c0 + chunk, n_f2);
       pin.v = -1;
+      pin_sm = 0;
     }
     const int64_t e = A.group ? A.group[ci] : ci;
     const int32_t x2 = f2c[e];
@@ -507,7 +515,17 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
       const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
                                                               ((unsigned long long)(unsigned)raw.y << 32));
       const uint32_t ml = (uint32_t)raw.z;
-      if (run >= 2 && ml >= 32 && !is_hit(A, mp) && ml <= (uint32_t)A.dcap) {
+      const bool miss = !is_hit(A, mp);
+      const uint32_t ml4 = (ml + 3) & ~3u;
+      pin_sm = 0;
+      if (run >= 2 && ml >= 32 && ml4 <= GCSM_PIN_SMEM_MAX) {  // fits the shared slice: pin hits and misses
+        warp_copy(sm, mp, ml, lane);
+        if (miss) acc.copied += 4ull * ml;
+        __syncwarp();
+        pin.v = x2;
+        pin.p = sm;
+        pin_sm = ml4;
+      } else if (run >= 2 && ml >= 32 && miss && ml <= (uint32_t)A.dcap) {
         warp_copy(pstage, mp, ml, lane);
         acc.copied += 4ull * ml;
         __syncwarp();
@@ -546,7 +564,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_extend(const MatchArgs A) {
         // last level, two lists already in device memory: merge without staging
         const bool merged = GCSM_PRESTAGE_MERGE && !LIST && p == k - 1 && !dset && nl == 2 &&
                             count2(A, L, drv, excl, nex, Lp.label, lane, &c);
-        if (!merged) stage_lists(A, L, nl, drv, dset != nullptr, dn, sm, gstage, lane, acc);
+        if (!merged) stage_lists(A, L, nl, drv, dset != nullptr, dn, sm + pin_sm, kSmemInts - pin_sm, gstage, lane, acc);
         if (merged) {
           if (P.kind) acc.rem += c;
           else acc.add += c;
@@ -711,11 +729,12 @@ cudaError_t upload_plans(DevPlan *dst, const DevPlan *plans, int n, cudaStream_t
 int match_grid(int device, int *warps_total) {
   int sms = 0, occ = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  cudaFuncSetAttribute(k_extend<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-  cudaFuncSetAttribute(k_extend<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_extend<false, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_extend<false, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_extend<true, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   cudaFuncSetAttribute(k_level2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   cudaFuncSetAttribute(k_level2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false>, kBlock, kSmemBytes);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false, 0>, kBlock, kSmemBytes);
   int occ2 = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_level2<false>, kBlock, kSmemBytes);
   if (occ2 < occ) occ = occ2;
@@ -736,8 +755,9 @@ cudaError_t launch_level2(const MatchArgs &a0, int grid, cudaStream_t s) {
 cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
   MatchArgs a = a0;
   a.acc_base = CNT_ACC_EXT;
-  if (a.listing) k_extend<true><<<grid, kBlock, kSmemBytes, s>>>(a);
-  else k_extend<false><<<grid, kBlock, kSmemBytes, s>>>(a);
+  if (a.listing) k_extend<true, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
+  else if (a.k == 4) k_extend<false, 4><<<grid, kBlock, kSmemBytes, s>>>(a);
+  else k_extend<false, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
   return cudaGetLastError();
 }
 
