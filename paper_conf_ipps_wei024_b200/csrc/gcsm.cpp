@@ -117,6 +117,10 @@ struct gcsm_ctx {
   int64_t *d_pidx = nullptr; size_t pidx_cap = 0;
   VDesc *d_pval = nullptr; size_t pval_cap = 0;
   int32_t *d_tup = nullptr; size_t tup_cap = 0;
+  int32_t *d_arena = nullptr; size_t arena_cap = 0;     // level-3 work sharing (k >= 5)
+  Task *d_tasks = nullptr; size_t tasks_cap = 0;
+  int32_t *d_task_ready = nullptr; size_t task_ready_cap = 0;
+  int32_t task_gen = 0;
 
 
   // cache / batch state
@@ -151,7 +155,7 @@ gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
   void *dev[] = {d_vdesc, d_plans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
-                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh};
+                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (void *p : dev)
     if (p) cudaFree(p);
   for (Slot &sl : slots) {
@@ -709,6 +713,19 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.tup_rem_cap = rem_cap;
   A.k = k;
   A.listing = listing ? 1 : 0;
+  if (k >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
+    const size_t na = (size_t)64 << 20, nt = (size_t)4 << 20;
+    const bool fresh_ready = ctx->d_task_ready == nullptr;
+    if (!dev_ensure(ctx->d_arena, ctx->arena_cap, na) || !dev_ensure(ctx->d_tasks, ctx->tasks_cap, nt) ||
+        !dev_ensure(ctx->d_task_ready, ctx->task_ready_cap, nt))
+      return ctx->fail(GCSM_ENOMEM, "work-sharing buffers");
+    if (fresh_ready) CK(cudaMemsetAsync(ctx->d_task_ready, 0, 4 * ctx->task_ready_cap, s));
+    A.arena = ctx->d_arena;
+    A.arena_cap = ctx->arena_cap;
+    A.tasks = ctx->d_tasks;
+    A.task_ready = ctx->d_task_ready;
+    A.task_cap = (uint32_t)std::min<size_t>(ctx->tasks_cap, ctx->task_ready_cap);
+  }
   CK(cudaEventRecord(sl.ev_m0, s));
   size_t nev = 0;
   for (const auto &ch : chunks) {
@@ -731,6 +748,10 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_group, s));
       launches += 6;
       A.group = ctx->d_group;
+      if (A.tasks) {
+        if (++ctx->task_gen <= 0) ctx->task_gen = 1;  // ready flags hold the launch's generation, never 0
+        A.task_gen = ctx->task_gen;
+      }
       CK(launch_extend(A, ctx->grid, s));
       ++launches;
     }

@@ -54,6 +54,8 @@ constexpr unsigned kFull = 0xffffffffu;
 constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 constexpr int kChunk = 32;  // frontier entries per k_extend work grab
+constexpr uint32_t kSplitMin = 64;  // level-3 sets larger than this are shared as tasks (k >= 5)
+constexpr uint32_t kTaskSize = 16;  // level-3 candidates per task
 
 struct LRef {
   const int32_t *m;  // main list
@@ -490,50 +492,107 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   Acc acc;
   Pinned pin;
   uint32_t pin_sm = 0;  // ints of the shared slice held by the pinned x2 list
-  int64_t ci = 0, c_end = 0;
+  int64_t ci = 0, c_end = 0, c_start = 0;
+  bool producing = true;  // phase 1: walk the (grouped) frontier; phase 2 (k >= 5): take shared level-3 tasks
+  const bool sharing = KK == 0 && !LIST && k >= 5 && A.tasks != nullptr;
   for (;;) {
-    if (ci >= c_end) {  // grab the next chunk of the (x2-grouped) frontier order
-      unsigned long long c0 = 0;
-      if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)chunk);
-      c0 = __shfl_sync(kFull, c0, 0);
-      if ((int64_t)c0 >= n_f2) break;
-      ci = (int64_t)c0;
-      c_end = min((int64_t)c0 + chunk, n_f2);
-      pin.v = -1;
-      pin_sm = 0;
-    }
-    const int64_t e = A.group ? A.group[ci] : ci;
-    const int32_t x2 = f2c[e];
-    if (x2 != pin.v) {
-      // run of entries sharing x2 in this chunk: stage x2's zero-copy main list once for all of them
-      int64_t j = ci + 1 + lane;
-      const bool same = j < c_end && f2c[A.group ? A.group[j] : j] == x2;
-      const unsigned run_mask = __ballot_sync(kFull, same);
-      const int run = 1 + (run_mask == kFull ? 32 : __ffs(~run_mask) - 1);  // entries of this run (capped at 33)
-      pin.v = -1;
-      const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + x2));
-      const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
-                                                              ((unsigned long long)(unsigned)raw.y << 32));
-      const uint32_t ml = (uint32_t)raw.z;
-      const bool miss = !is_hit(A, mp);
-      const uint32_t ml4 = (ml + 3) & ~3u;
-      pin_sm = 0;
-      if (run >= 2 && ml >= 32 && ml4 <= GCSM_PIN_SMEM_MAX) {  // fits the shared slice: pin hits and misses
-        warp_copy(sm, mp, ml, lane);
-        if (miss) acc.copied += 4ull * ml;
-        __syncwarp();
-        pin.v = x2;
-        pin.p = sm;
-        pin_sm = ml4;
-      } else if (run >= 2 && ml >= 32 && miss && ml <= (uint32_t)A.dcap) {
-        warp_copy(pstage, mp, ml, lane);
-        acc.copied += 4ull * ml;
-        __syncwarp();
-        pin.v = x2;
-        pin.p = pstage;
+    int64_t e;
+    bool task = false;
+    Task tk;
+    if (producing) {
+      if (ci >= c_end) {  // grab the next chunk of the (x2-grouped) frontier order
+        unsigned long long c0 = 0;
+        if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)chunk);
+        c0 = __shfl_sync(kFull, c0, 0);
+        if (sharing && c_end > 0 && lane == 0) {  // the previous chunk is finished (tasks published)
+          __threadfence();
+          atomicAdd(&A.cnt[CNT_PRODUCERS], (unsigned long long)(c_end - c_start));
+        }
+        if ((int64_t)c0 >= n_f2) {
+          if (!sharing) break;
+          producing = false;
+          pin.v = -1;
+          pin_sm = 0;
+          continue;
+        }
+        c_start = (int64_t)c0;
+        ci = (int64_t)c0;
+        c_end = min((int64_t)c0 + chunk, n_f2);
+        pin.v = -1;
+        pin_sm = 0;
       }
+      e = A.group ? A.group[ci] : ci;
+      const int32_t x2 = f2c[e];
+      if (x2 != pin.v) {
+        // run of entries sharing x2 in this chunk: stage x2's zero-copy main list once for all of them
+        int64_t j = ci + 1 + lane;
+        const bool same = j < c_end && f2c[A.group ? A.group[j] : j] == x2;
+        const unsigned run_mask = __ballot_sync(kFull, same);
+        const int run = 1 + (run_mask == kFull ? 32 : __ffs(~run_mask) - 1);  // entries of this run (capped at 33)
+        pin.v = -1;
+        const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + x2));
+        const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
+                                                                ((unsigned long long)(unsigned)raw.y << 32));
+        const uint32_t ml = (uint32_t)raw.z;
+        const bool miss = !is_hit(A, mp);
+        const uint32_t ml4 = (ml + 3) & ~3u;
+        pin_sm = 0;
+        if (run >= 2 && ml >= 32 && ml4 <= GCSM_PIN_SMEM_MAX) {  // fits the shared slice: pin hits and misses
+          warp_copy(sm, mp, ml, lane);
+          if (miss) acc.copied += 4ull * ml;
+          __syncwarp();
+          pin.v = x2;
+          pin.p = sm;
+          pin_sm = ml4;
+        } else if (run >= 2 && ml >= 32 && miss && ml <= (uint32_t)A.dcap) {
+          warp_copy(pstage, mp, ml, lane);
+          acc.copied += 4ull * ml;
+          __syncwarp();
+          pin.v = x2;
+          pin.p = pstage;
+        }
+      }
+      ++ci;
+    } else {
+      // phase 2: take a ticket (unique task index); wait until that task is published, or leave when every
+      // frontier entry has been walked (the task tail is final) and the ticket lies past it
+      unsigned long long h = 0;
+      if (lane == 0) h = atomicAdd(&A.cnt[CNT_HEAD], 1ull);
+      h = __shfl_sync(kFull, h, 0);
+      int state = 0;  // 1: task h is ready, 2: no such task will exist
+      if (lane == 0) {
+        unsigned ns = 64;
+        for (;;) {
+          const unsigned long long tail = *(volatile unsigned long long *)&A.cnt[CNT_TAIL];
+          if (h < tail) {
+            if (h >= A.task_cap) { state = 3; break; }  // reserved past the array: its owner kept the work
+            if (*(volatile int32_t *)&A.task_ready[h] == A.task_gen) { state = 1; break; }
+          } else {
+            const unsigned long long done = *(volatile unsigned long long *)&A.cnt[CNT_PRODUCERS];
+            __threadfence();  // the producers fence between publishing and counting an entry as walked
+            if ((int64_t)done >= n_f2 && h >= *(volatile unsigned long long *)&A.cnt[CNT_TAIL]) { state = 2; break; }
+          }
+          __nanosleep(ns);
+          if (ns < 4096) ns <<= 1;
+        }
+      }
+      state = __shfl_sync(kFull, state, 0);
+      if (state == 2) break;
+      if (state == 3) continue;
+      __syncwarp();
+      __threadfence();
+      // other SMs wrote the task and its arena slice during this launch: read them through L2 (ld.global.cg),
+      // never from a possibly stale L1 line
+      {
+        const unsigned long long *src = reinterpret_cast<const unsigned long long *>(&A.tasks[h]);
+        unsigned long long w[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) w[i] = __ldcg(src + i);
+        memcpy(&tk, w, sizeof(Task));
+      }
+      e = tk.e;
+      task = true;
     }
-    ++ci;
     const int32_t ui = f2u[e];
     const Unit U = A.units[ui];
     const DevPlan &P = A.plans[U.plan];
@@ -546,8 +605,20 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     uint32_t sz[GCSM_MAXK], it[GCSM_MAXK];
     set[2] = f2c + seg.x;
     sz[2] = (uint32_t)seg.y;
+    uint32_t end3 = 0xffffffffu;  // level-3 iteration bound (a task's slice)
     int lvl = 2;   // deepest position with a chosen element
     bool descend = true;
+    if (task) {
+      int32_t *own = stack;  // this warp's level-3 buffer: a private, L1-safe copy of the shared set
+      for (uint32_t i = lane; i < tk.n; i += 32) own[i] = __ldcg(A.arena + tk.off + i);
+      __syncwarp();
+      set[3] = own;
+      sz[3] = tk.n;
+      it[3] = tk.lo;
+      end3 = tk.hi;
+      lvl = 3;
+      descend = false;
+    }
     for (;;) {
       if (descend) {
         const int p = lvl + 1;  // compute candidates of position p
@@ -589,10 +660,56 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           it[p] = 0;
           lvl = p;
           descend = false;
+          if (p == 3 && sharing && sz[3] > kSplitMin) {
+            // share this level-3 set: copy it to the arena and publish slices of it as tasks
+            const uint32_t n3 = sz[3], nt = (n3 + kTaskSize - 1) / kTaskSize;
+            unsigned long long off = 0, t0 = 0;
+            if (lane == 0) {
+              off = atomicAdd(&A.cnt[CNT_ARENA], (unsigned long long)n3);
+              t0 = atomicAdd(&A.cnt[CNT_TAIL], (unsigned long long)nt);
+            }
+            off = __shfl_sync(kFull, off, 0);
+            t0 = __shfl_sync(kFull, t0, 0);
+            if (off + n3 <= A.arena_cap && t0 + nt <= A.task_cap) {
+              for (uint32_t i = lane; i < n3; i += 32) A.arena[off + i] = out[i];
+              for (uint32_t t = lane; t < nt; t += 32) {
+                Task q;
+                q.e = e;
+                q.off = off;
+                q.n = n3;
+                q.lo = t * kTaskSize;
+                q.hi = min(n3, (t + 1) * kTaskSize);
+                q.pad = 0;
+                A.tasks[t0 + t] = q;
+              }
+              __threadfence();
+              __syncwarp();
+              for (uint32_t t = lane; t < nt; t += 32) *(volatile int32_t *)&A.task_ready[t0 + t] = A.task_gen;
+              if (lane == 0) atomicAdd(&A.cnt[CNT_SPLIT], 1ull);
+              end3 = 0;  // all of it delegated
+            } else {
+              // no room: publish empty tasks for the reserved slots so takers do not wait forever
+              for (uint32_t t = lane; t < nt; t += 32) {
+                if (t0 + t < A.task_cap) {
+                  Task q;
+                  q.e = e;
+                  q.off = 0;
+                  q.n = 0;
+                  q.lo = q.hi = 0;
+                  q.pad = 0;
+                  A.tasks[t0 + t] = q;
+                }
+              }
+              __threadfence();
+              __syncwarp();
+              for (uint32_t t = lane; t < nt; t += 32)
+                if (t0 + t < A.task_cap) *(volatile int32_t *)&A.task_ready[t0 + t] = A.task_gen;
+            }
+          }
         }
       }
       // choose the next element at the deepest open position (>= 3)
-      while (lvl >= 3 && it[lvl] == sz[lvl]) --lvl;
+      while (lvl >= 3 && it[lvl] >= (lvl == 3 ? min(end3, sz[3]) : sz[lvl])) --lvl;
       if (lvl < 3) break;
       f[lvl] = set[lvl][it[lvl]++];
       descend = true;
@@ -752,9 +869,17 @@ cudaError_t launch_level2(const MatchArgs &a0, int grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
+__global__ void k_reset_sharing(unsigned long long *cnt) {
+  cnt[CNT_ARENA] = 0;
+  cnt[CNT_TAIL] = 0;
+  cnt[CNT_HEAD] = 0;
+  cnt[CNT_PRODUCERS] = 0;
+}
+
 cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
   MatchArgs a = a0;
   a.acc_base = CNT_ACC_EXT;
+  if (a.tasks) k_reset_sharing<<<1, 1, 0, s>>>(a.cnt);
   if (a.listing) k_extend<true, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
   else if (a.k == 4) k_extend<false, 4><<<grid, kBlock, kSmemBytes, s>>>(a);
   else k_extend<false, 0><<<grid, kBlock, kSmemBytes, s>>>(a);

@@ -21,7 +21,12 @@ enum Counter {
   // the HBM cache, zero-copy from pinned host memory, and from the device delta segments (ins/del of U)
   CNT_ACC_L2 = 10,
   CNT_ACC_EXT = 13,
-  CNT_N = 16
+  CNT_ARENA = 16,   // ints used in the level-3 task arena
+  CNT_TAIL = 17,    // level-3 tasks published (reserved)
+  CNT_HEAD = 18,    // level-3 tasks taken
+  CNT_PRODUCERS = 19,  // frontier entries fully walked (their tasks, if any, published)
+  CNT_SPLIT = 20,   // level-3 sets handed out as tasks (stats)
+  CNT_N = 24
 };
 
 struct MatchArgs {
@@ -49,6 +54,22 @@ struct MatchArgs {
   int32_t k;
   int32_t listing;
   int32_t acc_base;         // CNT_ACC_L2 or CNT_ACC_EXT (set by the launchers)
+  // level-3 work sharing (k >= 5): a warp whose level-3 candidate set is large copies it to the arena and
+  // publishes slices of it as tasks that idle warps take (STMatch-style work sharing)
+  int32_t *arena;
+  uint64_t arena_cap;       // ints
+  struct Task *tasks;
+  int32_t *task_ready;
+  uint32_t task_cap;
+  int32_t task_gen;         // ready-flag value of this launch (no per-launch clearing)
+};
+
+struct Task {
+  int64_t e;        // level-2 frontier entry (unit, x2)
+  uint64_t off;     // its level-3 candidate set in the arena
+  uint32_t n;       // set size
+  uint32_t lo, hi;  // the slice of positions this task iterates
+  uint32_t pad;
 };
 
 // plans live in a per-context device buffer (contexts may run concurrently)
