@@ -353,3 +353,54 @@ def test_pipelined_submit_wait(G, name):
     g.submit_batch(np.zeros((0, 2)), np.zeros((0, 2)))
     assert g.apply_batch(np.zeros((0, 2)), np.zeros((0, 2))) == (0, 0)
     g.close()
+
+
+# ------------------------------------------------------------------ full-size configs, bench launch configuration
+
+@pytest.mark.parametrize("cfg,queries", [("C2", ["k4", "c4"]), ("C3", ["house5", "bowtie5", "k5e"])])
+def test_full_size_sampled(G, cfg, queries):
+    """BASELINE configs[1]/[2] at full size (70M / 120M edges) with bench.py's launch configuration (default grid,
+    10 % budget, estimator cache): a sampled sub-batch (the first 256 updated edges of batch 0) against the oracle."""
+    w = gi.make_workload(cfg, n_batches=2)
+    ins, dele = w.batches[0]
+    si, sd = ins[:128], dele[:128]
+    for q in queries:
+        k, qe, ql = gi.query(q)
+        want = oracle.delta(w.n, w.row_ptr, w.col, w.labels, k, qe, ql, si, sd)
+        g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=0)
+        g.set_query(k, qe, ql)
+        g.set_cache_budget(int(w.adj_bytes * w.budget_frac))
+        assert g.apply_batch(si, sd) == want, q
+        st = g.stats()
+        assert st["cached_vertices"] > 0 and st["hit_bytes"] > 0
+        g.close()
+
+
+@pytest.mark.parametrize("r", [2, 3])
+def test_full_size_star_closed_form(G, r):
+    """Whole C2 batches at full size (4096 mixed updates, 70M edges) against the K_{1,r} degree closed form."""
+    w = gi.make_workload("C2", n_batches=2)
+    k = r + 1
+    qe = np.array([(0, i) for i in range(1, k)], np.int32)
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    g.set_query(k, qe)
+    g.set_cache_budget(w.adj_bytes // 10)
+    rp, col = w.row_ptr, w.col
+
+    def P(x):
+        out = np.ones_like(x, dtype=object)
+        for i in range(r):
+            out = out * (x - i)
+        return out
+
+    for ins, dele in w.batches:
+        I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+        rp1, col1 = oracle.apply_batch(w.n, rp, col, I, D)
+        U = np.unique(np.concatenate([I.ravel(), D.ravel()]))
+        d, d1 = np.diff(rp)[U].astype(object), np.diff(rp1)[U].astype(object)
+        # stable degree: old degree minus deleted incident edges
+        s = d - np.array([int(np.count_nonzero(D == u)) for u in U], dtype=object)
+        want = (int((P(d1) - P(s)).sum()), int((P(d) - P(s)).sum()))
+        assert g.apply_batch(ins, dele) == want
+        rp, col = rp1, col1
+    g.close()
