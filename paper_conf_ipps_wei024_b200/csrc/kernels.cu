@@ -45,6 +45,9 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GCSM_PIN_SMEM_MAX
 #define GCSM_PIN_SMEM_MAX 768  // largest x2 list (ints) pinned in the shared slice; larger ones go to HBM scratch
 #endif
+#ifndef GCSM_BM_INTS
+#define GCSM_BM_INTS 0  // per-warp membership bitmap of the run x2 list; measured slower than merge on C2 (off)
+#endif
 #ifndef GCSM_MINBLOCKS
 #define GCSM_MINBLOCKS 4  // resident 256-thread blocks per SM requested from ptxas for k_extend
 #endif
@@ -74,6 +77,7 @@ struct Acc {
 struct Pinned {
   int32_t v = -1;
   const int32_t *p = nullptr;
+  int32_t bm_v = -1;  // vertex whose main list is in the warp's bitmap (the run's x2), -1 = none
 };
 
 __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc,
@@ -340,6 +344,48 @@ __device__ __forceinline__ bool count2(const MatchArgs &A, const LRef *L, int dr
   return true;
 }
 
+// ---- run-shared bitmap count ------------------------------------------------------
+// The run's x2 list P is hashed once into a per-warp shared bitmap; each entry then streams its other list X
+// coalesced (32 consecutive elements per warp step, independent loads) and an element survives the bitmap
+// test only if its hash bit is set — about (matches + |P|/bits) of them — and is then verified exactly by a
+// binary search of P. Exact: every element of X ∩ P has its bit set; the bitmap only filters.
+constexpr int kBmLog2 = GCSM_BM_INTS > 0 ? 5 + __builtin_ctz(GCSM_BM_INTS) : 5;
+__device__ __forceinline__ uint32_t bm_hash(int32_t v) { return ((uint32_t)v * 2654435761u) >> (32 - kBmLog2); }
+
+__device__ __forceinline__ void bm_build(uint32_t *bm, const int32_t *P, uint32_t n, int lane) {
+  for (uint32_t i = lane; i < (uint32_t)GCSM_BM_INTS; i += 32) bm[i] = 0;
+  __syncwarp();
+  for (uint32_t i = lane; i < n; i += 32) {
+    const uint32_t h = bm_hash(P[i]);
+    atomicOr(&bm[h >> 5], 1u << (h & 31));
+  }
+  __syncwarp();
+}
+
+__device__ __forceinline__ uint32_t bm_count(const MatchArgs &A, const uint32_t *bm, const LRef &X, const LRef &P,
+                                             const int32_t *excl, int nexcl, int label, int lane) {
+  uint32_t cnt = 0;
+  auto visit = [&](const int32_t *seg, uint32_t n) {
+    for (uint32_t i = lane; i < n; i += 32) {
+      const int32_t v = seg[i];
+      const uint32_t h = bm_hash(v);
+      bool in = false;
+      if ((bm[h >> 5] >> (h & 31)) & 1u) in = bsearch_has(P.m, P.ml, v);
+      if (!in && P.xl) in = bsearch_has(P.x, P.xl, v);
+      if (!in) continue;
+      if (label >= 0 && A.lab[v] != (uint16_t)label) continue;
+      bool ex = false;
+      for (int e = 0; e < nexcl; ++e) ex |= v == excl[e];
+      cnt += !ex;
+    }
+  };
+  visit(X.m, X.ml);
+  if (X.xl) visit(X.x, X.xl);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
+  return cnt;
+}
+
 // Lists of position p for the current partial match f (positions 0..p-1).
 // Returns the number of probe lists written to L and sets *drv (index of the
 // smallest list) or uses the reused set.
@@ -480,7 +526,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   int32_t *gstage = stack + A.scratch_stride - 2 * (int64_t)A.dcap;
   int32_t *pstage = gstage - (int64_t)A.dcap;  // persistent copy of the current x2's main list
   extern __shared__ int4 smem_raw[];
-  int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
+  uint32_t *bm = reinterpret_cast<uint32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
+  int32_t *sm = reinterpret_cast<int32_t *>(bm) + GCSM_BM_INTS;  // pin area, then transient staging
+  constexpr uint32_t kSlice = kSmemInts - GCSM_BM_INTS;
   const int k = KK ? KK : A.k;
   int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
   const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
@@ -512,6 +560,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           if (!sharing) break;
           producing = false;
           pin.v = -1;
+          pin.bm_v = -1;
           pin_sm = 0;
           continue;
         }
@@ -519,6 +568,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         ci = (int64_t)c0;
         c_end = min((int64_t)c0 + chunk, n_f2);
         pin.v = -1;
+        pin.bm_v = -1;
         pin_sm = 0;
       }
       e = A.group ? A.group[ci] : ci;
@@ -537,6 +587,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const bool miss = !is_hit(A, mp);
         const uint32_t ml4 = (ml + 3) & ~3u;
         pin_sm = 0;
+        pin.bm_v = -1;
         if (run >= 2 && ml >= 32 && ml4 <= GCSM_PIN_SMEM_MAX) {  // fits the shared slice: pin hits and misses
           warp_copy(sm, mp, ml, lane);
           if (miss) acc.copied += 4ull * ml;
@@ -550,6 +601,10 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           __syncwarp();
           pin.v = x2;
           pin.p = pstage;
+        }
+        if (GCSM_BM_INTS > 0 && run >= 2 && ml >= 32 && (pin.v == x2 || !miss)) {
+          bm_build(bm, pin.v == x2 ? pin.p : mp, ml, lane);
+          pin.bm_v = x2;
         }
       }
       ++ci;
@@ -632,10 +687,26 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
         const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
         uint32_t c = 0;
-        // last level, two lists already in device memory: merge without staging
-        const bool merged = GCSM_PRESTAGE_MERGE && !LIST && p == k - 1 && !dset && nl == 2 &&
-                            count2(A, L, drv, excl, nex, Lp.label, lane, &c);
-        if (!merged) stage_lists(A, L, nl, drv, dset != nullptr, dn, sm + pin_sm, kSmemInts - pin_sm, gstage, lane, acc);
+        // last level, two lists, one of them the run's x2 list in the bitmap: stream the other one
+        bool merged = false;
+        if (GCSM_BM_INTS > 0 && !LIST && p == k - 1 && !dset && nl == 2 && pin.bm_v >= 0 && !task) {
+          const int pi = f[Lp.bpos[0]] == pin.bm_v ? 0 : (f[Lp.bpos[1]] == pin.bm_v ? 1 : -1);
+          if (pi >= 0) {
+            const LRef &X = L[1 - pi];
+            const uint32_t nx = X.ml + X.xl, np = L[pi].ml + L[pi].xl;
+            const uint32_t bm_cost = 8 * ((nx + 31) >> 5) + 24;
+            const uint32_t d = min(nx, np), big = max(nx, np);
+            const uint32_t bs_cost = ((d + 31) >> 5) * (7 * ilog2(big) + 12);
+            if (bm_cost <= bs_cost && X.dev) {
+              c = bm_count(A, bm, X, L[pi], excl, nex, Lp.label, lane);
+              merged = true;
+            }
+          }
+        }
+        if (!merged)
+          merged = GCSM_PRESTAGE_MERGE && !LIST && p == k - 1 && !dset && nl == 2 &&
+                   count2(A, L, drv, excl, nex, Lp.label, lane, &c);
+        if (!merged) stage_lists(A, L, nl, drv, dset != nullptr, dn, sm + pin_sm, kSlice - pin_sm, gstage, lane, acc);
         if (merged) {
           if (P.kind) acc.rem += c;
           else acc.add += c;
