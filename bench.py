@@ -49,6 +49,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=20.0)
     ap.add_argument("--quick", action="store_true", help="profiling mode: no clocks sampler / cpu baseline")
+    ap.add_argument("--emulate", action="store_true",
+                    help="test the N>1 plumbing on one GPU: gloo process group, every rank on cuda:0, shard-local "
+                         "counts (no NCCL communicator)")
     ap.add_argument("--serial", action="store_true",
                     help="synchronous apply_batch, query contexts one after the other (default at N=1: one host "
                          "thread per query context, each pipelining submit/wait so batch t+1's host steps overlap "
@@ -107,7 +110,13 @@ def dist_setup(args):
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     import torch
-    if world > 1:
+    if world > 1 and args.emulate:
+        import torch.distributed as dist
+        torch.cuda.set_device(0)
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("gloo")
+        local = 0
+    elif world > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local)
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
@@ -128,7 +137,7 @@ def allmax(world, x):
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([float(x)], device="cuda")
+    t = torch.tensor([float(x)], device="cuda" if dist.get_backend() == "nccl" else "cpu")
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -238,18 +247,22 @@ def main():
     import gcsm_inputs as gi
     import paper_conf_ipps_wei024_b200 as G
 
+    # the host cores are shared by the ranks of one node
+    per_rank = max(1, (os.cpu_count() or 1) // world)
+    os.environ.setdefault("GCSM_GEN_THREADS", str(per_rank))
     t0 = time.perf_counter()
     w = workload(args, world)
     gen_s = time.perf_counter() - t0
     queries = args.queries.split(",") if args.queries else w.queries
     frac = w.budget_frac if args.budget_frac is None else args.budget_frac
     budget = int(w.adj_bytes * frac)
-    nccl_id = G.distributed_nccl_id() if world > 1 else None
+    nccl_id = G.distributed_nccl_id() if world > 1 and not args.emulate else None
     ctxs = []
     for q in queries:
         k, qe, ql = gi.query(q)
         g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=local, rank=rank, world=world, nccl_id=nccl_id,
-                   cache_policy=args.cache_policy)
+                   cache_policy=args.cache_policy, local_counts=bool(args.emulate and world > 1),
+                   host_threads=per_rank if world > 1 else 0)
         g.set_query(k, qe, ql)
         g.set_cache_budget(budget)
         ctxs.append((q, g))

@@ -77,9 +77,9 @@ enum {
 typedef struct {
   int32_t device;          /* CUDA ordinal; -1 = the current device */
   int32_t rank, world;     /* world = 1: single GPU */
-  const void *nccl_id;     /* 128-byte ncclUniqueId when world > 1 (gcsm_nccl_unique_id on rank 0,
-                              broadcast by the caller, e.g. through torch.distributed); NULL with
-                              GCSM_FLAG_LOCAL_COUNTS */
+  const void *nccl_id;     /* 128-byte ncclUniqueId (gcsm_nccl_unique_id on rank 0, broadcast by the
+                              caller, e.g. through torch.distributed): required when world > 1, optional
+                              with world = 1 (a one-rank communicator); NULL with GCSM_FLAG_LOCAL_COUNTS */
   uint64_t seed;           /* estimator RNG seed (R22) */
   int32_t host_threads;    /* 0 = all cores */
   int32_t cache_policy;    /* GCSM_CACHE_* */

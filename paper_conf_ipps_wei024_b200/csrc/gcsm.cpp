@@ -253,7 +253,8 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   }
   ctx->mark.assign(n, 0);
   ctx->grid = match_grid(dev, &ctx->warps_total);
-  if (o.world > 1 && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
+  // a communicator whenever an id is given (world 1 included: the single-rank allreduce exercises the same path)
+  if (o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
     ncclUniqueId id;
     std::memcpy(&id, o.nccl_id, sizeof id);
     if (ncclCommInitRank(&ctx->comm, o.world, id, o.rank) != ncclSuccess) return bail(GCSM_ENCCL);

@@ -78,11 +78,13 @@ struct Pinned {
   int32_t v = -1;
   const int32_t *p = nullptr;
   int32_t bm_v = -1;  // vertex whose main list is in the warp's bitmap (the run's x2), -1 = none
+  int32_t rv = -1;    // vertex whose descriptor is cached in `raw` (the run's x2: no reload per entry)
+  int4 raw;
 };
 
 __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc,
                                         const Pinned &pin = Pinned()) {
-  const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
+  const int4 raw = v == pin.rv ? pin.raw : __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
   LRef r;
   r.m = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
                                           ((unsigned long long)(unsigned)raw.y << 32));
@@ -581,6 +583,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const int run = 1 + (run_mask == kFull ? 32 : __ffs(~run_mask) - 1);  // entries of this run (capped at 33)
         pin.v = -1;
         const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + x2));
+        pin.rv = x2;
+        pin.raw = raw;
         const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
                                                                 ((unsigned long long)(unsigned)raw.y << 32));
         const uint32_t ml = (uint32_t)raw.z;

@@ -404,3 +404,13 @@ def test_full_size_star_closed_form(G, r):
         assert g.apply_batch(ins, dele) == want
         rp, col = rp1, col1
     g.close()
+
+
+def test_nccl_single_rank_allreduce(G):
+    """The NCCL path on one GPU: a one-rank communicator from gcsm_nccl_unique_id; the counts go through
+    ncclAllReduce on the kernel stream and come back unchanged."""
+    w = gi.make_workload("C2", scale=12, n_edges=30_000, batch=256, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, "diamond", w.batches)
+    got, st, _ = lib_run(G, w.n, w.row_ptr, w.col, None, "diamond", w.batches, 0.1, nccl_id=G.nccl_unique_id())
+    assert got == want
+    assert st["ms_allreduce"] > 0
