@@ -152,6 +152,10 @@ CONFIGS = {
     "C3": dict(scale=22, n_edges=120_000_000, abc=(0.502, 0.166, 0.166), id_limit=3_000_000, L=8,
                queries=["house5", "bowtie5", "k5e"], stream=12 * 8192, batch=4096, inserts_only=False,
                budget=0.10),
+    # FR-shaped: 67.1M ids, 1.8B edges (14.4 GB of adjacency in pinned host memory), hub ~5.2K
+    "C4": dict(scale=26, n_edges=1_800_000_000, abc=(0.42, 0.176, 0.176), id_limit=0, L=0,
+               queries=["prism6", "k4tri6", "k6"], stream=12 * 8192, batch=4096, inserts_only=False,
+               budget=0.01),
 }
 
 
