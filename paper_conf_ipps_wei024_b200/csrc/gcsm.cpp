@@ -783,7 +783,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // ---- (5) reorganise the host lists. P:302 runs it after matching so the kernel reads consistent data: here
   // the merge writes fresh arrays and the ones the in-flight kernels may read are retired, not overwritten.
   Timer t5;
-  S.merge(sl.retired);
+  if (!S.merge(sl.retired)) return ctx->fail(GCSM_ENOMEM, "pinned allocation for the merged lists failed");
   tr.mark("merge");
   ctx->prev_cached = sel;
   std::sort(ctx->prev_cached.begin(), ctx->prev_cached.end());

@@ -48,6 +48,14 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GCSM_BM_INTS
 #define GCSM_BM_INTS 0  // per-warp membership bitmap of the run x2 list; measured slower than merge on C2 (off)
 #endif
+#ifndef GCSM_COLD_NOINLINE
+#define GCSM_COLD_NOINLINE 0  // 1: generic intersection / staging / probe helpers out of line (register pressure)
+#endif
+#if GCSM_COLD_NOINLINE
+#define GCSM_COLD __noinline__
+#else
+#define GCSM_COLD __forceinline__
+#endif
 #ifndef GCSM_MINBLOCKS
 #define GCSM_MINBLOCKS 4  // resident 256-thread blocks per SM requested from ptxas for k_extend
 #endif
@@ -135,7 +143,7 @@ __device__ __forceinline__ bool contains(const LRef &L, int32_t v) {
 // MATERIALIZE: survivors are compacted into out[]. Returns the survivor count
 // (warp-uniform).
 template <bool MATERIALIZE>
-__device__ __forceinline__ uint32_t warp_isect(const MatchArgs &A, const int32_t *dset, uint32_t dn, const LRef *L,
+__device__ GCSM_COLD uint32_t warp_isect(const MatchArgs &A, const int32_t *dset, uint32_t dn, const LRef *L,
                                                int nl, int drv, const int32_t *excl, int nexcl, int label,
                                                int32_t *out, int lane) {
   const int32_t *s0, *s1;
@@ -200,7 +208,7 @@ __device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint
 // bytes than the probes would (4 L <= 32 B x d x (log2 L - 3): one sector per
 // binary-search step below the first 8-int sector), into the warp's shared
 // memory slice if it fits, else (zero-copy lists only) into its HBM scratch.
-__device__ __forceinline__ void stage_lists(const MatchArgs &A, LRef *L, int nl, int drv, bool has_set, uint32_t dn,
+__device__ GCSM_COLD void stage_lists(const MatchArgs &A, LRef *L, int nl, int drv, bool has_set, uint32_t dn,
                                             int32_t *sm, uint32_t sm_cap, int32_t *gbuf, int lane, Acc &acc) {
   const uint32_t d = has_set ? dn : L[drv].ml + L[drv].xl;
   uint32_t sm_used = 0, g_used = 0;
@@ -305,7 +313,7 @@ __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, c
 }
 
 // lane-parallel count of x[0..nx) present in the sorted list y (label-filtered)
-__device__ __forceinline__ uint32_t probe_count(const int32_t *x, uint32_t nx, const int32_t *y, uint32_t ny, int label,
+__device__ GCSM_COLD uint32_t probe_count(const int32_t *x, uint32_t nx, const int32_t *y, uint32_t ny, int label,
                                                 const uint16_t *lab, int lane) {
   uint32_t cnt = 0;
   for (uint32_t i = lane; i < nx; i += 32) {

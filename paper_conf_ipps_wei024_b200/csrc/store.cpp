@@ -285,7 +285,7 @@ uint32_t HostStore::view_len(int32_t v, int vw) const {
   return s_len[i];
 }
 
-void HostStore::merge(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
+bool HostStore::merge(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
   const size_t nu = U.size();
   std::vector<int32_t *> target(nu, nullptr);
   std::vector<uint32_t> newlen(nu), newcap(nu);
@@ -296,6 +296,11 @@ void HostStore::merge(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
     newcap[i] = cap[x];
     if (newlen[i] > cap[x]) newcap[i] = round4(std::max<uint64_t>(4, 2ull * newlen[i]));  // double
     target[i] = newcap[i] ? alloc_list(newcap[i], &err) : nullptr;
+    if (err) {  // give back what this merge took; the store is unchanged
+      for (size_t j = 0; j < i; ++j)
+        if (target[j]) free_[newcap[j]].push_back(target[j]);
+      return false;
+    }
   }
   parallel_for(threads, (int64_t)nu, [&](int, int64_t lo, int64_t hi) {
     for (int64_t i = lo; i < hi; ++i) {
@@ -318,6 +323,7 @@ void HostStore::merge(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
   }
   maxdeg = (uint32_t)deg_hist.size() - 1;
   while (maxdeg > 0 && deg_hist[maxdeg] == 0) --maxdeg;
+  return true;
 }
 
 void HostStore::recycle(std::vector<std::pair<int32_t *, uint32_t>> &retired) {

@@ -54,7 +54,7 @@ class HostStore {
   // step ⑤: base(x) <- S(x) ∪ ins(x) for x ∈ U, always into a *fresh* array (a recycled one of the same
   // capacity class, or a doubled one when full) so that a batch whose kernels are still reading
   // the old arrays (pipelined submit) is not disturbed; the old arrays are appended to `retired`.
-  void merge(std::vector<std::pair<int32_t *, uint32_t>> &retired);
+  bool merge(std::vector<std::pair<int32_t *, uint32_t>> &retired);  // false: pinned allocation failed
   void recycle(std::vector<std::pair<int32_t *, uint32_t>> &retired);  // once their batch has completed
   void clear_batch();
 
