@@ -186,6 +186,7 @@ __device__ __forceinline__ bool is_device(const MatchArgs &A, const int32_t *p) 
 // warp keeps 2 KB in flight: a zero-copy list crosses PCIe at link speed
 // instead of one dependent 32 B sector per binary-search step.
 __device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
+  __syncwarp();  // every lane is done reading what this buffer held before (WAR across lanes)
   const uint32_t n4 = (n + 3) >> 2;
   const int4 *s4 = reinterpret_cast<const int4 *>(src);
   int4 *d4 = reinterpret_cast<int4 *>(dst);
@@ -363,6 +364,7 @@ constexpr int kBmLog2 = GCSM_BM_INTS > 0 ? 5 + __builtin_ctz(GCSM_BM_INTS) : 5;
 __device__ __forceinline__ uint32_t bm_hash(int32_t v) { return ((uint32_t)v * 2654435761u) >> (32 - kBmLog2); }
 
 __device__ __forceinline__ void bm_build(uint32_t *bm, const int32_t *P, uint32_t n, int lane) {
+  __syncwarp();
   for (uint32_t i = lane; i < (uint32_t)GCSM_BM_INTS; i += 32) bm[i] = 0;
   __syncwarp();
   for (uint32_t i = lane; i < n; i += 32) {
