@@ -70,8 +70,10 @@ enum {
 
 /* Option flags */
 enum {
-  GCSM_FLAG_LOCAL_COUNTS = 1u /* world > 1 without NCCL: return this rank's shard counts
-                                 (single-GPU "emulated world" used by the parity tests) */
+  GCSM_FLAG_LOCAL_COUNTS = 1u, /* world > 1 without NCCL: return this rank's shard counts
+                                  (single-GPU "emulated world" used by the parity tests) */
+  GCSM_FLAG_NO_SYMMETRY = 2u   /* count mode walks every embedding instead of one per Aut_L(Q) orbit
+                                  (symmetry breaking is on by default; list mode never uses it) */
 };
 
 typedef struct {
@@ -226,6 +228,14 @@ gcsm_status gcsm_measure_host_link(int32_t device, uint64_t bytes, double *zero_
  * 0 stable, 1 old N, 2 new N'). */
 gcsm_status gcsm_plan_inspect(int32_t k, int32_t m, const int32_t *qedges, const int32_t *order, int32_t *out_seed,
                               int32_t *out_order, int32_t *out_nb, int32_t *out_bq, int32_t *out_view);
+
+/* Pure host, no device: the symmetry-breaking restrictions the library uses for a query in count mode
+ * (Grochow-Kellis on Aut_L(Q), user order as the vertex order): pairs (u, w) meaning f(u) < f(w); exactly one
+ * embedding per Aut_L orbit satisfies all of them. out_pairs[2*cap]; *n_out = the number of pairs (ETRUNC if
+ * > cap); *aut = |Aut_L(Q)|. */
+gcsm_status gcsm_query_restrictions(int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                                    const int32_t *order, int32_t *out_pairs, int32_t cap, int32_t *n_out,
+                                    uint64_t *aut);
 
 /* Pure host, no device: the shard of each unit for world ranks (LPT on the
  * cost proxy cost[i], ties by index): out_rank[n_units]. */

@@ -24,6 +24,7 @@ __all__ = ["Gcsm", "GcsmError", "plan_inspect", "shard", "nccl_unique_id", "meas
 
 CACHE_POLICIES = {"estimator": 0, "degree": 1, "none": 2}
 FLAG_LOCAL_COUNTS = 1
+FLAG_NO_SYMMETRY = 2
 
 
 class GcsmError(RuntimeError):
@@ -56,7 +57,7 @@ class Gcsm:
     """One GCSM context (one GPU, one process). See include/gcsm.h for the semantics."""
 
     def __init__(self, n, row_ptr, col, labels=None, *, device=-1, rank=0, world=1, nccl_id=None, seed=0x6C53,
-                 host_threads=0, cache_policy="estimator", walks_override=0, local_counts=False):
+                 host_threads=0, cache_policy="estimator", walks_override=0, local_counts=False, symmetry=True):
         lib = _lib.load()
         self._lib = lib
         opt = Options()
@@ -70,7 +71,7 @@ class Gcsm:
         opt.host_threads = host_threads
         opt.cache_policy = CACHE_POLICIES[cache_policy] if isinstance(cache_policy, str) else int(cache_policy)
         opt.walks_override = walks_override
-        opt.flags = FLAG_LOCAL_COUNTS if local_counts else 0
+        opt.flags = (FLAG_LOCAL_COUNTS if local_counts else 0) | (0 if symmetry else FLAG_NO_SYMMETRY)
         self.n = int(n)
         self._rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
         self._col = np.ascontiguousarray(col, dtype=np.int32)
@@ -192,6 +193,19 @@ def plan_inspect(k, qedges, order=None):
         raise GcsmError(s, "bad query")
     return dict(seed=seed.reshape(m, 2), order=order_out.reshape(m, k), nb=nb.reshape(m, k), bq=bq.reshape(m, k, 8),
                 view=view.reshape(2, m, k, 8))
+
+
+def query_restrictions(k, qedges, qlabels=None, order=None):
+    """(pairs [(u, w): f(u) < f(w)], |Aut_L|) of the library's symmetry breaking (pure host)."""
+    qe = _i32(qedges).reshape(-1, 2)
+    out = np.zeros(2 * 64, np.int32)
+    n = ctypes.c_int32()
+    aut = ctypes.c_uint64()
+    s = _lib.load().gcsm_query_restrictions(k, len(qe), _ptr(qe), _ptr(_i32(qlabels)), _ptr(_i32(order)), _ptr(out),
+                                            64, ctypes.byref(n), ctypes.byref(aut))
+    if s:
+        raise GcsmError(s, "bad query")
+    return [tuple(out[2 * i:2 * i + 2].tolist()) for i in range(n.value)], aut.value
 
 
 def shard(cost, world):

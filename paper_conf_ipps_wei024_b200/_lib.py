@@ -19,7 +19,8 @@ STATUS = {0: "GCSM_OK", 1: "GCSM_EINVAL", 2: "GCSM_ENOMEM", 3: "GCSM_EDEVICE", 4
 SYMBOLS = ["gcsm_default_options", "gcsm_create", "gcsm_set_query", "gcsm_set_cache_budget", "gcsm_apply_batch",
            "gcsm_apply_batch_list", "gcsm_submit_batch", "gcsm_wait_batch", "gcsm_get_stats", "gcsm_query_automorphisms", "gcsm_last_error", "gcsm_destroy",
            "gcsm_nccl_unique_id", "gcsm_get_stream", "gcsm_export_csr", "gcsm_get_estimates", "gcsm_get_cached",
-           "gcsm_plan_inspect", "gcsm_shard", "gcsm_measure_host_link"]
+           "gcsm_plan_inspect", "gcsm_query_restrictions", "gcsm_shard",
+           "gcsm_measure_host_link"]
 
 
 class Options(ctypes.Structure):
@@ -72,6 +73,7 @@ def load():
         "gcsm_get_cached": (st, [P, P, U64, ctypes.POINTER(U64)]),
         "gcsm_plan_inspect": (st, [I32, I32, P, P, P, P, P, P, P]),
         "gcsm_shard": (st, [I64, P, I32, P]),
+        "gcsm_query_restrictions": (st, [I32, I32, P, P, P, P, I32, P, ctypes.POINTER(U64)]),
         "gcsm_measure_host_link": (st, [I32, U64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double),
                                         ctypes.POINTER(ctypes.c_double)]),
     }

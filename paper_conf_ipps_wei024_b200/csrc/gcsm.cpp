@@ -60,7 +60,8 @@ struct gcsm_ctx {
   std::string err;
   bool poisoned = false;
   HostStore store;
-  QueryPlan qp;
+  QueryPlan qp;   // plans without restrictions
+  QueryPlan qps;  // plans with the symmetry-breaking restrictions of Aut_L(Q)
   bool has_query = false;
   uint64_t budget = 0;
   cudaStream_t stream = nullptr;
@@ -80,6 +81,7 @@ struct gcsm_ctx {
     std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
     size_t nev = 0;
     bool inflight = false;
+    uint64_t aut_mul = 1;  // canonical-embedding counts x |Aut_L| (symmetry breaking)
     gcsm_stats st{};
     double host_ms = 0;
     // list mode
@@ -94,7 +96,8 @@ struct gcsm_ctx {
 
   // device buffers
   VDesc *d_vdesc = nullptr;
-  DevPlan *d_plans = nullptr;
+  DevPlan *d_plans = nullptr;   // the query's plans (estimator, list mode)
+  DevPlan *d_splans = nullptr;  // the same with symmetry-breaking restrictions (count mode)
   uint16_t *d_lab = nullptr;
   DRec *d_drec = nullptr; size_t drec_cap = 0;
   int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
@@ -154,7 +157,7 @@ struct gcsm_ctx {
 gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
-  void *dev[] = {d_vdesc, d_plans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
+  void *dev[] = {d_vdesc, d_plans, d_splans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (void *p : dev)
     if (p) cudaFree(p);
@@ -237,6 +240,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_plans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_splans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)n + 2047) / 2048 + 1)) != cudaSuccess)
     return bail(GCSM_ENOMEM);
@@ -279,15 +283,19 @@ gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *q
   if (ctx->poisoned) return GCSM_ESTATE;
   if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "set_query with a batch in flight");
   QueryPlan qp;
+  QueryPlan qps;
   std::string e = build_plan(k, m, qedges, qlabels, order, qp);
+  if (e.empty()) e = build_plan(k, m, qedges, qlabels, order, qps, !(ctx->opt.flags & GCSM_FLAG_NO_SYMMETRY));
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
   if (qp.labelled && !ctx->d_lab) {  // unlabelled graph: every data label is 0 (R5)
     CK(cudaMalloc(&ctx->d_lab, 2 * (size_t)ctx->store.n));
     CK(cudaMemset(ctx->d_lab, 0, 2 * (size_t)ctx->store.n));
   }
   CK(upload_plans(ctx->d_plans, qp.plans.data(), (int)qp.plans.size(), ctx->stream));
+  CK(upload_plans(ctx->d_splans, qps.plans.data(), (int)qps.plans.size(), ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
   ctx->qp = qp;
+  ctx->qps = qps;
   ctx->has_query = true;
   ctx->err.clear();
   return GCSM_OK;
@@ -482,6 +490,20 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   }
   st.ms_estimate = t2.ms();
   tr.mark("score");
+  // symmetry breaking (count mode): the kernels walk only the canonical embedding of every Aut_L orbit and the
+  // counts are scaled by |Aut_L| (Emb(G') \ Emb(G) is a union of orbits); the estimator above samples the full
+  // execution trees of the paper. Seeds violating a restriction between the two seed endpoints are dropped here.
+  const bool sym = !listing && ctx->qps.symmetry;
+  const QueryPlan &QK = sym ? ctx->qps : Q;
+  if (sym) {
+    size_t w = 0;
+    for (size_t i = 0; i < units.size(); ++i) {
+      const int rel = QK.plans[units[i].plan].seed_rel;
+      if (rel == 0 || (rel == 1 ? units[i].a < units[i].b : units[i].a > units[i].b)) units[w++] = units[i];
+    }
+    units.resize(w);
+  }
+  const int64_t gnu = (int64_t)units.size();
 
   // ---- (3) pack the cache + descriptors --------------------------------------------------
   Timer t3;
@@ -604,21 +626,21 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const size_t nU = S.U.size();
   const size_t nd = S.ins_val.size() + S.del_val.size();
   if (!host_ensure(sl.h_drec, sl.h_drec_cap, nU) || !host_ensure(sl.h_dlist, sl.h_dlist_cap, nd) ||
-      !host_ensure(sl.h_units, sl.h_units_cap, (size_t)nu))
+      !host_ensure(sl.h_units, sl.h_units_cap, (size_t)gnu))
     return ctx->fail(GCSM_ENOMEM, "pinned staging");
   for (size_t i = 0; i < nU; ++i)
     sl.h_drec[i] = DRec{S.ins_off[i], S.ins_off[i + 1] - S.ins_off[i], (uint32_t)S.ins_val.size() + S.del_off[i],
                           S.del_off[i + 1] - S.del_off[i]};
   std::memcpy(sl.h_dlist, S.ins_val.data(), S.ins_val.size() * 4);
   std::memcpy(sl.h_dlist + S.ins_val.size(), S.del_val.data(), S.del_val.size() * 4);
-  std::memcpy(sl.h_units, units.data(), sizeof(Unit) * (size_t)nu);
+  std::memcpy(sl.h_units, units.data(), sizeof(Unit) * (size_t)gnu);
   st.ms_pack = t3.ms();
   tr.mark("staging");
 
   cudaStream_t s = ctx->stream;
   if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
       !dev_ensure(ctx->d_drec, ctx->drec_cap, nU) || !dev_ensure(ctx->d_dlist, ctx->dlist_cap, nd) ||
-      !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)nu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)nu))
+      !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)gnu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)gnu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
   CK(cudaEventRecord(sl.ev_c0, s));
   const uint64_t retained_bytes = used - new_bytes;
@@ -645,10 +667,10 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   uint64_t launches = dirty.empty() ? 0 : 1;
   if (nU) CK(cudaMemcpyAsync(ctx->d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
   if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
-  if (nu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)nu, cudaMemcpyHostToDevice, s));
+  if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(sl.ev_c1, s));
   st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
-                 4 * nd + sizeof(Unit) * (size_t)nu;
+                 4 * nd + sizeof(Unit) * (size_t)gnu;
 
   // ---- (4) matching kernels --------------------------------------------------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
@@ -661,8 +683,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   int64_t f2_need = 0;
   if (k >= 4) {
     int64_t start = 0, acc = 0;
-    for (int64_t i = 0; i < nu; ++i) {
-      const DevPlan &P = Q.plans[units[i].plan];
+    for (int64_t i = 0; i < gnu; ++i) {
+      const DevPlan &P = QK.plans[units[i].plan];
       const LevelPlan &L2 = P.lv[2];
       const int32_t f[2] = {units[i].a, units[i].b};
       int64_t b = INT64_MAX;
@@ -675,13 +697,13 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       }
       acc += b;
     }
-    chunks.push_back({start, nu});
+    chunks.push_back({start, gnu});
     f2_need = std::max(f2_need, acc);
     if (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)) ||
         !dev_ensure(ctx->d_group, ctx->group_cap, (size_t)std::max<int64_t>(f2_need, 1)))
       return ctx->fail(GCSM_ENOMEM, "frontier");
   } else {
-    chunks.push_back({0, nu});
+    chunks.push_back({0, gnu});
   }
   // list mode buffers
   int32_t *d_tadd = nullptr, *d_trem = nullptr;
@@ -693,7 +715,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   }
   CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N, s));
   MatchArgs A{};
-  A.plans = ctx->d_plans;
+  A.plans = sym ? ctx->d_splans : ctx->d_plans;
   A.vdesc = ctx->d_vdesc;
   A.lab = ctx->d_lab;
   A.drec = ctx->d_drec;
@@ -778,6 +800,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   sl.d_trem = d_trem;
   sl.add_cap = add_cap;
   sl.rem_cap = rem_cap;
+  sl.aut_mul = sym ? QK.automorphisms : 1;
   tr.mark("enqueue");
 
   // ---- (5) reorganise the host lists. P:302 runs it after matching so the kernel reads consistent data: here
@@ -832,8 +855,8 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.ms_extend += b;
   }
   const unsigned long long *h = sl.h_cnt;
-  st.added = h[CNT_ADDED];
-  st.removed = h[CNT_REMOVED];
+  st.added = h[CNT_ADDED] * sl.aut_mul;
+  st.removed = h[CNT_REMOVED] * sl.aut_mul;
   st.hit_bytes_ext = h[CNT_ACC_EXT + 0];
   st.miss_bytes_ext = h[CNT_ACC_EXT + 1];
   st.delta_bytes_ext = h[CNT_ACC_EXT + 2];
@@ -964,6 +987,21 @@ gcsm_status gcsm_plan_inspect(int32_t k, int32_t m, const int32_t *qedges, const
     }
   }
   return GCSM_OK;
+}
+
+gcsm_status gcsm_query_restrictions(int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                                    const int32_t *order, int32_t *out_pairs, int32_t cap, int32_t *n_out,
+                                    uint64_t *aut) {
+  QueryPlan qp;
+  if (!build_plan(k, m, qedges, qlabels, order, qp, true).empty()) return GCSM_EINVAL;
+  const int32_t n = (int32_t)qp.restrictions.size();
+  if (n_out) *n_out = n;
+  if (aut) *aut = qp.automorphisms;
+  for (int32_t i = 0; i < n && i < cap && out_pairs; ++i) {
+    out_pairs[2 * i] = qp.restrictions[i].first;
+    out_pairs[2 * i + 1] = qp.restrictions[i].second;
+  }
+  return n > cap ? GCSM_ETRUNC : GCSM_OK;
 }
 
 gcsm_status gcsm_shard(int64_t n_units, const uint64_t *cost, int32_t world, int32_t *out_rank) {

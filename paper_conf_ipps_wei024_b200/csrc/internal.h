@@ -56,6 +56,8 @@ struct LevelPlan {
   int8_t rest[7];      // indices into bpos/bview
   int8_t ninj;         // matched positions to exclude (not backward neighbours)
   int8_t inj[7];
+  int8_t nlo, lo[7];   // symmetry breaking: f(order[p]) > f(position lo[i])
+  int8_t nhi, hi[7];   //                    f(order[p]) < f(position hi[i])
   int32_t label;       // required data label of order[p], -1 = any
 };
 
@@ -64,6 +66,7 @@ struct DevPlan {
   int32_t kind;              // 0 "+", 1 "-"
   int8_t order[GCSM_MAXK];   // query vertex at each term position
   int32_t label0, label1;    // labels of the seed endpoints (-1 = any)
+  int32_t seed_rel;          // symmetry breaking on the seed: 0 none, 1 f(order[0]) < f(order[1]), 2 >
   LevelPlan lv[GCSM_MAXK];   // valid for positions 2..k-1
 };
 
@@ -150,12 +153,15 @@ struct QueryPlan {
   int qlab[GCSM_MAXK];          // -1 = any
   bool labelled = false;
   uint64_t automorphisms = 0;
+  bool symmetry = false;                        // restrictions below are active in `plans`
+  std::vector<std::pair<int, int>> restrictions;  // (u, w): f(u) < f(w) selects one embedding per Aut_L orbit
   std::vector<DevPlan> plans;   // 2*m: index 2*term + kind
 };
 
 // Returns "" on success, else the EINVAL reason.
+// symmetry: add the symmetry-breaking restrictions of Aut_L(Q) (counts then scale by |Aut_L|)
 std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabels, const int32_t *order,
-                       QueryPlan &out);
+                       QueryPlan &out, bool symmetry = false);
 
 // ------------------------------------------------------------ RNG (estimator.cpp)
 uint64_t rng_mix(uint64_t z);

@@ -145,7 +145,7 @@ __device__ __forceinline__ bool contains(const LRef &L, int32_t v) {
 template <bool MATERIALIZE>
 __device__ GCSM_COLD uint32_t warp_isect(const MatchArgs &A, const int32_t *dset, uint32_t dn, const LRef *L,
                                                int nl, int drv, const int32_t *excl, int nexcl, int label,
-                                               int32_t *out, int lane) {
+                                               int32_t *out, int lane, int32_t vlo = INT_MIN, int32_t vhi = INT_MAX) {
   const int32_t *s0, *s1;
   uint32_t n0, n1;
   if (dset) {
@@ -160,6 +160,7 @@ __device__ GCSM_COLD uint32_t warp_isect(const MatchArgs &A, const int32_t *dset
     bool ok = i < total;
     int32_t v = 0;
     if (ok) v = i < n0 ? s0[i] : s1[i - n0];
+    ok = ok && v > vlo && v < vhi;  // symmetry-breaking range
     for (int e = 0; e < nexcl; ++e) ok = ok && v != excl[e];
     if (ok && label >= 0) ok = A.lab[v] == (uint16_t)label;
     for (int p = 0; p < nl; ++p)
@@ -315,11 +316,11 @@ __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, c
 
 // lane-parallel count of x[0..nx) present in the sorted list y (label-filtered)
 __device__ GCSM_COLD uint32_t probe_count(const int32_t *x, uint32_t nx, const int32_t *y, uint32_t ny, int label,
-                                                const uint16_t *lab, int lane) {
+                                                const uint16_t *lab, int lane, int32_t vlo, int32_t vhi) {
   uint32_t cnt = 0;
   for (uint32_t i = lane; i < nx; i += 32) {
     const int32_t v = x[i];
-    if (bsearch_has(y, ny, v) && (label < 0 || lab[v] == (uint16_t)label)) ++cnt;
+    if (v > vlo && v < vhi && bsearch_has(y, ny, v) && (label < 0 || lab[v] == (uint16_t)label)) ++cnt;
   }
 #pragma unroll
   for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
@@ -336,7 +337,8 @@ __device__ __forceinline__ uint32_t ilog2(uint32_t x) { return 31u - __clz(x | 1
 // memory and it is cheaper than per-lane binary search; the tiny delta runs are probed; excluded (matched,
 // non-adjacent) vertices that lie in the intersection are subtracted. Returns false if not applicable.
 __device__ __forceinline__ bool count2(const MatchArgs &A, const LRef *L, int drv, const int32_t *excl, int nexcl,
-                                       int label, int lane, uint32_t *out) {
+                                       int label, int lane, uint32_t *out, int32_t vlo = INT_MIN,
+                                       int32_t vhi = INT_MAX) {
   const LRef &X = L[drv], &Y = L[1 - drv];
   if (X.ml < 8 || Y.ml < 8 || !X.dev || !Y.dev) return false;
   const uint32_t d = X.ml + X.xl, big = Y.ml + Y.xl;
@@ -344,12 +346,12 @@ __device__ __forceinline__ bool count2(const MatchArgs &A, const LRef *L, int dr
   const uint32_t mg_cost = 10 * ilog2(min(X.ml, Y.ml)) + 7 * ((X.ml + Y.ml + 31) >> 5) + 30;
   if (mg_cost >= bs_cost) return false;
   uint32_t c = merge_count(X.m, X.ml, Y.m, Y.ml, label, A.lab, lane);
-  if (X.xl) c += probe_count(X.x, X.xl, Y.m, Y.ml, label, A.lab, lane);
-  if (Y.xl) c += probe_count(Y.x, Y.xl, X.m, X.ml, label, A.lab, lane);
-  if (X.xl && Y.xl) c += probe_count(X.x, X.xl, Y.x, Y.xl, label, A.lab, lane);
+  if (X.xl) c += probe_count(X.x, X.xl, Y.m, Y.ml, label, A.lab, lane, vlo, vhi);
+  if (Y.xl) c += probe_count(Y.x, Y.xl, X.m, X.ml, label, A.lab, lane, vlo, vhi);
+  if (X.xl && Y.xl) c += probe_count(X.x, X.xl, Y.x, Y.xl, label, A.lab, lane, vlo, vhi);
   for (int e = 0; e < nexcl; ++e) {
     const int32_t v = excl[e];
-    if ((label < 0 || A.lab[v] == (uint16_t)label) && contains(X, v) && contains(Y, v)) --c;
+    if (v > vlo && v < vhi && (label < 0 || A.lab[v] == (uint16_t)label) && contains(X, v) && contains(Y, v)) --c;
   }
   *out = c;
   return true;
@@ -375,11 +377,13 @@ __device__ __forceinline__ void bm_build(uint32_t *bm, const int32_t *P, uint32_
 }
 
 __device__ __forceinline__ uint32_t bm_count(const MatchArgs &A, const uint32_t *bm, const LRef &X, const LRef &P,
-                                             const int32_t *excl, int nexcl, int label, int lane) {
+                                             const int32_t *excl, int nexcl, int label, int lane, int32_t vlo,
+                                             int32_t vhi) {
   uint32_t cnt = 0;
   auto visit = [&](const int32_t *seg, uint32_t n) {
     for (uint32_t i = lane; i < n; i += 32) {
       const int32_t v = seg[i];
+      if (v <= vlo || v >= vhi) continue;
       const uint32_t h = bm_hash(v);
       bool in = false;
       if ((bm[h >> 5] >> (h & 31)) & 1u) in = bsearch_has(P.m, P.ml, v);
@@ -396,6 +400,38 @@ __device__ __forceinline__ uint32_t bm_count(const MatchArgs &A, const uint32_t 
 #pragma unroll
   for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
   return cnt;
+}
+
+// Symmetry-breaking range of position p: vlo < candidate < vhi (counts scale by |Aut_L|).
+__device__ __forceinline__ void range_of(const LevelPlan &Lp, const int32_t *f, int32_t *vlo, int32_t *vhi) {
+  int32_t lo = INT_MIN, hi = INT_MAX;
+  for (int i = 0; i < Lp.nlo; ++i) lo = max(lo, f[Lp.lo[i]]);
+  for (int i = 0; i < Lp.nhi; ++i) hi = min(hi, f[Lp.hi[i]]);
+  *vlo = lo;
+  *vhi = hi;
+}
+
+__device__ __forceinline__ uint32_t lower_idx(const int32_t *a, uint32_t n, int32_t v) {
+  uint32_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (a[mid] < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// Narrow the device-resident main runs to the range (vlo, vhi): the sorted lists lose the elements no
+// candidate may take, so every intersection below reads fewer of them.
+__device__ __forceinline__ void trim_lists(LRef *L, int nl, int32_t vlo, int32_t vhi) {
+  if (vlo == INT_MIN && vhi == INT_MAX) return;
+  for (int p = 0; p < nl; ++p) {
+    if (!L[p].dev || L[p].ml == 0) continue;
+    const uint32_t b = vlo == INT_MIN ? 0 : lower_idx(L[p].m, L[p].ml, vlo + 1);
+    const uint32_t e = vhi == INT_MAX ? L[p].ml : lower_idx(L[p].m, L[p].ml, vhi);
+    L[p].m += b;
+    L[p].ml = e > b ? e - b : 0;
+  }
 }
 
 // Lists of position p for the current partial match f (positions 0..p-1).
@@ -490,18 +526,21 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
     int drv;
     const int nl = gather_lists(A, L2, f, L, &drv, acc);
     stage_lists(A, L, nl, drv, false, 0, sm, kSmemInts, gstage, lane, acc);
+    int32_t vlo, vhi;
+    range_of(L2, f, &vlo, &vhi);
+    trim_lists(L, nl, vlo, vhi);
     int32_t excl[2];
     int nex = 0;
     for (int i = 0; i < L2.ninj; ++i) excl[nex++] = f[L2.inj[i]];
     if (A.k == 3 && !LIST) {
       uint32_t c;
-      if (nl != 2 || !count2(A, L, drv, excl, nex, L2.label, lane, &c))
-        c = warp_isect<false>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, nullptr, lane);
+      if (nl != 2 || !count2(A, L, drv, excl, nex, L2.label, lane, &c, vlo, vhi))
+        c = warp_isect<false>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, nullptr, lane, vlo, vhi);
       if (P.kind) acc.rem += c;
       else acc.add += c;
       continue;
     }
-    const uint32_t c = warp_isect<true>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, buf, lane);
+    const uint32_t c = warp_isect<true>(A, nullptr, 0, L, nl, drv, excl, nex, L2.label, buf, lane, vlo, vhi);
     __syncwarp();
     if (A.k == 3) {  // LIST
       if (P.kind) acc.rem += c;
@@ -701,6 +740,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
         const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
         uint32_t c = 0;
+        int32_t vlo, vhi;
+        range_of(Lp, f, &vlo, &vhi);
         // last level, two lists, one of them the run's x2 list in the bitmap: stream the other one
         bool merged = false;
         if (GCSM_BM_INTS > 0 && !LIST && p == k - 1 && !dset && nl == 2 && pin.bm_v >= 0 && !task) {
@@ -712,34 +753,32 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
             const uint32_t d = min(nx, np), big = max(nx, np);
             const uint32_t bs_cost = ((d + 31) >> 5) * (7 * ilog2(big) + 12);
             if (bm_cost <= bs_cost && X.dev) {
-              c = bm_count(A, bm, X, L[pi], excl, nex, Lp.label, lane);
+              c = bm_count(A, bm, X, L[pi], excl, nex, Lp.label, lane, vlo, vhi);
               merged = true;
             }
           }
         }
-        if (!merged)
-          merged = GCSM_PRESTAGE_MERGE && !LIST && p == k - 1 && !dset && nl == 2 &&
-                   count2(A, L, drv, excl, nex, Lp.label, lane, &c);
         if (!merged) stage_lists(A, L, nl, drv, dset != nullptr, dn, sm + pin_sm, kSlice - pin_sm, gstage, lane, acc);
+        if (!merged) trim_lists(L, nl, vlo, vhi);
         if (merged) {
           if (P.kind) acc.rem += c;
           else acc.add += c;
           descend = false;
         } else if (p == k - 1) {
           if (LIST) {
-            c = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, lastbuf, lane);
+            c = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, lastbuf, lane, vlo, vhi);
             __syncwarp();
             emit_tuples(A, P, f, P.kind, lastbuf, c, lane);
             __syncwarp();
-          } else if (dset || nl != 2 || !count2(A, L, drv, excl, nex, Lp.label, lane, &c)) {
-            c = warp_isect<false>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, nullptr, lane);
+          } else if (dset || nl != 2 || !count2(A, L, drv, excl, nex, Lp.label, lane, &c, vlo, vhi)) {
+            c = warp_isect<false>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, nullptr, lane, vlo, vhi);
           }
           if (P.kind) acc.rem += c;
           else acc.add += c;
           descend = false;
         } else {
           int32_t *out = stack + (int64_t)(p - 3) * A.dcap;
-          sz[p] = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, out, lane);
+          sz[p] = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, out, lane, vlo, vhi);
           __syncwarp();
           set[p] = out;
           it[p] = 0;

@@ -28,7 +28,7 @@ static View view_for(int j, int term, int kind) {
 }
 
 std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabels, const int32_t *order,
-                       QueryPlan &out) {
+                       QueryPlan &out, bool symmetry) {
   if (k < 2 || k > GCSM_MAXK) return "query size k must be in [2, 8]";
   if (m < 1 || m > k * (k - 1) / 2) return "query edge count m out of range";
   if (!qedges) return "qedges is NULL";
@@ -84,19 +84,38 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
     eidx[e[i].first][e[i].second] = eidx[e[i].second][e[i].first] = i;
   }
   // automorphisms (label preserving)
+  std::vector<std::vector<int>> auts;
   {
     int p[GCSM_MAXK];
     std::iota(p, p + k, 0);
-    uint64_t cnt = 0;
     do {
       bool ok = true;
       for (int u = 0; u < k && ok; ++u)
         if (q.qlab[p[u]] != q.qlab[u]) ok = false;
       for (int i = 0; i < m && ok; ++i)
         if (!adj[p[q.qe[i][0]]][p[q.qe[i][1]]]) ok = false;
-      cnt += ok;
+      if (ok) auts.emplace_back(p, p + k);
     } while (std::next_permutation(p, p + k));
-    q.automorphisms = cnt;
+    q.automorphisms = auts.size();
+  }
+  // Symmetry breaking (Grochow & Kellis): walk the user order; for the first vertex v with a non-trivial orbit
+  // under the current group require f(v) < f(w) for the rest of its orbit, then keep only v's stabiliser.
+  // Exactly one embedding of every Aut_L orbit {f o s} satisfies all restrictions (pinned by brute force in
+  // tests/test_abi.py), and Emb(G') \ Emb(G) is a union of orbits, so counts = |Aut_L| x restricted counts.
+  q.symmetry = symmetry && auts.size() > 1;
+  if (q.symmetry) {
+    std::vector<std::vector<int>> G = auts;
+    for (int r = 0; r < k && G.size() > 1; ++r) {
+      const int v = uo[r];
+      bool seen[GCSM_MAXK] = {};
+      for (const auto &p : G) seen[p[v]] = true;
+      for (int w = 0; w < k; ++w)
+        if (seen[w] && w != v) q.restrictions.push_back({v, w});
+      std::vector<std::vector<int>> H;
+      for (const auto &p : G)
+        if (p[v] == v) H.push_back(p);
+      G.swap(H);
+    }
   }
   q.plans.resize(2 * m);
   for (int term = 0; term < m; ++term) {
@@ -123,6 +142,21 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
       for (int s = 0; s < k; ++s) P.order[s] = (int8_t)ord[s];
       P.label0 = q.qlab[ord[0]];
       P.label1 = q.qlab[ord[1]];
+      int posof[GCSM_MAXK];
+      for (int s2 = 0; s2 < k; ++s2) posof[ord[s2]] = s2;
+      P.seed_rel = 0;
+      for (const auto &rw : q.restrictions) {
+        const int pu = posof[rw.first], pw = posof[rw.second];  // f(order[pu]) < f(order[pw])
+        if (std::max(pu, pw) == 1) {
+          P.seed_rel = pu == 0 ? 1 : 2;
+        } else if (pw > pu) {  // placed at pw: must exceed f at pu
+          LevelPlan &L = P.lv[pw];
+          L.lo[L.nlo++] = (int8_t)pu;
+        } else {  // placed at pu: must stay below f at pw
+          LevelPlan &L = P.lv[pu];
+          L.hi[L.nhi++] = (int8_t)pw;
+        }
+      }
       for (int p = 2; p < k; ++p) {
         LevelPlan &L = P.lv[p];
         L.label = q.qlab[ord[p]];
@@ -141,6 +175,19 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
         for (int pp = p - 1; pp >= 2 && L.reuse < 0; --pp) {
           const LevelPlan &E = P.lv[pp];
           if (E.label != L.label) continue;
+          // the earlier set was filtered by its own symmetry restrictions: they must bind here too
+          bool implied = true;
+          for (int a = 0; a < E.nlo && implied; ++a) {
+            bool f = false;
+            for (int b = 0; b < L.nlo; ++b) f |= E.lo[a] == L.lo[b];
+            implied = f;
+          }
+          for (int a = 0; a < E.nhi && implied; ++a) {
+            bool f = false;
+            for (int b = 0; b < L.nhi; ++b) f |= E.hi[a] == L.hi[b];
+            implied = f;
+          }
+          if (!implied) continue;
           bool sub = true;
           for (int a = 0; a < E.nb && sub; ++a) {
             bool found = false;

@@ -96,3 +96,28 @@ def test_no_cpu_fallback(pkg):
     with pytest.raises(pkg.GcsmError) as ei:
         pkg.Gcsm(w.n, w.row_ptr, w.col)
     assert ei.value.name in ("GCSM_EDEVICE", "GCSM_ENOMEM")
+
+
+@pytest.mark.parametrize("name", ["edge", "wedge", "triangle", "c4", "diamond", "k4", "star3", "path4", "house5u",
+                                  "house5", "bowtie5", "k5e", "k5", "prism6", "k4tri6"])
+def test_symmetry_breaking_restrictions_brute_force(pkg, name):
+    """Exactly one embedding per Aut_L orbit satisfies the library's restrictions:
+    |{f in Emb : f(u) < f(w) for all (u, w)}| * |Aut_L| = |Emb|, by brute force on random small graphs."""
+    k, qe, ql = gi.query(name)
+    pairs, aut = pkg.query_restrictions(k, qe, ql)
+    assert aut == oracle.automorphisms(k, qe, ql)
+    rng = np.random.default_rng(len(name))
+    for trial in range(3):
+        n = 7 if k <= 5 else 8
+        edges = gi.random_graph(n, 0.6, 1000 * trial + k)
+        labels = rng.integers(0, 3, n).astype(np.int32) if ql is not None else None
+        emb = oracle.brute_embeddings(n, edges, labels, k, qe.tolist(), ql)
+        canon = [f for f in emb if all(f[u] < f[w] for u, w in pairs)]
+        assert len(canon) * aut == len(emb)
+    # a random user order changes the restrictions, not their property
+    order = rng.permutation(k).astype(np.int32)
+    pairs2, aut2 = pkg.query_restrictions(k, qe, ql, order)
+    emb = oracle.brute_embeddings(7, gi.random_graph(7, 0.7, 5), None if ql is None else np.zeros(7, np.int32),
+                                  k, qe.tolist(), None if ql is None else np.zeros(k, np.int32))
+    if ql is None:
+        assert len([f for f in emb if all(f[u] < f[w] for u, w in pairs2)]) * aut2 == len(emb)

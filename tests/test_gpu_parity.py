@@ -414,3 +414,14 @@ def test_nccl_single_rank_allreduce(G):
     got, st, _ = lib_run(G, w.n, w.row_ptr, w.col, None, "diamond", w.batches, 0.1, nccl_id=G.nccl_unique_id())
     assert got == want
     assert st["ms_allreduce"] > 0
+
+
+@pytest.mark.parametrize("name", ["triangle", "k4", "c4", "diamond", "house5u", "prism6", "k4tri6"])
+def test_symmetry_breaking_on_off(G, name):
+    """Count mode walks one embedding per Aut_L orbit and scales by |Aut_L| (default); both settings equal the
+    oracle on a mixed stream."""
+    w = gi.make_workload("C2", scale=12, n_edges=40_000, batch=256, n_batches=3)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    on, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.1, symmetry=True)
+    off, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.1, symmetry=False)
+    assert on == want and off == want
