@@ -382,37 +382,46 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   st.n_ins = S.I.size();
   st.n_del = S.D.size();
   st.dropped = S.dropped;
+  // level-1 units: (term, kind, changed edge, orientation) slots enumerated in parallel, then compacted in slot
+  // order (deterministic); the cost proxy of a unit is the list lengths its first level reads
   std::vector<Unit> units;
   std::vector<uint64_t> cost;
-  units.reserve((S.I.size() + S.D.size()) * 2 * Q.m);
-  for (int term = 0; term < Q.m; ++term)
-    for (int kind = 0; kind < 2; ++kind) {
-      const DevPlan &P = Q.plans[2 * term + kind];
-      const std::vector<uint64_t> &E = kind ? S.D : S.I;
-      for (uint64_t key : E) {
+  {
+    const int64_t ni = (int64_t)S.I.size(), ndl = (int64_t)S.D.size(), per = 2 * (ni + ndl);
+    const int64_t slots = (int64_t)Q.m * per;
+    std::vector<Unit> all((size_t)slots);
+    std::vector<uint64_t> ac((size_t)slots, 0);  // 0 = filtered out
+    parallel_for(T, slots, [&](int, int64_t lo, int64_t hi) {
+      for (int64_t sidx = lo; sidx < hi; ++sidx) {
+        const int term = (int)(sidx / per);
+        int64_t r = sidx % per;
+        const int o = (int)(r & 1);
+        r >>= 1;
+        const int kind = r < ni ? 0 : 1;
+        const uint64_t key = kind ? S.D[r - ni] : S.I[r];
+        const DevPlan &P = Q.plans[2 * term + kind];
         const int32_t x = (int32_t)(key >> 32), y = (int32_t)(key & 0xffffffffu);
-        for (int o = 0; o < 2; ++o) {
-          const int32_t a = o ? y : x, b = o ? x : y;
-          if (P.label0 >= 0 && host_label(S, a) != P.label0) continue;
-          if (P.label1 >= 0 && host_label(S, b) != P.label1) continue;
-          units.push_back(Unit{a, b, 2 * term + kind, 0});
+        const int32_t a = o ? y : x, b = o ? x : y;
+        if (P.label0 >= 0 && host_label(S, a) != P.label0) continue;
+        if (P.label1 >= 0 && host_label(S, b) != P.label1) continue;
+        all[sidx] = Unit{a, b, 2 * term + kind, 0};
+        uint64_t c = 1;
+        if (k > 2) {
+          const LevelPlan &L2 = P.lv[2];
+          const int32_t f[2] = {a, b};
+          for (int bb = 0; bb < L2.nb; ++bb) c += S.view_len(f[L2.bpos[bb]], L2.bview[bb]);
         }
+        ac[sidx] = c;
       }
-    }
-  // cost proxy of a unit: the list lengths its first level reads
-  cost.resize(units.size());
-  parallel_for(T, (int64_t)units.size(), [&](int, int64_t lo, int64_t hi) {
-    for (int64_t i = lo; i < hi; ++i) {
-      const DevPlan &P = Q.plans[units[i].plan];
-      uint64_t c = 1;
-      if (k > 2) {
-        const LevelPlan &L2 = P.lv[2];
-        const int32_t f[2] = {units[i].a, units[i].b};
-        for (int b = 0; b < L2.nb; ++b) c += S.view_len(f[L2.bpos[b]], L2.bview[b]);
+    });
+    units.reserve((size_t)slots);
+    cost.reserve((size_t)slots);
+    for (int64_t sidx = 0; sidx < slots; ++sidx)
+      if (ac[sidx]) {
+        units.push_back(all[sidx]);
+        cost.push_back(ac[sidx]);
       }
-      cost[i] = c;
-    }
-  });
+  }
   if (ctx->opt.world > 1) {
     std::vector<int32_t> rk(units.size());
     shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data());
@@ -519,6 +528,36 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
   ctx->d_cache = ctx->d_cachebuf[tgt];
   if (use_cache && !ranked.empty()) {
+    // Only the head of the ranking can fit the budget: bucket the (positive) scores by their top 16 bits
+    // (monotone in the score), find the bucket where the cumulative list bytes pass the budget, and sort just
+    // the vertices at or above it. The longest-prefix selection (R23) is unchanged: it stops inside that bucket.
+    {
+      std::vector<uint64_t> vb(ranked.size());
+      parallel_for(T, (int64_t)ranked.size(), [&](int, int64_t lo, int64_t hi) {
+        for (int64_t i = lo; i < hi; ++i) vb[i] = (uint64_t)((S.view_len(ranked[i].second, VIEW_S) + 3u) & ~3u) * 4;
+      });
+      auto bucket = [](double x) {
+        uint64_t b;
+        std::memcpy(&b, &x, 8);
+        return (uint32_t)(b >> 48);
+      };
+      std::vector<uint64_t> hb(1u << 16, 0);
+      for (size_t i = 0; i < ranked.size(); ++i)
+        if (ranked[i].first > 0) hb[bucket(ranked[i].first)] += vb[i];
+      uint64_t cum = 0;
+      uint32_t cut = 0;
+      for (int64_t b = (1 << 16) - 1; b >= 0; --b) {
+        cum += hb[b];
+        if (cum > ctx->budget) {
+          cut = (uint32_t)b;
+          break;
+        }
+      }
+      size_t w = 0;
+      for (size_t i = 0; i < ranked.size(); ++i)
+        if (ranked[i].first > 0 && bucket(ranked[i].first) >= cut) ranked[w++] = ranked[i];
+      ranked.resize(w);
+    }
     parallel_sort(
         ranked,
         [](const std::pair<double, int32_t> &x, const std::pair<double, int32_t> &y) {

@@ -175,12 +175,22 @@ std::string HostStore::normalize(int64_t n_ins, const int32_t *ins, int64_t n_de
   I.clear();
   D.clear();
   dropped = 0;
-  for (uint64_t key : ki) {
-    if (has_edge((int32_t)(key >> 32), (int32_t)(key & 0xffffffffu))) ++dropped;
-    else I.push_back(key);
+  // existence checks: random probes into the host lists, in parallel
+  std::vector<uint8_t> ei(ki.size()), ed(kd.size());
+  parallel_for(threads, (int64_t)(ki.size() + kd.size()), [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      const uint64_t key = i < (int64_t)ki.size() ? ki[i] : kd[i - ki.size()];
+      const uint8_t h = has_edge((int32_t)(key >> 32), (int32_t)(key & 0xffffffffu));
+      if (i < (int64_t)ki.size()) ei[i] = h;
+      else ed[i - ki.size()] = h;
+    }
+  });
+  for (size_t i = 0; i < ki.size(); ++i) {
+    if (ei[i]) ++dropped;
+    else I.push_back(ki[i]);
   }
-  for (uint64_t key : kd) {
-    if (has_edge((int32_t)(key >> 32), (int32_t)(key & 0xffffffffu))) D.push_back(key);
+  for (size_t i = 0; i < kd.size(); ++i) {
+    if (ed[i]) D.push_back(kd[i]);
     else ++dropped;
   }
   // directed pairs grouped by source
