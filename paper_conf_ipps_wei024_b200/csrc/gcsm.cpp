@@ -774,6 +774,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.tup_rem = d_trem;
   A.tup_rem_cap = rem_cap;
   A.k = k;
+  A.n_plans = (int32_t)QK.plans.size();
   A.listing = listing ? 1 : 0;
   if (k >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
     const size_t na = (size_t)64 << 20, nt = (size_t)4 << 20;
@@ -905,6 +906,9 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
   st.host_copied_bytes = h[CNT_COPIED];
   st.d2h_bytes = sizeof(unsigned long long) * CNT_N;
   st.frontier = h[CNT_F2];
+  if (std::getenv("GCSM_TRACE"))
+    std::fprintf(stderr, "[gcsm kern] frontier=%llu runs=%llu pins=%llu pin_gb=%.3f copied_gb=%.3f\n", h[CNT_F2],
+                 h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_COPIED] / 1e9);
   bool trunc = false;
   if (sl.tup_add || sl.tup_rem) {
     const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);

@@ -843,6 +843,444 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   flush(A, acc, lane);
 }
 
+// ---- k = 4 count mode: the last level as one lean kernel ("k_last4") -------------------------
+// Every level-2 frontier entry (unit, x2) of a 4-vertex query needs one count: |∩ of position 3's backward lists|
+// under the entry's views, label, injectivity and symmetry range. The generic DFS kernel carries stacks, list
+// arrays indexed at run time (local memory) and a chain of dependent metadata loads per entry; here
+//   * the plan's position-3 rule is packed into one int4 per plan in shared memory (bit masks over positions
+//     0..2: no run-time-indexed arrays, so everything stays in registers);
+//   * a warp grabs up to 32 x2-grouped entries and each lane prefetches ONE entry's metadata (frontier slot,
+//     unit, descriptors and delta records of its seed-side lists) in parallel, parked in a per-warp shared
+//     record: the per-entry dependent global-load chain becomes one parallel round per grab;
+//   * the run's x2 list is pinned once per run (shared memory, else HBM scratch for zero-copy lists);
+//   * symmetry ranges trim sorted lists by a 32-way warp-parallel lower bound (2-3 ballot rounds instead of
+//     log2 L dependent loads by every lane);
+//   * the count is a merge path (both runs device-resident, when cheaper) or lane-parallel binary-search probes.
+struct LR {
+  const int32_t *m;  // main run (trimmed in place)
+  uint32_t ml;
+  const int32_t *x;  // delta run (device memory) or nullptr
+  uint32_t xl;
+  bool dev;
+};
+
+__device__ __forceinline__ uint32_t warp_lb(const int32_t *a, uint32_t n, int32_t v, int lane) {
+  uint32_t lo = 0, hi = n;
+  while (hi - lo > 32) {
+    const uint32_t step = (hi - lo + 31) >> 5;
+    const uint32_t p = lo + (uint32_t)lane * step;
+    const bool pr = p < hi && a[p] < v;
+    const uint32_t c = __popc(__ballot_sync(kFull, pr));
+    if (c == 0) return lo;  // a[lo] >= v
+    const uint32_t nlo = lo + (c - 1) * step + 1;
+    hi = min(hi, lo + c * step);
+    lo = nlo;
+  }
+  const bool pr = lo + (uint32_t)lane < hi && a[lo + lane] < v;
+  return lo + __popc(__ballot_sync(kFull, pr));
+}
+
+__device__ __forceinline__ void warp_trim(LR &L, int32_t vlo, int32_t vhi, int lane) {
+  if (L.ml == 0) return;
+  const uint32_t b = vlo == INT_MIN ? 0u : warp_lb(L.m, L.ml, vlo + 1, lane);
+  const uint32_t e = vhi == INT_MAX ? L.ml : warp_lb(L.m, L.ml, vhi, lane);
+  L.m += b;
+  L.ml = e > b ? e - b : 0u;
+}
+
+__device__ __forceinline__ bool lr_has(const LR &L, int32_t v) {
+  return bsearch_has(L.m, L.ml, v) || (L.xl != 0 && bsearch_has(L.x, L.xl, v));
+}
+
+// pack position 3 of a k = 4 plan: x = list_mask | probe_mask << 3 | reuse << 6 | inj << 8 | lo << 11 | hi << 14 |
+// kind << 17 | view(p) << (20 + 2p); y = label
+__device__ int4 pack_last4(const DevPlan &P) {
+  const LevelPlan &L = P.lv[3];
+  unsigned lm = 0, pm = 0, im = 0, lo = 0, hi = 0, vw = 0;
+  for (int b = 0; b < L.nb; ++b) {
+    lm |= 1u << L.bpos[b];
+    vw |= (unsigned)L.bview[b] << (2 * L.bpos[b]);
+  }
+  if (L.reuse >= 0)
+    for (int r = 0; r < L.nrest; ++r) pm |= 1u << L.bpos[L.rest[r]];
+  for (int i = 0; i < L.ninj; ++i) im |= 1u << L.inj[i];
+  for (int i = 0; i < L.nlo; ++i) lo |= 1u << L.lo[i];
+  for (int i = 0; i < L.nhi; ++i) hi |= 1u << L.hi[i];
+  const unsigned x = lm | pm << 3 | (L.reuse >= 0 ? 1u : 0u) << 6 | im << 8 | lo << 11 | hi << 14 |
+                     (unsigned)P.kind << 17 | vw << 20;
+  return make_int4((int)x, L.label, 0, 0);
+}
+
+// Prefetch side: vertex v's raw descriptor with the delta run of view vw resolved -> {ptr lo, ptr hi, len, xoff}
+// and the delta length in *xl.
+__device__ __forceinline__ int4 lr_fetch(const MatchArgs &A, int32_t v, int vw, int *xl) {
+  int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
+  const uint32_t upd = (uint32_t)raw.w;
+  *xl = 0;
+  raw.w = 0;
+  if (upd != 0 && vw != VIEW_S) {
+    const int4 e = __ldg(reinterpret_cast<const int4 *>(A.drec + (upd - 1)));
+    raw.w = vw == VIEW_NEW ? e.x : e.z;
+    *xl = vw == VIEW_NEW ? e.y : e.w;
+  }
+  return raw;
+}
+
+// Entry side: the list from a prefetched record; algorithmic bytes accounted (hit / miss / delta).
+__device__ __forceinline__ LR lr_make(const MatchArgs &A, const int4 r, int xl, Acc &acc) {
+  LR l;
+  l.m = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)r.x | ((unsigned long long)(unsigned)r.y << 32));
+  l.ml = (uint32_t)r.z;
+  l.x = xl ? A.dlist + r.w : nullptr;
+  l.xl = (uint32_t)xl;
+  l.dev = is_hit(A, l.m);
+  if (l.dev) acc.hit += 4ull * l.ml;
+  else acc.miss += 4ull * l.ml;
+  acc.delta += 4ull * l.xl;
+  return l;
+}
+
+// bulk-copy a zero-copy list when the staging rule of stage_lists says so (drv: always), into the free part of
+// the warp's shared slice, else its HBM staging buffer (out of line: rare, and its copy loop is register-hungry)
+__device__ __noinline__ void stage_slow(LR &L, bool drv, uint32_t d, int32_t *&sm, uint32_t &sm_left, int32_t *&g,
+                                        uint32_t &g_left, int lane, unsigned long long &copied) {
+  const uint32_t n = L.ml;
+  if (!drv) {
+    const uint32_t lg = 32u - __clz(n);
+    if (4ull * n > 32ull * d * (lg > 4 ? lg - 3 : 1)) return;
+  }
+  // a trimmed run starts anywhere: copy from its 16-byte granule (lists are allocated in granules)
+  const uint32_t mis = (uint32_t)((reinterpret_cast<uintptr_t>(L.m) >> 2) & 3u);
+  const uint32_t cn = n + mis, n4 = (cn + 3) & ~3u;
+  int32_t *dst;
+  if (n4 <= sm_left) {
+    dst = sm;
+    sm += n4;
+    sm_left -= n4;
+  } else if (n4 <= g_left) {
+    dst = g;
+    g += n4;
+    g_left -= n4;
+  } else {
+    return;
+  }
+  warp_copy(dst, L.m - mis, cn, lane);
+  __syncwarp();
+  copied += 4ull * cn;
+  L.m = dst + mis;
+  L.dev = true;
+}
+
+__device__ __forceinline__ void stage_one(LR &L, bool drv, uint32_t d, int32_t *&sm, uint32_t &sm_left,
+                                          int32_t *&g, uint32_t &g_left, int lane, Acc &acc) {
+  if (L.dev || L.ml < 32) return;
+  stage_slow(L, drv, d, sm, sm_left, g, g_left, lane, acc.copied);
+}
+
+__device__ __noinline__ void copy_list(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
+  warp_copy(dst, src, n, lane);
+  __syncwarp();
+}
+
+__device__ __forceinline__ uint32_t warp_sum(uint32_t c) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
+  return c;
+}
+
+__device__ __forceinline__ void swap_lr(LR &a, LR &b) {
+  const LR t = a;
+  a = b;
+  b = t;
+}
+
+// position 3's symmetry range of a packed plan for the partial match (a, b, x2); false if the plan's position 3
+// does not read x2's list
+__device__ __forceinline__ bool l4_range(unsigned pk, int32_t a, int32_t b, int32_t x2, int32_t *lo, int32_t *hi) {
+  const bool reuse = (pk >> 6) & 1u;
+  const unsigned need = reuse ? (pk >> 3) & 7u : pk & 7u;
+  const unsigned lom = (pk >> 11) & 7u, him = (pk >> 14) & 7u;
+  int32_t vlo = INT_MIN, vhi = INT_MAX;
+  if (lom & 1u) vlo = max(vlo, a);
+  if (lom & 2u) vlo = max(vlo, b);
+  if (lom & 4u) vlo = max(vlo, x2);
+  if (him & 1u) vhi = min(vhi, a);
+  if (him & 2u) vhi = min(vhi, b);
+  if (him & 4u) vhi = min(vhi, x2);
+  *lo = vlo;
+  *hi = vhi;
+  return (need & 4u) != 0;
+}
+
+#ifndef GCSM_PIN_RANGE
+#define GCSM_PIN_RANGE 0  // 1: pin only the run's symmetry-range slice of x2's list (search costs > bytes saved)
+#endif
+#ifndef GCSM_ZC_TRIM
+#define GCSM_ZC_TRIM 0
+#endif
+#ifndef GCSM_L4_MINBLOCKS
+#define GCSM_L4_MINBLOCKS 3
+#endif
+#ifndef GCSM_LAST4
+#define GCSM_LAST4 1
+#endif
+constexpr int kL4Meta = 32 * 4;  // int4 per warp: 32 entries x 4
+constexpr int kL4SmemBytes = kSmemBytes + kWarps * kL4Meta * 16 + GCSM_MAXPLANS * 16;
+
+__global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const MatchArgs A) {
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  extern __shared__ int4 smem_raw[];
+  int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + wib * kSmemInts;
+  int4 *meta = smem_raw + kSmemBytes / 16 + wib * kL4Meta;
+  int4 *lp = smem_raw + kSmemBytes / 16 + kWarps * kL4Meta;
+  for (int i = threadIdx.x; i < A.n_plans; i += blockDim.x) lp[i] = pack_last4(A.plans[i]);
+  __syncthreads();
+  int32_t *gstage = A.scratch + gw * A.scratch_stride + A.scratch_stride - 2 * (int64_t)A.dcap;
+  int32_t *pstage = gstage - (int64_t)A.dcap;
+  const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
+  const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
+  const int32_t *f2u = f2c + A.f2_cap;
+  const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t chunk = max((int64_t)1, min((int64_t)32, n_f2 / (4 * warps)));
+  Acc acc;
+  unsigned long long d_runs = 0, d_pinb = 0, d_pins = 0;
+  for (;;) {
+    unsigned long long c0 = 0;
+    if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)chunk);
+    c0 = __shfl_sync(kFull, c0, 0);
+    if ((int64_t)c0 >= n_f2) break;
+    const int n = (int)min((int64_t)chunk, n_f2 - (int64_t)c0);
+    // ---- one lane per entry: prefetch the entry's metadata in parallel
+    __syncwarp();
+    if (lane < n) {
+      const int64_t j = (int64_t)c0 + lane;
+      const int64_t e = A.group ? A.group[j] : j;
+      const int32_t x2 = f2c[e], ui = f2u[e];
+      const int4 u = __ldg(reinterpret_cast<const int4 *>(A.units + ui));  // a, b, plan
+      const unsigned pk = (unsigned)lp[u.z].x;
+      const unsigned need = (pk >> 6) & 1u ? (pk >> 3) & 7u : pk & 7u;
+      int4 r1 = make_int4(0, 0, 0, 0), r2 = make_int4(0, 0, 0, 0);
+      int2 seg = make_int2(0, 0);
+      int xl0 = 0, xl1 = 0;
+      if (need & 1u) r1 = lr_fetch(A, u.x, (pk >> 20) & 3u, &xl0);
+      if (need & 2u) r2 = lr_fetch(A, u.y, (pk >> 22) & 3u, &xl1);
+      if ((pk >> 6) & 1u) seg = A.useg[ui];
+      meta[4 * lane + 0] = make_int4(x2, u.z, u.x, u.y);
+      meta[4 * lane + 1] = r1;
+      meta[4 * lane + 2] = r2;
+      meta[4 * lane + 3] = make_int4(seg.x, seg.y, xl0, xl1);
+    }
+    __syncwarp();
+    int32_t pin_v = -1;  // x2 of the current run and its list slice (pinned copy, or in place)
+    const int32_t *pin_p = nullptr;
+    uint32_t pin_len = 0;
+    int4 xraw = make_int4(0, 0, 0, 0);
+    int4 xrec = make_int4(0, 0, 0, 0);  // x2's delta record (if updated)
+    uint32_t pin_sm = 0;
+    bool pin_dev = false, pin_hit = false;
+    for (int i = 0; i < n; ++i) {
+      const int4 m0 = meta[4 * i];
+      const int32_t x2 = m0.x, a = m0.z, b = m0.w;
+      if (x2 != pin_v) {  // new run: entries i..i+run-1 share x2
+        const bool same = i + 1 + lane < n && meta[4 * (i + 1 + lane)].x == x2;
+        const unsigned rm = __ballot_sync(kFull, same);
+        const int run = 1 + (rm == kFull ? 32 : __ffs(~rm) - 1);
+        // union of the symmetry ranges of the run's entries that read x2's list: only that slice is fetched
+        int32_t rlo = INT_MAX, rhi = INT_MIN;
+        if (lane < run) {
+          const int4 mr = meta[4 * (i + lane)];
+          int32_t lo, hi;
+          if (l4_range((unsigned)lp[mr.y].x, mr.z, mr.w, x2, &lo, &hi)) {
+            rlo = lo;
+            rhi = hi;
+          }
+        }
+        rlo = __reduce_min_sync(kFull, rlo);
+        rhi = __reduce_max_sync(kFull, rhi);
+        pin_v = x2;
+        xraw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + x2));
+        xrec = xraw.w ? __ldg(reinterpret_cast<const int4 *>(A.drec + ((uint32_t)xraw.w - 1))) : make_int4(0, 0, 0, 0);
+        const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)xraw.x |
+                                                                ((unsigned long long)(unsigned)xraw.y << 32));
+        const uint32_t ml = (uint32_t)xraw.z;
+        pin_hit = is_hit(A, mp);
+        uint32_t lb = 0, le = ml;
+        if (rlo > rhi) {
+          le = 0;  // no entry of the run reads x2's list
+        } else if (GCSM_PIN_RANGE && ml >= 32) {
+          if (rlo != INT_MIN) lb = warp_lb(mp, ml, rlo + 1, lane);
+          if (rhi != INT_MAX) le = max(lb, warp_lb(mp, ml, rhi, lane));
+        }
+        pin_p = mp + lb;
+        pin_len = le - lb;
+        pin_dev = pin_hit;
+        pin_sm = 0;
+        ++d_runs;
+        // copy from the 16-byte granule holding the slice's first element (lists are granule-aligned)
+        const uint32_t mis = lb & 3u, cn = pin_len + mis, cn4 = (cn + 3) & ~3u;
+        if (run >= 2 && pin_len >= 32 && !pin_hit) {
+          ++d_pins;
+          d_pinb += 4ull * cn;
+        }
+        if (run >= 2 && pin_len >= 32 && cn4 <= GCSM_PIN_SMEM_MAX) {
+          copy_list(sm, mp + (lb - mis), cn, lane);
+          if (!pin_hit) acc.copied += 4ull * cn;
+          pin_p = sm + mis;
+          pin_dev = true;
+          pin_sm = cn4;
+        } else if (run >= 2 && pin_len >= 32 && !pin_hit) {
+          copy_list(pstage, mp + (lb - mis), cn, lane);
+          acc.copied += 4ull * cn;
+          pin_p = pstage + mis;
+          pin_dev = true;
+        }
+      }
+      const unsigned pk = (unsigned)lp[m0.y].x;
+      const int label = lp[m0.y].y;
+      const bool reuse = (pk >> 6) & 1u;
+      const unsigned need = reuse ? (pk >> 3) & 7u : pk & 7u;
+      const unsigned im = (pk >> 8) & 7u, lom = (pk >> 11) & 7u, him = (pk >> 14) & 7u;
+      const int kind = (pk >> 17) & 1u;
+      int32_t vlo = INT_MIN, vhi = INT_MAX;
+      if (lom & 1u) vlo = max(vlo, a);
+      if (lom & 2u) vlo = max(vlo, b);
+      if (lom & 4u) vlo = max(vlo, x2);
+      if (him & 1u) vhi = min(vhi, a);
+      if (him & 2u) vhi = min(vhi, b);
+      if (him & 4u) vhi = min(vhi, x2);
+      const int32_t ex0 = (im & 1u) ? a : -1, ex1 = (im & 2u) ? b : -1, ex2 = (im & 4u) ? x2 : -1;
+      // the lists: slot 0 = driver, slots 1.. = probes (positions in ascending order; selects, no indexed arrays)
+      const int4 m3 = meta[4 * i + 3];
+      LR La, Lb, Lc;
+      La.xl = Lb.xl = Lc.xl = 0;
+      La.x = Lb.x = Lc.x = nullptr;
+      La.ml = Lb.ml = Lc.ml = 0;
+      La.m = Lb.m = Lc.m = nullptr;
+      La.dev = Lb.dev = Lc.dev = true;
+      if (need & 1u) La = lr_make(A, meta[4 * i + 1], m3.z, acc);
+      if (need & 2u) Lb = lr_make(A, meta[4 * i + 2], m3.w, acc);
+      if (need & 4u) {
+        const int vw = (pk >> 24) & 3u;
+        Lc.m = pin_p;
+        Lc.ml = pin_len;  // the run's range slice (every read below is range-checked or range-trimmed)
+        Lc.dev = pin_dev;
+        if (xraw.w != 0 && vw != VIEW_S) {
+          Lc.x = A.dlist + (vw == VIEW_NEW ? xrec.x : xrec.z);
+          Lc.xl = (uint32_t)(vw == VIEW_NEW ? xrec.y : xrec.w);
+        }
+        if (pin_hit) acc.hit += 4ull * (uint32_t)xraw.z;  // algorithmic: the whole list
+        else acc.miss += 4ull * (uint32_t)xraw.z;
+        acc.delta += 4ull * Lc.xl;
+      }
+      const LR first = (need & 1u) ? La : ((need & 2u) ? Lb : Lc);
+      const LR second = (need & 1u) ? ((need & 2u) ? Lb : Lc) : Lc;
+      const int nl = __popc(need) + (reuse ? 1 : 0);
+      LR L0, L1, L2;
+      if (reuse) {  // the unit's level-2 candidate set (code motion); not globally sorted (main then delta run)
+        L0.m = f2c + m3.x;
+        L0.ml = (uint32_t)m3.y;
+        L0.x = nullptr;
+        L0.xl = 0;
+        L0.dev = true;
+        L1 = first;
+        L2 = second;
+      } else {
+        L0 = first;
+        L1 = second;
+        L2 = Lc;
+      }
+#if GCSM_ZC_TRIM
+      // zero-copy lists: only their range slice is read and staged (costs PCIe round trips: measured slower)
+      if (!L0.dev && L0.ml >= 32) warp_trim(L0, vlo, vhi, lane);
+      if (nl >= 2 && !L1.dev && L1.ml >= 32) warp_trim(L1, vlo, vhi, lane);
+      if (nl >= 3 && !L2.dev && L2.ml >= 32) warp_trim(L2, vlo, vhi, lane);
+#endif
+      if (!reuse) {  // the smallest list drives
+        if (nl >= 2 && L1.ml + L1.xl < L0.ml + L0.xl) swap_lr(L0, L1);
+        if (nl >= 3 && L2.ml + L2.xl < L0.ml + L0.xl) swap_lr(L0, L2);
+      }
+      const uint32_t d = L0.ml + L0.xl;
+      int32_t *smf = sm + pin_sm, *gf = gstage;
+      uint32_t sml = kSmemInts - pin_sm, gl = 2u * (uint32_t)A.dcap;
+      stage_one(L0, true, d, smf, sml, gf, gl, lane, acc);
+      if (nl >= 2) stage_one(L1, false, d, smf, sml, gf, gl, lane, acc);
+      if (nl >= 3) stage_one(L2, false, d, smf, sml, gf, gl, lane, acc);
+      uint32_t c = 0;
+      bool done = false;
+      if (!reuse && nl == 2 && L0.dev && L1.dev && L0.ml >= 8 && L1.ml >= 8) {
+        // merge path on the range-trimmed main runs when cheaper than d/32 rounds of binary search
+        warp_trim(L0, vlo, vhi, lane);
+        warp_trim(L1, vlo, vhi, lane);
+        const uint32_t dd = L0.ml + L0.xl, big = L1.ml + L1.xl;
+        const uint32_t bs_cost = ((dd + 31) >> 5) * (7 * ilog2(big) + 12);
+        const uint32_t mg_cost = 10 * ilog2(min(L0.ml, L1.ml) | 1u) + 7 * ((L0.ml + L1.ml + 31) >> 5) + 30;
+        if (mg_cost < bs_cost && L0.ml > 0 && L1.ml > 0) {
+          c = merge_count(L0.m, L0.ml, L1.m, L1.ml, label, A.lab, lane);
+          if (L0.xl) c += probe_count(L0.x, L0.xl, L1.m, L1.ml, label, A.lab, lane, vlo, vhi);
+          if (L1.xl) c += probe_count(L1.x, L1.xl, L0.m, L0.ml, label, A.lab, lane, vlo, vhi);
+          if (L0.xl && L1.xl) c += probe_count(L0.x, L0.xl, L1.x, L1.xl, label, A.lab, lane, vlo, vhi);
+          const int32_t exs[3] = {ex0, ex1, ex2};
+#pragma unroll
+          for (int q = 0; q < 3; ++q) {
+            const int32_t v = exs[q];
+            if (v >= 0 && v > vlo && v < vhi && (label < 0 || A.lab[v] == (uint16_t)label) && lr_has(L0, v) &&
+                lr_has(L1, v))
+              --c;
+          }
+          done = true;
+        }
+      } else if (L0.dev && !reuse) {
+        warp_trim(L0, vlo, vhi, lane);
+      }
+      if (!done) {
+        if (nl == 1 && label < 0 && !reuse) {  // single list: its in-range size minus the excluded vertices it holds
+          uint32_t cx = 0;
+          for (uint32_t q = lane; q < L0.xl; q += 32) {
+            const int32_t v = L0.x[q];
+            cx += v > vlo && v < vhi;
+          }
+          c = (L0.dev ? L0.ml : 0u) + warp_sum(cx);
+          if (!L0.dev) {  // untrimmed zero-copy run: count in range
+            uint32_t cm = 0;
+            for (uint32_t q = lane; q < L0.ml; q += 32) {
+              const int32_t v = L0.m[q];
+              cm += v > vlo && v < vhi;
+            }
+            c += warp_sum(cm);
+          }
+          const int32_t exs[3] = {ex0, ex1, ex2};
+#pragma unroll
+          for (int q = 0; q < 3; ++q) {
+            const int32_t v = exs[q];
+            if (v >= 0 && v > vlo && v < vhi && lr_has(L0, v)) --c;
+          }
+        } else {  // lane-parallel probes of the driver's elements
+          uint32_t cnt = 0;
+          const uint32_t total = L0.ml + L0.xl;
+          for (uint32_t q = lane; q < total; q += 32) {
+            const int32_t v = q < L0.ml ? L0.m[q] : L0.x[q - L0.ml];
+            bool ok = v > vlo && v < vhi && v != ex0 && v != ex1 && v != ex2;
+            if (ok && nl >= 2) ok = lr_has(L1, v);
+            if (ok && nl >= 3) ok = lr_has(L2, v);
+            if (ok && label >= 0) ok = A.lab[v] == (uint16_t)label;
+            cnt += ok;
+          }
+          c = warp_sum(cnt);
+        }
+      }
+      if (kind) acc.rem += c;
+      else acc.add += c;
+    }
+  }
+  flush(A, acc, lane);
+  if (lane == 0) {
+    atomicAdd(&A.cnt[CNT_DBG_RUNS], d_runs);
+    atomicAdd(&A.cnt[CNT_DBG_PINBYTES], d_pinb);
+    atomicAdd(&A.cnt[CNT_DBG_PINS], d_pins);
+  }
+}
+
 // ---- counting sort of the level-2 frontier by its candidate vertex x2 (entries sharing x2 are
 // processed back to back by one warp, which stages x2's zero-copy list once per run).
 __global__ void k_group_hist(const int32_t *f2c, const unsigned long long *cnt, uint32_t *hist) {
@@ -975,6 +1413,7 @@ int match_grid(int device, int *warps_total) {
   cudaFuncSetAttribute(k_extend<true, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   cudaFuncSetAttribute(k_level2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   cudaFuncSetAttribute(k_level2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_last4, cudaFuncAttributeMaxDynamicSharedMemorySize, kL4SmemBytes);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false, 0>, kBlock, kSmemBytes);
   int occ2 = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_level2<false>, kBlock, kSmemBytes);
@@ -1005,6 +1444,7 @@ cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
   a.acc_base = CNT_ACC_EXT;
   if (a.tasks) k_reset_sharing<<<1, 1, 0, s>>>(a.cnt);
   if (a.listing) k_extend<true, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
+  else if (a.k == 4 && GCSM_LAST4) k_last4<<<grid, kBlock, kL4SmemBytes, s>>>(a);
   else if (a.k == 4) k_extend<false, 4><<<grid, kBlock, kSmemBytes, s>>>(a);
   else k_extend<false, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
   return cudaGetLastError();

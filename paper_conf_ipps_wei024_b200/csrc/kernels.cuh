@@ -26,6 +26,9 @@ enum Counter {
   CNT_HEAD = 18,    // level-3 tasks taken
   CNT_PRODUCERS = 19,  // frontier entries fully walked (their tasks, if any, published)
   CNT_SPLIT = 20,   // level-3 sets handed out as tasks (stats)
+  CNT_DBG_RUNS = 21,     // k_last4: x2 runs started (GCSM_TRACE)
+  CNT_DBG_PINBYTES = 22, // k_last4: zero-copy bytes copied by run pins
+  CNT_DBG_PINS = 23,     // k_last4: runs pinned
   CNT_N = 24
 };
 
@@ -52,6 +55,7 @@ struct MatchArgs {
   int32_t *tup_rem;
   uint64_t tup_rem_cap;
   int32_t k;
+  int32_t n_plans;          // plans[] entries (2 m)
   int32_t listing;
   int32_t acc_base;         // CNT_ACC_L2 or CNT_ACC_EXT (set by the launchers)
   // level-3 work sharing (k >= 5): a warp whose level-3 candidate set is large copies it to the arena and
