@@ -53,9 +53,8 @@ def parse():
                     help="test the N>1 plumbing on one GPU: gloo process group, every rank on cuda:0, shard-local "
                          "counts (no NCCL communicator)")
     ap.add_argument("--serial", action="store_true",
-                    help="synchronous apply_batch, query contexts one after the other (default at N=1: one host "
-                         "thread per query context, each pipelining submit/wait so batch t+1's host steps overlap "
-                         "batch t's kernels)")
+                    help="synchronous apply_batch per step (default: pipelined submit/wait, so batch t+1's host "
+                         "steps overlap batch t's kernels)")
     return ap.parse_args()
 
 
@@ -257,65 +256,43 @@ def main():
     frac = w.budget_frac if args.budget_frac is None else args.budget_frac
     budget = int(w.adj_bytes * frac)
     nccl_id = G.distributed_nccl_id() if world > 1 and not args.emulate else None
-    ctxs = []
-    for q in queries:
+    # one context per GPU holding every standing query of the config: the store, each batch's normalisation,
+    # overlays and merge, and ONE cache under the per-GPU budget are shared (gcsm_add_query)
+    g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=local, rank=rank, world=world, nccl_id=nccl_id,
+               cache_policy=args.cache_policy, local_counts=bool(args.emulate and world > 1),
+               host_threads=per_rank if world > 1 else 0)
+    for i, q in enumerate(queries):
         k, qe, ql = gi.query(q)
-        g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=local, rank=rank, world=world, nccl_id=nccl_id,
-                   cache_policy=args.cache_policy, local_counts=bool(args.emulate and world > 1),
-                   host_threads=per_rank if world > 1 else 0)
-        g.set_query(k, qe, ql)
-        g.set_cache_budget(budget)
-        ctxs.append((q, g))
+        if i == 0:
+            g.set_query(k, qe, ql)
+        else:
+            g.add_query(k, qe, ql)
+    g.set_cache_budget(budget)
     steps = args.warmup + args.steps
     assert len(w.batches) >= steps, "stream too short"
     batches = [(np.ascontiguousarray(a, dtype=np.int32), np.ascontiguousarray(b, dtype=np.int32))
                for a, b in w.batches[:steps]]
 
-    def run_one(q, g, i, out, slot):
-        a, r = g.apply_batch(*batches[i])
-        out[slot] = (q, a, r, g.stats())
+    def collect():
+        return [(q, *g.query_counts(i), g.query_stats(i)) for i, q in enumerate(queries)]
 
-    def run_pipelined(q, g, lo, hi, out, slot):
-        """batch i+1's host steps overlap batch i's kernels (gcsm_submit_batch / gcsm_wait_batch)"""
+    def do_step(i):
+        g.apply_batch(*batches[i])
+        return collect()
+
+    def timed_steps(lo, hi):
+        """per-step records [[(q, added, removed, stats) per query] per batch]"""
+        if args.serial:
+            return [do_step(i) for i in range(lo, hi)]
+        # pipelined: batch i+1's host steps overlap batch i's kernels (gcsm_submit_batch / gcsm_wait_batch)
         recs = []
         g.submit_batch(*batches[lo])
         for i in range(lo + 1, hi):
             g.submit_batch(*batches[i])
-            a, r = g.wait_batch()
-            recs.append((q, a, r, g.stats()))
-        a, r = g.wait_batch()
-        recs.append((q, a, r, g.stats()))
-        out[slot] = recs
-
-    def timed_steps(lo, hi):
-        """returns per-step records [[(q, a, r, stats) per context] per batch]"""
-        if args.serial or world > 1:
-            return [do_step(i) for i in range(lo, hi)]
-        outs = [None] * len(ctxs)
-        ths = [threading.Thread(target=run_pipelined, args=(q, g, lo, hi, outs, slot))
-               for slot, (q, g) in enumerate(ctxs)]
-        for t in ths:
-            t.start()
-        for t in ths:
-            t.join()
-        if any(o is None for o in outs):
-            raise RuntimeError("a query context failed")
-        return [[outs[c][i] for c in range(len(ctxs))] for i in range(hi - lo)]
-
-    def do_step(i):
-        recs = [None] * len(ctxs)
-        # world > 1: serial, so every rank issues its contexts' NCCL allreduces in the same order
-        if args.serial or len(ctxs) == 1 or world > 1:
-            for slot, (q, g) in enumerate(ctxs):
-                run_one(q, g, i, recs, slot)
-        else:  # independent standing queries: one host thread each (ctypes releases the GIL)
-            ths = [threading.Thread(target=run_one, args=(q, g, i, recs, slot)) for slot, (q, g) in enumerate(ctxs)]
-            for t in ths:
-                t.start()
-            for t in ths:
-                t.join()
-        if any(r is None for r in recs):
-            raise RuntimeError("a query context failed")
+            g.wait_batch()
+            recs.append(collect())
+        g.wait_batch()
+        recs.append(collect())
         return recs
 
     for i in range(args.warmup):
@@ -324,7 +301,7 @@ def main():
     clocks = Clocks(local)
     if not args.quick and rank == 0:
         clocks.start()
-    streams = [torch.cuda.ExternalStream(g.stream_ptr()) for _, g in ctxs]
+    streams = [torch.cuda.ExternalStream(g.stream_ptr())]
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier(world)
     torch.cuda.synchronize()
@@ -357,6 +334,8 @@ def main():
                 if key not in ("added", "removed"):
                     d[key] += st[key]
     K = args.steps
+    shared = {x: per_q[queries[0]][x] for x in ("h2d_bytes", "d2h_bytes", "kernel_launches", "cache_bytes",
+                                                 "cached_vertices")}
     value = edges / (ms_dev / 1e3)
     e2e_value = edges / (ms_host / 1e3)
     # dominant kernel: k_extend of the heaviest query; algorithmic HBM bytes = cache + delta list bytes it reads
@@ -399,9 +378,8 @@ def main():
     cpu = None
     if not args.no_cpu_baseline and not args.quick and world == 1:
         cpu = cpu_baseline(w, queries, args.cpu_seconds)
-    h2d = sum(d["h2d_bytes"] for d in per_q.values()) / K + sum(8 * len(b[0]) + 8 * len(b[1])
-                                                               for b in batches[args.warmup:]) / K
-    d2h = sum(d["d2h_bytes"] for d in per_q.values()) / K
+    h2d = shared["h2d_bytes"] / K + sum(8 * len(b[0]) + 8 * len(b[1]) for b in batches[args.warmup:]) / K
+    d2h = shared["d2h_bytes"] / K
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms_dev / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
@@ -411,13 +389,15 @@ def main():
                                f"{frac:.0%} of adjacency", "queries": queries, "global_batch": args.batch * world,
                    "graph_vertices": w.n, "graph_edges": int(w.row_ptr[-1] // 2), "budget_bytes": budget,
                    "cache_policy": args.cache_policy,
-                   "parallelism": f"units LPT-sharded over {world} GPU(s); "
-                                  f"{'serial synchronous' if (args.serial or world > 1) else 'concurrent pipelined'} query contexts",
+                   "cache_mb": shared["cache_bytes"] / K / 2**20,
+                   "parallelism": f"units LPT-sharded over {world} GPU(s); one context per GPU with all queries "
+                                  f"(shared store, batch steps and cache budget), "
+                                  f"{'synchronous' if args.serial else 'pipelined submit/wait'} batches",
                    "l2": "inputs larger than L2 (560 MB pinned host graph; cache repacked every batch)"},
         "roofline": roofline,
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)},
-        "gpu_launches": int(sum(d["kernel_launches"] for d in per_q.values())),
+        "gpu_launches": int(shared["kernel_launches"]),
         "clocks": clk,
         "cache_hit_rate": tot_hit / tot_all if tot_all else None,
         "host_link": link,
@@ -434,8 +414,7 @@ def main():
         "gen_seconds": gen_s,
     }
     print(json.dumps(line), flush=True)
-    for _, g in ctxs:
-        g.close()
+    g.close()
 
 
 if __name__ == "__main__":

@@ -146,6 +146,21 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
 gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
                            const int32_t *order);
 
+/* Adds another standing query to the context (gcsm_set_query replaces all of them with one). Arguments as
+ * gcsm_set_query; *qid (may be NULL) receives its index (query 0 is the set_query one). Up to 8 queries. The
+ * queries share the host store, each batch's normalisation, overlays and merge (steps (1) and (5) of Fig. 3)
+ * and ONE device cache under the per-GPU budget, filled by ranking vertices on the SUM of the queries'
+ * estimated access frequencies (eq. (3) per query; P:339's top-K rule on the sum). Every query gets
+ * its own level-1 units, estimator walks, kernels and counters: gcsm_apply_batch / gcsm_wait_batch return
+ * query 0's counts, gcsm_get_query_stats any query's. List mode needs exactly one query (EINVAL otherwise).
+ * ESTATE before gcsm_set_query or with a batch in flight; EINVAL for a bad pattern or a 9th query (nothing
+ * changes). With world > 1 this is collective. */
+gcsm_status gcsm_add_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                           const int32_t *order, int32_t *qid);
+
+/* Number of standing queries (0 before gcsm_set_query). */
+int32_t gcsm_num_queries(const gcsm_ctx *ctx);
+
 /* Per-GPU byte budget of the HBM list cache ("GPU buffer"); it counts
  * cached list payload (16-byte aligned lists). 0 = pure zero-copy. Applies
  * from the next batch. ENOMEM if the device buffer cannot be allocated. */
@@ -180,8 +195,12 @@ gcsm_status gcsm_apply_batch_list(gcsm_ctx *ctx, int64_t n_ins, const int32_t *i
 gcsm_status gcsm_submit_batch(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del);
 gcsm_status gcsm_wait_batch(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed);
 
-/* Last batch's statistics. */
+/* Last batch's statistics (query 0; the shared steps' times are the batch's). */
 gcsm_status gcsm_get_stats(const gcsm_ctx *ctx, gcsm_stats *out);
+
+/* Last batch's statistics of query qid (its counts in added / removed, its kernels' times and bytes, its
+ * estimator time; the shared steps as in gcsm_get_stats). EINVAL for an unknown qid. */
+gcsm_status gcsm_get_query_stats(const gcsm_ctx *ctx, int32_t qid, gcsm_stats *out);
 
 /* |Aut_L(Q)| (label-preserving automorphisms) of the current query, 0 if none. */
 uint64_t gcsm_query_automorphisms(const gcsm_ctx *ctx);

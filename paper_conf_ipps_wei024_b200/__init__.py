@@ -95,6 +95,26 @@ class Gcsm:
                                              _ptr(_i32(order))), "set_query")
         self.k = int(k)
 
+    def add_query(self, k, qedges, qlabels=None, order=None) -> int:
+        """Another standing query sharing the store, the batch steps and the cache budget; returns its id."""
+        qe = _i32(qedges).reshape(-1, 2)
+        qid = ctypes.c_int32()
+        self._check(self._lib.gcsm_add_query(self._h, int(k), len(qe), _ptr(qe), _ptr(_i32(qlabels)),
+                                             _ptr(_i32(order)), ctypes.byref(qid)), "add_query")
+        return qid.value
+
+    def num_queries(self) -> int:
+        return int(self._lib.gcsm_num_queries(self._h))
+
+    def query_stats(self, qid: int) -> dict:
+        st = Stats()
+        self._check(self._lib.gcsm_get_query_stats(self._h, int(qid), ctypes.byref(st)), "get_query_stats")
+        return {name: getattr(st, name) for name, _ in Stats._fields_}
+
+    def query_counts(self, qid: int):
+        st = self.query_stats(qid)
+        return st["added"], st["removed"]
+
     def set_cache_budget(self, nbytes: int):
         self._check(self._lib.gcsm_set_cache_budget(self._h, int(nbytes)), "set_cache_budget")
 

@@ -17,7 +17,8 @@ STATUS = {0: "GCSM_OK", 1: "GCSM_EINVAL", 2: "GCSM_ENOMEM", 3: "GCSM_EDEVICE", 4
 
 # exported symbols of include/gcsm.h (checked by tests/test_abi.py)
 SYMBOLS = ["gcsm_default_options", "gcsm_create", "gcsm_set_query", "gcsm_set_cache_budget", "gcsm_apply_batch",
-           "gcsm_apply_batch_list", "gcsm_submit_batch", "gcsm_wait_batch", "gcsm_get_stats", "gcsm_query_automorphisms", "gcsm_last_error", "gcsm_destroy",
+           "gcsm_apply_batch_list", "gcsm_submit_batch", "gcsm_wait_batch", "gcsm_get_stats", "gcsm_add_query", "gcsm_num_queries",
+           "gcsm_get_query_stats", "gcsm_query_automorphisms", "gcsm_last_error", "gcsm_destroy",
            "gcsm_nccl_unique_id", "gcsm_get_stream", "gcsm_export_csr", "gcsm_get_estimates", "gcsm_get_cached",
            "gcsm_plan_inspect", "gcsm_query_restrictions", "gcsm_shard",
            "gcsm_measure_host_link"]
@@ -63,6 +64,9 @@ def load():
         "gcsm_submit_batch": (st, [P, I64, P, I64, P]),
         "gcsm_wait_batch": (st, [P, ctypes.POINTER(U64), ctypes.POINTER(U64)]),
         "gcsm_get_stats": (st, [P, ctypes.POINTER(Stats)]),
+        "gcsm_add_query": (st, [P, I32, I32, P, P, P, ctypes.POINTER(I32)]),
+        "gcsm_num_queries": (I32, [P]),
+        "gcsm_get_query_stats": (st, [P, I32, ctypes.POINTER(Stats)]),
         "gcsm_query_automorphisms": (U64, [P]),
         "gcsm_last_error": (ctypes.c_char_p, [P]),
         "gcsm_destroy": (None, [P]),

@@ -60,8 +60,17 @@ struct gcsm_ctx {
   std::string err;
   bool poisoned = false;
   HostStore store;
-  QueryPlan qp;   // plans without restrictions
-  QueryPlan qps;  // plans with the symmetry-breaking restrictions of Aut_L(Q)
+  // Standing queries (gcsm_set_query sets query 0, gcsm_add_query appends): they share the host store, the batch
+  // normalisation / overlays / merge and ONE cache under the per-GPU budget (ranked by the sum of the queries'
+  // estimates); each has its own units, estimator run, plans, kernels and counters.
+  struct Query {
+    QueryPlan qp;   // plans without restrictions
+    QueryPlan qps;  // plans with the symmetry-breaking restrictions of Aut_L(Q)
+    DevPlan *d_plans = nullptr, *d_splans = nullptr;
+    EstimatorOutput est;  // last batch's estimator output
+    gcsm_stats stats{};   // last completed batch
+  };
+  std::vector<Query> qs;
   bool has_query = false;
   uint64_t budget = 0;
   cudaStream_t stream = nullptr;
@@ -75,14 +84,17 @@ struct gcsm_ctx {
     Unit *h_units = nullptr; size_t h_units_cap = 0;
     uint64_t *h_gather = nullptr; size_t h_gather_cap = 0;
     uint64_t *h_fresh = nullptr; size_t h_fresh_cap = 0;
-    unsigned long long *h_cnt = nullptr;
-    cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr, ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr,
-                ev_c1 = nullptr, ev_done = nullptr;
-    std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
-    size_t nev = 0;
+    unsigned long long *h_cnt = nullptr;  // CNT_N per query
+    cudaEvent_t ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr, ev_c1 = nullptr, ev_done = nullptr;
+    struct PerQuery {
+      cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr;
+      std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
+      size_t nev = 0;
+      uint64_t aut_mul = 1;  // canonical-embedding counts x |Aut_L| (symmetry breaking)
+      gcsm_stats st{};
+    };
+    std::vector<PerQuery> q;
     bool inflight = false;
-    uint64_t aut_mul = 1;  // canonical-embedding counts x |Aut_L| (symmetry breaking)
-    gcsm_stats st{};
     double host_ms = 0;
     // list mode
     int32_t *tup_add = nullptr, *tup_rem = nullptr, *d_tadd = nullptr, *d_trem = nullptr;
@@ -96,8 +108,6 @@ struct gcsm_ctx {
 
   // device buffers
   VDesc *d_vdesc = nullptr;
-  DevPlan *d_plans = nullptr;   // the query's plans (estimator, list mode)
-  DevPlan *d_splans = nullptr;  // the same with symmetry-breaking restrictions (count mode)
   uint16_t *d_lab = nullptr;
   DRec *d_drec = nullptr; size_t drec_cap = 0;
   int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
@@ -108,7 +118,7 @@ struct gcsm_ctx {
   uint32_t *d_hist = nullptr;                         // n counters + scan
   uint32_t *d_bsum = nullptr;
   int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
-  unsigned long long *d_cnt = nullptr;
+  unsigned long long *d_cnt = nullptr; size_t cnt_queries = 0;  // CNT_N per query
   char *d_cache = nullptr; size_t cache_cap = 0;   // the buffer this batch's kernels read
   char *d_cachebuf[2] = {nullptr, nullptr};        // double buffer: last batch's cache stays readable
   int cache_cur = 0;                               // buffer holding the previous batch's cache
@@ -130,9 +140,7 @@ struct gcsm_ctx {
   std::vector<int32_t> cached;       // ascending
   std::vector<int32_t> prev_cached, prev_U;
   std::vector<uint8_t> mark;         // scratch (n)
-  EstimatorOutput est;
   EstimatorScratch est_scratch;
-  gcsm_stats stats{};
   uint64_t batch_seq = 0;
   std::vector<int32_t> degree_order;  // GCSM_CACHE_DEGREE ranking
 
@@ -157,7 +165,10 @@ struct gcsm_ctx {
 gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
-  void *dev[] = {d_vdesc, d_plans, d_splans, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
+  for (Query &q : qs)
+    for (DevPlan *p : {q.d_plans, q.d_splans})
+      if (p) cudaFree(p);
+  void *dev[] = {d_vdesc, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (void *p : dev)
     if (p) cudaFree(p);
@@ -165,9 +176,13 @@ gcsm_ctx::~gcsm_ctx() {
     void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt};
     for (void *p : host)
       if (p) cudaFreeHost(p);
-    for (cudaEvent_t e : {sl.ev_m0, sl.ev_m1, sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done})
+    for (cudaEvent_t e : {sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done})
       if (e) cudaEventDestroy(e);
-    for (cudaEvent_t e : sl.kev) cudaEventDestroy(e);
+    for (auto &pq : sl.q) {
+      for (cudaEvent_t e : {pq.ev_m0, pq.ev_m1})
+        if (e) cudaEventDestroy(e);
+      for (cudaEvent_t e : pq.kev) cudaEventDestroy(e);
+    }
   }
   if (stream) cudaStreamDestroy(stream);
 }
@@ -232,15 +247,15 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
   for (auto &sl : ctx->slots) {
-    for (cudaEvent_t *ev : {&sl.ev_m0, &sl.ev_m1, &sl.ev_a0, &sl.ev_a1, &sl.ev_c0, &sl.ev_c1, &sl.ev_done})
+    for (cudaEvent_t *ev : {&sl.ev_a0, &sl.ev_a1, &sl.ev_c0, &sl.ev_c1, &sl.ev_done})
       if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
-    if (cudaHostAlloc(&sl.h_cnt, sizeof(unsigned long long) * CNT_N, cudaHostAllocDefault) != cudaSuccess)
+    if (cudaHostAlloc(&sl.h_cnt, sizeof(unsigned long long) * CNT_N * GCSM_MAX_QUERIES, cudaHostAllocDefault) !=
+        cudaSuccess)
       return bail(GCSM_ENOMEM);
   }
   if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
-  if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N) != cudaSuccess) return bail(GCSM_ENOMEM);
-  if (cudaMalloc(&ctx->d_plans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
-  if (cudaMalloc(&ctx->d_splans, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N * GCSM_MAX_QUERIES) != cudaSuccess)
+    return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)n + 2047) / 2048 + 1)) != cudaSuccess)
     return bail(GCSM_ENOMEM);
@@ -277,29 +292,60 @@ gcsm_status gcsm_get_stream(const gcsm_ctx *ctx, void **stream) {
   return GCSM_OK;
 }
 
-gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
-                           const int32_t *order) {
+static gcsm_status add_query_impl(gcsm_ctx *ctx, bool reset, int32_t k, int32_t m, const int32_t *qedges,
+                                  const int32_t *qlabels, const int32_t *order, int32_t *qid) {
   if (!ctx) return GCSM_EINVAL;
   if (ctx->poisoned) return GCSM_ESTATE;
-  if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "set_query with a batch in flight");
-  QueryPlan qp;
-  QueryPlan qps;
-  std::string e = build_plan(k, m, qedges, qlabels, order, qp);
-  if (e.empty()) e = build_plan(k, m, qedges, qlabels, order, qps, !(ctx->opt.flags & GCSM_FLAG_NO_SYMMETRY));
+  if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "set_query / add_query with a batch in flight");
+  if (!reset && !ctx->has_query) return ctx->fail(GCSM_ESTATE, "add_query before set_query");
+  if (!reset && ctx->qs.size() >= GCSM_MAX_QUERIES) return ctx->fail(GCSM_EINVAL, "too many standing queries");
+  gcsm_ctx::Query q;
+  std::string e = build_plan(k, m, qedges, qlabels, order, q.qp);
+  if (e.empty()) e = build_plan(k, m, qedges, qlabels, order, q.qps, !(ctx->opt.flags & GCSM_FLAG_NO_SYMMETRY));
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
-  if (qp.labelled && !ctx->d_lab) {  // unlabelled graph: every data label is 0 (R5)
+  if (q.qp.labelled && !ctx->d_lab) {  // unlabelled graph: every data label is 0 (R5)
     CK(cudaMalloc(&ctx->d_lab, 2 * (size_t)ctx->store.n));
     CK(cudaMemset(ctx->d_lab, 0, 2 * (size_t)ctx->store.n));
   }
-  CK(upload_plans(ctx->d_plans, qp.plans.data(), (int)qp.plans.size(), ctx->stream));
-  CK(upload_plans(ctx->d_splans, qps.plans.data(), (int)qps.plans.size(), ctx->stream));
+  const size_t slot = reset ? 0 : ctx->qs.size();
+  DevPlan *dp = slot < ctx->qs.size() ? ctx->qs[slot].d_plans : nullptr;
+  DevPlan *dsp = slot < ctx->qs.size() ? ctx->qs[slot].d_splans : nullptr;
+  if (!dp && cudaMalloc(&dp, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess)
+    return ctx->fail(GCSM_ENOMEM, "plan buffer");
+  if (!dsp && cudaMalloc(&dsp, sizeof(DevPlan) * GCSM_MAXPLANS) != cudaSuccess) {
+    if (slot >= ctx->qs.size()) cudaFree(dp);
+    return ctx->fail(GCSM_ENOMEM, "plan buffer");
+  }
+  q.d_plans = dp;
+  q.d_splans = dsp;
+  CK(upload_plans(dp, q.qp.plans.data(), (int)q.qp.plans.size(), ctx->stream));
+  CK(upload_plans(dsp, q.qps.plans.data(), (int)q.qps.plans.size(), ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
-  ctx->qp = qp;
-  ctx->qps = qps;
+  if (reset) {
+    for (size_t i = 1; i < ctx->qs.size(); ++i) {
+      cudaFree(ctx->qs[i].d_plans);
+      cudaFree(ctx->qs[i].d_splans);
+    }
+    ctx->qs.clear();
+  }
+  ctx->qs.push_back(std::move(q));
+  if (qid) *qid = (int32_t)ctx->qs.size() - 1;
   ctx->has_query = true;
   ctx->err.clear();
   return GCSM_OK;
 }
+
+gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                           const int32_t *order) {
+  return add_query_impl(ctx, true, k, m, qedges, qlabels, order, nullptr);
+}
+
+gcsm_status gcsm_add_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
+                           const int32_t *order, int32_t *qid) {
+  return add_query_impl(ctx, false, k, m, qedges, qlabels, order, qid);
+}
+
+int32_t gcsm_num_queries(const gcsm_ctx *ctx) { return ctx && ctx->has_query ? (int32_t)ctx->qs.size() : 0; }
 
 gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
   if (!ctx) return GCSM_EINVAL;
@@ -360,11 +406,13 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const bool listing = tup_add || tup_rem;
   if (listing && ctx->opt.world > 1 && !(ctx->opt.flags & GCSM_FLAG_LOCAL_COUNTS))
     return ctx->fail(GCSM_EINVAL, "list mode is single-GPU");
+  if (listing && ctx->qs.size() != 1) return ctx->fail(GCSM_EINVAL, "list mode needs exactly one query");
   Timer total;
   Trace tr;
   HostStore &S = ctx->store;
-  const QueryPlan &Q = ctx->qp;
-  const int k = Q.k;
+  const int nq = (int)ctx->qs.size();
+  int kmax = 2;
+  for (const auto &q : ctx->qs) kmax = std::max(kmax, q.qp.k);
   const int T = ctx->opt.host_threads;
   gcsm_stats st{};
   st.batches = ctx->batch_seq + 1;
@@ -382,114 +430,148 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   st.n_ins = S.I.size();
   st.n_del = S.D.size();
   st.dropped = S.dropped;
-  // level-1 units: (term, kind, changed edge, orientation) slots enumerated in parallel, then compacted in slot
-  // order (deterministic); the cost proxy of a unit is the list lengths its first level reads
-  std::vector<Unit> units;
-  std::vector<uint64_t> cost;
-  {
-    const int64_t ni = (int64_t)S.I.size(), ndl = (int64_t)S.D.size(), per = 2 * (ni + ndl);
-    const int64_t slots = (int64_t)Q.m * per;
-    std::vector<Unit> all((size_t)slots);
-    std::vector<uint64_t> ac((size_t)slots, 0);  // 0 = filtered out
-    parallel_for(T, slots, [&](int, int64_t lo, int64_t hi) {
-      for (int64_t sidx = lo; sidx < hi; ++sidx) {
-        const int term = (int)(sidx / per);
-        int64_t r = sidx % per;
-        const int o = (int)(r & 1);
-        r >>= 1;
-        const int kind = r < ni ? 0 : 1;
-        const uint64_t key = kind ? S.D[r - ni] : S.I[r];
-        const DevPlan &P = Q.plans[2 * term + kind];
-        const int32_t x = (int32_t)(key >> 32), y = (int32_t)(key & 0xffffffffu);
-        const int32_t a = o ? y : x, b = o ? x : y;
-        if (P.label0 >= 0 && host_label(S, a) != P.label0) continue;
-        if (P.label1 >= 0 && host_label(S, b) != P.label1) continue;
-        all[sidx] = Unit{a, b, 2 * term + kind, 0};
-        uint64_t c = 1;
-        if (k > 2) {
-          const LevelPlan &L2 = P.lv[2];
-          const int32_t f[2] = {a, b};
-          for (int bb = 0; bb < L2.nb; ++bb) c += S.view_len(f[L2.bpos[bb]], L2.bview[bb]);
-        }
-        ac[sidx] = c;
-      }
-    });
-    units.reserve((size_t)slots);
-    cost.reserve((size_t)slots);
-    for (int64_t sidx = 0; sidx < slots; ++sidx)
-      if (ac[sidx]) {
-        units.push_back(all[sidx]);
-        cost.push_back(ac[sidx]);
-      }
-  }
-  if (ctx->opt.world > 1) {
-    std::vector<int32_t> rk(units.size());
-    shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data());
-    size_t w = 0;
-    for (size_t i = 0; i < units.size(); ++i)
-      if (rk[i] == ctx->opt.rank) {
-        units[w] = units[i];
-        cost[w] = cost[i];
-        ++w;
-      }
-    units.resize(w);
-    cost.resize(w);
-  }
-  {  // heaviest units first (dynamic scheduling tail)
-    std::vector<size_t> idx(units.size());
-    std::iota(idx.begin(), idx.end(), 0);
-    parallel_sort(idx, [&](size_t x, size_t y) { return cost[x] > cost[y]; }, T, /*stable=*/true);
-    std::vector<Unit> u2(units.size());
-    std::vector<uint64_t> c2(units.size());
-    for (size_t i = 0; i < idx.size(); ++i) {
-      u2[i] = units[idx[i]];
-      c2[i] = cost[idx[i]];
-    }
-    units.swap(u2);
-    cost.swap(c2);
-  }
-  const int64_t nu = (int64_t)units.size();
-  tr.mark("units");
-  st.units = st.n1 = (uint64_t)nu;
   const uint64_t D = std::max<uint64_t>(1, std::max<uint64_t>(S.maxdeg, S.maxdeg_new));
+  std::vector<std::vector<Unit>> qunits((size_t)nq);
+  std::vector<int64_t> qnu((size_t)nq, 0);
+  for (int qi = 0; qi < nq; ++qi) {
+    const QueryPlan &Q = ctx->qs[qi].qp;
+    const int k = Q.k;
+    std::vector<Unit> &units = qunits[qi];
+    // level-1 units: (term, kind, changed edge, orientation) slots enumerated in parallel, then compacted in slot
+    // order (deterministic); the cost proxy of a unit is the list lengths its first level reads
+    std::vector<uint64_t> cost;
+    {
+      const int64_t ni = (int64_t)S.I.size(), ndl = (int64_t)S.D.size(), per = 2 * (ni + ndl);
+      const int64_t slots = (int64_t)Q.m * per;
+      std::vector<Unit> all((size_t)slots);
+      std::vector<uint64_t> ac((size_t)slots, 0);  // 0 = filtered out
+      parallel_for(T, slots, [&](int, int64_t lo, int64_t hi) {
+        for (int64_t sidx = lo; sidx < hi; ++sidx) {
+          const int term = (int)(sidx / per);
+          int64_t r = sidx % per;
+          const int o = (int)(r & 1);
+          r >>= 1;
+          const int kind = r < ni ? 0 : 1;
+          const uint64_t key = kind ? S.D[r - ni] : S.I[r];
+          const DevPlan &P = Q.plans[2 * term + kind];
+          const int32_t x = (int32_t)(key >> 32), y = (int32_t)(key & 0xffffffffu);
+          const int32_t a = o ? y : x, b = o ? x : y;
+          if (P.label0 >= 0 && host_label(S, a) != P.label0) continue;
+          if (P.label1 >= 0 && host_label(S, b) != P.label1) continue;
+          all[sidx] = Unit{a, b, 2 * term + kind, 0};
+          uint64_t c = 1;
+          if (k > 2) {
+            const LevelPlan &L2 = P.lv[2];
+            const int32_t f[2] = {a, b};
+            for (int bb = 0; bb < L2.nb; ++bb) c += S.view_len(f[L2.bpos[bb]], L2.bview[bb]);
+          }
+          ac[sidx] = c;
+        }
+      });
+      units.reserve((size_t)slots);
+      cost.reserve((size_t)slots);
+      for (int64_t sidx = 0; sidx < slots; ++sidx)
+        if (ac[sidx]) {
+          units.push_back(all[sidx]);
+          cost.push_back(ac[sidx]);
+        }
+    }
+    if (ctx->opt.world > 1) {
+      std::vector<int32_t> rk(units.size());
+      shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data());
+      size_t w = 0;
+      for (size_t i = 0; i < units.size(); ++i)
+        if (rk[i] == ctx->opt.rank) {
+          units[w] = units[i];
+          cost[w] = cost[i];
+          ++w;
+        }
+      units.resize(w);
+      cost.resize(w);
+    }
+    {  // heaviest units first (dynamic scheduling tail)
+      std::vector<size_t> idx(units.size());
+      std::iota(idx.begin(), idx.end(), 0);
+      parallel_sort(idx, [&](size_t x, size_t y) { return cost[x] > cost[y]; }, T, /*stable=*/true);
+      std::vector<Unit> u2(units.size());
+      std::vector<uint64_t> c2(units.size());
+      for (size_t i = 0; i < idx.size(); ++i) {
+        u2[i] = units[idx[i]];
+        c2[i] = cost[idx[i]];
+      }
+      units.swap(u2);
+      cost.swap(c2);
+    }
+
+    qnu[qi] = (int64_t)units.size();
+  }
+  tr.mark("units");
+  st.units = st.n1 = (uint64_t)qnu[0];
   st.max_degree = D;
   st.ms_normalize = t1.ms();
 
-  // ---- (2) estimator ---------------------------------------------------------------------
+  // ---- (2) estimator (per query; one ranking: the sum of the queries' estimated accesses per vertex) -------
   Timer t2;
-  ctx->est.ids.clear();
-  ctx->est.levcnt.clear();
   std::vector<std::pair<double, int32_t>> ranked;  // (score, id)
-  const bool use_cache = ctx->budget > 0 && ctx->opt.cache_policy != GCSM_CACHE_NONE && k > 2;
-  uint64_t M = 0;
-  if (k > 2 && nu > 0) {
-    M = ctx->opt.walks_override ? ctx->opt.walks_override : walk_budget((uint64_t)nu, D, k);
-    st.walks = M;
-    if (ctx->opt.cache_policy == GCSM_CACHE_ESTIMATOR && ctx->budget > 0) {
-      EstimatorInput in;
-      in.plans = Q.plans.data();
-      in.units = units.data();
-      in.n_units = nu;
-      in.N1 = (uint64_t)nu;
-      in.D = D;
-      in.M = M;
-      in.seed = ctx->opt.seed;
-      in.batch_seq = ctx->batch_seq;
-      in.labels = S.lab.empty() ? nullptr : S.lab.data();
-      in.threads = T;
-      in.view = [&S](int32_t v, int vw) { return S.view(v, vw); };
-      in.n = S.n;
-      run_estimator(in, ctx->est_scratch, ctx->est);
-      tr.mark("walks");
-      if (use_cache) {
-        ranked.resize(ctx->est.ids.size());
-        parallel_for(T, (int64_t)ranked.size(), [&](int, int64_t lo, int64_t hi) {
-          for (int64_t i = lo; i < hi; ++i)
-            ranked[i] = {estimate_value(&ctx->est.levcnt[8 * i], k, (uint64_t)nu, D, M), ctx->est.ids[i]};
-        });
+  const bool use_cache = ctx->budget > 0 && ctx->opt.cache_policy != GCSM_CACHE_NONE && kmax > 2;
+  std::vector<double> qms_est((size_t)nq, 0.0);
+  std::vector<uint64_t> qwalks((size_t)nq, 0);
+  for (int qi = 0; qi < nq; ++qi) {
+    Timer tq;
+    const QueryPlan &Q = ctx->qs[qi].qp;
+    const int k = Q.k;
+    const int64_t nu = qnu[qi];
+    EstimatorOutput &est = ctx->qs[qi].est;
+    est.ids.clear();
+    est.levcnt.clear();
+    if (k > 2 && nu > 0) {
+      const uint64_t M = ctx->opt.walks_override ? ctx->opt.walks_override : walk_budget((uint64_t)nu, D, k);
+      qwalks[qi] = M;
+      if (ctx->opt.cache_policy == GCSM_CACHE_ESTIMATOR && ctx->budget > 0) {
+        EstimatorInput in;
+        in.plans = Q.plans.data();
+        in.units = qunits[qi].data();
+        in.n_units = nu;
+        in.N1 = (uint64_t)nu;
+        in.D = D;
+        in.M = M;
+        in.seed = qi == 0 ? ctx->opt.seed : rng_chain(ctx->opt.seed, 0x51ull + (uint64_t)qi);  // own stream per query
+        in.batch_seq = ctx->batch_seq;
+        in.labels = S.lab.empty() ? nullptr : S.lab.data();
+        in.threads = T;
+        in.view = [&S](int32_t v, int vw) { return S.view(v, vw); };
+        in.n = S.n;
+        run_estimator(in, ctx->est_scratch, est);
+        tr.mark("walks");
+        if (use_cache) {
+          std::vector<std::pair<double, int32_t>> r(est.ids.size());
+          parallel_for(T, (int64_t)r.size(), [&](int, int64_t lo, int64_t hi) {
+            for (int64_t i = lo; i < hi; ++i)
+              r[i] = {estimate_value(&est.levcnt[8 * i], k, (uint64_t)nu, D, M), est.ids[i]};
+          });
+          if (ranked.empty()) {
+            ranked.swap(r);
+          } else {  // both ascending by id: merge, summing the scores of a vertex both queries access
+            std::vector<std::pair<double, int32_t>> m2;
+            m2.reserve(ranked.size() + r.size());
+            size_t x = 0, y = 0;
+            while (x < ranked.size() || y < r.size()) {
+              if (y == r.size() || (x < ranked.size() && ranked[x].second < r[y].second)) m2.push_back(ranked[x++]);
+              else if (x == ranked.size() || r[y].second < ranked[x].second) m2.push_back(r[y++]);
+              else {
+                m2.push_back({ranked[x].first + r[y].first, ranked[x].second});
+                ++x;
+                ++y;
+              }
+            }
+            ranked.swap(m2);
+          }
+        }
       }
     }
+    qms_est[qi] = tq.ms();
   }
+  st.walks = qwalks[0];
   if (use_cache && ctx->opt.cache_policy == GCSM_CACHE_DEGREE) {
     ranked.reserve(S.n);
     for (int32_t v = 0; v < S.n; ++v) {
@@ -502,17 +584,22 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // symmetry breaking (count mode): the kernels walk only the canonical embedding of every Aut_L orbit and the
   // counts are scaled by |Aut_L| (Emb(G') \ Emb(G) is a union of orbits); the estimator above samples the full
   // execution trees of the paper. Seeds violating a restriction between the two seed endpoints are dropped here.
-  const bool sym = !listing && ctx->qps.symmetry;
-  const QueryPlan &QK = sym ? ctx->qps : Q;
-  if (sym) {
-    size_t w = 0;
-    for (size_t i = 0; i < units.size(); ++i) {
-      const int rel = QK.plans[units[i].plan].seed_rel;
-      if (rel == 0 || (rel == 1 ? units[i].a < units[i].b : units[i].a > units[i].b)) units[w++] = units[i];
+  std::vector<int64_t> uoff((size_t)nq + 1, 0);
+  for (int qi = 0; qi < nq; ++qi) {
+    const bool sym = !listing && ctx->qs[qi].qps.symmetry;
+    std::vector<Unit> &units = qunits[qi];
+    if (sym) {
+      const QueryPlan &QK = ctx->qs[qi].qps;
+      size_t w = 0;
+      for (size_t i = 0; i < units.size(); ++i) {
+        const int rel = QK.plans[units[i].plan].seed_rel;
+        if (rel == 0 || (rel == 1 ? units[i].a < units[i].b : units[i].a > units[i].b)) units[w++] = units[i];
+      }
+      units.resize(w);
     }
-    units.resize(w);
+    uoff[qi + 1] = uoff[qi] + (int64_t)units.size();
   }
-  const int64_t gnu = (int64_t)units.size();
+  const int64_t gnu = uoff[nq];
 
   // ---- (3) pack the cache + descriptors --------------------------------------------------
   Timer t3;
@@ -672,7 +759,9 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
                           S.del_off[i + 1] - S.del_off[i]};
   std::memcpy(sl.h_dlist, S.ins_val.data(), S.ins_val.size() * 4);
   std::memcpy(sl.h_dlist + S.ins_val.size(), S.del_val.data(), S.del_val.size() * 4);
-  std::memcpy(sl.h_units, units.data(), sizeof(Unit) * (size_t)gnu);
+  for (int qi = 0; qi < nq; ++qi)
+    if (!qunits[qi].empty())
+      std::memcpy(sl.h_units + uoff[qi], qunits[qi].data(), sizeof(Unit) * qunits[qi].size());
   st.ms_pack = t3.ms();
   tr.mark("staging");
 
@@ -711,50 +800,57 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
                  4 * nd + sizeof(Unit) * (size_t)gnu;
 
-  // ---- (4) matching kernels --------------------------------------------------------------
+  // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
-  const int nbuf = std::max(1, std::max(k - 4, 0) + (listing ? 1 : 0));
+  const int nbuf = std::max(1, std::max(kmax - 4, 0) + (listing ? 1 : 0));
   const size_t stride = (size_t)(nbuf + 3) * (size_t)dcap;  // stacks + pinned-x2 + 2 HBM staging buffers
   if (!dev_ensure(ctx->d_scratch, ctx->scratch_cap, stride * (size_t)ctx->warps_total))
     return ctx->fail(GCSM_ENOMEM, "scratch");
-  // level-2 frontier chunks: per unit an upper bound on its candidates
-  std::vector<std::pair<int64_t, int64_t>> chunks;
+  // level-2 frontier chunks: per unit an upper bound on its candidates (unit indices local to the query)
+  std::vector<std::vector<std::pair<int64_t, int64_t>>> qchunks((size_t)nq);
   int64_t f2_need = 0;
-  if (k >= 4) {
-    int64_t start = 0, acc = 0;
-    for (int64_t i = 0; i < gnu; ++i) {
-      const DevPlan &P = QK.plans[units[i].plan];
-      const LevelPlan &L2 = P.lv[2];
-      const int32_t f[2] = {units[i].a, units[i].b};
-      int64_t b = INT64_MAX;
-      for (int j = 0; j < L2.nb; ++j) b = std::min<int64_t>(b, S.view_len(f[L2.bpos[j]], L2.bview[j]));
-      if (acc + b > kF2CapLimit && i > start) {
-        chunks.push_back({start, i});
-        f2_need = std::max(f2_need, acc);
-        start = i;
-        acc = 0;
+  for (int qi = 0; qi < nq; ++qi) {
+    const bool sym = !listing && ctx->qs[qi].qps.symmetry;
+    const QueryPlan &QK = sym ? ctx->qs[qi].qps : ctx->qs[qi].qp;
+    const std::vector<Unit> &units = qunits[qi];
+    const int64_t qn = (int64_t)units.size();
+    auto &chunks = qchunks[qi];
+    if (QK.k >= 4) {
+      int64_t start = 0, acc = 0;
+      for (int64_t i = 0; i < qn; ++i) {
+        const DevPlan &P = QK.plans[units[i].plan];
+        const LevelPlan &L2 = P.lv[2];
+        const int32_t f[2] = {units[i].a, units[i].b};
+        int64_t b = INT64_MAX;
+        for (int j = 0; j < L2.nb; ++j) b = std::min<int64_t>(b, S.view_len(f[L2.bpos[j]], L2.bview[j]));
+        if (acc + b > kF2CapLimit && i > start) {
+          chunks.push_back({start, i});
+          f2_need = std::max(f2_need, acc);
+          start = i;
+          acc = 0;
+        }
+        acc += b;
       }
-      acc += b;
+      chunks.push_back({start, qn});
+      f2_need = std::max(f2_need, acc);
+    } else {
+      chunks.push_back({0, qn});
     }
-    chunks.push_back({start, gnu});
-    f2_need = std::max(f2_need, acc);
-    if (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)) ||
-        !dev_ensure(ctx->d_group, ctx->group_cap, (size_t)std::max<int64_t>(f2_need, 1)))
-      return ctx->fail(GCSM_ENOMEM, "frontier");
-  } else {
-    chunks.push_back({0, gnu});
   }
-  // list mode buffers
+  if (kmax >= 4 && (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)) ||
+                    !dev_ensure(ctx->d_group, ctx->group_cap, (size_t)std::max<int64_t>(f2_need, 1))))
+    return ctx->fail(GCSM_ENOMEM, "frontier");
+  // list mode buffers (one query)
   int32_t *d_tadd = nullptr, *d_trem = nullptr;
   if (listing) {
+    const int k = ctx->qs[0].qp.k;
     const size_t need = (size_t)k * (add_cap + rem_cap);
     if (!dev_ensure(ctx->d_tup, ctx->tup_cap, std::max<size_t>(need, 1))) return ctx->fail(GCSM_ENOMEM, "tuples");
     d_tadd = ctx->d_tup;
     d_trem = ctx->d_tup + (size_t)k * add_cap;
   }
-  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N, s));
+  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
   MatchArgs A{};
-  A.plans = sym ? ctx->d_splans : ctx->d_plans;
   A.vdesc = ctx->d_vdesc;
   A.lab = ctx->d_lab;
   A.drec = ctx->d_drec;
@@ -766,83 +862,109 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.scratch_end = ctx->d_scratch + stride * (size_t)ctx->warps_total;
   A.scratch_stride = (int64_t)stride;
   A.dcap = dcap;
-  A.cnt = ctx->d_cnt;
   A.cache_lo = ctx->d_cache;
   A.cache_hi = ctx->d_cache ? ctx->d_cache + ctx->cache_cap : nullptr;
   A.tup_add = d_tadd;
   A.tup_add_cap = add_cap;
   A.tup_rem = d_trem;
   A.tup_rem_cap = rem_cap;
-  A.k = k;
-  A.n_plans = (int32_t)QK.plans.size();
   A.listing = listing ? 1 : 0;
-  if (k >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
+  if (kmax >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
     const size_t na = (size_t)64 << 20, nt = (size_t)4 << 20;
     const bool fresh_ready = ctx->d_task_ready == nullptr;
     if (!dev_ensure(ctx->d_arena, ctx->arena_cap, na) || !dev_ensure(ctx->d_tasks, ctx->tasks_cap, nt) ||
         !dev_ensure(ctx->d_task_ready, ctx->task_ready_cap, nt))
       return ctx->fail(GCSM_ENOMEM, "work-sharing buffers");
     if (fresh_ready) CK(cudaMemsetAsync(ctx->d_task_ready, 0, 4 * ctx->task_ready_cap, s));
-    A.arena = ctx->d_arena;
-    A.arena_cap = ctx->arena_cap;
-    A.tasks = ctx->d_tasks;
-    A.task_ready = ctx->d_task_ready;
-    A.task_cap = (uint32_t)std::min<size_t>(ctx->tasks_cap, ctx->task_ready_cap);
   }
-  CK(cudaEventRecord(sl.ev_m0, s));
-  size_t nev = 0;
-  for (const auto &ch : chunks) {
-    if (ch.second <= ch.first) continue;
-    A.units = ctx->d_units + ch.first;
-    A.n_units = ch.second - ch.first;
-    while (sl.kev.size() < nev + 3) {
-      cudaEvent_t ev;
-      CK(cudaEventCreate(&ev));
-      sl.kev.push_back(ev);
+  while (sl.q.size() < (size_t)nq) {
+    sl.q.emplace_back();
+    CK(cudaEventCreate(&sl.q.back().ev_m0));
+    CK(cudaEventCreate(&sl.q.back().ev_m1));
+  }
+  for (int qi = 0; qi < nq; ++qi) {
+    auto &pq = sl.q[qi];
+    const bool sym = !listing && ctx->qs[qi].qps.symmetry;
+    const QueryPlan &QK = sym ? ctx->qs[qi].qps : ctx->qs[qi].qp;
+    const int k = QK.k;
+    unsigned long long *qcnt = ctx->d_cnt + (size_t)qi * CNT_N;
+    A.plans = sym ? ctx->qs[qi].d_splans : ctx->qs[qi].d_plans;
+    A.n_plans = (int32_t)QK.plans.size();
+    A.k = k;
+    A.cnt = qcnt;
+    A.group = nullptr;
+    A.tasks = nullptr;
+    if (k >= 5 && !listing) {
+      A.arena = ctx->d_arena;
+      A.arena_cap = ctx->arena_cap;
+      A.tasks = ctx->d_tasks;
+      A.task_ready = ctx->d_task_ready;
+      A.task_cap = (uint32_t)std::min<size_t>(ctx->tasks_cap, ctx->task_ready_cap);
     }
-    // reset the work cursors and the frontier size of this chunk
-    CK(cudaMemsetAsync(ctx->d_cnt + CNT_F2, 0, sizeof(unsigned long long), s));
-    CK(cudaMemsetAsync(ctx->d_cnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), s));
-    CK(cudaEventRecord(sl.kev[nev], s));
-    CK(launch_level2(A, ctx->grid, s));
-    CK(cudaEventRecord(sl.kev[nev + 1], s));
-    ++launches;
-    if (k >= 4) {
-      CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_group, s));
-      launches += 6;
-      A.group = ctx->d_group;
-      if (A.tasks) {
-        if (++ctx->task_gen <= 0) ctx->task_gen = 1;  // ready flags hold the launch's generation, never 0
-        A.task_gen = ctx->task_gen;
+    CK(cudaEventRecord(pq.ev_m0, s));
+    size_t nev = 0;
+    for (const auto &ch : qchunks[qi]) {
+      if (ch.second <= ch.first) continue;
+      A.units = ctx->d_units + uoff[qi] + ch.first;
+      A.n_units = ch.second - ch.first;
+      while (pq.kev.size() < nev + 3) {
+        cudaEvent_t ev;
+        CK(cudaEventCreate(&ev));
+        pq.kev.push_back(ev);
       }
-      CK(launch_extend(A, ctx->grid, s));
+      // reset the work cursors and the frontier size of this chunk
+      CK(cudaMemsetAsync(qcnt + CNT_F2, 0, sizeof(unsigned long long), s));
+      CK(cudaMemsetAsync(qcnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), s));
+      CK(cudaEventRecord(pq.kev[nev], s));
+      CK(launch_level2(A, ctx->grid, s));
+      CK(cudaEventRecord(pq.kev[nev + 1], s));
       ++launches;
+      if (k >= 4) {
+        CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_group, s));
+        launches += 6;
+        A.group = ctx->d_group;
+        if (A.tasks) {
+          if (++ctx->task_gen <= 0) ctx->task_gen = 1;  // ready flags hold the launch's generation, never 0
+          A.task_gen = ctx->task_gen;
+        }
+        CK(launch_extend(A, ctx->grid, s));
+        ++launches;
+      }
+      CK(cudaEventRecord(pq.kev[nev + 2], s));
+      nev += 3;
     }
-    CK(cudaEventRecord(sl.kev[nev + 2], s));
-    nev += 3;
+    CK(cudaEventRecord(pq.ev_m1, s));
+    pq.nev = nev;
+    pq.aut_mul = sym ? QK.automorphisms : 1;
   }
-  CK(cudaEventRecord(sl.ev_m1, s));
   // ---- (4b) count allreduce over NVLink (world > 1) -------------------------------------
   CK(cudaEventRecord(sl.ev_a0, s));
   if (ctx->comm) {
-    if (ncclAllReduce(ctx->d_cnt, ctx->d_cnt, 2, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
-      return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
+    for (int qi = 0; qi < nq; ++qi) {
+      unsigned long long *qcnt = ctx->d_cnt + (size_t)qi * CNT_N;
+      if (ncclAllReduce(qcnt, qcnt, 2, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
+        return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
+    }
   }
   CK(cudaEventRecord(sl.ev_a1, s));
-  CK(cudaMemcpyAsync(sl.h_cnt, ctx->d_cnt, sizeof(unsigned long long) * CNT_N, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(sl.h_cnt, ctx->d_cnt, sizeof(unsigned long long) * CNT_N * (size_t)nq, cudaMemcpyDeviceToHost,
+                     s));
   CK(cudaEventRecord(sl.ev_done, s));
-  sl.nev = nev;
-  sl.st = st;
-  sl.st.kernel_launches = launches;
+  st.kernel_launches = launches;
+  for (int qi = 0; qi < nq; ++qi) {  // shared steps' times and sizes, plus the query's own
+    gcsm_stats &q = sl.q[qi].st;
+    q = st;
+    q.units = q.n1 = (uint64_t)qnu[qi];
+    q.walks = qwalks[qi];
+    q.ms_estimate = qms_est[qi];
+  }
   sl.tup_add = tup_add;
   sl.tup_rem = tup_rem;
   sl.d_tadd = d_tadd;
   sl.d_trem = d_trem;
   sl.add_cap = add_cap;
   sl.rem_cap = rem_cap;
-  sl.aut_mul = sym ? QK.automorphisms : 1;
   tr.mark("enqueue");
-
   // ---- (5) reorganise the host lists. P:302 runs it after matching so the kernel reads consistent data: here
   // the merge writes fresh arrays and the ones the in-flight kernels may read are retired, not overwritten.
   Timer t5;
@@ -860,7 +982,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   ctx->cached = ctx->prev_cached;
   ctx->prev_U = S.U;
   S.clear_batch();
-  sl.st.ms_merge = t5.ms();
+  for (auto &pq : sl.q) pq.st.ms_merge = t5.ms();
   ++ctx->batch_seq;
   sl.inflight = true;
   sl.host_ms = total.ms();
@@ -868,6 +990,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   ctx->err.clear();
   return GCSM_OK;
 }
+
 
 // Waits for the oldest in-flight batch and collects its counts and statistics.
 static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) {
@@ -877,55 +1000,60 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
   Timer tw;
   auto &sl = ctx->slots[ctx->waited & 1];
   CK(cudaEventSynchronize(sl.ev_done));
-  gcsm_stats st = sl.st;
-  const int k = ctx->qp.k;
-  if (sl.h_cnt[CNT_OVERFLOW]) return ctx->fail(GCSM_EDEVICE, "internal: level-2 frontier overflow");
-  float ms_m = 0, ms_a = 0, ms_c = 0;
-  cudaEventElapsedTime(&ms_m, sl.ev_m0, sl.ev_m1);
+  const int nq = (int)ctx->qs.size();
+  float ms_a = 0, ms_c = 0;
   cudaEventElapsedTime(&ms_a, sl.ev_a0, sl.ev_a1);
   cudaEventElapsedTime(&ms_c, sl.ev_c0, sl.ev_c1);
-  st.ms_match = ms_m;
-  st.ms_allreduce = ms_a;
-  st.ms_copy = ms_c;
-  for (size_t i = 0; i < sl.nev; i += 3) {
-    float a = 0, b = 0;
-    cudaEventElapsedTime(&a, sl.kev[i], sl.kev[i + 1]);
-    cudaEventElapsedTime(&b, sl.kev[i + 1], sl.kev[i + 2]);
-    st.ms_level2 += a;
-    st.ms_extend += b;
-  }
-  const unsigned long long *h = sl.h_cnt;
-  st.added = h[CNT_ADDED] * sl.aut_mul;
-  st.removed = h[CNT_REMOVED] * sl.aut_mul;
-  st.hit_bytes_ext = h[CNT_ACC_EXT + 0];
-  st.miss_bytes_ext = h[CNT_ACC_EXT + 1];
-  st.delta_bytes_ext = h[CNT_ACC_EXT + 2];
-  st.hit_bytes = h[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
-  st.miss_bytes = h[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
-  st.delta_bytes = h[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
-  st.host_copied_bytes = h[CNT_COPIED];
-  st.d2h_bytes = sizeof(unsigned long long) * CNT_N;
-  st.frontier = h[CNT_F2];
-  if (std::getenv("GCSM_TRACE"))
-    std::fprintf(stderr, "[gcsm kern] frontier=%llu runs=%llu pins=%llu pin_gb=%.3f copied_gb=%.3f\n", h[CNT_F2],
-                 h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_COPIED] / 1e9);
   bool trunc = false;
-  if (sl.tup_add || sl.tup_rem) {
-    const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);
-    const uint64_t nr = std::min<uint64_t>(h[CNT_TUP_REM], sl.rem_cap);
-    if (na) CK(cudaMemcpy(sl.tup_add, sl.d_tadd, sizeof(int32_t) * k * na, cudaMemcpyDeviceToHost));
-    if (nr) CK(cudaMemcpy(sl.tup_rem, sl.d_trem, sizeof(int32_t) * k * nr, cudaMemcpyDeviceToHost));
-    st.d2h_bytes += sizeof(int32_t) * k * (na + nr);
-    trunc = h[CNT_TUP_ADD] > sl.add_cap || h[CNT_TUP_REM] > sl.rem_cap;
-    sl.tup_add = sl.tup_rem = nullptr;
+  for (int qi = 0; qi < nq; ++qi) {
+    auto &pq = sl.q[qi];
+    gcsm_stats st = pq.st;
+    const unsigned long long *h = sl.h_cnt + (size_t)qi * CNT_N;
+    if (h[CNT_OVERFLOW]) return ctx->fail(GCSM_EDEVICE, "internal: level-2 frontier overflow");
+    float ms_m = 0;
+    cudaEventElapsedTime(&ms_m, pq.ev_m0, pq.ev_m1);
+    st.ms_match = ms_m;
+    st.ms_allreduce = ms_a;
+    st.ms_copy = ms_c;
+    for (size_t i = 0; i < pq.nev; i += 3) {
+      float a = 0, b = 0;
+      cudaEventElapsedTime(&a, pq.kev[i], pq.kev[i + 1]);
+      cudaEventElapsedTime(&b, pq.kev[i + 1], pq.kev[i + 2]);
+      st.ms_level2 += a;
+      st.ms_extend += b;
+    }
+    st.added = h[CNT_ADDED] * pq.aut_mul;
+    st.removed = h[CNT_REMOVED] * pq.aut_mul;
+    st.hit_bytes_ext = h[CNT_ACC_EXT + 0];
+    st.miss_bytes_ext = h[CNT_ACC_EXT + 1];
+    st.delta_bytes_ext = h[CNT_ACC_EXT + 2];
+    st.hit_bytes = h[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
+    st.miss_bytes = h[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
+    st.delta_bytes = h[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
+    st.host_copied_bytes = h[CNT_COPIED];
+    st.d2h_bytes = sizeof(unsigned long long) * CNT_N * (size_t)nq;
+    st.frontier = h[CNT_F2];
+    if (std::getenv("GCSM_TRACE"))
+      std::fprintf(stderr, "[gcsm kern] q=%d frontier=%llu runs=%llu pins=%llu pin_gb=%.3f copied_gb=%.3f\n", qi,
+                   h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_COPIED] / 1e9);
+    if (qi == 0 && (sl.tup_add || sl.tup_rem)) {
+      const int k = ctx->qs[0].qp.k;
+      const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);
+      const uint64_t nr = std::min<uint64_t>(h[CNT_TUP_REM], sl.rem_cap);
+      if (na) CK(cudaMemcpy(sl.tup_add, sl.d_tadd, sizeof(int32_t) * k * na, cudaMemcpyDeviceToHost));
+      if (nr) CK(cudaMemcpy(sl.tup_rem, sl.d_trem, sizeof(int32_t) * k * nr, cudaMemcpyDeviceToHost));
+      st.d2h_bytes += sizeof(int32_t) * k * (na + nr);
+      trunc = h[CNT_TUP_ADD] > sl.add_cap || h[CNT_TUP_REM] > sl.rem_cap;
+      sl.tup_add = sl.tup_rem = nullptr;
+    }
+    st.ms_total = sl.host_ms + tw.ms();
+    ctx->qs[qi].stats = st;
   }
   ctx->store.recycle(sl.retired);  // arrays the batch's kernels could read are free again
   sl.inflight = false;
   ++ctx->waited;
-  st.ms_total = sl.host_ms + tw.ms();
-  ctx->stats = st;
-  if (added) *added = st.added;
-  if (removed) *removed = st.removed;
+  if (added) *added = ctx->qs[0].stats.added;
+  if (removed) *removed = ctx->qs[0].stats.removed;
   if (trunc) return ctx->fail(GCSM_ETRUNC, "tuple buffer too small");
   ctx->err.clear();
   return GCSM_OK;
@@ -969,12 +1097,22 @@ gcsm_status gcsm_wait_batch(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) {
 
 gcsm_status gcsm_get_stats(const gcsm_ctx *ctx, gcsm_stats *out) {
   if (!ctx || !out) return GCSM_EINVAL;
-  *out = ctx->stats;
+  if (ctx->qs.empty()) {
+    std::memset(out, 0, sizeof *out);
+    return GCSM_OK;
+  }
+  *out = ctx->qs[0].stats;
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_get_query_stats(const gcsm_ctx *ctx, int32_t qid, gcsm_stats *out) {
+  if (!ctx || !out || qid < 0 || (size_t)qid >= ctx->qs.size()) return GCSM_EINVAL;
+  *out = ctx->qs[qid].stats;
   return GCSM_OK;
 }
 
 uint64_t gcsm_query_automorphisms(const gcsm_ctx *ctx) {
-  return ctx && ctx->has_query ? ctx->qp.automorphisms : 0;
+  return ctx && ctx->has_query ? ctx->qs[0].qp.automorphisms : 0;
 }
 
 gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col, uint64_t col_cap) {
@@ -990,11 +1128,13 @@ gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col,
 
 gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levcnt, uint64_t cap, uint64_t *n_out) {
   if (!ctx || !n_out) return GCSM_EINVAL;
-  const uint64_t n = ctx->est.ids.size();
+  static const EstimatorOutput none;
+  const EstimatorOutput &est = ctx->qs.empty() ? none : ctx->qs[0].est;
+  const uint64_t n = est.ids.size();
   *n_out = n;
   const uint64_t w = std::min(n, cap);
-  if (ids && w) std::memcpy(ids, ctx->est.ids.data(), 4 * w);
-  if (levcnt && w) std::memcpy(levcnt, ctx->est.levcnt.data(), 8 * 8 * w);
+  if (ids && w) std::memcpy(ids, est.ids.data(), 4 * w);
+  if (levcnt && w) std::memcpy(levcnt, est.levcnt.data(), 8 * 8 * w);
   return n > cap ? GCSM_ETRUNC : GCSM_OK;
 }
 

@@ -364,16 +364,19 @@ def test_full_size_sampled(G, cfg, queries):
     w = gi.make_workload(cfg, n_batches=2)
     ins, dele = w.batches[0]
     si, sd = ins[:128], dele[:128]
-    for q in queries:
+    g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=0)  # bench.py: one context holding every query
+    for i, q in enumerate(queries):
+        k, qe, ql = gi.query(q)
+        (g.set_query if i == 0 else g.add_query)(k, qe, ql)
+    g.set_cache_budget(int(w.adj_bytes * w.budget_frac))
+    g.apply_batch(si, sd)
+    for i, q in enumerate(queries):
         k, qe, ql = gi.query(q)
         want = oracle.delta(w.n, w.row_ptr, w.col, w.labels, k, qe, ql, si, sd)
-        g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=0)
-        g.set_query(k, qe, ql)
-        g.set_cache_budget(int(w.adj_bytes * w.budget_frac))
-        assert g.apply_batch(si, sd) == want, q
-        st = g.stats()
+        assert g.query_counts(i) == want, q
+        st = g.query_stats(i)
         assert st["cached_vertices"] > 0 and st["hit_bytes"] > 0
-        g.close()
+    g.close()
 
 
 @pytest.mark.parametrize("r", [2, 3])
@@ -425,3 +428,60 @@ def test_symmetry_breaking_on_off(G, name):
     on, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.1, symmetry=True)
     off, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.1, symmetry=False)
     assert on == want and off == want
+
+
+# ------------------------------------------------------------------ standing queries sharing one context
+
+@pytest.mark.parametrize("policy", ["estimator", "degree", "none"])
+def test_multi_query_context(G, policy):
+    """gcsm_add_query: several queries share the store, the batch steps and one cache budget; every query's
+    counts equal the oracle's on every batch (mixed k, labels off, pipelined submit/wait)."""
+    names = ["k4", "c4", "triangle", "house5u", "path4"]
+    w = gi.make_workload("C2", scale=12, n_edges=40_000, batch=256, n_batches=4)
+    want = {q: oracle_run(w.n, w.row_ptr, w.col, None, q, w.batches)[0] for q in names}
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0, cache_policy=policy)
+    k, qe, ql = gi.query(names[0])
+    g.set_query(k, qe, ql)
+    for i, q in enumerate(names[1:], 1):
+        k, qe, ql = gi.query(q)
+        assert g.add_query(k, qe, ql) == i
+    assert g.num_queries() == len(names)
+    g.set_cache_budget(w.adj_bytes // 10)
+    got = {q: [] for q in names}
+    g.submit_batch(*w.batches[0])
+    for b in list(w.batches[1:]) + [None]:
+        if b is not None:
+            g.submit_batch(*b)
+        a0 = g.wait_batch()
+        for i, q in enumerate(names):
+            got[q].append(g.query_counts(i))
+        assert a0 == got[names[0]][-1]
+    assert got == want
+    st = g.query_stats(1)
+    assert st["cache_bytes"] <= w.adj_bytes // 10 and st["units"] > 0
+    with pytest.raises(G.GcsmError) as ei:
+        g.apply_batch_list(np.zeros((0, 2)), np.zeros((0, 2)))
+    assert ei.value.name == "GCSM_EINVAL"
+    # set_query resets to one query
+    k, qe, ql = gi.query("triangle")
+    g.set_query(k, qe, ql)
+    assert g.num_queries() == 1
+    g.close()
+
+
+def test_multi_query_limits(G):
+    w = gi.make_workload("C2", scale=10, n_edges=5_000, batch=64, n_batches=1)
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    k, qe, ql = gi.query("triangle")
+    with pytest.raises(G.GcsmError) as ei:
+        g.add_query(k, qe, ql)  # before set_query
+    assert ei.value.name == "GCSM_ESTATE"
+    g.set_query(k, qe, ql)
+    for _ in range(7):
+        g.add_query(k, qe, ql)
+    with pytest.raises(G.GcsmError) as ei:
+        g.add_query(k, qe, ql)
+    assert ei.value.name == "GCSM_EINVAL"
+    a = g.apply_batch(*w.batches[0])
+    assert all(g.query_counts(i) == a for i in range(8))
+    g.close()
