@@ -32,6 +32,11 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 METRIC = "updated edges/sec per batch (C2: LJ-shaped 4.19M-vertex / 70M-edge R-MAT, 4-clique + 4-cycle)"
+METRICS = {"C1": "updated edges/sec per batch (C1: 1K-vertex / 8K-edge R-MAT, triangle)", "C2": METRIC,
+           "C3": "updated edges/sec per batch (C3: Orkut-shaped 3M-vertex / 120M-edge R-MAT, 8 labels, 5-vertex "
+                 "labelled patterns)",
+           "C4": "updated edges/sec per batch (C4: FR-shaped 67M-vertex / 1.8B-edge R-MAT in pinned host memory, "
+                 "6-vertex patterns, budget 1%)"}
 UNIT = "updated_edges/s"
 
 
@@ -222,7 +227,7 @@ def run_reference(args):
             edges += len(si) + len(sd)
     T = sum(times)
     v = edges / T
-    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+    line = {"impl": "reference", "metric": METRICS.get(w.name, METRIC), "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / max(len(times), 1),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic", "config": {"workload": f"{w.name} (BASELINE configs[1])", "queries": queries,
@@ -381,19 +386,25 @@ def main():
     h2d = shared["h2d_bytes"] / K + sum(8 * len(b[0]) + 8 * len(b[1]) for b in batches[args.warmup:]) / K
     d2h = shared["d2h_bytes"] / K
     line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
+        "metric": METRICS.get(w.name, METRIC), "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms_dev / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "int32", "data": "synthetic (seeded R-MAT graph + P:331 update stream, generated on the box)",
-        "config": {"workload": f"{w.name} (BASELINE configs[1]): R-MAT s=22, 70M edges, queries "
-                               f"{'+'.join(queries)}, {args.batch} mixed updates per GPU per step, cache budget "
-                               f"{frac:.0%} of adjacency", "queries": queries, "global_batch": args.batch * world,
+        "config": {"workload": f"{w.name} (BASELINE configs[{int(w.name[1:]) - 1}]): R-MAT s={w.meta['scale']}, "
+                               f"{w.meta['n_edges'] / 1e6:.0f}M edges"
+                               + (f" ({w.meta['planted'][0]} planted {w.meta['planted'][1]}-cliques)"
+                                  if w.meta['planted'][0] else "")
+                               + (f", {w.meta['L']} labels" if w.meta['L'] else "")
+                               + f", queries {'+'.join(queries)}, {args.batch} mixed updates per GPU per step, "
+                                 f"cache budget {frac:.0%} of adjacency", "queries": queries,
+                   "global_batch": args.batch * world,
                    "graph_vertices": w.n, "graph_edges": int(w.row_ptr[-1] // 2), "budget_bytes": budget,
                    "cache_policy": args.cache_policy,
                    "cache_mb": shared["cache_bytes"] / K / 2**20,
                    "parallelism": f"units LPT-sharded over {world} GPU(s); one context per GPU with all queries "
                                   f"(shared store, batch steps and cache budget), "
                                   f"{'synchronous' if args.serial else 'pipelined submit/wait'} batches",
-                   "l2": "inputs larger than L2 (560 MB pinned host graph; cache repacked every batch)"},
+                   "l2": f"inputs larger than L2 ({w.adj_bytes / 1e6:.0f} MB pinned host graph; cache repacked "
+                         f"every batch)"},
         "roofline": roofline,
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)},

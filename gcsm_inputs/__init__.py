@@ -29,7 +29,8 @@ def _load():
         P = ctypes.c_void_p
         lib.gi_rmat_edges.restype = ctypes.c_int64
         lib.gi_rmat_edges.argtypes = [ctypes.c_int32, ctypes.c_int64, ctypes.c_double, ctypes.c_double,
-                                      ctypes.c_double, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int32, P]
+                                      ctypes.c_double, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int32, P,
+                                      ctypes.c_int64, ctypes.c_int32]
         lib.gi_build_csr.restype = ctypes.c_int32
         lib.gi_build_csr.argtypes = [ctypes.c_int32, ctypes.c_int64, P, ctypes.c_int32, P, P]
         lib.gi_labels.restype = None
@@ -51,10 +52,14 @@ def _threads() -> int:
 # ---------------------------------------------------------------- graphs
 
 def rmat_edges(scale: int, n_edges: int, a: float, b: float, c: float, seed: int,
-               id_limit: int = 0) -> np.ndarray:
-    """Exactly ``n_edges`` unique undirected R-MAT edges as an int32 [m,2] array (u<v)."""
+               id_limit: int = 0, planted: tuple = (0, 0)) -> np.ndarray:
+    """Exactly ``n_edges`` unique undirected R-MAT edges as an int32 [m,2] array (u<v).
+
+    ``planted=(groups, size)``: the edges of ``groups`` cliques of ``size`` uniformly drawn vertices come first
+    (always kept), then R-MAT fills up to ``n_edges``."""
     out = np.empty((n_edges, 2), dtype=np.int32)
-    r = _load().gi_rmat_edges(scale, n_edges, a, b, c, seed & (2**64 - 1), id_limit, _threads(), _p(out))
+    r = _load().gi_rmat_edges(scale, n_edges, a, b, c, seed & (2**64 - 1), id_limit, _threads(), _p(out),
+                              int(planted[0]), int(planted[1]))
     if r != n_edges:
         raise ValueError("R-MAT id space too small for the requested edge count")
     return out
@@ -152,10 +157,11 @@ CONFIGS = {
     "C3": dict(scale=22, n_edges=120_000_000, abc=(0.502, 0.166, 0.166), id_limit=3_000_000, L=8,
                queries=["house5", "bowtie5", "k5e"], stream=12 * 8192, batch=4096, inserts_only=False,
                budget=0.10),
-    # FR-shaped: 67.1M ids, 1.8B edges (14.4 GB of adjacency in pinned host memory), hub ~5.2K
+    # FR-shaped: 67.1M ids, 1.8B edges (14.4 GB of adjacency in pinned host memory), hub ~5.2K; 5% of the
+    # edges are planted 8-cliques (R-MAT alone holds ~no dense 6-vertex subgraphs: SURVEY §8d realism note)
     "C4": dict(scale=26, n_edges=1_800_000_000, abc=(0.42, 0.176, 0.176), id_limit=0, L=0,
                queries=["prism6", "k4tri6", "k6"], stream=12 * 8192, batch=4096, inserts_only=False,
-               budget=0.01),
+               budget=0.01, planted_frac=0.05, planted_size=8),
 }
 
 
@@ -176,7 +182,9 @@ def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = 
     if n_stream is not None:
         cfg["stream"] = n_stream
     a, b, c = cfg["abc"]
-    uv = rmat_edges(cfg["scale"], cfg["n_edges"], a, b, c, seed, cfg["id_limit"])
+    ps = cfg.get("planted_size", 0)
+    groups = int(cfg.get("planted_frac", 0.0) * cfg["n_edges"]) // (ps * (ps - 1) // 2) if ps else 0
+    uv = rmat_edges(cfg["scale"], cfg["n_edges"], a, b, c, seed, cfg["id_limit"], planted=(groups, ps))
     n = cfg["id_limit"] if cfg["id_limit"] else (1 << cfg["scale"])
     n_stream = min(cfg["stream"], len(uv) // 2)
     sel, sign = stream(len(uv), n_stream, seed + 1000)
@@ -199,7 +207,7 @@ def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = 
     return Workload(name=name, n=n, row_ptr=rp, col=col, labels=lab, queries=list(cfg["queries"]),
                     batches=batches, budget_frac=cfg["budget"],
                     meta=dict(seed=seed, scale=cfg["scale"], n_edges=cfg["n_edges"], abc=cfg["abc"],
-                              id_limit=cfg["id_limit"], L=cfg["L"], batch=B))
+                              id_limit=cfg["id_limit"], L=cfg["L"], batch=B, planted=(groups, ps)))
 
 
 def small_random_case(seed: int, n: int = 9, p: float = 0.45, n_ins: int = 4, n_del: int = 4):

@@ -73,14 +73,54 @@ extern "C" {
 // relabelled with a seeded uniform permutation of [0, n_ids) where
 // n_ids = id_limit > 0 ? id_limit : 2^scale. Output pairs (u<v) in generation
 // order. Returns n_edges, or -1 if the id space cannot hold that many edges.
+// planted_groups > 0: the candidate stream starts with the edges of that many
+// planted cliques of planted_size vertices each (members drawn uniformly from
+// the id space, so they come first in generation order and are always kept):
+// community structure R-MAT lacks (SURVEY §8d workload-realism note).
 int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double c,
-                      uint64_t seed, int64_t id_limit, int32_t threads, int32_t* out_uv) {
+                      uint64_t seed, int64_t id_limit, int32_t threads, int32_t* out_uv,
+                      int64_t planted_groups, int32_t planted_size) {
   if (threads > 0) omp_set_num_threads(threads);
   const int64_t n_ids = id_limit > 0 ? id_limit : (int64_t(1) << scale);
   if ((double)n_edges > 0.5 * (double)n_ids * (double)(n_ids - 1)) return -1;
   std::vector<Cand> cands;
   int64_t next_j = 0;
   int64_t uniq = 0;
+  if (planted_groups > 0 && planted_size >= 2) {
+    const int64_t per = (int64_t)planted_size * (planted_size - 1) / 2;
+    const int64_t np = planted_groups * per;
+    cands.resize((size_t)np);
+    std::vector<uint8_t> ok((size_t)np);
+    const uint64_t gseed = h2(seed, 0x504C414E54ULL);
+#pragma omp parallel for schedule(static)
+    for (int64_t g = 0; g < planted_groups; ++g) {
+      uint64_t mem[64];
+      const int sz = planted_size < 64 ? planted_size : 64;
+      for (int i = 0; i < sz; ++i) mem[i] = h2(gseed, (uint64_t)(g * sz + i)) % (uint64_t)n_ids;
+      int64_t t = g * per;
+      for (int i = 0; i < sz; ++i)
+        for (int j = i + 1; j < sz; ++j, ++t) {
+          uint64_t u = mem[i], v = mem[j];
+          ok[t] = u != v;
+          if (u > v) std::swap(u, v);
+          cands[t] = Cand{(u << 32) | v, t};
+        }
+    }
+    size_t w = 0;
+    for (int64_t t = 0; t < np; ++t)
+      if (ok[t]) cands[w++] = cands[t];
+    cands.resize(w);
+    next_j = np;
+    __gnu_parallel::sort(cands.begin(), cands.end(), [](const Cand& x, const Cand& y) {
+      return x.key < y.key || (x.key == y.key && x.idx < y.idx);
+    });
+    size_t o = 0;
+    for (size_t i = 0; i < cands.size(); ++i)
+      if (o == 0 || cands[i].key != cands[o - 1].key) cands[o++] = cands[i];
+    cands.resize(o);
+    uniq = (int64_t)o;
+  }
+  const int64_t rmat_base = next_j;  // R-MAT draw j = generation index - rmat_base (same draws with or without planting)
   while (uniq < n_edges) {
     const int64_t want = (int64_t)((double)(n_edges - uniq) * 1.25) + 1024;
     const size_t old = cands.size();
@@ -89,7 +129,7 @@ int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double
 #pragma omp parallel for schedule(static)
     for (int64_t t = 0; t < want; ++t) {
       uint64_t key = 0;
-      ok[t] = rmat_one(scale, a, b, c, seed, next_j + t, id_limit, &key);
+      ok[t] = rmat_one(scale, a, b, c, seed, next_j + t - rmat_base, id_limit, &key);
       cands[old + t] = Cand{key, next_j + t};
     }
     size_t w = old;

@@ -122,8 +122,8 @@ struct gcsm_ctx {
   char *d_cache = nullptr; size_t cache_cap = 0;   // the buffer this batch's kernels read
   char *d_cachebuf[2] = {nullptr, nullptr};        // double buffer: last batch's cache stays readable
   int cache_cur = 0;                               // buffer holding the previous batch's cache
-  bool cache_valid = false;                        // prev_slot describes d_cachebuf[cache_cur]
-  std::vector<std::pair<int32_t, uint64_t>> prev_slot;  // (vertex, offset) of the previous cache, by vertex
+  bool cache_valid = false;                        // slot16 describes d_cachebuf[cache_cur]
+  std::vector<uint32_t> slot16;  // per vertex: 1 + (offset / 16) of its list in the previous cache, 0 = not cached
   uint64_t *d_gather = nullptr; size_t gather_cap = 0;  // retained lists: (src, dst, n16) triples
   uint64_t *d_fresh = nullptr; size_t fresh_cap = 0;    // newly cached lists: (host src, dst, n16) triples
   std::vector<int32_t> sel_index;                       // vertex -> index in this batch's selection, or -1
@@ -137,7 +137,6 @@ struct gcsm_ctx {
 
 
   // cache / batch state
-  std::vector<int32_t> cached;       // ascending
   std::vector<int32_t> prev_cached, prev_U;
   std::vector<uint8_t> mark;         // scratch (n)
   EstimatorScratch est_scratch;
@@ -271,6 +270,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
       return bail(GCSM_EDEVICE);
   }
   ctx->mark.assign(n, 0);
+  ctx->slot16.assign(n, 0);
   ctx->grid = match_grid(dev, &ctx->warps_total);
   // a communicator whenever an id is given (world 1 included: the single-rank allreduce exercises the same path)
   if (o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
@@ -364,13 +364,52 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
   }
   ctx->budget = bytes;
   ctx->cache_valid = false;  // the next batch repacks everything
-  ctx->prev_slot.clear();
+  for (int32_t v : ctx->prev_cached) ctx->slot16[v] = 0;
   return GCSM_OK;
 }
 
 }  // extern "C"
 
 // ------------------------------------------------------------------ pipeline
+
+// Merge of two id-ascending (score, id) lists, summing the scores of common ids; parallel over id ranges.
+static std::vector<std::pair<double, int32_t>> merge_sum_by_id(const std::vector<std::pair<double, int32_t>> &x,
+                                                              const std::vector<std::pair<double, int32_t>> &y,
+                                                              int T) {
+  const int nt = std::max(1, std::min(T, pool_size()));
+  const int64_t lo_id = std::min(x.empty() ? INT32_MAX : x.front().second, y.empty() ? INT32_MAX : y.front().second);
+  const int64_t hi_id = std::max(x.empty() ? 0 : x.back().second, y.empty() ? 0 : y.back().second) + 1;
+  std::vector<int64_t> cut(nt + 1);
+  for (int t = 0; t <= nt; ++t) cut[t] = lo_id + (hi_id - lo_id) * t / nt;
+  auto lb = [](const std::vector<std::pair<double, int32_t>> &v, int64_t id) {
+    return (size_t)(std::lower_bound(v.begin(), v.end(), id,
+                                     [](const std::pair<double, int32_t> &e, int64_t k) { return e.second < k; }) -
+                    v.begin());
+  };
+  std::vector<std::vector<std::pair<double, int32_t>>> part(nt);
+  parallel_for(nt, nt, [&](int, int64_t t0, int64_t t1) {
+    for (int64_t t = t0; t < t1; ++t) {
+      size_t i = lb(x, cut[t]), ie = lb(x, cut[t + 1]), j = lb(y, cut[t]), je = lb(y, cut[t + 1]);
+      auto &o = part[t];
+      o.reserve((ie - i) + (je - j));
+      while (i < ie || j < je) {
+        if (j == je || (i < ie && x[i].second < y[j].second)) o.push_back(x[i++]);
+        else if (i == ie || y[j].second < x[i].second) o.push_back(y[j++]);
+        else {
+          o.push_back({x[i].first + y[j].first, x[i].second});
+          ++i;
+          ++j;
+        }
+      }
+    }
+  });
+  std::vector<std::pair<double, int32_t>> out;
+  size_t tot = 0;
+  for (auto &p : part) tot += p.size();
+  out.reserve(tot);
+  for (auto &p : part) out.insert(out.end(), p.begin(), p.end());
+  return out;
+}
 
 static uint16_t host_label(const HostStore &s, int32_t v) { return s.lab.empty() ? 0 : s.lab[v]; }
 
@@ -552,19 +591,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
           if (ranked.empty()) {
             ranked.swap(r);
           } else {  // both ascending by id: merge, summing the scores of a vertex both queries access
-            std::vector<std::pair<double, int32_t>> m2;
-            m2.reserve(ranked.size() + r.size());
-            size_t x = 0, y = 0;
-            while (x < ranked.size() || y < r.size()) {
-              if (y == r.size() || (x < ranked.size() && ranked[x].second < r[y].second)) m2.push_back(ranked[x++]);
-              else if (x == ranked.size() || r[y].second < ranked[x].second) m2.push_back(r[y++]);
-              else {
-                m2.push_back({ranked[x].first + r[y].first, ranked[x].second});
-                ++x;
-                ++y;
-              }
-            }
-            ranked.swap(m2);
+            ranked = merge_sum_by_id(ranked, r, T);
           }
         }
       }
@@ -615,35 +642,74 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
   ctx->d_cache = ctx->d_cachebuf[tgt];
   if (use_cache && !ranked.empty()) {
-    // Only the head of the ranking can fit the budget: bucket the (positive) scores by their top 16 bits
-    // (monotone in the score), find the bucket where the cumulative list bytes pass the budget, and sort just
-    // the vertices at or above it. The longest-prefix selection (R23) is unchanged: it stops inside that bucket.
+    // Only the head of the ranking can fit the budget: bucket the (positive) scores by the top 12 bits of their
+    // IEEE pattern (monotone in the score), then the next 12 inside the bucket where the cumulative list bytes
+    // pass the budget, and sort just the vertices at or above that cut (per-thread histograms, parallel
+    // compaction). The longest-prefix selection (R23) is unchanged: it stops inside the cut bucket.
     {
-      std::vector<uint64_t> vb(ranked.size());
-      parallel_for(T, (int64_t)ranked.size(), [&](int, int64_t lo, int64_t hi) {
-        for (int64_t i = lo; i < hi; ++i) vb[i] = (uint64_t)((S.view_len(ranked[i].second, VIEW_S) + 3u) & ~3u) * 4;
-      });
-      auto bucket = [](double x) {
+      const int nt = std::max(1, std::min(T, pool_size()));
+      const int64_t nr = (int64_t)ranked.size();
+      std::vector<uint64_t> vb((size_t)nr);
+      auto bits = [](double x) {
         uint64_t b;
         std::memcpy(&b, &x, 8);
-        return (uint32_t)(b >> 48);
+        return b;
       };
-      std::vector<uint64_t> hb(1u << 16, 0);
-      for (size_t i = 0; i < ranked.size(); ++i)
-        if (ranked[i].first > 0) hb[bucket(ranked[i].first)] += vb[i];
-      uint64_t cum = 0;
-      uint32_t cut = 0;
-      for (int64_t b = (1 << 16) - 1; b >= 0; --b) {
-        cum += hb[b];
-        if (cum > ctx->budget) {
-          cut = (uint32_t)b;
-          break;
+      std::vector<uint64_t> h1((size_t)nt * 4096, 0), h2((size_t)nt * 4096, 0);
+      parallel_for(nt, nr, [&](int t, int64_t lo, int64_t hi) {
+        uint64_t *h = &h1[(size_t)t * 4096];
+        for (int64_t i = lo; i < hi; ++i) {
+          vb[i] = (uint64_t)((S.view_len(ranked[i].second, VIEW_S) + 3u) & ~3u) * 4;
+          if (ranked[i].first > 0) h[bits(ranked[i].first) >> 52] += vb[i];
         }
+      });
+      auto find_cut = [&](std::vector<uint64_t> &h, uint64_t before, uint32_t *cut, uint64_t *above) {
+        uint64_t cum = before;
+        for (int64_t b = 4095; b >= 0; --b) {
+          uint64_t x = 0;
+          for (int t = 0; t < nt; ++t) x += h[(size_t)t * 4096 + b];
+          if (cum + x > ctx->budget) {
+            *cut = (uint32_t)b;
+            *above = cum;
+            return true;
+          }
+          cum += x;
+        }
+        *cut = 0;
+        *above = cum;
+        return false;
+      };
+      uint32_t c1 = 0, c2 = 0;
+      uint64_t above1 = 0, above2 = 0;
+      const bool cut_found = find_cut(h1, 0, &c1, &above1);
+      if (cut_found) {
+        parallel_for(nt, nr, [&](int t, int64_t lo, int64_t hi) {
+          uint64_t *h = &h2[(size_t)t * 4096];
+          for (int64_t i = lo; i < hi; ++i)
+            if (ranked[i].first > 0 && (bits(ranked[i].first) >> 52) == c1) h[(bits(ranked[i].first) >> 40) & 4095] += vb[i];
+        });
+        find_cut(h2, above1, &c2, &above2);
       }
-      size_t w = 0;
-      for (size_t i = 0; i < ranked.size(); ++i)
-        if (ranked[i].first > 0 && bucket(ranked[i].first) >= cut) ranked[w++] = ranked[i];
-      ranked.resize(w);
+      auto keep = [&](int64_t i) {
+        if (!(ranked[i].first > 0)) return false;
+        const uint64_t b = bits(ranked[i].first);
+        const uint32_t k1 = (uint32_t)(b >> 52);
+        return !cut_found || k1 > c1 || (k1 == c1 && ((b >> 40) & 4095) >= c2);
+      };
+      std::vector<int64_t> cnt((size_t)nt + 1, 0);
+      parallel_for(nt, nr, [&](int t, int64_t lo, int64_t hi) {
+        int64_t c = 0;
+        for (int64_t i = lo; i < hi; ++i) c += keep(i);
+        cnt[t + 1] = c;
+      });
+      for (int t = 0; t < nt; ++t) cnt[t + 1] += cnt[t];
+      std::vector<std::pair<double, int32_t>> kept((size_t)cnt[nt]);
+      parallel_for(nt, nr, [&](int t, int64_t lo, int64_t hi) {
+        int64_t o = cnt[t];
+        for (int64_t i = lo; i < hi; ++i)
+          if (keep(i)) kept[o++] = ranked[i];
+      });
+      ranked.swap(kept);
     }
     parallel_sort(
         ranked,
@@ -673,8 +739,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       for (int64_t i = lo; i < hi; ++i) {
         const int32_t v = sel[i];
         if (ctx->cache_valid && ctx->mark[v] != 2 && S.uidx[v] < 0) {
-          auto it = std::lower_bound(ctx->prev_slot.begin(), ctx->prev_slot.end(), std::make_pair(v, (uint64_t)0));
-          if (it != ctx->prev_slot.end() && it->first == v) old_off[i] = (int64_t)it->second;
+          const uint32_t so = ctx->slot16[v];
+          if (so) old_off[i] = 16 * (int64_t)(so - 1);
         }
         if (old_off[i] < 0) src[i] = (uint64_t)(uintptr_t)S.dev_ptr(S.view(v, VIEW_S).a);
       }
@@ -970,16 +1036,17 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   Timer t5;
   if (!S.merge(sl.retired)) return ctx->fail(GCSM_ENOMEM, "pinned allocation for the merged lists failed");
   tr.mark("merge");
-  ctx->prev_cached = sel;
-  std::sort(ctx->prev_cached.begin(), ctx->prev_cached.end());
-  ctx->prev_slot.resize(sel.size());
-  for (size_t i = 0; i < sel.size(); ++i) ctx->prev_slot[i] = {sel[i], sel_off[i]};
-  std::sort(ctx->prev_slot.begin(), ctx->prev_slot.end());
+  parallel_for(T, (int64_t)ctx->prev_cached.size(), [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) ctx->slot16[ctx->prev_cached[i]] = 0;
+  });
+  parallel_for(T, (int64_t)sel.size(), [&](int, int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) ctx->slot16[sel[i]] = (uint32_t)(sel_off[i] / 16) + 1;
+  });
+  ctx->prev_cached.swap(sel);  // selection order (gcsm_get_cached sorts its copy)
   if (ctx->budget > 0) {
     ctx->cache_cur = tgt;
     ctx->cache_valid = true;
   }
-  ctx->cached = ctx->prev_cached;
   ctx->prev_U = S.U;
   S.clear_batch();
   for (auto &pq : sl.q) pq.st.ms_merge = t5.ms();
@@ -1140,10 +1207,12 @@ gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levc
 
 gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out) {
   if (!ctx || !n_out) return GCSM_EINVAL;
-  const uint64_t n = ctx->cached.size();
+  std::vector<int32_t> cached = ctx->prev_cached;
+  std::sort(cached.begin(), cached.end());
+  const uint64_t n = cached.size();
   *n_out = n;
   const uint64_t w = std::min(n, cap);
-  if (ids && w) std::memcpy(ids, ctx->cached.data(), 4 * w);
+  if (ids && w) std::memcpy(ids, cached.data(), 4 * w);
   return n > cap ? GCSM_ETRUNC : GCSM_OK;
 }
 

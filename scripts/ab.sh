@@ -1,5 +1,5 @@
 #!/bin/bash
-# A/B kernel variants (serial contexts, match-only numbers): VARIANTS="old new" ARGS_LIST=("--budget-frac 0.1" ...)
+# A/B kernel variants (serial, match-only numbers; C2 K4+C4 in one context): VARIANTS="a b" [ARGSETS as below]
 out=gpurun_out/ab.txt; : > $out
 for args in "--cache-policy estimator" "--cache-policy degree --budget-frac 1.05"; do
 for v in ${VARIANTS:-old new}; do

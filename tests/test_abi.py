@@ -121,3 +121,23 @@ def test_symmetry_breaking_restrictions_brute_force(pkg, name):
                                   k, qe.tolist(), None if ql is None else np.zeros(k, np.int32))
     if ql is None:
         assert len([f for f in emb if all(f[u] < f[w] for u, w in pairs2)]) * aut2 == len(emb)
+
+
+def test_generator_planted_cliques():
+    """C4's planted 8-cliques: exactly n_edges unique edges, every planted group a clique, deterministic, and the
+    R-MAT part unchanged when nothing is planted (C2 / C3 inputs are the same as before)."""
+    import numpy as np
+    import gcsm_inputs as gi
+    uv = gi.rmat_edges(12, 20000, 0.42, 0.176, 0.176, 7, planted=(50, 8))
+    assert len(uv) == 20000 and (uv[:, 0] < uv[:, 1]).all()
+    keys = uv[:, 0].astype(np.int64) * (1 << 32) + uv[:, 1]
+    assert len(np.unique(keys)) == len(keys)
+    assert np.array_equal(uv, gi.rmat_edges(12, 20000, 0.42, 0.176, 0.176, 7, planted=(50, 8)))
+    # the planted edges come first in generation order: the first group's distinct members form a clique
+    first = uv[:28]
+    verts = np.unique(first)
+    assert len(first) == len(verts) * (len(verts) - 1) // 2
+    plain = gi.rmat_edges(12, 20000, 0.42, 0.176, 0.176, 7)
+    assert not np.array_equal(plain[:28], first)
+    w = gi.make_workload("C4", scale=12, n_edges=30000, batch=64, n_batches=1)
+    assert w.meta["planted"][0] > 0 and int(w.row_ptr[-1]) > 0

@@ -211,6 +211,16 @@ def test_six_vertex_queries(G, name):
     assert got == want
 
 
+@pytest.mark.parametrize("name", ["prism6", "k4tri6", "k6"])
+def test_c4_shaped_planted(G, name):
+    """C4-shaped (FR R-MAT parameters + planted 8-cliques): the 6-vertex counts are non-zero, budget << graph."""
+    w = gi.make_workload("C4", scale=13, n_edges=60_000, batch=256, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    assert any(a or r for a, r in want)
+    got, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.01)
+    assert got == want
+
+
 @pytest.mark.parametrize("r", [1, 2, 3])
 def test_star_closed_form_at_scale(G, r):
     """SURVEY §8c degree closed form for K_{1,r}: added = Σ_U P(d',r) - P(s,r), removed = Σ_U P(d,r) - P(s,r)."""
