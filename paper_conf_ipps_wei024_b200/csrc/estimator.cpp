@@ -226,24 +226,22 @@ uint64_t walk_budget(uint64_t N1, uint64_t D, int k) {
 
 namespace {
 
+constexpr int kPartLog2 = 14;  // ids per reduction partition (16K x levels x 8 B stays in L2)
+
 struct Walker {
   const EstimatorInput &in;
   EstimatorScratch &scr;
   const DevPlan *P = nullptr;
   int32_t f[GCSM_MAXK];
   std::vector<uint32_t> keep_[GCSM_MAXK];
+  std::vector<EstRec> *out = nullptr;  // this thread's partition buffers
   Walker(const EstimatorInput &i, EstimatorScratch &s) : in(i), scr(s) {}
 
   bool member(const HList &L, int32_t v) const {
     return std::binary_search(L.a, L.a + L.na, v) || (L.nb && std::binary_search(L.b, L.b + L.nb, v));
   }
 
-  void record(int32_t v, int level, uint64_t B) {
-    __atomic_fetch_add(&scr.sums[(size_t)(level - 1) * (size_t)scr.n + (size_t)v], B, __ATOMIC_RELAXED);
-    uint64_t *w = &scr.touched[(uint32_t)v >> 6];
-    const uint64_t bit = 1ull << (v & 63);
-    if (!(__atomic_load_n(w, __ATOMIC_RELAXED) & bit)) __atomic_fetch_or(w, bit, __ATOMIC_RELAXED);
-  }
+  void record(int32_t v, int level, uint64_t B) { out[(uint32_t)v >> kPartLog2].push_back({v, (uint32_t)level, B}); }
 
   // node at `level` (positions 0..level matched), multiplicity B, key
   void visit(int level, int64_t B, uint64_t key) {
@@ -301,17 +299,22 @@ void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOut
   const int k = in.plans[0].k;
   if (k <= 2 || in.n_units == 0) return;
   const int levels = k - 2;
-  if (scr.n != in.n || scr.levels < levels) {
+  const int T = std::max(1, std::min(in.threads, pool_size()));
+  const int parts = (int)(((int64_t)in.n + (1 << kPartLog2) - 1) >> kPartLog2);
+  if (scr.n != in.n || scr.threads != T || scr.parts != parts) {
     scr.n = in.n;
-    scr.levels = levels;
-    scr.sums.assign((size_t)levels * (size_t)in.n, 0);
-    scr.touched.assign(((size_t)in.n + 63) / 64, 0);
+    scr.threads = T;
+    scr.parts = parts;
+    scr.buf.assign((size_t)T * parts, {});
   }
-  const int T = std::max(1, in.threads);
+  for (auto &b : scr.buf) b.clear();
   const uint64_t root = rng_mix(in.seed);
   const double p1 = 1.0 / (double)in.N1;
   std::vector<std::unique_ptr<Walker>> walkers(T);
-  for (auto &w : walkers) w.reset(new Walker(in, scr));
+  for (int t = 0; t < T; ++t) {
+    walkers[t].reset(new Walker(in, scr));
+    walkers[t]->out = &scr.buf[(size_t)t * parts];
+  }
   parallel_dyn(T, in.n_units, 64, [&](int tid, int64_t ui) {
     const Unit &u = in.units[ui];
     const int term = u.plan >> 1, kind = u.plan & 1;
@@ -326,36 +329,41 @@ void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOut
     w.f[1] = u.b;
     w.visit(1, B, key);
   });
-  // touched vertices in ascending order (bitmap scan), their sums, then a sparse reset
-  const int64_t nw = (int64_t)scr.touched.size();
-  const int chunks = std::min<int64_t>(T, nw);
-  std::vector<int64_t> cnt(chunks + 1, 0);
-  parallel_for(chunks, nw, [&](int c, int64_t lo, int64_t hi) {
-    int64_t x = 0;
-    for (int64_t i = lo; i < hi; ++i) x += __builtin_popcountll(scr.touched[i]);
-    cnt[c + 1] = x;
-  });
-  for (int c = 0; c < chunks; ++c) cnt[c + 1] += cnt[c];
-  out.ids.resize(cnt[chunks]);
-  out.levcnt.assign(8 * (size_t)cnt[chunks], 0);
-  parallel_for(chunks, nw, [&](int c, int64_t lo, int64_t hi) {
-    int64_t o = cnt[c];
-    for (int64_t i = lo; i < hi; ++i) {
-      uint64_t w = scr.touched[i];
-      while (w) {
-        const int b = __builtin_ctzll(w);
-        w &= w - 1;
-        const int32_t v = (int32_t)(i * 64 + b);
-        out.ids[o] = v;
-        for (int l = 0; l < levels; ++l) {
-          uint64_t &x = scr.sums[(size_t)l * (size_t)scr.n + (size_t)v];
-          out.levcnt[8 * (size_t)o + l] = x;
-          x = 0;
-        }
-        ++o;
+  // reduce each vertex-range partition in a dense window (one thread per partition), ids in ascending order
+  std::vector<std::vector<int32_t>> pid((size_t)parts);
+  std::vector<std::vector<uint64_t>> plev((size_t)parts);
+  parallel_dyn(T, parts, 1, [&](int, int64_t p) {
+    size_t nrec = 0;
+    for (int t = 0; t < T; ++t) nrec += scr.buf[(size_t)t * parts + p].size();
+    if (!nrec) return;
+    const int64_t base = p << kPartLog2;
+    const int64_t span = std::min<int64_t>((int64_t)1 << kPartLog2, (int64_t)in.n - base);
+    thread_local std::vector<uint64_t> win;
+    thread_local std::vector<uint8_t> hit;
+    win.assign((size_t)span * levels, 0);
+    hit.assign((size_t)span, 0);
+    for (int t = 0; t < T; ++t)
+      for (const EstRec &r : scr.buf[(size_t)t * parts + p]) {
+        const int64_t o = r.v - base;
+        win[(size_t)o * levels + (r.level - 1)] += r.B;
+        hit[o] = 1;
       }
-      scr.touched[i] = 0;
-    }
+    auto &ids = pid[p];
+    auto &lev = plev[p];
+    for (int64_t o = 0; o < span; ++o)
+      if (hit[o]) {
+        ids.push_back((int32_t)(base + o));
+        for (int l = 0; l < 8; ++l) lev.push_back(l < levels ? win[(size_t)o * levels + l] : 0);
+      }
+  });
+  std::vector<size_t> off((size_t)parts + 1, 0);
+  for (int p = 0; p < parts; ++p) off[p + 1] = off[p] + pid[p].size();
+  out.ids.resize(off[parts]);
+  out.levcnt.resize(8 * off[parts]);
+  parallel_dyn(T, parts, 8, [&](int, int64_t p) {
+    if (pid[p].empty()) return;
+    std::memcpy(out.ids.data() + off[p], pid[p].data(), 4 * pid[p].size());
+    std::memcpy(out.levcnt.data() + 8 * off[p], plev[p].data(), 8 * plev[p].size());
   });
 }
 

@@ -26,13 +26,20 @@ struct EstimatorInput {
   std::function<HList(int32_t, int)> view;  // (vertex, View) -> host list view
 };
 
-// Persistent dense accumulators (n x (k-2) sums + a touched bitmap), reset
-// sparsely after each batch: O(records) accumulation, ids come out sorted.
+// Persistent per-batch scratch. Every node's read of a list is a record (vertex, level, B); records go to
+// thread-local buffers partitioned by vertex range (kPartLog2 ids per partition), and each partition is then
+// reduced by one thread in a cache-resident dense window: no scattered atomics into n-sized arrays, ids come
+// out sorted, and the integer sums are identical to any other summation order.
+struct EstRec {
+  int32_t v;
+  uint32_t level;
+  uint64_t B;
+};
 struct EstimatorScratch {
   int32_t n = 0;
-  int levels = 0;
-  std::vector<uint64_t> sums;     // [levels][n]
-  std::vector<uint64_t> touched;  // n bits
+  int threads = 0;
+  int parts = 0;
+  std::vector<std::vector<EstRec>> buf;  // [thread * parts + partition]
 };
 
 struct EstimatorOutput {
