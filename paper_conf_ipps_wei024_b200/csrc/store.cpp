@@ -43,17 +43,21 @@ const int32_t *HostStore::dev_ptr(const int32_t *host) const {
   return nullptr;
 }
 
-int32_t *HostStore::alloc_list(uint32_t capacity, bool *cuda_err) {
-  auto fit = free_.find(capacity);
-  if (fit != free_.end() && !fit->second.empty()) {
-    int32_t *p = fit->second.back();
-    fit->second.pop_back();
-    return p;
-  }
+int32_t *HostStore::alloc_list(uint32_t &capacity, bool *cuda_err) {
+  // recycled array of the smallest capacity in [capacity, 2 capacity] (a retired list of a similar size)
+  for (auto fit = free_.lower_bound(capacity); fit != free_.end() && fit->first <= 2ull * capacity; ++fit)
+    if (!fit->second.empty()) {
+      int32_t *p = fit->second.back();
+      fit->second.pop_back();
+      capacity = fit->first;  // the caller records the array's real capacity
+      return p;
+    }
   const size_t bytes = (size_t)capacity * 4;
   if (chunks_.empty() || chunks_.back().used + bytes > chunks_.back().size) {
     Chunk c;
-    size_t sz = std::max<size_t>((size_t)256 << 20, 4 * bytes);
+    // grow by an eighth of the store at least: pinning memory (cudaHostAlloc) costs ~0.1-0.2 s per GB, so it
+    // must be rare, not a per-batch stall
+    size_t sz = std::max<size_t>(std::max<size_t>((size_t)256 << 20, 4 * bytes), store_bytes_ / 8);
     if (!new_chunk(sz, c)) {
       *cuda_err = true;
       return nullptr;
@@ -120,7 +124,8 @@ std::string HostStore::init(int32_t n_, const int64_t *rp, const int32_t *col, c
   deg_hist.assign((size_t)maxdeg + 1, 0);
   for (int32_t v = 0; v < n; ++v) deg_hist[len[v]]++;
   Chunk c;
-  if (!new_chunk(total * 4 + ((size_t)64 << 20), c)) {
+  store_bytes_ = total * 4;
+  if (!new_chunk(total * 4 + std::max<size_t>((size_t)64 << 20, total / 2), c)) {  // slack: 1/8 of the store
     *cuda_err = true;
     return "cudaHostAlloc of the pinned store failed";
   }
@@ -305,7 +310,7 @@ bool HostStore::merge(std::vector<std::pair<int32_t *, uint32_t>> &retired) {
     newlen[i] = s_len[i] + (ins_off[i + 1] - ins_off[i]);
     newcap[i] = cap[x];
     if (newlen[i] > cap[x]) newcap[i] = round4(std::max<uint64_t>(4, 2ull * newlen[i]));  // double
-    target[i] = newcap[i] ? alloc_list(newcap[i], &err) : nullptr;
+    target[i] = newcap[i] ? alloc_list(newcap[i], &err) : nullptr;  // may raise newcap[i] (recycled array)
     if (err) {  // give back what this merge took; the store is unchanged
       for (size_t j = 0; j < i; ++j)
         if (target[j]) free_[newcap[j]].push_back(target[j]);

@@ -15,6 +15,7 @@
 #include <cstdint>
 #include <string>
 #include <unordered_map>
+#include <map>
 #include <vector>
 
 #include "estimator.h"
@@ -73,9 +74,11 @@ class HostStore {
  private:
   std::vector<Chunk> chunks_;
   Chunk overlay_[2];
-  std::unordered_map<uint32_t, std::vector<int32_t *>> free_;  // recycled arrays by capacity
-  int32_t *alloc_list(uint32_t capacity, bool *cuda_err);
+  std::map<uint32_t, std::vector<int32_t *>> free_;  // recycled arrays by capacity
+  // an array of >= capacity ints: a recycled one of up to 2x (capacity is raised to its size) or a fresh one
+  int32_t *alloc_list(uint32_t &capacity, bool *cuda_err);
   bool new_chunk(size_t bytes, Chunk &c);
+  size_t store_bytes_ = 0;  // pinned list capacity at init (growth quantum)
   bool has_edge(int32_t u, int32_t v) const;
 };
 
