@@ -207,6 +207,8 @@ static void coin_filter(const int32_t *v, uint32_t n, uint64_t key, uint64_t T, 
   else coin_filter_scalar(v, n, key, T, out);
 }
 
+double stirling_small(int k) { return stirling_fc(k); }
+
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k) {
   // M = floor(N1 * D^(k-2) / 32^k), clamped to [1, 2^62] (R21), exact integer arithmetic.
   if (N1 == 0) return 1;

@@ -48,6 +48,7 @@ struct EstimatorOutput {
 };
 
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k);
+double stirling_small(int k);  // BTRD's Stirling correction for k < 10 (lgamma; the GPU sampler's table)
 void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOutput &out);
 double estimate_value(const uint64_t *lev, int k, uint64_t N1, uint64_t D, uint64_t M);
 

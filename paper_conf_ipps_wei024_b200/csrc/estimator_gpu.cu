@@ -1,0 +1,745 @@
+// estimator_gpu.cu — steps ② (random-walk access-frequency estimation, §IV) and ③ (cache ranking and
+// packing) on sm_100a, enqueued on the context's stream before the matching kernels.
+//
+// ② k_walks: warp per level-1 node (a unit with its host-drawn B_1 ~ Bin(M, 1/N1)), DFS over the merged
+//    walks of §IV-B inside the warp: a node at level l records B on every list its next position reads (eq. (3),
+//    P:204; R17) into dense per-query integer sums; its children are the candidates of the next position (R18),
+//    the lanes taking 32 consecutive driver elements, each child drawing B' ~ Bin(B, 1/D) from its own key
+//    (R20, R22) and surviving if B' > 0 and it belongs to every other backward list. Integer atomics make the sums
+//    independent of the visiting order, so they equal the host walker's and the oracle's bit for bit.
+// ③ the touched vertices (a bitmap, compacted in id order) get their estimate (eq. (3) averaged over M, summed
+//    over standing queries); the ranking cut of R23 (estimate desc, id asc, longest prefix under the budget) is
+//    found without a sort: byte-weighted histograms over the score's IEEE bits, 12 bits per pass, narrow the cut
+//    to one exact score value (positive doubles order like their bit patterns); the vertices strictly above it all
+//    fit; the ties at it are taken in id order while they fit (an inclusive scan). The selected lists are copied
+//    into this batch's cache buffer from where their descriptors point (the previous buffer: HBM -> HBM, else the
+//    pinned host store over PCIe), then the descriptors are switched (previous selection back to host, new one to
+//    its slot).
+//
+// Floating point: the binomial samplers and the score are transcribed from the host code with explicit
+// round-to-nearest intrinsics (__dmul_rn, __dadd_rn, __dsub_rn, __ddiv_rn, __dsqrt_rn) so nvcc cannot contract
+// them into FMAs: the same IEEE operation sequence gives the same doubles. BINV's r0 = (1-p)^n comes from a host
+// table (glibc pow), BTRD's Stirling terms for k < 10 from a host table (glibc lgamma); BTRD's log is CUDA's
+// (max 1 ulp; it decides only comparisons that are not within an ulp of a tie — DESIGN.md).
+#include <cub/cub.cuh>
+
+#include "estimator_gpu.cuh"
+
+namespace gcsm {
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+__device__ __forceinline__ unsigned long long dmix(unsigned long long z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+__device__ __forceinline__ unsigned long long dchain(unsigned long long h, unsigned long long x) {
+  return dmix(h + 0x9E3779B97F4A7C15ULL * (x + 1));
+}
+
+#define DM(a, b) __dmul_rn((a), (b))
+#define DA(a, b) __dadd_rn((a), (b))
+#define DS(a, b) __dsub_rn((a), (b))
+#define DV(a, b) __ddiv_rn((a), (b))
+
+struct DUni {
+  unsigned long long key, j;
+  __device__ __forceinline__ double next() {
+    ++j;
+    return DM((double)(dmix(key + 0xD1B54A32D192ED03ULL * j) >> 11), 1.0 / 9007199254740992.0);
+  }
+};
+
+struct BinTab {
+  double pD;
+  const double *r0tab;
+  int64_t r0n;
+  const double *sfc;  // 10 entries
+  int32_t *err;
+};
+
+__device__ __forceinline__ double d_sfc(const BinTab &T, int64_t k) {
+  if (k < 10) return T.sfc[k];
+  const double r = DV(1.0, (double)(k + 1)), r2 = DM(r, r);
+  return DM(DS(1.0 / 12.0, DM(DS(1.0 / 360.0, DM(1.0 / 1260.0, r2)), r2)), r);
+}
+
+// BINV (n p < 10): estimator.cpp binv with r0 = (1-p)^n from the host table.
+__device__ int64_t d_binv(DUni &U, int64_t n, double p, double r0) {
+  const double q = DS(1.0, p);
+  const double s = DV(p, q), a = DM((double)(n + 1), s);
+  for (;;) {
+    double r = r0, u = U.next();
+    int64_t x = 0;
+    while (u > r) {
+      u = DS(u, r);
+      x += 1;
+      if (x > n) break;
+      r = DM(r, DS(DV(a, (double)x), s));
+    }
+    if (x <= n) return x;
+  }
+}
+
+// BTRD (n p >= 10): estimator.cpp btrd, operation for operation.
+__device__ int64_t d_btrd(DUni &U, int64_t n, double p, const BinTab &T) {
+  const double q = DS(1.0, p);
+  const double m = floor(DM((double)(n + 1), p));
+  const double r = DV(p, q), nr = DM((double)(n + 1), r), npq = DM(DM((double)n, p), q);
+  const double spq = __dsqrt_rn(npq);
+  const double b = DA(1.15, DM(2.53, spq));
+  const double a = DA(DA(-0.0873, DM(0.0248, b)), DM(0.01, p));
+  const double c = DA(DM((double)n, p), 0.5);
+  const double alpha = DM(DA(2.83, DV(5.1, b)), spq);
+  const double vr = DS(0.92, DV(4.2, b));
+  const double urvr = DM(0.86, vr);
+  const int64_t mi = (int64_t)m;
+  for (;;) {
+    double v = U.next(), u;
+    if (v <= urvr) {
+      u = DS(DV(v, vr), 0.43);
+      return (int64_t)floor(DA(DM(DA(DV(DM(2.0, a), DS(0.5, fabs(u))), b), u), c));
+    }
+    if (v >= vr) {
+      u = DS(U.next(), 0.5);
+    } else {
+      u = DS(DV(v, vr), 0.93);
+      u = DS(u < 0 ? -0.5 : 0.5, u);
+      v = DM(U.next(), vr);
+    }
+    const double us = DS(0.5, fabs(u));
+    const double kd = floor(DA(DM(DA(DV(DM(2.0, a), us), b), u), c));
+    if (kd < 0.0 || kd > (double)n) continue;
+    const int64_t ki = (int64_t)kd;
+    v = DV(DM(v, alpha), DA(DV(a, DM(us, us)), b));
+    const int64_t km = ki > mi ? ki - mi : mi - ki;
+    if (km <= 15) {
+      double f = 1.0;
+      if (mi < ki) {
+        for (int64_t i = mi + 1; i <= ki; ++i) f = DM(f, DS(DV(nr, (double)i), r));
+      } else if (mi > ki) {
+        for (int64_t i = ki + 1; i <= mi; ++i) v = DM(v, DS(DV(nr, (double)i), r));
+      }
+      if (v <= f) return ki;
+      continue;
+    }
+    v = log(v);
+    const double kmd = (double)km;
+    const double rho = DM(DV(kmd, npq), DA(DV(DA(DM(DA(DV(kmd, 3.0), 0.625), kmd), 1.0 / 6.0), npq), 0.5));
+    const double t = DV(DM(-kmd, kmd), DM(2.0, npq));
+    if (v < DS(t, rho)) return ki;
+    if (v > DA(t, rho)) continue;
+    const double nm = (double)(n - mi + 1);
+    const double h = DA(DA(DM(DA(m, 0.5), log(DV(DA(m, 1.0), DM(r, nm)))), d_sfc(T, mi)), d_sfc(T, n - mi));
+    const double nk = (double)(n - ki + 1);
+    const double rhs = DS(DS(DA(DA(h, DM((double)(n + 1), log(DV(nm, nk)))),
+                                DM(DA(kd, 0.5), log(DV(DM(nk, r), DA(kd, 1.0))))),
+                             d_sfc(T, ki)),
+                          d_sfc(T, n - ki));
+    if (v <= rhs) return ki;
+  }
+}
+
+// estimator.cpp binomial(key, n, p) for p = 1/D.
+__device__ __forceinline__ int64_t d_binomial(unsigned long long key, int64_t n, const BinTab &T) {
+  const double p = T.pD;
+  if (n <= 0 || p <= 0.0) return 0;
+  if (p >= 1.0) return n;
+  DUni U{key, 0};
+  if (p > 0.5) {  // unreachable: p = 1/D with an integer D >= 2
+    atomicExch(T.err, 1);
+    return 0;
+  }
+  if (DM((double)n, p) < 10.0) {
+    if (n >= T.r0n) {
+      atomicExch(T.err, 2);
+      return 0;
+    }
+    return d_binv(U, n, p, T.r0tab[n]);
+  }
+  return d_btrd(U, n, p, T);
+}
+
+struct LR {
+  const int32_t *m;
+  uint32_t ml;
+  const int32_t *x;
+  uint32_t xl;
+};
+
+__device__ __forceinline__ LR view_of(const VDesc *vdesc, const DRec *drec, const int32_t *dlist, int32_t v, int vw) {
+  const int4 raw = __ldg(reinterpret_cast<const int4 *>(vdesc + v));
+  LR r;
+  r.m = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x | ((unsigned long long)(unsigned)raw.y << 32));
+  r.ml = (uint32_t)raw.z;
+  r.x = nullptr;
+  r.xl = 0;
+  const uint32_t upd = (uint32_t)raw.w;
+  if (upd != 0 && vw != VIEW_S) {
+    const int4 e = __ldg(reinterpret_cast<const int4 *>(drec + (upd - 1)));
+    if (vw == VIEW_NEW) {
+      r.x = dlist + e.x;
+      r.xl = (uint32_t)e.y;
+    } else {
+      r.x = dlist + e.z;
+      r.xl = (uint32_t)e.w;
+    }
+  }
+  return r;
+}
+
+__device__ __forceinline__ bool has(const int32_t *a, uint32_t n, int32_t v) {
+  uint32_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    const int32_t x = a[mid];
+    if (x < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo < n && a[lo] == v;
+}
+
+struct WalkArgs {
+  const DevPlan *plans;
+  const EstUnit *units;
+  int64_t n_units;
+  unsigned long long *levcnt;
+  int32_t levels;
+  const VDesc *vdesc;
+  const DRec *drec;
+  const int32_t *dlist;
+  const uint16_t *lab;
+  uint32_t *touched;
+  unsigned long long *cursor;
+  BinTab T;
+  double sfc[10];
+};
+
+constexpr int kEW = 8;  // warps per block
+struct EstLv {
+  int32_t pos, ns, si, pad;
+  unsigned long long B, key;
+  int32_t sv[32];
+  unsigned long long sB[32], skey[32];
+};
+struct EstW {
+  int32_t f[GCSM_MAXK];
+  EstLv lv[GCSM_MAXK - 1];  // index = tree level 1..k-2
+};
+
+__global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
+  __shared__ EstW sw[kEW];
+  __shared__ double sfc_s[10];
+  if (threadIdx.x < 10) sfc_s[threadIdx.x] = A.sfc[threadIdx.x];
+  __syncthreads();
+  BinTab T = A.T;
+  T.sfc = sfc_s;
+  const int lane = threadIdx.x & 31;
+  EstW &W = sw[threadIdx.x >> 5];
+  for (;;) {
+    unsigned long long u = 0;
+    if (lane == 0) u = atomicAdd(A.cursor, 1ull);
+    u = __shfl_sync(FULL, u, 0);
+    if (u >= (unsigned long long)A.n_units) return;
+    const EstUnit U = A.units[u];
+    const DevPlan *P = A.plans + U.plan;
+    const int k = P->k;
+    __syncwarp();
+    if (lane == 0) {
+      W.f[0] = U.a;
+      W.f[1] = U.b;
+      W.lv[1].B = U.B;
+      W.lv[1].key = U.key;
+    }
+    __syncwarp();
+    int level = 1;
+    bool fresh = true;
+    while (level >= 1) {
+      EstLv &S = W.lv[level];
+      const LevelPlan &Lp = P->lv[level + 1];
+      const int nb = Lp.nb;
+      if (fresh) {  // a node at `level` (positions 0..level matched) reads its next position's backward lists
+        fresh = false;
+        if (lane < nb) {
+          const int32_t v = W.f[Lp.bpos[lane]];
+          atomicAdd(A.levcnt + (size_t)v * A.levels + (level - 1), S.B);
+          atomicOr(A.touched + (v >> 5), 1u << (v & 31));
+        }
+        if (level == k - 2) {  // its children are leaves: they read nothing (R17)
+          --level;
+          __syncwarp();
+          continue;
+        }
+        if (lane == 0) {
+          S.pos = 0;
+          S.ns = 0;
+          S.si = 0;
+        }
+        __syncwarp();
+        continue;
+      }
+      const int si = S.si, ns = S.ns;
+      if (si < ns) {  // descend into the next surviving child
+        __syncwarp();
+        if (lane == 0) {
+          S.si = si + 1;
+          W.f[level + 1] = S.sv[si];
+          W.lv[level + 1].B = S.sB[si];
+          W.lv[level + 1].key = S.skey[si];
+        }
+        __syncwarp();
+        ++level;
+        fresh = true;
+        continue;
+      }
+      // next 32 driver elements of this node's candidate set
+      const int p = level + 1;
+      LR L[7];
+      int drv = 0;
+      uint32_t best = 0xffffffffu;
+      for (int b = 0; b < nb; ++b) {
+        L[b] = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
+        const uint32_t t = L[b].ml + L[b].xl;
+        if (t < best) {
+          best = t;
+          drv = b;
+        }
+      }
+      const uint32_t pos = (uint32_t)S.pos;
+      if (pos >= best) {
+        __syncwarp();
+        --level;
+        continue;
+      }
+      const uint32_t idx = pos + lane;
+      bool ok = false;
+      int32_t v = 0;
+      unsigned long long Bc = 0, ck = 0;
+      if (idx < best) {
+        v = idx < L[drv].ml ? L[drv].m[idx] : L[drv].x[idx - L[drv].ml];
+        ok = true;
+        for (int s = 0; s < p; ++s) ok &= W.f[s] != v;
+        if (ok && Lp.label >= 0) ok = (A.lab ? (int32_t)A.lab[v] : 0) == Lp.label;
+        if (ok) {
+          ck = dchain(S.key, (unsigned long long)(uint32_t)v);
+          const int64_t bc = d_binomial(ck, (int64_t)S.B, T);
+          Bc = (unsigned long long)bc;
+          ok = bc > 0;
+        }
+        if (ok)
+          for (int b = 0; b < nb; ++b)
+            if (b != drv && !(has(L[b].m, L[b].ml, v) || (L[b].xl && has(L[b].x, L[b].xl, v)))) {
+              ok = false;
+              break;
+            }
+      }
+      const unsigned mask = __ballot_sync(FULL, ok);
+      __syncwarp();
+      if (ok) {
+        const int r = __popc(mask & ((1u << lane) - 1u));
+        S.sv[r] = v;
+        S.sB[r] = Bc;
+        S.skey[r] = ck;
+      }
+      if (lane == 0) {
+        S.ns = __popc(mask);
+        S.si = 0;
+        S.pos = (int32_t)(pos + 32);
+      }
+      __syncwarp();
+    }
+  }
+}
+
+// ---- touched set, scores ----------------------------------------------------------------------------------
+
+__global__ void k_clear_rows(const int32_t *tids, const SelState *st, unsigned long long *lev, int levels) {
+  const unsigned long long n = st->n_touched;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    for (int l = 0; l < levels; ++l) lev[(size_t)tids[i] * levels + l] = 0;
+}
+
+__global__ void k_deg_bits(const VDesc *vdesc, int32_t n, uint32_t *touched) {
+  const int64_t W = ((int64_t)n + 31) / 32;
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = 0;
+    for (int b = 0; b < 32; ++b) {
+      const int64_t v = w * 32 + b;
+      if (v < n && vdesc[v].len > 0) bits |= 1u << b;
+    }
+    touched[w] = bits;
+  }
+}
+
+__global__ void k_wcount(const uint32_t *touched, int64_t W, uint32_t *wcnt) {
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w <= W; w += (int64_t)gridDim.x * blockDim.x)
+    wcnt[w] = w < W ? __popc(touched[w]) : 0u;
+}
+
+__global__ void k_wwrite(const uint32_t *touched, int64_t W, const uint32_t *woff, int32_t *tids, SelState *st) {
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = touched[w];
+    uint32_t o = woff[w];
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      tids[o++] = (int32_t)(w * 32 + b);
+      bits &= bits - 1;
+    }
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    st->n_touched = woff[W];
+    st->above = 0;
+    st->prefix = 0;
+    st->mask = 0;
+    st->found = 1;
+    st->sel_bytes = 0;
+  }
+}
+
+struct ScoreArgs {
+  int32_t nq;
+  int32_t policy;
+  const unsigned long long *lev[GCSM_MAX_QUERIES];
+  int32_t levels[GCSM_MAX_QUERIES];
+  double N1[GCSM_MAX_QUERIES], M[GCSM_MAX_QUERIES];
+  double powD[GCSM_MAX_QUERIES][8];
+};
+
+// eq. (3) averaged over M (estimator.cpp estimate_value), summed over the queries in registration order
+__global__ void k_score(const ScoreArgs S, const int32_t *tids, const SelState *st, const VDesc *vdesc,
+                        unsigned long long *bits, unsigned long long *bytes) {
+  const unsigned long long n = st->n_touched;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const int32_t v = tids[i];
+    const uint32_t len = vdesc[v].len;
+    double s = 0.0;
+    if (S.policy == 2) {
+      s = (double)len;
+    } else {
+      for (int q = 0; q < S.nq; ++q) {
+        const int L = S.levels[q];
+        const unsigned long long *lv = S.lev[q] + (size_t)v * L;
+        double e = 0.0;
+        for (int l = 0; l < L; ++l) e = DA(e, DM(DM(S.N1[q], S.powD[q][l]), (double)lv[l]));
+        e = DV(e, S.M[q]);
+        s = DA(s, e);
+      }
+    }
+    bits[i] = (unsigned long long)__double_as_longlong(s);
+    bytes[i] = (unsigned long long)((len + 3u) & ~3u) * 4ull;
+  }
+}
+
+// ---- the ranking cut (R23) without a sort --------------------------------------------------------------------
+
+__device__ __forceinline__ int cut_shift(int level) { return level < 5 ? 52 - 12 * level : 0; }
+__device__ __forceinline__ unsigned long long cut_wmask(int level) { return level < 5 ? 4095ull : 15ull; }
+
+__global__ void __launch_bounds__(256) k_hist(const unsigned long long *bits, const unsigned long long *bytes,
+                                              const SelState *st, unsigned long long *hist, int level) {
+  __shared__ unsigned long long h[4096];
+  for (int i = threadIdx.x; i < 4096; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  const unsigned long long n = st->n_touched, mask = st->mask, prefix = st->prefix;
+  const int sh = cut_shift(level);
+  const unsigned long long wm = cut_wmask(level);
+  if (st->found)
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+         i += (unsigned long long)gridDim.x * blockDim.x) {
+      const unsigned long long b = bits[i];
+      if ((long long)b > 0 && (b & mask) == prefix && bytes[i]) atomicAdd(&h[(b >> sh) & wm], bytes[i]);
+    }
+  __syncthreads();
+  for (int i = threadIdx.x; i < 4096; i += blockDim.x)
+    if (h[i]) atomicAdd(hist + (size_t)level * 4096 + i, h[i]);
+}
+
+// One block of 1024 threads: bins in descending order, 4 per thread; the first bin where the cumulative bytes
+// pass the budget is the cut bucket of this level.
+__global__ void __launch_bounds__(1024) k_cut(const unsigned long long *hist, SelState *st, uint64_t budget, int level) {
+  using BS = cub::BlockScan<unsigned long long, 1024>;
+  __shared__ typename BS::TempStorage tmp;
+  __shared__ int win;
+  if (!st->found) return;
+  if (threadIdx.x == 0) win = 1 << 30;
+  const unsigned long long *h = hist + (size_t)level * 4096;
+  const int nbins = level < 5 ? 4096 : 16;
+  unsigned long long v[4], tot = 0;
+  for (int j = 0; j < 4; ++j) {
+    const int d = 4 * threadIdx.x + j;  // descending position
+    v[j] = d < nbins ? h[nbins - 1 - d] : 0ull;
+    tot += v[j];
+  }
+  unsigned long long before;
+  BS(tmp).ExclusiveSum(tot, before);
+  __syncthreads();
+  const unsigned long long above = st->above;
+  unsigned long long cum = above + before;
+  int mine = -1;
+  unsigned long long mine_cum = 0;
+  for (int j = 0; j < 4; ++j) {
+    if (cum + v[j] > budget) {
+      mine = 4 * threadIdx.x + j;
+      mine_cum = cum;
+      break;
+    }
+    cum += v[j];
+  }
+  if (mine >= 0) atomicMin(&win, mine);
+  __syncthreads();
+  if (mine >= 0 && mine == win) {
+    const int bin = nbins - 1 - mine;
+    const int sh = cut_shift(level);
+    st->prefix |= (unsigned long long)bin << sh;
+    st->mask |= cut_wmask(level) << sh;
+    st->above = mine_cum;
+  }
+  if (threadIdx.x == 0 && win == (1 << 30)) st->found = 0;  // everything fits (level 0)
+}
+
+__global__ void k_ties(const unsigned long long *bits, const unsigned long long *bytes, const SelState *st, int64_t cap,
+                       unsigned long long *out) {
+  const unsigned long long n = st->n_touched;
+  const bool found = st->found != 0;
+  const unsigned long long prefix = st->prefix;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cap; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = ((unsigned long long)i < n && found && bits[i] == prefix) ? bytes[i] : 0ull;
+}
+
+// selection flag; scan[i] (tie prefix in, selected bytes out)
+__global__ void k_select(const unsigned long long *bits, const unsigned long long *bytes, SelState *st, int64_t cap,
+                         uint64_t budget, unsigned long long *scan, uint8_t *flag) {
+  const unsigned long long n = st->n_touched;
+  const bool found = st->found != 0;
+  const unsigned long long prefix = st->prefix, above = st->above;
+  unsigned long long used = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cap; i += (int64_t)gridDim.x * blockDim.x) {
+    bool sel = false;
+    if ((unsigned long long)i < n) {
+      const unsigned long long b = bits[i];
+      sel = (long long)b > 0 && (!found || b > prefix || (b == prefix && above + scan[i] <= budget));
+    }
+    flag[i] = sel;
+    const unsigned long long sb = sel ? bytes[i] : 0ull;
+    scan[i] = sb;
+    used += sb;
+  }
+  for (int o = 16; o; o >>= 1) used += __shfl_xor_sync(FULL, used, o);
+  if ((threadIdx.x & 31) == 0 && used) atomicAdd(&st->sel_bytes, used);
+}
+
+// warp per 32 touched entries: copy each selected list (16-byte granules) from where its descriptor points
+__global__ void __launch_bounds__(256) k_copy(const int32_t *tids, const SelState *st, const uint8_t *flag,
+                                              const unsigned long long *off, const unsigned long long *bytes,
+                                              const VDesc *vdesc, char *cache) {
+  const unsigned long long n = st->n_touched;
+  const int lane = threadIdx.x & 31;
+  const unsigned long long nw = (unsigned long long)gridDim.x * (blockDim.x >> 5);
+  for (unsigned long long base = ((unsigned long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32;
+       base < n; base += nw * 32) {
+    const unsigned long long i = base + lane;
+    const bool sel = i < n && flag[i];
+    unsigned mask = __ballot_sync(FULL, sel);
+    while (mask) {
+      const int j = __ffs(mask) - 1;
+      mask &= mask - 1;
+      const unsigned long long e = base + j;
+      const int32_t v = tids[e];
+      const uint4 *src = reinterpret_cast<const uint4 *>(vdesc[v].ptr);
+      uint4 *dst = reinterpret_cast<uint4 *>(cache + off[e]);
+      const unsigned long long g = bytes[e] / 16;
+      unsigned long long t = lane;
+      for (; t + 96 < g; t += 128) {  // 4 x 16 B loads in flight per lane
+        const uint4 a = src[t], b = src[t + 32], c = src[t + 64], d = src[t + 96];
+        dst[t] = a;
+        dst[t + 32] = b;
+        dst[t + 64] = c;
+        dst[t + 96] = d;
+      }
+      for (; t < g; t += 32) dst[t] = src[t];
+    }
+  }
+}
+
+__global__ void k_reset_prev(const int32_t *prev, const SelState *st, VDesc *vdesc, const unsigned long long *hptr) {
+  const unsigned long long n = st->prev_sel;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const int32_t v = prev[i];
+    vdesc[v].ptr = reinterpret_cast<const int32_t *>(hptr[v]);
+  }
+}
+
+__global__ void k_set_new(const int32_t *tids, const SelState *st, const uint8_t *flag, const unsigned long long *off,
+                          VDesc *vdesc, char *cache) {
+  const unsigned long long n = st->n_touched;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    if (flag[i]) vdesc[tids[i]].ptr = reinterpret_cast<const int32_t *>(cache + off[i]);
+}
+
+__global__ void k_sel_stats(SelState *st, unsigned long long *cnt, int has_cache) {
+  if (!has_cache) {
+    st->prev_sel = 0;
+    st->sel_bytes = 0;
+  }
+  cnt[0] = st->prev_sel;
+  cnt[1] = st->sel_bytes;
+  cnt[2] = (unsigned long long)st->err;
+}
+
+__global__ void k_zero_touched_count(SelState *st) { st->n_touched = 0; }
+
+__global__ void k_patch_host(VDesc *vdesc, unsigned long long *hptr, const int64_t *idx, const VDesc *val, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = idx[i];
+    vdesc[v] = val[i];
+    hptr[v] = (unsigned long long)val[i].ptr;
+  }
+}
+
+__global__ void k_est_gather(const int32_t *tids, int64_t n, const unsigned long long *lev, int levels,
+                             unsigned long long *out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    for (int l = 0; l < 8; ++l) out[i * 8 + l] = l < levels ? lev[(size_t)tids[i] * levels + l] : 0ull;
+}
+
+int gs_grid(int64_t n, int per = 256) { return (int)std::max<int64_t>(1, std::min<int64_t>((n + per - 1) / per, 148 * 8)); }
+
+}  // namespace
+
+size_t cache_step_tmp_bytes(int32_t n) {
+  size_t a = 0, b = 0, c = 0;
+  const int64_t W = ((int64_t)n + 31) / 32;
+  cub::DeviceScan::ExclusiveSum(nullptr, a, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(W + 1));
+  // num_items types must match the launches in launch_cache_step (cub's dispatch, hence its scratch size,
+  // depends on them)
+  cub::DeviceScan::InclusiveSum(nullptr, b, (unsigned long long *)nullptr, (unsigned long long *)nullptr, (int)n);
+  size_t b2 = 0;
+  cub::DeviceScan::ExclusiveSum(nullptr, b2, (unsigned long long *)nullptr, (unsigned long long *)nullptr, (int)n);
+  b = std::max(b, b2);
+  cub::DeviceSelect::Flagged(nullptr, c, (int32_t *)nullptr, (uint8_t *)nullptr, (int32_t *)nullptr,
+                             (unsigned long long *)nullptr, (int)n);
+  return std::max(a, std::max(b, c)) + 256;
+}
+
+cudaError_t launch_patch_vdesc_host(VDesc *vdesc, unsigned long long *hptr, const int64_t *idx, const VDesc *val,
+                                    int64_t n, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  k_patch_host<<<gs_grid(n), 256, 0, s>>>(vdesc, hptr, idx, val, n);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_estimates_gather(const int32_t *tids, int64_t n, const unsigned long long *levcnt, int levels,
+                                    unsigned long long *lev_out, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  k_est_gather<<<gs_grid(n), 256, 0, s>>>(tids, n, levcnt, levels, lev_out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *launches) {
+  const int64_t n = c.n, W = (n + 31) / 32;
+  const int G = 148 * 4;
+  uint64_t L = 0;
+  cudaError_t e;
+#define LK(...)                              \
+  do {                                       \
+    __VA_ARGS__;                             \
+    if ((e = cudaGetLastError()) != cudaSuccess) return e; \
+    ++L;                                     \
+  } while (0)
+  if (c.reset_first) {
+    LK(k_reset_prev<<<G, 256, 0, s>>>(c.prev_sel, c.st, c.vdesc, c.hptr));
+    if ((e = cudaMemsetAsync(&c.st->prev_sel, 0, sizeof(unsigned long long), s)) != cudaSuccess) return e;
+  }
+  // last batch's estimator sums are cleared (rows of its touched set)
+  for (int q = 0; q < c.nq; ++q)
+    if (c.q[q].levcnt && c.q[q].k > 2) LK(k_clear_rows<<<G, 256, 0, s>>>(c.tids, c.st, c.q[q].levcnt, c.q[q].k - 2));
+  if (c.policy == 0) {
+    LK(k_zero_touched_count<<<1, 1, 0, s>>>(c.st));
+    LK(k_reset_prev<<<G, 256, 0, s>>>(c.prev_sel, c.st, c.vdesc, c.hptr));
+    LK(k_sel_stats<<<1, 1, 0, s>>>(c.st, c.cnt_cached, 0));
+    *launches += L;
+    return cudaSuccess;
+  }
+  if ((e = cudaMemsetAsync(c.touched, 0, sizeof(uint32_t) * (size_t)W, s)) != cudaSuccess) return e;
+  if (c.policy == 2) {
+    LK(k_deg_bits<<<gs_grid(W), 256, 0, s>>>(c.vdesc, c.n, c.touched));
+  } else {
+    if ((e = cudaMemsetAsync(c.cursor, 0, sizeof(unsigned long long) * c.nq, s)) != cudaSuccess) return e;
+    for (int q = 0; q < c.nq; ++q) {
+      const EstQuery &Q = c.q[q];
+      if (Q.k <= 2 || Q.n_units <= 0) continue;
+      WalkArgs A;
+      A.plans = Q.plans;
+      A.units = Q.units;
+      A.n_units = Q.n_units;
+      A.levcnt = Q.levcnt;
+      A.levels = Q.k - 2;
+      A.vdesc = c.vdesc;
+      A.drec = c.drec;
+      A.dlist = c.dlist;
+      A.lab = c.lab;
+      A.touched = c.touched;
+      A.cursor = c.cursor + q;
+      A.T.pD = c.pD;
+      A.T.r0tab = c.r0tab;
+      A.T.r0n = c.r0n;
+      A.T.sfc = nullptr;  // set to the block's shared copy of A.sfc
+      A.T.err = &c.st->err;
+      for (int i = 0; i < 10; ++i) A.sfc[i] = c.sfc[i];
+      const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((Q.n_units + kEW - 1) / kEW, 148 * 6));
+      LK(k_walks<<<grid, kEW * 32, 0, s>>>(A));
+    }
+  }
+  // touched set in id order
+  uint32_t *wcnt = c.wcnt;
+  uint32_t *woff = c.woff;
+  LK(k_wcount<<<gs_grid(W + 1), 256, 0, s>>>(c.touched, W, wcnt));
+  size_t tb = c.cub_tmp_bytes;
+  if ((e = cub::DeviceScan::ExclusiveSum(c.cub_tmp, tb, wcnt, woff, (int)(W + 1), s)) != cudaSuccess) return e;
+  ++L;
+  LK(k_wwrite<<<gs_grid(W), 256, 0, s>>>(c.touched, W, woff, c.tids, c.st));
+  ScoreArgs S{};
+  S.nq = c.nq;
+  S.policy = c.policy;
+  for (int q = 0; q < c.nq; ++q) {
+    S.lev[q] = c.q[q].levcnt;
+    S.levels[q] = c.q[q].k > 2 ? c.q[q].k - 2 : 0;
+    S.N1[q] = (double)c.q[q].N1;
+    S.M[q] = (double)c.q[q].M;
+    for (int l = 0; l < 8; ++l) S.powD[q][l] = c.q[q].powD[l];
+    if (!c.q[q].levcnt || c.q[q].n_units <= 0) S.levels[q] = 0, S.M[q] = 1.0;
+  }
+  LK(k_score<<<G, 256, 0, s>>>(S, c.tids, c.st, c.vdesc, c.bits, c.bytes));
+  if ((e = cudaMemsetAsync(c.hist, 0, sizeof(unsigned long long) * 6 * 4096, s)) != cudaSuccess) return e;
+  for (int lv = 0; lv < 6; ++lv) {
+    LK(k_hist<<<G, 256, 0, s>>>(c.bits, c.bytes, c.st, c.hist, lv));
+    LK(k_cut<<<1, 1024, 0, s>>>(c.hist, c.st, c.budget, lv));
+  }
+  LK(k_ties<<<G, 256, 0, s>>>(c.bits, c.bytes, c.st, n, c.off));
+  tb = c.cub_tmp_bytes;
+  if ((e = cub::DeviceScan::InclusiveSum(c.cub_tmp, tb, c.off, c.scan, (int)n, s)) != cudaSuccess) return e;
+  ++L;
+  LK(k_select<<<G, 256, 0, s>>>(c.bits, c.bytes, c.st, n, c.budget, c.scan, c.flag));
+  tb = c.cub_tmp_bytes;
+  if ((e = cub::DeviceScan::ExclusiveSum(c.cub_tmp, tb, c.scan, c.off, (int)n, s)) != cudaSuccess) return e;
+  ++L;
+  LK(k_copy<<<G, 256, 0, s>>>(c.tids, c.st, c.flag, c.off, c.bytes, c.vdesc, c.cache));
+  LK(k_reset_prev<<<G, 256, 0, s>>>(c.prev_sel, c.st, c.vdesc, c.hptr));
+  LK(k_set_new<<<G, 256, 0, s>>>(c.tids, c.st, c.flag, c.off, c.vdesc, c.cache));
+  tb = c.cub_tmp_bytes;
+  if ((e = cub::DeviceSelect::Flagged(c.cub_tmp, tb, c.tids, c.flag, c.prev_sel, &c.st->prev_sel, (int)n, s)) != cudaSuccess)
+    return e;
+  ++L;
+  LK(k_sel_stats<<<1, 1, 0, s>>>(c.st, c.cnt_cached, 1));
+#undef LK
+  *launches += L;
+  return cudaSuccess;
+}
+
+}  // namespace gcsm

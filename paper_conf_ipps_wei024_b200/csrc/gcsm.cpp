@@ -17,6 +17,7 @@
 
 #include "estimator.h"
 #include "internal.h"
+#include "estimator_gpu.cuh"
 #include "kernels.cuh"
 #include "store.h"
 
@@ -85,6 +86,11 @@ struct gcsm_ctx {
     uint64_t *h_gather = nullptr; size_t h_gather_cap = 0;
     uint64_t *h_fresh = nullptr; size_t h_fresh_cap = 0;
     unsigned long long *h_cnt = nullptr;  // CNT_N per query
+    EstUnit *h_eunits = nullptr; size_t h_eunits_cap = 0;  // level-1 walk nodes (GPU estimator)
+    int32_t *h_ulist = nullptr; size_t h_ulist_cap = 0;    // stable lists S(x) of U, packed (GPU path)
+    int32_t *d_ulist = nullptr; size_t d_ulist_cap = 0;    // their device copy (read by this batch's kernels)
+    size_t ulist_n = 0;
+    double *h_r0 = nullptr; size_t h_r0_cap = 0;           // BINV table staging
     cudaEvent_t ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr, ev_c1 = nullptr, ev_done = nullptr;
     struct PerQuery {
       cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr;
@@ -134,6 +140,26 @@ struct gcsm_ctx {
   Task *d_tasks = nullptr; size_t tasks_cap = 0;
   int32_t *d_task_ready = nullptr; size_t task_ready_cap = 0;
   int32_t task_gen = 0;
+  // GPU estimator + cache packer (steps 2-3 on the device, estimator_gpu.cu; default). GCSM_HOST_EST=1 at create
+  // selects the host walker and host packer instead (the paper's CPU placement, kept for A/B measurements).
+  bool gpu_est = true;
+  bool gpu_ready = false;          // the n-sized buffers below exist
+  bool cache_reset = false;        // the last selection's descriptors must go back to host before the next batch
+  unsigned long long *d_hptr = nullptr;  // host address of every vertex's main list
+  uint32_t *d_touched = nullptr, *d_wcnt = nullptr, *d_woff = nullptr;
+  int32_t *d_tids = nullptr, *d_prev_sel = nullptr;
+  unsigned long long *d_bits = nullptr, *d_bytes = nullptr, *d_scan = nullptr, *d_off = nullptr;
+  uint8_t *d_flag = nullptr;
+  unsigned long long *d_selhist = nullptr, *d_ecursor = nullptr;
+  SelState *d_sel = nullptr;
+  void *d_cubtmp = nullptr; size_t cubtmp_bytes = 0;
+  unsigned long long *d_levcnt[GCSM_MAX_QUERIES] = {};
+  int lev_levels[GCSM_MAX_QUERIES] = {-1, -1, -1, -1, -1, -1, -1, -1};
+  EstUnit *d_eunits = nullptr; size_t eunits_cap = 0;
+  double *d_r0 = nullptr; size_t r0_cap = 0;
+  size_t r0_n = 0;                 // entries of the device table of (1 - pD)^n
+  double r0_pD = -1.0;
+  bool est_valid = false;          // the device holds a batch's estimator output (gcsm_get_estimates)
 
 
   // cache / batch state
@@ -171,8 +197,16 @@ gcsm_ctx::~gcsm_ctx() {
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (void *p : dev)
     if (p) cudaFree(p);
+  void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
+                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0};
+  for (void *p : dev2)
+    if (p) cudaFree(p);
+  for (unsigned long long *p : d_levcnt)
+    if (p) cudaFree(p);
   for (Slot &sl : slots) {
-    void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt};
+    void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt,
+                    sl.h_eunits, sl.h_ulist, sl.h_r0};
+    if (sl.d_ulist) cudaFree(sl.d_ulist);
     for (void *p : host)
       if (p) cudaFreeHost(p);
     for (cudaEvent_t e : {sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done})
@@ -271,6 +305,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   }
   ctx->mark.assign(n, 0);
   ctx->slot16.assign(n, 0);
+  if (const char *he = std::getenv("GCSM_HOST_EST")) ctx->gpu_est = std::atoi(he) == 0;
   ctx->grid = match_grid(dev, &ctx->warps_total);
   // a communicator whenever an id is given (world 1 included: the single-rank allreduce exercises the same path)
   if (o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
@@ -321,6 +356,10 @@ static gcsm_status add_query_impl(gcsm_ctx *ctx, bool reset, int32_t k, int32_t 
   CK(upload_plans(dp, q.qp.plans.data(), (int)q.qp.plans.size(), ctx->stream));
   CK(upload_plans(dsp, q.qps.plans.data(), (int)q.qps.plans.size(), ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
+  if (reset)
+    for (int &l : ctx->lev_levels) l = -1;  // walk sums of other patterns are stale: re-zeroed on next use
+  else
+    ctx->lev_levels[slot] = -1;
   if (reset) {
     for (size_t i = 1; i < ctx->qs.size(); ++i) {
       cudaFree(ctx->qs[i].d_plans);
@@ -365,6 +404,7 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
   ctx->budget = bytes;
   ctx->cache_valid = false;  // the next batch repacks everything
   for (int32_t v : ctx->prev_cached) ctx->slot16[v] = 0;
+  ctx->cache_reset = true;   // GPU packer: the previous selection's descriptors may point into a freed buffer
   return GCSM_OK;
 }
 
@@ -431,6 +471,145 @@ struct Trace {
     if (on) std::fprintf(stderr, "[gcsm trace]%s\n", line.c_str());
   }
 };
+
+// GPU path of steps (2)-(3) (estimator_gpu.cu): uploads the batch's delta records, units, changed descriptors (host
+// addresses) and level-1 walk nodes, then enqueues the walks, the ranking cut and the cache copy on the stream.
+static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStream_t s, size_t ndirty, size_t nU,
+                                     size_t nd, int64_t gnu, const std::vector<std::vector<EstUnit>> &qeu,
+                                     uint64_t maxB, uint64_t D, const std::vector<int64_t> &qnu,
+                                     const std::vector<uint64_t> &qwalks, bool use_cache, uint64_t *launches) {
+  HostStore &S = ctx->store;
+  const int32_t n = S.n;
+  const int nq = (int)ctx->qs.size();
+  if (!ctx->gpu_ready) {
+    const size_t W = ((size_t)n + 31) / 32 + 1;
+    std::vector<unsigned long long> hp((size_t)n);
+    for (int32_t v = 0; v < n; ++v) hp[v] = (unsigned long long)(uintptr_t)S.dev_ptr(S.lst[v]);
+    ctx->cubtmp_bytes = cache_step_tmp_bytes(n);
+    if (cudaMalloc(&ctx->d_hptr, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_touched, 4 * W) != cudaSuccess ||
+        cudaMalloc(&ctx->d_wcnt, 4 * W) != cudaSuccess || cudaMalloc(&ctx->d_woff, 4 * W) != cudaSuccess ||
+        cudaMalloc(&ctx->d_tids, 4 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_prev_sel, 4 * (size_t)n) != cudaSuccess ||
+        cudaMalloc(&ctx->d_bits, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_bytes, 8 * (size_t)n) != cudaSuccess ||
+        cudaMalloc(&ctx->d_scan, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_off, 8 * (size_t)n) != cudaSuccess ||
+        cudaMalloc(&ctx->d_flag, (size_t)n) != cudaSuccess ||
+        cudaMalloc(&ctx->d_selhist, 8 * 6 * 4096) != cudaSuccess ||
+        cudaMalloc(&ctx->d_ecursor, 8 * GCSM_MAX_QUERIES) != cudaSuccess ||
+        cudaMalloc(&ctx->d_sel, sizeof(SelState)) != cudaSuccess ||
+        cudaMalloc(&ctx->d_cubtmp, ctx->cubtmp_bytes) != cudaSuccess)
+      return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
+    CK(cudaMemcpyAsync(ctx->d_hptr, hp.data(), 8 * (size_t)n, cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(ctx->d_sel, 0, sizeof(SelState), s));
+    CK(cudaStreamSynchronize(s));  // hp is pageable and local
+    ctx->gpu_ready = true;
+  }
+  const bool est_on = use_cache && ctx->opt.cache_policy == GCSM_CACHE_ESTIMATOR;
+  for (int qi = 0; qi < nq; ++qi) {  // dense per-vertex walk sums (zero outside the last touched set)
+    const int L = ctx->qs[qi].qp.k - 2;
+    if (L <= 0 || ctx->lev_levels[qi] == L) continue;
+    if (ctx->d_levcnt[qi]) cudaFree(ctx->d_levcnt[qi]);
+    ctx->d_levcnt[qi] = nullptr;
+    if (cudaMalloc(&ctx->d_levcnt[qi], 8 * (size_t)n * L) != cudaSuccess)
+      return ctx->fail(GCSM_ENOMEM, "estimator sums");
+    CK(cudaMemsetAsync(ctx->d_levcnt[qi], 0, 8 * (size_t)n * L, s));
+    ctx->lev_levels[qi] = L;
+  }
+  // binomial tables: BINV's r0 = (1 - 1/D)^n (host pow, as the host walker computes it) for n up to the largest
+  // level-1 multiplicity inside BINV's domain n p < 10 (children draw with n <= their parent's B); rebuilt when
+  // D changes or the batch needs more entries, staged in this slot's pinned buffer and copied on the stream
+  const double pD = 1.0 / (double)D;
+  if (est_on) {
+    int64_t nlim = (int64_t)std::ceil(10.0 / pD) + 2;
+    while (nlim > 0 && (double)nlim * pD >= 10.0) --nlim;
+    const size_t need = (size_t)std::min<int64_t>((int64_t)maxB, nlim) + 1;
+    if (pD != ctx->r0_pD || need > ctx->r0_n) {
+      const size_t want = std::min<size_t>((size_t)nlim + 1, std::max<size_t>(2 * need, 4096));
+      if (!host_ensure(sl.h_r0, sl.h_r0_cap, want)) return ctx->fail(GCSM_ENOMEM, "r0 table");
+      double *h = sl.h_r0;
+      parallel_for(ctx->opt.host_threads, (int64_t)want, [&](int, int64_t lo, int64_t hi) {
+        for (int64_t i = lo; i < hi; ++i) h[i] = std::pow(1.0 - pD, (double)i);
+      });
+      if (!dev_ensure(ctx->d_r0, ctx->r0_cap, want)) return ctx->fail(GCSM_ENOMEM, "r0 table");
+      CK(cudaMemcpyAsync(ctx->d_r0, h, 8 * want, cudaMemcpyHostToDevice, s));
+      ctx->r0_pD = pD;
+      ctx->r0_n = want;
+    }
+  }
+  // uploads
+  size_t neu = 0;
+  for (const auto &eu : qeu) neu += eu.size();
+  if (!host_ensure(sl.h_eunits, sl.h_eunits_cap, neu) || !dev_ensure(ctx->d_eunits, ctx->eunits_cap, neu))
+    return ctx->fail(GCSM_ENOMEM, "walk roots");
+  {
+    size_t o = 0;
+    for (const auto &eu : qeu) {
+      if (!eu.empty()) std::memcpy(sl.h_eunits + o, eu.data(), sizeof(EstUnit) * eu.size());
+      o += eu.size();
+    }
+  }
+  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
+  if (sl.ulist_n) CK(cudaMemcpyAsync(sl.d_ulist, sl.h_ulist, 4 * sl.ulist_n, cudaMemcpyHostToDevice, s));
+  if (nU) CK(cudaMemcpyAsync(ctx->d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
+  if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
+  if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
+  if (neu) CK(cudaMemcpyAsync(ctx->d_eunits, sl.h_eunits, sizeof(EstUnit) * neu, cudaMemcpyHostToDevice, s));
+  if (ndirty) {
+    CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * ndirty, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * ndirty, cudaMemcpyHostToDevice, s));
+    CK(launch_patch_vdesc_host(ctx->d_vdesc, ctx->d_hptr, ctx->d_pidx, ctx->d_pval, (int64_t)ndirty, s));
+    ++*launches;
+  }
+  CacheStep c{};
+  c.n = n;
+  c.nq = nq;
+  size_t o = 0;
+  for (int qi = 0; qi < nq; ++qi) {
+    EstQuery &q = c.q[qi];
+    const int k = ctx->qs[qi].qp.k;
+    q.plans = ctx->qs[qi].d_plans;
+    q.units = ctx->d_eunits + o;
+    q.n_units = est_on ? (int64_t)qeu[qi].size() : 0;
+    o += qeu[qi].size();
+    q.levcnt = k > 2 ? ctx->d_levcnt[qi] : nullptr;
+    q.k = k;
+    q.N1 = (uint64_t)std::max<int64_t>(qnu[qi], 1);
+    q.M = std::max<uint64_t>(qwalks[qi], 1);
+    for (int l = 0; l < 8; ++l) q.powD[l] = std::pow((double)D, (double)l);
+  }
+  c.policy = use_cache ? (ctx->opt.cache_policy == GCSM_CACHE_DEGREE ? 2 : 1) : 0;
+  c.reset_first = ctx->cache_reset;
+  ctx->cache_reset = false;
+  c.budget = ctx->budget;
+  c.vdesc = ctx->d_vdesc;
+  c.hptr = ctx->d_hptr;
+  c.drec = ctx->d_drec;
+  c.dlist = ctx->d_dlist;
+  c.lab = ctx->d_lab;
+  c.pD = pD;
+  c.r0tab = ctx->d_r0;
+  c.r0n = (int64_t)ctx->r0_n;
+  for (int i = 0; i < 10; ++i) c.sfc[i] = stirling_small(i);
+  c.touched = ctx->d_touched;
+  c.wcnt = ctx->d_wcnt;
+  c.woff = ctx->d_woff;
+  c.tids = ctx->d_tids;
+  c.bits = ctx->d_bits;
+  c.bytes = ctx->d_bytes;
+  c.scan = ctx->d_scan;
+  c.off = ctx->d_off;
+  c.flag = ctx->d_flag;
+  c.prev_sel = ctx->d_prev_sel;
+  c.hist = ctx->d_selhist;
+  c.st = ctx->d_sel;
+  c.cursor = ctx->d_ecursor;
+  c.cub_tmp = ctx->d_cubtmp;
+  c.cub_tmp_bytes = ctx->cubtmp_bytes;
+  c.cache = ctx->d_cache;
+  c.cnt_cached = ctx->d_cnt + CNT_CACHED;
+  CK(launch_cache_step(c, s, launches));
+  ctx->est_valid = est_on;
+  CK(cudaEventRecord(sl.ev_c1, s));
+  return GCSM_OK;
+}
 
 // Host steps (1)-(3) of one batch, its GPU work (3)-(4b) enqueued on the stream, and its host merge (5) into
 // fresh arrays; returns without waiting for the kernels (gcsm_wait_batch collects the counts).
@@ -555,7 +734,51 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const bool use_cache = ctx->budget > 0 && ctx->opt.cache_policy != GCSM_CACHE_NONE && kmax > 2;
   std::vector<double> qms_est((size_t)nq, 0.0);
   std::vector<uint64_t> qwalks((size_t)nq, 0);
-  for (int qi = 0; qi < nq; ++qi) {
+  // GPU path: the level-1 nodes of the walks (a unit, its key of R22 and its draw B_1 ~ Bin(M, 1/N1)) are
+  // made here (N1 draws); everything below level 1 runs in k_walks (estimator_gpu.cu)
+  std::vector<std::vector<EstUnit>> qeu(ctx->gpu_est ? (size_t)nq : 0);
+  uint64_t eu_maxB = 0;
+  if (ctx->gpu_est) {
+    for (int qi = 0; qi < nq; ++qi) {
+      Timer tq;
+      const QueryPlan &Q = ctx->qs[qi].qp;
+      const int k = Q.k;
+      const int64_t nu = qnu[qi];
+      if (k > 2 && nu > 0) {
+        const uint64_t M = ctx->opt.walks_override ? ctx->opt.walks_override : walk_budget((uint64_t)nu, D, k);
+        qwalks[qi] = M;
+        if (ctx->opt.cache_policy == GCSM_CACHE_ESTIMATOR && ctx->budget > 0) {
+          const uint64_t seed = qi == 0 ? ctx->opt.seed : rng_chain(ctx->opt.seed, 0x51ull + (uint64_t)qi);
+          const uint64_t root = rng_mix(seed);
+          const double p1 = 1.0 / (double)nu;
+          const std::vector<Unit> &units = qunits[qi];
+          std::vector<EstUnit> all((size_t)nu);
+          parallel_for(T, nu, [&](int, int64_t lo, int64_t hi) {
+            for (int64_t i = lo; i < hi; ++i) {
+              const Unit &u = units[i];
+              const uint64_t key =
+                  rng_chain(rng_chain(rng_chain(rng_chain(rng_chain(root, ctx->batch_seq), (uint64_t)(u.plan >> 1)),
+                                                (uint64_t)(u.plan & 1)),
+                                      (uint64_t)(uint32_t)u.a),
+                            (uint64_t)(uint32_t)u.b);
+              const int64_t B = binomial(key, (int64_t)M, p1);
+              all[i] = EstUnit{u.a, u.b, u.plan, 0, (unsigned long long)std::max<int64_t>(B, 0), key};
+            }
+          });
+          std::vector<EstUnit> &eu = qeu[qi];
+          eu.reserve(all.size());
+          for (const EstUnit &x : all)
+            if (x.B > 0) {
+              eu.push_back(x);
+              eu_maxB = std::max<uint64_t>(eu_maxB, x.B);
+            }
+        }
+      }
+      qms_est[qi] = tq.ms();
+    }
+    tr.mark("walk_roots");
+  }
+  for (int qi = 0; qi < nq && !ctx->gpu_est; ++qi) {
     Timer tq;
     const QueryPlan &Q = ctx->qs[qi].qp;
     const int k = Q.k;
@@ -599,7 +822,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     qms_est[qi] = tq.ms();
   }
   st.walks = qwalks[0];
-  if (use_cache && ctx->opt.cache_policy == GCSM_CACHE_DEGREE) {
+  if (use_cache && ctx->opt.cache_policy == GCSM_CACHE_DEGREE && !ctx->gpu_est) {
     ranked.reserve(S.n);
     for (int32_t v = 0; v < S.n; ++v) {
       const uint32_t d = S.view_len(v, VIEW_S);
@@ -641,7 +864,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   uint64_t new_bytes = 0;
   const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
   ctx->d_cache = ctx->d_cachebuf[tgt];
-  if (use_cache && !ranked.empty()) {
+  if (use_cache && !ranked.empty() && !ctx->gpu_est) {
     // Only the head of the ranking can fit the budget: bucket the (positive) scores by the top 12 bits of their
     // IEEE pattern (monotone in the score), then the next 12 inside the bucket where the cumulative list bytes
     // pass the budget, and sort just the vertices at or above that cut (per-thread histograms, parallel
@@ -775,8 +998,10 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   st.cache_bytes = used;
   // descriptors to patch: previous cache / updated sets and the new ones
   std::vector<int32_t> dirty;
+  static const std::vector<int32_t> kNone;
   {
-    const std::vector<int32_t> *srcs[4] = {&ctx->prev_cached, &ctx->prev_U, &S.U, &sel};
+    const std::vector<int32_t> *srcs[4] = {ctx->gpu_est ? &kNone : &ctx->prev_cached, &ctx->prev_U, &S.U,
+                                           ctx->gpu_est ? &kNone : &sel};
     std::vector<int64_t> base(5, 0);
     for (int i = 0; i < 4; ++i) base[i + 1] = base[i] + (int64_t)srcs[i]->size();
     const int nt = std::max(1, std::min(T, pool_size()));
@@ -799,6 +1024,21 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   if (!host_ensure(sl.h_pidx, sl.h_pidx_cap, dirty.size()) ||
       !host_ensure(sl.h_pval, sl.h_pval_cap, dirty.size()))
     return ctx->fail(GCSM_ENOMEM, "pinned staging");
+  // GPU path: the stable lists S(x) of U travel with the batch (packed, 16-byte aligned, one DMA into this slot's
+  // device buffer): every kernel of the batch reads them from HBM instead of re-reading the host overlays
+  std::vector<uint64_t> ul_off;
+  if (ctx->gpu_est) {
+    const size_t nU0 = S.U.size();
+    ul_off.assign(nU0 + 1, 0);
+    for (size_t i = 0; i < nU0; ++i) ul_off[i + 1] = ul_off[i] + ((S.s_len[i] + 3u) & ~3u);
+    sl.ulist_n = ul_off[nU0];
+    if (!host_ensure(sl.h_ulist, sl.h_ulist_cap, sl.ulist_n) || !dev_ensure(sl.d_ulist, sl.d_ulist_cap, sl.ulist_n))
+      return ctx->fail(GCSM_ENOMEM, "stable lists of U");
+    parallel_for(T, (int64_t)nU0, [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i)
+        if (S.s_len[i]) std::memcpy(sl.h_ulist + ul_off[i], S.s_ptr[i], 4 * (size_t)S.s_len[i]);
+    });
+  }
   parallel_for(T, (int64_t)dirty.size(), [&](int, int64_t lo, int64_t hi) {
     for (int64_t i = lo; i < hi; ++i) {
       const int32_t v = dirty[i];
@@ -808,6 +1048,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       d.len = ui >= 0 ? S.s_len[ui] : S.len[v];
       const int32_t si = ctx->sel_index[v];
       d.ptr = si >= 0 ? (const int32_t *)(ctx->d_cache + sel_off[si]) : S.dev_ptr(ui >= 0 ? S.s_ptr[ui] : S.lst[v]);
+      if (ctx->gpu_est && ui >= 0) d.ptr = sl.d_ulist + ul_off[ui];
       sl.h_pidx[i] = v;
       sl.h_pval[i] = d;
     }
@@ -837,6 +1078,16 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)gnu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)gnu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
   CK(cudaEventRecord(sl.ev_c0, s));
+  uint64_t launches = 0;
+  if (ctx->gpu_est) {
+    gcsm_status gs = enqueue_gpu_cache(ctx, sl, s, dirty.size(), nU, nd, gnu, qeu, eu_maxB, D, qnu, qwalks, use_cache,
+                                       &launches);
+    if (gs != GCSM_OK) return gs;
+    st.h2d_bytes = (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU + 4 * nd +
+                   sizeof(Unit) * (size_t)gnu;
+    for (const auto &eu : qeu) st.h2d_bytes += sizeof(EstUnit) * eu.size();
+    st.h2d_bytes += 4 * sl.ulist_n;
+  } else {
   const uint64_t retained_bytes = used - new_bytes;
   if (!gather.empty()) {  // HBM -> HBM copy of the retained lists from the previous buffer
     if (!host_ensure(sl.h_gather, sl.h_gather_cap, gather.size()) ||
@@ -858,13 +1109,15 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(launch_patch_vdesc(ctx->d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
-  uint64_t launches = dirty.empty() ? 0 : 1;
+  launches += dirty.empty() ? 0 : 1;
   if (nU) CK(cudaMemcpyAsync(ctx->d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
   if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
   if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(sl.ev_c1, s));
   st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
                  4 * nd + sizeof(Unit) * (size_t)gnu;
+  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
+  }
 
   // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
@@ -915,7 +1168,6 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     d_tadd = ctx->d_tup;
     d_trem = ctx->d_tup + (size_t)k * add_cap;
   }
-  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
   MatchArgs A{};
   A.vdesc = ctx->d_vdesc;
   A.lab = ctx->d_lab;
@@ -930,6 +1182,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.dcap = dcap;
   A.cache_lo = ctx->d_cache;
   A.cache_hi = ctx->d_cache ? ctx->d_cache + ctx->cache_cap : nullptr;
+  A.ubuf_lo = ctx->gpu_est ? reinterpret_cast<const char *>(sl.d_ulist) : nullptr;
+  A.ubuf_hi = ctx->gpu_est ? reinterpret_cast<const char *>(sl.d_ulist + sl.ulist_n) : nullptr;
   A.tup_add = d_tadd;
   A.tup_add_cap = add_cap;
   A.tup_rem = d_trem;
@@ -1036,13 +1290,15 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   Timer t5;
   if (!S.merge(sl.retired)) return ctx->fail(GCSM_ENOMEM, "pinned allocation for the merged lists failed");
   tr.mark("merge");
-  parallel_for(T, (int64_t)ctx->prev_cached.size(), [&](int, int64_t lo, int64_t hi) {
-    for (int64_t i = lo; i < hi; ++i) ctx->slot16[ctx->prev_cached[i]] = 0;
-  });
-  parallel_for(T, (int64_t)sel.size(), [&](int, int64_t lo, int64_t hi) {
-    for (int64_t i = lo; i < hi; ++i) ctx->slot16[sel[i]] = (uint32_t)(sel_off[i] / 16) + 1;
-  });
-  ctx->prev_cached.swap(sel);  // selection order (gcsm_get_cached sorts its copy)
+  if (!ctx->gpu_est) {
+    parallel_for(T, (int64_t)ctx->prev_cached.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i) ctx->slot16[ctx->prev_cached[i]] = 0;
+    });
+    parallel_for(T, (int64_t)sel.size(), [&](int, int64_t lo, int64_t hi) {
+      for (int64_t i = lo; i < hi; ++i) ctx->slot16[sel[i]] = (uint32_t)(sel_off[i] / 16) + 1;
+    });
+    ctx->prev_cached.swap(sel);  // selection order (gcsm_get_cached sorts its copy)
+  }
   if (ctx->budget > 0) {
     ctx->cache_cur = tgt;
     ctx->cache_valid = true;
@@ -1077,6 +1333,12 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     gcsm_stats st = pq.st;
     const unsigned long long *h = sl.h_cnt + (size_t)qi * CNT_N;
     if (h[CNT_OVERFLOW]) return ctx->fail(GCSM_EDEVICE, "internal: level-2 frontier overflow");
+    if (ctx->gpu_est) {  // the GPU packer's selection (query 0's counter block; shared by all queries)
+      const unsigned long long *h0 = sl.h_cnt;
+      if (h0[CNT_CACHED + 2]) return ctx->fail(GCSM_EDEVICE, "internal: GPU estimator binomial table");
+      st.cached_vertices = h0[CNT_CACHED];
+      st.cache_bytes = h0[CNT_CACHED + 1];
+    }
     float ms_m = 0;
     cudaEventElapsedTime(&ms_m, pq.ev_m0, pq.ev_m1);
     st.ms_match = ms_m;
@@ -1195,6 +1457,40 @@ gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col,
 
 gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levcnt, uint64_t cap, uint64_t *n_out) {
   if (!ctx || !n_out) return GCSM_EINVAL;
+  if (ctx->gpu_est) {  // device-resident walk sums of the last batch (query 0): rows of the touched set, non-zero
+    *n_out = 0;
+    if (!ctx->est_valid || ctx->qs.empty() || ctx->qs[0].qp.k <= 2 || !ctx->d_levcnt[0]) return GCSM_OK;
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) return GCSM_EDEVICE;
+    SelState st;
+    if (cudaMemcpy(&st, ctx->d_sel, sizeof st, cudaMemcpyDeviceToHost) != cudaSuccess) return GCSM_EDEVICE;
+    const int64_t nt = (int64_t)st.n_touched;
+    std::vector<int32_t> tid((size_t)nt);
+    std::vector<unsigned long long> rows((size_t)nt * 8);
+    unsigned long long *d_rows = nullptr;
+    if (nt) {
+      if (cudaMalloc(&d_rows, 8 * 8 * (size_t)nt) != cudaSuccess) return GCSM_ENOMEM;
+      cudaError_t e = launch_estimates_gather(ctx->d_tids, nt, ctx->d_levcnt[0], ctx->qs[0].qp.k - 2, d_rows,
+                                              ctx->stream);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+      if (e == cudaSuccess) e = cudaMemcpy(rows.data(), d_rows, 8 * 8 * (size_t)nt, cudaMemcpyDeviceToHost);
+      if (e == cudaSuccess) e = cudaMemcpy(tid.data(), ctx->d_tids, 4 * (size_t)nt, cudaMemcpyDeviceToHost);
+      cudaFree(d_rows);
+      if (e != cudaSuccess) return GCSM_EDEVICE;
+    }
+    uint64_t w = 0;
+    for (int64_t i = 0; i < nt; ++i) {
+      unsigned long long sum = 0;
+      for (int l = 0; l < 8; ++l) sum |= rows[(size_t)i * 8 + l];
+      if (!sum) continue;  // read only by other queries' walks
+      if (w < cap) {
+        if (ids) ids[w] = tid[i];
+        if (levcnt) std::memcpy(levcnt + 8 * w, &rows[(size_t)i * 8], 64);
+      }
+      ++w;
+    }
+    *n_out = w;
+    return w > cap ? GCSM_ETRUNC : GCSM_OK;
+  }
   static const EstimatorOutput none;
   const EstimatorOutput &est = ctx->qs.empty() ? none : ctx->qs[0].est;
   const uint64_t n = est.ids.size();
@@ -1207,6 +1503,17 @@ gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levc
 
 gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out) {
   if (!ctx || !n_out) return GCSM_EINVAL;
+  if (ctx->gpu_est) {  // the GPU packer's last selection (ids ascending)
+    *n_out = 0;
+    if (!ctx->gpu_ready) return GCSM_OK;
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) return GCSM_EDEVICE;
+    SelState st;
+    if (cudaMemcpy(&st, ctx->d_sel, sizeof st, cudaMemcpyDeviceToHost) != cudaSuccess) return GCSM_EDEVICE;
+    const uint64_t n = st.prev_sel, w = std::min<uint64_t>(n, cap);
+    *n_out = n;
+    if (ids && w && cudaMemcpy(ids, ctx->d_prev_sel, 4 * w, cudaMemcpyDeviceToHost) != cudaSuccess) return GCSM_EDEVICE;
+    return n > cap ? GCSM_ETRUNC : GCSM_OK;
+  }
   std::vector<int32_t> cached = ctx->prev_cached;
   std::sort(cached.begin(), cached.end());
   const uint64_t n = cached.size();

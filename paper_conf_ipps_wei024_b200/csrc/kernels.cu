@@ -111,8 +111,10 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
     }
   }
   const char *p = reinterpret_cast<const char *>(r.m);
-  r.dev = p >= A.cache_lo && p < A.cache_hi;
-  if (r.dev) acc.hit += 4ull * r.ml;
+  const bool in_cache = p >= A.cache_lo && p < A.cache_hi, in_ubuf = p >= A.ubuf_lo && p < A.ubuf_hi;
+  r.dev = in_cache || in_ubuf;
+  if (in_cache) acc.hit += 4ull * r.ml;
+  else if (in_ubuf) acc.delta += 4ull * r.ml;  // the batch's uploaded stable lists of U (device-resident deltas)
   else acc.miss += 4ull * r.ml;
   acc.delta += 4ull * r.xl;
   if (v == pin.v) {  // served from this warp's staged copy
@@ -172,8 +174,10 @@ __device__ GCSM_COLD uint32_t warp_isect(const MatchArgs &A, const int32_t *dset
   return found;
 }
 
+// device-resident main list: the HBM cache or the batch's uploaded stable lists of U
 __device__ __forceinline__ bool is_hit(const MatchArgs &A, const int32_t *p) {
-  return reinterpret_cast<const char *>(p) >= A.cache_lo && reinterpret_cast<const char *>(p) < A.cache_hi;
+  const char *c = reinterpret_cast<const char *>(p);
+  return (c >= A.cache_lo && c < A.cache_hi) || (c >= A.ubuf_lo && c < A.ubuf_hi);
 }
 
 // A list already in device memory outside the cache (a warp's staged copy in its HBM scratch).
@@ -933,8 +937,11 @@ __device__ __forceinline__ LR lr_make(const MatchArgs &A, const int4 r, int xl, 
   l.ml = (uint32_t)r.z;
   l.x = xl ? A.dlist + r.w : nullptr;
   l.xl = (uint32_t)xl;
+  const char *c = reinterpret_cast<const char *>(l.m);
+  const bool in_ubuf = c >= A.ubuf_lo && c < A.ubuf_hi;
   l.dev = is_hit(A, l.m);
-  if (l.dev) acc.hit += 4ull * l.ml;
+  if (in_ubuf) acc.delta += 4ull * l.ml;
+  else if (l.dev) acc.hit += 4ull * l.ml;
   else acc.miss += 4ull * l.ml;
   acc.delta += 4ull * l.xl;
   return l;

@@ -29,7 +29,8 @@ enum Counter {
   CNT_DBG_RUNS = 21,     // k_last4: x2 runs started (GCSM_TRACE)
   CNT_DBG_PINBYTES = 22, // k_last4: zero-copy bytes copied by run pins
   CNT_DBG_PINS = 23,     // k_last4: runs pinned
-  CNT_N = 24
+  CNT_CACHED = 24,       // GPU packer (query 0's block): cached vertices, cached bytes, internal error flag
+  CNT_N = 27
 };
 
 struct MatchArgs {
@@ -50,6 +51,7 @@ struct MatchArgs {
   int32_t dcap;             // ints per stack level (>= max list length)
   unsigned long long *cnt;  // CNT_N counters
   const char *cache_lo, *cache_hi;  // HBM cache address range (hit/miss accounting)
+  const char *ubuf_lo, *ubuf_hi;    // the batch's uploaded stable lists of U (device-resident, delta accounting)
   int32_t *tup_add;         // list mode: k ints per tuple
   uint64_t tup_add_cap;
   int32_t *tup_rem;

@@ -71,8 +71,8 @@ def test_c1_triangle_budgets(G, budget):
     assert got == want
     assert want[0][0] > 0
     assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
-    if budget == 0:
-        assert st["hit_bytes"] == 0 and st["miss_bytes"] > 0
+    if budget == 0:  # no cache; a triangle reads only the updated vertices' lists, uploaded with the batch
+        assert st["hit_bytes"] == 0 and st["cached_vertices"] == 0 and st["delta_bytes"] > 0
     if budget == 1.0:
         assert st["cached_vertices"] > 0
 
@@ -279,6 +279,68 @@ def test_estimator_and_cache_parity(G, name, labelled):
         assert np.array_equal(g.cached(), oracle.select_cache(e["est"], sz, budget & ~15))
         rp, col = oracle.apply_batch(w.n, rp, col, I, D)
     g.close()
+
+
+@pytest.mark.parametrize("name,M", [("k4", 10**9), ("house5u", 10**9), ("prism6", 10**9)])
+def test_estimator_btrd_range(G, name, M):
+    """Walk budgets large enough that children draw B' ~ Bin(B, 1/D) with B/D >= 10 (BTRD, R20) on the device:
+    per-vertex per-level sums and the cached set still equal the oracle's."""
+    w = gi.make_workload("C2", scale=11, n_edges=12_000, batch=96, n_batches=1)
+    k, qe, ql = gi.query(name)
+    seed = 0x5EED
+    budget = w.adj_bytes // 20
+    g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0, seed=seed, walks_override=M)
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(budget)
+    ins, dele = w.batches[0]
+    g.apply_batch(ins, dele)
+    e = oracle.estimate(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele, seed=seed, batch_seq=0, M=M)
+    assert e["M"] == M and g.stats()["walks"] == M
+    assert M // e["N1"] >= 10 * e["D"]  # level-1 children are in BTRD's range
+    ids, lev = g.estimates()
+    want_ids = np.nonzero(e["levcnt"].sum(1))[0]
+    assert np.array_equal(ids, want_ids)
+    assert np.array_equal(lev[:, :k - 2], e["levcnt"][want_ids])
+    I, D, _ = oracle.normalize_batch(w.n, w.row_ptr, w.col, ins, dele)
+    rps, _ = oracle.stable_graph(w.n, w.row_ptr, w.col, D)
+    sz = 16 * ((np.diff(rps) + 3) // 4)
+    assert np.array_equal(g.cached(), oracle.select_cache(e["est"], sz, budget & ~15))
+    g.close()
+
+
+def test_degree_policy_cached_set(G):
+    """Naive ablation (degree-ranked cache): the device ranking is R23 applied to the stable degrees."""
+    w = gi.make_workload("C2", scale=12, n_edges=30_000, batch=256, n_batches=2)
+    k, qe, ql = gi.query("k4")
+    budget = w.adj_bytes // 10
+    g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0, cache_policy="degree")
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(budget)
+    rp, col = w.row_ptr, w.col
+    for ins, dele in w.batches:
+        g.apply_batch(ins, dele)
+        I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+        rps, _ = oracle.stable_graph(w.n, rp, col, D)
+        deg = np.diff(rps).astype(np.float64)
+        sz = 16 * ((np.diff(rps) + 3) // 4)
+        assert np.array_equal(g.cached(), oracle.select_cache(deg, sz, budget & ~15))
+        rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+    g.close()
+
+
+def test_budget_change_between_batches(G):
+    """Growing the budget reallocates the cache buffers: descriptors of the old selection must not dangle."""
+    w = gi.make_workload("C2", scale=12, n_edges=30_000, batch=256, n_batches=4)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, "c4", w.batches)
+    k, qe, ql = gi.query("c4")
+    g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0)
+    g.set_query(k, qe, ql)
+    got = []
+    for i, (ins, dele) in enumerate(w.batches):
+        g.set_cache_budget([w.adj_bytes // 50, w.adj_bytes // 5, 0, w.adj_bytes][i])
+        got.append(g.apply_batch(ins, dele))
+    g.close()
+    assert got == want
 
 
 # ------------------------------------------------------------------ multi-GPU sharding, emulated world on one GPU
