@@ -205,6 +205,12 @@ struct WalkArgs {
   const DevPlan *plans;
   const EstUnit *units;
   int64_t n_units;
+  const int2 *items;
+  int64_t n_items;
+  EstNode2 *f2;
+  int64_t f2_cap;
+  unsigned long long *f2_count;
+  unsigned long long *cursor2;
   unsigned long long *levcnt;
   int32_t levels;
   const VDesc *vdesc;
@@ -229,6 +235,94 @@ struct EstW {
   EstLv lv[GCSM_MAXK - 1];  // index = tree level 1..k-2
 };
 
+// Level 1 (phase A): warp per work item (a unit and kEstItem of its driver elements). The item at index 0 records
+// the level-1 node's reads; children with B' > 0 are recorded directly when they are the last sampled level (k = 4)
+// or appended to the level-2 node list (k >= 5) for k_walks.
+__global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
+  __shared__ double sfc_s[10];
+  if (threadIdx.x < 10) sfc_s[threadIdx.x] = A.sfc[threadIdx.x];
+  __syncthreads();
+  BinTab T = A.T;
+  T.sfc = sfc_s;
+  const int lane = threadIdx.x & 31;
+  for (;;) {
+    unsigned long long it = 0;
+    if (lane == 0) it = atomicAdd(A.cursor, 1ull);
+    it = __shfl_sync(FULL, it, 0);
+    if (it >= (unsigned long long)A.n_items) return;
+    const int2 item = A.items[it];
+    const EstUnit U = A.units[item.x];
+    const DevPlan *P = A.plans + U.plan;
+    const int k = P->k;
+    const LevelPlan &Lp = P->lv[2];
+    const int nb = Lp.nb;
+    const int32_t f01[2] = {U.a, U.b};
+    if (item.y == 0 && lane < nb) {
+      const int32_t v = f01[Lp.bpos[lane]];
+      atomicAdd(A.levcnt + (size_t)v * A.levels, U.B);
+      atomicOr(A.touched + (v >> 5), 1u << (v & 31));
+    }
+    if (k <= 3) continue;  // level 1 is the last sampled level
+    LR L[7];
+    int drv = 0;
+    uint32_t best = 0xffffffffu;
+    for (int b = 0; b < nb; ++b) {
+      L[b] = view_of(A.vdesc, A.drec, A.dlist, f01[Lp.bpos[b]], Lp.bview[b]);
+      const uint32_t t = L[b].ml + L[b].xl;
+      if (t < best) {
+        best = t;
+        drv = b;
+      }
+    }
+    const uint32_t end = min(best, (uint32_t)item.y + (uint32_t)kEstItem);
+    const LevelPlan &L3 = P->lv[3];
+    for (uint32_t pos = (uint32_t)item.y; pos < end; pos += 32) {
+      const uint32_t idx = pos + lane;
+      bool ok = false;
+      int32_t v = 0;
+      unsigned long long Bc = 0, ck = 0;
+      if (idx < end) {
+        v = idx < L[drv].ml ? L[drv].m[idx] : L[drv].x[idx - L[drv].ml];
+        ok = v != U.a && v != U.b;
+        if (ok && Lp.label >= 0) ok = (A.lab ? (int32_t)A.lab[v] : 0) == Lp.label;
+        if (ok) {
+          ck = dchain(U.key, (unsigned long long)(uint32_t)v);
+          const int64_t bc = d_binomial(ck, (int64_t)U.B, T);
+          Bc = (unsigned long long)bc;
+          ok = bc > 0;
+        }
+        if (ok)
+          for (int b = 0; b < nb; ++b)
+            if (b != drv && !(has(L[b].m, L[b].ml, v) || (L[b].xl && has(L[b].x, L[b].xl, v)))) {
+              ok = false;
+              break;
+            }
+      }
+      if (k == 4) {  // the child is a level-2 node of the last sampled level: its reads, then nothing below
+        if (ok) {
+          const int32_t f3[3] = {U.a, U.b, v};
+          for (int b = 0; b < L3.nb; ++b) {
+            const int32_t w = f3[L3.bpos[b]];
+            atomicAdd(A.levcnt + (size_t)w * A.levels + 1, Bc);
+            atomicOr(A.touched + (w >> 5), 1u << (w & 31));
+          }
+        }
+      } else {
+        const unsigned mask = __ballot_sync(FULL, ok);
+        unsigned long long base = 0;
+        if (lane == 0 && mask) base = atomicAdd(A.f2_count, (unsigned long long)__popc(mask));
+        base = __shfl_sync(FULL, base, 0);
+        if (ok) {
+          const unsigned long long slot = base + __popc(mask & ((1u << lane) - 1u));
+          if (slot < (unsigned long long)A.f2_cap) A.f2[slot] = EstNode2{U.a, U.b, v, U.plan, Bc, ck};
+          else atomicExch(A.T.err, 3);
+        }
+      }
+    }
+  }
+}
+
+// Levels >= 2 (phase B, k >= 5): warp per level-2 node, DFS over the rest of its subtree.
 __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
   __shared__ EstW sw[kEW];
   __shared__ double sfc_s[10];
@@ -238,25 +332,27 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
   T.sfc = sfc_s;
   const int lane = threadIdx.x & 31;
   EstW &W = sw[threadIdx.x >> 5];
+  const unsigned long long n2 = min(*(volatile unsigned long long *)A.f2_count, (unsigned long long)A.f2_cap);
   for (;;) {
     unsigned long long u = 0;
-    if (lane == 0) u = atomicAdd(A.cursor, 1ull);
+    if (lane == 0) u = atomicAdd(A.cursor2, 1ull);
     u = __shfl_sync(FULL, u, 0);
-    if (u >= (unsigned long long)A.n_units) return;
-    const EstUnit U = A.units[u];
-    const DevPlan *P = A.plans + U.plan;
+    if (u >= n2) return;
+    const EstNode2 N = A.f2[u];
+    const DevPlan *P = A.plans + N.plan;
     const int k = P->k;
     __syncwarp();
     if (lane == 0) {
-      W.f[0] = U.a;
-      W.f[1] = U.b;
-      W.lv[1].B = U.B;
-      W.lv[1].key = U.key;
+      W.f[0] = N.f0;
+      W.f[1] = N.f1;
+      W.f[2] = N.f2;
+      W.lv[2].B = N.B;
+      W.lv[2].key = N.key;
     }
     __syncwarp();
-    int level = 1;
+    int level = 2;
     bool fresh = true;
-    while (level >= 1) {
+    while (level >= 2) {
       EstLv &S = W.lv[level];
       const LevelPlan &Lp = P->lv[level + 1];
       const int nb = Lp.nb;
@@ -670,7 +766,7 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
   if (c.policy == 2) {
     LK(k_deg_bits<<<gs_grid(W), 256, 0, s>>>(c.vdesc, c.n, c.touched));
   } else {
-    if ((e = cudaMemsetAsync(c.cursor, 0, sizeof(unsigned long long) * c.nq, s)) != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(c.cursor, 0, sizeof(unsigned long long) * 3 * c.nq, s)) != cudaSuccess) return e;
     for (int q = 0; q < c.nq; ++q) {
       const EstQuery &Q = c.q[q];
       if (Q.k <= 2 || Q.n_units <= 0) continue;
@@ -678,6 +774,12 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.plans = Q.plans;
       A.units = Q.units;
       A.n_units = Q.n_units;
+      A.items = Q.items;
+      A.n_items = Q.n_items;
+      A.f2 = c.f2;
+      A.f2_cap = Q.f2_cap;
+      A.f2_count = c.cursor + 3 * q + 2;
+      A.cursor2 = c.cursor + 3 * q + 1;
       A.levcnt = Q.levcnt;
       A.levels = Q.k - 2;
       A.vdesc = c.vdesc;
@@ -685,15 +787,16 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.dlist = c.dlist;
       A.lab = c.lab;
       A.touched = c.touched;
-      A.cursor = c.cursor + q;
+      A.cursor = c.cursor + 3 * q;
       A.T.pD = c.pD;
       A.T.r0tab = c.r0tab;
       A.T.r0n = c.r0n;
       A.T.sfc = nullptr;  // set to the block's shared copy of A.sfc
       A.T.err = &c.st->err;
       for (int i = 0; i < 10; ++i) A.sfc[i] = c.sfc[i];
-      const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((Q.n_units + kEW - 1) / kEW, 148 * 6));
-      LK(k_walks<<<grid, kEW * 32, 0, s>>>(A));
+      const int ga = (int)std::max<int64_t>(1, std::min<int64_t>((Q.n_items + kEW - 1) / kEW, 148 * 8));
+      LK(k_walks_l1<<<ga, kEW * 32, 0, s>>>(A));
+      if (Q.k >= 5) LK(k_walks<<<148 * 2, kEW * 32, 0, s>>>(A));
     }
   }
   // touched set in id order

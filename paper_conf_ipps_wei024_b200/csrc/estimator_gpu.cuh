@@ -21,10 +21,21 @@ struct alignas(16) EstUnit {
   unsigned long long B, key;
 };
 
+// Level-2 node of the walks (k >= 5): positions 0..2 matched, multiplicity B, key.
+struct alignas(16) EstNode2 {
+  int32_t f0, f1, f2, plan;
+  unsigned long long B, key;
+};
+
+constexpr int kEstItem = 1024;  // level-1 driver elements per work item (a hub's children spread over warps)
+
 struct EstQuery {
   const DevPlan *plans;     // unrestricted plans (the walks sample the paper's full trees, R27)
   const EstUnit *units;     // B > 0 only, heaviest first
   int64_t n_units;
+  const int2 *items;        // (unit, first driver index): max(1, ceil(driver / kEstItem)) per unit
+  int64_t n_items;
+  int64_t f2_cap;           // level-2 node capacity (k >= 5): sum of the units' driver lengths
   unsigned long long *levcnt;  // dense: n x levels (zero outside the touched set)
   int32_t k;
   uint64_t N1, M;
@@ -73,7 +84,8 @@ struct CacheStep {
   int32_t *prev_sel;        // last selection (ids ascending)
   unsigned long long *hist; // 6 x 4096
   SelState *st;
-  unsigned long long *cursor;  // per query work cursor (nq)
+  unsigned long long *cursor;  // 3 per query: item cursor, level-2 node cursor, level-2 node count
+  EstNode2 *f2;             // level-2 nodes (shared by the queries, one after the other)
   void *cub_tmp;
   size_t cub_tmp_bytes;
   // cache buffers

@@ -27,15 +27,28 @@ namespace {
 
 constexpr int64_t kF2CapLimit = 64ll << 20;  // level-2 frontier entries per chunk
 
+// Growth inside a submit must not wait for the previous batch's kernels: device buffers are re-allocated
+// stream-ordered on the context's stream (cudaFreeAsync / cudaMallocAsync), replaced pinned buffers are parked
+// until the context is destroyed (cudaFreeHost would synchronise the device). Set by submit_impl.
+thread_local cudaStream_t g_alloc_stream = nullptr;
+thread_local std::vector<void *> *g_retired_pinned = nullptr;
+
 template <typename T>
 bool dev_ensure(T *&p, size_t &cap, size_t need) {
   if (need <= cap && p) return true;
-  if (p) cudaFree(p);
+  if (p) {
+    if (g_alloc_stream) cudaFreeAsync(p, g_alloc_stream);
+    else cudaFree(p);
+  }
   p = nullptr;
   cap = 0;
   size_t n = std::max<size_t>(need, 1);
   n = 2 * n;
-  if (cudaMalloc((void **)&p, n * sizeof(T)) != cudaSuccess) return false;
+  if (g_alloc_stream) {
+    if (cudaMallocAsync((void **)&p, n * sizeof(T), g_alloc_stream) != cudaSuccess) return false;
+  } else if (cudaMalloc((void **)&p, n * sizeof(T)) != cudaSuccess) {
+    return false;
+  }
   cap = n;
   return true;
 }
@@ -43,7 +56,10 @@ bool dev_ensure(T *&p, size_t &cap, size_t need) {
 template <typename T>
 bool host_ensure(T *&p, size_t &cap, size_t need) {
   if (need <= cap && p) return true;
-  if (p) cudaFreeHost(p);
+  if (p) {
+    if (g_retired_pinned) g_retired_pinned->push_back(p);
+    else cudaFreeHost(p);
+  }
   p = nullptr;
   cap = 0;
   size_t n = std::max<size_t>(need, 1);
@@ -87,6 +103,7 @@ struct gcsm_ctx {
     uint64_t *h_fresh = nullptr; size_t h_fresh_cap = 0;
     unsigned long long *h_cnt = nullptr;  // CNT_N per query
     EstUnit *h_eunits = nullptr; size_t h_eunits_cap = 0;  // level-1 walk nodes (GPU estimator)
+    int2 *h_eitems = nullptr; size_t h_eitems_cap = 0;     // their work items
     int32_t *h_ulist = nullptr; size_t h_ulist_cap = 0;    // stable lists S(x) of U, packed (GPU path)
     int32_t *d_ulist = nullptr; size_t d_ulist_cap = 0;    // their device copy (read by this batch's kernels)
     size_t ulist_n = 0;
@@ -156,10 +173,13 @@ struct gcsm_ctx {
   unsigned long long *d_levcnt[GCSM_MAX_QUERIES] = {};
   int lev_levels[GCSM_MAX_QUERIES] = {-1, -1, -1, -1, -1, -1, -1, -1};
   EstUnit *d_eunits = nullptr; size_t eunits_cap = 0;
+  int2 *d_eitems = nullptr; size_t eitems_cap = 0;
+  EstNode2 *d_ef2 = nullptr; size_t ef2_cap = 0;
   double *d_r0 = nullptr; size_t r0_cap = 0;
   size_t r0_n = 0;                 // entries of the device table of (1 - pD)^n
   double r0_pD = -1.0;
   bool est_valid = false;          // the device holds a batch's estimator output (gcsm_get_estimates)
+  std::vector<void *> retired_pinned;  // pinned staging replaced by a larger one (freed at destroy)
 
 
   // cache / batch state
@@ -198,14 +218,15 @@ gcsm_ctx::~gcsm_ctx() {
   for (void *p : dev)
     if (p) cudaFree(p);
   void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
-                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0};
+                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2};
   for (void *p : dev2)
     if (p) cudaFree(p);
   for (unsigned long long *p : d_levcnt)
     if (p) cudaFree(p);
+  for (void *p : retired_pinned) cudaFreeHost(p);
   for (Slot &sl : slots) {
     void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt,
-                    sl.h_eunits, sl.h_ulist, sl.h_r0};
+                    sl.h_eunits, sl.h_ulist, sl.h_r0, sl.h_eitems};
     if (sl.d_ulist) cudaFree(sl.d_ulist);
     for (void *p : host)
       if (p) cudaFreeHost(p);
@@ -476,6 +497,7 @@ struct Trace {
 // addresses) and level-1 walk nodes, then enqueues the walks, the ranking cut and the cache copy on the stream.
 static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStream_t s, size_t ndirty, size_t nU,
                                      size_t nd, int64_t gnu, const std::vector<std::vector<EstUnit>> &qeu,
+                                     const std::vector<std::vector<int2>> &qitems, const std::vector<int64_t> &qf2cap,
                                      uint64_t maxB, uint64_t D, const std::vector<int64_t> &qnu,
                                      const std::vector<uint64_t> &qwalks, bool use_cache, uint64_t *launches) {
   HostStore &S = ctx->store;
@@ -493,7 +515,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
         cudaMalloc(&ctx->d_scan, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_off, 8 * (size_t)n) != cudaSuccess ||
         cudaMalloc(&ctx->d_flag, (size_t)n) != cudaSuccess ||
         cudaMalloc(&ctx->d_selhist, 8 * 6 * 4096) != cudaSuccess ||
-        cudaMalloc(&ctx->d_ecursor, 8 * GCSM_MAX_QUERIES) != cudaSuccess ||
+        cudaMalloc(&ctx->d_ecursor, 8 * 3 * GCSM_MAX_QUERIES) != cudaSuccess ||
         cudaMalloc(&ctx->d_sel, sizeof(SelState)) != cudaSuccess ||
         cudaMalloc(&ctx->d_cubtmp, ctx->cubtmp_bytes) != cudaSuccess)
       return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
@@ -535,15 +557,22 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
     }
   }
   // uploads
-  size_t neu = 0;
+  size_t neu = 0, nit = 0;
+  int64_t f2max = 0;
   for (const auto &eu : qeu) neu += eu.size();
-  if (!host_ensure(sl.h_eunits, sl.h_eunits_cap, neu) || !dev_ensure(ctx->d_eunits, ctx->eunits_cap, neu))
+  for (const auto &it : qitems) nit += it.size();
+  for (int64_t c2 : qf2cap) f2max = std::max(f2max, c2);
+  if (!host_ensure(sl.h_eunits, sl.h_eunits_cap, neu) || !dev_ensure(ctx->d_eunits, ctx->eunits_cap, neu) ||
+      !host_ensure(sl.h_eitems, sl.h_eitems_cap, nit) || !dev_ensure(ctx->d_eitems, ctx->eitems_cap, nit) ||
+      (f2max > 0 && !dev_ensure(ctx->d_ef2, ctx->ef2_cap, (size_t)f2max)))
     return ctx->fail(GCSM_ENOMEM, "walk roots");
   {
-    size_t o = 0;
-    for (const auto &eu : qeu) {
-      if (!eu.empty()) std::memcpy(sl.h_eunits + o, eu.data(), sizeof(EstUnit) * eu.size());
-      o += eu.size();
+    size_t o = 0, oi = 0;
+    for (int qi = 0; qi < nq; ++qi) {
+      if (!qeu[qi].empty()) std::memcpy(sl.h_eunits + o, qeu[qi].data(), sizeof(EstUnit) * qeu[qi].size());
+      if (!qitems[qi].empty()) std::memcpy(sl.h_eitems + oi, qitems[qi].data(), sizeof(int2) * qitems[qi].size());
+      o += qeu[qi].size();
+      oi += qitems[qi].size();
     }
   }
   CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
@@ -552,6 +581,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
   if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   if (neu) CK(cudaMemcpyAsync(ctx->d_eunits, sl.h_eunits, sizeof(EstUnit) * neu, cudaMemcpyHostToDevice, s));
+  if (nit) CK(cudaMemcpyAsync(ctx->d_eitems, sl.h_eitems, sizeof(int2) * nit, cudaMemcpyHostToDevice, s));
   if (ndirty) {
     CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * ndirty, cudaMemcpyHostToDevice, s));
     CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * ndirty, cudaMemcpyHostToDevice, s));
@@ -561,14 +591,18 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   CacheStep c{};
   c.n = n;
   c.nq = nq;
-  size_t o = 0;
+  size_t o = 0, oi = 0;
   for (int qi = 0; qi < nq; ++qi) {
     EstQuery &q = c.q[qi];
     const int k = ctx->qs[qi].qp.k;
     q.plans = ctx->qs[qi].d_plans;
     q.units = ctx->d_eunits + o;
     q.n_units = est_on ? (int64_t)qeu[qi].size() : 0;
+    q.items = ctx->d_eitems + oi;
+    q.n_items = est_on ? (int64_t)qitems[qi].size() : 0;
+    q.f2_cap = qf2cap[qi];
     o += qeu[qi].size();
+    oi += qitems[qi].size();
     q.levcnt = k > 2 ? ctx->d_levcnt[qi] : nullptr;
     q.k = k;
     q.N1 = (uint64_t)std::max<int64_t>(qnu[qi], 1);
@@ -601,6 +635,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.hist = ctx->d_selhist;
   c.st = ctx->d_sel;
   c.cursor = ctx->d_ecursor;
+  c.f2 = ctx->d_ef2;
   c.cub_tmp = ctx->d_cubtmp;
   c.cub_tmp_bytes = ctx->cubtmp_bytes;
   c.cache = ctx->d_cache;
@@ -627,6 +662,16 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   if (listing && ctx->qs.size() != 1) return ctx->fail(GCSM_EINVAL, "list mode needs exactly one query");
   Timer total;
   Trace tr;
+  struct AllocScope {  // stream-ordered growth for this submit only
+    AllocScope(cudaStream_t st, std::vector<void *> *r) {
+      g_alloc_stream = st;
+      g_retired_pinned = r;
+    }
+    ~AllocScope() {
+      g_alloc_stream = nullptr;
+      g_retired_pinned = nullptr;
+    }
+  } alloc_scope(ctx->stream, &ctx->retired_pinned);
   HostStore &S = ctx->store;
   const int nq = (int)ctx->qs.size();
   int kmax = 2;
@@ -737,6 +782,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // GPU path: the level-1 nodes of the walks (a unit, its key of R22 and its draw B_1 ~ Bin(M, 1/N1)) are
   // made here (N1 draws); everything below level 1 runs in k_walks (estimator_gpu.cu)
   std::vector<std::vector<EstUnit>> qeu(ctx->gpu_est ? (size_t)nq : 0);
+  std::vector<std::vector<int2>> qitems(ctx->gpu_est ? (size_t)nq : 0);
+  std::vector<int64_t> qf2cap((size_t)nq, 0);
   uint64_t eu_maxB = 0;
   if (ctx->gpu_est) {
     for (int qi = 0; qi < nq; ++qi) {
@@ -772,6 +819,20 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
               eu.push_back(x);
               eu_maxB = std::max<uint64_t>(eu_maxB, x.B);
             }
+          // work items: kEstItem driver elements of a unit's level-1 candidate scan each (hubs spread over warps);
+          // level-2 node capacity = the sum of the driver lengths (k >= 5)
+          std::vector<int2> &items = qitems[qi];
+          int64_t cap2 = 0;
+          for (size_t i = 0; i < eu.size(); ++i) {
+            const LevelPlan &L2 = Q.plans[eu[i].plan].lv[2];
+            const int32_t f[2] = {eu[i].a, eu[i].b};
+            int64_t dl = INT64_MAX;
+            for (int bb = 0; bb < L2.nb; ++bb) dl = std::min<int64_t>(dl, S.view_len(f[L2.bpos[bb]], L2.bview[bb]));
+            if (dl == INT64_MAX) dl = 0;
+            cap2 += dl;
+            for (int64_t st0 = 0; st0 == 0 || st0 < dl; st0 += kEstItem) items.push_back(int2{(int)i, (int)st0});
+          }
+          qf2cap[qi] = k >= 5 ? cap2 : 0;
         }
       }
       qms_est[qi] = tq.ms();
@@ -1080,8 +1141,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   CK(cudaEventRecord(sl.ev_c0, s));
   uint64_t launches = 0;
   if (ctx->gpu_est) {
-    gcsm_status gs = enqueue_gpu_cache(ctx, sl, s, dirty.size(), nU, nd, gnu, qeu, eu_maxB, D, qnu, qwalks, use_cache,
-                                       &launches);
+    gcsm_status gs = enqueue_gpu_cache(ctx, sl, s, dirty.size(), nU, nd, gnu, qeu, qitems, qf2cap, eu_maxB, D, qnu,
+                                       qwalks, use_cache, &launches);
     if (gs != GCSM_OK) return gs;
     st.h2d_bytes = (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU + 4 * nd +
                    sizeof(Unit) * (size_t)gnu;
