@@ -269,9 +269,9 @@ def main():
     for i, q in enumerate(queries):
         k, qe, ql = gi.query(q)
         if i == 0:
-            g.set_query(k, qe, ql)
+            g.set_query(k, qe, ql, gi.order(q))
         else:
-            g.add_query(k, qe, ql)
+            g.add_query(k, qe, ql, gi.order(q))
     g.set_cache_budget(budget)
     steps = args.warmup + args.steps
     assert len(w.batches) >= steps, "stream too short"

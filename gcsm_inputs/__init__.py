@@ -122,6 +122,22 @@ QUERIES = {
 }
 
 
+# Matching orders (user order; each term's order follows from it by reading R11). The paper leaves matching-order
+# optimisation to future work; these were picked by measurement with scripts/order_probe.py on the
+# config's graph shape (profiles/order_probe_r01.txt): for prism6 starting from a rung (0,3) and closing both
+# triangles last cuts the C4-shaped match 2.5x. Counts do not depend on the order (GPU invariance tests).
+ORDERS = {
+    "prism6": [0, 3, 4, 1, 2, 5],
+    "bowtie5": [0, 3, 4, 1, 2],
+}
+
+
+def order(name: str):
+    """The catalogue's matching order for a query (None = the identity order)."""
+    o = ORDERS.get(name)
+    return None if o is None else np.asarray(o, dtype=np.int32)
+
+
 def query(name: str):
     k, edges, lab = QUERIES[name]
     qe = np.asarray(edges, dtype=np.int32).reshape(-1, 2)

@@ -141,3 +141,13 @@ def test_generator_planted_cliques():
     assert not np.array_equal(plain[:28], first)
     w = gi.make_workload("C4", scale=12, n_edges=30000, batch=64, n_batches=1)
     assert w.meta["planted"][0] > 0 and int(w.row_ptr[-1]) > 0
+
+
+def test_catalogue_orders_are_valid(pkg):
+    """The catalogue's matching orders are permutations the plan builder accepts (connected per-term orders)."""
+    import gcsm_inputs as gi
+    for name in gi.ORDERS:
+        k, qe, _ = gi.query(name)
+        o = gi.order(name)
+        assert sorted(o.tolist()) == list(range(k))
+        pkg.plan_inspect(k, qe, o)
