@@ -220,7 +220,6 @@ struct WalkArgs {
   uint32_t *touched;
   unsigned long long *cursor;
   BinTab T;
-  double sfc[10];
 };
 
 constexpr int kEW = 8;  // warps per block
@@ -239,11 +238,7 @@ struct EstW {
 // the level-1 node's reads; children with B' > 0 are recorded directly when they are the last sampled level (k = 4)
 // or appended to the level-2 node list (k >= 5) for k_walks.
 __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
-  __shared__ double sfc_s[10];
-  if (threadIdx.x < 10) sfc_s[threadIdx.x] = A.sfc[threadIdx.x];
-  __syncthreads();
-  BinTab T = A.T;
-  T.sfc = sfc_s;
+  const BinTab T = A.T;
   const int lane = threadIdx.x & 31;
   for (;;) {
     unsigned long long it = 0;
@@ -325,11 +320,7 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
 // Levels >= 2 (phase B, k >= 5): warp per level-2 node, DFS over the rest of its subtree.
 __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
   __shared__ EstW sw[kEW];
-  __shared__ double sfc_s[10];
-  if (threadIdx.x < 10) sfc_s[threadIdx.x] = A.sfc[threadIdx.x];
-  __syncthreads();
-  BinTab T = A.T;
-  T.sfc = sfc_s;
+  const BinTab T = A.T;
   const int lane = threadIdx.x & 31;
   EstW &W = sw[threadIdx.x >> 5];
   const unsigned long long n2 = min(*(volatile unsigned long long *)A.f2_count, (unsigned long long)A.f2_cap);
@@ -791,9 +782,8 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.T.pD = c.pD;
       A.T.r0tab = c.r0tab;
       A.T.r0n = c.r0n;
-      A.T.sfc = nullptr;  // set to the block's shared copy of A.sfc
+      A.T.sfc = c.sfc_dev;
       A.T.err = &c.st->err;
-      for (int i = 0; i < 10; ++i) A.sfc[i] = c.sfc[i];
       const int ga = (int)std::max<int64_t>(1, std::min<int64_t>((Q.n_items + kEW - 1) / kEW, 148 * 8));
       LK(k_walks_l1<<<ga, kEW * 32, 0, s>>>(A));
       if (Q.k >= 5) LK(k_walks<<<148 * 2, kEW * 32, 0, s>>>(A));

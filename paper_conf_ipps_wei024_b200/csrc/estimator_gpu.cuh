@@ -70,7 +70,7 @@ struct CacheStep {
   double pD;                // 1 / D
   const double *r0tab;      // (1 - pD)^n for n < r0n (host std::pow)
   int64_t r0n;
-  double sfc[10];           // BTRD's Stirling correction for k < 10 (host lgamma)
+  const double *sfc_dev;    // BTRD's Stirling correction for k < 10 (host lgamma), 10 doubles in device memory
   // scratch (capacity n unless noted)
   uint32_t *touched;        // ceil(n/32) words
   uint32_t *wcnt;           // ceil(n/32) + 1

@@ -176,6 +176,7 @@ struct gcsm_ctx {
   int2 *d_eitems = nullptr; size_t eitems_cap = 0;
   EstNode2 *d_ef2 = nullptr; size_t ef2_cap = 0;
   double *d_r0 = nullptr; size_t r0_cap = 0;
+  double *d_sfc = nullptr;         // BTRD Stirling table (10 doubles)
   size_t r0_n = 0;                 // entries of the device table of (1 - pD)^n
   double r0_pD = -1.0;
   bool est_valid = false;          // the device holds a batch's estimator output (gcsm_get_estimates)
@@ -218,7 +219,7 @@ gcsm_ctx::~gcsm_ctx() {
   for (void *p : dev)
     if (p) cudaFree(p);
   void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
-                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2};
+                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2, d_sfc};
   for (void *p : dev2)
     if (p) cudaFree(p);
   for (unsigned long long *p : d_levcnt)
@@ -520,6 +521,10 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
         cudaMalloc(&ctx->d_cubtmp, ctx->cubtmp_bytes) != cudaSuccess)
       return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
     CK(cudaMemcpyAsync(ctx->d_hptr, hp.data(), 8 * (size_t)n, cudaMemcpyHostToDevice, s));
+    double sfc[10];
+    for (int i = 0; i < 10; ++i) sfc[i] = stirling_small(i);
+    if (cudaMalloc(&ctx->d_sfc, sizeof sfc) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
+    CK(cudaMemcpyAsync(ctx->d_sfc, sfc, sizeof sfc, cudaMemcpyHostToDevice, s));
     CK(cudaMemsetAsync(ctx->d_sel, 0, sizeof(SelState), s));
     CK(cudaStreamSynchronize(s));  // hp is pageable and local
     ctx->gpu_ready = true;
@@ -621,7 +626,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.pD = pD;
   c.r0tab = ctx->d_r0;
   c.r0n = (int64_t)ctx->r0_n;
-  for (int i = 0; i < 10; ++i) c.sfc[i] = stirling_small(i);
+  c.sfc_dev = ctx->d_sfc;
   c.touched = ctx->d_touched;
   c.wcnt = ctx->d_wcnt;
   c.woff = ctx->d_woff;

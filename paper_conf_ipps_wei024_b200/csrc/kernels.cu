@@ -65,8 +65,14 @@ constexpr unsigned kFull = 0xffffffffu;
 constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 constexpr int kChunk = 32;  // frontier entries per k_extend work grab
-constexpr uint32_t kSplitMin = 64;  // level-3 sets larger than this are shared as tasks (k >= 5)
-constexpr uint32_t kTaskSize = 16;  // level-3 candidates per task
+#ifndef GCSM_SPLIT_MIN
+#define GCSM_SPLIT_MIN 64
+#endif
+#ifndef GCSM_TASK_SIZE
+#define GCSM_TASK_SIZE 16
+#endif
+constexpr uint32_t kSplitMin = GCSM_SPLIT_MIN;  // level-3 sets larger than this are shared as tasks (k >= 5)
+constexpr uint32_t kTaskSize = GCSM_TASK_SIZE;  // level-3 candidates per task
 
 struct LRef {
   const int32_t *m;  // main list
