@@ -66,10 +66,10 @@ constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 constexpr int kChunk = 32;  // frontier entries per k_extend work grab
 #ifndef GCSM_SPLIT_MIN
-#define GCSM_SPLIT_MIN 64
+#define GCSM_SPLIT_MIN 8
 #endif
 #ifndef GCSM_TASK_SIZE
-#define GCSM_TASK_SIZE 16
+#define GCSM_TASK_SIZE 2
 #endif
 constexpr uint32_t kSplitMin = GCSM_SPLIT_MIN;  // level-3 sets larger than this are shared as tasks (k >= 5)
 constexpr uint32_t kTaskSize = GCSM_TASK_SIZE;  // level-3 candidates per task
