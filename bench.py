@@ -43,8 +43,8 @@ UNIT = "updated_edges/s"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=8)
-    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--steps", type=int, default=16)
+    ap.add_argument("--warmup", type=int, default=4)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2")
     ap.add_argument("--queries", default=None, help="comma list (default: the config's queries)")
@@ -78,7 +78,7 @@ class Clocks:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
@@ -87,7 +87,11 @@ class Clocks:
 
     def _read(self):
         for line in self.proc.stdout:
-            self.rows.append([x.strip() for x in line.split(",")])
+            self.rows.append((time.perf_counter(), [x.strip() for x in line.split(",")]))
+
+    def mark(self, t0, t1):
+        """the timed region: samples taken inside it (or the nearest one) are reported"""
+        self.t0, self.t1 = t0, t1
 
     def stop(self):
         if not self.proc:
@@ -98,6 +102,11 @@ class Clocks:
             self.proc.wait(timeout=2)
         except Exception:
             self.proc.kill()
+        t0, t1 = getattr(self, "t0", 0.0), getattr(self, "t1", float("inf"))
+        rows = [r for t, r in self.rows if t0 <= t <= t1 + 0.05]
+        if not rows and self.rows:  # region shorter than the sampling period: the sample closest to it
+            rows = [min(self.rows, key=lambda tr: abs(tr[0] - 0.5 * (t0 + t1)))[1]]
+        self.rows = rows
         sm = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
         mx = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
@@ -300,12 +309,14 @@ def main():
         recs.append(collect())
         return recs
 
-    for i in range(args.warmup):
-        do_step(i)
-
+    # the clocks sampler (nvidia-smi) starts before the warm-up: its start-up must not land in the timed region
     clocks = Clocks(local)
     if not args.quick and rank == 0:
         clocks.start()
+        time.sleep(1.0)
+    for i in range(args.warmup):
+        do_step(i)
+
     streams = [torch.cuda.ExternalStream(g.stream_ptr())]
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier(world)
@@ -319,6 +330,8 @@ def main():
     barrier(world)
     ms_dev = allmax(world, ev0.elapsed_time(ev1))
     ms_host = allmax(world, 1e3 * (th1 - th0))
+    if not args.quick and rank == 0:
+        clocks.mark(th0, th1)
     clk = clocks.stop() if (not args.quick and rank == 0) else None
 
     # per query aggregates over the timed steps
