@@ -162,6 +162,8 @@ __device__ __forceinline__ int64_t d_binomial(unsigned long long key, int64_t n,
   return d_btrd(U, n, p, T);
 }
 
+__device__ __noinline__ int64_t d_binomial_ool(unsigned long long key, int64_t n, BinTab T) { return d_binomial(key, n, T); }
+
 struct LR {
   const int32_t *m;
   uint32_t ml;
@@ -224,8 +226,11 @@ struct WalkArgs {
 
 constexpr int kEW = 8;  // warps per block
 struct EstLv {
-  int32_t pos, ns, si, pad;
+  int32_t pos, ns, si, drv;
   unsigned long long B, key;
+  unsigned long long T53;  // BINV's first-uniform threshold floor(r0 2^53) of this node (all ones: no shortcut)
+  const int32_t *dm, *dx;  // the node's driver list (main, delta segment), fixed at node entry
+  uint32_t dml, dxl;
   int32_t sv[32];
   unsigned long long sB[32], skey[32];
 };
@@ -359,10 +364,33 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
           __syncwarp();
           continue;
         }
+        // the node's driver (smallest backward list) and its BINV shortcut are fixed for all of its chunks
+        LR L[7];
+        int drv = 0;
+        uint32_t best = 0xffffffffu;
+        for (int b = 0; b < nb; ++b) {
+          L[b] = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
+          const uint32_t t = L[b].ml + L[b].xl;
+          if (t < best) {
+            best = t;
+            drv = b;
+          }
+        }
+        const int64_t Bn = (int64_t)S.B;
+        const double pD = T.pD;
+        unsigned long long t53 = ~0ull;
+        if (Bn > 0 && pD > 0.0 && pD <= 0.5 && DM((double)Bn, pD) < 10.0 && Bn < T.r0n)
+          t53 = (unsigned long long)floor(DM(T.r0tab[Bn], 9007199254740992.0));
         if (lane == 0) {
           S.pos = 0;
           S.ns = 0;
           S.si = 0;
+          S.drv = drv;
+          S.dm = L[drv].m;
+          S.dml = L[drv].ml;
+          S.dx = L[drv].x;
+          S.dxl = L[drv].xl;
+          S.T53 = t53;
         }
         __syncwarp();
         continue;
@@ -381,59 +409,85 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
         fresh = true;
         continue;
       }
-      // next 32 driver elements of this node's candidate set
-      const int p = level + 1;
-      LR L[7];
-      int drv = 0;
-      uint32_t best = 0xffffffffu;
-      for (int b = 0; b < nb; ++b) {
-        L[b] = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
-        const uint32_t t = L[b].ml + L[b].xl;
-        if (t < best) {
-          best = t;
-          drv = b;
-        }
-      }
+      // the next (up to) 4 chunks of 32 driver elements: 4 loads per lane in flight, the BINV first-uniform test
+      // (B' = 0 exactly when it fails, as in the host walker's pre-filter) inline, full draws out of line
+      const uint32_t dml = S.dml, best = dml + S.dxl;
       const uint32_t pos = (uint32_t)S.pos;
       if (pos >= best) {
         __syncwarp();
         --level;
         continue;
       }
-      const uint32_t idx = pos + lane;
-      bool ok = false;
-      int32_t v = 0;
-      unsigned long long Bc = 0, ck = 0;
-      if (idx < best) {
-        v = idx < L[drv].ml ? L[drv].m[idx] : L[drv].x[idx - L[drv].ml];
-        ok = true;
-        for (int s = 0; s < p; ++s) ok &= W.f[s] != v;
-        if (ok && Lp.label >= 0) ok = (A.lab ? (int32_t)A.lab[v] : 0) == Lp.label;
-        if (ok) {
-          ck = dchain(S.key, (unsigned long long)(uint32_t)v);
-          const int64_t bc = d_binomial(ck, (int64_t)S.B, T);
-          Bc = (unsigned long long)bc;
-          ok = bc > 0;
+      const int p = level + 1;
+      const int32_t *dm = S.dm, *dx = S.dx;
+      const unsigned long long key = S.key, t53 = S.T53;
+      const int64_t Bn = (int64_t)S.B;
+      int32_t v[4];
+      bool ok[4];
+      unsigned long long Bc[4], ck[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t idx = pos + 32 * j + lane;
+        ok[j] = idx < best;
+        v[j] = ok[j] ? (idx < dml ? dm[idx] : dx[idx - dml]) : 0;
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        for (int s2 = 0; s2 < p; ++s2) ok[j] = ok[j] && W.f[s2] != v[j];
+        if (ok[j] && Lp.label >= 0) ok[j] = (A.lab ? (int32_t)A.lab[v[j]] : 0) == Lp.label;
+        Bc[j] = 0;
+        ck[j] = 0;
+        if (ok[j]) {
+          ck[j] = dchain(key, (unsigned long long)(uint32_t)v[j]);
+          // in BINV's range a first uniform <= r0 means B' = 0 (binv's loop never runs)
+          ok[j] = t53 == ~0ull || (dmix(ck[j] + 0xD1B54A32D192ED03ULL) >> 11) > t53;
         }
-        if (ok)
-          for (int b = 0; b < nb; ++b)
-            if (b != drv && !(has(L[b].m, L[b].ml, v) || (L[b].xl && has(L[b].x, L[b].xl, v)))) {
-              ok = false;
-              break;
-            }
       }
-      const unsigned mask = __ballot_sync(FULL, ok);
+#pragma unroll 1
+      for (int j = 0; j < 4; ++j)
+        if (ok[j]) {
+          const int64_t bc = d_binomial_ool(ck[j], Bn, T);
+          Bc[j] = (unsigned long long)bc;
+          ok[j] = bc > 0;
+        }
+      if (__any_sync(FULL, ok[0] || ok[1] || ok[2] || ok[3])) {  // membership in the other backward lists
+        const int drv = S.drv;
+        for (int b = 0; b < nb; ++b) {
+          if (b == drv) continue;
+          const LR Lb = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
+#pragma unroll 1
+          for (int j = 0; j < 4; ++j)
+            if (ok[j]) ok[j] = has(Lb.m, Lb.ml, v[j]) || (Lb.xl && has(Lb.x, Lb.xl, v[j]));
+        }
+      }
+      // whole chunks while their survivors fit the 32-entry buffer (chunk 0 always does); the rest is redone
+      unsigned msk[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) msk[j] = __ballot_sync(FULL, ok[j]);
+      int taken = 0, tot = 0;
+      int basej[4] = {0, 0, 0, 0};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = __popc(msk[j]);
+        if (taken == j && (j == 0 || tot + c <= 32)) {
+          basej[j] = tot;
+          tot += c;
+          taken = j + 1;
+        }
+      }
       __syncwarp();
-      if (ok) {
-        const int r = __popc(mask & ((1u << lane) - 1u));
-        S.sv[r] = v;
-        S.sB[r] = Bc;
-        S.skey[r] = ck;
-      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (j < taken && ok[j]) {
+          const int r = basej[j] + __popc(msk[j] & ((1u << lane) - 1u));
+          S.sv[r] = v[j];
+          S.sB[r] = Bc[j];
+          S.skey[r] = ck[j];
+        }
       if (lane == 0) {
-        S.ns = __popc(mask);
+        S.ns = tot;
         S.si = 0;
-        S.pos = (int32_t)(pos + 32);
+        S.pos = (int32_t)(pos + 32 * taken);
       }
       __syncwarp();
     }
