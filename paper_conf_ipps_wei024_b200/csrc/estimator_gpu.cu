@@ -570,6 +570,7 @@ __global__ void k_score(const ScoreArgs S, const int32_t *tids, const SelState *
         s = DA(s, e);
       }
     }
+    if (vdesc[v].upd != 0) s = 0.0;  // x ∈ U: S(x) is already in HBM with the batch (R32), it takes no budget
     bits[i] = (unsigned long long)__double_as_longlong(s);
     bytes[i] = (unsigned long long)((len + 3u) & ~3u) * 4ull;
   }

@@ -931,6 +931,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const int tgt = ctx->cache_valid ? 1 - ctx->cache_cur : ctx->cache_cur;
   ctx->d_cache = ctx->d_cachebuf[tgt];
   if (use_cache && !ranked.empty() && !ctx->gpu_est) {
+    // x ∈ U: its list is device-resident with the batch only on the GPU path; the host path keeps the paper's
+    // ranking over every vertex (R32)
     // Only the head of the ranking can fit the budget: bucket the (positive) scores by the top 12 bits of their
     // IEEE pattern (monotone in the score), then the next 12 inside the bucket where the cumulative list bytes
     // pass the budget, and sort just the vertices at or above that cut (per-thread histograms, parallel

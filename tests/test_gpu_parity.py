@@ -73,8 +73,8 @@ def test_c1_triangle_budgets(G, budget):
     assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
     if budget == 0:  # no cache; a triangle reads only the updated vertices' lists, uploaded with the batch
         assert st["hit_bytes"] == 0 and st["cached_vertices"] == 0 and st["delta_bytes"] > 0
-    if budget == 1.0:
-        assert st["cached_vertices"] > 0
+    if budget == 1.0:  # every list a triangle reads belongs to U: device-resident with the batch (R32), no misses
+        assert st["miss_bytes"] == 0
 
 
 # ------------------------------------------------------------------ fuzz
@@ -252,6 +252,15 @@ def test_star_closed_form_at_scale(G, r):
 
 # ------------------------------------------------------------------ estimator ② and packer ③ parity
 
+def without_updated(score, I, D):
+    """DESIGN.md R32: the stable lists of the batch's updated vertices are uploaded with the batch (device-resident
+    for all of its kernels), so the ranking of R23 runs over the other vertices."""
+    s = np.array(score, dtype=np.float64, copy=True)
+    U = np.unique(np.concatenate([np.asarray(I).ravel(), np.asarray(D).ravel()]))
+    s[U] = 0.0
+    return s
+
+
 @pytest.mark.parametrize("name,labelled", [("diamond", False), ("k4", False), ("house5u", False), ("house5", True)])
 def test_estimator_and_cache_parity(G, name, labelled):
     w = gi.make_workload("C3" if labelled else "C2", scale=12, n_edges=30_000, batch=256, n_batches=2)
@@ -276,7 +285,7 @@ def test_estimator_and_cache_parity(G, name, labelled):
         I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
         rps, _ = oracle.stable_graph(w.n, rp, col, D)
         sz = 16 * ((np.diff(rps) + 3) // 4)
-        assert np.array_equal(g.cached(), oracle.select_cache(e["est"], sz, budget & ~15))
+        assert np.array_equal(g.cached(), oracle.select_cache(without_updated(e["est"], I, D), sz, budget & ~15))
         rp, col = oracle.apply_batch(w.n, rp, col, I, D)
     g.close()
 
@@ -304,7 +313,7 @@ def test_estimator_btrd_range(G, name, M):
     I, D, _ = oracle.normalize_batch(w.n, w.row_ptr, w.col, ins, dele)
     rps, _ = oracle.stable_graph(w.n, w.row_ptr, w.col, D)
     sz = 16 * ((np.diff(rps) + 3) // 4)
-    assert np.array_equal(g.cached(), oracle.select_cache(e["est"], sz, budget & ~15))
+    assert np.array_equal(g.cached(), oracle.select_cache(without_updated(e["est"], I, D), sz, budget & ~15))
     g.close()
 
 
@@ -323,7 +332,7 @@ def test_degree_policy_cached_set(G):
         rps, _ = oracle.stable_graph(w.n, rp, col, D)
         deg = np.diff(rps).astype(np.float64)
         sz = 16 * ((np.diff(rps) + 3) // 4)
-        assert np.array_equal(g.cached(), oracle.select_cache(deg, sz, budget & ~15))
+        assert np.array_equal(g.cached(), oracle.select_cache(without_updated(deg, I, D), sz, budget & ~15))
         rp, col = oracle.apply_batch(w.n, rp, col, I, D)
     g.close()
 
