@@ -1431,8 +1431,9 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.d2h_bytes = sizeof(unsigned long long) * CNT_N * (size_t)nq;
     st.frontier = h[CNT_F2];
     if (std::getenv("GCSM_TRACE"))
-      std::fprintf(stderr, "[gcsm kern] q=%d frontier=%llu runs=%llu pins=%llu pin_gb=%.3f copied_gb=%.3f\n", qi,
-                   h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_COPIED] / 1e9);
+      std::fprintf(stderr, "[gcsm kern] q=%d frontier=%llu runs=%llu pins=%llu pin_gb=%.3f split_gb=%.3f copied_gb=%.3f\n",
+                   qi, h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_DBG_SPLIT] / 1e9,
+                   h[CNT_COPIED] / 1e9);
     if (qi == 0 && (sl.tup_add || sl.tup_rem)) {
       const int k = ctx->qs[0].qp.k;
       const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);

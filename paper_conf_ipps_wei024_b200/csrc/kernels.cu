@@ -65,6 +65,9 @@ constexpr unsigned kFull = 0xffffffffu;
 constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 constexpr int kChunk = 32;  // frontier entries per k_extend work grab
+#ifndef GCSM_L4_GRAB
+#define GCSM_L4_GRAB 64  // k_last4: frontier entries per work grab (processed in rounds of 32)
+#endif
 #ifndef GCSM_SPLIT_MIN
 #define GCSM_SPLIT_MIN 8
 #endif
@@ -1055,15 +1058,26 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
   const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
   const int32_t *f2u = f2c + A.f2_cap;
   const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const int64_t chunk = max((int64_t)1, min((int64_t)32, n_f2 / (4 * warps)));
+  // work grab: up to GCSM_L4_GRAB entries (rounds of 32), fewer when the frontier would leave warps idle. A run of
+  // entries sharing x2 is cut only at grab boundaries, where its zero-copy list is fetched again.
+  const int64_t chunk = max((int64_t)1, min((int64_t)GCSM_L4_GRAB, n_f2 / (8 * warps)));
   Acc acc;
-  unsigned long long d_runs = 0, d_pinb = 0, d_pins = 0;
+  unsigned long long d_runs = 0, d_pinb = 0, d_pins = 0, d_split = 0;
   for (;;) {
-    unsigned long long c0 = 0;
-    if (lane == 0) c0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)chunk);
-    c0 = __shfl_sync(kFull, c0, 0);
-    if ((int64_t)c0 >= n_f2) break;
-    const int n = (int)min((int64_t)chunk, n_f2 - (int64_t)c0);
+    unsigned long long g0 = 0;
+    if (lane == 0) g0 = atomicAdd(&A.cnt[CNT_CURSOR1], (unsigned long long)chunk);
+    g0 = __shfl_sync(kFull, g0, 0);
+    if ((int64_t)g0 >= n_f2) break;
+    const int64_t gend = min((int64_t)g0 + chunk, n_f2);
+    int32_t pin_v = -1;  // x2 of the current run and its list slice (pinned copy, or in place): kept across rounds
+    const int32_t *pin_p = nullptr;
+    uint32_t pin_len = 0;
+    int4 xraw = make_int4(0, 0, 0, 0);
+    int4 xrec = make_int4(0, 0, 0, 0);  // x2's delta record (if updated)
+    uint32_t pin_sm = 0;
+    bool pin_dev = false, pin_hit = false;
+    for (int64_t c0 = (int64_t)g0; c0 < gend; c0 += 32) {
+    const int n = (int)min((int64_t)32, gend - c0);
     // ---- one lane per entry: prefetch the entry's metadata in parallel
     __syncwarp();
     if (lane < n) {
@@ -1085,23 +1099,21 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
       meta[4 * lane + 3] = make_int4(seg.x, seg.y, xl0, xl1);
     }
     __syncwarp();
-    int32_t pin_v = -1;  // x2 of the current run and its list slice (pinned copy, or in place)
-    const int32_t *pin_p = nullptr;
-    uint32_t pin_len = 0;
-    int4 xraw = make_int4(0, 0, 0, 0);
-    int4 xrec = make_int4(0, 0, 0, 0);  // x2's delta record (if updated)
-    uint32_t pin_sm = 0;
-    bool pin_dev = false, pin_hit = false;
     for (int i = 0; i < n; ++i) {
       const int4 m0 = meta[4 * i];
       const int32_t x2 = m0.x, a = m0.z, b = m0.w;
-      if (x2 != pin_v) {  // new run: entries i..i+run-1 share x2
-        const bool same = i + 1 + lane < n && meta[4 * (i + 1 + lane)].x == x2;
+      if (x2 != pin_v) {  // new run: entries i..i+run-1 share x2 (it may continue into the grab's next rounds)
+        const int64_t jn = c0 + i + 1 + lane;
+        const bool same = jn < gend && f2c[A.group ? A.group[jn] : jn] == x2;
         const unsigned rm = __ballot_sync(kFull, same);
         const int run = 1 + (rm == kFull ? 32 : __ffs(~rm) - 1);
         // union of the symmetry ranges of the run's entries that read x2's list: only that slice is fetched
+        // (entries of later rounds are not prefetched yet: then the whole list)
         int32_t rlo = INT_MAX, rhi = INT_MIN;
-        if (lane < run) {
+        if (i + run > n) {
+          rlo = INT_MIN;
+          rhi = INT_MAX;
+        } else if (lane < run) {
           const int4 mr = meta[4 * (i + lane)];
           int32_t lo, hi;
           if (l4_range((unsigned)lp[mr.y].x, mr.z, mr.w, x2, &lo, &hi)) {
@@ -1135,6 +1147,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
         if (run >= 2 && pin_len >= 32 && !pin_hit) {
           ++d_pins;
           d_pinb += 4ull * cn;
+          // GCSM_TRACE: a run continuing the previous grab's run (same x2 across the grab boundary) fetches again
+          if (i == 0 && c0 == (int64_t)g0 && c0 > 0 && f2c[A.group ? A.group[c0 - 1] : c0 - 1] == x2) d_split += 4ull * cn;
         }
         if (run >= 2 && pin_len >= 32 && cn4 <= GCSM_PIN_SMEM_MAX) {
           copy_list(sm, mp + (lb - mis), cn, lane);
@@ -1285,12 +1299,14 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
       if (kind) acc.rem += c;
       else acc.add += c;
     }
+    }
   }
   flush(A, acc, lane);
   if (lane == 0) {
     atomicAdd(&A.cnt[CNT_DBG_RUNS], d_runs);
     atomicAdd(&A.cnt[CNT_DBG_PINBYTES], d_pinb);
     atomicAdd(&A.cnt[CNT_DBG_PINS], d_pins);
+    atomicAdd(&A.cnt[CNT_DBG_SPLIT], d_split);
   }
 }
 

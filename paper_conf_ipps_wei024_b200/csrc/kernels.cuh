@@ -16,6 +16,7 @@ enum Counter {
   CNT_TUP_REM = 7,
   CNT_CURSOR0 = 8,  // work cursors (reset per launch)
   CNT_CURSOR1 = 9,
+  CNT_DBG_SPLIT = 2,     // k_last4: bytes pinned again for runs split across work grabs (GCSM_TRACE)
   CNT_COPIED = 3,   // bytes bulk-copied from host memory by the kernels' staging (real zero-copy reads)
   // per kernel, 3 consecutive slots: list bytes (algorithmic: 4 B x list length per use) served from
   // the HBM cache, zero-copy from pinned host memory, and from the device delta segments (ins/del of U)
