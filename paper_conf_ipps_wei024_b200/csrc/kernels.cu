@@ -64,7 +64,10 @@ constexpr unsigned kFull = 0xffffffffu;
 #endif
 constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
-constexpr int kChunk = 32;  // frontier entries per k_extend work grab
+#ifndef GCSM_EXT_CHUNK
+#define GCSM_EXT_CHUNK 32
+#endif
+constexpr int kChunk = GCSM_EXT_CHUNK;  // frontier entries per k_extend work grab
 #ifndef GCSM_L4_GRAB
 #define GCSM_L4_GRAB 64  // k_last4: frontier entries per work grab (processed in rounds of 32)
 #endif
