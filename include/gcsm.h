@@ -103,7 +103,8 @@ typedef struct {
   uint64_t cache_bytes;     /* bytes of cached lists (<= budget) */
   uint64_t hit_bytes;       /* list bytes the kernels read from the HBM cache (algorithmic, §8d) */
   uint64_t miss_bytes;      /* list bytes the kernels read zero-copy from host memory */
-  uint64_t delta_bytes;     /* list bytes read from the device-resident ins/del segments of updated vertices */
+  uint64_t delta_bytes;     /* list bytes read from device-resident batch data: the ins/del segments of updated
+                               vertices and (GPU estimator path) their stable lists S(x), uploaded with the batch */
   uint64_t hit_bytes_ext, miss_bytes_ext, delta_bytes_ext; /* the same, k_extend only (levels >= 3) */
   uint64_t host_copied_bytes; /* bytes the kernels bulk-copied from host memory (staging; real zero-copy reads) */
   uint64_t frontier;        /* level-2 partial matches materialised */
@@ -112,9 +113,11 @@ typedef struct {
   uint64_t d2h_bytes;       /* bytes copied device -> host (counters, tuples) */
   uint64_t added, removed;  /* last batch's global counts */
   double ms_normalize;      /* (1) normalise + overlay + units */
-  double ms_estimate;       /* (2) */
-  double ms_pack;           /* (3) host packing */
-  double ms_copy;           /* (3) H2D: cache DMA + descriptors + deltas */
+  double ms_estimate;       /* (2) host part: level-1 walk roots on the GPU path (default), all walks with
+                               GCSM_HOST_EST=1 */
+  double ms_pack;           /* (3) host part: descriptors / staging (GPU path), ranking + layout (host path) */
+  double ms_copy;           /* (3) GPU path: uploads + walks + ranking + cache copy on the stream (CUDA events);
+                               host path: H2D of the cache, descriptors and deltas */
   double ms_match;          /* (4) kernels (CUDA events) */
   double ms_level2;         /* (4) k_level2 launches only (CUDA events) */
   double ms_extend;         /* (4) k_extend launches only (CUDA events) */
@@ -223,13 +226,16 @@ gcsm_status gcsm_get_stream(const gcsm_ctx *ctx, void **stream);
  * if col_cap >= row_ptr[n], else ETRUNC. */
 gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col, uint64_t col_cap);
 
-/* Last batch's estimator output (step 2): the vertices with a non-zero count,
+/* Last batch's estimator output (step 2) for query 0: the vertices with a non-zero count,
  * ascending, and per vertex the per-level sums of walk multiplicities B for
  * tree levels 1..k-2 (eq. (3)): levcnt[i*8 + (l-1)]. *n_out = the number of
- * such vertices (ETRUNC if > cap; the first cap are written). */
+ * such vertices (ETRUNC if > cap; the first cap are written). On the GPU path the
+ * sums live in device memory: the call synchronises the context's stream. */
 gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levcnt, uint64_t cap, uint64_t *n_out);
 
-/* Last batch's cached vertex set (step 3), ascending. */
+/* Last batch's cached vertex set (step 3), ascending: the longest prefix of (estimate desc, id asc)
+ * that fits the budget (R23), over the vertices not updated by the batch on the GPU path (their
+ * stable lists are uploaded with the batch, R32). Synchronises the context's stream. */
 gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out);
 
 /* Roofline denominators the hot path needs and MEASURED_PEAKS.json lacks
