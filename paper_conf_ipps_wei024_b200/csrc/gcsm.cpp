@@ -109,6 +109,7 @@ struct gcsm_ctx {
     size_t ulist_n = 0;
     double *h_r0 = nullptr; size_t h_r0_cap = 0;           // BINV table staging
     cudaEvent_t ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr, ev_c1 = nullptr, ev_done = nullptr;
+    cudaEvent_t ev_up = nullptr, ev_l2 = nullptr;  // uploads done (fork) / hoisted level-2 work done (join)
     struct PerQuery {
       cudaEvent_t ev_m0 = nullptr, ev_m1 = nullptr;
       std::vector<cudaEvent_t> kev;  // per frontier chunk: level2 start, extend start, extend end
@@ -136,8 +137,9 @@ struct gcsm_ctx {
   int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
   Unit *d_units = nullptr; size_t units_cap = 0;
   int2 *d_useg = nullptr; size_t useg_cap = 0;
-  int32_t *d_f2 = nullptr; size_t f2_cap = 0;  // 2 * f2 entries ints
-  int32_t *d_group = nullptr; size_t group_cap = 0;  // frontier entries grouped by candidate
+  int32_t *d_f2q[GCSM_MAX_QUERIES] = {};  size_t f2q_cap[GCSM_MAX_QUERIES] = {};  // per query: 2 * f2 entries ints
+  int32_t *d_groupq[GCSM_MAX_QUERIES] = {};  size_t groupq_cap[GCSM_MAX_QUERIES] = {};  // frontier grouped by x2
+  cudaStream_t stream2 = nullptr;  // GPU path: the first level-2 kernels run here, beside the cache step
   uint32_t *d_hist = nullptr;                         // n counters + scan
   uint32_t *d_bsum = nullptr;
   int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
@@ -214,8 +216,12 @@ gcsm_ctx::~gcsm_ctx() {
   for (Query &q : qs)
     for (DevPlan *p : {q.d_plans, q.d_splans})
       if (p) cudaFree(p);
-  void *dev[] = {d_vdesc, d_lab, d_drec, d_dlist, d_units, d_useg, d_f2, d_scratch, d_cnt, d_cachebuf[0],
-                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_group, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
+  void *dev[] = {d_vdesc, d_lab, d_drec, d_dlist, d_units, d_useg, d_scratch, d_cnt, d_cachebuf[0],
+                 d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
+  for (int q = 0; q < GCSM_MAX_QUERIES; ++q) {
+    if (d_f2q[q]) cudaFree(d_f2q[q]);
+    if (d_groupq[q]) cudaFree(d_groupq[q]);
+  }
   for (void *p : dev)
     if (p) cudaFree(p);
   void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
@@ -231,7 +237,7 @@ gcsm_ctx::~gcsm_ctx() {
     if (sl.d_ulist) cudaFree(sl.d_ulist);
     for (void *p : host)
       if (p) cudaFreeHost(p);
-    for (cudaEvent_t e : {sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done})
+    for (cudaEvent_t e : {sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done, sl.ev_up, sl.ev_l2})
       if (e) cudaEventDestroy(e);
     for (auto &pq : sl.q) {
       for (cudaEvent_t e : {pq.ev_m0, pq.ev_m1})
@@ -239,7 +245,9 @@ gcsm_ctx::~gcsm_ctx() {
       for (cudaEvent_t e : pq.kev) cudaEventDestroy(e);
     }
   }
+  if (stream2) cudaStreamSynchronize(stream2);
   if (stream) cudaStreamDestroy(stream);
+  if (stream2) cudaStreamDestroy(stream2);
 }
 
 extern "C" {
@@ -301,9 +309,12 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
     return s;
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
+  if (cudaStreamCreateWithFlags(&ctx->stream2, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
   for (auto &sl : ctx->slots) {
     for (cudaEvent_t *ev : {&sl.ev_a0, &sl.ev_a1, &sl.ev_c0, &sl.ev_c1, &sl.ev_done})
       if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
+    for (cudaEvent_t *ev : {&sl.ev_up, &sl.ev_l2})
+      if (cudaEventCreateWithFlags(ev, cudaEventDisableTiming) != cudaSuccess) return bail(GCSM_EDEVICE);
     if (cudaHostAlloc(&sl.h_cnt, sizeof(unsigned long long) * CNT_N * GCSM_MAX_QUERIES, cudaHostAllocDefault) !=
         cudaSuccess)
       return bail(GCSM_ENOMEM);
@@ -593,6 +604,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
     CK(launch_patch_vdesc_host(ctx->d_vdesc, ctx->d_hptr, ctx->d_pidx, ctx->d_pval, (int64_t)ndirty, s));
     ++*launches;
   }
+  CK(cudaEventRecord(sl.ev_up, s));  // the batch's data is on the device: the level-2 kernels may start (stream2)
   CacheStep c{};
   c.n = n;
   c.nq = nq;
@@ -1195,8 +1207,9 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     return ctx->fail(GCSM_ENOMEM, "scratch");
   // level-2 frontier chunks: per unit an upper bound on its candidates (unit indices local to the query)
   std::vector<std::vector<std::pair<int64_t, int64_t>>> qchunks((size_t)nq);
-  int64_t f2_need = 0;
+  std::vector<int64_t> qf2need((size_t)nq, 0);
   for (int qi = 0; qi < nq; ++qi) {
+    int64_t &f2_need = qf2need[qi];
     const bool sym = !listing && ctx->qs[qi].qps.symmetry;
     const QueryPlan &QK = sym ? ctx->qs[qi].qps : ctx->qs[qi].qp;
     const std::vector<Unit> &units = qunits[qi];
@@ -1224,9 +1237,11 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       chunks.push_back({0, qn});
     }
   }
-  if (kmax >= 4 && (!dev_ensure(ctx->d_f2, ctx->f2_cap, (size_t)std::max<int64_t>(2 * f2_need, 2)) ||
-                    !dev_ensure(ctx->d_group, ctx->group_cap, (size_t)std::max<int64_t>(f2_need, 1))))
-    return ctx->fail(GCSM_ENOMEM, "frontier");
+  for (int qi = 0; qi < nq; ++qi)
+    if (ctx->qs[qi].qp.k >= 4 &&
+        (!dev_ensure(ctx->d_f2q[qi], ctx->f2q_cap[qi], (size_t)std::max<int64_t>(2 * qf2need[qi], 2)) ||
+         !dev_ensure(ctx->d_groupq[qi], ctx->groupq_cap[qi], (size_t)std::max<int64_t>(qf2need[qi], 1))))
+      return ctx->fail(GCSM_ENOMEM, "frontier");
   // list mode buffers (one query)
   int32_t *d_tadd = nullptr, *d_trem = nullptr;
   if (listing) {
@@ -1241,9 +1256,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.lab = ctx->d_lab;
   A.drec = ctx->d_drec;
   A.dlist = ctx->d_dlist;
-  A.useg = ctx->d_useg;
-  A.f2 = reinterpret_cast<int2 *>(ctx->d_f2);
-  A.f2_cap = f2_need;
+
   A.scratch = ctx->d_scratch;
   A.scratch_end = ctx->d_scratch + stride * (size_t)ctx->warps_total;
   A.scratch_stride = (int64_t)stride;
@@ -1270,47 +1283,83 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     CK(cudaEventCreate(&sl.q.back().ev_m0));
     CK(cudaEventCreate(&sl.q.back().ev_m1));
   }
-  for (int qi = 0; qi < nq; ++qi) {
-    auto &pq = sl.q[qi];
+  // per query and chunk: the kernel arguments (frontier buffers are per query, the unit segments per chunk)
+  auto setup = [&](int qi, const std::pair<int64_t, int64_t> &ch) {
     const bool sym = !listing && ctx->qs[qi].qps.symmetry;
     const QueryPlan &QK = sym ? ctx->qs[qi].qps : ctx->qs[qi].qp;
-    const int k = QK.k;
-    unsigned long long *qcnt = ctx->d_cnt + (size_t)qi * CNT_N;
     A.plans = sym ? ctx->qs[qi].d_splans : ctx->qs[qi].d_plans;
     A.n_plans = (int32_t)QK.plans.size();
-    A.k = k;
-    A.cnt = qcnt;
+    A.k = QK.k;
+    A.cnt = ctx->d_cnt + (size_t)qi * CNT_N;
+    A.f2 = reinterpret_cast<int2 *>(ctx->d_f2q[qi]);
+    A.f2_cap = qf2need[qi];
+    A.units = ctx->d_units + uoff[qi] + ch.first;
+    A.n_units = ch.second - ch.first;
+    A.useg = ctx->d_useg + uoff[qi] + ch.first;
     A.group = nullptr;
     A.tasks = nullptr;
-    if (k >= 5 && !listing) {
+    if (QK.k >= 5 && !listing) {
       A.arena = ctx->d_arena;
       A.arena_cap = ctx->arena_cap;
       A.tasks = ctx->d_tasks;
       A.task_ready = ctx->d_task_ready;
       A.task_cap = (uint32_t)std::min<size_t>(ctx->tasks_cap, ctx->task_ready_cap);
     }
+  };
+  // level 2 + grouping of a chunk (events e0 / e1 around the level-2 kernel) on stream `st`
+  auto level2 = [&](int qi, size_t ev0, cudaStream_t st) -> gcsm_status {
+    auto &pq = sl.q[qi];
+    unsigned long long *qcnt = ctx->d_cnt + (size_t)qi * CNT_N;
+    CK(cudaMemsetAsync(qcnt + CNT_F2, 0, sizeof(unsigned long long), st));
+    CK(cudaMemsetAsync(qcnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), st));
+    CK(cudaEventRecord(pq.kev[ev0], st));
+    CK(launch_level2(A, ctx->grid, st));
+    CK(cudaEventRecord(pq.kev[ev0 + 1], st));
+    ++launches;
+    if (A.k >= 4) {
+      CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_groupq[qi], st));
+      launches += 6;
+    }
+    return GCSM_OK;
+  };
+  for (int qi = 0; qi < nq; ++qi)
+    while (sl.q[qi].kev.size() < 4 * std::max<size_t>(qchunks[qi].size(), 1)) {
+      cudaEvent_t ev;
+      CK(cudaEventCreate(&ev));
+      sl.q[qi].kev.push_back(ev);
+    }
+  // GPU path: the first chunk's level-2 kernels read only the seeds' lists — the batch's uploaded U lists (R32) —
+  // so they run on stream2 while the cache step runs on the main stream; the extensions wait for both
+  const bool hoist = ctx->gpu_est;
+  if (hoist) {
+    CK(cudaStreamWaitEvent(ctx->stream2, sl.ev_up, 0));
+    for (int qi = 0; qi < nq; ++qi) {
+      if (qchunks[qi].empty() || qchunks[qi][0].second <= qchunks[qi][0].first) continue;
+      setup(qi, qchunks[qi][0]);
+      gcsm_status g2 = level2(qi, 0, ctx->stream2);
+      if (g2 != GCSM_OK) return g2;
+    }
+    CK(cudaEventRecord(sl.ev_l2, ctx->stream2));
+    CK(cudaStreamWaitEvent(s, sl.ev_l2, 0));
+  }
+  for (int qi = 0; qi < nq; ++qi) {
+    auto &pq = sl.q[qi];
+    const bool sym = !listing && ctx->qs[qi].qps.symmetry;
+    const QueryPlan &QK = sym ? ctx->qs[qi].qps : ctx->qs[qi].qp;
+    const int k = QK.k;
     CK(cudaEventRecord(pq.ev_m0, s));
     size_t nev = 0;
-    for (const auto &ch : qchunks[qi]) {
+    for (size_t c = 0; c < qchunks[qi].size(); ++c) {
+      const auto &ch = qchunks[qi][c];
       if (ch.second <= ch.first) continue;
-      A.units = ctx->d_units + uoff[qi] + ch.first;
-      A.n_units = ch.second - ch.first;
-      while (pq.kev.size() < nev + 3) {
-        cudaEvent_t ev;
-        CK(cudaEventCreate(&ev));
-        pq.kev.push_back(ev);
+      setup(qi, ch);
+      if (!(hoist && c == 0)) {
+        gcsm_status g2 = level2(qi, nev, s);
+        if (g2 != GCSM_OK) return g2;
       }
-      // reset the work cursors and the frontier size of this chunk
-      CK(cudaMemsetAsync(qcnt + CNT_F2, 0, sizeof(unsigned long long), s));
-      CK(cudaMemsetAsync(qcnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), s));
-      CK(cudaEventRecord(pq.kev[nev], s));
-      CK(launch_level2(A, ctx->grid, s));
-      CK(cudaEventRecord(pq.kev[nev + 1], s));
-      ++launches;
+      CK(cudaEventRecord(pq.kev[nev + 2], s));
       if (k >= 4) {
-        CK(launch_group_frontier(A, S.n, ctx->d_hist, ctx->d_bsum, ctx->d_group, s));
-        launches += 6;
-        A.group = ctx->d_group;
+        A.group = ctx->d_groupq[qi];
         if (A.tasks) {
           if (++ctx->task_gen <= 0) ctx->task_gen = 1;  // ready flags hold the launch's generation, never 0
           A.task_gen = ctx->task_gen;
@@ -1318,8 +1367,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
         CK(launch_extend(A, ctx->grid, s));
         ++launches;
       }
-      CK(cudaEventRecord(pq.kev[nev + 2], s));
-      nev += 3;
+      CK(cudaEventRecord(pq.kev[nev + 3], s));
+      nev += 4;
     }
     CK(cudaEventRecord(pq.ev_m1, s));
     pq.nev = nev;
@@ -1407,18 +1456,16 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
       st.cached_vertices = h0[CNT_CACHED];
       st.cache_bytes = h0[CNT_CACHED + 1];
     }
-    float ms_m = 0;
-    cudaEventElapsedTime(&ms_m, pq.ev_m0, pq.ev_m1);
-    st.ms_match = ms_m;
     st.ms_allreduce = ms_a;
     st.ms_copy = ms_c;
-    for (size_t i = 0; i < pq.nev; i += 3) {
+    for (size_t i = 0; i < pq.nev; i += 4) {  // per chunk: level 2 (e0 -> e1), extension (e2 -> e3)
       float a = 0, b = 0;
       cudaEventElapsedTime(&a, pq.kev[i], pq.kev[i + 1]);
-      cudaEventElapsedTime(&b, pq.kev[i + 1], pq.kev[i + 2]);
+      cudaEventElapsedTime(&b, pq.kev[i + 2], pq.kev[i + 3]);
       st.ms_level2 += a;
       st.ms_extend += b;
     }
+    st.ms_match = st.ms_level2 + st.ms_extend;  // kernel time (the first level-2 launches overlap the cache step)
     st.added = h[CNT_ADDED] * pq.aut_mul;
     st.removed = h[CNT_REMOVED] * pq.aut_mul;
     st.hit_bytes_ext = h[CNT_ACC_EXT + 0];
