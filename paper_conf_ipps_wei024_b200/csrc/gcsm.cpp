@@ -105,6 +105,8 @@ struct gcsm_ctx {
     EstUnit *h_eunits = nullptr; size_t h_eunits_cap = 0;  // level-1 walk nodes (GPU estimator)
     int2 *h_eitems = nullptr; size_t h_eitems_cap = 0;     // their work items
     int32_t *h_ulist = nullptr; size_t h_ulist_cap = 0;    // stable lists S(x) of U, packed (GPU path)
+    int4 *h_srec = nullptr; size_t h_srec_cap = 0;         // sampled-index updates of the previous batch's U
+    int32_t *h_sstage = nullptr; size_t h_sstage_cap = 0;
     int32_t *d_ulist = nullptr; size_t d_ulist_cap = 0;    // their device copy (read by this batch's kernels)
     size_t ulist_n = 0;
     double *h_r0 = nullptr; size_t h_r0_cap = 0;           // BINV table staging
@@ -179,6 +181,14 @@ struct gcsm_ctx {
   EstNode2 *d_ef2 = nullptr; size_t ef2_cap = 0;
   double *d_r0 = nullptr; size_t r0_cap = 0;
   double *d_sfc = nullptr;         // BTRD Stirling table (10 doubles)
+  // sampled index of the host lists (every 32nd element of each list of >= 64 elements): lets k_last4 fetch only
+  // the symmetry-range slice of a zero-copy list. Per-vertex slots, relocated to an append area when a merged list
+  // outgrows its slot (none left: the vertex is not indexed and its lists are fetched whole)
+  int32_t *d_sidx = nullptr; uint32_t *d_soff = nullptr;
+  size_t sidx_capacity = 0, sidx_next = 0;
+  std::vector<uint32_t> soff_h, scap_h;
+  int4 *d_srec = nullptr; size_t srec_cap = 0;
+  int32_t *d_sstage = nullptr; size_t sstage_cap = 0;
   size_t r0_n = 0;                 // entries of the device table of (1 - pD)^n
   double r0_pD = -1.0;
   bool est_valid = false;          // the device holds a batch's estimator output (gcsm_get_estimates)
@@ -225,7 +235,8 @@ gcsm_ctx::~gcsm_ctx() {
   for (void *p : dev)
     if (p) cudaFree(p);
   void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
-                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2, d_sfc};
+                  d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2, d_sfc, d_sidx, d_soff,
+                  d_srec, d_sstage};
   for (void *p : dev2)
     if (p) cudaFree(p);
   for (unsigned long long *p : d_levcnt)
@@ -233,7 +244,7 @@ gcsm_ctx::~gcsm_ctx() {
   for (void *p : retired_pinned) cudaFreeHost(p);
   for (Slot &sl : slots) {
     void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt,
-                    sl.h_eunits, sl.h_ulist, sl.h_r0, sl.h_eitems};
+                    sl.h_eunits, sl.h_ulist, sl.h_r0, sl.h_eitems, sl.h_srec, sl.h_sstage};
     if (sl.d_ulist) cudaFree(sl.d_ulist);
     for (void *p : host)
       if (p) cudaFreeHost(p);
@@ -536,6 +547,32 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
     for (int i = 0; i < 10; ++i) sfc[i] = stirling_small(i);
     if (cudaMalloc(&ctx->d_sfc, sizeof sfc) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
     CK(cudaMemcpyAsync(ctx->d_sfc, sfc, sizeof sfc, cudaMemcpyHostToDevice, s));
+    {  // sampled index of every list of >= 64 elements
+      ctx->soff_h.assign((size_t)n, 0xffffffffu);
+      ctx->scap_h.assign((size_t)n, 0);
+      size_t total = 0;
+      for (int32_t v = 0; v < n; ++v)
+        if (S.len[v] >= 64) {
+          const uint32_t ns = (S.len[v] + 31) / 32;
+          ctx->soff_h[v] = (uint32_t)total;
+          ctx->scap_h[v] = ns + 1;
+          total += ns + 1;
+        }
+      ctx->sidx_capacity = total + total / 2 + ((size_t)1 << 20);
+      ctx->sidx_next = total;
+      std::vector<int32_t> smp(total);
+      parallel_for(ctx->opt.host_threads, n, [&](int, int64_t lo, int64_t hi) {
+        for (int64_t v = lo; v < hi; ++v)
+          if (ctx->soff_h[v] != 0xffffffffu)
+            for (uint32_t j = 0; 32 * j < S.len[v]; ++j) smp[ctx->soff_h[v] + j] = S.lst[v][32 * j];
+      });
+      if (ctx->sidx_capacity >= ((size_t)1 << 31) || cudaMalloc(&ctx->d_sidx, 4 * ctx->sidx_capacity) != cudaSuccess ||
+          cudaMalloc(&ctx->d_soff, 4 * (size_t)n) != cudaSuccess)
+        return ctx->fail(GCSM_ENOMEM, "sampled list index");
+      CK(cudaMemcpyAsync(ctx->d_sidx, smp.data(), 4 * total, cudaMemcpyHostToDevice, s));
+      CK(cudaMemcpyAsync(ctx->d_soff, ctx->soff_h.data(), 4 * (size_t)n, cudaMemcpyHostToDevice, s));
+      CK(cudaStreamSynchronize(s));  // pageable sources
+    }
     CK(cudaMemsetAsync(ctx->d_sel, 0, sizeof(SelState), s));
     CK(cudaStreamSynchronize(s));  // hp is pageable and local
     ctx->gpu_ready = true;
@@ -598,6 +635,42 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   if (neu) CK(cudaMemcpyAsync(ctx->d_eunits, sl.h_eunits, sizeof(EstUnit) * neu, cudaMemcpyHostToDevice, s));
   if (nit) CK(cudaMemcpyAsync(ctx->d_eitems, sl.h_eitems, sizeof(int2) * nit, cudaMemcpyHostToDevice, s));
+  {  // the previous batch's updated vertices were merged into new lists: refresh their samples
+    const std::vector<int32_t> &pu = ctx->prev_U;
+    size_t nst = 0;
+    for (int32_t v : pu)
+      if (S.len[v] >= 64) nst += (S.len[v] + 31) / 32;
+    if (!pu.empty()) {
+      if (!host_ensure(sl.h_srec, sl.h_srec_cap, pu.size()) || !host_ensure(sl.h_sstage, sl.h_sstage_cap, nst + 1) ||
+          !dev_ensure(ctx->d_srec, ctx->srec_cap, pu.size()) || !dev_ensure(ctx->d_sstage, ctx->sstage_cap, nst + 1))
+        return ctx->fail(GCSM_ENOMEM, "sampled index staging");
+      size_t pos = 0;
+      for (size_t i = 0; i < pu.size(); ++i) {
+        const int32_t v = pu[i];
+        int32_t off = -1, ns = 0;
+        if (S.len[v] >= 64) {
+          ns = (int32_t)((S.len[v] + 31) / 32);
+          if ((uint32_t)ns <= ctx->scap_h[v] && ctx->soff_h[v] != 0xffffffffu) {
+            off = (int32_t)ctx->soff_h[v];
+          } else if (ctx->sidx_next + 2 * (size_t)ns <= ctx->sidx_capacity) {
+            off = (int32_t)ctx->sidx_next;
+            ctx->scap_h[v] = 2 * (uint32_t)ns;
+            ctx->sidx_next += 2 * (size_t)ns;
+          }
+          if (off >= 0)
+            for (int32_t j = 0; j < ns; ++j) sl.h_sstage[pos + j] = S.lst[v][32 * j];
+        }
+        if (off < 0) ctx->scap_h[v] = 0;
+        ctx->soff_h[v] = off >= 0 ? (uint32_t)off : 0xffffffffu;
+        sl.h_srec[i] = int4{v, off, off >= 0 ? ns : 0, (int)pos};
+        if (off >= 0) pos += (size_t)ns;
+      }
+      CK(cudaMemcpyAsync(ctx->d_srec, sl.h_srec, sizeof(int4) * pu.size(), cudaMemcpyHostToDevice, s));
+      if (pos) CK(cudaMemcpyAsync(ctx->d_sstage, sl.h_sstage, 4 * pos, cudaMemcpyHostToDevice, s));
+      CK(launch_sidx_update(ctx->d_sidx, ctx->d_soff, ctx->d_srec, (int64_t)pu.size(), ctx->d_sstage, s));
+      ++*launches;
+    }
+  }
   if (ndirty) {
     CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * ndirty, cudaMemcpyHostToDevice, s));
     CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * ndirty, cudaMemcpyHostToDevice, s));
@@ -1265,6 +1338,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.cache_hi = ctx->d_cache ? ctx->d_cache + ctx->cache_cap : nullptr;
   A.ubuf_lo = ctx->gpu_est ? reinterpret_cast<const char *>(sl.d_ulist) : nullptr;
   A.ubuf_hi = ctx->gpu_est ? reinterpret_cast<const char *>(sl.d_ulist + sl.ulist_n) : nullptr;
+  A.sidx = ctx->gpu_est && !std::getenv("GCSM_NO_SIDX") ? ctx->d_sidx : nullptr;
+  A.soff = ctx->d_soff;
   A.tup_add = d_tadd;
   A.tup_add_cap = add_cap;
   A.tup_rem = d_trem;

@@ -1136,6 +1136,21 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
         uint32_t lb = 0, le = ml;
         if (rlo > rhi) {
           le = 0;  // no entry of the run reads x2's list
+        } else if (!pin_hit && A.sidx && ml >= 64 && (rlo != INT_MIN || rhi != INT_MAX) &&
+                   __ldg(A.soff + x2) != 0xffffffffu) {
+          // zero-copy list with a sampled index in HBM (every 32nd element): the run's symmetry-range slice is
+          // located without touching host memory and only that slice crosses PCIe (32-element granularity;
+          // every read below is range-checked or range-trimmed)
+          const int32_t *smp = A.sidx + __ldg(A.soff + x2);
+          const uint32_t ns = (ml + 31) >> 5;
+          if (rlo != INT_MIN) {
+            const uint32_t j = warp_lb(smp, ns, rlo + 1, lane);  // samples <= rlo
+            lb = j ? 32u * (j - 1) : 0u;
+          }
+          if (rhi != INT_MAX) {
+            const uint32_t j = warp_lb(smp, ns, rhi, lane);  // samples < rhi: list[32 j] >= rhi when j < ns
+            le = max(lb, min(ml, 32u * j));
+          }
         } else if (GCSM_PIN_RANGE && ml >= 32) {
           if (rlo != INT_MIN) lb = warp_lb(mp, ml, rlo + 1, lane);
           if (rhi != INT_MAX) le = max(lb, warp_lb(mp, ml, rhi, lane));
@@ -1500,6 +1515,25 @@ cudaError_t launch_gather_lists(char *dst, const char *src, const uint64_t *tri,
   if (n <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>((n + 7) / 8, 148 * 16);
   k_gather<<<grid, 256, 0, s>>>(dst, src, tri, n);
+  return cudaGetLastError();
+}
+
+__global__ void k_sidx_update(int32_t *sidx, uint32_t *soff, const int4 *rec, int64_t n, const int32_t *staged) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n;
+       i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const int4 r = rec[i];  // vertex, offset (or -1), count, staging position
+    if (r.y >= 0)
+      for (int j = lane; j < r.z; j += 32) sidx[(uint32_t)r.y + j] = staged[(uint32_t)r.w + j];
+    if (lane == 0) soff[r.x] = r.y >= 0 ? (uint32_t)r.y : 0xffffffffu;
+  }
+}
+
+cudaError_t launch_sidx_update(int32_t *sidx, uint32_t *soff, const int4 *rec, int64_t n, const int32_t *staged,
+                               cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  const int grid = (int)std::min<int64_t>((n + 7) / 8, 148 * 8);
+  k_sidx_update<<<grid, 256, 0, s>>>(sidx, soff, rec, n, staged);
   return cudaGetLastError();
 }
 

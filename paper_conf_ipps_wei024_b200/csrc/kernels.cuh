@@ -53,6 +53,8 @@ struct MatchArgs {
   unsigned long long *cnt;  // CNT_N counters
   const char *cache_lo, *cache_hi;  // HBM cache address range (hit/miss accounting)
   const char *ubuf_lo, *ubuf_hi;    // the batch's uploaded stable lists of U (device-resident, delta accounting)
+  const int32_t *sidx;              // sampled index of the host lists: every 32nd element (nullptr: none)
+  const uint32_t *soff;             // per vertex: offset of its samples in sidx, 0xffffffff = not indexed
   int32_t *tup_add;         // list mode: k ints per tuple
   uint64_t tup_add_cap;
   int32_t *tup_rem;
@@ -90,5 +92,8 @@ cudaError_t launch_group_frontier(const MatchArgs &a, int32_t n_vertices, uint32
                                   int32_t *group, cudaStream_t s);
 cudaError_t launch_gather_lists(char *dst, const char *src, const uint64_t *tri, int64_t n, cudaStream_t s);
 cudaError_t launch_patch_vdesc(VDesc *vdesc, const int64_t *idx, const VDesc *val, int64_t n, cudaStream_t s);
+// sampled-index updates: rec[i] = (vertex, offset, count, staging position); samples staged contiguously
+cudaError_t launch_sidx_update(int32_t *sidx, uint32_t *soff, const int4 *rec, int64_t n, const int32_t *staged,
+                               cudaStream_t s);
 
 }  // namespace gcsm
