@@ -53,7 +53,7 @@ struct MatchArgs {
   unsigned long long *cnt;  // CNT_N counters
   const char *cache_lo, *cache_hi;  // HBM cache address range (hit/miss accounting)
   const char *ubuf_lo, *ubuf_hi;    // the batch's uploaded stable lists of U (device-resident, delta accounting)
-  const int32_t *sidx;              // sampled index of the host lists: every 32nd element (nullptr: none)
+  const int32_t *sidx;              // sampled index of the host lists: every GCSM_SIDX_STRIDE-th element (nullptr: none)
   const uint32_t *soff;             // per vertex: offset of its samples in sidx, 0xffffffff = not indexed
   int32_t *tup_add;         // list mode: k ints per tuple
   uint64_t tup_add_cap;
