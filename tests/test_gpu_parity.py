@@ -566,3 +566,29 @@ def test_multi_query_limits(G):
     a = g.apply_batch(*w.batches[0])
     assert all(g.query_counts(i) == a for i in range(8))
     g.close()
+
+
+@pytest.mark.parametrize("name", ["c4", "k4"])
+def test_sampled_index_on_off(G, name, monkeypatch):
+    """The sampled index only narrows which slice of a zero-copy x2 list crosses PCIe: counts equal the
+    oracle with it on and off over a 4-batch stream (the previous batch's updated vertices get their samples
+    refreshed), and with it on the kernels never copy more bytes from host memory than with it off."""
+    w = gi.make_workload("C2", scale=16, n_edges=600_000, batch=1024, n_batches=4)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    k, qe, ql = gi.query(name)
+    copied = {}
+    for mode in ("on", "off"):
+        if mode == "off":
+            monkeypatch.setenv("GCSM_NO_SIDX", "1")
+        g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+        g.set_query(k, qe, ql)
+        g.set_cache_budget(w.adj_bytes // 20)
+        got, cb = [], 0
+        for ins, dele in w.batches:
+            got.append(g.apply_batch(ins, dele))
+            cb += g.stats()["host_copied_bytes"]
+        g.close()
+        assert got == want, mode
+        copied[mode] = cb
+    monkeypatch.delenv("GCSM_NO_SIDX", raising=False)
+    assert copied["on"] <= copied["off"], copied
