@@ -108,6 +108,14 @@ struct gcsm_ctx {
     int4 *h_srec = nullptr; size_t h_srec_cap = 0;         // sampled-index updates of the previous batch's U
     int32_t *h_sstage = nullptr; size_t h_sstage_cap = 0;
     int32_t *d_ulist = nullptr; size_t d_ulist_cap = 0;    // their device copy (read by this batch's kernels)
+    // per-batch device state (double buffered so that batch t+1's cache step can run while batch t matches):
+    // descriptors (copied from the previous batch's, then patched), delta records and lists, units, counters
+    VDesc *d_vdesc = nullptr;
+    DRec *d_drec = nullptr; size_t drec_cap = 0;
+    int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
+    Unit *d_units = nullptr; size_t units_cap = 0;
+    int2 *d_useg = nullptr; size_t useg_cap = 0;
+    unsigned long long *d_cnt = nullptr;  // CNT_N per query
     size_t ulist_n = 0;
     double *h_r0 = nullptr; size_t h_r0_cap = 0;           // BINV table staging
     cudaEvent_t ev_a0 = nullptr, ev_a1 = nullptr, ev_c0 = nullptr, ev_c1 = nullptr, ev_done = nullptr;
@@ -133,19 +141,17 @@ struct gcsm_ctx {
   int grid = 0, warps_total = 0;
 
   // device buffers
-  VDesc *d_vdesc = nullptr;
   uint16_t *d_lab = nullptr;
-  DRec *d_drec = nullptr; size_t drec_cap = 0;
-  int32_t *d_dlist = nullptr; size_t dlist_cap = 0;
-  Unit *d_units = nullptr; size_t units_cap = 0;
-  int2 *d_useg = nullptr; size_t useg_cap = 0;
   int32_t *d_f2q[GCSM_MAX_QUERIES] = {};  size_t f2q_cap[GCSM_MAX_QUERIES] = {};  // per query: 2 * f2 entries ints
   int32_t *d_groupq[GCSM_MAX_QUERIES] = {};  size_t groupq_cap[GCSM_MAX_QUERIES] = {};  // frontier grouped by x2
   cudaStream_t stream2 = nullptr;  // GPU path: the first level-2 kernels run here, beside the cache step
+  // GPU path: batch t+1's cache step (uploads, walks, ranking, k_copy, descriptor switch into its own descriptor
+  // copy) runs here while batch t's extension kernels run on `stream` (GCSM_NO_OVERLAP=1 at create: on `stream`)
+  cudaStream_t stream3 = nullptr;
+  bool overlap = false;
   uint32_t *d_hist = nullptr;                         // n counters + scan
   uint32_t *d_bsum = nullptr;
   int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
-  unsigned long long *d_cnt = nullptr; size_t cnt_queries = 0;  // CNT_N per query
   char *d_cache = nullptr; size_t cache_cap = 0;   // the buffer this batch's kernels read
   char *d_cachebuf[2] = {nullptr, nullptr};        // double buffer: last batch's cache stays readable
   int cache_cur = 0;                               // buffer holding the previous batch's cache
@@ -226,7 +232,8 @@ gcsm_ctx::~gcsm_ctx() {
   for (Query &q : qs)
     for (DevPlan *p : {q.d_plans, q.d_splans})
       if (p) cudaFree(p);
-  void *dev[] = {d_vdesc, d_lab, d_drec, d_dlist, d_units, d_useg, d_scratch, d_cnt, d_cachebuf[0],
+  if (stream3) cudaStreamSynchronize(stream3);
+  void *dev[] = {d_lab, d_scratch, d_cachebuf[0],
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (int q = 0; q < GCSM_MAX_QUERIES; ++q) {
     if (d_f2q[q]) cudaFree(d_f2q[q]);
@@ -246,6 +253,9 @@ gcsm_ctx::~gcsm_ctx() {
     void *host[] = {sl.h_pidx, sl.h_pval, sl.h_drec, sl.h_dlist, sl.h_units, sl.h_gather, sl.h_fresh, sl.h_cnt,
                     sl.h_eunits, sl.h_ulist, sl.h_r0, sl.h_eitems, sl.h_srec, sl.h_sstage};
     if (sl.d_ulist) cudaFree(sl.d_ulist);
+    for (void *p : {(void *)sl.d_vdesc, (void *)sl.d_drec, (void *)sl.d_dlist, (void *)sl.d_units, (void *)sl.d_useg,
+                    (void *)sl.d_cnt})
+      if (p) cudaFree(p);
     for (void *p : host)
       if (p) cudaFreeHost(p);
     for (cudaEvent_t e : {sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done, sl.ev_up, sl.ev_l2})
@@ -259,6 +269,7 @@ gcsm_ctx::~gcsm_ctx() {
   if (stream2) cudaStreamSynchronize(stream2);
   if (stream) cudaStreamDestroy(stream);
   if (stream2) cudaStreamDestroy(stream2);
+  if (stream3) cudaStreamDestroy(stream3);
 }
 
 extern "C" {
@@ -321,6 +332,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
   if (cudaStreamCreateWithFlags(&ctx->stream2, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
+  if (cudaStreamCreateWithFlags(&ctx->stream3, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
   for (auto &sl : ctx->slots) {
     for (cudaEvent_t *ev : {&sl.ev_a0, &sl.ev_a1, &sl.ev_c0, &sl.ev_c1, &sl.ev_done})
       if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
@@ -330,17 +342,19 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
         cudaSuccess)
       return bail(GCSM_ENOMEM);
   }
-  if (cudaMalloc(&ctx->d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
-  if (cudaMalloc(&ctx->d_cnt, sizeof(unsigned long long) * CNT_N * GCSM_MAX_QUERIES) != cudaSuccess)
-    return bail(GCSM_ENOMEM);
+  for (auto &sl : ctx->slots)
+    if (cudaMalloc(&sl.d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess ||
+        cudaMalloc(&sl.d_cnt, sizeof(unsigned long long) * CNT_N * GCSM_MAX_QUERIES) != cudaSuccess)
+      return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
   if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)n + 2047) / 2048 + 1)) != cudaSuccess)
     return bail(GCSM_ENOMEM);
   {
     std::vector<VDesc> vd(n);
     for (int32_t v = 0; v < n; ++v) vd[v] = VDesc{ctx->store.dev_ptr(ctx->store.lst[v]), ctx->store.len[v], 0};
-    if (cudaMemcpy(ctx->d_vdesc, vd.data(), sizeof(VDesc) * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
-      return bail(GCSM_EDEVICE);
+    for (auto &sl : ctx->slots)
+      if (cudaMemcpy(sl.d_vdesc, vd.data(), sizeof(VDesc) * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
+        return bail(GCSM_EDEVICE);
   }
   if (labels) {
     if (cudaMalloc(&ctx->d_lab, 2 * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
@@ -350,6 +364,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   ctx->mark.assign(n, 0);
   ctx->slot16.assign(n, 0);
   if (const char *he = std::getenv("GCSM_HOST_EST")) ctx->gpu_est = std::atoi(he) == 0;
+  ctx->overlap = ctx->gpu_est && !std::getenv("GCSM_NO_OVERLAP");
   ctx->grid = match_grid(dev, &ctx->warps_total);
   // a communicator whenever an id is given (world 1 included: the single-rank allreduce exercises the same path)
   if (o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
@@ -628,11 +643,11 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
       oi += qitems[qi].size();
     }
   }
-  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
+  CK(cudaMemsetAsync(sl.d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
   if (sl.ulist_n) CK(cudaMemcpyAsync(sl.d_ulist, sl.h_ulist, 4 * sl.ulist_n, cudaMemcpyHostToDevice, s));
-  if (nU) CK(cudaMemcpyAsync(ctx->d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
-  if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
-  if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
+  if (nU) CK(cudaMemcpyAsync(sl.d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
+  if (nd) CK(cudaMemcpyAsync(sl.d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
+  if (gnu) CK(cudaMemcpyAsync(sl.d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   if (neu) CK(cudaMemcpyAsync(ctx->d_eunits, sl.h_eunits, sizeof(EstUnit) * neu, cudaMemcpyHostToDevice, s));
   if (nit) CK(cudaMemcpyAsync(ctx->d_eitems, sl.h_eitems, sizeof(int2) * nit, cudaMemcpyHostToDevice, s));
   {  // the previous batch's updated vertices were merged into new lists: refresh their samples
@@ -674,7 +689,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   if (ndirty) {
     CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * ndirty, cudaMemcpyHostToDevice, s));
     CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * ndirty, cudaMemcpyHostToDevice, s));
-    CK(launch_patch_vdesc_host(ctx->d_vdesc, ctx->d_hptr, ctx->d_pidx, ctx->d_pval, (int64_t)ndirty, s));
+    CK(launch_patch_vdesc_host(sl.d_vdesc, ctx->d_hptr, ctx->d_pidx, ctx->d_pval, (int64_t)ndirty, s));
     ++*launches;
   }
   CK(cudaEventRecord(sl.ev_up, s));  // the batch's data is on the device: the level-2 kernels may start (stream2)
@@ -703,10 +718,10 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.reset_first = ctx->cache_reset;
   ctx->cache_reset = false;
   c.budget = ctx->budget;
-  c.vdesc = ctx->d_vdesc;
+  c.vdesc = sl.d_vdesc;
   c.hptr = ctx->d_hptr;
-  c.drec = ctx->d_drec;
-  c.dlist = ctx->d_dlist;
+  c.drec = sl.d_drec;
+  c.dlist = sl.d_dlist;
   c.lab = ctx->d_lab;
   c.pD = pD;
   c.r0tab = ctx->d_r0;
@@ -729,7 +744,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.cub_tmp = ctx->d_cubtmp;
   c.cub_tmp_bytes = ctx->cubtmp_bytes;
   c.cache = ctx->d_cache;
-  c.cnt_cached = ctx->d_cnt + CNT_CACHED;
+  c.cnt_cached = sl.d_cnt + CNT_CACHED;
   CK(launch_cache_step(c, s, launches));
   ctx->est_valid = est_on;
   CK(cudaEventRecord(sl.ev_c1, s));
@@ -761,7 +776,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       g_alloc_stream = nullptr;
       g_retired_pinned = nullptr;
     }
-  } alloc_scope(ctx->stream, &ctx->retired_pinned);
+  } alloc_scope(ctx->overlap ? nullptr : ctx->stream, &ctx->retired_pinned);  // two streams: synchronous growth
   HostStore &S = ctx->store;
   const int nq = (int)ctx->qs.size();
   int kmax = 2;
@@ -1226,14 +1241,21 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   tr.mark("staging");
 
   cudaStream_t s = ctx->stream;
+  // the cache step's stream: with overlap it runs beside the previous batch's matching (it writes only this slot's
+  // descriptors, delta records, units and counters and the other cache buffer; the previous use of this slot was
+  // batch t-2, already collected by gcsm_wait_batch)
+  cudaStream_t cs = ctx->overlap ? ctx->stream3 : s;
   if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
-      !dev_ensure(ctx->d_drec, ctx->drec_cap, nU) || !dev_ensure(ctx->d_dlist, ctx->dlist_cap, nd) ||
-      !dev_ensure(ctx->d_units, ctx->units_cap, (size_t)gnu) || !dev_ensure(ctx->d_useg, ctx->useg_cap, (size_t)gnu))
+      !dev_ensure(sl.d_drec, sl.drec_cap, nU) || !dev_ensure(sl.d_dlist, sl.dlist_cap, nd) ||
+      !dev_ensure(sl.d_units, sl.units_cap, (size_t)gnu) || !dev_ensure(sl.d_useg, sl.useg_cap, (size_t)gnu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
-  CK(cudaEventRecord(sl.ev_c0, s));
+  CK(cudaEventRecord(sl.ev_c0, cs));
+  if (ctx->batch_seq > 0)  // this batch's descriptors start as the previous batch's (after its cache step)
+    CK(cudaMemcpyAsync(sl.d_vdesc, ctx->slots[(ctx->batch_seq + 1) & 1].d_vdesc, sizeof(VDesc) * (size_t)S.n,
+                       cudaMemcpyDeviceToDevice, cs));
   uint64_t launches = 0;
   if (ctx->gpu_est) {
-    gcsm_status gs = enqueue_gpu_cache(ctx, sl, s, dirty.size(), nU, nd, gnu, qeu, qitems, qf2cap, eu_maxB, D, qnu,
+    gcsm_status gs = enqueue_gpu_cache(ctx, sl, cs, dirty.size(), nU, nd, gnu, qeu, qitems, qf2cap, eu_maxB, D, qnu,
                                        qwalks, use_cache, &launches);
     if (gs != GCSM_OK) return gs;
     st.h2d_bytes = (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU + 4 * nd +
@@ -1261,16 +1283,17 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   (void)retained_bytes;
   CK(cudaMemcpyAsync(ctx->d_pidx, sl.h_pidx, sizeof(int64_t) * dirty.size(), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(ctx->d_pval, sl.h_pval, sizeof(VDesc) * dirty.size(), cudaMemcpyHostToDevice, s));
-  CK(launch_patch_vdesc(ctx->d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
+  CK(launch_patch_vdesc(sl.d_vdesc, ctx->d_pidx, ctx->d_pval, (int64_t)dirty.size(), s));
   launches += dirty.empty() ? 0 : 1;
-  if (nU) CK(cudaMemcpyAsync(ctx->d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
-  if (nd) CK(cudaMemcpyAsync(ctx->d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
-  if (gnu) CK(cudaMemcpyAsync(ctx->d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
+  if (nU) CK(cudaMemcpyAsync(sl.d_drec, sl.h_drec, sizeof(DRec) * nU, cudaMemcpyHostToDevice, s));
+  if (nd) CK(cudaMemcpyAsync(sl.d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
+  if (gnu) CK(cudaMemcpyAsync(sl.d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(sl.ev_c1, s));
   st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
                  4 * nd + sizeof(Unit) * (size_t)gnu;
-  CK(cudaMemsetAsync(ctx->d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
+  CK(cudaMemsetAsync(sl.d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
   }
+  if (cs != s) CK(cudaStreamWaitEvent(s, sl.ev_c1, 0));  // the matching kernels read the cache step's output
 
   // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
@@ -1325,10 +1348,10 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     d_trem = ctx->d_tup + (size_t)k * add_cap;
   }
   MatchArgs A{};
-  A.vdesc = ctx->d_vdesc;
+  A.vdesc = sl.d_vdesc;
   A.lab = ctx->d_lab;
-  A.drec = ctx->d_drec;
-  A.dlist = ctx->d_dlist;
+  A.drec = sl.d_drec;
+  A.dlist = sl.d_dlist;
 
   A.scratch = ctx->d_scratch;
   A.scratch_end = ctx->d_scratch + stride * (size_t)ctx->warps_total;
@@ -1365,12 +1388,12 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     A.plans = sym ? ctx->qs[qi].d_splans : ctx->qs[qi].d_plans;
     A.n_plans = (int32_t)QK.plans.size();
     A.k = QK.k;
-    A.cnt = ctx->d_cnt + (size_t)qi * CNT_N;
+    A.cnt = sl.d_cnt + (size_t)qi * CNT_N;
     A.f2 = reinterpret_cast<int2 *>(ctx->d_f2q[qi]);
     A.f2_cap = qf2need[qi];
-    A.units = ctx->d_units + uoff[qi] + ch.first;
+    A.units = sl.d_units + uoff[qi] + ch.first;
     A.n_units = ch.second - ch.first;
-    A.useg = ctx->d_useg + uoff[qi] + ch.first;
+    A.useg = sl.d_useg + uoff[qi] + ch.first;
     A.group = nullptr;
     A.tasks = nullptr;
     if (QK.k >= 5 && !listing) {
@@ -1384,7 +1407,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // level 2 + grouping of a chunk (events e0 / e1 around the level-2 kernel) on stream `st`
   auto level2 = [&](int qi, size_t ev0, cudaStream_t st) -> gcsm_status {
     auto &pq = sl.q[qi];
-    unsigned long long *qcnt = ctx->d_cnt + (size_t)qi * CNT_N;
+    unsigned long long *qcnt = sl.d_cnt + (size_t)qi * CNT_N;
     CK(cudaMemsetAsync(qcnt + CNT_F2, 0, sizeof(unsigned long long), st));
     CK(cudaMemsetAsync(qcnt + CNT_CURSOR0, 0, 2 * sizeof(unsigned long long), st));
     CK(cudaEventRecord(pq.kev[ev0], st));
@@ -1408,6 +1431,9 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   const bool hoist = ctx->gpu_est;
   if (hoist) {
     CK(cudaStreamWaitEvent(ctx->stream2, sl.ev_up, 0));
+    // the frontier buffers and grouping counters are shared with the previous batch's matching (stream order on
+    // `stream` no longer implies it when the cache step runs beside it)
+    if (ctx->batch_seq > 0) CK(cudaStreamWaitEvent(ctx->stream2, ctx->slots[(ctx->batch_seq + 1) & 1].ev_done, 0));
     for (int qi = 0; qi < nq; ++qi) {
       if (qchunks[qi].empty() || qchunks[qi][0].second <= qchunks[qi][0].first) continue;
       setup(qi, qchunks[qi][0]);
@@ -1453,13 +1479,13 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   CK(cudaEventRecord(sl.ev_a0, s));
   if (ctx->comm) {
     for (int qi = 0; qi < nq; ++qi) {
-      unsigned long long *qcnt = ctx->d_cnt + (size_t)qi * CNT_N;
+      unsigned long long *qcnt = sl.d_cnt + (size_t)qi * CNT_N;
       if (ncclAllReduce(qcnt, qcnt, 2, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
         return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
     }
   }
   CK(cudaEventRecord(sl.ev_a1, s));
-  CK(cudaMemcpyAsync(sl.h_cnt, ctx->d_cnt, sizeof(unsigned long long) * CNT_N * (size_t)nq, cudaMemcpyDeviceToHost,
+  CK(cudaMemcpyAsync(sl.h_cnt, sl.d_cnt, sizeof(unsigned long long) * CNT_N * (size_t)nq, cudaMemcpyDeviceToHost,
                      s));
   CK(cudaEventRecord(sl.ev_done, s));
   st.kernel_launches = launches;
