@@ -139,6 +139,7 @@ struct gcsm_ctx {
   uint64_t waited = 0;  // batches whose results have been collected
   ncclComm_t comm = nullptr;
   int grid = 0, warps_total = 0;
+  int ext_grid = 0;  // blocks of the extension kernels (GCSM_EXT_RESERVE blocks left for the overlapped cache step)
 
   // device buffers
   uint16_t *d_lab = nullptr;
@@ -332,7 +333,13 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
   if (cudaStreamCreateWithFlags(&ctx->stream2, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
-  if (cudaStreamCreateWithFlags(&ctx->stream3, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
+  {  // the cache step's stream may take the higher scheduling priority (GCSM_CS_PRIO=1): its blocks go first when
+     // the extension kernels' blocks retire
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    const int prio = std::getenv("GCSM_CS_PRIO") ? hi : lo;
+    if (cudaStreamCreateWithPriority(&ctx->stream3, cudaStreamNonBlocking, prio) != cudaSuccess) return bail(GCSM_EDEVICE);
+  }
   for (auto &sl : ctx->slots) {
     for (cudaEvent_t *ev : {&sl.ev_a0, &sl.ev_a1, &sl.ev_c0, &sl.ev_c1, &sl.ev_done})
       if (cudaEventCreate(ev) != cudaSuccess) return bail(GCSM_EDEVICE);
@@ -366,6 +373,9 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   if (const char *he = std::getenv("GCSM_HOST_EST")) ctx->gpu_est = std::atoi(he) == 0;
   ctx->overlap = ctx->gpu_est && !std::getenv("GCSM_NO_OVERLAP");
   ctx->grid = match_grid(dev, &ctx->warps_total);
+  ctx->ext_grid = ctx->grid;
+  if (const char *r = std::getenv("GCSM_EXT_RESERVE"))
+    if (ctx->overlap) ctx->ext_grid = std::max(1, ctx->grid - std::atoi(r));
   // a communicator whenever an id is given (world 1 included: the single-rank allreduce exercises the same path)
   if (o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
     ncclUniqueId id;
@@ -1465,7 +1475,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
           if (++ctx->task_gen <= 0) ctx->task_gen = 1;  // ready flags hold the launch's generation, never 0
           A.task_gen = ctx->task_gen;
         }
-        CK(launch_extend(A, ctx->grid, s));
+        CK(launch_extend(A, ctx->ext_grid, s));
         ++launches;
       }
       CK(cudaEventRecord(pq.kev[nev + 3], s));

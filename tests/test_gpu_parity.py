@@ -592,3 +592,36 @@ def test_sampled_index_on_off(G, name, monkeypatch):
         copied[mode] = cb
     monkeypatch.delenv("GCSM_NO_SIDX", raising=False)
     assert copied["on"] <= copied["off"], copied
+
+
+@pytest.mark.parametrize("overlap", ["on", "off"])
+def test_pipelined_cache_step_overlap(G, overlap, monkeypatch):
+    """Batch t+1's GPU cache step runs on its own stream beside batch t's matching (DESIGN.md §1c step 6; off:
+    GCSM_NO_OVERLAP=1 at create). Two standing queries, C2-shaped graph, 5 pipelined batches: each query's counts
+    equal the oracle's and the final graph equals the oracle's either way."""
+    if overlap == "off":
+        monkeypatch.setenv("GCSM_NO_OVERLAP", "1")
+    w = gi.make_workload("C2", scale=16, n_edges=600_000, batch=2048, n_batches=5)
+    names = ["k4", "c4"]
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    g.set_query(*gi.query(names[0]))
+    qids = [0] + [g.add_query(*gi.query(nm)) for nm in names[1:]]
+    g.set_cache_budget(w.adj_bytes // 10)
+    got = {nm: [] for nm in names}
+
+    def collect():
+        g.wait_batch()
+        for nm, qi in zip(names, qids):
+            got[nm].append(g.query_counts(qi))
+
+    g.submit_batch(*w.batches[0])
+    for b in w.batches[1:]:
+        g.submit_batch(*b)
+        collect()
+    collect()
+    rp2, col2 = g.export_csr()
+    g.close()
+    for nm in names:
+        want, (rp1, col1) = oracle_run(w.n, w.row_ptr, w.col, None, nm, w.batches)
+        assert got[nm] == want, nm
+    assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
