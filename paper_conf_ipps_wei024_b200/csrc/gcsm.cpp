@@ -333,11 +333,13 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   };
   if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
   if (cudaStreamCreateWithFlags(&ctx->stream2, cudaStreamNonBlocking) != cudaSuccess) return bail(GCSM_EDEVICE);
-  {  // the cache step's stream may take the higher scheduling priority (GCSM_CS_PRIO=1): its blocks go first when
-     // the extension kernels' blocks retire
+  {  // the cache step's stream takes the higher scheduling priority (it feeds the next batch's matching): its blocks
+     // go first when the extension kernels' blocks retire (GCSM_CS_PRIO=0: default priority; A/B in
+     // profiles/ab_r01_reserve.txt)
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    const int prio = std::getenv("GCSM_CS_PRIO") ? hi : lo;
+    const char *pe = std::getenv("GCSM_CS_PRIO");
+    const int prio = (pe && std::atoi(pe) == 0) ? lo : hi;
     if (cudaStreamCreateWithPriority(&ctx->stream3, cudaStreamNonBlocking, prio) != cudaSuccess) return bail(GCSM_EDEVICE);
   }
   for (auto &sl : ctx->slots) {
