@@ -230,12 +230,12 @@ gcsm_status gcsm_export_csr(const gcsm_ctx *ctx, int64_t *row_ptr, int32_t *col,
  * ascending, and per vertex the per-level sums of walk multiplicities B for
  * tree levels 1..k-2 (eq. (3)): levcnt[i*8 + (l-1)]. *n_out = the number of
  * such vertices (ETRUNC if > cap; the first cap are written). On the GPU path the
- * sums live in device memory: the call synchronises the context's stream. */
+ * sums live in device memory: the call synchronises the context's streams. */
 gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levcnt, uint64_t cap, uint64_t *n_out);
 
 /* Last batch's cached vertex set (step 3), ascending: the longest prefix of (estimate desc, id asc)
  * that fits the budget (R23), over the vertices not updated by the batch on the GPU path (their
- * stable lists are uploaded with the batch, R32). Synchronises the context's stream. */
+ * stable lists are uploaded with the batch, R32). Synchronises the context's streams. */
 gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uint64_t *n_out);
 
 /* Roofline denominators the hot path needs and MEASURED_PEAKS.json lacks

@@ -1689,7 +1689,8 @@ gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levc
   if (ctx->gpu_est) {  // device-resident walk sums of the last batch (query 0): rows of the touched set, non-zero
     *n_out = 0;
     if (!ctx->est_valid || ctx->qs.empty() || ctx->qs[0].qp.k <= 2 || !ctx->d_levcnt[0]) return GCSM_OK;
-    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) return GCSM_EDEVICE;
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess || cudaStreamSynchronize(ctx->stream3) != cudaSuccess)
+      return GCSM_EDEVICE;
     SelState st;
     if (cudaMemcpy(&st, ctx->d_sel, sizeof st, cudaMemcpyDeviceToHost) != cudaSuccess) return GCSM_EDEVICE;
     const int64_t nt = (int64_t)st.n_touched;
@@ -1701,6 +1702,7 @@ gcsm_status gcsm_get_estimates(const gcsm_ctx *ctx, int32_t *ids, uint64_t *levc
       cudaError_t e = launch_estimates_gather(ctx->d_tids, nt, ctx->d_levcnt[0], ctx->qs[0].qp.k - 2, d_rows,
                                               ctx->stream);
       if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream3);
       if (e == cudaSuccess) e = cudaMemcpy(rows.data(), d_rows, 8 * 8 * (size_t)nt, cudaMemcpyDeviceToHost);
       if (e == cudaSuccess) e = cudaMemcpy(tid.data(), ctx->d_tids, 4 * (size_t)nt, cudaMemcpyDeviceToHost);
       cudaFree(d_rows);
@@ -1735,7 +1737,8 @@ gcsm_status gcsm_get_cached(const gcsm_ctx *ctx, int32_t *ids, uint64_t cap, uin
   if (ctx->gpu_est) {  // the GPU packer's last selection (ids ascending)
     *n_out = 0;
     if (!ctx->gpu_ready) return GCSM_OK;
-    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) return GCSM_EDEVICE;
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess || cudaStreamSynchronize(ctx->stream3) != cudaSuccess)
+      return GCSM_EDEVICE;
     SelState st;
     if (cudaMemcpy(&st, ctx->d_sel, sizeof st, cudaMemcpyDeviceToHost) != cudaSuccess) return GCSM_EDEVICE;
     const uint64_t n = st.prev_sel, w = std::min<uint64_t>(n, cap);
