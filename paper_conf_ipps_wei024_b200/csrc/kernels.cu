@@ -59,9 +59,6 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GCSM_MINBLOCKS
 #define GCSM_MINBLOCKS 4  // resident 256-thread blocks per SM requested from ptxas for k_extend
 #endif
-#ifndef GCSM_MERGE_INT4
-#define GCSM_MERGE_INT4 0
-#endif
 constexpr uint32_t kSmemInts = GCSM_SMEM_INTS;  // per-warp shared staging slice
 constexpr int kSmemBytes = kWarps * kSmemInts * 4;
 #ifndef GCSM_EXT_CHUNK
@@ -268,12 +265,8 @@ __device__ GCSM_COLD void stage_lists(const MatchArgs &A, LRef *L, int nl, int d
 // co-rank binary search and merges its range sequentially, counting a[i] == b[j] when it consumes a[i] (ties
 // take A first, so an equal pair is counted exactly once even across lane boundaries). O((na+nb)/32 + log)
 // instructions per lane instead of ceil(d/32) * log2(L) dependent probes.
-__device__ __forceinline__ int32_t pick4(const int4 &w, uint32_t k) {
-  return k == 0 ? w.x : (k == 1 ? w.y : (k == 2 ? w.z : w.w));
-}
-
-// Both runs are 16-byte aligned and allocated in 16-byte granules, so each lane reads its segment as int4
-// windows (one load per 4 elements, L1-friendly).
+// (Runs start anywhere once range-trimmed, so the lanes read scalars; an int4-window variant faulted on trimmed
+// runs and was removed.)
 __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, const int32_t *b, uint32_t nb,
                                                 int label, const uint16_t *lab, int lane) {
   const uint32_t T = na + nb;
@@ -286,7 +279,6 @@ __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, c
     else hi = i;
   }
   uint32_t i = lo, j = d0 - lo, cnt = 0;
-#if !GCSM_MERGE_INT4
   // branch-free steps; an equal pair advances both runs (still counted once: the co-rank split puts a[i]
   // before an equal b[j], so the lane owning a[i] counts it and the next lane starts past it)
   while (i + j < d1) {
@@ -297,34 +289,6 @@ __device__ __forceinline__ uint32_t merge_count(const int32_t *a, uint32_t na, c
     i += le;
     j += ge;
   }
-#else
-  const int4 *a4 = reinterpret_cast<const int4 *>(a);
-  const int4 *b4 = reinterpret_cast<const int4 *>(b);
-  int4 wa = make_int4(0, 0, 0, 0), wb = make_int4(0, 0, 0, 0);
-  if (i < na) wa = a4[i >> 2];
-  if (j < nb) wb = b4[j >> 2];
-  int32_t ai = i < na ? pick4(wa, i & 3) : INT_MAX, bj = j < nb ? pick4(wb, j & 3) : INT_MAX;
-  for (uint32_t st = d0; st < d1; ++st) {
-    if (ai <= bj) {
-      if (ai == bj && (label < 0 || lab[ai] == (uint16_t)label)) ++cnt;
-      ++i;
-      if (i < na) {
-        if ((i & 3) == 0) wa = a4[i >> 2];
-        ai = pick4(wa, i & 3);
-      } else {
-        ai = INT_MAX;
-      }
-    } else {
-      ++j;
-      if (j < nb) {
-        if ((j & 3) == 0) wb = b4[j >> 2];
-        bj = pick4(wb, j & 3);
-      } else {
-        bj = INT_MAX;
-      }
-    }
-  }
-#endif
 #pragma unroll
   for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
   return cnt;
