@@ -1256,7 +1256,9 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // the cache step's stream: with overlap it runs beside the previous batch's matching (it writes only this slot's
   // descriptors, delta records, units and counters and the other cache buffer; the previous use of this slot was
   // batch t-2, already collected by gcsm_wait_batch)
-  cudaStream_t cs = ctx->overlap ? ctx->stream3 : s;
+  // (not with a 6-vertex query: its level->=2 walks read zero-copy lists and contend for the host link with the
+  // extension kernels they would run beside — C4: 3.67 K vs 3.89 K updated edges/s)
+  cudaStream_t cs = (ctx->overlap && kmax <= 5) ? ctx->stream3 : s;
   if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
       !dev_ensure(sl.d_drec, sl.drec_cap, nU) || !dev_ensure(sl.d_dlist, sl.dlist_cap, nd) ||
       !dev_ensure(sl.d_units, sl.units_cap, (size_t)gnu) || !dev_ensure(sl.d_useg, sl.useg_cap, (size_t)gnu))
