@@ -23,8 +23,7 @@ _lib = None
 def _load():
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            _build_lib()
+        _build_lib()  # rebuilds only when gen.cpp is newer than the library
         lib = ctypes.CDLL(LIB_PATH)
         P = ctypes.c_void_p
         lib.gi_rmat_edges.restype = ctypes.c_int64
@@ -33,8 +32,13 @@ def _load():
                                       ctypes.c_int64, ctypes.c_int32]
         lib.gi_build_csr.restype = ctypes.c_int32
         lib.gi_build_csr.argtypes = [ctypes.c_int32, ctypes.c_int64, P, ctypes.c_int32, P, P]
+        lib.gi_build_csr_skip.restype = ctypes.c_int32
+        lib.gi_build_csr_skip.argtypes = [ctypes.c_int32, ctypes.c_int64, P, P, ctypes.c_int32, P, P]
         lib.gi_labels.restype = None
         lib.gi_labels.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_uint64, P]
+        lib.gi_grid_edges.restype = ctypes.c_int64
+        lib.gi_grid_edges.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_double, ctypes.c_double,
+                                      ctypes.c_uint64, P, ctypes.c_int64]
         lib.gi_stream.restype = ctypes.c_int64
         lib.gi_stream.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_uint64, P, P]
         _lib = lib
@@ -65,12 +69,24 @@ def rmat_edges(scale: int, n_edges: int, a: float, b: float, c: float, seed: int
     return out
 
 
-def csr_from_edges(n: int, uv: np.ndarray):
-    """Symmetric CSR (row_ptr int64[n+1], col int32[2m]) with sorted rows."""
+def grid_edges(W: int, H: int, p_keep: float, p_diag: float, seed: int) -> np.ndarray:
+    """Road-network-shaped edges (RoadNetPA/CA, Table I; Fig. 11): a W x H lattice thinned to p_keep plus cell
+    diagonals with p_diag, ids permuted; int32 [m,2] (u<v) in generation order."""
+    cap = 3 * W * H
+    out = np.empty((cap, 2), dtype=np.int32)
+    m = _load().gi_grid_edges(W, H, p_keep, p_diag, seed & (2**64 - 1), _p(out), cap)
+    return out[:m].copy()
+
+
+def csr_from_edges(n: int, uv: np.ndarray, skip: np.ndarray | None = None):
+    """Symmetric CSR (row_ptr int64[n+1], col int32[2m]) with sorted rows; `skip` (bool[m]) leaves edges out."""
     uv = np.ascontiguousarray(uv, dtype=np.int32).reshape(-1, 2)
+    m = len(uv) - (0 if skip is None else int(np.count_nonzero(skip)))
     rp = np.empty(n + 1, dtype=np.int64)
-    col = np.empty(2 * len(uv), dtype=np.int32)
-    if _load().gi_build_csr(n, len(uv), _p(uv), _threads(), _p(rp), _p(col)) != 0:
+    col = np.empty(2 * m, dtype=np.int32)
+    sk = None if skip is None else np.ascontiguousarray(skip, dtype=np.uint8)
+    if _load().gi_build_csr_skip(n, len(uv), _p(uv), None if sk is None else _p(sk), _threads(), _p(rp),
+                                 _p(col)) != 0:
         raise ValueError("bad edge list (out of range or self loop)")
     return rp, col
 
@@ -119,6 +135,13 @@ QUERIES = {
     "prism6": (6, [(0, 1), (0, 2), (1, 2), (3, 4), (3, 5), (4, 5), (0, 3), (1, 4), (2, 5)], None),
     "k4tri6": (6, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3), (0, 4), (1, 4), (2, 5), (3, 5)], None),
     "k6": (6, [(i, j) for i in range(6) for j in range(i + 1, 6)], None),
+    # 7- and 8-vertex patterns (the paper's query sizes reach 7; the ABI accepts k <= 8)
+    "wheel7": (7, [(0, i) for i in range(1, 7)] + [(i, i % 6 + 1) for i in range(1, 7)], None),
+    "k4k4_7": (7, [(i, j) for i in range(4) for j in range(i + 1, 4)]
+               + [(i, j) for i in (0, 4, 5, 6) for j in (0, 4, 5, 6) if i < j], None),
+    "k7": (7, [(i, j) for i in range(7) for j in range(i + 1, 7)], None),
+    "cube8": (8, [(i, i ^ (1 << b)) for i in range(8) for b in range(3) if i < i ^ (1 << b)], None),
+    "k8": (8, [(i, j) for i in range(8) for j in range(i + 1, 8)], None),
 }
 
 
@@ -130,6 +153,46 @@ ORDERS = {
     "prism6": [0, 3, 4, 1, 2, 5],
     "bowtie5": [0, 3, 4, 1, 2],
 }
+
+
+def _connected(k, edges):
+    adj = {i: set() for i in range(k)}
+    for a, b in edges:
+        adj[a].add(b)
+        adj[b].add(a)
+    seen, todo = {0}, [0]
+    while todo:
+        x = todo.pop()
+        for y in adj[x] - seen:
+            seen.add(y)
+            todo.append(y)
+    return len(seen) == k
+
+
+def motifs(size: int):
+    """All connected simple graphs on `size` vertices up to isomorphism (the motifs of Fig. 11):
+    2 of size 3, 6 of size 4, 21 of size 5. Each as (name, edge list) in a canonical form (the lexicographically
+    smallest edge bitmask over all vertex permutations), ordered by (edge count, canonical mask)."""
+    import itertools
+    pairs = [(i, j) for i in range(size) for j in range(i + 1, size)]
+    index = {p: t for t, p in enumerate(pairs)}
+    perms = list(itertools.permutations(range(size)))
+    seen = {}
+    for mask in range(1, 1 << len(pairs)):
+        edges = [pairs[t] for t in range(len(pairs)) if mask >> t & 1]
+        if not _connected(size, edges):
+            continue
+        canon = min(sum(1 << index[tuple(sorted((p[a], p[b])))] for a, b in edges) for p in perms)
+        if canon not in seen:
+            seen[canon] = [pairs[t] for t in range(len(pairs)) if canon >> t & 1]
+    out = sorted(seen.items(), key=lambda kv: (bin(kv[0]).count("1"), kv[0]))
+    return [(f"m{size}_{i}", e) for i, (_, e) in enumerate(out)]
+
+
+for _size in (3, 4, 5):
+    for _name, _edges in motifs(_size):
+        QUERIES[_name] = (_size, _edges, None)
+MOTIFS = {sz: [nm for nm, _ in motifs(sz)] for sz in (3, 4, 5)}
 
 
 def order(name: str):
@@ -178,6 +241,10 @@ CONFIGS = {
     "C4": dict(scale=26, n_edges=1_800_000_000, abc=(0.42, 0.176, 0.176), id_limit=0, L=0,
                queries=["prism6", "k4tri6", "k6"], stream=12 * 8192, batch=4096, inserts_only=False,
                budget=0.01, planted_frac=0.05, planted_size=8),
+    # RoadNetPA-shaped (Table I: 1.09M vertices, 1.54M edges, max degree 9; Fig. 11 motif counting):
+    # a 1044 x 1044 thinned lattice with cell diagonals; all connected 3-, 4- and 5-vertex motifs as standing queries
+    "PA": dict(grid=(1044, 1044, 0.65, 0.12), queries=MOTIFS[3] + MOTIFS[4] + MOTIFS[5], stream=12 * 8192,
+               batch=4096, inserts_only=False, budget=0.10, L=0, idx=6),
 }
 
 
@@ -185,8 +252,10 @@ def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = 
                   batch: int | None = None, n_batches: int | None = None, n_stream: int | None = None) -> Workload:
     """Build G_0 and the batch stream of a config (optionally scaled down for tests)."""
     cfg = dict(CONFIGS[name])
-    idx = int(name[1:])
+    idx = cfg.get("idx", None) or int(name[1:])
     seed = 0x6C53 + idx
+    if "grid" in cfg:
+        return _grid_workload(name, cfg, seed, scale, batch, n_batches, n_stream)
     if scale is not None:
         cfg["scale"] = scale
         if cfg["id_limit"]:
@@ -208,8 +277,7 @@ def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = 
         sign[:] = 1
     ins_mask = np.zeros(len(uv), dtype=bool)
     ins_mask[sel[sign > 0]] = True
-    g0 = uv[~ins_mask]
-    rp, col = csr_from_edges(n, g0)
+    rp, col = csr_from_edges(n, uv, skip=ins_mask)  # G_0 = the generated graph minus the insertion-marked edges
     lab = labels(n, cfg["L"], seed + 2000) if cfg["L"] else None
     B = cfg["batch"]
     nb = n_stream // B
@@ -224,6 +292,32 @@ def make_workload(name: str, *, n_edges: int | None = None, scale: int | None = 
                     batches=batches, budget_frac=cfg["budget"],
                     meta=dict(seed=seed, scale=cfg["scale"], n_edges=cfg["n_edges"], abc=cfg["abc"],
                               id_limit=cfg["id_limit"], L=cfg["L"], batch=B, planted=(groups, ps)))
+
+
+def _grid_workload(name, cfg, seed, scale, batch, n_batches, n_stream) -> Workload:
+    W, H, pk, pd = cfg["grid"]
+    if scale is not None:  # tests: a (2^scale)-vertex lattice of the same shape
+        W = H = max(4, int(round((1 << scale) ** 0.5)))
+    uv = grid_edges(W, H, pk, pd, seed)
+    n = W * H
+    B = batch if batch is not None else cfg["batch"]
+    n_stream = min(n_stream if n_stream is not None else cfg["stream"], len(uv) // 2)
+    sel, sign = stream(len(uv), n_stream, seed + 1000)
+    ins_mask = np.zeros(len(uv), dtype=bool)
+    ins_mask[sel[sign > 0]] = True
+    rp, col = csr_from_edges(n, uv[~ins_mask])
+    nb = n_stream // B
+    if n_batches is not None:
+        nb = min(nb, n_batches)
+    batches = []
+    for t in range(nb):
+        s = sel[t * B:(t + 1) * B]
+        g = sign[t * B:(t + 1) * B]
+        batches.append((np.ascontiguousarray(uv[s[g > 0]]), np.ascontiguousarray(uv[s[g < 0]])))
+    return Workload(name=name, n=n, row_ptr=rp, col=col, labels=None, queries=list(cfg["queries"]),
+                    batches=batches, budget_frac=cfg["budget"],
+                    meta=dict(seed=seed, scale=None, n_edges=len(uv), abc=None, id_limit=0, L=0, batch=B,
+                              planted=(0, 0), grid=(W, H, pk, pd)))
 
 
 def small_random_case(seed: int, n: int = 9, p: float = 0.45, n_ins: int = 4, n_del: int = 4):

@@ -20,6 +20,14 @@
 #include <vector>
 #include <parallel/algorithm>
 #include <omp.h>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+
+static double gi_now() {
+  return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+#define GI_T(label) do { if (std::getenv("GI_TIMING")) std::fprintf(stderr, "[gi] %s %.2f s\n", label, gi_now() - t_start); } while (0)
 
 namespace {
 
@@ -37,30 +45,96 @@ struct Cand {
   int64_t idx;   // generation index (earlier wins)
 };
 
+// Integer thresholds of the R-MAT quadrant test: u01(x) < t  <=>  (x >> 11) < ceil(t * 2^53) (x >> 11 is an
+// integer below 2^53 and the scaling by 2^-53 is exact), so the draws are the same as comparing doubles.
+struct RmatT {
+  uint64_t ta, tab, tabc;
+  uint64_t lvl[64];  // sm64(l + 1): the per-level half of h2(base, l + 1)
+};
+inline uint64_t ceil53(double t) {
+  const double x = t * 9007199254740992.0;
+  const uint64_t f = (uint64_t)x;
+  return (double)f == x ? f : f + 1;
+}
+inline RmatT rmat_thresholds(double a, double b, double c, int scale) {
+  RmatT T;
+  T.ta = ceil53(a);
+  T.tab = ceil53(a + b);
+  T.tabc = ceil53(a + b + c);
+  for (int l = 0; l < scale && l < 64; ++l) T.lvl[l] = sm64((uint64_t)l + 1);
+  return T;
+}
+
 // One R-MAT draw for candidate index j. Returns false for self loops / rejected ids.
-inline bool rmat_one(int scale, double a, double b, double c, uint64_t seed, int64_t j,
-                     int64_t id_limit, uint64_t* key) {
+inline bool rmat_one(int scale, const RmatT& T, uint64_t seed, int64_t j, int64_t id_limit, uint64_t* key) {
   uint64_t u = 0, v = 0;
   const uint64_t base = h2(seed, (uint64_t)j);
   for (int l = 0; l < scale; ++l) {
-    const double r = u01(h2(base, (uint64_t)l + 1));
-    u <<= 1;
-    v <<= 1;
-    if (r < a) {
-    } else if (r < a + b) {
-      v |= 1;
-    } else if (r < a + b + c) {
-      u |= 1;
-    } else {
-      u |= 1;
-      v |= 1;
-    }
+    const uint64_t z = sm64(base ^ T.lvl[l]) >> 11;  // h2(base, l + 1)
+    const uint64_t ge_a = z >= T.ta, ge_ab = z >= T.tab, ge_abc = z >= T.tabc;
+    u = (u << 1) | ge_ab;                          // quadrants c, d
+    v = (v << 1) | ((ge_a & (1 - ge_ab)) | ge_abc);  // quadrants b, d
   }
   if (u == v) return false;
   if (id_limit > 0 && ((int64_t)u >= id_limit || (int64_t)v >= id_limit)) return false;
   if (u > v) std::swap(u, v);
   *key = (u << 32) | v;
   return true;
+}
+
+// Parallel sort of candidates by (key, idx) or by idx: one MSD pass into 2^bits buckets by the top bits of the
+// sort field (counting sort over thread-local histograms), then each bucket sorted on its own.
+template <bool BY_KEY>
+void bucket_sort(std::vector<Cand>& v, int bits, uint64_t maxval) {
+  const int64_t n = (int64_t)v.size();
+  if (n < (1 << 16)) {
+    if (BY_KEY) std::sort(v.begin(), v.end(), [](const Cand& x, const Cand& y) {
+      return x.key < y.key || (x.key == y.key && x.idx < y.idx); });
+    else std::sort(v.begin(), v.end(), [](const Cand& x, const Cand& y) { return x.idx < y.idx; });
+    return;
+  }
+  int shift = 0;
+  while (shift < 64 && (maxval >> shift) >= (1ull << bits)) ++shift;
+  const int nb = 1 << bits;
+  const int nt = omp_get_max_threads();
+  std::vector<int64_t> hist((size_t)nt * nb, 0);
+  auto field = [&](const Cand& c) -> uint64_t { return BY_KEY ? c.key : (uint64_t)c.idx; };
+#pragma omp parallel
+  {
+    const int t = omp_get_thread_num();
+    const int64_t lo = n * t / nt, hi = n * (t + 1) / nt;
+    int64_t* h = &hist[(size_t)t * nb];
+    for (int64_t i = lo; i < hi; ++i) h[field(v[i]) >> shift]++;
+  }
+  std::vector<int64_t> start((size_t)nb + 1, 0);
+  {  // bucket-major, thread-minor exclusive scan (a stable scatter)
+    int64_t run = 0;
+    for (int bkt = 0; bkt < nb; ++bkt) {
+      start[bkt] = run;
+      for (int t = 0; t < nt; ++t) {
+        const int64_t c = hist[(size_t)t * nb + bkt];
+        hist[(size_t)t * nb + bkt] = run;
+        run += c;
+      }
+    }
+    start[nb] = run;
+  }
+  std::vector<Cand> out((size_t)n);
+#pragma omp parallel
+  {
+    const int t = omp_get_thread_num();
+    const int64_t lo = n * t / nt, hi = n * (t + 1) / nt;
+    int64_t* h = &hist[(size_t)t * nb];
+    for (int64_t i = lo; i < hi; ++i) out[(size_t)h[field(v[i]) >> shift]++] = v[i];
+  }
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int bkt = 0; bkt < nb; ++bkt) {
+    auto b0 = out.begin() + start[bkt], b1 = out.begin() + start[bkt + 1];
+    if (BY_KEY) std::sort(b0, b1, [](const Cand& x, const Cand& y) {
+      return x.key < y.key || (x.key == y.key && x.idx < y.idx); });
+    else std::sort(b0, b1, [](const Cand& x, const Cand& y) { return x.idx < y.idx; });
+  }
+  v.swap(out);
 }
 
 }  // namespace
@@ -81,6 +155,8 @@ int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double
                       uint64_t seed, int64_t id_limit, int32_t threads, int32_t* out_uv,
                       int64_t planted_groups, int32_t planted_size) {
   if (threads > 0) omp_set_num_threads(threads);
+  const double t_start = gi_now();
+  const RmatT T = rmat_thresholds(a, b, c, scale);
   const int64_t n_ids = id_limit > 0 ? id_limit : (int64_t(1) << scale);
   if ((double)n_edges > 0.5 * (double)n_ids * (double)(n_ids - 1)) return -1;
   std::vector<Cand> cands;
@@ -111,9 +187,7 @@ int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double
       if (ok[t]) cands[w++] = cands[t];
     cands.resize(w);
     next_j = np;
-    __gnu_parallel::sort(cands.begin(), cands.end(), [](const Cand& x, const Cand& y) {
-      return x.key < y.key || (x.key == y.key && x.idx < y.idx);
-    });
+    bucket_sort<true>(cands, 14, (uint64_t)n_ids << 32);
     size_t o = 0;
     for (size_t i = 0; i < cands.size(); ++i)
       if (o == 0 || cands[i].key != cands[o - 1].key) cands[o++] = cands[i];
@@ -129,7 +203,7 @@ int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double
 #pragma omp parallel for schedule(static)
     for (int64_t t = 0; t < want; ++t) {
       uint64_t key = 0;
-      ok[t] = rmat_one(scale, a, b, c, seed, next_j + t - rmat_base, id_limit, &key);
+      ok[t] = rmat_one(scale, T, seed, next_j + t - rmat_base, id_limit, &key);
       cands[old + t] = Cand{key, next_j + t};
     }
     size_t w = old;
@@ -137,19 +211,19 @@ int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double
       if (ok[t]) cands[w++] = cands[old + t];
     cands.resize(w);
     next_j += want;
-    __gnu_parallel::sort(cands.begin(), cands.end(), [](const Cand& x, const Cand& y) {
-      return x.key < y.key || (x.key == y.key && x.idx < y.idx);
-    });
+    GI_T("draw");
+    bucket_sort<true>(cands, 14, (uint64_t)n_ids << 32);
     size_t o = 0;
     for (size_t i = 0; i < cands.size(); ++i)
       if (o == 0 || cands[i].key != cands[o - 1].key) cands[o++] = cands[i];
     cands.resize(o);
     uniq = (int64_t)o;
+    GI_T("sort+unique");
   }
   // keep the n_edges earliest by generation index, in generation order
-  __gnu_parallel::sort(cands.begin(), cands.end(),
-                       [](const Cand& x, const Cand& y) { return x.idx < y.idx; });
+  bucket_sort<false>(cands, 14, (uint64_t)next_j);
   cands.resize((size_t)n_edges);
+  GI_T("idx sort");
   // seeded permutation of vertex ids (Fisher-Yates, counter-based draws)
   std::vector<int32_t> perm((size_t)n_ids);
   std::iota(perm.begin(), perm.end(), 0);
@@ -170,29 +244,81 @@ int64_t gi_rmat_edges(int32_t scale, int64_t n_edges, double a, double b, double
   return n_edges;
 }
 
-// Symmetric CSR of an undirected simple edge list (u != v, no duplicates):
-// row_ptr[n+1], col[2m], each row sorted ascending.
-int32_t gi_build_csr(int32_t n, int64_t m, const int32_t* uv, int32_t threads, int64_t* row_ptr,
-                     int32_t* col) {
+// Road-network-shaped graph (RoadNetPA / RoadNetCA of Table I; the motif experiment of Fig. 11,
+// every vertex has a small degree): a W x H lattice whose edges are kept with probability p_keep,
+// plus one diagonal per cell with probability p_diag (road junctions close triangles), cells in row-major
+// order, each cell emitting (right, down, diagonal); then the vertex ids are relabelled with a seeded uniform
+// permutation. Writes up to cap pairs (u < v) in generation order; returns the number of edges.
+int64_t gi_grid_edges(int32_t W, int32_t H, double p_keep, double p_diag, uint64_t seed, int32_t* out_uv,
+                      int64_t cap) {
+  const int64_t n = (int64_t)W * H;
+  std::vector<int32_t> perm((size_t)n);
+  std::iota(perm.begin(), perm.end(), 0);
+  const uint64_t pseed = h2(seed, 0x47524944ULL);
+  for (int64_t i = n - 1; i > 0; --i) {
+    const int64_t j = (int64_t)(h2(pseed, (uint64_t)i) % (uint64_t)(i + 1));
+    std::swap(perm[i], perm[j]);
+  }
+  int64_t m = 0;
+  auto emit = [&](int64_t a, int64_t b) {
+    if (m < cap) {
+      int32_t u = perm[(size_t)a], v = perm[(size_t)b];
+      if (u > v) std::swap(u, v);
+      out_uv[2 * m] = u;
+      out_uv[2 * m + 1] = v;
+    }
+    ++m;
+  };
+  for (int64_t y = 0; y < H; ++y)
+    for (int64_t x = 0; x < W; ++x) {
+      const int64_t c = y * W + x;
+      if (x + 1 < W && u01(h2(seed, 3 * (uint64_t)c)) < p_keep) emit(c, c + 1);
+      if (y + 1 < H && u01(h2(seed, 3 * (uint64_t)c + 1)) < p_keep) emit(c, c + W);
+      if (x + 1 < W && y + 1 < H && u01(h2(seed, 3 * (uint64_t)c + 2)) < p_diag) {
+        if (h2(seed ^ 0xD1A6ULL, (uint64_t)c) & 1) emit(c, c + W + 1);
+        else emit(c + 1, c + W);
+      }
+    }
+  return m;
+}
+
+// Symmetric CSR of an undirected simple edge list (u != v, no duplicates): row_ptr[n+1], col[2m'], each row
+// sorted ascending. skip: NULL, or m flags (1 = leave edge e out: the insertion-marked edges of the stream,
+// P:331). Parallel: atomic degree counts and slot claims, then per-row sorts. Returns -1 on a bad edge.
+int32_t gi_build_csr_skip(int32_t n, int64_t m, const int32_t* uv, const uint8_t* skip, int32_t threads,
+                          int64_t* row_ptr, int32_t* col) {
   if (threads > 0) omp_set_num_threads(threads);
   std::vector<int64_t> deg((size_t)n + 1, 0);
+  int bad = 0;
+#pragma omp parallel for schedule(static) reduction(| : bad)
   for (int64_t e = 0; e < m; ++e) {
+    if (skip && skip[e]) continue;
     const int32_t u = uv[2 * e], v = uv[2 * e + 1];
-    if (u < 0 || v < 0 || u >= n || v >= n || u == v) return -1;
-    deg[u]++;
-    deg[v]++;
+    if (u < 0 || v < 0 || u >= n || v >= n || u == v) {
+      bad = 1;
+      continue;
+    }
+    __atomic_fetch_add(&deg[u], 1, __ATOMIC_RELAXED);
+    __atomic_fetch_add(&deg[v], 1, __ATOMIC_RELAXED);
   }
+  if (bad) return -1;
   row_ptr[0] = 0;
   for (int32_t i = 0; i < n; ++i) row_ptr[i + 1] = row_ptr[i] + deg[i];
   std::vector<int64_t> pos(row_ptr, row_ptr + n);
+#pragma omp parallel for schedule(static)
   for (int64_t e = 0; e < m; ++e) {
+    if (skip && skip[e]) continue;
     const int32_t u = uv[2 * e], v = uv[2 * e + 1];
-    col[pos[u]++] = v;
-    col[pos[v]++] = u;
+    col[__atomic_fetch_add(&pos[u], 1, __ATOMIC_RELAXED)] = v;
+    col[__atomic_fetch_add(&pos[v], 1, __ATOMIC_RELAXED)] = u;
   }
 #pragma omp parallel for schedule(dynamic, 4096)
   for (int32_t i = 0; i < n; ++i) std::sort(col + row_ptr[i], col + row_ptr[i + 1]);
   return 0;
+}
+
+int32_t gi_build_csr(int32_t n, int64_t m, const int32_t* uv, int32_t threads, int64_t* row_ptr, int32_t* col) {
+  return gi_build_csr_skip(n, m, uv, nullptr, threads, row_ptr, col);
 }
 
 // Labels uniform over [0, L).

@@ -88,6 +88,9 @@ typedef struct {
   uint64_t walks_override; /* 0 = M = |ΔE| D^(k-2) / 32^k (R21) */
   uint32_t flags;          /* GCSM_FLAG_* */
   uint32_t reserved;
+  uint64_t staging_bytes;  /* per-GPU HBM arena of the fetch-once staging of zero-copy lists within a batch
+                              (not a cache: emptied every batch): 0 = default (a quarter of the
+                              free HBM when first needed, at most 16 GiB), 1 = off */
 } gcsm_options;
 
 /* Per-batch statistics (Table II-style breakdown; hit rate §8d). */
@@ -124,6 +127,13 @@ typedef struct {
   double ms_allreduce;      /* (4b) */
   double ms_merge;          /* (5) */
   double ms_total;          /* whole gcsm_apply_batch, host wall clock */
+  uint64_t stage_fill_bytes; /* bytes copied host -> the batch's staging arena (fetch-once staging; each list at
+                                most once per batch; included in host_copied_bytes) */
+  uint64_t stage_lists;      /* lists staged */
+  uint64_t stage_hit_bytes;  /* algorithmic list bytes then served from the arena (HBM) instead of zero-copy */
+  uint64_t bcomp_hit_bytes, bcomp_miss_bytes, bcomp_delta_bytes; /* B_comp: bytes of the DISTINCT
+                                main lists the query's kernels touched, by home (HBM cache / pinned host / uploaded
+                                lists of U); only with GCSM_BCOMP=1 at create (measurement mode), else 0 */
 } gcsm_stats;
 
 /* Fills *opt with the defaults (device -1, world 1, seed 0x6C53, all cores,
@@ -150,7 +160,7 @@ gcsm_status gcsm_set_query(gcsm_ctx *ctx, int32_t k, int32_t m, const int32_t *q
                            const int32_t *order);
 
 /* Adds another standing query to the context (gcsm_set_query replaces all of them with one). Arguments as
- * gcsm_set_query; *qid (may be NULL) receives its index (query 0 is the set_query one). Up to 8 queries. The
+ * gcsm_set_query; *qid (may be NULL) receives its index (query 0 is the set_query one). Up to 32 queries. The
  * queries share the host store, each batch's normalisation, overlays and merge (steps (1) and (5) of Fig. 3)
  * and ONE device cache under the per-GPU budget, filled by ranking vertices on the SUM of the queries'
  * estimated access frequencies (eq. (3) per query; P:339's top-K rule on the sum). Every query gets
@@ -211,6 +221,15 @@ uint64_t gcsm_query_automorphisms(const gcsm_ctx *ctx);
 /* Static-lifetime (per ctx) message for the last error; "" if none. */
 const char *gcsm_last_error(const gcsm_ctx *ctx);
 
+/* Measurement modes for the following batches (flags = GCSM_MEASURE_*; 0 = off, the default). With
+ * GCSM_MEASURE_BCOMP the kernels also mark, per query, the vertices whose main list they read, and the batch's
+ * statistics report B_comp (bytes of the DISTINCT lists touched, by home: HBM cache, pinned host,
+ * uploaded lists of U) in bcomp_*_bytes; it costs one atomic per list read and serialises each batch's
+ * kernels on the context stream, so timed runs leave it off. EINVAL for unknown flags, ENOMEM if the bitmap
+ * (n bits) cannot be allocated. Also enabled at create by the environment variable GCSM_BCOMP=1. */
+enum { GCSM_MEASURE_BCOMP = 1u };
+gcsm_status gcsm_set_measure(gcsm_ctx *ctx, uint32_t flags);
+
 /* Frees everything (pinned store, device buffers, stream, communicator). NULL-safe. */
 void gcsm_destroy(gcsm_ctx *ctx);
 
@@ -261,6 +280,12 @@ gcsm_status gcsm_plan_inspect(int32_t k, int32_t m, const int32_t *qedges, const
 gcsm_status gcsm_query_restrictions(int32_t k, int32_t m, const int32_t *qedges, const int32_t *qlabels,
                                     const int32_t *order, int32_t *out_pairs, int32_t cap, int32_t *n_out,
                                     uint64_t *aut);
+
+/* Pure host, no device: the estimator's binomial sampler (§IV-B: B ~ Bin(n, p)), as the walks draw it:
+ * out[i] = Bin(n, p) drawn from the counter-based key chain(key0, i) (reading R22; BINV for n p < 10, BTRD
+ * otherwise, R20). For the distribution tests of the product's sampler (chi-square against the exact pmf).
+ * count >= 0, n >= 0, 0 <= p <= 1, else EINVAL. */
+gcsm_status gcsm_binomial_samples(uint64_t key0, int64_t n, double p, int64_t count, int64_t *out);
 
 /* Pure host, no device: the shard of each unit for world ranks (LPT on the
  * cost proxy cost[i], ties by index): out_rank[n_units]. */

@@ -16,8 +16,9 @@ Functions (pins in tests/test_oracle_*.py):
   static_count     O2  |Emb(Q, G)|                             (pinned: K_n / stars / K_ab closed forms)
   ivm_count        a5  eq. (1) terms with stable split (R7)    (pinned: equals delta on fuzz cases)
   access_counts    a3  exact C_v of the execution trees        (pinned: brute-force tree walk in Python)
-  estimate         a3  merged random walks, eq. (3), §IV-B     (pinned: eq. (6) unbiasedness, eq. (7) variance,
-                                                                 P:339 ">= |ΔE|" property, binomial chi-square)
+  estimate         a3  M plain random walks of §IV-A, eq. (3) (pinned: eq. (6) unbiasedness vs the exact C_v,
+                                                                 eq. (7) variance bound, ">= |ΔE|" property,
+                                                                 a one-unit closed form of the walk distribution)
   select_cache     a4  top-K prefix under a byte budget (R23)  (pinned: brute-force prefix search)
 """
 from __future__ import annotations
@@ -59,12 +60,10 @@ def _load():
         lib.ivm_units.restype = I64
         lib.ivm_units.argtypes = [I32, I32, P, P, P, P, I64, P, I64, P, P, I64]
         lib.ivm_run.restype = ctypes.c_int
-        lib.ivm_run.argtypes = [I32, I32, P, P, P, P, P, P, P, I32, I32, P, P, P, I64, P, I32, U64, U64, I64, I64,
+        lib.ivm_run.argtypes = [I32, I32, P, P, P, P, P, P, P, I32, I32, P, P, P, I64, P, I32, U64, I64, I64,
                                 P, P, P]
         lib.o_apply.restype = ctypes.c_int
         lib.o_apply.argtypes = [I32, P, P, I64, P, I64, P, P, P]
-        lib.o_binom_many.restype = None
-        lib.o_binom_many.argtypes = [U64, I64, ctypes.c_double, I64, P]
         _lib = lib
     return _lib
 
@@ -264,7 +263,7 @@ class _Views:
 
 
 def _ivm(mode, n, rp, col, labels, k, qe, ql, ins, dele, user_order=None, unit_filter=None, threads=None,
-         seed=0, batch_seq=0, M=None, D=None):
+         seed=0, M=None, D=None):
     I, Dl, _ = normalize_batch(n, rp, col, ins, dele)
     V = _Views(n, rp, col, I, Dl)
     U = units(k, qe, ql, labels, I, Dl, user_order)
@@ -280,7 +279,7 @@ def _ivm(mode, n, rp, col, labels, k, qe, ql, ins, dele, user_order=None, unit_f
         M = walks(len(U), Dv, k)
     r = _load().ivm_run(mode, n, _p(V.stable[0]), _p(V.stable[1]), _p(V.old[0]), _p(V.old[1]), _p(V.new[0]),
                         _p(V.new[1]), _p(labels), k, len(qe), _p(qe), _p(ql), _p(uo), len(U), _p(U),
-                        _threads(threads), seed & (2**64 - 1), batch_seq, int(M), Dv, _p(out), _p(access), _p(lev))
+                        _threads(threads), seed & (2**64 - 1), int(M), Dv, _p(out), _p(access), _p(lev))
     if r:
         raise ValueError("bad query")
     return dict(added=_u128(out[0], out[1]), removed=_u128(out[2], out[3]), access=access,
@@ -305,14 +304,19 @@ def walks(N1: int, D: int, k: int) -> int:
     return int(min(max((N1 * D ** max(k - 2, 0)) // 32 ** k, 1), 2 ** 62))
 
 
-def estimate(n, rp, col, labels, k, qe, ql, ins, dele, seed, batch_seq=0, user_order=None, M=None, threads=None,
+def estimate(n, rp, col, labels, k, qe, ql, ins, dele, seed, M=None, user_order=None, threads=None,
              unit_filter=None):
-    """Merged random walks (§IV-B) with the counter RNG of R22.
+    """Access-frequency estimate by M plain random walks (§IV-A), one walk at a time.
 
-    Returns dict(levcnt=[n, k-2] per-level sums of B, N1, D, M, est=[n] float64)
-    where est_v = (1/M) Σ_l N1 D^(l-1) levcnt[v, l-1]  (eq. (3)).
+    A walk picks one level-1 unit (term, sign, oriented changed edge; R15/R16) with probability 1/|ΔE|
+    (|ΔE| = N1), records the lists its node accesses (R17), computes the candidate set V of the next position,
+    picks one element with probability 1/|V| and continues with probability |V|/D (D of R19). Drawn from the
+    oracle's own PCG32 streams (one per walk index, `seed`), never the product's generator.
+
+    Returns dict(levcnt=[n, k-2] number of walks whose level-l node read v's list, N1, D, M,
+    est=[n] float64) where est_v = (1/M) Σ_l |ΔE| D^(l-1) levcnt[v, l-1]  (eq. (3), averaged over M).
     """
-    r = _ivm(2, n, rp, col, labels, k, qe, ql, ins, dele, user_order, unit_filter, threads, seed, batch_seq, M)
+    r = _ivm(2, n, rp, col, labels, k, qe, ql, ins, dele, user_order, unit_filter, threads, seed, M)
     lev = r["levcnt"].astype(np.float64)
     est = np.zeros(n)
     if k > 2:
@@ -323,18 +327,26 @@ def estimate(n, rp, col, labels, k, qe, ql, ins, dele, seed, batch_seq=0, user_o
     return r
 
 
-def binom_samples(key0: int, n: int, p: float, count: int) -> np.ndarray:
-    out = np.zeros(count, np.int64)
-    _load().o_binom_many(key0 & (2**64 - 1), n, p, count, _p(out))
-    return out
+def estimate_from_levels(levcnt, k, N1, D, M):
+    """eq. (3) averaged over M for per-level sums (rows of any estimator's output): Σ_l N1 D^(l-1) lev[:, l-1] / M."""
+    lev = np.asarray(levcnt, dtype=np.float64)
+    est = np.zeros(lev.shape[0])
+    for l in range(1, k - 1):
+        est += float(N1) * float(D) ** (l - 1) * lev[:, l - 1]
+    return est / float(M)
 
 
 # ------------------------------------------------------------------ cache selection
 
-def select_cache(score, list_bytes, budget):
+def select_cache(score, list_bytes, budget, exclude=None):
     """a4 (P:339, reading R23): order vertices with score > 0 by (score desc, id asc);
-    keep the longest prefix whose list bytes fit the budget. Returns sorted ids."""
-    ids = [v for v in range(len(score)) if score[v] > 0]
+    keep the longest prefix whose list bytes fit the budget. Returns sorted ids.
+
+    exclude: vertices that take no part in the ranking. Reading R32: on the GPU path the stable lists of the
+    batch's updated vertices U travel with the batch into HBM, so they compete for no budget; pass U there.
+    The paper's own rule ranks every vertex (exclude=None)."""
+    ex = set() if exclude is None else {int(v) for v in np.asarray(exclude).ravel()}
+    ids = [v for v in range(len(score)) if score[v] > 0 and v not in ex]
     ids.sort(key=lambda v: (-score[v], v))
     used, keep = 0, []
     for v in ids:

@@ -20,9 +20,13 @@
  *                DESIGN.md reading R7; used for
  *                  * its counts (must equal o3_delta: pins reading R7),
  *                  * exact per-vertex access counts C_v (Fig. 15),
- *                  * the merged random walks of §IV-B, eq. (3)
- *                    (P:204), with the counter-based RNG of reading R22 and
- *                    binomial sampling (BINV / BTRD, Hörmann 1993).
+ *                  * M plain random walks of §IV-A, one at a
+ *                    time, exactly as the paper states them (pick a unit
+ *                    with probability 1/|ΔE|, a child with 1/|V|, continue
+ *                    with |V|/D), drawn from the oracle's own PCG32 streams;
+ *                    eq. (3) weighs what they record. The paper's
+ *                    merged form (§IV-B, binomial multiplicities) is the
+ *                    product's business and is NOT reproduced here.
  *
  * Match semantics (readings R1-R5): non-induced, injective,
  * vertex-labelled embeddings of an undirected simple query graph.
@@ -464,124 +468,15 @@ int ivm_plan(int32_t k, int32_t m, const int32_t *qe, const int32_t *user_order,
   return 0;
 }
 
-/* ---------------------------------------------------------- counter-based RNG */
-/* DESIGN.md reading R22: splitmix64 finaliser, keys chained per tree node. */
-static uint64_t o_mix(uint64_t z) {
-  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
-  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
-  return z ^ (z >> 31);
-}
-static uint64_t o_chain(uint64_t h, uint64_t x) { return o_mix(h + 0x9E3779B97F4A7C15ULL * (x + 1)); }
-
-typedef struct { uint64_t key; uint64_t j; } ostream_t;
-static double o_unif(ostream_t *s) {
-  s->j += 1;
-  return (double)(o_mix(s->key + 0xD1B54A32D192ED03ULL * s->j) >> 11) * (1.0 / 9007199254740992.0);
-}
-
-/* Stirling-series correction fc(k) = ln k! - [(k+1/2) ln(k+1) - (k+1) + ln(2 pi)/2] */
-static double o_fc(int64_t k) {
-  if (k < 10) {
-    double kk = (double)k;
-    return lgamma(kk + 1.0) - ((kk + 0.5) * log(kk + 1.0) - (kk + 1.0) + 0.5 * log(2.0 * M_PI));
-  }
-  double r = 1.0 / (double)(k + 1), r2 = r * r;
-  return (1.0 / 12.0 - (1.0 / 360.0 - (1.0 / 1260.0) * r2) * r2) * r;
-}
-
-/* Bin(n, p), p <= 1/2: inversion (BINV) when n p < 10, else BTRD (Hörmann 1993). */
-static int64_t o_binom_half(ostream_t *s, int64_t n, double p) {
-  if (n <= 0 || p <= 0.0) return 0;
-  const double q = 1.0 - p;
-  if ((double)n * p < 10.0) {
-    const double sr = p / q, a = (double)(n + 1) * sr;
-    const double r0 = pow(q, (double)n);
-    for (;;) {
-      double r = r0, u = o_unif(s);
-      int64_t x = 0;
-      while (u > r) {
-        u -= r;
-        x += 1;
-        if (x > n) break;
-        r *= (a / (double)x - sr);
-      }
-      if (x <= n) return x;
-    }
-  }
-  const double m = floor((double)(n + 1) * p);
-  const double r = p / q, nr = (double)(n + 1) * r, npq = (double)n * p * q;
-  const double spq = sqrt(npq);
-  const double b = 1.15 + 2.53 * spq;
-  const double a = -0.0873 + 0.0248 * b + 0.01 * p;
-  const double c = (double)n * p + 0.5;
-  const double alpha = (2.83 + 5.1 / b) * spq;
-  const double vr = 0.92 - 4.2 / b;
-  const double urvr = 0.86 * vr;
-  for (;;) {
-    double v = o_unif(s), u;
-    if (v <= urvr) {
-      u = v / vr - 0.43;
-      return (int64_t)floor((2.0 * a / (0.5 - fabs(u)) + b) * u + c);
-    }
-    if (v >= vr) {
-      u = o_unif(s) - 0.5;
-    } else {
-      u = v / vr - 0.93;
-      u = (u < 0 ? -0.5 : 0.5) - u;
-      v = o_unif(s) * vr;
-    }
-    const double us = 0.5 - fabs(u);
-    const double kd = floor((2.0 * a / us + b) * u + c);
-    if (kd < 0.0 || kd > (double)n) continue;
-    const int64_t kk = (int64_t)kd, mm = (int64_t)m;
-    v = v * alpha / (a / (us * us) + b);
-    const int64_t km = kk > mm ? kk - mm : mm - kk;
-    if (km <= 15) {
-      double f = 1.0;
-      if (mm < kk) {
-        for (int64_t i = mm + 1; i <= kk; ++i) f *= (nr / (double)i - r);
-      } else if (mm > kk) {
-        for (int64_t i = kk + 1; i <= mm; ++i) v *= (nr / (double)i - r);
-      }
-      if (v <= f) return kk;
-      continue;
-    }
-    v = log(v);
-    const double kmd = (double)km;
-    const double rho = (kmd / npq) * (((kmd / 3.0 + 0.625) * kmd + 1.0 / 6.0) / npq + 0.5);
-    const double t = -kmd * kmd / (2.0 * npq);
-    if (v < t - rho) return kk;
-    if (v > t + rho) continue;
-    const double nm = (double)(n - mm + 1);
-    const double h = (m + 0.5) * log((m + 1.0) / (r * nm)) + o_fc(mm) + o_fc(n - mm);
-    const double nk = (double)(n - kk + 1);
-    if (v <= h + (double)(n + 1) * log(nm / nk) + (kd + 0.5) * log(nk * r / (kd + 1.0)) - o_fc(kk) - o_fc(n - kk))
-      return kk;
-  }
-}
-
-static int64_t o_binom(uint64_t key, int64_t n, double p) {
-  ostream_t s = {key, 0};
-  if (n <= 0 || p <= 0.0) return 0;
-  if (p >= 1.0) return n;
-  if (p > 0.5) return n - o_binom_half(&s, n, 1.0 - p);
-  return o_binom_half(&s, n, p);
-}
-
-/* Exported for the distribution pin (tests compare against scipy's pmf). */
-void o_binom_many(uint64_t key0, int64_t n, double p, int64_t count, int64_t *out) {
-  for (int64_t i = 0; i < count; ++i) out[i] = o_binom(o_chain(key0, (uint64_t)i), n, p);
-}
-
 /* ---------------------------------------------------------- the nested loops */
 typedef struct {
   const ograph *g[3]; /* indexed by view: STABLE, OLD, NEW */
   const int32_t *lab;
   const oquery *q;
   oterm terms[OMAXM];
-  int mode; /* 0 count, 1 access, 2 estimate */
-  /* estimate */
-  uint64_t seed, batch_seq;
+  int mode; /* 0 count, 1 access, 2 plain random walks */
+  /* walks */
+  uint64_t seed;
   int64_t M, N1, D;
   /* outputs (shared; atomics) */
   uint64_t *access;  /* n (mode 1) */
@@ -622,7 +517,7 @@ static int64_t ivm_candidates(ivm_state *s, int p, int32_t *out) {
   return n;
 }
 
-static void ivm_visit(ivm_state *s, int level, int64_t B, uint64_t key) {
+static void ivm_visit(ivm_state *s, int level) {
   /* node at `level` has positions 0..level matched; it computes position level+1 */
   const int k = s->c->q->k;
   if (level >= k - 1) { s->count += 1; return; } /* leaf: a complete embedding */
@@ -630,25 +525,83 @@ static void ivm_visit(ivm_state *s, int level, int64_t B, uint64_t key) {
   const oterm *t = s->t;
   if (s->c->mode == 1)
     for (int b = 0; b < t->nb[p]; ++b) __atomic_fetch_add(&s->c->access[s->f[t->bq[p][b]]], 1, __ATOMIC_RELAXED);
-  if (s->c->mode == 2) {
-    for (int b = 0; b < t->nb[p]; ++b)
-      __atomic_fetch_add(&s->c->levcnt[(int64_t)s->f[t->bq[p][b]] * (k - 2) + (level - 1)], (uint64_t)B,
-                         __ATOMIC_RELAXED);
-    if (level == k - 2) return; /* children are leaves: they access nothing */
-  }
   int32_t *cand = (int32_t *)malloc(sizeof(int32_t) * (size_t)(s->c->D + 1));
   const int64_t nc = ivm_candidates(s, p, cand);
   for (int64_t i = 0; i < nc; ++i) {
     s->f[p] = cand[i];
-    if (s->c->mode == 2) {
-      const uint64_t ck = o_chain(key, (uint64_t)(uint32_t)cand[i]);
-      const int64_t Bc = o_binom(ck, B, 1.0 / (double)s->c->D);
-      if (Bc > 0) ivm_visit(s, level + 1, Bc, ck);
-    } else {
-      ivm_visit(s, level + 1, 0, 0);
-    }
+    ivm_visit(s, level + 1);
   }
   free(cand);
+}
+
+/* ---------------------------------------------------------- plain random walks (§IV-A) */
+/* The oracle's own generator: PCG32 (O'Neill 2014, XSH-RR 64/32), one stream per walk index, so the result is
+ * the same for any thread count. The paper fixes no RNG; this one shares nothing with the product's. */
+typedef struct { uint64_t state, inc; } opcg;
+static uint32_t opcg_next(opcg *r) {
+  const uint64_t old = r->state;
+  r->state = old * 6364136223846793005ULL + r->inc;
+  const uint32_t xs = (uint32_t)(((old >> 18) ^ old) >> 27), rot = (uint32_t)(old >> 59);
+  return (xs >> rot) | (xs << ((32u - rot) & 31u));
+}
+static void opcg_seed(opcg *r, uint64_t initstate, uint64_t stream) {
+  r->state = 0;
+  r->inc = (stream << 1) | 1u;
+  opcg_next(r);
+  r->state += initstate;
+  opcg_next(r);
+}
+/* uniform integer in [0, n), n >= 1, by rejection of the top partial block of 2^64 */
+static uint64_t opcg_below(opcg *r, uint64_t n) {
+  const uint64_t lim = UINT64_MAX - UINT64_MAX % n;
+  for (;;) {
+    const uint64_t x = ((uint64_t)opcg_next(r) << 32) | opcg_next(r);
+    if (x < lim) return x % n;
+  }
+}
+
+/* One random walk of §IV-A: "randomly select one edge from ΔE, with a probability of 1/|ΔE|" (here one level-1
+ * unit of the forest of all terms, R15/R16); "compute the set of matching vertices V for the next pattern
+ * vertex", "randomly select one vertex from V, with a probability of 1/|V|", then "continue the walk with a
+ * probability of |V|/D". Each node on the path records the lists it accesses (R17: the backward lists of the
+ * next position; leaves access nothing): levcnt[v][l-1] counts the walk's level-l node reading v's list, and
+ * eq. (3) weighs it by |ΔE| D^(l-1) (done in Python). */
+static void ow_walk(const ivm_ctx *c, int64_t w, int32_t *cand) {
+  opcg r;
+  opcg_seed(&r, c->seed, (uint64_t)w);
+  const int k = c->q->k;
+  const int32_t *un = c->units + 4 * (int64_t)opcg_below(&r, (uint64_t)c->N1);
+  ivm_state s;
+  memset(&s, 0, sizeof s);
+  s.c = c;
+  s.t = &c->terms[un[0]];
+  s.kind = un[1];
+  s.f[0] = un[2];
+  s.f[1] = un[3];
+  for (int level = 1; level <= k - 2; ++level) {
+    const int p = level + 1;
+    for (int b = 0; b < s.t->nb[p]; ++b)
+      __atomic_fetch_add(&c->levcnt[(int64_t)s.f[s.t->bq[p][b]] * (k - 2) + (level - 1)], 1, __ATOMIC_RELAXED);
+    if (level == k - 2) break; /* the next node is a leaf: it accesses nothing */
+    const int64_t nv = ivm_candidates(&s, p, cand);
+    if (nv == 0) break;
+    s.f[p] = cand[opcg_below(&r, (uint64_t)nv)];
+    if (opcg_below(&r, (uint64_t)c->D) >= (uint64_t)nv) break; /* continue with probability |V|/D */
+  }
+}
+
+typedef struct {
+  pool_t *pool;
+  const ivm_ctx *c;
+} ow_arg;
+
+static void *ow_worker(void *vp) {
+  ow_arg *a = (ow_arg *)vp;
+  int32_t *cand = (int32_t *)malloc(sizeof(int32_t) * (size_t)(a->c->D + 1));
+  for (int64_t ch; (ch = pool_take(a->pool)) >= 0;)
+    for (int64_t w = ch * 256; w < a->c->M && w < (ch + 1) * 256; ++w) ow_walk(a->c, w, cand);
+  free(cand);
+  return NULL;
 }
 
 typedef struct {
@@ -669,15 +622,7 @@ static void *ivm_worker(void *vp) {
     s.kind = un[1];
     s.f[0] = un[2];
     s.f[1] = un[3];
-    int64_t B = 0;
-    uint64_t key = 0;
-    if (c->mode == 2) {
-      key = o_chain(o_chain(o_chain(o_chain(o_chain(o_mix(c->seed), c->batch_seq), (uint64_t)un[0]),
-                                        (uint64_t)un[1]), (uint64_t)(uint32_t)un[2]), (uint64_t)(uint32_t)un[3]);
-      B = o_binom(key, c->M, 1.0 / (double)c->N1);
-      if (B == 0) continue;
-    }
-    ivm_visit(&s, 1, B, key);
+    ivm_visit(&s, 1);
     if (un[1] == 0) a->added += s.count;
     else a->removed += s.count;
   }
@@ -721,13 +666,13 @@ int64_t ivm_units(int32_t k, int32_t m, const int32_t *qe, const int32_t *ql, co
  * (STABLE = E∩E', OLD = E, NEW = E'), each a CSR over the same n.
  * mode 0: out_counts[0..3] = added lo/hi, removed lo/hi.
  * mode 1: access[n] += number of tree nodes (levels 1..k-2) reading v's list.
- * mode 2: merged random walks; levcnt[n*(k-2)] += sum of B over nodes at
- *         level l (1..k-2) reading v's list; M walks, N1 = n_units, D.
+ * mode 2: M plain random walks (ow_walk, seeded by `seed`); levcnt[n*(k-2)] += number of walks whose level-l
+ *         node (1..k-2) reads v's list; N1 = n_units, D.
  */
 int ivm_run(int32_t mode, int32_t n, const int64_t *rp_s, const int32_t *col_s, const int64_t *rp_o,
             const int32_t *col_o, const int64_t *rp_n, const int32_t *col_n, const int32_t *lab, int32_t k, int32_t m,
             const int32_t *qe, const int32_t *ql, const int32_t *user_order, int64_t n_units, const int32_t *units,
-            int32_t threads, uint64_t seed, uint64_t batch_seq, int64_t M, int64_t D, uint64_t *out_counts,
+            int32_t threads, uint64_t seed, int64_t M, int64_t D, uint64_t *out_counts,
             uint64_t *access, uint64_t *levcnt) {
   oquery q;
   if (query_init(&q, k, m, qe, ql)) return -1;
@@ -735,7 +680,7 @@ int ivm_run(int32_t mode, int32_t n, const int64_t *rp_s, const int32_t *col_s, 
   ivm_ctx *c = (ivm_ctx *)calloc(1, sizeof(ivm_ctx));
   c->g[V_STABLE] = &gs; c->g[V_OLD] = &go; c->g[V_NEW] = &gn;
   c->lab = lab; c->q = &q; c->mode = mode;
-  c->seed = seed; c->batch_seq = batch_seq; c->M = M; c->N1 = n_units; c->D = D;
+  c->seed = seed; c->M = M; c->N1 = n_units; c->D = D;
   c->access = access; c->levcnt = levcnt; c->n_units = n_units; c->units = units;
   int uo[OMAXK], num[OMAXM][2], eidx[OMAXM];
   for (int i = 0; i < k; ++i) uo[i] = user_order ? user_order[i] : i;
@@ -749,10 +694,19 @@ int ivm_run(int32_t mode, int32_t n, const int64_t *rp_s, const int32_t *col_s, 
     }
     c->D = d;
   }
-  pool_t pool = {n_units, 0, PTHREAD_MUTEX_INITIALIZER, NULL};
   if (threads < 1) threads = 1;
-  ivm_arg *args = (ivm_arg *)calloc((size_t)threads, sizeof(ivm_arg));
   void *ptrs[256];
+  if (mode == 2) {
+    pool_t wpool = {(M + 255) / 256, 0, PTHREAD_MUTEX_INITIALIZER, NULL};
+    ow_arg wargs[256];
+    if (n_units > 0 && k > 2)
+      for (int t = 0; t < threads && t < 256; ++t) { wargs[t] = (ow_arg){&wpool, c}; ptrs[t] = &wargs[t]; }
+    if (n_units > 0 && k > 2) run_threads(threads, ow_worker, ptrs);
+    free(c);
+    return 0;
+  }
+  pool_t pool = {n_units, 0, PTHREAD_MUTEX_INITIALIZER, NULL};
+  ivm_arg *args = (ivm_arg *)calloc((size_t)threads, sizeof(ivm_arg));
   for (int t = 0; t < threads && t < 256; ++t) { args[t] = (ivm_arg){&pool, c, 0, 0}; ptrs[t] = &args[t]; }
   run_threads(threads, ivm_worker, ptrs);
   u128 ad = 0, rm = 0;

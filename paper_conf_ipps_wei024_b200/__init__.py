@@ -57,7 +57,8 @@ class Gcsm:
     """One GCSM context (one GPU, one process). See include/gcsm.h for the semantics."""
 
     def __init__(self, n, row_ptr, col, labels=None, *, device=-1, rank=0, world=1, nccl_id=None, seed=0x6C53,
-                 host_threads=0, cache_policy="estimator", walks_override=0, local_counts=False, symmetry=True):
+                 host_threads=0, cache_policy="estimator", walks_override=0, local_counts=False, symmetry=True,
+                 staging_bytes=0):
         lib = _lib.load()
         self._lib = lib
         opt = Options()
@@ -71,6 +72,7 @@ class Gcsm:
         opt.host_threads = host_threads
         opt.cache_policy = CACHE_POLICIES[cache_policy] if isinstance(cache_policy, str) else int(cache_policy)
         opt.walks_override = walks_override
+        opt.staging_bytes = int(staging_bytes)
         opt.flags = (FLAG_LOCAL_COUNTS if local_counts else 0) | (0 if symmetry else FLAG_NO_SYMMETRY)
         self.n = int(n)
         self._rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
@@ -114,6 +116,10 @@ class Gcsm:
     def query_counts(self, qid: int):
         st = self.query_stats(qid)
         return st["added"], st["removed"]
+
+    def set_measure(self, bcomp: bool):
+        """Measurement mode (gcsm_set_measure): B_comp of the following batches in stats()['bcomp_*_bytes']."""
+        self._check(self._lib.gcsm_set_measure(self._h, 1 if bcomp else 0), "set_measure")
 
     def set_cache_budget(self, nbytes: int):
         self._check(self._lib.gcsm_set_cache_budget(self._h, int(nbytes)), "set_cache_budget")
@@ -235,6 +241,15 @@ def shard(cost, world):
     s = _lib.load().gcsm_shard(len(c), _ptr(c), int(world), _ptr(out))
     if s:
         raise GcsmError(s, "bad shard arguments")
+    return out
+
+
+def binomial_samples(key0, n, p, count):
+    """The estimator's host binomial sampler (gcsm_binomial_samples): count draws of Bin(n, p)."""
+    out = np.zeros(int(count), np.int64)
+    s = _lib.load().gcsm_binomial_samples(int(key0) & (2**64 - 1), int(n), float(p), int(count), _ptr(out))
+    if s:
+        raise GcsmError(s, "gcsm_binomial_samples")
     return out
 
 

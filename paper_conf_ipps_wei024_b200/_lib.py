@@ -21,14 +21,14 @@ SYMBOLS = ["gcsm_default_options", "gcsm_create", "gcsm_set_query", "gcsm_set_ca
            "gcsm_get_query_stats", "gcsm_query_automorphisms", "gcsm_last_error", "gcsm_destroy",
            "gcsm_nccl_unique_id", "gcsm_get_stream", "gcsm_export_csr", "gcsm_get_estimates", "gcsm_get_cached",
            "gcsm_plan_inspect", "gcsm_query_restrictions", "gcsm_shard",
-           "gcsm_measure_host_link"]
+           "gcsm_measure_host_link", "gcsm_binomial_samples", "gcsm_set_measure"]
 
 
 class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("nccl_id", ctypes.c_void_p), ("seed", ctypes.c_uint64), ("host_threads", ctypes.c_int32),
                 ("cache_policy", ctypes.c_int32), ("walks_override", ctypes.c_uint64), ("flags", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32)]
+                ("reserved", ctypes.c_uint32), ("staging_bytes", ctypes.c_uint64)]
 
 
 class Stats(ctypes.Structure):
@@ -38,7 +38,10 @@ class Stats(ctypes.Structure):
                  "delta_bytes_ext", "host_copied_bytes", "frontier", "kernel_launches", "h2d_bytes", "d2h_bytes", "added", "removed"]] + \
               [(name, ctypes.c_double) for name in
                ["ms_normalize", "ms_estimate", "ms_pack", "ms_copy", "ms_match", "ms_level2", "ms_extend",
-                "ms_allreduce", "ms_merge", "ms_total"]]
+                "ms_allreduce", "ms_merge", "ms_total"]] + \
+              [(name, ctypes.c_uint64) for name in
+               ["stage_fill_bytes", "stage_lists", "stage_hit_bytes", "bcomp_hit_bytes", "bcomp_miss_bytes",
+                "bcomp_delta_bytes"]]
 
 
 _lib = None
@@ -77,6 +80,8 @@ def load():
         "gcsm_get_cached": (st, [P, P, U64, ctypes.POINTER(U64)]),
         "gcsm_plan_inspect": (st, [I32, I32, P, P, P, P, P, P, P]),
         "gcsm_shard": (st, [I64, P, I32, P]),
+        "gcsm_binomial_samples": (st, [U64, I64, ctypes.c_double, I64, P]),
+        "gcsm_set_measure": (st, [P, ctypes.c_uint32]),
         "gcsm_query_restrictions": (st, [I32, I32, P, P, P, P, I32, P, ctypes.POINTER(U64)]),
         "gcsm_measure_host_link": (st, [I32, U64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double),
                                         ctypes.POINTER(ctypes.c_double)]),

@@ -150,6 +150,7 @@ struct gcsm_ctx {
   // copy) runs here while batch t's extension kernels run on `stream` (GCSM_NO_OVERLAP=1 at create: on `stream`)
   cudaStream_t stream3 = nullptr;
   bool overlap = false;
+  int overlap_kmax = 5;  // largest query size whose batches overlap the cache step (GCSM_OVERLAP_KMAX)
   uint32_t *d_hist = nullptr;                         // n counters + scan
   uint32_t *d_bsum = nullptr;
   int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
@@ -182,7 +183,7 @@ struct gcsm_ctx {
   SelState *d_sel = nullptr;
   void *d_cubtmp = nullptr; size_t cubtmp_bytes = 0;
   unsigned long long *d_levcnt[GCSM_MAX_QUERIES] = {};
-  int lev_levels[GCSM_MAX_QUERIES] = {-1, -1, -1, -1, -1, -1, -1, -1};
+  int lev_levels[GCSM_MAX_QUERIES];  // -1 until allocated (set in gcsm_create)
   EstUnit *d_eunits = nullptr; size_t eunits_cap = 0;
   int2 *d_eitems = nullptr; size_t eitems_cap = 0;
   EstNode2 *d_ef2 = nullptr; size_t ef2_cap = 0;
@@ -199,6 +200,17 @@ struct gcsm_ctx {
   size_t r0_n = 0;                 // entries of the device table of (1 - pD)^n
   double r0_pD = -1.0;
   bool est_valid = false;          // the device holds a batch's estimator output (gcsm_get_estimates)
+  // fetch-once staging of zero-copy lists within a batch (kernels.cu stage_resolve): per-vertex
+  // state words, the arena (emptied every batch: a new epoch) and its bump counter
+  unsigned long long *d_stage_state = nullptr;
+  int32_t *d_stage_arena = nullptr;
+  size_t stage_cap = 0;            // ints
+  unsigned long long *d_stage_bump = nullptr;
+  bool stage_failed = false;       // allocation failed once: stay off
+  uint32_t stage_min = 1;          // shortest list (ints) routed through the arena (GCSM_STAGE_MIN)
+  // B_comp measurement mode (GCSM_BCOMP=1 at create): bitmap of the vertices whose main list a query's kernels read
+  uint32_t *d_touched_bc = nullptr;
+  bool bcomp = false;
   std::vector<void *> retired_pinned;  // pinned staging replaced by a larger one (freed at destroy)
 
 
@@ -244,7 +256,7 @@ gcsm_ctx::~gcsm_ctx() {
     if (p) cudaFree(p);
   void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
                   d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2, d_sfc, d_sidx, d_soff,
-                  d_srec, d_sstage};
+                  d_srec, d_sstage, d_stage_state, d_stage_arena, d_stage_bump, d_touched_bc};
   for (void *p : dev2)
     if (p) cudaFree(p);
   for (unsigned long long *p : d_levcnt)
@@ -372,8 +384,13 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   }
   ctx->mark.assign(n, 0);
   ctx->slot16.assign(n, 0);
+  for (int q = 0; q < GCSM_MAX_QUERIES; ++q) ctx->lev_levels[q] = -1;
   if (const char *he = std::getenv("GCSM_HOST_EST")) ctx->gpu_est = std::atoi(he) == 0;
   ctx->overlap = ctx->gpu_est && !std::getenv("GCSM_NO_OVERLAP");
+  if (const char *ok = std::getenv("GCSM_OVERLAP_KMAX")) ctx->overlap_kmax = std::atoi(ok);
+  if (const char *sm = std::getenv("GCSM_STAGE_MB")) ctx->opt.staging_bytes = std::strtoull(sm, nullptr, 10) << 20;
+  if (const char *sm = std::getenv("GCSM_STAGE_MIN")) ctx->stage_min = (uint32_t)std::max(1, std::atoi(sm));
+  if (std::getenv("GCSM_BCOMP") && gcsm_set_measure(ctx, GCSM_MEASURE_BCOMP) != GCSM_OK) return bail(GCSM_ENOMEM);
   ctx->grid = match_grid(dev, &ctx->warps_total);
   ctx->ext_grid = ctx->grid;
   if (const char *r = std::getenv("GCSM_EXT_RESERVE"))
@@ -389,6 +406,22 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
 }
 
 void gcsm_destroy(gcsm_ctx *ctx) { delete ctx; }
+
+gcsm_status gcsm_set_measure(gcsm_ctx *ctx, uint32_t flags) {
+  if (!ctx || (flags & ~(uint32_t)GCSM_MEASURE_BCOMP)) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  const bool on = (flags & GCSM_MEASURE_BCOMP) != 0;
+  if (on && !ctx->d_touched_bc) {
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return GCSM_EDEVICE;
+    if (cudaMalloc(&ctx->d_touched_bc, 4 * (((size_t)ctx->store.n + 31) / 32)) != cudaSuccess) {
+      cudaGetLastError();
+      ctx->d_touched_bc = nullptr;
+      return GCSM_ENOMEM;
+    }
+  }
+  ctx->bcomp = on;
+  return GCSM_OK;
+}
 
 const char *gcsm_last_error(const gcsm_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
 
@@ -788,11 +821,16 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       g_alloc_stream = nullptr;
       g_retired_pinned = nullptr;
     }
-  } alloc_scope(ctx->overlap ? nullptr : ctx->stream, &ctx->retired_pinned);  // two streams: synchronous growth
-  HostStore &S = ctx->store;
+  };
   const int nq = (int)ctx->qs.size();
   int kmax = 2;
   for (const auto &q : ctx->qs) kmax = std::max(kmax, q.qp.k);
+  // one predicate for the cache step's stream and the allocation mode: with the cache step on its own stream
+  // (overlap, every standing query within the overlap size limit) buffers grow synchronously; otherwise
+  // stream-ordered on the context stream
+  const bool two_streams = ctx->overlap && kmax <= ctx->overlap_kmax;
+  AllocScope alloc_scope(two_streams ? nullptr : ctx->stream, &ctx->retired_pinned);
+  HostStore &S = ctx->store;
   const int T = ctx->opt.host_threads;
   gcsm_stats st{};
   st.batches = ctx->batch_seq + 1;
@@ -1256,9 +1294,15 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // the cache step's stream: with overlap it runs beside the previous batch's matching (it writes only this slot's
   // descriptors, delta records, units and counters and the other cache buffer; the previous use of this slot was
   // batch t-2, already collected by gcsm_wait_batch)
-  // (not with a 6-vertex query: its level->=2 walks read zero-copy lists and contend for the host link with the
-  // extension kernels they would run beside — C4: 3.67 K vs 3.89 K updated edges/s)
-  cudaStream_t cs = (ctx->overlap && kmax <= 5) ? ctx->stream3 : s;
+  // (not with a query larger than overlap_kmax, default 5: a 6-vertex query's level->=2 walks read zero-copy lists
+  // and contend for the host link with the extension kernels they would run beside; GCSM_OVERLAP_KMAX
+  // at create moves the limit)
+  // Invariant of the overlapped step: k_sidx_update (in the cache step of t+1) rewrites the sampled index of batch
+  // t's updated vertices while batch t's kernels may run; they never read it for those vertices, because the
+  // descriptor of every x in U_t points into batch t's uploaded U buffer (is_hit() is true, the sampled index is
+  // consulted only for zero-copy lists). A change that lets an updated vertex's descriptor point at host memory
+  // must double-buffer soff per slot first.
+  cudaStream_t cs = two_streams ? ctx->stream3 : s;
   if (!dev_ensure(ctx->d_pidx, ctx->pidx_cap, dirty.size()) || !dev_ensure(ctx->d_pval, ctx->pval_cap, dirty.size()) ||
       !dev_ensure(sl.d_drec, sl.drec_cap, nU) || !dev_ensure(sl.d_dlist, sl.dlist_cap, nd) ||
       !dev_ensure(sl.d_units, sl.units_cap, (size_t)gnu) || !dev_ensure(sl.d_useg, sl.useg_cap, (size_t)gnu))
@@ -1308,6 +1352,38 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   CK(cudaMemsetAsync(sl.d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
   }
   if (cs != s) CK(cudaStreamWaitEvent(s, sl.ev_c1, 0));  // the matching kernels read the cache step's output
+
+  // fetch-once staging (k >= 5 extension kernels): allocated when first needed; this batch's epoch and an empty
+  // arena (the bump counter is reset on the context stream, after the previous batch's kernels)
+  const bool staging = kmax >= 5 && !listing && ctx->opt.staging_bytes != 1 && !ctx->stage_failed;
+  uint32_t stage_epoch = 0;
+  if (staging) {
+    if (!ctx->d_stage_arena) {
+      size_t freeb = 0, totalb = 0;
+      cudaMemGetInfo(&freeb, &totalb);
+      size_t bytes = ctx->opt.staging_bytes ? ctx->opt.staging_bytes : std::min<size_t>(freeb / 4, (size_t)16 << 30);
+      bytes &= ~(size_t)127;
+      if (bytes < 4096 || cudaMalloc(&ctx->d_stage_arena, bytes) != cudaSuccess ||
+          cudaMalloc(&ctx->d_stage_state, 8 * (size_t)S.n) != cudaSuccess ||
+          cudaMalloc(&ctx->d_stage_bump, 8) != cudaSuccess) {
+        cudaGetLastError();
+        for (void *p : {(void *)ctx->d_stage_arena, (void *)ctx->d_stage_state, (void *)ctx->d_stage_bump})
+          if (p) cudaFree(p);
+        ctx->d_stage_arena = nullptr;
+        ctx->d_stage_state = nullptr;
+        ctx->d_stage_bump = nullptr;
+        ctx->stage_failed = true;
+      } else {
+        ctx->stage_cap = bytes / 4;
+        CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.n, s));
+      }
+    }
+    if (ctx->d_stage_arena) {
+      stage_epoch = (uint32_t)(ctx->batch_seq % ((1u << 24) - 1)) + 1;  // 24 bits, never 0
+      if (stage_epoch == 1 && ctx->batch_seq > 0) CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.n, s));
+      CK(cudaMemsetAsync(ctx->d_stage_bump, 0, 8, s));
+    }
+  }
 
   // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
@@ -1382,6 +1458,15 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.tup_rem = d_trem;
   A.tup_rem_cap = rem_cap;
   A.listing = listing ? 1 : 0;
+  if (stage_epoch) {
+    A.stage_state = ctx->d_stage_state;
+    A.stage_arena = ctx->d_stage_arena;
+    A.stage_cap = ctx->stage_cap;
+    A.stage_bump = ctx->d_stage_bump;
+    A.stage_epoch = stage_epoch;
+    A.stage_min = ctx->stage_min;
+  }
+  A.touched = ctx->bcomp ? ctx->d_touched_bc : nullptr;
   if (kmax >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
     const size_t na = (size_t)64 << 20, nt = (size_t)4 << 20;
     const bool fresh_ready = ctx->d_task_ready == nullptr;
@@ -1442,7 +1527,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     }
   // GPU path: the first chunk's level-2 kernels read only the seeds' lists — the batch's uploaded U lists (R32) —
   // so they run on stream2 while the cache step runs on the main stream; the extensions wait for both
-  const bool hoist = ctx->gpu_est;
+  const bool hoist = ctx->gpu_est && !ctx->bcomp;  // measurement mode: every kernel of a query on `s`, in order
   if (hoist) {
     CK(cudaStreamWaitEvent(ctx->stream2, sl.ev_up, 0));
     // the frontier buffers and grouping counters are shared with the previous batch's matching (stream order on
@@ -1463,6 +1548,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     const QueryPlan &QK = sym ? ctx->qs[qi].qps : ctx->qs[qi].qp;
     const int k = QK.k;
     CK(cudaEventRecord(pq.ev_m0, s));
+    if (ctx->bcomp) CK(cudaMemsetAsync(ctx->d_touched_bc, 0, 4 * (((size_t)S.n + 31) / 32), s));
     size_t nev = 0;
     for (size_t c = 0; c < qchunks[qi].size(); ++c) {
       const auto &ch = qchunks[qi][c];
@@ -1486,6 +1572,11 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       nev += 4;
     }
     CK(cudaEventRecord(pq.ev_m1, s));
+    if (ctx->bcomp) {
+      CK(launch_bcomp(ctx->d_touched_bc, S.n, sl.d_vdesc, A.cache_lo, A.cache_hi, A.ubuf_lo, A.ubuf_hi,
+                      sl.d_cnt + (size_t)qi * CNT_N + CNT_BCOMP, s));
+      ++launches;
+    }
     pq.nev = nev;
     pq.aut_mul = sym ? QK.automorphisms : 1;
   }
@@ -1589,7 +1680,13 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.hit_bytes = h[CNT_ACC_L2 + 0] + st.hit_bytes_ext;
     st.miss_bytes = h[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
     st.delta_bytes = h[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
-    st.host_copied_bytes = h[CNT_COPIED];
+    st.host_copied_bytes = h[CNT_COPIED] + h[CNT_STAGE_FILL];  // warp staging copies + arena fills
+    st.stage_fill_bytes = h[CNT_STAGE_FILL];
+    st.stage_lists = h[CNT_STAGE_LISTS];
+    st.stage_hit_bytes = h[CNT_STAGE_HIT];
+    st.bcomp_hit_bytes = h[CNT_BCOMP + 0];
+    st.bcomp_miss_bytes = h[CNT_BCOMP + 1];
+    st.bcomp_delta_bytes = h[CNT_BCOMP + 2];
     st.d2h_bytes = sizeof(unsigned long long) * CNT_N * (size_t)nq;
     st.frontier = h[CNT_F2];
     if (std::getenv("GCSM_TRACE"))
@@ -1795,6 +1892,12 @@ gcsm_status gcsm_query_restrictions(int32_t k, int32_t m, const int32_t *qedges,
     out_pairs[2 * i + 1] = qp.restrictions[i].second;
   }
   return n > cap ? GCSM_ETRUNC : GCSM_OK;
+}
+
+gcsm_status gcsm_binomial_samples(uint64_t key0, int64_t n, double p, int64_t count, int64_t *out) {
+  if (count < 0 || n < 0 || !(p >= 0.0 && p <= 1.0) || (count > 0 && !out)) return GCSM_EINVAL;
+  for (int64_t i = 0; i < count; ++i) out[i] = binomial(rng_chain(key0, (uint64_t)i), n, p);
+  return GCSM_OK;
 }
 
 gcsm_status gcsm_shard(int64_t n_units, const uint64_t *cost, int32_t world, int32_t *out_rank) {

@@ -22,7 +22,7 @@
 #define GCSM_MAXK 8
 #define GCSM_MAXM 28
 #define GCSM_MAXPLANS (2 * GCSM_MAXM)
-#define GCSM_MAX_QUERIES 8  // standing queries per context (gcsm_add_query)
+#define GCSM_MAX_QUERIES 32  // standing queries per context (gcsm_add_query; all 29 connected 3-5-vertex motifs fit)
 
 namespace gcsm {
 

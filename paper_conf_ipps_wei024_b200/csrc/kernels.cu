@@ -87,7 +87,106 @@ struct LRef {
 
 struct Acc {
   unsigned long long add = 0, rem = 0, hit = 0, miss = 0, delta = 0, copied = 0;
+  unsigned long long sfill = 0, slists = 0, shit = 0;  // fetch-once staging: bytes filled, lists, bytes served
 };
+
+// Warp-cooperative bulk copy of a list (16-byte aligned source; lists are
+// allocated in 16-byte granules so reading up to round4(n) ints stays inside
+// the allocation). 4 x 16 B loads per lane are issued before any store, so a
+// warp keeps 2 KB in flight: a zero-copy list crosses PCIe at link speed
+// instead of one dependent 32 B sector per binary-search step.
+__device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
+  __syncwarp();  // every lane is done reading what this buffer held before (WAR across lanes)
+  const uint32_t n4 = (n + 3) >> 2;
+  const int4 *s4 = reinterpret_cast<const int4 *>(src);
+  int4 *d4 = reinterpret_cast<int4 *>(dst);
+  for (uint32_t base = 0; base < n4; base += 128) {
+    const uint32_t i0 = base + lane, i1 = i0 + 32, i2 = i0 + 64, i3 = i0 + 96;
+    int4 v0, v1, v2, v3;
+    if (i0 < n4) v0 = s4[i0];
+    if (i1 < n4) v1 = s4[i1];
+    if (i2 < n4) v2 = s4[i2];
+    if (i3 < n4) v3 = s4[i3];
+    if (i0 < n4) d4[i0] = v0;
+    if (i1 < n4) d4[i1] = v1;
+    if (i2 < n4) d4[i2] = v2;
+    if (i3 < n4) d4[i3] = v3;
+  }
+}
+
+// ---- fetch-once staging of zero-copy lists within a batch -------------------------------------
+// The first warp of the batch that needs vertex v's zero-copy main list claims it (CAS of its state word from an
+// older epoch to "loading"), copies it over PCIe into the batch arena (bump-allocated, 128-byte granules so that
+// no two lists share an L1 line) and publishes (epoch, ready, offset); every later read of that list in the batch,
+// by any warp or any later kernel of the batch, is an HBM read. A warp that finds the list loading waits for it
+// (the loader waits on nothing, so this cannot deadlock). Arena full: the list stays zero-copy ("no room").
+// The arena holds the batch's MAIN lists (v not in U: base(v), unchanged during the batch); the next batch has a
+// new epoch, so nothing stale is ever served.
+constexpr unsigned long long kStReady = 1ull << 39, kStOff = (1ull << 39) - 1;
+
+__device__ __noinline__ const int32_t *stage_resolve(const MatchArgs &A, int32_t v, const int32_t *hp, uint32_t ml,
+                                                     unsigned long long &sfill, unsigned long long &slists,
+                                                     unsigned long long &shit, int lane) {
+  const unsigned long long ep = (unsigned long long)A.stage_epoch << 40;
+  unsigned long long res = 0;
+  int claimed = 0;
+  if (lane == 0) {
+    unsigned long long *w = A.stage_state + v;
+    unsigned long long cur = __ldcg(w);
+    unsigned ns = 32;
+    for (;;) {
+      if ((cur & ~((1ull << 40) - 1)) == ep) {  // this batch's: ready, no room, or being loaded
+        if (cur & kStReady) {
+          res = cur & kStOff;
+          break;
+        }
+        __nanosleep(ns);
+        if (ns < 2048) ns <<= 1;
+        cur = __ldcg(w);
+        continue;
+      }
+      const unsigned long long prev = atomicCAS(w, cur, ep | kStOff);  // claim: loading
+      if (prev == cur) {
+        claimed = 1;
+        break;
+      }
+      cur = prev;
+    }
+    if (claimed) {
+      const unsigned long long n32 = ((unsigned long long)ml + 31) & ~31ull;
+      const unsigned long long off = atomicAdd(A.stage_bump, n32);
+      if (off + n32 > A.stage_cap) {
+        atomicExch(w, ep | kStReady | kStOff);  // no room this batch: zero-copy for everyone
+        claimed = 0;
+        res = kStOff;
+      } else {
+        res = off;
+      }
+    } else {
+      __threadfence();  // acquire: the arena copy published before the state word
+    }
+  }
+  claimed = __shfl_sync(kFull, claimed, 0);
+  res = __shfl_sync(kFull, res, 0);
+  if (claimed) {
+    int32_t *dst = A.stage_arena + res;
+    warp_copy(dst, hp, ml, lane);
+    __syncwarp();
+    __threadfence();  // release: the copy before the state word
+    if (lane == 0) atomicExch(A.stage_state + v, ep | kStReady | res);
+    sfill += 4ull * ml;
+    slists += 1;
+    return dst;
+  }
+  __syncwarp();
+  if (res == kStOff) return hp;
+  shit += 4ull * ml;
+  return A.stage_arena + res;
+}
+
+__device__ __forceinline__ void mark_touched(const MatchArgs &A, int32_t v) {
+  if (A.touched) atomicOr(A.touched + (v >> 5), 1u << (v & 31));
+}
 
 // Persistent per-warp copy of one vertex's main list (the position-2 vertex x2 of a run of frontier entries
 // grouped by x2): `v` = -1 when empty.
@@ -99,7 +198,7 @@ struct Pinned {
   int4 raw;
 };
 
-__device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc,
+__device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view, Acc &acc, int lane,
                                         const Pinned &pin = Pinned()) {
   const int4 raw = v == pin.rv ? pin.raw : __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
   LRef r;
@@ -126,9 +225,13 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
   else if (in_ubuf) acc.delta += 4ull * r.ml;  // the batch's uploaded stable lists of U (device-resident deltas)
   else acc.miss += 4ull * r.ml;
   acc.delta += 4ull * r.xl;
+  if (lane == 0) mark_touched(A, v);
   if (v == pin.v) {  // served from this warp's staged copy
     r.m = pin.p;
     r.dev = true;
+  } else if (!r.dev && A.stage_state && r.ml >= A.stage_min) {  // fetched once per batch into HBM
+    r.m = stage_resolve(A, v, r.m, r.ml, acc.sfill, acc.slists, acc.shit, lane);
+    r.dev = reinterpret_cast<const char *>(r.m) != p;
   }
   return r;
 }
@@ -192,30 +295,6 @@ __device__ __forceinline__ bool is_hit(const MatchArgs &A, const int32_t *p) {
 // A list already in device memory outside the cache (a warp's staged copy in its HBM scratch).
 __device__ __forceinline__ bool is_device(const MatchArgs &A, const int32_t *p) {
   return p >= A.scratch && p < A.scratch_end;
-}
-
-// Warp-cooperative bulk copy of a list (16-byte aligned source; lists are
-// allocated in 16-byte granules so reading up to round4(n) ints stays inside
-// the allocation). 4 x 16 B loads per lane are issued before any store, so a
-// warp keeps 2 KB in flight: a zero-copy list crosses PCIe at link speed
-// instead of one dependent 32 B sector per binary-search step.
-__device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
-  __syncwarp();  // every lane is done reading what this buffer held before (WAR across lanes)
-  const uint32_t n4 = (n + 3) >> 2;
-  const int4 *s4 = reinterpret_cast<const int4 *>(src);
-  int4 *d4 = reinterpret_cast<int4 *>(dst);
-  for (uint32_t base = 0; base < n4; base += 128) {
-    const uint32_t i0 = base + lane, i1 = i0 + 32, i2 = i0 + 64, i3 = i0 + 96;
-    int4 v0, v1, v2, v3;
-    if (i0 < n4) v0 = s4[i0];
-    if (i1 < n4) v1 = s4[i1];
-    if (i2 < n4) v2 = s4[i2];
-    if (i3 < n4) v3 = s4[i3];
-    if (i0 < n4) d4[i0] = v0;
-    if (i1 < n4) d4[i1] = v1;
-    if (i2 < n4) d4[i2] = v2;
-    if (i3 < n4) d4[i3] = v3;
-  }
 }
 
 // Staging policy: a zero-copy driver list is bulk-copied once
@@ -418,19 +497,19 @@ __device__ __forceinline__ void trim_lists(LRef *L, int nl, int32_t vlo, int32_t
 // Returns the number of probe lists written to L and sets *drv (index of the
 // smallest list) or uses the reused set.
 __device__ __forceinline__ int gather_lists(const MatchArgs &A, const LevelPlan &Lp, const int32_t *f, LRef *L,
-                                            int *drv, Acc &acc, const Pinned &pin = Pinned()) {
+                                            int *drv, Acc &acc, int lane, const Pinned &pin = Pinned()) {
   int nl = 0;
   uint32_t best = 0xffffffffu;
   *drv = 0;
   if (Lp.reuse >= 0) {
     for (int r = 0; r < Lp.nrest; ++r) {
       const int b = Lp.rest[r];
-      L[nl++] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, pin);
+      L[nl++] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, lane, pin);
     }
     return nl;
   }
   for (int b = 0; b < Lp.nb; ++b) {
-    L[nl] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, pin);
+    L[nl] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, lane, pin);
     const uint32_t sz = L[nl].ml + L[nl].xl;
     if (sz < best) {
       best = sz;
@@ -465,6 +544,9 @@ __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int la
     if (acc.miss) atomicAdd(&A.cnt[A.acc_base + 1], acc.miss);
     if (acc.delta) atomicAdd(&A.cnt[A.acc_base + 2], acc.delta);
     if (acc.copied) atomicAdd(&A.cnt[CNT_COPIED], acc.copied);
+    if (acc.sfill) atomicAdd(&A.cnt[CNT_STAGE_FILL], acc.sfill);
+    if (acc.slists) atomicAdd(&A.cnt[CNT_STAGE_LISTS], acc.slists);
+    if (acc.shit) atomicAdd(&A.cnt[CNT_STAGE_HIT], acc.shit);
   }
 }
 
@@ -504,7 +586,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
     const LevelPlan &L2 = P.lv[2];
     LRef L[7];
     int drv;
-    const int nl = gather_lists(A, L2, f, L, &drv, acc);
+    const int nl = gather_lists(A, L2, f, L, &drv, acc, lane);
     stage_lists(A, L, nl, drv, false, 0, sm, kSmemInts, gstage, lane, acc);
     int32_t vlo, vhi;
     range_of(L2, f, &vlo, &vhi);
@@ -617,7 +699,16 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
                                                                 ((unsigned long long)(unsigned)raw.y << 32));
         const uint32_t ml = (uint32_t)raw.z;
-        const bool miss = !is_hit(A, mp);
+        bool miss = !is_hit(A, mp), staged = false;
+        if (lane == 0) mark_touched(A, x2);
+        if (miss && A.stage_state && ml >= A.stage_min) {  // the run's x2 list, fetched once per batch
+          const int32_t *sp = stage_resolve(A, x2, mp, ml, acc.sfill, acc.slists, acc.shit, lane);
+          if (sp != mp) {
+            mp = sp;
+            miss = false;
+            staged = true;
+          }
+        }
         const uint32_t ml4 = (ml + 3) & ~3u;
         pin_sm = 0;
         pin.bm_v = -1;
@@ -634,6 +725,10 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           __syncwarp();
           pin.v = x2;
           pin.p = pstage;
+        }
+        if (staged && pin.v != x2) {  // served in place from the batch arena (HBM) for the whole run
+          pin.v = x2;
+          pin.p = mp;
         }
         if (GCSM_BM_INTS > 0 && run >= 2 && ml >= 32 && (pin.v == x2 || !miss)) {
           bm_build(bm, pin.v == x2 ? pin.p : mp, ml, lane);
@@ -713,7 +808,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const LevelPlan &Lp = P.lv[p];
         LRef L[7];
         int drv;
-        const int nl = gather_lists(A, Lp, f, L, &drv, acc, pin);
+        const int nl = gather_lists(A, Lp, f, L, &drv, acc, lane, pin);
         int32_t excl[GCSM_MAXK];
         int nex = 0;
         for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
@@ -1057,8 +1152,14 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
       int4 r1 = make_int4(0, 0, 0, 0), r2 = make_int4(0, 0, 0, 0);
       int2 seg = make_int2(0, 0);
       int xl0 = 0, xl1 = 0;
-      if (need & 1u) r1 = lr_fetch(A, u.x, (pk >> 20) & 3u, &xl0);
-      if (need & 2u) r2 = lr_fetch(A, u.y, (pk >> 22) & 3u, &xl1);
+      if (need & 1u) {
+        r1 = lr_fetch(A, u.x, (pk >> 20) & 3u, &xl0);
+        mark_touched(A, u.x);
+      }
+      if (need & 2u) {
+        r2 = lr_fetch(A, u.y, (pk >> 22) & 3u, &xl1);
+        mark_touched(A, u.y);
+      }
       if ((pk >> 6) & 1u) seg = A.useg[ui];
       meta[4 * lane + 0] = make_int4(x2, u.z, u.x, u.y);
       meta[4 * lane + 1] = r1;
@@ -1091,6 +1192,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
         rlo = __reduce_min_sync(kFull, rlo);
         rhi = __reduce_max_sync(kFull, rhi);
         pin_v = x2;
+        if (lane == 0 && rlo <= rhi) mark_touched(A, x2);
         xraw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + x2));
         xrec = xraw.w ? __ldg(reinterpret_cast<const int4 *>(A.drec + ((uint32_t)xraw.w - 1))) : make_int4(0, 0, 0, 0);
         const int32_t *mp = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)xraw.x |
@@ -1438,6 +1540,7 @@ int match_grid(int device, int *warps_total) {
 cudaError_t launch_level2(const MatchArgs &a0, int grid, cudaStream_t s) {
   MatchArgs a = a0;
   a.acc_base = CNT_ACC_L2;
+  a.stage_state = nullptr;  // level 2 reads the seeds' lists (the batch's uploaded U lists on the GPU path)
   if (a.listing) k_level2<true><<<grid, kBlock, kSmemBytes, s>>>(a);
   else k_level2<false><<<grid, kBlock, kSmemBytes, s>>>(a);
   return cudaGetLastError();
@@ -1498,6 +1601,35 @@ cudaError_t launch_sidx_update(int32_t *sidx, uint32_t *soff, const int4 *rec, i
   if (n <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>((n + 7) / 8, 148 * 8);
   k_sidx_update<<<grid, 256, 0, s>>>(sidx, soff, rec, n, staged);
+  return cudaGetLastError();
+}
+
+__global__ void k_bcomp(const uint32_t *touched, int32_t n, const VDesc *vdesc, const char *cache_lo,
+                        const char *cache_hi, const char *ubuf_lo, const char *ubuf_hi, unsigned long long *out) {
+  unsigned long long b[3] = {0, 0, 0};
+  const int64_t W = ((int64_t)n + 31) >> 5;
+  for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = touched[w];
+    while (bits) {
+      const int i = __ffs(bits) - 1;
+      bits &= bits - 1;
+      const VDesc d = vdesc[w * 32 + i];
+      const char *p = reinterpret_cast<const char *>(d.ptr);
+      const int where = (p >= cache_lo && p < cache_hi) ? 0 : ((p >= ubuf_lo && p < ubuf_hi) ? 2 : 1);
+      b[where] += 4ull * d.len;
+    }
+  }
+  for (int j = 0; j < 3; ++j) {
+    unsigned long long x = b[j];
+    for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
+    if ((threadIdx.x & 31) == 0 && x) atomicAdd(out + j, x);
+  }
+}
+
+cudaError_t launch_bcomp(const uint32_t *touched, int32_t n, const VDesc *vdesc, const char *cache_lo,
+                         const char *cache_hi, const char *ubuf_lo, const char *ubuf_hi, unsigned long long *out,
+                         cudaStream_t s) {
+  k_bcomp<<<148 * 4, 256, 0, s>>>(touched, n, vdesc, cache_lo, cache_hi, ubuf_lo, ubuf_hi, out);
   return cudaGetLastError();
 }
 

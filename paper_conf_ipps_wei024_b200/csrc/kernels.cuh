@@ -31,7 +31,15 @@ enum Counter {
   CNT_DBG_PINBYTES = 22, // k_last4: zero-copy bytes copied by run pins
   CNT_DBG_PINS = 23,     // k_last4: runs pinned
   CNT_CACHED = 24,       // GPU packer (query 0's block): cached vertices, cached bytes, internal error flag
-  CNT_N = 27
+  // fetch-once staging of zero-copy lists: bytes copied host -> batch arena, lists staged,
+  // algorithmic bytes then served from the arena (HBM)
+  CNT_STAGE_FILL = 27,
+  CNT_STAGE_LISTS = 28,
+  CNT_STAGE_HIT = 29,
+  // B_comp (measurement mode only): bytes of the DISTINCT main lists the query's kernels touched,
+  // by where they lived: HBM cache, pinned host (zero-copy), the batch's uploaded lists of U
+  CNT_BCOMP = 30,
+  CNT_N = 33
 };
 
 struct MatchArgs {
@@ -71,6 +79,15 @@ struct MatchArgs {
   int32_t *task_ready;
   uint32_t task_cap;
   int32_t task_gen;         // ready-flag value of this launch (no per-launch clearing)
+  // fetch-once staging of zero-copy lists within a batch: per vertex state word (epoch << 40 | ready << 39 |
+  // offset), the batch arena and its bump counter; nullptr = off
+  unsigned long long *stage_state;
+  int32_t *stage_arena;
+  unsigned long long stage_cap;  // ints
+  unsigned long long *stage_bump;
+  uint32_t stage_epoch;          // 24 bits, never 0
+  uint32_t stage_min;            // shortest list (ints) routed through the arena
+  uint32_t *touched;             // B_comp measurement: bitmap of vertices whose main list was read (nullptr = off)
 };
 
 struct Task {
@@ -91,6 +108,11 @@ cudaError_t launch_extend(const MatchArgs &a, int grid, cudaStream_t s);
 cudaError_t launch_group_frontier(const MatchArgs &a, int32_t n_vertices, uint32_t *hist, uint32_t *bsum,
                                   int32_t *group, cudaStream_t s);
 cudaError_t launch_gather_lists(char *dst, const char *src, const uint64_t *tri, int64_t n, cudaStream_t s);
+// B_comp (measurement mode): sum the main-list bytes of the vertices in the touched bitmap by where they live;
+// out[0..2] += (HBM cache, pinned host, uploaded U lists)
+cudaError_t launch_bcomp(const uint32_t *touched, int32_t n, const VDesc *vdesc, const char *cache_lo,
+                         const char *cache_hi, const char *ubuf_lo, const char *ubuf_hi, unsigned long long *out,
+                         cudaStream_t s);
 cudaError_t launch_patch_vdesc(VDesc *vdesc, const int64_t *idx, const VDesc *val, int64_t n, cudaStream_t s);
 // sampled-index updates: rec[i] = (vertex, offset, count, staging position); samples staged contiguously
 cudaError_t launch_sidx_update(int32_t *sidx, uint32_t *soff, const int4 *rec, int64_t n, const int32_t *staged,

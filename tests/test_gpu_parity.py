@@ -79,10 +79,11 @@ def test_c1_triangle_budgets(G, budget):
 
 # ------------------------------------------------------------------ fuzz
 
-FUZZ = ["edge", "wedge", "triangle", "path4", "c4", "diamond", "k4", "star3", "house5u", "k5", "prism6", "k4tri6"]
+FUZZ = ["edge", "wedge", "triangle", "path4", "c4", "diamond", "k4", "star3", "house5u", "k5", "prism6", "k4tri6",
+        "wheel7", "k4k4_7", "k7", "cube8", "k8"]
 
 
-@pytest.mark.parametrize("seed", range(36))
+@pytest.mark.parametrize("seed", range(51))
 def test_fuzz_small_graphs(G, seed):
     rng = np.random.default_rng(1000 + seed)
     n = int(rng.integers(8, 14))
@@ -96,6 +97,15 @@ def test_fuzz_small_graphs(G, seed):
         ql = rng.integers(0, 2, k).astype(np.int32)
     order = rng.permutation(k).astype(np.int32) if seed % 4 == 2 else None
     rp, col = oracle.csr(n, g0)
+    if k >= 7:  # 7- and 8-vertex patterns: counts (their tuple lists on dense graphs run to millions)
+        want, _ = oracle_run(n, rp, col, labels, (k, qe, ql), [(ins, dele)])
+        for sym in (True, False):
+            g = G.Gcsm(n, rp, col, labels, device=0, symmetry=sym)
+            g.set_query(k, qe, ql, order)
+            g.set_cache_budget([0, 64, 1 << 20][seed % 3])
+            assert g.apply_batch(ins, dele) == want[0]
+            g.close()
+        return
     want, _ = oracle_run(n, rp, col, labels, (k, qe, ql), [(ins, dele)], listing=True)
     g = G.Gcsm(n, rp, col, labels, device=0)
     g.set_query(k, qe, ql, order)
@@ -103,6 +113,15 @@ def test_fuzz_small_graphs(G, seed):
     a, r, ta, tr = g.apply_batch_list(ins, dele, 1 << 16, 1 << 16)
     g.close()
     assert (a, r, tuples_set(ta), tuples_set(tr)) == want[0]
+
+
+@pytest.mark.parametrize("name", ["wheel7", "k4k4_7", "k7", "cube8"])
+def test_seven_eight_vertex_lists(G, name):
+    """k = 7 / 8 in list mode (every tuple, no symmetry breaking) on a sparse graph with planted cliques."""
+    w = gi.make_workload("C4", scale=9, n_edges=2_500, batch=64, n_batches=2)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches, listing=True)
+    got, _, _ = lib_run(G, w.n, w.row_ptr, w.col, None, name, w.batches, 0.05, listing=True)
+    assert got == want
 
 
 def test_degenerate_cases(G):
@@ -211,7 +230,7 @@ def test_six_vertex_queries(G, name):
     assert got == want
 
 
-@pytest.mark.parametrize("name", ["prism6", "k4tri6", "k6"])
+@pytest.mark.parametrize("name", ["prism6", "k4tri6", "k6", "wheel7", "k4k4_7"])
 def test_c4_shaped_planted(G, name):
     """C4-shaped (FR R-MAT parameters + planted 8-cliques): the 6-vertex counts are non-zero, budget << graph."""
     w = gi.make_workload("C4", scale=13, n_edges=60_000, batch=256, n_batches=2)
@@ -250,71 +269,147 @@ def test_star_closed_form_at_scale(G, r):
     g.close()
 
 
-# ------------------------------------------------------------------ estimator ② and packer ③ parity
+# ------------------------------------------------------------------ estimator ② and packer ③
+# The oracle estimates by plain walks (§IV-A) with its own generator, so the product's merged walks (§IV-B) are
+# pinned STATISTICALLY against the exact access counts C_v (eq. (6)/(7)), while the host walker (the paper's
+# CPU placement, GCSM_HOST_EST=1) and the GPU walker are compared bit-exactly with each other (product-internal).
 
-def without_updated(score, I, D):
-    """DESIGN.md R32: the stable lists of the batch's updated vertices are uploaded with the batch (device-resident
-    for all of its kernels), so the ranking of R23 runs over the other vertices."""
-    s = np.array(score, dtype=np.float64, copy=True)
-    U = np.unique(np.concatenate([np.asarray(I).ravel(), np.asarray(D).ravel()]))
-    s[U] = 0.0
-    return s
+def updated_vertices(I, D):
+    return np.unique(np.concatenate([np.asarray(I).ravel(), np.asarray(D).ravel()]))
+
+
+def host_est_ctx(G, *args, **kw):
+    import os
+    os.environ["GCSM_HOST_EST"] = "1"
+    try:
+        return G.Gcsm(*args, **kw)
+    finally:
+        del os.environ["GCSM_HOST_EST"]
+
+
+def product_estimate(g, n, k):
+    """eq. (3) over the product's per-level sums (query 0), as a dense vector."""
+    st = g.stats()
+    ids, lev = g.estimates()
+    est = np.zeros(n)
+    est[ids] = oracle.estimate_from_levels(lev[:, :k - 2], k, st["n1"], st["max_degree"], st["walks"])
+    return est, ids, lev, st
+
+
+def _eq6_case():
+    w = gi.make_workload("C1", scale=8, n_edges=1500, batch=24)
+    ins = w.batches[0][0][:12]
+    E = oracle.edges_of(w.row_ptr, w.col)
+    dele = E[np.random.default_rng(9).choice(len(E), 8, replace=False)]
+    return w, ins, dele
+
+
+@pytest.mark.parametrize("name", ["diamond", "house5u", "k4", "prism6"])
+def test_gpu_estimator_unbiased_eq6(G, name):
+    """The DEVICE walker (merged walks, §IV-B) against the oracle's exact C_v: the mean of eq. (3) over 60 seeds lies
+    within 5 standard errors of C_v (eq. (6)), the spread respects eq. (7) (merged walks: independent binomials,
+    R20, so a factor 2 of slack), every estimated vertex is accessed in the exact trees, and every sampled vertex's
+    un-averaged estimate is >= |ΔE|."""
+    w, ins, dele = _eq6_case()
+    k, qe, ql = gi.query(name)
+    C = oracle.access_counts(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele).astype(float)
+    I, D, _ = oracle.normalize_batch(w.n, w.row_ptr, w.col, ins, dele)
+    N1 = len(oracle.units(k, qe, ql, None, I, D))
+    R, M = 60, 3000
+    ests = []
+    for r in range(R):
+        g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0, seed=1000 + r, walks_override=M)
+        g.set_query(k, qe, ql)
+        g.set_cache_budget(w.adj_bytes // 10)
+        assert g.apply_batch(ins, dele) == oracle.delta(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele)
+        est, ids, lev, st = product_estimate(g, w.n, k)
+        g.close()
+        assert (st["n1"], st["walks"]) == (N1, M)
+        Dmax = st["max_degree"]
+        ests.append(est)
+    ests = np.array(ests)
+    mean, sd = ests.mean(0), ests.std(0, ddof=1)
+    hot = C > 0
+    bound7 = np.sqrt((k - 1) * N1 * float(Dmax) ** (k - 2) * C / M)
+    se = np.maximum(sd, bound7 / 4) / np.sqrt(R)
+    z = np.abs(mean[hot] - C[hot]) / se[hot]
+    assert np.mean(z < 5) > 0.995 and z.max() < 8, (z.max(), np.mean(z < 5))
+    assert np.all(ests[:, ~hot] == 0)
+    assert np.all(sd[hot] ** 2 <= 2.0 * bound7[hot] ** 2 + 1e-9)
+    for row in ests:
+        s_ = row > 0
+        assert np.all(row[s_] * M >= N1 * (1 - 1e-12))
 
 
 @pytest.mark.parametrize("name,labelled", [("diamond", False), ("k4", False), ("house5u", False), ("house5", True)])
-def test_estimator_and_cache_parity(G, name, labelled):
+def test_gpu_walker_equals_host_walker(G, name, labelled):
+    """Product-internal: the device walker draws exactly what the host walker draws (R30), batch after batch; the
+    two packers select by R23 (GPU path: over the vertices not updated by the batch, R32) — checked against the
+    oracle's independent ranking on the product's own estimates; counts equal the oracle's."""
     w = gi.make_workload("C3" if labelled else "C2", scale=12, n_edges=30_000, batch=256, n_batches=2)
     labels = w.labels if labelled else None
     k, qe, ql = gi.query(name)
     seed = 0xBEEF
     budget = w.adj_bytes // 25
     g = G.Gcsm(w.n, w.row_ptr, w.col, labels, device=0, seed=seed)
-    g.set_query(k, qe, ql)
-    g.set_cache_budget(budget)
+    h = host_est_ctx(G, w.n, w.row_ptr, w.col, labels, device=0, seed=seed)
+    for c in (g, h):
+        c.set_query(k, qe, ql)
+        c.set_cache_budget(budget)
     rp, col = w.row_ptr, w.col
     for t, (ins, dele) in enumerate(w.batches):
-        g.apply_batch(ins, dele)
-        st = g.stats()
-        e = oracle.estimate(w.n, rp, col, labels, k, qe, ql, ins, dele, seed=seed, batch_seq=t)
-        assert (st["n1"], st["max_degree"], st["walks"]) == (e["N1"], e["D"], e["M"])
-        ids, lev = g.estimates()
-        want_ids = np.nonzero(e["levcnt"].sum(1))[0]
-        assert np.array_equal(ids, want_ids)
-        assert np.array_equal(lev[:, :k - 2], e["levcnt"][want_ids])
-        # the cache: longest prefix of (estimate desc, id asc) whose 16-byte-aligned stable lists fit (R23)
+        want = oracle.delta(w.n, rp, col, labels, k, qe, ql, ins, dele)
+        assert g.apply_batch(ins, dele) == want
+        assert h.apply_batch(ins, dele) == want
         I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+        eg, ids_g, lev_g, st_g = product_estimate(g, w.n, k)
+        eh, ids_h, lev_h, st_h = product_estimate(h, w.n, k)
+        N1 = len(oracle.units(k, qe, ql, labels, I, D))
+        Dmax = oracle._Views(w.n, rp, col, I, D).max_degree()
+        assert (st_g["n1"], st_g["max_degree"], st_g["walks"]) == (N1, Dmax, oracle.walks(N1, Dmax, k))
+        assert (st_h["n1"], st_h["max_degree"], st_h["walks"]) == (st_g["n1"], st_g["max_degree"], st_g["walks"])
+        assert np.array_equal(ids_g, ids_h)
+        assert np.array_equal(lev_g[:, :k - 2], lev_h[:, :k - 2])
+        # every estimated vertex is one the exact execution trees access (eq. (6) support)
+        C = oracle.access_counts(w.n, rp, col, labels, k, qe, ql, ins, dele)
+        assert np.all(C[ids_g] > 0)
         rps, _ = oracle.stable_graph(w.n, rp, col, D)
         sz = 16 * ((np.diff(rps) + 3) // 4)
-        assert np.array_equal(g.cached(), oracle.select_cache(without_updated(e["est"], I, D), sz, budget & ~15))
+        assert np.array_equal(g.cached(), oracle.select_cache(eg, sz, budget & ~15, exclude=updated_vertices(I, D)))
+        assert np.array_equal(h.cached(), oracle.select_cache(eh, sz, budget & ~15))
         rp, col = oracle.apply_batch(w.n, rp, col, I, D)
     g.close()
+    h.close()
 
 
 @pytest.mark.parametrize("name,M", [("k4", 10**9), ("house5u", 10**9), ("prism6", 10**9)])
-def test_estimator_btrd_range(G, name, M):
-    """Walk budgets large enough that children draw B' ~ Bin(B, 1/D) with B/D >= 10 (BTRD, R20) on the device:
-    per-vertex per-level sums and the cached set still equal the oracle's."""
+def test_gpu_walker_btrd_range(G, name, M):
+    """Walk budgets large enough that children draw B' ~ Bin(B, 1/D) with B/D >= 10 (BTRD, R20) on the device: the
+    per-vertex per-level sums still equal the host walker's, and the cached set is R23 on them."""
     w = gi.make_workload("C2", scale=11, n_edges=12_000, batch=96, n_batches=1)
     k, qe, ql = gi.query(name)
     seed = 0x5EED
     budget = w.adj_bytes // 20
     g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0, seed=seed, walks_override=M)
-    g.set_query(k, qe, ql)
-    g.set_cache_budget(budget)
+    h = host_est_ctx(G, w.n, w.row_ptr, w.col, None, device=0, seed=seed, walks_override=M)
     ins, dele = w.batches[0]
-    g.apply_batch(ins, dele)
-    e = oracle.estimate(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele, seed=seed, batch_seq=0, M=M)
-    assert e["M"] == M and g.stats()["walks"] == M
-    assert M // e["N1"] >= 10 * e["D"]  # level-1 children are in BTRD's range
-    ids, lev = g.estimates()
-    want_ids = np.nonzero(e["levcnt"].sum(1))[0]
-    assert np.array_equal(ids, want_ids)
-    assert np.array_equal(lev[:, :k - 2], e["levcnt"][want_ids])
+    want = oracle.delta(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele)
+    for c in (g, h):
+        c.set_query(k, qe, ql)
+        c.set_cache_budget(budget)
+        assert c.apply_batch(ins, dele) == want
+    eg, ids_g, lev_g, st = product_estimate(g, w.n, k)
+    _, ids_h, lev_h, _ = product_estimate(h, w.n, k)
+    assert st["walks"] == M
+    assert M // st["n1"] >= 10 * st["max_degree"]  # level-1 children are in BTRD's range
+    assert np.array_equal(ids_g, ids_h)
+    assert np.array_equal(lev_g[:, :k - 2], lev_h[:, :k - 2])
     I, D, _ = oracle.normalize_batch(w.n, w.row_ptr, w.col, ins, dele)
     rps, _ = oracle.stable_graph(w.n, w.row_ptr, w.col, D)
     sz = 16 * ((np.diff(rps) + 3) // 4)
-    assert np.array_equal(g.cached(), oracle.select_cache(without_updated(e["est"], I, D), sz, budget & ~15))
+    assert np.array_equal(g.cached(), oracle.select_cache(eg, sz, budget & ~15, exclude=updated_vertices(I, D)))
     g.close()
+    h.close()
 
 
 def test_degree_policy_cached_set(G):
@@ -332,7 +427,7 @@ def test_degree_policy_cached_set(G):
         rps, _ = oracle.stable_graph(w.n, rp, col, D)
         deg = np.diff(rps).astype(np.float64)
         sz = 16 * ((np.diff(rps) + 3) // 4)
-        assert np.array_equal(g.cached(), oracle.select_cache(without_updated(deg, I, D), sz, budget & ~15))
+        assert np.array_equal(g.cached(), oracle.select_cache(deg, sz, budget & ~15, exclude=updated_vertices(I, D)))
         rp, col = oracle.apply_batch(w.n, rp, col, I, D)
     g.close()
 
@@ -558,13 +653,13 @@ def test_multi_query_limits(G):
         g.add_query(k, qe, ql)  # before set_query
     assert ei.value.name == "GCSM_ESTATE"
     g.set_query(k, qe, ql)
-    for _ in range(7):
+    for _ in range(31):
         g.add_query(k, qe, ql)
     with pytest.raises(G.GcsmError) as ei:
         g.add_query(k, qe, ql)
     assert ei.value.name == "GCSM_EINVAL"
     a = g.apply_batch(*w.batches[0])
-    assert all(g.query_counts(i) == a for i in range(8))
+    assert all(g.query_counts(i) == a for i in range(32))
     g.close()
 
 
@@ -625,3 +720,33 @@ def test_pipelined_cache_step_overlap(G, overlap, monkeypatch):
         want, (rp1, col1) = oracle_run(w.n, w.row_ptr, w.col, None, nm, w.batches)
         assert got[nm] == want, nm
     assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
+
+
+# ------------------------------------------------------------------ NEXT-4: motif counting (Fig. 11)
+
+def test_motif_census_road_net(G):
+    """All 29 connected 3-, 4- and 5-vertex motifs as standing queries of ONE context on a road-net-shaped graph
+    (low skew): every motif's (added, removed) equals the oracle's, over a 3-batch stream, and the
+    final graph equals the oracle's G_t."""
+    w = gi.make_workload("PA", scale=14, batch=512, n_batches=3)
+    names = gi.MOTIFS[3] + gi.MOTIFS[4] + gi.MOTIFS[5]
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    for i, q in enumerate(names):
+        k, qe, ql = gi.query(q)
+        (g.set_query if i == 0 else g.add_query)(k, qe, ql)
+    g.set_cache_budget(w.adj_bytes // 10)
+    rp, col = w.row_ptr, w.col
+    nonzero = 0
+    for ins, dele in w.batches:
+        g.apply_batch(ins, dele)
+        for i, q in enumerate(names):
+            k, qe, ql = gi.query(q)
+            want = oracle.delta(w.n, rp, col, None, k, qe, ql, ins, dele)
+            assert g.query_counts(i) == want, q
+            nonzero += want != (0, 0)
+        I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+        rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+    assert nonzero >= 30
+    rp2, col2 = g.export_csr()
+    assert np.array_equal(rp, rp2) and np.array_equal(col, col2)
+    g.close()

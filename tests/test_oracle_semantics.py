@@ -306,3 +306,32 @@ def test_apply_batch_vs_set_algebra(seed):
     s = oracle.stable_graph(n, rp, col, D)
     e = {tuple(x) for x in oracle.edges_of(*s).tolist()}
     assert e == {tuple(x) for x in g0.tolist()} - {tuple(x) for x in D.tolist()}
+
+
+def test_motif_catalogue():
+    """Fig. 11 counts 'all size-3, 4, and 5 motifs': the connected simple graphs on 3, 4, 5 vertices up
+    to isomorphism number 2, 6 and 21 (OEIS A001349); each is connected and no two are isomorphic (networkx)."""
+    nx = pytest.importorskip("networkx")
+    for size, want in ((3, 2), (4, 6), (5, 21)):
+        cat = gi.motifs(size)
+        assert len(cat) == want
+        graphs = []
+        for name, edges in cat:
+            h = nx.Graph()
+            h.add_nodes_from(range(size))
+            h.add_edges_from(edges)
+            assert nx.is_connected(h), name
+            graphs.append(h)
+        for i in range(len(graphs)):
+            for j in range(i + 1, len(graphs)):
+                assert not nx.is_isomorphic(graphs[i], graphs[j])
+    assert gi.MOTIFS[3] == ["m3_0", "m3_1"]
+    assert gi.query("m3_1")[1].tolist() == [[0, 1], [0, 2], [1, 2]]  # the triangle
+
+
+def test_road_net_shape():
+    """PA-shaped input (Table I RoadNetPA: 1.09M vertices, 1.54M edges, small degrees): low skew, small max degree."""
+    w = gi.make_workload("PA", scale=14, n_batches=1, batch=256)
+    deg = np.diff(w.row_ptr)
+    assert deg.max() <= 8 and 2.0 < deg.mean() < 3.5
+    assert w.n == 128 * 128
