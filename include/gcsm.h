@@ -88,6 +88,9 @@ typedef struct {
   uint64_t walks_override; /* 0 = M = |ΔE| D^(k-2) / 32^k (R21) */
   uint32_t flags;          /* GCSM_FLAG_* */
   uint32_t reserved;
+  int64_t vertex_capacity; /* ids the graph may grow into: 0 = n (no growth). Insertions may name ids in
+                              [n, vertex_capacity): new vertices, each given an empty list with the average
+                              degree as capacity; gcsm_add_vertices adds labelled ones */
   uint64_t staging_bytes;  /* per-GPU HBM arena of the fetch-once staging of zero-copy lists within a batch
                               (not a cache: emptied every batch): 0 = default (a quarter of the
                               free HBM when first needed, at most 16 GiB), 1 = off */
@@ -134,6 +137,7 @@ typedef struct {
   uint64_t bcomp_hit_bytes, bcomp_miss_bytes, bcomp_delta_bytes; /* B_comp: bytes of the DISTINCT
                                 main lists the query's kernels touched, by home (HBM cache / pinned host / uploaded
                                 lists of U); only with GCSM_BCOMP=1 at create (measurement mode), else 0 */
+  uint64_t peer_bytes;       /* algorithmic list bytes read from a linked peer's HBM cache (gcsm_link_peers) */
 } gcsm_stats;
 
 /* Fills *opt with the defaults (device -1, world 1, seed 0x6C53, all cores,
@@ -147,7 +151,7 @@ void gcsm_default_options(gcsm_options *opt);
  * The graph is copied into the library's pinned, GPU-mapped host store with
  * 2x capacity per list. opt may be NULL (defaults). EINVAL on any
  * violation (nothing allocated). With world > 1 this is collective (NCCL
- * communicator creation). */
+ * communicator creation). Per-vertex device arrays are sized for opt->vertex_capacity ids. */
 gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels,
                         const gcsm_options *opt, gcsm_ctx **out);
 
@@ -181,9 +185,10 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes);
 
 /* Applies one batch: ins[2*n_ins], del[2*n_del] (pairs of vertex ids, any
  * orientation; duplicates collapse; inserting an existing edge or deleting an
- * absent one is a counted no-op, R8). EINVAL (no mutation) on a self loop, an
- * id outside [0,n), or an edge in both lists. On success *added / *removed
- * are the global embedding counts (every rank gets the same values). */
+ * absent one is a counted no-op, R8). An insertion may name ids in [n, vertex_capacity): those vertices join
+ * the graph. EINVAL (no mutation) on a self loop, an id outside [0, vertex_capacity), a deletion
+ * naming an id >= n (deletions involve existing vertices), or an edge in both lists. On success *added /
+ * *removed are the global embedding counts (every rank gets the same values). */
 gcsm_status gcsm_apply_batch(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del,
                              uint64_t *added, uint64_t *removed);
 
@@ -220,6 +225,25 @@ uint64_t gcsm_query_automorphisms(const gcsm_ctx *ctx);
 
 /* Static-lifetime (per ctx) message for the last error; "" if none. */
 const char *gcsm_last_error(const gcsm_ctx *ctx);
+
+/* Current number of vertices (ids [0, n)); grows by insertions naming new ids or gcsm_add_vertices. */
+int32_t gcsm_num_vertices(const gcsm_ctx *ctx);
+
+/* Adds `count` isolated vertices (ids n .. n+count-1, *first_id = n) with labels[count] (NULL: label 0), each
+ * with an empty list of the average degree's capacity. EINVAL beyond the vertex capacity
+ * (gcsm_options.vertex_capacity) or for labels on an unlabelled graph; ESTATE with a batch in flight. */
+gcsm_status gcsm_add_vertices(gcsm_ctx *ctx, int32_t count, const int32_t *labels, int32_t *first_id);
+
+/* NVLink peer cache (host data movement is the bottleneck): links n contexts
+ * (2 <= n <= 8) of this process — one per GPU, or several on one GPU — so that a list missing from a context's
+ * own HBM cache is read from a linked context's HBM cache (peer access over NVLink / NVSwitch) before falling
+ * back to zero-copy host reads. The contexts must hold the same graph and apply the same batches in lockstep
+ * (same vertex capacity and batch count at link time), each driven by ITS OWN host thread: a context's submit
+ * of batch t waits (host rendezvous) until every linked context has enqueued its cache step of batch t, and its
+ * matching kernels wait (device events) for those cache steps; a context's cache step of batch t+2 waits for
+ * every peer's batch t. n = 0 or 1 unlinks the given contexts (gcsm_destroy also unlinks the group).
+ * EINVAL on bad arguments or a mismatch, ESTATE with a batch in flight, EDEVICE without peer access. */
+gcsm_status gcsm_link_peers(gcsm_ctx *const *ctxs, int32_t n);
 
 /* Measurement modes for the following batches (flags = GCSM_MEASURE_*; 0 = off, the default). With
  * GCSM_MEASURE_BCOMP the kernels also mark, per query, the vertices whose main list they read, and the batch's

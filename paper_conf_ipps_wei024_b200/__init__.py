@@ -58,7 +58,7 @@ class Gcsm:
 
     def __init__(self, n, row_ptr, col, labels=None, *, device=-1, rank=0, world=1, nccl_id=None, seed=0x6C53,
                  host_threads=0, cache_policy="estimator", walks_override=0, local_counts=False, symmetry=True,
-                 staging_bytes=0):
+                 staging_bytes=0, vertex_capacity=0):
         lib = _lib.load()
         self._lib = lib
         opt = Options()
@@ -73,6 +73,7 @@ class Gcsm:
         opt.cache_policy = CACHE_POLICIES[cache_policy] if isinstance(cache_policy, str) else int(cache_policy)
         opt.walks_override = walks_override
         opt.staging_bytes = int(staging_bytes)
+        opt.vertex_capacity = int(vertex_capacity)
         opt.flags = (FLAG_LOCAL_COUNTS if local_counts else 0) | (0 if symmetry else FLAG_NO_SYMMETRY)
         self.n = int(n)
         self._rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
@@ -163,8 +164,18 @@ class Gcsm:
     def automorphisms(self) -> int:
         return int(self._lib.gcsm_query_automorphisms(self._h))
 
+    def num_vertices(self) -> int:
+        return int(self._lib.gcsm_num_vertices(self._h))
+
+    def add_vertices(self, count, labels=None) -> int:
+        """count new isolated vertices; returns the first new id."""
+        first = ctypes.c_int32()
+        lab = None if labels is None else _i32(labels)
+        self._check(self._lib.gcsm_add_vertices(self._h, int(count), _ptr(lab), ctypes.byref(first)), "add_vertices")
+        return first.value
+
     def export_csr(self):
-        rp = np.zeros(self.n + 1, np.int64)
+        rp = np.zeros(self.num_vertices() + 1, np.int64)
         self._lib.gcsm_export_csr(self._h, _ptr(rp), None, 0)
         col = np.zeros(int(rp[-1]), np.int32)
         self._check(self._lib.gcsm_export_csr(self._h, _ptr(rp), _ptr(col), len(col)), "export_csr")
@@ -242,6 +253,16 @@ def shard(cost, world):
     if s:
         raise GcsmError(s, "bad shard arguments")
     return out
+
+
+def link_peers(contexts):
+    """NVLink peer cache (gcsm_link_peers): the contexts read each other's HBM caches; drive each from its own
+    host thread, in lockstep. An empty or one-element list unlinks."""
+    arr = (ctypes.c_void_p * max(len(contexts), 1))(*[c._h.value if hasattr(c._h, "value") else c._h
+                                                       for c in contexts])
+    s = _lib.load().gcsm_link_peers(arr, len(contexts))
+    if s:
+        raise GcsmError(s, "gcsm_link_peers")
 
 
 def binomial_samples(key0, n, p, count):

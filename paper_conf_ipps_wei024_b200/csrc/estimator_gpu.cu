@@ -222,6 +222,10 @@ struct WalkArgs {
   uint32_t *touched;
   unsigned long long *cursor;
   BinTab T;
+  StageRef stage;            // fetch-once staging (stage.state == nullptr: off)
+  uint32_t stage_min;
+  unsigned long long *stage_cnt;
+  const char *dev_lo[2], *dev_hi[2];
 };
 
 constexpr int kEW = 8;  // warps per block
@@ -231,6 +235,7 @@ struct EstLv {
   unsigned long long T53;  // BINV's first-uniform threshold floor(r0 2^53) of this node (all ones: no shortcut)
   const int32_t *dm, *dx;  // the node's driver list (main, delta segment), fixed at node entry
   uint32_t dml, dxl;
+  const int32_t *pm[7];    // every backward main list as read (staged copy when zero-copy and staging is on)
   int32_t sv[32];
   unsigned long long sB[32], skey[32];
 };
@@ -329,11 +334,19 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
   const int lane = threadIdx.x & 31;
   EstW &W = sw[threadIdx.x >> 5];
   const unsigned long long n2 = min(*(volatile unsigned long long *)A.f2_count, (unsigned long long)A.f2_cap);
+  unsigned long long wfill = 0, wlists = 0, whit = 0;  // fetch-once staging counters
   for (;;) {
     unsigned long long u = 0;
     if (lane == 0) u = atomicAdd(A.cursor2, 1ull);
     u = __shfl_sync(FULL, u, 0);
-    if (u >= n2) return;
+    if (u >= n2) {
+      if (lane == 0 && A.stage_cnt && (wfill | wlists | whit)) {
+        atomicAdd(A.stage_cnt + 0, wfill);
+        atomicAdd(A.stage_cnt + 1, wlists);
+        atomicAdd(A.stage_cnt + 2, whit);
+      }
+      return;
+    }
     const EstNode2 N = A.f2[u];
     const DevPlan *P = A.plans + N.plan;
     const int k = P->k;
@@ -370,12 +383,18 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
         uint32_t best = 0xffffffffu;
         for (int b = 0; b < nb; ++b) {
           L[b] = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
+          const char *pc = reinterpret_cast<const char *>(L[b].m);
+          if (A.stage.state && L[b].ml >= A.stage_min && !(pc >= A.dev_lo[0] && pc < A.dev_hi[0]) &&
+              !(pc >= A.dev_lo[1] && pc < A.dev_hi[1]))  // zero-copy: fetched once per batch into HBM
+            L[b].m = stage_fetch(A.stage, W.f[Lp.bpos[b]], L[b].m, L[b].ml, wfill, wlists, whit, lane);
           const uint32_t t = L[b].ml + L[b].xl;
           if (t < best) {
             best = t;
             drv = b;
           }
         }
+        if (lane == 0)
+          for (int b = 0; b < nb; ++b) S.pm[b] = L[b].m;
         const int64_t Bn = (int64_t)S.B;
         const double pD = T.pD;
         unsigned long long t53 = ~0ull;
@@ -455,9 +474,10 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
         for (int b = 0; b < nb; ++b) {
           if (b == drv) continue;
           const LR Lb = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
+          const int32_t *bm = S.pm[b];
 #pragma unroll 1
           for (int j = 0; j < 4; ++j)
-            if (ok[j]) ok[j] = has(Lb.m, Lb.ml, v[j]) || (Lb.xl && has(Lb.x, Lb.xl, v[j]));
+            if (ok[j]) ok[j] = has(bm, Lb.ml, v[j]) || (Lb.xl && has(Lb.x, Lb.xl, v[j]));
         }
       }
       // whole chunks while their survivors fit the 32-entry buffer (chunk 0 always does); the rest is redone
@@ -839,6 +859,13 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.T.r0n = c.r0n;
       A.T.sfc = c.sfc_dev;
       A.T.err = &c.st->err;
+      A.stage = c.stage;
+      A.stage_min = c.stage_min;
+      A.stage_cnt = c.stage_cnt;
+      for (int r = 0; r < 2; ++r) {
+        A.dev_lo[r] = c.dev_lo[r];
+        A.dev_hi[r] = c.dev_hi[r];
+      }
       const int ga = (int)std::max<int64_t>(1, std::min<int64_t>((Q.n_items + kEW - 1) / kEW, 148 * 8));
       LK(k_walks_l1<<<ga, kEW * 32, 0, s>>>(A));
       if (Q.k >= 5) LK(k_walks<<<148 * 2, kEW * 32, 0, s>>>(A));

@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 
 #include "internal.h"
+#include "stage.cuh"
 
 namespace gcsm {
 
@@ -92,6 +93,12 @@ struct CacheStep {
   char *cache;              // this batch's buffer (written)
   // stats
   unsigned long long *cnt_cached;  // 3 counters: vertices, bytes, internal error
+  // fetch-once staging of the walks' zero-copy lists (stage.state == nullptr: off); lists already in device memory
+  // at walk time (the last batch's cache, the batch's U lists) are read in place
+  StageRef stage{};
+  uint32_t stage_min = 1;
+  unsigned long long *stage_cnt = nullptr;  // fill bytes, lists, hit bytes
+  const char *dev_lo[2] = {nullptr, nullptr}, *dev_hi[2] = {nullptr, nullptr};
 };
 
 size_t cache_step_tmp_bytes(int32_t n);

@@ -8,7 +8,9 @@
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
+#include <condition_variable>
 #include <cstring>
+#include <memory>
 #include <mutex>
 #include <new>
 #include <numeric>
@@ -19,6 +21,7 @@
 #include "internal.h"
 #include "estimator_gpu.cuh"
 #include "kernels.cuh"
+#include "stage.cuh"
 #include "store.h"
 
 using namespace gcsm;
@@ -68,6 +71,17 @@ bool host_ensure(T *&p, size_t &cap, size_t need) {
   cap = n;
   return true;
 }
+
+// NVLink peer cache: contexts linked by gcsm_link_peers read each other's HBM caches. The
+// per-batch rendezvous below orders the cross-context reads: a context's matching of batch t starts
+// after every peer's cache step of batch t (their descriptors and cache are final), and a context's cache step of
+// batch t+2 (which rewrites the slot and buffer of batch t) waits for every peer's batch t.
+struct PeerGroup {
+  std::mutex mu;
+  std::condition_variable cv;
+  std::vector<gcsm_ctx *> members;
+  std::vector<uint64_t> enq;  // per member: batches whose cache step has been enqueued
+};
 
 }  // namespace
 
@@ -134,6 +148,7 @@ struct gcsm_ctx {
     int32_t *tup_add = nullptr, *tup_rem = nullptr, *d_tadd = nullptr, *d_trem = nullptr;
     uint64_t add_cap = 0, rem_cap = 0;
     std::vector<std::pair<int32_t *, uint32_t>> retired;  // host arrays replaced by this batch's merge
+    const char *cache_lo = nullptr, *cache_hi = nullptr;  // the HBM cache this batch's kernels read (peers too)
   };
   Slot slots[2];
   uint64_t waited = 0;  // batches whose results have been collected
@@ -165,6 +180,7 @@ struct gcsm_ctx {
   int64_t *d_pidx = nullptr; size_t pidx_cap = 0;
   VDesc *d_pval = nullptr; size_t pval_cap = 0;
   int32_t *d_tup = nullptr; size_t tup_cap = 0;
+  unsigned long long *d_red = nullptr; size_t red_cap = 0;  // packed (added, removed) of every query: one allreduce
   int32_t *d_arena = nullptr; size_t arena_cap = 0;     // level-3 work sharing (k >= 5)
   Task *d_tasks = nullptr; size_t tasks_cap = 0;
   int32_t *d_task_ready = nullptr; size_t task_ready_cap = 0;
@@ -208,6 +224,8 @@ struct gcsm_ctx {
   unsigned long long *d_stage_bump = nullptr;
   bool stage_failed = false;       // allocation failed once: stay off
   uint32_t stage_min = 1;          // shortest list (ints) routed through the arena (GCSM_STAGE_MIN)
+  uint32_t walk_stage_epoch = 0;   // this batch's walks stage through the arena too (0 = no)
+  int32_t stage_policy = 1;        // smem staging model for device-resident probe lists (GCSM_STAGE_POLICY)
   // B_comp measurement mode (GCSM_BCOMP=1 at create): bitmap of the vertices whose main list a query's kernels read
   uint32_t *d_touched_bc = nullptr;
   bool bcomp = false;
@@ -221,6 +239,8 @@ struct gcsm_ctx {
   uint64_t batch_seq = 0;
   std::vector<int32_t> degree_order;  // GCSM_CACHE_DEGREE ranking
 
+  std::shared_ptr<PeerGroup> peers;  // gcsm_link_peers
+  int peer_idx = -1;
   bool in_batch = false;  // between a successful normalise and the end of submit: failures poison the ctx
   gcsm_status fail(gcsm_status s, const std::string &m) {
     err = m;
@@ -239,14 +259,17 @@ struct gcsm_ctx {
     if (e_ != cudaSuccess) return ctx->cuda_fail(e_, #call); \
   } while (0)
 
+static void peer_leave(gcsm_ctx *ctx);
+
 gcsm_ctx::~gcsm_ctx() {
+  peer_leave(this);
   if (stream) cudaStreamSynchronize(stream);
   if (comm) ncclCommDestroy(comm);
   for (Query &q : qs)
     for (DevPlan *p : {q.d_plans, q.d_splans})
       if (p) cudaFree(p);
   if (stream3) cudaStreamSynchronize(stream3);
-  void *dev[] = {d_lab, d_scratch, d_cachebuf[0],
+  void *dev[] = {d_lab, d_scratch, d_red, d_cachebuf[0],
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (int q = 0; q < GCSM_MAX_QUERIES; ++q) {
     if (d_f2q[q]) cudaFree(d_f2q[q]);
@@ -283,6 +306,18 @@ gcsm_ctx::~gcsm_ctx() {
   if (stream) cudaStreamDestroy(stream);
   if (stream2) cudaStreamDestroy(stream2);
   if (stream3) cudaStreamDestroy(stream3);
+}
+
+// Leaves the peer group (the remaining members are unlinked too: a group is all or nothing).
+static void peer_leave(gcsm_ctx *ctx) {
+  if (!ctx || !ctx->peers) return;
+  std::shared_ptr<PeerGroup> pg = ctx->peers;
+  std::lock_guard<std::mutex> lk(pg->mu);
+  for (gcsm_ctx *p : pg->members) {
+    p->peers.reset();
+    p->peer_idx = -1;
+  }
+  pg->members.clear();
 }
 
 extern "C" {
@@ -334,7 +369,12 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   }
   ctx->device = dev;
   bool cuda_err = false;
-  std::string e = ctx->store.init(n, row_ptr, col, labels, threads, &cuda_err);
+  if (o.vertex_capacity < 0 || o.vertex_capacity > INT32_MAX) {
+    delete ctx;
+    return GCSM_EINVAL;
+  }
+  const int32_t ncap = (int32_t)std::max<int64_t>(n, o.vertex_capacity);
+  std::string e = ctx->store.init(n, row_ptr, col, labels, threads, &cuda_err, ncap);
   if (!e.empty()) {
     delete ctx;
     return cuda_err ? GCSM_EDEVICE : GCSM_EINVAL;
@@ -364,32 +404,33 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
       return bail(GCSM_ENOMEM);
   }
   for (auto &sl : ctx->slots)
-    if (cudaMalloc(&sl.d_vdesc, sizeof(VDesc) * (size_t)n) != cudaSuccess ||
+    if (cudaMalloc(&sl.d_vdesc, sizeof(VDesc) * (size_t)ncap) != cudaSuccess ||
         cudaMalloc(&sl.d_cnt, sizeof(unsigned long long) * CNT_N * GCSM_MAX_QUERIES) != cudaSuccess)
       return bail(GCSM_ENOMEM);
-  if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
-  if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)n + 2047) / 2048 + 1)) != cudaSuccess)
+  if (cudaMalloc(&ctx->d_hist, sizeof(uint32_t) * (size_t)ncap) != cudaSuccess) return bail(GCSM_ENOMEM);
+  if (cudaMalloc(&ctx->d_bsum, sizeof(uint32_t) * (((size_t)ncap + 2047) / 2048 + 1)) != cudaSuccess)
     return bail(GCSM_ENOMEM);
   {
-    std::vector<VDesc> vd(n);
+    std::vector<VDesc> vd(ncap, VDesc{nullptr, 0, 0});  // ids [n, ncap): empty until they join
     for (int32_t v = 0; v < n; ++v) vd[v] = VDesc{ctx->store.dev_ptr(ctx->store.lst[v]), ctx->store.len[v], 0};
     for (auto &sl : ctx->slots)
-      if (cudaMemcpy(sl.d_vdesc, vd.data(), sizeof(VDesc) * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
+      if (cudaMemcpy(sl.d_vdesc, vd.data(), sizeof(VDesc) * (size_t)ncap, cudaMemcpyHostToDevice) != cudaSuccess)
         return bail(GCSM_EDEVICE);
   }
   if (labels) {
-    if (cudaMalloc(&ctx->d_lab, 2 * (size_t)n) != cudaSuccess) return bail(GCSM_ENOMEM);
-    if (cudaMemcpy(ctx->d_lab, ctx->store.lab.data(), 2 * (size_t)n, cudaMemcpyHostToDevice) != cudaSuccess)
+    if (cudaMalloc(&ctx->d_lab, 2 * (size_t)ncap) != cudaSuccess) return bail(GCSM_ENOMEM);
+    if (cudaMemcpy(ctx->d_lab, ctx->store.lab.data(), 2 * (size_t)ncap, cudaMemcpyHostToDevice) != cudaSuccess)
       return bail(GCSM_EDEVICE);
   }
-  ctx->mark.assign(n, 0);
-  ctx->slot16.assign(n, 0);
+  ctx->mark.assign(ncap, 0);
+  ctx->slot16.assign(ncap, 0);
   for (int q = 0; q < GCSM_MAX_QUERIES; ++q) ctx->lev_levels[q] = -1;
   if (const char *he = std::getenv("GCSM_HOST_EST")) ctx->gpu_est = std::atoi(he) == 0;
   ctx->overlap = ctx->gpu_est && !std::getenv("GCSM_NO_OVERLAP");
   if (const char *ok = std::getenv("GCSM_OVERLAP_KMAX")) ctx->overlap_kmax = std::atoi(ok);
   if (const char *sm = std::getenv("GCSM_STAGE_MB")) ctx->opt.staging_bytes = std::strtoull(sm, nullptr, 10) << 20;
   if (const char *sm = std::getenv("GCSM_STAGE_MIN")) ctx->stage_min = (uint32_t)std::max(1, std::atoi(sm));
+  if (const char *sp = std::getenv("GCSM_STAGE_POLICY")) ctx->stage_policy = std::atoi(sp);
   if (std::getenv("GCSM_BCOMP") && gcsm_set_measure(ctx, GCSM_MEASURE_BCOMP) != GCSM_OK) return bail(GCSM_ENOMEM);
   ctx->grid = match_grid(dev, &ctx->warps_total);
   ctx->ext_grid = ctx->grid;
@@ -407,13 +448,76 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
 
 void gcsm_destroy(gcsm_ctx *ctx) { delete ctx; }
 
+int32_t gcsm_num_vertices(const gcsm_ctx *ctx) { return ctx ? ctx->store.n : 0; }
+
+gcsm_status gcsm_link_peers(gcsm_ctx *const *ctxs, int32_t n) {
+  if (n < 0 || n > GCSM_MAX_PEERS + 1 || (n > 0 && !ctxs)) return GCSM_EINVAL;
+  for (int32_t i = 0; i < n; ++i) {
+    if (!ctxs[i]) return GCSM_EINVAL;
+    if (ctxs[i]->poisoned) return GCSM_ESTATE;
+    if (ctxs[i]->waited != ctxs[i]->batch_seq) return ctxs[i]->fail(GCSM_ESTATE, "link_peers with a batch in flight");
+    for (int32_t j = 0; j < i; ++j)
+      if (ctxs[j] == ctxs[i]) return GCSM_EINVAL;
+    if (ctxs[i]->store.ncap != ctxs[0]->store.ncap || ctxs[i]->batch_seq != ctxs[0]->batch_seq)
+      return ctxs[i]->fail(GCSM_EINVAL, "linked contexts need the same vertex capacity and batch count");
+  }
+  for (int32_t i = 0; i < n; ++i) peer_leave(ctxs[i]);
+  if (n < 2) return GCSM_OK;
+  for (int32_t i = 0; i < n; ++i)  // peer access between distinct devices (NVLink through NVSwitch)
+    for (int32_t j = 0; j < n; ++j) {
+      const int di = ctxs[i]->device, dj = ctxs[j]->device;
+      if (di == dj) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, di, dj);
+      if (!can) return ctxs[i]->fail(GCSM_EDEVICE, "no peer access between the linked devices");
+      cudaSetDevice(di);
+      const cudaError_t e = cudaDeviceEnablePeerAccess(dj, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return ctxs[i]->cuda_fail(e, "peer access");
+      cudaGetLastError();
+    }
+  auto pg = std::make_shared<PeerGroup>();
+  pg->members.assign(ctxs, ctxs + n);
+  pg->enq.assign((size_t)n, ctxs[0]->batch_seq);
+  for (int32_t i = 0; i < n; ++i) {
+    ctxs[i]->peers = pg;
+    ctxs[i]->peer_idx = i;
+    cudaSetDevice(ctxs[i]->device);
+  }
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_add_vertices(gcsm_ctx *ctx, int32_t count, const int32_t *labels, int32_t *first_id) {
+  if (!ctx || count < 0) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "add_vertices with a batch in flight");
+  HostStore &S = ctx->store;
+  if ((int64_t)S.n + count > (int64_t)S.ncap) return ctx->fail(GCSM_EINVAL, "vertex capacity exceeded");
+  if (labels) {
+    if (S.lab.empty()) return ctx->fail(GCSM_EINVAL, "labels for new vertices of an unlabelled graph");
+    for (int32_t i = 0; i < count; ++i)
+      if (labels[i] < 0 || labels[i] > 65535) return ctx->fail(GCSM_EINVAL, "label out of [0, 65535]");
+  }
+  const int32_t first = S.n;
+  if (!S.grow(S.n + count)) return ctx->fail(GCSM_ENOMEM, "pinned allocation for new vertices failed");
+  if (labels) {
+    for (int32_t i = 0; i < count; ++i) S.lab[first + i] = (uint16_t)labels[i];
+    if (ctx->d_lab) {
+      if (cudaSetDevice(ctx->device) != cudaSuccess) return ctx->fail(GCSM_EDEVICE, "cudaSetDevice");
+      CK(cudaMemcpy(ctx->d_lab + first, S.lab.data() + first, 2 * (size_t)count, cudaMemcpyHostToDevice));
+    }
+  }
+  if (first_id) *first_id = first;
+  ctx->err.clear();
+  return GCSM_OK;
+}
+
 gcsm_status gcsm_set_measure(gcsm_ctx *ctx, uint32_t flags) {
   if (!ctx || (flags & ~(uint32_t)GCSM_MEASURE_BCOMP)) return GCSM_EINVAL;
   if (ctx->poisoned) return GCSM_ESTATE;
   const bool on = (flags & GCSM_MEASURE_BCOMP) != 0;
   if (on && !ctx->d_touched_bc) {
     if (cudaSetDevice(ctx->device) != cudaSuccess) return GCSM_EDEVICE;
-    if (cudaMalloc(&ctx->d_touched_bc, 4 * (((size_t)ctx->store.n + 31) / 32)) != cudaSuccess) {
+    if (cudaMalloc(&ctx->d_touched_bc, 4 * (((size_t)ctx->store.ncap + 31) / 32)) != cudaSuccess) {
       cudaGetLastError();
       ctx->d_touched_bc = nullptr;
       return GCSM_ENOMEM;
@@ -443,8 +547,8 @@ static gcsm_status add_query_impl(gcsm_ctx *ctx, bool reset, int32_t k, int32_t 
   if (e.empty()) e = build_plan(k, m, qedges, qlabels, order, q.qps, !(ctx->opt.flags & GCSM_FLAG_NO_SYMMETRY));
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
   if (q.qp.labelled && !ctx->d_lab) {  // unlabelled graph: every data label is 0 (R5)
-    CK(cudaMalloc(&ctx->d_lab, 2 * (size_t)ctx->store.n));
-    CK(cudaMemset(ctx->d_lab, 0, 2 * (size_t)ctx->store.n));
+    CK(cudaMalloc(&ctx->d_lab, 2 * (size_t)ctx->store.ncap));
+    CK(cudaMemset(ctx->d_lab, 0, 2 * (size_t)ctx->store.ncap));
   }
   const size_t slot = reset ? 0 : ctx->qs.size();
   DevPlan *dp = slot < ctx->qs.size() ? ctx->qs[slot].d_plans : nullptr;
@@ -586,30 +690,31 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   HostStore &S = ctx->store;
   const int32_t n = S.n;
   const int nq = (int)ctx->qs.size();
-  if (!ctx->gpu_ready) {
-    const size_t W = ((size_t)n + 31) / 32 + 1;
-    std::vector<unsigned long long> hp((size_t)n);
+  if (!ctx->gpu_ready) {  // n-sized buffers at the vertex capacity (ids may grow into it)
+    const int32_t nc = S.ncap;
+    const size_t W = ((size_t)nc + 31) / 32 + 1;
+    std::vector<unsigned long long> hp((size_t)nc, 0ull);
     for (int32_t v = 0; v < n; ++v) hp[v] = (unsigned long long)(uintptr_t)S.dev_ptr(S.lst[v]);
-    ctx->cubtmp_bytes = cache_step_tmp_bytes(n);
-    if (cudaMalloc(&ctx->d_hptr, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_touched, 4 * W) != cudaSuccess ||
+    ctx->cubtmp_bytes = cache_step_tmp_bytes(nc);
+    if (cudaMalloc(&ctx->d_hptr, 8 * (size_t)nc) != cudaSuccess || cudaMalloc(&ctx->d_touched, 4 * W) != cudaSuccess ||
         cudaMalloc(&ctx->d_wcnt, 4 * W) != cudaSuccess || cudaMalloc(&ctx->d_woff, 4 * W) != cudaSuccess ||
-        cudaMalloc(&ctx->d_tids, 4 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_prev_sel, 4 * (size_t)n) != cudaSuccess ||
-        cudaMalloc(&ctx->d_bits, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_bytes, 8 * (size_t)n) != cudaSuccess ||
-        cudaMalloc(&ctx->d_scan, 8 * (size_t)n) != cudaSuccess || cudaMalloc(&ctx->d_off, 8 * (size_t)n) != cudaSuccess ||
-        cudaMalloc(&ctx->d_flag, (size_t)n) != cudaSuccess ||
+        cudaMalloc(&ctx->d_tids, 4 * (size_t)nc) != cudaSuccess || cudaMalloc(&ctx->d_prev_sel, 4 * (size_t)nc) != cudaSuccess ||
+        cudaMalloc(&ctx->d_bits, 8 * (size_t)nc) != cudaSuccess || cudaMalloc(&ctx->d_bytes, 8 * (size_t)nc) != cudaSuccess ||
+        cudaMalloc(&ctx->d_scan, 8 * (size_t)nc) != cudaSuccess || cudaMalloc(&ctx->d_off, 8 * (size_t)nc) != cudaSuccess ||
+        cudaMalloc(&ctx->d_flag, (size_t)nc) != cudaSuccess ||
         cudaMalloc(&ctx->d_selhist, 8 * 6 * 4096) != cudaSuccess ||
         cudaMalloc(&ctx->d_ecursor, 8 * 3 * GCSM_MAX_QUERIES) != cudaSuccess ||
         cudaMalloc(&ctx->d_sel, sizeof(SelState)) != cudaSuccess ||
         cudaMalloc(&ctx->d_cubtmp, ctx->cubtmp_bytes) != cudaSuccess)
       return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
-    CK(cudaMemcpyAsync(ctx->d_hptr, hp.data(), 8 * (size_t)n, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->d_hptr, hp.data(), 8 * (size_t)nc, cudaMemcpyHostToDevice, s));
     double sfc[10];
     for (int i = 0; i < 10; ++i) sfc[i] = stirling_small(i);
     if (cudaMalloc(&ctx->d_sfc, sizeof sfc) != cudaSuccess) return ctx->fail(GCSM_ENOMEM, "GPU estimator buffers");
     CK(cudaMemcpyAsync(ctx->d_sfc, sfc, sizeof sfc, cudaMemcpyHostToDevice, s));
     {  // sampled index of every list of >= 64 elements
-      ctx->soff_h.assign((size_t)n, 0xffffffffu);
-      ctx->scap_h.assign((size_t)n, 0);
+      ctx->soff_h.assign((size_t)nc, 0xffffffffu);
+      ctx->scap_h.assign((size_t)nc, 0);
       size_t total = 0;
       for (int32_t v = 0; v < n; ++v)
         if (S.len[v] >= 64) {
@@ -627,10 +732,10 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
             for (uint32_t j = 0; 32 * j < S.len[v]; ++j) smp[ctx->soff_h[v] + j] = S.lst[v][32 * j];
       });
       if (ctx->sidx_capacity >= ((size_t)1 << 31) || cudaMalloc(&ctx->d_sidx, 4 * ctx->sidx_capacity) != cudaSuccess ||
-          cudaMalloc(&ctx->d_soff, 4 * (size_t)n) != cudaSuccess)
+          cudaMalloc(&ctx->d_soff, 4 * (size_t)nc) != cudaSuccess)
         return ctx->fail(GCSM_ENOMEM, "sampled list index");
       CK(cudaMemcpyAsync(ctx->d_sidx, smp.data(), 4 * total, cudaMemcpyHostToDevice, s));
-      CK(cudaMemcpyAsync(ctx->d_soff, ctx->soff_h.data(), 4 * (size_t)n, cudaMemcpyHostToDevice, s));
+      CK(cudaMemcpyAsync(ctx->d_soff, ctx->soff_h.data(), 4 * (size_t)nc, cudaMemcpyHostToDevice, s));
       CK(cudaStreamSynchronize(s));  // pageable sources
     }
     CK(cudaMemsetAsync(ctx->d_sel, 0, sizeof(SelState), s));
@@ -643,9 +748,9 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
     if (L <= 0 || ctx->lev_levels[qi] == L) continue;
     if (ctx->d_levcnt[qi]) cudaFree(ctx->d_levcnt[qi]);
     ctx->d_levcnt[qi] = nullptr;
-    if (cudaMalloc(&ctx->d_levcnt[qi], 8 * (size_t)n * L) != cudaSuccess)
+    if (cudaMalloc(&ctx->d_levcnt[qi], 8 * (size_t)S.ncap * L) != cudaSuccess)
       return ctx->fail(GCSM_ENOMEM, "estimator sums");
-    CK(cudaMemsetAsync(ctx->d_levcnt[qi], 0, 8 * (size_t)n * L, s));
+    CK(cudaMemsetAsync(ctx->d_levcnt[qi], 0, 8 * (size_t)S.ncap * L, s));
     ctx->lev_levels[qi] = L;
   }
   // binomial tables: BINV's r0 = (1 - 1/D)^n (host pow, as the host walker computes it) for n up to the largest
@@ -790,6 +895,16 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.cub_tmp_bytes = ctx->cubtmp_bytes;
   c.cache = ctx->d_cache;
   c.cnt_cached = sl.d_cnt + CNT_CACHED;
+  if (ctx->walk_stage_epoch && !std::getenv("GCSM_NO_WALK_STAGE")) {  // the walks' zero-copy lists through the arena
+    c.stage = StageRef{ctx->d_stage_state, ctx->d_stage_arena, ctx->stage_cap, ctx->d_stage_bump,
+                       ctx->walk_stage_epoch};
+    c.stage_min = ctx->stage_min;
+    c.stage_cnt = sl.d_cnt + CNT_STAGE_FILL;  // query 0's counters
+    c.dev_lo[0] = ctx->cache_valid ? ctx->d_cachebuf[ctx->cache_cur] : nullptr;  // lists cached by the last batch
+    c.dev_hi[0] = c.dev_lo[0] ? c.dev_lo[0] + ctx->cache_cap : nullptr;
+    c.dev_lo[1] = reinterpret_cast<const char *>(sl.d_ulist);  // the batch's U lists
+    c.dev_hi[1] = reinterpret_cast<const char *>(sl.d_ulist + sl.ulist_n);
+  }
   CK(launch_cache_step(c, s, launches));
   ctx->est_valid = est_on;
   CK(cudaEventRecord(sl.ev_c1, s));
@@ -840,6 +955,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   std::string e = S.normalize(n_ins, ins, n_del, del);
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
   ctx->in_batch = true;
+  if (S.grow_n > S.n && !S.grow(S.grow_n))  // new vertices named by the insertions
+    return ctx->fail(GCSM_ENOMEM, "pinned allocation for new vertices failed");
   tr.mark("normalize");
   bool cuda_err = false;
   if (!S.build_overlay((int)(ctx->batch_seq & 1), &cuda_err))
@@ -1237,7 +1354,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       for (int64_t i = lo; i < hi; ++i) ctx->mark[dirty[i]] = 0;
     });
   }
-  if (ctx->sel_index.size() != (size_t)S.n) ctx->sel_index.assign(S.n, -1);
+  if (ctx->sel_index.size() != (size_t)S.ncap) ctx->sel_index.assign(S.ncap, -1);
   for (size_t i = 0; i < sel.size(); ++i) ctx->sel_index[sel[i]] = (int32_t)i;
   if (!host_ensure(sl.h_pidx, sl.h_pidx_cap, dirty.size()) ||
       !host_ensure(sl.h_pval, sl.h_pval_cap, dirty.size()))
@@ -1307,6 +1424,46 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
       !dev_ensure(sl.d_drec, sl.drec_cap, nU) || !dev_ensure(sl.d_dlist, sl.dlist_cap, nd) ||
       !dev_ensure(sl.d_units, sl.units_cap, (size_t)gnu) || !dev_ensure(sl.d_useg, sl.useg_cap, (size_t)gnu))
     return ctx->fail(GCSM_ENOMEM, "device buffers");
+  if (ctx->peers && ctx->batch_seq >= 2) {  // peers may still read this slot's descriptors and cache (batch t-2)
+    std::lock_guard<std::mutex> lk(ctx->peers->mu);
+    for (gcsm_ctx *p : ctx->peers->members)
+      if (p != ctx) CK(cudaStreamWaitEvent(cs, p->slots[ctx->batch_seq & 1].ev_done, 0));
+  }
+  // fetch-once staging (k >= 5 extension kernels, and the walks when the cache step shares the context stream):
+  // allocated when first needed; this batch's epoch and an empty arena (the bump counter is reset on the context
+  // stream, after the previous batch's kernels and before this batch's walks / matching)
+  const bool staging = kmax >= 5 && !listing && ctx->opt.staging_bytes != 1 && !ctx->stage_failed;
+  uint32_t stage_epoch = 0;
+  if (staging) {
+    if (!ctx->d_stage_arena) {
+      size_t freeb = 0, totalb = 0;
+      cudaMemGetInfo(&freeb, &totalb);
+      size_t bytes = ctx->opt.staging_bytes ? ctx->opt.staging_bytes : std::min<size_t>(freeb / 4, (size_t)16 << 30);
+      bytes &= ~(size_t)127;
+      if (bytes < 4096 || cudaMalloc(&ctx->d_stage_arena, bytes) != cudaSuccess ||
+          cudaMalloc(&ctx->d_stage_state, 8 * (size_t)S.ncap) != cudaSuccess ||
+          cudaMalloc(&ctx->d_stage_bump, 8) != cudaSuccess) {
+        cudaGetLastError();
+        for (void *p : {(void *)ctx->d_stage_arena, (void *)ctx->d_stage_state, (void *)ctx->d_stage_bump})
+          if (p) cudaFree(p);
+        ctx->d_stage_arena = nullptr;
+        ctx->d_stage_state = nullptr;
+        ctx->d_stage_bump = nullptr;
+        ctx->stage_failed = true;
+      } else {
+        ctx->stage_cap = bytes / 4;
+        CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.ncap, s));
+      }
+    }
+    if (ctx->d_stage_arena) {
+      stage_epoch = (uint32_t)(ctx->batch_seq % ((1u << 24) - 1)) + 1;  // 24 bits, never 0
+      if (stage_epoch == 1 && ctx->batch_seq > 0) CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.ncap, s));
+      CK(cudaMemsetAsync(ctx->d_stage_bump, 0, 8, s));
+    }
+  }
+
+  ctx->walk_stage_epoch = (stage_epoch && ctx->gpu_est && !two_streams) ? stage_epoch : 0;
+
   CK(cudaEventRecord(sl.ev_c0, cs));
   if (ctx->batch_seq > 0)  // this batch's descriptors start as the previous batch's (after its cache step)
     CK(cudaMemcpyAsync(sl.d_vdesc, ctx->slots[(ctx->batch_seq + 1) & 1].d_vdesc, sizeof(VDesc) * (size_t)S.n,
@@ -1352,42 +1509,32 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   CK(cudaMemsetAsync(sl.d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
   }
   if (cs != s) CK(cudaStreamWaitEvent(s, sl.ev_c1, 0));  // the matching kernels read the cache step's output
-
-  // fetch-once staging (k >= 5 extension kernels): allocated when first needed; this batch's epoch and an empty
-  // arena (the bump counter is reset on the context stream, after the previous batch's kernels)
-  const bool staging = kmax >= 5 && !listing && ctx->opt.staging_bytes != 1 && !ctx->stage_failed;
-  uint32_t stage_epoch = 0;
-  if (staging) {
-    if (!ctx->d_stage_arena) {
-      size_t freeb = 0, totalb = 0;
-      cudaMemGetInfo(&freeb, &totalb);
-      size_t bytes = ctx->opt.staging_bytes ? ctx->opt.staging_bytes : std::min<size_t>(freeb / 4, (size_t)16 << 30);
-      bytes &= ~(size_t)127;
-      if (bytes < 4096 || cudaMalloc(&ctx->d_stage_arena, bytes) != cudaSuccess ||
-          cudaMalloc(&ctx->d_stage_state, 8 * (size_t)S.n) != cudaSuccess ||
-          cudaMalloc(&ctx->d_stage_bump, 8) != cudaSuccess) {
-        cudaGetLastError();
-        for (void *p : {(void *)ctx->d_stage_arena, (void *)ctx->d_stage_state, (void *)ctx->d_stage_bump})
-          if (p) cudaFree(p);
-        ctx->d_stage_arena = nullptr;
-        ctx->d_stage_state = nullptr;
-        ctx->d_stage_bump = nullptr;
-        ctx->stage_failed = true;
-      } else {
-        ctx->stage_cap = bytes / 4;
-        CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.n, s));
+  sl.cache_lo = ctx->d_cache;
+  sl.cache_hi = ctx->d_cache ? ctx->d_cache + ctx->cache_cap : nullptr;
+  // peer cache: rendezvous with the linked contexts at batch t (each has enqueued its cache step of t), then this
+  // context's matching waits for theirs
+  int npeer = 0;
+  gcsm_ctx *peer_of[GCSM_MAX_PEERS] = {};
+  if (ctx->peers) {
+    PeerGroup &pg = *ctx->peers;
+    std::unique_lock<std::mutex> lk(pg.mu);
+    pg.enq[ctx->peer_idx] = ctx->batch_seq + 1;
+    pg.cv.notify_all();
+    pg.cv.wait(lk, [&] {
+      for (uint64_t x : pg.enq)
+        if (x < ctx->batch_seq + 1) return false;
+      return true;
+    });
+    for (gcsm_ctx *p : pg.members)
+      if (p != ctx && npeer < GCSM_MAX_PEERS) {
+        CK(cudaStreamWaitEvent(s, p->slots[ctx->batch_seq & 1].ev_c1, 0));
+        peer_of[npeer++] = p;
       }
-    }
-    if (ctx->d_stage_arena) {
-      stage_epoch = (uint32_t)(ctx->batch_seq % ((1u << 24) - 1)) + 1;  // 24 bits, never 0
-      if (stage_epoch == 1 && ctx->batch_seq > 0) CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.n, s));
-      CK(cudaMemsetAsync(ctx->d_stage_bump, 0, 8, s));
-    }
   }
 
   // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
-  const int nbuf = std::max(1, std::max(kmax - 4, 0) + (listing ? 1 : 0));
+  const int nbuf = std::max(1, std::max(kmax - 4, 0) + (listing ? 1 : 0) + (kmax >= 5 ? 1 : 0));  // + hoisted set
   const size_t stride = (size_t)(nbuf + 3) * (size_t)dcap;  // stacks + pinned-x2 + 2 HBM staging buffers
   if (!dev_ensure(ctx->d_scratch, ctx->scratch_cap, stride * (size_t)ctx->warps_total))
     return ctx->fail(GCSM_ENOMEM, "scratch");
@@ -1467,6 +1614,14 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     A.stage_min = ctx->stage_min;
   }
   A.touched = ctx->bcomp ? ctx->d_touched_bc : nullptr;
+  A.stage_policy = ctx->stage_policy;
+  A.npeer = npeer;
+  for (int p = 0; p < npeer; ++p) {
+    const gcsm_ctx::Slot &ps = peer_of[p]->slots[ctx->batch_seq & 1];
+    A.peer_vdesc[p] = ps.d_vdesc;
+    A.peer_lo[p] = ps.cache_lo;
+    A.peer_hi[p] = ps.cache_hi;
+  }
   if (kmax >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
     const size_t na = (size_t)64 << 20, nt = (size_t)4 << 20;
     const bool fresh_ready = ctx->d_task_ready == nullptr;
@@ -1582,12 +1737,13 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   }
   // ---- (4b) count allreduce over NVLink (world > 1) -------------------------------------
   CK(cudaEventRecord(sl.ev_a0, s));
-  if (ctx->comm) {
-    for (int qi = 0; qi < nq; ++qi) {
-      unsigned long long *qcnt = sl.d_cnt + (size_t)qi * CNT_N;
-      if (ncclAllReduce(qcnt, qcnt, 2, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
-        return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
-    }
+  if (ctx->comm) {  // ONE allreduce for every standing query: (added, removed) gathered into a packed buffer
+    if (!dev_ensure(ctx->d_red, ctx->red_cap, 2 * (size_t)nq)) return ctx->fail(GCSM_ENOMEM, "allreduce buffer");
+    const size_t pitch = sizeof(unsigned long long) * CNT_N, w16 = 2 * sizeof(unsigned long long);
+    CK(cudaMemcpy2DAsync(ctx->d_red, w16, sl.d_cnt, pitch, w16, (size_t)nq, cudaMemcpyDeviceToDevice, s));
+    if (ncclAllReduce(ctx->d_red, ctx->d_red, 2 * (size_t)nq, ncclUint64, ncclSum, ctx->comm, s) != ncclSuccess)
+      return ctx->fail(GCSM_ENCCL, "ncclAllReduce failed");
+    CK(cudaMemcpy2DAsync(sl.d_cnt, pitch, ctx->d_red, w16, w16, (size_t)nq, cudaMemcpyDeviceToDevice, s));
   }
   CK(cudaEventRecord(sl.ev_a1, s));
   CK(cudaMemcpyAsync(sl.h_cnt, sl.d_cnt, sizeof(unsigned long long) * CNT_N * (size_t)nq, cudaMemcpyDeviceToHost,
@@ -1681,6 +1837,7 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.miss_bytes = h[CNT_ACC_L2 + 1] + st.miss_bytes_ext;
     st.delta_bytes = h[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
     st.host_copied_bytes = h[CNT_COPIED] + h[CNT_STAGE_FILL];  // warp staging copies + arena fills
+    st.peer_bytes = h[CNT_PEER];
     st.stage_fill_bytes = h[CNT_STAGE_FILL];
     st.stage_lists = h[CNT_STAGE_LISTS];
     st.stage_hit_bytes = h[CNT_STAGE_HIT];
@@ -1690,9 +1847,10 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.d2h_bytes = sizeof(unsigned long long) * CNT_N * (size_t)nq;
     st.frontier = h[CNT_F2];
     if (std::getenv("GCSM_TRACE"))
-      std::fprintf(stderr, "[gcsm kern] q=%d frontier=%llu runs=%llu pins=%llu pin_gb=%.3f split_gb=%.3f copied_gb=%.3f\n",
+      std::fprintf(stderr, "[gcsm kern] q=%d frontier=%llu runs=%llu pins=%llu pin_gb=%.3f split_gb=%.3f copied_gb=%.3f "
+                   "entries=%llu pruned=%llu l3=%llu l4=%llu last_drv=%llu\n",
                    qi, h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_DBG_SPLIT] / 1e9,
-                   h[CNT_COPIED] / 1e9);
+                   h[CNT_COPIED] / 1e9, h[CNT_X_ENTRIES], h[CNT_X_PRUNED], h[CNT_X_L3], h[CNT_X_L4], h[CNT_X_LAST]);
     if (qi == 0 && (sl.tup_add || sl.tup_rem)) {
       const int k = ctx->qs[0].qp.k;
       const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);

@@ -22,6 +22,7 @@
 #define GCSM_MAXK 8
 #define GCSM_MAXM 28
 #define GCSM_MAXPLANS (2 * GCSM_MAXM)
+#define GCSM_MAX_PEERS 7     // linked peer contexts whose HBM caches a context reads (gcsm_link_peers)
 #define GCSM_MAX_QUERIES 32  // standing queries per context (gcsm_add_query; all 29 connected 3-5-vertex motifs fit)
 
 namespace gcsm {
@@ -59,6 +60,9 @@ struct LevelPlan {
   int8_t inj[7];
   int8_t nlo, lo[7];   // symmetry breaking: f(order[p]) > f(position lo[i])
   int8_t nhi, hi[7];   //                    f(order[p]) < f(position hi[i])
+  int8_t hmask;        // last position (k >= 5) only: backward lists (bit b = bpos[b]) whose positions are <= 2,
+                       // i.e. fixed once a level-2 partial match is chosen; their intersection is hoisted to the
+                       // level-2 entry (loop-invariant code motion): empty -> the entry's subtree holds no match
   int32_t label;       // required data label of order[p], -1 = any
 };
 

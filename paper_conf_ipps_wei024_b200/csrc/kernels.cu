@@ -28,6 +28,7 @@
 #include <cstdio>
 
 #include "kernels.cuh"
+#include "stage.cuh"
 
 namespace gcsm {
 
@@ -88,100 +89,29 @@ struct LRef {
 struct Acc {
   unsigned long long add = 0, rem = 0, hit = 0, miss = 0, delta = 0, copied = 0;
   unsigned long long sfill = 0, slists = 0, shit = 0;  // fetch-once staging: bytes filled, lists, bytes served
+  unsigned long long peer = 0;                         // bytes read from a linked peer's HBM cache
 };
 
-// Warp-cooperative bulk copy of a list (16-byte aligned source; lists are
-// allocated in 16-byte granules so reading up to round4(n) ints stays inside
-// the allocation). 4 x 16 B loads per lane are issued before any store, so a
-// warp keeps 2 KB in flight: a zero-copy list crosses PCIe at link speed
-// instead of one dependent 32 B sector per binary-search step.
-__device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
-  __syncwarp();  // every lane is done reading what this buffer held before (WAR across lanes)
-  const uint32_t n4 = (n + 3) >> 2;
-  const int4 *s4 = reinterpret_cast<const int4 *>(src);
-  int4 *d4 = reinterpret_cast<int4 *>(dst);
-  for (uint32_t base = 0; base < n4; base += 128) {
-    const uint32_t i0 = base + lane, i1 = i0 + 32, i2 = i0 + 64, i3 = i0 + 96;
-    int4 v0, v1, v2, v3;
-    if (i0 < n4) v0 = s4[i0];
-    if (i1 < n4) v1 = s4[i1];
-    if (i2 < n4) v2 = s4[i2];
-    if (i3 < n4) v3 = s4[i3];
-    if (i0 < n4) d4[i0] = v0;
-    if (i1 < n4) d4[i1] = v1;
-    if (i2 < n4) d4[i2] = v2;
-    if (i3 < n4) d4[i3] = v3;
+// NVLink peer cache (NEXT-3): vertex v's main list in a linked peer's HBM cache for this batch, or nullptr. The
+// peers apply the same batches, so for v not updated by the batch (upd == 0) their copy of base(v) is ours; a
+// peer's descriptors and cache are final before this batch's kernels start and stay until they finish
+// (gcsm_link_peers).
+__device__ __forceinline__ const int32_t *peer_lookup(const MatchArgs &A, int32_t v, uint32_t ml) {
+  for (int p = 0; p < A.npeer; ++p) {
+    const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.peer_vdesc[p] + v));
+    const char *q = reinterpret_cast<const char *>((unsigned long long)(unsigned)raw.x |
+                                                   ((unsigned long long)(unsigned)raw.y << 32));
+    if (q >= A.peer_lo[p] && q < A.peer_hi[p] && (uint32_t)raw.z == ml && raw.w == 0)
+      return reinterpret_cast<const int32_t *>(q);
   }
+  return nullptr;
 }
-
-// ---- fetch-once staging of zero-copy lists within a batch -------------------------------------
-// The first warp of the batch that needs vertex v's zero-copy main list claims it (CAS of its state word from an
-// older epoch to "loading"), copies it over PCIe into the batch arena (bump-allocated, 128-byte granules so that
-// no two lists share an L1 line) and publishes (epoch, ready, offset); every later read of that list in the batch,
-// by any warp or any later kernel of the batch, is an HBM read. A warp that finds the list loading waits for it
-// (the loader waits on nothing, so this cannot deadlock). Arena full: the list stays zero-copy ("no room").
-// The arena holds the batch's MAIN lists (v not in U: base(v), unchanged during the batch); the next batch has a
-// new epoch, so nothing stale is ever served.
-constexpr unsigned long long kStReady = 1ull << 39, kStOff = (1ull << 39) - 1;
 
 __device__ __noinline__ const int32_t *stage_resolve(const MatchArgs &A, int32_t v, const int32_t *hp, uint32_t ml,
                                                      unsigned long long &sfill, unsigned long long &slists,
                                                      unsigned long long &shit, int lane) {
-  const unsigned long long ep = (unsigned long long)A.stage_epoch << 40;
-  unsigned long long res = 0;
-  int claimed = 0;
-  if (lane == 0) {
-    unsigned long long *w = A.stage_state + v;
-    unsigned long long cur = __ldcg(w);
-    unsigned ns = 32;
-    for (;;) {
-      if ((cur & ~((1ull << 40) - 1)) == ep) {  // this batch's: ready, no room, or being loaded
-        if (cur & kStReady) {
-          res = cur & kStOff;
-          break;
-        }
-        __nanosleep(ns);
-        if (ns < 2048) ns <<= 1;
-        cur = __ldcg(w);
-        continue;
-      }
-      const unsigned long long prev = atomicCAS(w, cur, ep | kStOff);  // claim: loading
-      if (prev == cur) {
-        claimed = 1;
-        break;
-      }
-      cur = prev;
-    }
-    if (claimed) {
-      const unsigned long long n32 = ((unsigned long long)ml + 31) & ~31ull;
-      const unsigned long long off = atomicAdd(A.stage_bump, n32);
-      if (off + n32 > A.stage_cap) {
-        atomicExch(w, ep | kStReady | kStOff);  // no room this batch: zero-copy for everyone
-        claimed = 0;
-        res = kStOff;
-      } else {
-        res = off;
-      }
-    } else {
-      __threadfence();  // acquire: the arena copy published before the state word
-    }
-  }
-  claimed = __shfl_sync(kFull, claimed, 0);
-  res = __shfl_sync(kFull, res, 0);
-  if (claimed) {
-    int32_t *dst = A.stage_arena + res;
-    warp_copy(dst, hp, ml, lane);
-    __syncwarp();
-    __threadfence();  // release: the copy before the state word
-    if (lane == 0) atomicExch(A.stage_state + v, ep | kStReady | res);
-    sfill += 4ull * ml;
-    slists += 1;
-    return dst;
-  }
-  __syncwarp();
-  if (res == kStOff) return hp;
-  shit += 4ull * ml;
-  return A.stage_arena + res;
+  const StageRef R{A.stage_state, A.stage_arena, A.stage_cap, A.stage_bump, A.stage_epoch};
+  return stage_fetch(R, v, hp, ml, sfill, slists, shit, lane);
 }
 
 __device__ __forceinline__ void mark_touched(const MatchArgs &A, int32_t v) {
@@ -229,7 +159,15 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
   if (v == pin.v) {  // served from this warp's staged copy
     r.m = pin.p;
     r.dev = true;
-  } else if (!r.dev && A.stage_state && r.ml >= A.stage_min) {  // fetched once per batch into HBM
+  } else if (!r.dev && A.npeer && (uint32_t)raw.w == 0 && r.ml > 0) {  // a peer's HBM cache, then the arena
+    const int32_t *q = peer_lookup(A, v, r.ml);
+    if (q) {
+      r.m = q;
+      r.dev = true;
+      acc.peer += 4ull * r.ml;
+    }
+  }
+  if (!r.dev && A.stage_state && r.ml >= A.stage_min) {  // fetched once per batch into HBM
     r.m = stage_resolve(A, v, r.m, r.ml, acc.sfill, acc.slists, acc.shit, lane);
     r.dev = reinterpret_cast<const char *>(r.m) != p;
   }
@@ -313,10 +251,15 @@ __device__ GCSM_COLD void stage_lists(const MatchArgs &A, LRef *L, int nl, int d
     const bool hit = L[p].dev;
     const bool driver = !has_set && p == drv;
     bool stage;
+    const uint32_t lg = 32u - __clz(n);
     if (driver) {
       stage = !hit;
+    } else if (hit && A.stage_policy == 1) {
+      // device-resident probe list (HBM cache, arena, U lists): latency model — a copy into shared memory costs
+      // one dependent round per 512 ints (4 x 16 B per lane in flight), the probes cost one per binary-search step
+      // below the last 128-byte line, for every 32 driver elements
+      stage = !__isShared(L[p].m) && (n + 511) / 512 <= ((d + 31) / 32) * (lg > 5 ? lg - 5 : 1);
     } else {
-      const uint32_t lg = 32u - __clz(n);
       stage = 4ull * n <= 32ull * d * (lg > 4 ? lg - 3 : 1);
     }
     if (!stage) continue;
@@ -547,6 +490,7 @@ __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int la
     if (acc.sfill) atomicAdd(&A.cnt[CNT_STAGE_FILL], acc.sfill);
     if (acc.slists) atomicAdd(&A.cnt[CNT_STAGE_LISTS], acc.slists);
     if (acc.shit) atomicAdd(&A.cnt[CNT_STAGE_HIT], acc.shit);
+    if (acc.peer) atomicAdd(&A.cnt[CNT_PEER], acc.peer);
   }
 }
 
@@ -644,6 +588,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   constexpr uint32_t kSlice = kSmemInts - GCSM_BM_INTS;
   const int k = KK ? KK : A.k;
   int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
+  int32_t *hbuf = stack + (int64_t)((k > 4 ? k - 4 : 0) + (LIST ? 1 : 0)) * A.dcap;  // hoisted last-level set
   const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
   const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
   const int32_t *f2u = f2c + A.f2_cap;
@@ -652,6 +597,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   const int64_t chunk = max((int64_t)1, min((int64_t)kChunk, n_f2 / (4 * warps)));
   Acc acc;
   Pinned pin;
+  unsigned long long x_entries = 0, x_pruned = 0, x_l3 = 0, x_l4 = 0, x_last = 0;  // work profile
   uint32_t pin_sm = 0;  // ints of the shared slice held by the pinned x2 list
   int64_t ci = 0, c_end = 0, c_start = 0;
   bool producing = true;  // phase 1: walk the (grouped) frontier; phase 2 (k >= 5): take shared level-3 tasks
@@ -701,6 +647,14 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const uint32_t ml = (uint32_t)raw.z;
         bool miss = !is_hit(A, mp), staged = false;
         if (lane == 0) mark_touched(A, x2);
+        if (miss && A.npeer && raw.w == 0 && ml > 0) {  // a linked peer's HBM cache holds it
+          const int32_t *q = peer_lookup(A, x2, ml);
+          if (q) {
+            mp = q;
+            miss = false;
+            staged = true;  // device-resident: served in place for the run unless pinned in shared memory
+          }
+        }
         if (miss && A.stage_state && ml >= A.stage_min) {  // the run's x2 list, fetched once per batch
           const int32_t *sp = stage_resolve(A, x2, mp, ml, acc.sfill, acc.slists, acc.shit, lane);
           if (sp != mp) {
@@ -780,6 +734,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     const Unit U = A.units[ui];
     const DevPlan &P = A.plans[U.plan];
     const int2 seg = A.useg[ui];
+    if (!task) ++x_entries;
     int32_t f[GCSM_MAXK];
     f[0] = U.a;
     f[1] = U.b;
@@ -791,6 +746,32 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     uint32_t end3 = 0xffffffffu;  // level-3 iteration bound (a task's slice)
     int lvl = 2;   // deepest position with a chosen element
     bool descend = true;
+    // hoisted last-level set (LevelPlan::hmask): ∩ of the last position's lists fixed at level 2, label-filtered
+    const int32_t *hset = nullptr;
+    uint32_t hn = 0;
+    if (KK == 0 && P.lv[k - 1].hmask) {
+      const LevelPlan &Lh = P.lv[k - 1];
+      LRef Lx[7];
+      int nx = 0, hdrv = 0;
+      uint32_t best = 0xffffffffu;
+      for (int b = 0; b < Lh.nb; ++b)
+        if ((Lh.hmask >> b) & 1) {
+          Lx[nx] = list_of(A, f[Lh.bpos[b]], Lh.bview[b], acc, lane, pin);
+          const uint32_t szx = Lx[nx].ml + Lx[nx].xl;
+          if (szx < best) {
+            best = szx;
+            hdrv = nx;
+          }
+          ++nx;
+        }
+      hn = warp_isect<true>(A, nullptr, 0, Lx, nx, hdrv, nullptr, 0, Lh.label, hbuf, lane);
+      __syncwarp();
+      hset = hbuf;
+      if (hn == 0) {  // no candidate for the last position anywhere below this entry
+        ++x_pruned;
+        continue;
+      }
+    }
     if (task) {
       int32_t *own = stack;  // this warp's level-3 buffer: a private, L1-safe copy of the shared set
       for (uint32_t i = lane; i < tk.n; i += 32) own[i] = __ldcg(A.arena + tk.off + i);
@@ -807,13 +788,21 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         const int p = lvl + 1;  // compute candidates of position p
         const LevelPlan &Lp = P.lv[p];
         LRef L[7];
-        int drv;
-        const int nl = gather_lists(A, Lp, f, L, &drv, acc, lane, pin);
+        int drv = 0;
+        int nl = (p == k - 1 && hset) ? 0 : gather_lists(A, Lp, f, L, &drv, acc, lane, pin);
         int32_t excl[GCSM_MAXK];
         int nex = 0;
         for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
-        const uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
+        uint32_t dn = Lp.reuse >= 0 ? sz[Lp.reuse] : 0;
+        if (p == k - 1 && hset) {  // hoisted set drives; probes = the lists not hoisted
+          int w2 = 0;
+          for (int b = 0; b < Lp.nb; ++b)
+            if (!((Lp.hmask >> b) & 1)) L[w2++] = list_of(A, f[Lp.bpos[b]], Lp.bview[b], acc, lane, pin);
+          nl = w2;
+          dset = hset;
+          dn = hn;
+        }
         uint32_t c = 0;
         int32_t vlo, vhi;
         range_of(Lp, f, &vlo, &vhi);
@@ -840,6 +829,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           else acc.add += c;
           descend = false;
         } else if (p == k - 1) {
+          x_last += dset ? dn : (nl ? L[drv].ml + L[drv].xl : 0);
           if (LIST) {
             c = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, lastbuf, lane, vlo, vhi);
             __syncwarp();
@@ -854,6 +844,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         } else {
           int32_t *out = stack + (int64_t)(p - 3) * A.dcap;
           sz[p] = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, out, lane, vlo, vhi);
+          if (p == 3) x_l3 += sz[p];
+          else if (p == 4) x_l4 += sz[p];
           __syncwarp();
           set[p] = out;
           it[p] = 0;
@@ -916,6 +908,13 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     (void)lvl;
   }
   flush(A, acc, lane);
+  if (lane == 0) {
+    atomicAdd(&A.cnt[CNT_X_ENTRIES], x_entries);
+    atomicAdd(&A.cnt[CNT_X_PRUNED], x_pruned);
+    atomicAdd(&A.cnt[CNT_X_L3], x_l3);
+    atomicAdd(&A.cnt[CNT_X_L4], x_l4);
+    atomicAdd(&A.cnt[CNT_X_LAST], x_last);
+  }
 }
 
 // ---- k = 4 count mode: the last level as one lean kernel ("k_last4") -------------------------
@@ -1137,7 +1136,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
     int4 xraw = make_int4(0, 0, 0, 0);
     int4 xrec = make_int4(0, 0, 0, 0);  // x2's delta record (if updated)
     uint32_t pin_sm = 0;
-    bool pin_dev = false, pin_hit = false;
+    bool pin_dev = false, pin_hit = false, pin_peer = false;
     for (int64_t c0 = (int64_t)g0; c0 < gend; c0 += 32) {
     const int n = (int)min((int64_t)32, gend - c0);
     // ---- one lane per entry: prefetch the entry's metadata in parallel
@@ -1199,6 +1198,15 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
                                                                 ((unsigned long long)(unsigned)xraw.y << 32));
         const uint32_t ml = (uint32_t)xraw.z;
         pin_hit = is_hit(A, mp);
+        pin_peer = false;
+        if (!pin_hit && A.npeer && xraw.w == 0 && ml > 0) {  // a linked peer's HBM cache holds x2's list
+          const int32_t *q = peer_lookup(A, x2, ml);
+          if (q) {
+            mp = q;
+            pin_hit = true;
+            pin_peer = true;
+          }
+        }
         uint32_t lb = 0, le = ml;
         if (rlo > rhi) {
           le = 0;  // no entry of the run reads x2's list
@@ -1280,8 +1288,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
           Lc.x = A.dlist + (vw == VIEW_NEW ? xrec.x : xrec.z);
           Lc.xl = (uint32_t)(vw == VIEW_NEW ? xrec.y : xrec.w);
         }
-        if (pin_hit) acc.hit += 4ull * (uint32_t)xraw.z;  // algorithmic: the whole list
+        if (pin_hit && !pin_peer) acc.hit += 4ull * (uint32_t)xraw.z;  // algorithmic: the whole list
         else acc.miss += 4ull * (uint32_t)xraw.z;
+        if (pin_peer) acc.peer += 4ull * (uint32_t)xraw.z;
         acc.delta += 4ull * Lc.xl;
       }
       const LR first = (need & 1u) ? La : ((need & 2u) ? Lb : Lc);

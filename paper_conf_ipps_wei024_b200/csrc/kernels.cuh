@@ -39,7 +39,15 @@ enum Counter {
   // B_comp (measurement mode only): bytes of the DISTINCT main lists the query's kernels touched,
   // by where they lived: HBM cache, pinned host (zero-copy), the batch's uploaded lists of U
   CNT_BCOMP = 30,
-  CNT_N = 33
+  CNT_PEER = 33,  // NVLink peer cache (NEXT-3): algorithmic list bytes read from a linked peer's HBM cache
+  // k_extend work profile (GCSM_TRACE): entries walked, entries pruned by the hoisted last-level set, level-3 and
+  // level-4 nodes, last-level driver elements
+  CNT_X_ENTRIES = 34,
+  CNT_X_PRUNED = 35,
+  CNT_X_L3 = 36,
+  CNT_X_L4 = 37,
+  CNT_X_LAST = 38,
+  CNT_N = 39
 };
 
 struct MatchArgs {
@@ -87,7 +95,13 @@ struct MatchArgs {
   unsigned long long *stage_bump;
   uint32_t stage_epoch;          // 24 bits, never 0
   uint32_t stage_min;            // shortest list (ints) routed through the arena
+  int32_t stage_policy;          // shared-memory staging of device-resident probe lists: 0 bytes model, 1 latency
   uint32_t *touched;             // B_comp measurement: bitmap of vertices whose main list was read (nullptr = off)
+  // NVLink peer cache: the linked peers' descriptor arrays and cache address ranges of this
+  // batch; a zero-copy miss whose list a peer holds in HBM is read from there (peer / NVLink) instead
+  int32_t npeer;
+  const VDesc *peer_vdesc[GCSM_MAX_PEERS];
+  const char *peer_lo[GCSM_MAX_PEERS], *peer_hi[GCSM_MAX_PEERS];
 };
 
 struct Task {

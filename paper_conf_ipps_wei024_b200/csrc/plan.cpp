@@ -203,6 +203,18 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
             if (!covered) L.rest[L.nrest++] = (int8_t)b;
           }
         }
+        // loop-invariant code motion of the last level (k >= 5): the lists of backward positions <= 2 are fixed
+        // for a whole level-2 entry; with >= 2 of them their intersection is computed once per entry
+        L.hmask = 0;
+        if (p == k - 1 && k >= 5 && L.reuse < 0) {
+          int cnt = 0, msk = 0;
+          for (int b = 0; b < L.nb; ++b)
+            if (L.bpos[b] <= 2) {
+              msk |= 1 << b;
+              ++cnt;
+            }
+          if (cnt >= 2) L.hmask = (int8_t)msk;
+        }
       }
     }
   }

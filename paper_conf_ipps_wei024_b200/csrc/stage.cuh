@@ -1,0 +1,116 @@
+// stage.cuh — device helpers shared by the matching kernels (kernels.cu) and the GPU walks (estimator_gpu.cu):
+// the warp-cooperative bulk list copy and the fetch-once staging of zero-copy lists within a batch
+// (DESIGN.md §1d).
+#pragma once
+#include <cstdint>
+
+namespace gcsm {
+
+struct StageRef {
+  unsigned long long *state;  // per vertex: epoch << 40 | ready << 39 | offset (ints)
+  int32_t *arena;
+  unsigned long long cap;     // ints
+  unsigned long long *bump;
+  uint32_t epoch;             // 24 bits, never 0
+};
+
+#ifdef __CUDACC__
+namespace {
+// Warp-cooperative bulk copy of a list (16-byte aligned source; lists are
+// allocated in 16-byte granules so reading up to round4(n) ints stays inside
+// the allocation). 4 x 16 B loads per lane are issued before any store, so a
+// warp keeps 2 KB in flight: a zero-copy list crosses PCIe at link speed
+// instead of one dependent 32 B sector per binary-search step.
+__device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
+  __syncwarp();  // every lane is done reading what this buffer held before (WAR across lanes)
+  const uint32_t n4 = (n + 3) >> 2;
+  const int4 *s4 = reinterpret_cast<const int4 *>(src);
+  int4 *d4 = reinterpret_cast<int4 *>(dst);
+  for (uint32_t base = 0; base < n4; base += 128) {
+    const uint32_t i0 = base + lane, i1 = i0 + 32, i2 = i0 + 64, i3 = i0 + 96;
+    int4 v0, v1, v2, v3;
+    if (i0 < n4) v0 = s4[i0];
+    if (i1 < n4) v1 = s4[i1];
+    if (i2 < n4) v2 = s4[i2];
+    if (i3 < n4) v3 = s4[i3];
+    if (i0 < n4) d4[i0] = v0;
+    if (i1 < n4) d4[i1] = v1;
+    if (i2 < n4) d4[i2] = v2;
+    if (i3 < n4) d4[i3] = v3;
+  }
+}
+
+// ---- fetch-once staging of zero-copy lists within a batch -------------------------------------
+// The first warp of the batch that needs vertex v's zero-copy main list claims it (CAS of its state word from an
+// older epoch to "loading"), copies it over PCIe into the batch arena (bump-allocated, 128-byte granules so that
+// no two lists share an L1 line) and publishes (epoch, ready, offset); every later read of that list in the batch,
+// by any warp or any later kernel of the batch, is an HBM read. A warp that finds the list loading waits for it
+// (the loader waits on nothing, so this cannot deadlock). Arena full: the list stays zero-copy ("no room").
+// The arena holds the batch's MAIN lists (v not in U: base(v), unchanged during the batch); the next batch has a
+// new epoch, so nothing stale is ever served.
+constexpr unsigned long long kStReady = 1ull << 39, kStOff = (1ull << 39) - 1;
+
+__device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v, const int32_t *hp, uint32_t ml,
+                                                   unsigned long long &sfill, unsigned long long &slists,
+                                                   unsigned long long &shit, int lane) {
+  const unsigned long long ep = (unsigned long long)A.epoch << 40;
+  unsigned long long res = 0;
+  int claimed = 0;
+  if (lane == 0) {
+    unsigned long long *w = A.state + v;
+    unsigned long long cur = __ldcg(w);
+    unsigned ns = 32;
+    for (;;) {
+      if ((cur & ~((1ull << 40) - 1)) == ep) {  // this batch's: ready, no room, or being loaded
+        if (cur & kStReady) {
+          res = cur & kStOff;
+          break;
+        }
+        __nanosleep(ns);
+        if (ns < 2048) ns <<= 1;
+        cur = __ldcg(w);
+        continue;
+      }
+      const unsigned long long prev = atomicCAS(w, cur, ep | kStOff);  // claim: loading
+      if (prev == cur) {
+        claimed = 1;
+        break;
+      }
+      cur = prev;
+    }
+    if (claimed) {
+      const unsigned long long n32 = ((unsigned long long)ml + 31) & ~31ull;
+      const unsigned long long off = atomicAdd(A.bump, n32);
+      if (off + n32 > A.cap) {
+        atomicExch(w, ep | kStReady | kStOff);  // no room this batch: zero-copy for everyone
+        claimed = 0;
+        res = kStOff;
+      } else {
+        res = off;
+      }
+    } else {
+      __threadfence();  // acquire: the arena copy published before the state word
+    }
+  }
+  claimed = __shfl_sync(0xffffffffu, claimed, 0);
+  res = __shfl_sync(0xffffffffu, res, 0);
+  if (claimed) {
+    int32_t *dst = A.arena + res;
+    warp_copy(dst, hp, ml, lane);
+    __syncwarp();
+    __threadfence();  // release: the copy before the state word
+    if (lane == 0) atomicExch(A.state + v, ep | kStReady | res);
+    sfill += 4ull * ml;
+    slists += 1;
+    return dst;
+  }
+  __syncwarp();
+  if (res == kStOff) return hp;
+  shit += 4ull * ml;
+  return A.arena + res;
+}
+
+}  // namespace
+#endif  // __CUDACC__
+
+}  // namespace gcsm

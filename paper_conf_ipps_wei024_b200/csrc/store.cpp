@@ -71,9 +71,10 @@ int32_t *HostStore::alloc_list(uint32_t &capacity, bool *cuda_err) {
 }
 
 std::string HostStore::init(int32_t n_, const int64_t *rp, const int32_t *col, const int32_t *labels, int threads_,
-                            bool *cuda_err) {
+                            bool *cuda_err, int32_t ncap_) {
   *cuda_err = false;
   n = n_;
+  ncap = std::max(n_, ncap_);
   threads = std::max(1, threads_);
   if (n < 1) return "n must be >= 1";
   if (!rp || (rp[n] > 0 && !col)) return "row_ptr/col is NULL";
@@ -103,12 +104,12 @@ std::string HostStore::init(int32_t n_, const int64_t *rp, const int32_t *col, c
     case 4: return "graph is not symmetric";
     default: break;
   }
-  lst.assign(n, nullptr);
-  len.assign(n, 0);
-  cap.assign(n, 0);
-  uidx.assign(n, -1);
+  lst.assign(ncap, nullptr);
+  len.assign(ncap, 0);
+  cap.assign(ncap, 0);
+  uidx.assign(ncap, -1);
   if (labels) {
-    lab.resize(n);
+    lab.assign(ncap, 0);
     for (int32_t v = 0; v < n; ++v) lab[v] = (uint16_t)labels[v];
   }
   uint64_t total = 0;
@@ -145,6 +146,26 @@ std::string HostStore::init(int32_t n_, const int64_t *rp, const int32_t *col, c
   return "";
 }
 
+bool HostStore::grow(int32_t new_n) {
+  if (new_n <= n) return true;
+  if (new_n > ncap) return false;
+  const uint32_t avg = n > 0 ? (uint32_t)std::min<uint64_t>(edges2 / (uint64_t)n, 1u << 20) : 0;
+  const uint32_t c0 = round4(std::max<uint32_t>(4, avg));
+  bool err = false;
+  for (int32_t v = n; v < new_n; ++v) {
+    uint32_t c = c0;
+    int32_t *p = alloc_list(c, &err);
+    if (err) return false;
+    lst[v] = p;
+    cap[v] = c;
+    len[v] = 0;
+  }
+  if (deg_hist.empty()) deg_hist.assign(1, 0);
+  deg_hist[0] += (uint64_t)(new_n - n);
+  n = new_n;
+  return true;
+}
+
 bool HostStore::has_edge(int32_t u, int32_t v) const {
   if (len[u] > len[v]) std::swap(u, v);
   return std::binary_search(lst[u], lst[u] + len[u], v);
@@ -157,7 +178,8 @@ std::string HostStore::normalize(int64_t n_ins, const int32_t *ins, int64_t n_de
     out.resize(m);
     for (int64_t i = 0; i < m; ++i) {
       int32_t u = e[2 * i], v = e[2 * i + 1];
-      if (u < 0 || v < 0 || u >= n || v >= n) return "vertex id out of range";
+      if (u < 0 || v < 0 || u >= ncap || v >= ncap) return "vertex id out of range";
+      if (e == del && (u >= n || v >= n)) return "a deleted edge names a vertex that does not exist (P:65)";
       if (u == v) return "self loop in batch";
       if (u > v) std::swap(u, v);
       out[i] = ((uint64_t)(uint32_t)u << 32) | (uint32_t)v;
@@ -177,6 +199,8 @@ std::string HostStore::normalize(int64_t n_ins, const int32_t *ins, int64_t n_de
     else ++j;
   }
   // --- no mutation before this point ---
+  grow_n = n;
+  for (uint64_t key : ki) grow_n = std::max<int32_t>(grow_n, (int32_t)(key & 0xffffffffu) + 1);
   I.clear();
   D.clear();
   dropped = 0;

@@ -33,10 +33,12 @@ class HostStore {
  public:
   ~HostStore();
   // returns "" or an error message; *cuda_err set if the failure is a CUDA error
+  // ncap >= n: vertex-id capacity (ids in [n, ncap) may join later, P:65 / P:273)
   std::string init(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels, int threads,
-                   bool *cuda_err);
+                   bool *cuda_err, int32_t ncap = 0);
 
-  int32_t n = 0;
+  int32_t n = 0;     // current vertex count (ids [0, n))
+  int32_t ncap = 0;  // capacity: every per-vertex array is sized ncap
   int threads = 1;
   std::vector<int32_t *> lst;   // host address of each list (pinned, mapped)
   std::vector<uint32_t> len, cap;
@@ -47,8 +49,13 @@ class HostStore {
   const int32_t *dev_ptr(const int32_t *host) const;  // device-visible address of a pinned host address
 
   // ---- batch (steps ① / a0-a1) ----
-  // Validates and normalises; on EINVAL returns the message and mutates nothing.
+  // Validates and normalises; on EINVAL returns the message and mutates nothing. Insertions may name ids in
+  // [n, ncap) (new vertices): grow_n is then the vertex count the batch needs (grow() applies it).
   std::string normalize(int64_t n_ins, const int32_t *ins, int64_t n_del, const int32_t *del);
+  int32_t grow_n = 0;
+  // New vertices [n, new_n) ("allocate an array with an initial size of the average degree of the graph
+  // for each new vertex"): empty lists of that capacity; false if the pinned allocation fails.
+  bool grow(int32_t new_n);
   bool build_overlay(int slot, bool *cuda_err);  // S(x) for x ∈ U with deletions (per in-flight slot)
   HList view(int32_t v, int view) const;
   uint32_t view_len(int32_t v, int view) const;

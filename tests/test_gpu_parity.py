@@ -750,3 +750,198 @@ def test_motif_census_road_net(G):
     rp2, col2 = g.export_csr()
     assert np.array_equal(rp, rp2) and np.array_equal(col, col2)
     g.close()
+
+
+# ------------------------------------------------------------------ NEXT-4: vertex-id growth
+
+def _growth_batches(w, n0, ncap, seed, n_batches=3):
+    """Mixed batches that also attach new ids in [n0, ncap): a new vertex x gets edges to both endpoints of an
+    existing edge (a, b), so it closes triangles / diamonds / K4s at once; later batches join new ids together
+    and delete some of their edges again."""
+    rng = np.random.default_rng(seed)
+    E = oracle.edges_of(w.row_ptr, w.col)
+    out = []
+    nxt = n0
+    joined = []
+    for t in range(n_batches):
+        ins, dele = [tuple(e) for e in w.batches[t][0]], [tuple(e) for e in w.batches[t][1]]
+        for _ in range(40):
+            if nxt >= ncap:
+                break
+            a, b = E[rng.integers(len(E))]
+            ins += [(nxt, int(a)), (int(b), nxt)]
+            joined.append(nxt)
+            nxt += 1
+        if len(joined) >= 4:
+            for _ in range(10):
+                x, y = rng.choice(joined, 2, replace=False)
+                ins.append((int(x), int(y)))
+        out.append((np.array(sorted(set(ins)), np.int32).reshape(-1, 2), np.array(dele, np.int32).reshape(-1, 2)))
+    return out
+
+
+@pytest.mark.parametrize("name", ["triangle", "diamond", "k4", "house5u"])
+def test_vertex_growth(G, name):
+    """Insertions naming ids in [n, vertex_capacity) add vertices, each with an empty list of the average
+    degree's capacity; the oracle sees the same ids as isolated vertices of the capacity-sized universe
+    (reading R9), so the counts and the final graph must agree batch by batch."""
+    w = gi.make_workload("C2", scale=11, n_edges=12000, batch=200)
+    n0, ncap = w.n, w.n + 150
+    batches = _growth_batches(w, n0, ncap, 11)
+    rp = np.concatenate([w.row_ptr, np.full(ncap - n0, w.row_ptr[-1], np.int64)])
+    want, (rp1, col1) = oracle_run(ncap, rp, w.col, None, name, batches)
+    k, qe, ql = gi.query(name)
+    g = G.Gcsm(n0, w.row_ptr, w.col, device=0, vertex_capacity=ncap)
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(w.adj_bytes // 10)
+    got = [g.apply_batch(*b) for b in batches]
+    assert got == want
+    assert any(a for a, _ in want)
+    n1 = g.num_vertices()
+    assert n0 < n1 <= ncap
+    rp2, col2 = g.export_csr()
+    assert np.array_equal(rp2, rp1[:n1 + 1]) and np.array_equal(col2, col1) and rp1[n1] == rp1[-1]
+    # a deletion naming a vertex that does not exist (P:65), or an id beyond the capacity: EINVAL, nothing changes
+    bad = [([(0, ncap)], [])] + ([([], [(0, ncap - 1)])] if n1 < ncap else [])
+    for ins, dele in bad:
+        with pytest.raises(G.GcsmError) as ei:
+            g.apply_batch(ins, dele)
+        assert ei.value.name == "GCSM_EINVAL"
+    assert g.num_vertices() == n1
+    g.close()
+
+
+def test_add_vertices_labelled(G):
+    """gcsm_add_vertices with labels, then edges to them: labelled house5 counts equal the oracle's."""
+    w = gi.make_workload("C3", scale=11, n_edges=12000, batch=200, n_batches=2)
+    n0, extra = w.n, 80
+    lab_new = np.random.default_rng(5).integers(0, 8, extra).astype(np.int32)
+    labels = np.concatenate([w.labels, lab_new])
+    k, qe, ql = gi.query("house5")
+    g = G.Gcsm(n0, w.row_ptr, w.col, w.labels, device=0, vertex_capacity=n0 + extra)
+    g.set_query(k, qe, ql)
+    g.set_cache_budget(w.adj_bytes // 10)
+    assert g.add_vertices(extra, lab_new) == n0 and g.num_vertices() == n0 + extra
+    with pytest.raises(G.GcsmError):
+        g.add_vertices(1)  # capacity exhausted
+    batches = _growth_batches(w, n0, n0 + extra, 12, n_batches=2)
+    rp = np.concatenate([w.row_ptr, np.full(extra, w.row_ptr[-1], np.int64)])
+    want, _ = oracle_run(n0 + extra, rp, w.col, labels, "house5", batches)
+    assert [g.apply_batch(*b) for b in batches] == want
+    g.close()
+
+
+# ------------------------------------------------------------------ NEXT-3: NVLink peer cache
+
+@pytest.mark.parametrize("name", ["c4", "house5u", "prism6"])
+def test_peer_cache_two_contexts(G, name):
+    """Two contexts on one GPU (an emulated 2-rank world: each counts its own shard of the units) link their HBM
+    caches (gcsm_link_peers): a list missing from one context's cache is read from the other's. Each context is
+    driven by its own host thread in lockstep; the shard counts sum to the oracle's, batch by batch, and some
+    list bytes are served by the peer."""
+    import threading
+    w = gi.make_workload("C2" if name != "prism6" else "C4", scale=13, n_edges=60_000, batch=512, n_batches=3)
+    k, qe, ql = gi.query(name)
+    want, _ = oracle_run(w.n, w.row_ptr, w.col, None, name, w.batches)
+    ctxs = [G.Gcsm(w.n, w.row_ptr, w.col, device=0, rank=r, world=2, local_counts=True, seed=0x77 + r)
+            for r in range(2)]
+    for c in ctxs:
+        c.set_query(k, qe, ql, gi.order(name))
+        c.set_cache_budget(w.adj_bytes // 20)
+    G.link_peers(ctxs)
+    out = [[], []]
+    errs = []
+
+    def drive(r):
+        try:
+            for ins, dele in w.batches:
+                out[r].append((ctxs[r].apply_batch(ins, dele), ctxs[r].stats()["peer_bytes"]))
+        except Exception as e:  # noqa: BLE001
+            errs.append(e)
+
+    th = [threading.Thread(target=drive, args=(r,)) for r in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=600)
+    assert not errs, errs
+    got = [(a0 + a1, r0 + r1) for ((a0, r0), _), ((a1, r1), _) in zip(out[0], out[1])]
+    assert got == want
+    assert sum(p for _, p in out[0]) + sum(p for _, p in out[1]) > 0
+    G.link_peers([])
+    G.link_peers(ctxs[:1])  # unlink (n < 2) is accepted
+    for c in ctxs:
+        c.close()
+
+
+def _star_closed_form(n, rp, col, ins, dele, r):
+    """K_{1,r} added = Σ_U P(d',r) - P(s,r), removed = Σ_U P(d,r) - P(s,r) (O(|U|) arithmetic)."""
+    I, D, _ = oracle.normalize_batch(n, rp, col, ins, dele)
+    U = np.unique(np.concatenate([I.ravel(), D.ravel()]))
+    d = np.diff(rp)[U].astype(object)
+    cnt = lambda E: np.array([0 if len(E) == 0 else int(np.count_nonzero(E == u)) for u in U], dtype=object)
+    di, dd = cnt(I), cnt(D)
+    s, d1 = d - dd, d - dd + di
+
+    def P(x):
+        out = np.ones_like(x, dtype=object)
+        for i in range(r):
+            out = out * (x - i)
+        return out
+    return (int((P(d1) - P(s)).sum()), int((P(d) - P(s)).sum())), (I, D)
+
+
+def test_full_size_c2_whole_batch(G):
+    """One WHOLE 4096-update C2 batch (70M edges, bench launch configuration: one context holding K4 + C4 with the
+    catalogue orders, 10 % budget) against the oracle."""
+    w = gi.make_workload("C2", n_batches=1)
+    ins, dele = w.batches[0]
+    queries = ["k4", "c4"]
+    g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0)
+    for i, q in enumerate(queries):
+        k, qe, ql = gi.query(q)
+        (g.set_query if i == 0 else g.add_query)(k, qe, ql, gi.order(q))
+    g.set_cache_budget(int(w.adj_bytes * w.budget_frac))
+    g.apply_batch(ins, dele)
+    for i, q in enumerate(queries):
+        k, qe, ql = gi.query(q)
+        assert g.query_counts(i) == oracle.delta(w.n, w.row_ptr, w.col, None, k, qe, ql, ins, dele), q
+    g.close()
+
+
+def test_full_size_c4(G):
+    """BASELINE configs[3] at FULL size (67M vertices, 1.8B edges in pinned host memory, planted 8-cliques, 1 %
+    budget, bench.py's context: prism6 + K4+2tri6 + K6 with the catalogue orders, plus a K_{1,3} star): on two
+    batches, a sampled sub-batch (64 updated edges) against the oracle for every 6-vertex query, and the rest of
+    the batch against the star's degree closed form."""
+    w = gi.make_workload("C4", n_batches=2)
+    queries = ["prism6", "k4tri6", "k6"]
+    star = (4, np.array([(0, 1), (0, 2), (0, 3)], np.int32), None)
+    g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0)
+    for i, q in enumerate(queries):
+        k, qe, ql = gi.query(q)
+        (g.set_query if i == 0 else g.add_query)(k, qe, ql, gi.order(q))
+    g.add_query(*star)
+    g.set_cache_budget(int(w.adj_bytes * w.budget_frac))
+    rp, col = w.row_ptr, w.col
+    nonzero = 0
+    for t, (ins, dele) in enumerate(w.batches):
+        si, sd = ins[:32], dele[:32]
+        ri, rd = ins[32:], dele[32:]
+        g.apply_batch(si, sd)
+        for i, q in enumerate(queries):
+            k, qe, ql = gi.query(q)
+            want = oracle.delta(w.n, rp, col, None, k, qe, ql, si, sd)
+            assert g.query_counts(i) == want, (t, q)
+            nonzero += want != (0, 0)
+        cf, (I, D) = _star_closed_form(w.n, rp, col, si, sd, 3)
+        assert g.query_counts(3) == cf
+        rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+        g.apply_batch(ri, rd)  # the rest of the batch, on the star closed form
+        cf, (I, D) = _star_closed_form(w.n, rp, col, ri, rd, 3)
+        assert g.query_counts(3) == cf
+        assert g.query_stats(0)["stage_fill_bytes"] > 0  # the fetch-once staging ran at full size
+        if t + 1 < len(w.batches):
+            rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+    assert nonzero >= 2
+    g.close()

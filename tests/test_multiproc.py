@@ -94,3 +94,71 @@ def test_gloo_world2_shard_and_allreduce():
     a, b = set(res[0][4]), set(res[1][4])
     assert not (a & b) and len(a | b) == res[0][7]     # disjoint cover of the units
     assert a and b                                     # both ranks got work
+
+
+def _lib_worker(rank, world, port, out_q):
+    """One rank of an emulated world on cuda:0: ITS OWN libgcsm context (rank, world, shard-local counts), the
+    count allreduce over gloo; rank 0 checks the sums against the oracle."""
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import gcsm_inputs as gi
+        import oracle
+        import paper_conf_ipps_wei024_b200 as G
+        torch.cuda.set_device(0)
+        w = gi.make_workload("C2", scale=12, n_edges=30_000, batch=256, n_batches=3)
+        queries = ["diamond", "k4", "house5u"]
+        g = G.Gcsm(w.n, w.row_ptr, w.col, device=0, rank=rank, world=world, local_counts=True)
+        for i, q in enumerate(queries):
+            k, qe, ql = gi.query(q)
+            (g.set_query if i == 0 else g.add_query)(k, qe, ql)
+        g.set_cache_budget(w.adj_bytes // 10)
+        got, mine = [], []
+        for ins, dele in w.batches:
+            g.apply_batch(ins, dele)
+            c = [g.query_counts(i) for i in range(len(queries))]
+            mine.append(c)
+            t = torch.tensor(c, dtype=torch.int64)
+            dist.all_reduce(t)
+            got.append([tuple(x) for x in t.tolist()])
+        g.close()
+        want = None
+        if rank == 0:
+            want, rp, col = [], w.row_ptr, w.col
+            for ins, dele in w.batches:
+                want.append([oracle.delta(w.n, rp, col, None, *gi.query(q), ins, dele) for q in queries])
+                I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+                rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+        out_q.put((rank, got, mine, want))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+def test_libgcsm_world2_gloo():
+    """N > 1 through the library itself (not the oracle's IVM): two processes, each its own context on cuda:0 with
+    rank / world = 2, shard-local counts summed by a gloo allreduce, equal to the oracle on every batch and query;
+    both ranks did work."""
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import __graft_entry__
+    __graft_entry__.build()
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_lib_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=600) for _ in range(world)], key=lambda x: x[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    want = res[0][3]
+    for rank, got, mine, _ in res:
+        assert got == want
+    assert any(any(a or r for a, r in b) for b in res[0][2]) and any(any(a or r for a, r in b) for b in res[1][2])
