@@ -43,6 +43,8 @@ METRICS = {"C1": "updated edges/sec per batch (C1: 1K-vertex / 8K-edge R-MAT, tr
            "C2": "updated edges/sec per batch (C2: LJ-shaped 4.19M-vertex / 70M-edge R-MAT, 4-clique + 4-cycle)",
            "C3": "updated edges/sec per batch (C3: Orkut-shaped 3M-vertex / 120M-edge R-MAT, 8 labels, 5-vertex "
                  "labelled patterns)",
+           "PA": "updated edges/sec per batch (PA: RoadNetPA-shaped 1.09M-vertex lattice, all 29 connected 3-5-vertex "
+                 "motifs as standing queries)",
            "C4": "updated edges/sec per batch (C4: FR-shaped 67M-vertex / 1.8B-edge R-MAT in pinned host memory, "
                  "6-vertex patterns, budget 1%)"}
 UNIT = "updated_edges/s"
@@ -183,7 +185,10 @@ def load_traffic(config, query):
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return d.get(f"{config}:{query}", d.get(query) if config == "C2" else None)
+        e = d.get(f"{config}:{query}", d.get(query) if config == "C2" else None)
+        if isinstance(e, dict):
+            return e.get("dram_bytes")
+        return e
     return None
 
 
@@ -192,6 +197,17 @@ def workload(args, world, extra_steps=1):
     steps = args.warmup + args.steps + extra_steps
     gb = args.batch * world
     return gi.make_workload(args.config, batch=gb, n_stream=max(12 * 8192, steps * gb))
+
+
+def workload_name(w):
+    if w.meta.get("grid"):
+        W, H, pk, pd = w.meta["grid"]
+        return (f"{w.name} (RoadNetPA-shaped, Fig. 11 motif counting, SURVEY 8f NEXT-4): {W}x{H} lattice kept with "
+                f"p={pk} plus cell diagonals p={pd}, {w.meta['n_edges'] / 1e6:.2f}M edges")
+    return (f"{w.name} (BASELINE configs[{int(w.name[1:]) - 1}]): R-MAT s={w.meta['scale']}, "
+            f"{w.meta['n_edges'] / 1e6:.0f}M edges"
+            + (f" ({w.meta['planted'][0]} planted {w.meta['planted'][1]}-cliques)" if w.meta['planted'][0] else "")
+            + (f", {w.meta['L']} labels" if w.meta['L'] else ""))
 
 
 def sample_of(ins, dele, s):
@@ -306,7 +322,7 @@ def run_reference(args):
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / max(len(times), 1),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic (seeded R-MAT graph + P:331 update stream, generated on the box)",
-            "config": {"workload": f"{w.name} (BASELINE configs[{int(w.name[1:]) - 1}])", "queries": queries,
+            "config": {"workload": workload_name(w), "queries": queries,
                        "global_batch": s, "graph_vertices": w.n, "graph_edges": int(w.row_ptr[-1] // 2),
                        "parallelism": "host threads"},
             "cpu_baseline": {"value": v, "unit": UNIT, **host_info(), "kind": "oracle",
@@ -534,13 +550,9 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms_dev / K, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "int32",
         "data": "synthetic (seeded R-MAT graph + P:331 update stream, generated on the box)",
-        "config": {"workload": f"{w.name} (BASELINE configs[{int(w.name[1:]) - 1}]): R-MAT s={w.meta['scale']}, "
-                               f"{w.meta['n_edges'] / 1e6:.0f}M edges"
-                               + (f" ({w.meta['planted'][0]} planted {w.meta['planted'][1]}-cliques)"
-                                  if w.meta['planted'][0] else "")
-                               + (f", {w.meta['L']} labels" if w.meta['L'] else "")
-                               + f", queries {'+'.join(queries)}, {args.batch} mixed updates per GPU per step, "
-                                 f"cache budget {frac:.0%} of adjacency", "queries": queries,
+        "config": {"workload": workload_name(w),
+                   "detail": f"queries {'+'.join(queries)}, {args.batch} mixed updates per GPU per step, "
+                             f"cache budget {frac:.0%} of adjacency", "queries": queries,
                    "global_batch": args.batch * world,
                    "graph_vertices": w.n, "graph_edges": int(w.row_ptr[-1] // 2), "budget_bytes": budget,
                    "cache_policy": args.cache_policy,

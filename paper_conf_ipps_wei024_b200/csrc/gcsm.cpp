@@ -1534,7 +1534,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
 
   // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
   const int dcap = (int)((D + 32 + 31) & ~uint64_t(31));
-  const int nbuf = std::max(1, std::max(kmax - 4, 0) + (listing ? 1 : 0) + (kmax >= 5 ? 1 : 0));  // + hoisted set
+  // stacks + (list mode) last-level buffer + (k >= 5) hoisted set, filter set, level-3 iteration list
+  const int nbuf = std::max(1, std::max(kmax - 4, 0) + (listing ? 1 : 0) + (kmax >= 5 ? 3 : 0));
   const size_t stride = (size_t)(nbuf + 3) * (size_t)dcap;  // stacks + pinned-x2 + 2 HBM staging buffers
   if (!dev_ensure(ctx->d_scratch, ctx->scratch_cap, stride * (size_t)ctx->warps_total))
     return ctx->fail(GCSM_ENOMEM, "scratch");
@@ -1615,6 +1616,8 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   }
   A.touched = ctx->bcomp ? ctx->d_touched_bc : nullptr;
   A.stage_policy = ctx->stage_policy;
+  A.filter3 = std::getenv("GCSM_NO_FILTER3") ? 0 : 1;
+  A.hoist = std::getenv("GCSM_NO_HOIST") ? 0 : 1;
   A.npeer = npeer;
   for (int p = 0; p < npeer; ++p) {
     const gcsm_ctx::Slot &ps = peer_of[p]->slots[ctx->batch_seq & 1];
@@ -1848,9 +1851,9 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.frontier = h[CNT_F2];
     if (std::getenv("GCSM_TRACE"))
       std::fprintf(stderr, "[gcsm kern] q=%d frontier=%llu runs=%llu pins=%llu pin_gb=%.3f split_gb=%.3f copied_gb=%.3f "
-                   "entries=%llu pruned=%llu l3=%llu l4=%llu last_drv=%llu\n",
+                   "entries=%llu pruned=%llu l3=%llu l3kept=%llu l4=%llu last_drv=%llu\n",
                    qi, h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_DBG_SPLIT] / 1e9,
-                   h[CNT_COPIED] / 1e9, h[CNT_X_ENTRIES], h[CNT_X_PRUNED], h[CNT_X_L3], h[CNT_X_L4], h[CNT_X_LAST]);
+                   h[CNT_COPIED] / 1e9, h[CNT_X_ENTRIES], h[CNT_X_PRUNED], h[CNT_X_L3], h[CNT_X_L3F], h[CNT_X_L4], h[CNT_X_LAST]);
     if (qi == 0 && (sl.tup_add || sl.tup_rem)) {
       const int k = ctx->qs[0].qp.k;
       const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);

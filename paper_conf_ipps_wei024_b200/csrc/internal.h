@@ -60,6 +60,10 @@ struct LevelPlan {
   int8_t inj[7];
   int8_t nlo, lo[7];   // symmetry breaking: f(order[p]) > f(position lo[i])
   int8_t nhi, hi[7];   //                    f(order[p]) < f(position hi[i])
+  int8_t fmask;        // position 4 (k >= 5) only, when position 3 is one of its backward neighbours: the backward
+                       // lists at positions <= 2 (bit b); their intersection F is fixed per level-2 entry and every
+                       // level-3 node whose list misses F has no position-4 candidate (lane-parallel filter)
+  int8_t f3;           // index b of position 3 among the backward lists (with fmask)
   int8_t hmask;        // last position (k >= 5) only: backward lists (bit b = bpos[b]) whose positions are <= 2,
                        // i.e. fixed once a level-2 partial match is chosen; their intersection is hoisted to the
                        // level-2 entry (loop-invariant code motion): empty -> the entry's subtree holds no match

@@ -574,6 +574,99 @@ __global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
   flush(A, acc, lane);
 }
 
+__device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
+  return x;
+}
+
+// Level-3 filter (LevelPlan::fmask): position 4's candidates for a level-3 node x3 lie in
+// F ∩ view(N(x3)), where F (sorted, label-filtered) is the intersection of position 4's lists fixed for the whole
+// level-2 entry. Lane i tests node i: does its own list meet F? Nodes that cannot (almost all of them on C4) are
+// dropped from the level-3 set before the warp-wide DFS visits them; the test ignores injectivity and symmetry
+// ranges, so it only ever keeps too much (exact). Survivors go to out (may be set3 itself: compaction in place);
+// returns their number.
+__device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const int32_t *set3, uint32_t n3,
+                                               int32_t *out, const int32_t *F, uint32_t nF1, uint32_t nF, Acc &acc,
+                                               int lane) {
+  uint32_t w = 0;
+  unsigned long long hb = 0, mb = 0, db = 0, sb = 0, pb = 0;  // per-lane algorithmic bytes: hit, miss, delta, staged, peer
+  for (uint32_t base = 0; base < n3; base += 32) {
+    const uint32_t i = base + lane;
+    const bool act = i < n3;
+    const int32_t v = act ? set3[i] : 0;
+    const int32_t *m = nullptr, *x = nullptr;
+    uint32_t ml = 0, xl = 0;
+    bool need = false;
+    if (act) {
+      const int4 raw = __ldg(reinterpret_cast<const int4 *>(A.vdesc + v));
+      m = reinterpret_cast<const int32_t *>((unsigned long long)(unsigned)raw.x |
+                                            ((unsigned long long)(unsigned)raw.y << 32));
+      ml = (uint32_t)raw.z;
+      const uint32_t upd = (uint32_t)raw.w;
+      if (upd != 0 && vw != VIEW_S) {
+        const int4 e = __ldg(reinterpret_cast<const int4 *>(A.drec + (upd - 1)));
+        x = A.dlist + (vw == VIEW_NEW ? e.x : e.z);
+        xl = (uint32_t)(vw == VIEW_NEW ? e.y : e.w);
+      }
+      mark_touched(A, v);
+      db += 4ull * xl;
+      const char *pc = reinterpret_cast<const char *>(m);
+      if (pc >= A.cache_lo && pc < A.cache_hi) {
+        hb += 4ull * ml;
+      } else if (pc >= A.ubuf_lo && pc < A.ubuf_hi) {
+        db += 4ull * ml;
+      } else {
+        mb += 4ull * ml;
+        const int32_t *q = (A.npeer && upd == 0 && ml > 0) ? peer_lookup(A, v, ml) : nullptr;
+        if (q) {
+          m = q;
+          pb += 4ull * ml;
+        } else if (A.stage_state && ml >= A.stage_min) {
+          const unsigned long long st = __ldcg(A.stage_state + v);
+          if ((st >> 40) == A.stage_epoch && (st & kStReady) && (st & kStOff) != kStOff) {
+            m = A.stage_arena + (st & kStOff);
+            sb += 4ull * ml;
+          } else {
+            need = true;
+          }
+        }
+      }
+    }
+    // lists not staged yet: the warp fetches them once (every later reader in the batch finds them in HBM)
+    for (unsigned nm = __ballot_sync(kFull, need); nm; nm &= nm - 1) {
+      const int l = __ffs(nm) - 1;
+      const int32_t vl = __shfl_sync(kFull, v, l);
+      const unsigned long long hp = __shfl_sync(kFull, (unsigned long long)m, l);
+      const uint32_t mll = __shfl_sync(kFull, ml, l);
+      const int32_t *q = stage_resolve(A, vl, reinterpret_cast<const int32_t *>(hp), mll, acc.sfill, acc.slists,
+                                       acc.shit, lane);
+      if (lane == l) m = q;
+    }
+    bool hit = false;
+    if (act) {
+      if (ml + xl <= nF) {  // stream the node's list, probe F (its two sorted runs)
+        const int32_t *F2 = F + nF1;
+        const uint32_t nF2 = nF - nF1;
+        for (uint32_t j = 0; j < ml && !hit; ++j) hit = bsearch_has(F, nF1, m[j]) || (nF2 && bsearch_has(F2, nF2, m[j]));
+        for (uint32_t j = 0; j < xl && !hit; ++j) hit = bsearch_has(F, nF1, x[j]) || (nF2 && bsearch_has(F2, nF2, x[j]));
+      } else {  // stream F, probe the node's list
+        for (uint32_t j = 0; j < nF && !hit; ++j) hit = bsearch_has(m, ml, F[j]) || (xl && bsearch_has(x, xl, F[j]));
+      }
+    }
+    const unsigned hm = __ballot_sync(kFull, hit);
+    if (hit) out[w + __popc(hm & ((1u << lane) - 1u))] = v;
+    w += __popc(hm);
+    __syncwarp();
+  }
+  acc.hit += warp_sum64(hb);
+  acc.miss += warp_sum64(mb);
+  acc.delta += warp_sum64(db);
+  acc.shit += warp_sum64(sb);
+  acc.peer += warp_sum64(pb);
+  return w;
+}
+
 // Levels 3..k-1 (DFS): warp per level-2 frontier entry.
 template <bool LIST, int KK>  // KK: compile-time query size (4: the level-3 count only), 0 = any
 __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchArgs A) {
@@ -589,6 +682,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   const int k = KK ? KK : A.k;
   int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
   int32_t *hbuf = stack + (int64_t)((k > 4 ? k - 4 : 0) + (LIST ? 1 : 0)) * A.dcap;  // hoisted last-level set
+  int32_t *fbuf = hbuf + A.dcap;                                                        // level-3 filter set F
+  int32_t *ibuf = fbuf + A.dcap;                                 // level-3 iteration list (filtered, set reused)
   const int64_t n_f2 = (int64_t)*(volatile unsigned long long *)&A.cnt[CNT_F2];
   const int32_t *f2c = reinterpret_cast<const int32_t *>(A.f2);
   const int32_t *f2u = f2c + A.f2_cap;
@@ -597,7 +692,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   const int64_t chunk = max((int64_t)1, min((int64_t)kChunk, n_f2 / (4 * warps)));
   Acc acc;
   Pinned pin;
-  unsigned long long x_entries = 0, x_pruned = 0, x_l3 = 0, x_l4 = 0, x_last = 0;  // work profile
+  unsigned long long x_entries = 0, x_pruned = 0, x_l3 = 0, x_l4 = 0, x_last = 0, x_l3f = 0;  // work profile
   uint32_t pin_sm = 0;  // ints of the shared slice held by the pinned x2 list
   int64_t ci = 0, c_end = 0, c_start = 0;
   bool producing = true;  // phase 1: walk the (grouped) frontier; phase 2 (k >= 5): take shared level-3 tasks
@@ -749,7 +844,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     // hoisted last-level set (LevelPlan::hmask): ∩ of the last position's lists fixed at level 2, label-filtered
     const int32_t *hset = nullptr;
     uint32_t hn = 0;
-    if (KK == 0 && P.lv[k - 1].hmask) {
+    if (KK == 0 && P.lv[k - 1].hmask && A.hoist) {
       const LevelPlan &Lh = P.lv[k - 1];
       LRef Lx[7];
       int nx = 0, hdrv = 0;
@@ -772,9 +867,60 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         continue;
       }
     }
+    // level-3 filter set F (LevelPlan::fmask): ∩ of position 4's lists fixed for this entry, label-filtered
+    uint32_t nF = 0, nF1 = 0;  // F = fset[0..nF1) ∪ fset[nF1..nF), two sorted runs
+    const int32_t *fset = fbuf;
+    const bool filt = KK == 0 && k >= 5 && P.lv[4].fmask != 0 && A.filter3;
+    if (filt) {
+      const LevelPlan &L4 = P.lv[4];
+      LRef Lx[7];
+      int nx = 0, fdrv = 0;
+      uint32_t best = 0xffffffffu;
+      for (int b = 0; b < L4.nb; ++b)
+        if ((L4.fmask >> b) & 1) {
+          Lx[nx] = list_of(A, f[L4.bpos[b]], L4.bview[b], acc, lane, pin);
+          const uint32_t szx = Lx[nx].ml + Lx[nx].xl;
+          if (szx < best) {
+            best = szx;
+            fdrv = nx;
+          }
+          ++nx;
+        }
+      // F as two sorted runs: survivors of the driver's main run, then of its delta run (an updated vertex's
+      // view is main ∪ delta, each sorted, not sorted together); the filter binary-searches each run
+      const LRef dfull = Lx[fdrv];
+      Lx[fdrv].xl = 0;
+      nF1 = warp_isect<true>(A, nullptr, 0, Lx, nx, fdrv, nullptr, 0, L4.label, fbuf, lane);
+      __syncwarp();
+      nF = nF1;
+      if (dfull.xl) {
+        Lx[fdrv].m = dfull.x;
+        Lx[fdrv].ml = dfull.xl;
+        Lx[fdrv].dev = true;
+        nF += warp_isect<true>(A, nullptr, 0, Lx, nx, fdrv, nullptr, 0, L4.label, fbuf + nF1, lane);
+        __syncwarp();
+      }
+      if (nF == 0) {  // no position-4 candidate for any level-3 node of this entry
+        ++x_pruned;
+        continue;
+      }
+    }
+    // level 3 is iterated over it3p[0..it3n): position 3's set itself, or — when the level-3 filter ran and a later
+    // position reuses position 3's whole set (code motion) — the filter's survivors in their own buffer
+    const int32_t *it3p = nullptr;
+    uint32_t it3n = 0;
+    bool reuse3 = false;
+    for (int q = 4; q < k; ++q) reuse3 |= P.lv[q].reuse == 3;
     if (task) {
       int32_t *own = stack;  // this warp's level-3 buffer: a private, L1-safe copy of the shared set
       for (uint32_t i = lane; i < tk.n; i += 32) own[i] = __ldcg(A.arena + tk.off + i);
+      it3p = own;
+      it3n = tk.n;
+      if (tk.pad) {  // the producer's filtered iteration list follows the set in the arena
+        it3n = tk.pad - 1;
+        for (uint32_t i = lane; i < it3n; i += 32) ibuf[i] = __ldcg(A.arena + tk.off + tk.n + i);
+        it3p = ibuf;
+      }
       __syncwarp();
       set[3] = own;
       sz[3] = tk.n;
@@ -846,31 +992,47 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           sz[p] = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, out, lane, vlo, vhi);
           if (p == 3) x_l3 += sz[p];
           else if (p == 4) x_l4 += sz[p];
+          if (p == 3) {
+            it3p = out;
+            it3n = sz[3];
+          }
+          if (p == 3 && filt && sz[3]) {  // keep only the level-3 nodes whose own list meets F
+            __syncwarp();
+            int32_t *dst = reuse3 ? ibuf : out;
+            it3n = filter_level3(A, P.lv[4].bview[P.lv[4].f3], out, sz[3], dst, fset, nF1, nF, acc, lane);
+            it3p = dst;
+            if (!reuse3) sz[3] = it3n;
+            x_l3f += it3n;
+          }
           __syncwarp();
           set[p] = out;
           it[p] = 0;
           lvl = p;
           descend = false;
-          if (p == 3 && sharing && sz[3] > kSplitMin) {
-            // share this level-3 set: copy it to the arena and publish slices of it as tasks
-            const uint32_t n3 = sz[3], nt = (n3 + kTaskSize - 1) / kTaskSize;
+          if (p == 3 && sharing && it3n > kSplitMin) {
+            // share this level-3 set: copy it (and a separate iteration list) to the arena and publish slices of the
+            // iteration list as tasks
+            const bool sep = it3p != out;
+            const uint32_t n3 = sz[3], ni = it3n, nt = (ni + kTaskSize - 1) / kTaskSize;
             unsigned long long off = 0, t0 = 0;
             if (lane == 0) {
-              off = atomicAdd(&A.cnt[CNT_ARENA], (unsigned long long)n3);
+              off = atomicAdd(&A.cnt[CNT_ARENA], (unsigned long long)(n3 + (sep ? ni : 0)));
               t0 = atomicAdd(&A.cnt[CNT_TAIL], (unsigned long long)nt);
             }
             off = __shfl_sync(kFull, off, 0);
             t0 = __shfl_sync(kFull, t0, 0);
-            if (off + n3 <= A.arena_cap && t0 + nt <= A.task_cap) {
+            if (off + n3 + (sep ? ni : 0) <= A.arena_cap && t0 + nt <= A.task_cap) {
               for (uint32_t i = lane; i < n3; i += 32) A.arena[off + i] = out[i];
+              if (sep)
+                for (uint32_t i = lane; i < ni; i += 32) A.arena[off + n3 + i] = it3p[i];
               for (uint32_t t = lane; t < nt; t += 32) {
                 Task q;
                 q.e = e;
                 q.off = off;
                 q.n = n3;
                 q.lo = t * kTaskSize;
-                q.hi = min(n3, (t + 1) * kTaskSize);
-                q.pad = 0;
+                q.hi = min(ni, (t + 1) * kTaskSize);
+                q.pad = sep ? ni + 1 : 0;
                 A.tasks[t0 + t] = q;
               }
               __threadfence();
@@ -900,9 +1062,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         }
       }
       // choose the next element at the deepest open position (>= 3)
-      while (lvl >= 3 && it[lvl] >= (lvl == 3 ? min(end3, sz[3]) : sz[lvl])) --lvl;
+      while (lvl >= 3 && it[lvl] >= (lvl == 3 ? min(end3, it3n) : sz[lvl])) --lvl;
       if (lvl < 3) break;
-      f[lvl] = set[lvl][it[lvl]++];
+      f[lvl] = (lvl == 3 ? it3p : set[lvl])[it[lvl]++];
       descend = true;
     }
     (void)lvl;
@@ -914,6 +1076,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     atomicAdd(&A.cnt[CNT_X_L3], x_l3);
     atomicAdd(&A.cnt[CNT_X_L4], x_l4);
     atomicAdd(&A.cnt[CNT_X_LAST], x_last);
+    atomicAdd(&A.cnt[CNT_X_L3F], x_l3f);
   }
 }
 

@@ -47,7 +47,8 @@ enum Counter {
   CNT_X_L3 = 36,
   CNT_X_L4 = 37,
   CNT_X_LAST = 38,
-  CNT_N = 39
+  CNT_X_L3F = 39,  // level-3 nodes kept by the level-3 filter
+  CNT_N = 40
 };
 
 struct MatchArgs {
@@ -96,6 +97,8 @@ struct MatchArgs {
   uint32_t stage_epoch;          // 24 bits, never 0
   uint32_t stage_min;            // shortest list (ints) routed through the arena
   int32_t stage_policy;          // shared-memory staging of device-resident probe lists: 0 bytes model, 1 latency
+  int32_t filter3;               // level-3 filter on (LevelPlan::fmask)
+  int32_t hoist;                 // hoisted last-level set on (LevelPlan::hmask)
   uint32_t *touched;             // B_comp measurement: bitmap of vertices whose main list was read (nullptr = off)
   // NVLink peer cache: the linked peers' descriptor arrays and cache address ranges of this
   // batch; a zero-copy miss whose list a peer holds in HBM is read from there (peer / NVLink) instead

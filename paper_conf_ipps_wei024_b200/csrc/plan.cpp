@@ -205,6 +205,20 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
         }
         // loop-invariant code motion of the last level (k >= 5): the lists of backward positions <= 2 are fixed
         // for a whole level-2 entry; with >= 2 of them their intersection is computed once per entry
+        // level-3 filter (k >= 5): position 4's lists at positions <= 2 against each level-3 node's own list
+        L.fmask = 0;
+        L.f3 = -1;
+        if (p == 4 && k >= 5) {
+          int msk = 0, b3 = -1;
+          for (int b = 0; b < L.nb; ++b) {
+            if (L.bpos[b] <= 2) msk |= 1 << b;
+            if (L.bpos[b] == 3) b3 = b;
+          }
+          if (b3 >= 0 && msk) {
+            L.fmask = (int8_t)msk;
+            L.f3 = (int8_t)b3;
+          }
+        }
         L.hmask = 0;
         if (p == k - 1 && k >= 5 && L.reuse < 0) {
           int cnt = 0, msk = 0;
@@ -216,6 +230,7 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
           if (cnt >= 2) L.hmask = (int8_t)msk;
         }
       }
+
     }
   }
   out = q;
