@@ -458,7 +458,8 @@ def main():
     keys = ("ms_total", "ms_match", "ms_level2", "ms_extend", "ms_normalize", "ms_estimate", "ms_pack", "ms_copy",
             "ms_allreduce", "ms_merge", "hit_bytes", "miss_bytes", "delta_bytes", "hit_bytes_ext", "miss_bytes_ext",
             "delta_bytes_ext", "host_copied_bytes", "cache_bytes", "cached_vertices", "units", "frontier",
-            "h2d_bytes", "d2h_bytes", "kernel_launches", "stage_fill_bytes", "stage_lists", "stage_hit_bytes")
+            "h2d_bytes", "d2h_bytes", "kernel_launches", "stage_fill_bytes", "stage_lists", "stage_hit_bytes",
+            "ms_walks", "walk_alg_bytes", "walk_fill_bytes")
     for step in recs:
         edges += step[0][3]["n_ins"] + step[0][3]["n_del"]
         for q, a, r, st in step:
@@ -472,25 +473,29 @@ def main():
                                                  "cached_vertices")}
     value = edges / (ms_dev / 1e3)
     e2e_value = edges / (ms_host / 1e3)
-    # dominant kernel: the last-level kernel (k_last4 / k_extend) of the heaviest query
-    dom_q = max(per_q, key=lambda q: per_q[q]["ms_extend"] + per_q[q]["ms_level2"])
+    # dominant kernel (CUDA-event times): the matching extension (k_last4 / k_extend) of a query, or a query's GPU
+    # random walks (k_walks_l1 + k_walks, step 2)
+    cands = []
+    for q, d in per_q.items():
+        cands.append((d["ms_extend"], q, "ext"))
+        cands.append((d["ms_walks"], q, "walks"))
+    _, dom_q, dom_kind = max(cands)
     dq = per_q[dom_q]
-    kern = "k_extend" if dq["ms_extend"] > 0 else "k_level2"
-    if kern == "k_extend":
-        if gi.query(dom_q)[0] == 4:
-            kern = "k_last4"  # k = 4 count mode: the last level runs in the lean kernel
+    if dom_kind == "walks":
+        kern = "k_walks"
+        hit, miss, dlt = dq["walk_alg_bytes"], 0, 0  # walks' list bytes (arena / cache / U lists: HBM-resident)
+        kms = dq["ms_walks"] / K
+    else:
+        kern = "k_last4" if gi.query(dom_q)[0] == 4 else "k_extend"  # k = 4: the lean last-level kernel (§5)
         hit, miss, dlt = dq["hit_bytes_ext"], dq["miss_bytes_ext"], dq["delta_bytes_ext"]
         kms = dq["ms_extend"] / K
-    else:
-        hit, miss, dlt = dq["hit_bytes"], dq["miss_bytes"], dq["delta_bytes"]
-        kms = dq["ms_level2"] / K
     # per link: algorithmic list bytes served from HBM (the cache, the batch's device-resident delta
     # data and lists of U, and lists staged in the batch arena) vs the HBM peak; bytes that really crossed the host
     # link (bulk copies of zero-copy lists: the arena fills and the warps' staging) vs the measured zero-copy peak
-    stage_hit = dq["stage_hit_bytes"]
+    stage_hit = dq["stage_hit_bytes"] if dom_kind == "ext" else 0
     b_hbm = (hit + dlt + stage_hit) / K
     b_alg = (hit + dlt + miss) / K
-    b_host = dq["host_copied_bytes"] / K
+    b_host = (dq["host_copied_bytes"] if dom_kind == "ext" else dq["walk_fill_bytes"]) / K
     peak, peak_kind = load_peaks()
     sec = kms / 1e3 if kms > 0 else float("inf")
     link = None
@@ -516,7 +521,8 @@ def main():
     top = link_obj if bound == "host_link" else hbm_obj
     bq = (bcomp or {}).get(dom_q)
     roofline = {"bound": bound, "kernel": f"{kern} ({dom_q})", "achieved": top["achieved"], "peak": top["peak"],
-                "unit": "GB/s", "frac": top["frac"], "traffic": load_traffic(w.name, dom_q),
+                "unit": "GB/s", "frac": top["frac"],
+                "traffic": load_traffic(w.name, dom_q + (":walks" if dom_kind == "walks" else "")),
                 "launch_ms": kms, "algorithmic_bytes_per_launch": b_alg,
                 "hbm": hbm_obj, "host_link": link_obj,
                 "b_comp": None if bq is None else {
@@ -581,6 +587,7 @@ def main():
                           "miss_gb": d["miss_bytes"] / K / 1e9, "host_copied_gb": d["host_copied_bytes"] / K / 1e9,
                           "stage_fill_gb": d["stage_fill_bytes"] / K / 1e9,
                           "stage_hit_gb": d["stage_hit_bytes"] / K / 1e9,
+                          "ms_walks": d["ms_walks"] / K, "walk_alg_gb": d["walk_alg_bytes"] / K / 1e9,
                           "bcomp_miss_gb": None if bcomp is None else bcomp[q]["bcomp_miss_bytes"] / 1e9,
                           "bcomp_hit_gb": None if bcomp is None else bcomp[q]["bcomp_hit_bytes"] / 1e9,
                           "frontier": d["frontier"] / K} for q, d in per_q.items()},

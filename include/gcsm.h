@@ -138,6 +138,10 @@ typedef struct {
                                 main lists the query's kernels touched, by home (HBM cache / pinned host / uploaded
                                 lists of U); only with GCSM_BCOMP=1 at create (measurement mode), else 0 */
   uint64_t peer_bytes;       /* algorithmic list bytes read from a linked peer's HBM cache (gcsm_link_peers) */
+  uint64_t walk_fill_bytes;  /* bytes the GPU walks (step 2) fetched into the staging arena (all queries) */
+  uint64_t walk_stage_lists; /* lists they staged */
+  uint64_t walk_alg_bytes;   /* this query's walks: algorithmic list bytes (driver scans + probed lists, §8d) */
+  double ms_walks;           /* this query's GPU walk kernels (k_walks_l1 + k_walks, CUDA events; 0 if none) */
 } gcsm_stats;
 
 /* Fills *opt with the defaults (device -1, world 1, seed 0x6C53, all cores,

@@ -42,7 +42,8 @@ class Stats(ctypes.Structure):
                 "ms_allreduce", "ms_merge", "ms_total"]] + \
               [(name, ctypes.c_uint64) for name in
                ["stage_fill_bytes", "stage_lists", "stage_hit_bytes", "bcomp_hit_bytes", "bcomp_miss_bytes",
-                "bcomp_delta_bytes", "peer_bytes"]]
+                "bcomp_delta_bytes", "peer_bytes", "walk_fill_bytes", "walk_stage_lists", "walk_alg_bytes"]] + \
+              [("ms_walks", ctypes.c_double)]
 
 
 _lib = None

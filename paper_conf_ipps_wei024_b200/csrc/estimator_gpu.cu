@@ -21,7 +21,6 @@
 // them into FMAs: the same IEEE operation sequence gives the same doubles. BINV's r0 = (1-p)^n comes from a host
 // table (glibc pow), BTRD's Stirling terms for k < 10 from a host table (glibc lgamma); BTRD's log is CUDA's
 // (max 1 ulp; it decides only comparisons that are not within an ulp of a tie — DESIGN.md).
-#include <cub/cub.cuh>
 
 #include "estimator_gpu.cuh"
 
@@ -223,6 +222,7 @@ struct WalkArgs {
   unsigned long long *cursor;
   BinTab T;
   StageRef stage;            // fetch-once staging (stage.state == nullptr: off)
+  unsigned long long *alg_cnt;  // algorithmic list bytes read (or nullptr)
   uint32_t stage_min;
   unsigned long long *stage_cnt;
   const char *dev_lo[2], *dev_hi[2];
@@ -328,13 +328,17 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
 }
 
 // Levels >= 2 (phase B, k >= 5): warp per level-2 node, DFS over the rest of its subtree.
-__global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
+#ifndef GCSM_WALK_MINBLOCKS
+#define GCSM_WALK_MINBLOCKS 3  // resident 256-thread blocks per SM for k_walks (latency hiding of its list reads)
+#endif
+__global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const WalkArgs A) {
   __shared__ EstW sw[kEW];
   const BinTab T = A.T;
   const int lane = threadIdx.x & 31;
   EstW &W = sw[threadIdx.x >> 5];
   const unsigned long long n2 = min(*(volatile unsigned long long *)A.f2_count, (unsigned long long)A.f2_cap);
   unsigned long long wfill = 0, wlists = 0, whit = 0;  // fetch-once staging counters
+  unsigned long long walg = 0;                         // algorithmic list bytes (driver scans + probes)
   for (;;) {
     unsigned long long u = 0;
     if (lane == 0) u = atomicAdd(A.cursor2, 1ull);
@@ -345,6 +349,7 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
         atomicAdd(A.stage_cnt + 1, wlists);
         atomicAdd(A.stage_cnt + 2, whit);
       }
+      if (lane == 0 && A.alg_cnt && walg) atomicAdd(A.alg_cnt, walg);
       return;
     }
     const EstNode2 N = A.f2[u];
@@ -383,18 +388,33 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
         uint32_t best = 0xffffffffu;
         for (int b = 0; b < nb; ++b) {
           L[b] = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
-          const char *pc = reinterpret_cast<const char *>(L[b].m);
-          if (A.stage.state && L[b].ml >= A.stage_min && !(pc >= A.dev_lo[0] && pc < A.dev_hi[0]) &&
-              !(pc >= A.dev_lo[1] && pc < A.dev_hi[1]))  // zero-copy: fetched once per batch into HBM
-            L[b].m = stage_fetch(A.stage, W.f[Lp.bpos[b]], L[b].m, L[b].ml, wfill, wlists, whit, lane);
           const uint32_t t = L[b].ml + L[b].xl;
           if (t < best) {
             best = t;
             drv = b;
           }
         }
+        // zero-copy lists: the driver (scanned whole) is fetched once per batch into HBM; a probed list (only
+        // for the rare children with B' > 0) uses the staged copy when one exists, else a few in-place reads
+        for (int b = 0; b < nb; ++b) {
+          const char *pc = reinterpret_cast<const char *>(L[b].m);
+          if (!A.stage.state || L[b].ml < A.stage_min || (pc >= A.dev_lo[0] && pc < A.dev_hi[0]) ||
+              (pc >= A.dev_lo[1] && pc < A.dev_hi[1]))
+            continue;
+          const int32_t vb = W.f[Lp.bpos[b]];
+          if (b == drv) {
+            L[b].m = stage_fetch(A.stage, vb, L[b].m, L[b].ml, wfill, wlists, whit, lane);
+          } else {
+            const unsigned long long st = stage_word(A.stage.state + vb);
+            if ((st >> 40) == A.stage.epoch && (st & kStReady) && (st & kStOff) != kStOff) {
+              L[b].m = A.stage.arena + (st & kStOff);
+              whit += 4ull * L[b].ml;
+            }
+          }
+        }
         if (lane == 0)
           for (int b = 0; b < nb; ++b) S.pm[b] = L[b].m;
+        walg += 4ull * (L[drv].ml + L[drv].xl);  // the driver is scanned whole
         const int64_t Bn = (int64_t)S.B;
         const double pD = T.pD;
         unsigned long long t53 = ~0ull;
@@ -475,6 +495,7 @@ __global__ void __launch_bounds__(kEW * 32) k_walks(const WalkArgs A) {
           if (b == drv) continue;
           const LR Lb = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
           const int32_t *bm = S.pm[b];
+          walg += 4ull * (Lb.ml + Lb.xl);  // probed (binary search: an upper bound of the bytes it needs)
 #pragma unroll 1
           for (int j = 0; j < 4; ++j)
             if (ok[j]) ok[j] = has(bm, Lb.ml, v[j]) || (Lb.xl && has(Lb.x, Lb.xl, v[j]));
@@ -623,8 +644,7 @@ __global__ void __launch_bounds__(256) k_hist(const unsigned long long *bits, co
 // One block of 1024 threads: bins in descending order, 4 per thread; the first bin where the cumulative bytes
 // pass the budget is the cut bucket of this level.
 __global__ void __launch_bounds__(1024) k_cut(const unsigned long long *hist, SelState *st, uint64_t budget, int level) {
-  using BS = cub::BlockScan<unsigned long long, 1024>;
-  __shared__ typename BS::TempStorage tmp;
+  __shared__ unsigned long long wsum[32];
   __shared__ int win;
   if (!st->found) return;
   if (threadIdx.x == 0) win = 1 << 30;
@@ -636,8 +656,25 @@ __global__ void __launch_bounds__(1024) k_cut(const unsigned long long *hist, Se
     v[j] = d < nbins ? h[nbins - 1 - d] : 0ull;
     tot += v[j];
   }
-  unsigned long long before;
-  BS(tmp).ExclusiveSum(tot, before);
+  // exclusive block scan of the per-thread totals (warp shuffles, then the 32 warp totals)
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  unsigned long long x = tot;
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[wi] = x;
+  __syncthreads();
+  if (wi == 0) {
+    unsigned long long t = wsum[lane];
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(FULL, t, o);
+      if (lane >= o) t += y;
+    }
+    wsum[lane] = t;
+  }
+  __syncthreads();
+  const unsigned long long before = x - tot + (wi ? wsum[wi - 1] : 0ull);
   __syncthreads();
   const unsigned long long above = st->above;
   unsigned long long cum = above + before;
@@ -772,21 +809,133 @@ __global__ void k_est_gather(const int32_t *tids, int64_t n, const unsigned long
 
 int gs_grid(int64_t n, int per = 256) { return (int)std::max<int64_t>(1, std::min<int64_t>((n + per - 1) / per, 148 * 8)); }
 
+// ---- device-wide scans and the flagged select of the ranking (hand-written; three passes: 2048-element block
+// scans, one block scanning the block totals, the carries added back). The element count is the host bound n,
+// or the device-resident count *nd when given (the batch's touched set), so only live elements are scanned.
+constexpr int kScanT = 256, kScanIt = 8, kScanBlk = kScanT * kScanIt;
+
+__device__ __forceinline__ int64_t live_n(const unsigned long long *nd, int64_t n) {
+  return nd ? (int64_t)min((unsigned long long)n, *nd) : n;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kScanT) k_scan_blocks(const T *in, T *out, const unsigned long long *nd, int64_t nmax,
+                                                        T *bsum, int inclusive) {
+  __shared__ T ws[kScanT / 32];
+  const int64_t n = live_n(nd, nmax);
+  const int64_t base = (int64_t)blockIdx.x * kScanBlk + (int64_t)threadIdx.x * kScanIt;
+  T v[kScanIt], run = 0;
+#pragma unroll
+  for (int i = 0; i < kScanIt; ++i) {
+    const T x = base + i < n ? in[base + i] : (T)0;
+    v[i] = inclusive ? run + x : run;
+    run += x;
+  }
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  T xs = run;  // inclusive scan of the per-thread totals in the warp
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const T y = __shfl_up_sync(FULL, xs, o);
+    if (lane >= o) xs += y;
+  }
+  if (lane == 31) ws[w] = xs;
+  __syncthreads();
+  if (w == 0) {
+    T t = lane < kScanT / 32 ? ws[lane] : (T)0;
+#pragma unroll
+    for (int o = 1; o < kScanT / 32; o <<= 1) {
+      const T y = __shfl_up_sync(FULL, t, o);
+      if (lane >= o) t += y;
+    }
+    if (lane < kScanT / 32) ws[lane] = t;
+  }
+  __syncthreads();
+  const T excl = xs - run + (w ? ws[w - 1] : (T)0);
+#pragma unroll
+  for (int i = 0; i < kScanIt; ++i)
+    if (base + i < n) out[base + i] = v[i] + excl;
+  if (threadIdx.x == kScanT - 1) bsum[blockIdx.x] = excl + run;  // 0 for blocks past the live count
+}
+
+template <typename T>
+__global__ void __launch_bounds__(1024) k_scan_totals(T *bsum, int64_t nb) {  // exclusive, in place
+  __shared__ T ws[32];
+  __shared__ T carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int64_t s0 = 0; s0 < nb; s0 += 1024) {
+    const int64_t i = s0 + threadIdx.x;
+    const T v = i < nb ? bsum[i] : (T)0;
+    T x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const T y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) ws[w] = x;
+    __syncthreads();
+    if (w == 0) {
+      T t = ws[lane];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const T y = __shfl_up_sync(FULL, t, o);
+        if (lane >= o) t += y;
+      }
+      ws[lane] = t;
+    }
+    __syncthreads();
+    const T incl = x + (w ? ws[w - 1] : (T)0);
+    if (i < nb) bsum[i] = carry + incl - v;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry += incl;
+    __syncthreads();
+  }
+}
+
+template <typename T>
+__global__ void k_scan_carry(T *out, const unsigned long long *nd, int64_t nmax, const T *bsum) {
+  const int64_t n = live_n(nd, nmax);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] += bsum[i / kScanBlk];
+}
+
+template <typename T>
+cudaError_t scan(const T *in, T *out, const unsigned long long *nd, int64_t nmax, bool inclusive, void *tmp,
+                 cudaStream_t s, uint64_t &L) {
+  if (nmax <= 0) return cudaSuccess;
+  const int64_t nb = (nmax + kScanBlk - 1) / kScanBlk;
+  T *bsum = reinterpret_cast<T *>(tmp);
+  k_scan_blocks<T><<<(unsigned)nb, kScanT, 0, s>>>(in, out, nd, nmax, bsum, inclusive ? 1 : 0);
+  k_scan_totals<T><<<1, 1024, 0, s>>>(bsum, nb);
+  k_scan_carry<T><<<gs_grid(nmax), 256, 0, s>>>(out, nd, nmax, bsum);
+  L += 3;
+  return cudaGetLastError();
+}
+
+// out[pos(i)] = in[i] for the flagged i < n (order kept), *count = their number; pos = exclusive scan of the flags
+__global__ void k_flags_u32(const uint8_t *flag, uint32_t *f32, const unsigned long long *nd, int64_t nmax) {
+  const int64_t n = live_n(nd, nmax);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    f32[i] = flag[i] ? 1u : 0u;
+}
+
+__global__ void k_select_scatter(const int32_t *in, const uint8_t *flag, const uint32_t *pos,
+                                 const unsigned long long *nd, int64_t nmax, int32_t *out, unsigned long long *count) {
+  const int64_t n = live_n(nd, nmax);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (flag[i]) out[pos[i]] = in[i];
+    if (i == n - 1) *count = (unsigned long long)pos[i] + (flag[i] ? 1ull : 0ull);
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0 && n == 0) *count = 0;
+}
+
 }  // namespace
 
 size_t cache_step_tmp_bytes(int32_t n) {
-  size_t a = 0, b = 0, c = 0;
-  const int64_t W = ((int64_t)n + 31) / 32;
-  cub::DeviceScan::ExclusiveSum(nullptr, a, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(W + 1));
-  // num_items types must match the launches in launch_cache_step (cub's dispatch, hence its scratch size,
-  // depends on them)
-  cub::DeviceScan::InclusiveSum(nullptr, b, (unsigned long long *)nullptr, (unsigned long long *)nullptr, (int)n);
-  size_t b2 = 0;
-  cub::DeviceScan::ExclusiveSum(nullptr, b2, (unsigned long long *)nullptr, (unsigned long long *)nullptr, (int)n);
-  b = std::max(b, b2);
-  cub::DeviceSelect::Flagged(nullptr, c, (int32_t *)nullptr, (uint8_t *)nullptr, (int32_t *)nullptr,
-                             (unsigned long long *)nullptr, (int)n);
-  return std::max(a, std::max(b, c)) + 256;
+  // the scans' block totals (u64), then the select's u32 flags and positions
+  const size_t nb = ((size_t)n + 2 + kScanBlk - 1) / kScanBlk + 1;
+  return 8 * nb + 8 * ((size_t)n + 2) + 256;
 }
 
 cudaError_t launch_patch_vdesc_host(VDesc *vdesc, unsigned long long *hptr, const int64_t *idx, const VDesc *val,
@@ -862,22 +1011,23 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.stage = c.stage;
       A.stage_min = c.stage_min;
       A.stage_cnt = c.stage_cnt;
+      A.alg_cnt = c.alg_cnt[q];
       for (int r = 0; r < 2; ++r) {
         A.dev_lo[r] = c.dev_lo[r];
         A.dev_hi[r] = c.dev_hi[r];
       }
       const int ga = (int)std::max<int64_t>(1, std::min<int64_t>((Q.n_items + kEW - 1) / kEW, 148 * 8));
+      if (c.ev_walk && q < GCSM_MAX_QUERIES) cudaEventRecord(c.ev_walk[2 * q], s);
       LK(k_walks_l1<<<ga, kEW * 32, 0, s>>>(A));
-      if (Q.k >= 5) LK(k_walks<<<148 * 2, kEW * 32, 0, s>>>(A));
+      if (Q.k >= 5) LK(k_walks<<<148 * GCSM_WALK_MINBLOCKS, kEW * 32, 0, s>>>(A));
+      if (c.ev_walk && q < GCSM_MAX_QUERIES) cudaEventRecord(c.ev_walk[2 * q + 1], s);
     }
   }
   // touched set in id order
   uint32_t *wcnt = c.wcnt;
   uint32_t *woff = c.woff;
   LK(k_wcount<<<gs_grid(W + 1), 256, 0, s>>>(c.touched, W, wcnt));
-  size_t tb = c.cub_tmp_bytes;
-  if ((e = cub::DeviceScan::ExclusiveSum(c.cub_tmp, tb, wcnt, woff, (int)(W + 1), s)) != cudaSuccess) return e;
-  ++L;
+  if ((e = scan<uint32_t>(wcnt, woff, nullptr, W + 1, false, c.cub_tmp, s, L)) != cudaSuccess) return e;
   LK(k_wwrite<<<gs_grid(W), 256, 0, s>>>(c.touched, W, woff, c.tids, c.st));
   ScoreArgs S{};
   S.nq = c.nq;
@@ -897,20 +1047,23 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
     LK(k_cut<<<1, 1024, 0, s>>>(c.hist, c.st, c.budget, lv));
   }
   LK(k_ties<<<G, 256, 0, s>>>(c.bits, c.bytes, c.st, n, c.off));
-  tb = c.cub_tmp_bytes;
-  if ((e = cub::DeviceScan::InclusiveSum(c.cub_tmp, tb, c.off, c.scan, (int)n, s)) != cudaSuccess) return e;
-  ++L;
+  if ((e = scan<unsigned long long>(c.off, c.scan, &c.st->n_touched, n, true, c.cub_tmp, s, L)) != cudaSuccess)
+    return e;
   LK(k_select<<<G, 256, 0, s>>>(c.bits, c.bytes, c.st, n, c.budget, c.scan, c.flag));
-  tb = c.cub_tmp_bytes;
-  if ((e = cub::DeviceScan::ExclusiveSum(c.cub_tmp, tb, c.scan, c.off, (int)n, s)) != cudaSuccess) return e;
-  ++L;
+  if ((e = scan<unsigned long long>(c.scan, c.off, &c.st->n_touched, n, false, c.cub_tmp, s, L)) != cudaSuccess)
+    return e;
   LK(k_copy<<<G, 256, 0, s>>>(c.tids, c.st, c.flag, c.off, c.bytes, c.vdesc, c.cache));
   LK(k_reset_prev<<<G, 256, 0, s>>>(c.prev_sel, c.st, c.vdesc, c.hptr));
   LK(k_set_new<<<G, 256, 0, s>>>(c.tids, c.st, c.flag, c.off, c.vdesc, c.cache));
-  tb = c.cub_tmp_bytes;
-  if ((e = cub::DeviceSelect::Flagged(c.cub_tmp, tb, c.tids, c.flag, c.prev_sel, &c.st->prev_sel, (int)n, s)) != cudaSuccess)
-    return e;
-  ++L;
+  {  // the selection, compacted in id order (the next batch's previous selection)
+    const size_t nb = ((size_t)n + kScanBlk - 1) / kScanBlk + 1;
+    uint32_t *f32 = reinterpret_cast<uint32_t *>(reinterpret_cast<char *>(c.cub_tmp) + 8 * nb);
+    uint32_t *pos = f32 + (n + 1);  // two u32 arrays of n + 1 in the 8 (n + 2) bytes
+    LK(k_flags_u32<<<gs_grid(n), 256, 0, s>>>(c.flag, f32, &c.st->n_touched, n));
+    if ((e = scan<uint32_t>(f32, pos, &c.st->n_touched, n, false, c.cub_tmp, s, L)) != cudaSuccess) return e;
+    LK(k_select_scatter<<<gs_grid(n), 256, 0, s>>>(c.tids, c.flag, pos, &c.st->n_touched, n, c.prev_sel,
+                                                  &c.st->prev_sel));
+  }
   LK(k_sel_stats<<<1, 1, 0, s>>>(c.st, c.cnt_cached, 1));
 #undef LK
   *launches += L;

@@ -95,6 +95,8 @@ struct CacheStep {
   unsigned long long *cnt_cached;  // 3 counters: vertices, bytes, internal error
   // fetch-once staging of the walks' zero-copy lists (stage.state == nullptr: off); lists already in device memory
   // at walk time (the last batch's cache, the batch's U lists) are read in place
+  cudaEvent_t *ev_walk = nullptr;  // 2 per query: around its walk kernels (timing, may be null)
+  unsigned long long *alg_cnt[GCSM_MAX_QUERIES] = {};  // per query: algorithmic list bytes of its walks
   StageRef stage{};
   uint32_t stage_min = 1;
   unsigned long long *stage_cnt = nullptr;  // fill bytes, lists, hit bytes

@@ -149,6 +149,8 @@ struct gcsm_ctx {
     uint64_t add_cap = 0, rem_cap = 0;
     std::vector<std::pair<int32_t *, uint32_t>> retired;  // host arrays replaced by this batch's merge
     const char *cache_lo = nullptr, *cache_hi = nullptr;  // the HBM cache this batch's kernels read (peers too)
+    std::vector<cudaEvent_t> ev_walk;  // 2 per query around its walk kernels
+    bool walks_timed = false;
   };
   Slot slots[2];
   uint64_t waited = 0;  // batches whose results have been collected
@@ -296,6 +298,7 @@ gcsm_ctx::~gcsm_ctx() {
       if (p) cudaFreeHost(p);
     for (cudaEvent_t e : {sl.ev_a0, sl.ev_a1, sl.ev_c0, sl.ev_c1, sl.ev_done, sl.ev_up, sl.ev_l2})
       if (e) cudaEventDestroy(e);
+    for (cudaEvent_t e : sl.ev_walk) cudaEventDestroy(e);
     for (auto &pq : sl.q) {
       for (cudaEvent_t e : {pq.ev_m0, pq.ev_m1})
         if (e) cudaEventDestroy(e);
@@ -895,11 +898,19 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.cub_tmp_bytes = ctx->cubtmp_bytes;
   c.cache = ctx->d_cache;
   c.cnt_cached = sl.d_cnt + CNT_CACHED;
+  while (sl.ev_walk.size() < 2 * (size_t)nq) {  // walk timing events (per query)
+    cudaEvent_t ev;
+    CK(cudaEventCreate(&ev));
+    sl.ev_walk.push_back(ev);
+  }
+  c.ev_walk = sl.ev_walk.data();
+  for (int qi = 0; qi < nq && qi < GCSM_MAX_QUERIES; ++qi) c.alg_cnt[qi] = sl.d_cnt + (size_t)qi * CNT_N + CNT_WALG;
+  sl.walks_timed = est_on;
   if (ctx->walk_stage_epoch && !std::getenv("GCSM_NO_WALK_STAGE")) {  // the walks' zero-copy lists through the arena
     c.stage = StageRef{ctx->d_stage_state, ctx->d_stage_arena, ctx->stage_cap, ctx->d_stage_bump,
                        ctx->walk_stage_epoch};
     c.stage_min = ctx->stage_min;
-    c.stage_cnt = sl.d_cnt + CNT_STAGE_FILL;  // query 0's counters
+    c.stage_cnt = sl.d_cnt + CNT_WFILL;  // query 0's block
     c.dev_lo[0] = ctx->cache_valid ? ctx->d_cachebuf[ctx->cache_cur] : nullptr;  // lists cached by the last batch
     c.dev_hi[0] = c.dev_lo[0] ? c.dev_lo[0] + ctx->cache_cap : nullptr;
     c.dev_lo[1] = reinterpret_cast<const char *>(sl.d_ulist);  // the batch's U lists
@@ -1841,6 +1852,15 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.delta_bytes = h[CNT_ACC_L2 + 2] + st.delta_bytes_ext;
     st.host_copied_bytes = h[CNT_COPIED] + h[CNT_STAGE_FILL];  // warp staging copies + arena fills
     st.peer_bytes = h[CNT_PEER];
+    st.walk_alg_bytes = h[CNT_WALG];
+    st.walk_fill_bytes = sl.h_cnt[CNT_WFILL];  // the cache step's walks (all queries)
+    st.walk_stage_lists = sl.h_cnt[CNT_WLISTS];
+    st.ms_walks = 0;
+    if (sl.walks_timed && (size_t)(2 * qi + 1) < sl.ev_walk.size() && ctx->qs[qi].qp.k > 2) {
+      float mw = 0;
+      if (cudaEventElapsedTime(&mw, sl.ev_walk[2 * qi], sl.ev_walk[2 * qi + 1]) == cudaSuccess) st.ms_walks = mw;
+      cudaGetLastError();
+    }
     st.stage_fill_bytes = h[CNT_STAGE_FILL];
     st.stage_lists = h[CNT_STAGE_LISTS];
     st.stage_hit_bytes = h[CNT_STAGE_HIT];

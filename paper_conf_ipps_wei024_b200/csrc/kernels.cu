@@ -623,7 +623,7 @@ __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const
           m = q;
           pb += 4ull * ml;
         } else if (A.stage_state && ml >= A.stage_min) {
-          const unsigned long long st = __ldcg(A.stage_state + v);
+          const unsigned long long st = stage_word(A.stage_state + v);
           if ((st >> 40) == A.stage_epoch && (st & kStReady) && (st & kStOff) != kStOff) {
             m = A.stage_arena + (st & kStOff);
             sb += 4ull * ml;

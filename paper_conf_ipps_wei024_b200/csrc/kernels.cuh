@@ -48,7 +48,11 @@ enum Counter {
   CNT_X_L4 = 37,
   CNT_X_LAST = 38,
   CNT_X_L3F = 39,  // level-3 nodes kept by the level-3 filter
-  CNT_N = 40
+  CNT_WFILL = 40,  // the walks' fetch-once staging (query 0's block): bytes filled, lists, bytes served
+  CNT_WLISTS = 41,
+  CNT_WHIT = 42,
+  CNT_WALG = 43,   // per query: algorithmic list bytes its walks read (driver scans + membership probes, §8d)
+  CNT_N = 44
 };
 
 struct MatchArgs {

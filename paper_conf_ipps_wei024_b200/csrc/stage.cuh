@@ -50,6 +50,13 @@ __device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint
 // new epoch, so nothing stale is ever served.
 constexpr unsigned long long kStReady = 1ull << 39, kStOff = (1ull << 39) - 1;
 
+// the state word with acquire semantics (device scope): the arena copy published before it is visible after it
+__device__ __forceinline__ unsigned long long stage_word(const unsigned long long *w) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(w) : "memory");
+  return v;
+}
+
 __device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v, const int32_t *hp, uint32_t ml,
                                                    unsigned long long &sfill, unsigned long long &slists,
                                                    unsigned long long &shit, int lane) {
@@ -58,7 +65,7 @@ __device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v,
   int claimed = 0;
   if (lane == 0) {
     unsigned long long *w = A.state + v;
-    unsigned long long cur = __ldcg(w);
+    unsigned long long cur = stage_word(w);
     unsigned ns = 32;
     for (;;) {
       if ((cur & ~((1ull << 40) - 1)) == ep) {  // this batch's: ready, no room, or being loaded
@@ -68,7 +75,7 @@ __device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v,
         }
         __nanosleep(ns);
         if (ns < 2048) ns <<= 1;
-        cur = __ldcg(w);
+        cur = stage_word(w);
         continue;
       }
       const unsigned long long prev = atomicCAS(w, cur, ep | kStOff);  // claim: loading
@@ -88,8 +95,6 @@ __device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v,
       } else {
         res = off;
       }
-    } else {
-      __threadfence();  // acquire: the arena copy published before the state word
     }
   }
   claimed = __shfl_sync(0xffffffffu, claimed, 0);

@@ -1,6 +1,8 @@
 """Summarise .ncu-rep captures into profiles/ (text + JSON the bench reads for `roofline.traffic`).
 
-usage: python scripts/ncu_summary.py <round tag> <query>=<report.ncu-rep> ... [--launches file.csv]
+usage: python scripts/ncu_summary.py <round tag> <key>[@<launch index>,...]=<report.ncu-rep> ...
+  every launch of the report goes into profiles/ncu_<tag>.md; the traffic entry <key> (profiles/ncu_traffic.json,
+  read by bench.py) takes the launch given after '@' (default: the last one), or several as key1@i,key2@j
 """
 import csv
 import io
@@ -59,12 +61,19 @@ def main():
         if arg.startswith("--"):
             continue
         q, rep = arg.split("=", 1)
-        for i, d in enumerate(raw(rep)):
+        picks = {}  # launch index -> traffic key
+        for part in q.split(","):
+            key, _, idx = part.partition("@")
+            picks[int(idx) if idx else -1] = key
+        launches = raw(rep)
+        if -1 in picks:
+            picks[len(launches) - 1] = picks.pop(-1)
+        for i, d in enumerate(launches):
             name = d.get("Kernel Name", ("?", ""))[0]
             dur = num(d, "gpu__time_duration.sum")
             rd, wr = num(d, "dram__bytes_read.sum"), num(d, "dram__bytes_write.sum")
             sysr = num(d, "syslts__t_sectors_srcunit_tex_aperture_sysmem_op_read_lookup_miss.sum")
-            md.append(f"## {q}: `{name}` (launch {i})")
+            md.append(f"## {picks.get(i, q)}: `{name}` (launch {i})")
             md.append("")
             md.append("| metric | value | unit |")
             md.append("|---|---|---|")
@@ -77,8 +86,9 @@ def main():
                           f"{((rd or 0) + (wr or 0)) / dur / 1e9:.1f} GB/s; sysmem (zero-copy) reads "
                           f"{(sysr or 0) * 32 / 1e9:.3f} GB/launch = {(sysr or 0) * 32 / dur / 1e9:.1f} GB/s")
             md.append("")
-            traffic[q] = {"kernel": name, "dram_bytes": (rd or 0) + (wr or 0),
-                          "sysmem_read_bytes": (sysr or 0) * 32, "duration_s": dur, "tag": tag}
+            if i in picks:
+                traffic[picks[i]] = {"kernel": name, "dram_bytes": (rd or 0) + (wr or 0),
+                                     "sysmem_read_bytes": (sysr or 0) * 32, "duration_s": dur, "tag": tag}
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     with open(os.path.join(ROOT, "profiles", f"ncu_{tag}.md"), "w") as f:
         f.write("\n".join(md) + "\n")
