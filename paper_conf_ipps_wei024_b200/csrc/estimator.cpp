@@ -15,10 +15,10 @@
 //
 // Output: for every vertex read at least once, Σ B per tree level l = 1..k-2.
 // Implementation notes (exact reorderings, same distribution and same draws):
-//  * the binomial B' of a child only depends on the child's key, so a child
-//    whose draw is 0 is discarded before its (costly) membership probes when
-//    the inversion branch is used (B/D < 10): the first uniform decides B' = 0.
-#include <immintrin.h>
+//  * in the inversion branch (B/D < 10) the children with B' > 0 are found by
+//    skip sampling (geometric gaps over segments of the driver, then B' drawn
+//    conditioned on >= 1): the same law as one independent binomial per child,
+//    with work proportional to the children drawn, not to the driver (skip_gap).
 
 #include <algorithm>
 #include <cmath>
@@ -145,69 +145,54 @@ int64_t binomial(uint64_t key, int64_t n, double p) {
   return (double)n * p < 10.0 ? binv(U, n, p) : btrd(U, n, p);
 }
 
-// Exact B' = 0 decision of the inversion branch before the draw completes:
-// Bin(n, p) with n p < 10 and 0 < p <= 1/2 is 0 iff the first uniform <= (1-p)^n
-// (binv's r0, computed once per parent: every child of a node shares n and p).
-static inline bool first_uniform_le(uint64_t key, double r0) {
-  Uniforms U{key};
-  return !(U.next() > r0);
-}
+double stirling_small(int k) { return stirling_fc(k); }
 
-// Children of one node whose draw B' ~ Bin(B, p) is non-zero under the inversion branch: the first uniform of
-// the child's stream exceeds r0 = (1-p)^B. With u = m * 2^-53 (m = mix(key' + C) >> 11, exact) the test
-// u > r0 is the integer test m > floor(r0 * 2^53) — the same decision, evaluated 8 children at a time.
-static inline uint64_t mix_s(uint64_t z) {
-  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
-  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
-  return z ^ (z >> 31);
-}
-
-static void coin_filter_scalar(const int32_t *v, uint32_t n, uint64_t key, uint64_t T, std::vector<uint32_t> &out) {
-  for (uint32_t i = 0; i < n; ++i) {
-    const uint64_t ck = mix_s(key + 0x9E3779B97F4A7C15ULL * ((uint64_t)(uint32_t)v[i] + 1));
-    if ((mix_s(ck + 0xD1B54A32D192ED03ULL) >> 11) > T) out.push_back(i);
+// ---- skip sampling of a node's children in BINV's domain -------------------------------------
+// Every child of a node with multiplicity B draws B' ~ Bin(B, p), p = 1/D, independently (R20); in BINV's domain
+// B' > 0 has probability q = 1 - r0, r0 = (1-p)^B, which is small at levels >= 2 (C4: ~2.5 %). Instead of one
+// coin per driver element, the driver is cut into segments of kSkipSeg elements and each segment's selected
+// elements are found by geometric gaps G with P(G >= g) = r0^g (iid Bernoulli(q) per element), drawn from the
+// segment's own counter stream; a selected element that is a child then draws B' from Bin(B, p) conditioned on
+// B' >= 1 (its own stream, keyed by the child as before). The law of the children's draws is exactly the
+// independent binomials' — only the random numbers differ. The device walker computes the same doubles in the
+// same order (round-to-nearest, no contraction), so both draw the same children.
+int64_t binom_pos(uint64_t ck, int64_t n, double p, double r0) {
+  Uniforms U{ck};
+  const double q = 1.0 - p, s = p / q, a = (double)(n + 1) * s;
+  for (;;) {
+    double u = r0 + (1.0 - r0) * U.next();  // uniform on (r0, 1]: the inversion never stops at 0
+    double r = r0;
+    int64_t x = 0;
+    while (u > r) {
+      u -= r;
+      x += 1;
+      if (x > n) break;
+      r *= (a / (double)x - s);
+    }
+    if (x > n) continue;
+    return x < 1 ? 1 : x;
   }
 }
 
-__attribute__((target("avx512f,avx512dq"))) static inline __m512i mix_v(__m512i z, __m512i C1, __m512i C2) {
-  z = _mm512_mullo_epi64(_mm512_xor_si512(z, _mm512_srli_epi64(z, 30)), C1);
-  z = _mm512_mullo_epi64(_mm512_xor_si512(z, _mm512_srli_epi64(z, 27)), C2);
-  return _mm512_xor_si512(z, _mm512_srli_epi64(z, 31));
+void skip_table(double r0, double *pw) {
+  pw[0] = r0;
+  for (int i = 1; i < kSkipLog + 1; ++i) pw[i] = pw[i - 1] * pw[i - 1];
 }
 
-__attribute__((target("avx512f,avx512dq"))) static void coin_filter_avx512(const int32_t *v, uint32_t n, uint64_t key,
-                                                                           uint64_t T, std::vector<uint32_t> &out) {
-  const __m512i G = _mm512_set1_epi64((long long)0x9E3779B97F4A7C15ULL);
-  const __m512i K = _mm512_set1_epi64((long long)key);
-  const __m512i C1 = _mm512_set1_epi64((long long)0xBF58476D1CE4E5B9ULL);
-  const __m512i C2 = _mm512_set1_epi64((long long)0x94D049BB133111EBULL);
-  const __m512i D1 = _mm512_set1_epi64((long long)0xD1B54A32D192ED03ULL);
-  const __m512i one = _mm512_set1_epi64(1);
-  const __m512i TT = _mm512_set1_epi64((long long)T);
-  uint32_t i = 0;
-  for (; i + 8 <= n; i += 8) {
-    const __m512i x = _mm512_add_epi64(_mm512_cvtepu32_epi64(_mm256_loadu_si256((const __m256i *)(v + i))), one);
-    const __m512i ck = mix_v(_mm512_add_epi64(K, _mm512_mullo_epi64(G, x)), C1, C2);
-    const __m512i m = _mm512_srli_epi64(mix_v(_mm512_add_epi64(ck, D1), C1, C2), 11);
-    __mmask8 k = _mm512_cmpgt_epu64_mask(m, TT);
-    while (k) {
-      out.push_back(i + (uint32_t)__builtin_ctz(k));
-      k &= (__mmask8)(k - 1);
+uint32_t skip_gap(const double *pw, double u) {  // the largest g < 2 kSkipSeg with r0^g >= u
+  double cur = 1.0;
+  uint32_t g = 0;
+  for (int i = kSkipLog; i >= 0; --i) {
+    const double c = cur * pw[i];
+    if (c >= u) {
+      cur = c;
+      g += 1u << i;
     }
   }
-  for (; i < n; ++i) {
-    const uint64_t ck = mix_s(key + 0x9E3779B97F4A7C15ULL * ((uint64_t)(uint32_t)v[i] + 1));
-    if ((mix_s(ck + 0xD1B54A32D192ED03ULL) >> 11) > T) out.push_back(i);
-  }
+  return g;
 }
 
-static void coin_filter(const int32_t *v, uint32_t n, uint64_t key, uint64_t T, std::vector<uint32_t> &out) {
-  static const bool avx512 = __builtin_cpu_supports("avx512f") && __builtin_cpu_supports("avx512dq");
-  if (avx512) coin_filter_avx512(v, n, key, T, out);
-  else coin_filter_scalar(v, n, key, T, out);
-}
-
-double stirling_small(int k) { return stirling_fc(k); }
+uint64_t skip_uniform_bits(uint64_t segkey, uint64_t j) { return rng_mix(segkey + 0xD1B54A32D192ED03ULL * j) >> 11; }
 
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k) {
   // M = floor(N1 * D^(k-2) / 32^k), clamped to [1, 2^62] (R21), exact integer arithmetic.
@@ -269,7 +254,6 @@ struct Walker {
         if (f[s] == v) return;
       if (Lp.label >= 0 && (in.labels ? (int32_t)in.labels[v] : 0) != Lp.label) return;
       const uint64_t ck = rng_chain(key, (uint64_t)(uint32_t)v);
-      if (fast && first_uniform_le(ck, r0)) return;  // B' = 0: skip the probes
       for (int b = 0; b < Lp.nb; ++b)
         if (b != drv && !member(L[b], v)) return;
       const int64_t Bc = binomial(ck, B, pD);
@@ -277,15 +261,33 @@ struct Walker {
       f[p] = v;
       visit(level + 1, Bc, ck);
     };
-    if (fast) {  // vectorised B' = 0 pre-filter (same decision as first_uniform_le)
-      const uint64_t T = (uint64_t)std::floor(r0 * 9007199254740992.0);
-      std::vector<uint32_t> &keep = keep_[level];  // reused per depth (no per-node allocation)
-      keep.clear();
-      coin_filter(L[drv].a, L[drv].na, key, T, keep);
-      for (uint32_t i : keep) consider(L[drv].a[i]);
-      keep.clear();
-      if (L[drv].nb) coin_filter(L[drv].b, L[drv].nb, key, T, keep);
-      for (uint32_t i : keep) consider(L[drv].b[i]);
+    if (fast) {  // skip sampling over segments of the driver (main then delta segment)
+      auto consider_sel = [&](int32_t v) {
+        for (int s = 0; s < p; ++s)
+          if (f[s] == v) return;
+        if (Lp.label >= 0 && (in.labels ? (int32_t)in.labels[v] : 0) != Lp.label) return;
+        for (int b = 0; b < Lp.nb; ++b)
+          if (b != drv && !member(L[b], v)) return;
+        const uint64_t ck = rng_chain(key, (uint64_t)(uint32_t)v);
+        const int64_t Bc = binom_pos(ck, B, pD, r0);
+        f[p] = v;
+        visit(level + 1, Bc, ck);
+      };
+      double pw[kSkipLog + 1];
+      skip_table(r0, pw);
+      const uint32_t na = L[drv].na, nd = na + L[drv].nb;
+      for (uint32_t s0 = 0; s0 < nd; s0 += kSkipSeg) {
+        const uint32_t s1 = std::min<uint32_t>(nd, s0 + kSkipSeg);
+        const uint64_t segkey = rng_chain(key, kSkipTag + s0 / kSkipSeg);
+        uint32_t pos = s0;
+        for (uint64_t j = 1;; ++j) {
+          const uint32_t g = skip_gap(pw, (double)skip_uniform_bits(segkey, j) * (1.0 / 9007199254740992.0));
+          if (g >= s1 - pos) break;
+          pos += g;
+          consider_sel(pos < na ? L[drv].a[pos] : L[drv].b[pos - na]);
+          if (++pos >= s1) break;
+        }
+      }
     } else {
       for (uint32_t i = 0; i < L[drv].na; ++i) consider(L[drv].a[i]);
       for (uint32_t i = 0; i < L[drv].nb; ++i) consider(L[drv].b[i]);

@@ -47,6 +47,15 @@ struct EstimatorOutput {
   std::vector<uint64_t> levcnt;  // 8 per id: Σ B at levels 1..k-2
 };
 
+// skip sampling of children in BINV's domain (estimator.cpp; the device walker mirrors it bit for bit)
+constexpr uint32_t kSkipSeg = 1024;   // driver elements per segment (= kEstItem, the level-1 work item)
+constexpr int kSkipLog = 10;          // r0^(2^i), i = 0..10: gaps up to 2 kSkipSeg - 1
+constexpr uint64_t kSkipTag = 0x53B1000000000000ULL;  // segment s's stream: rng_chain(node key, kSkipTag + s)
+int64_t binom_pos(uint64_t ck, int64_t n, double p, double r0);  // Bin(n, p) | >= 1, n p < 10, r0 = (1-p)^n
+void skip_table(double r0, double *pw);
+uint32_t skip_gap(const double *pw, double u);
+uint64_t skip_uniform_bits(uint64_t segkey, uint64_t j);
+
 uint64_t walk_budget(uint64_t N1, uint64_t D, int k);
 double stirling_small(int k);  // BTRD's Stirling correction for k < 10 (lgamma; the GPU sampler's table)
 void run_estimator(const EstimatorInput &in, EstimatorScratch &scr, EstimatorOutput &out);

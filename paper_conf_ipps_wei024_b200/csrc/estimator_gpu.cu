@@ -22,6 +22,7 @@
 // table (glibc pow), BTRD's Stirling terms for k < 10 from a host table (glibc lgamma); BTRD's log is CUDA's
 // (max 1 ulp; it decides only comparisons that are not within an ulp of a tie — DESIGN.md).
 
+#include "estimator.h"
 #include "estimator_gpu.cuh"
 
 namespace gcsm {
@@ -163,6 +164,58 @@ __device__ __forceinline__ int64_t d_binomial(unsigned long long key, int64_t n,
 
 __device__ __noinline__ int64_t d_binomial_ool(unsigned long long key, int64_t n, BinTab T) { return d_binomial(key, n, T); }
 
+// ---- skip sampling (estimator.cpp skip_table / skip_gap / binom_pos, operation for operation) ------------------
+static_assert(kSkipSeg == (uint32_t)kEstItem, "a level-1 work item is one skip segment");
+__device__ __forceinline__ void d_skip_table(double r0, double *pw) {
+  pw[0] = r0;
+#pragma unroll
+  for (int i = 1; i < kSkipLog + 1; ++i) pw[i] = DM(pw[i - 1], pw[i - 1]);
+}
+__device__ __forceinline__ uint32_t d_skip_gap(const double *pw, double u) {
+  double cur = 1.0;
+  uint32_t g = 0;
+#pragma unroll
+  for (int i = kSkipLog; i >= 0; --i) {
+    const double c = DM(cur, pw[i]);
+    if (c >= u) {
+      cur = c;
+      g += 1u << i;
+    }
+  }
+  return g;
+}
+__device__ __noinline__ int64_t d_binom_pos(unsigned long long ck, int64_t n, double p, double r0) {
+  DUni U{ck, 0};
+  const double q = DS(1.0, p);
+  const double s = DV(p, q), a = DM((double)(n + 1), s);
+  for (;;) {
+    double u = DA(r0, DM(DS(1.0, r0), U.next()));
+    double r = r0;
+    int64_t x = 0;
+    while (u > r) {
+      u = DS(u, r);
+      x += 1;
+      if (x > n) break;
+      r = DM(r, DS(DV(a, (double)x), s));
+    }
+    if (x > n) continue;
+    return x < 1 ? 1 : x;
+  }
+}
+__device__ __forceinline__ double d_skip_uniform(unsigned long long segkey, unsigned long long j) {
+  return DM((double)(dmix(segkey + 0xD1B54A32D192ED03ULL * j) >> 11), 1.0 / 9007199254740992.0);
+}
+// inclusive warp scan of (g + 1): the driver offset (from the step's start) just past each lane's selection
+__device__ __forceinline__ uint32_t skip_scan(uint32_t g, int lane) {
+  uint32_t x = g + 1;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  return x;
+}
+
 struct LR {
   const int32_t *m;
   uint32_t ml;
@@ -232,7 +285,10 @@ constexpr int kEW = 8;  // warps per block
 struct EstLv {
   int32_t pos, ns, si, drv;
   unsigned long long B, key;
-  unsigned long long T53;  // BINV's first-uniform threshold floor(r0 2^53) of this node (all ones: no shortcut)
+  unsigned long long T53;  // 1: the node samples its children by skip sampling (BINV's domain), ~0: one draw each
+  unsigned long long uj;   // skip sampling: uniforms consumed in the current segment
+  double r0;               // (1 - 1/D)^B (host table)
+  double pw[kSkipLog + 1]; // r0^(2^i)
   const int32_t *dm, *dx;  // the node's driver list (main, delta segment), fixed at node entry
   uint32_t dml, dxl;
   const int32_t *pm[7];    // every backward main list as read (staged copy when zero-copy and staging is on)
@@ -281,6 +337,66 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
     }
     const uint32_t end = min(best, (uint32_t)item.y + (uint32_t)kEstItem);
     const LevelPlan &L3 = P->lv[3];
+    // emit one step's children: (k = 4) the reads of the level-2 nodes, (k >= 5) level-2 walk nodes
+    auto emit = [&](bool ok, int32_t v, unsigned long long Bc, unsigned long long ck) {
+      if (k == 4) {
+        if (ok) {
+          const int32_t f3[3] = {U.a, U.b, v};
+          for (int b = 0; b < L3.nb; ++b) {
+            const int32_t w = f3[L3.bpos[b]];
+            atomicAdd(A.levcnt + (size_t)w * A.levels + 1, Bc);
+            atomicOr(A.touched + (w >> 5), 1u << (w & 31));
+          }
+        }
+      } else {
+        const unsigned mask = __ballot_sync(FULL, ok);
+        unsigned long long base = 0;
+        if (lane == 0 && mask) base = atomicAdd(A.f2_count, (unsigned long long)__popc(mask));
+        base = __shfl_sync(FULL, base, 0);
+        if (ok) {
+          const unsigned long long slot = base + __popc(mask & ((1u << lane) - 1u));
+          if (slot < (unsigned long long)A.f2_cap) A.f2[slot] = EstNode2{U.a, U.b, v, U.plan, Bc, ck};
+          else atomicExch(A.T.err, 3);
+        }
+      }
+    };
+    if ((int64_t)U.B < T.r0n && DM((double)U.B, T.pD) < 10.0) {  // BINV's domain: skip sampling of the item
+      const double r0 = T.r0tab[U.B];
+      double pw[kSkipLog + 1];
+      d_skip_table(r0, pw);
+      const unsigned long long segkey = dchain(U.key, kSkipTag + (unsigned long long)item.y / kSkipSeg);
+      uint32_t pos = (uint32_t)item.y;
+      unsigned long long uj = 0;
+      while (pos < end) {
+        const uint32_t g = d_skip_gap(pw, d_skip_uniform(segkey, uj + lane + 1));
+        const uint32_t sel = pos + skip_scan(g, lane) - 1;
+        const bool valid = sel < end;  // a prefix of the lanes
+        const int nv = __popc(__ballot_sync(FULL, valid));
+        bool ok = valid;
+        int32_t v = 0;
+        unsigned long long Bc = 0, ck = 0;
+        if (ok) {
+          v = sel < L[drv].ml ? L[drv].m[sel] : L[drv].x[sel - L[drv].ml];
+          ok = v != U.a && v != U.b;
+          if (ok && Lp.label >= 0) ok = (A.lab ? (int32_t)A.lab[v] : 0) == Lp.label;
+          if (ok)
+            for (int b = 0; b < nb; ++b)
+              if (b != drv && !(has(L[b].m, L[b].ml, v) || (L[b].xl && has(L[b].x, L[b].xl, v)))) {
+                ok = false;
+                break;
+              }
+          if (ok) {
+            ck = dchain(U.key, (unsigned long long)(uint32_t)v);
+            Bc = (unsigned long long)d_binom_pos(ck, (int64_t)U.B, T.pD, r0);
+          }
+        }
+        emit(ok, v, Bc, ck);
+        if (nv < 32) break;
+        pos = __shfl_sync(FULL, sel, 31) + 1;
+        uj += 32;
+      }
+      continue;
+    }
     for (uint32_t pos = (uint32_t)item.y; pos < end; pos += 32) {
       const uint32_t idx = pos + lane;
       bool ok = false;
@@ -303,26 +419,7 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
               break;
             }
       }
-      if (k == 4) {  // the child is a level-2 node of the last sampled level: its reads, then nothing below
-        if (ok) {
-          const int32_t f3[3] = {U.a, U.b, v};
-          for (int b = 0; b < L3.nb; ++b) {
-            const int32_t w = f3[L3.bpos[b]];
-            atomicAdd(A.levcnt + (size_t)w * A.levels + 1, Bc);
-            atomicOr(A.touched + (w >> 5), 1u << (w & 31));
-          }
-        }
-      } else {
-        const unsigned mask = __ballot_sync(FULL, ok);
-        unsigned long long base = 0;
-        if (lane == 0 && mask) base = atomicAdd(A.f2_count, (unsigned long long)__popc(mask));
-        base = __shfl_sync(FULL, base, 0);
-        if (ok) {
-          const unsigned long long slot = base + __popc(mask & ((1u << lane) - 1u));
-          if (slot < (unsigned long long)A.f2_cap) A.f2[slot] = EstNode2{U.a, U.b, v, U.plan, Bc, ck};
-          else atomicExch(A.T.err, 3);
-        }
-      }
+      emit(ok, v, Bc, ck);  // the child is a level-2 node (k = 4: of the last sampled level)
     }
   }
 }
@@ -394,15 +491,20 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
             drv = b;
           }
         }
-        // zero-copy lists: the driver (scanned whole) is fetched once per batch into HBM; a probed list (only
-        // for the rare children with B' > 0) uses the staged copy when one exists, else a few in-place reads
+        const int64_t Bn0 = (int64_t)S.B;
+        const bool fast0 = Bn0 > 0 && T.pD > 0.0 && T.pD <= 0.5 && DM((double)Bn0, T.pD) < 10.0 && Bn0 < T.r0n;
+        // zero-copy lists: a driver scanned whole (one draw per child) is fetched once per batch into HBM; under
+        // skip sampling only the selected elements are read (a fraction 1 - r0 of the driver: C4 level 2 ~2.5 %,
+        // level 3 ~0.02 %), in place unless that fraction is large; a probed list (only for the children drawn)
+        // uses the staged copy when one exists, else a few in-place reads
+        const bool stage_drv = !fast0 || DS(1.0, T.r0tab[Bn0]) > 0.125;
         for (int b = 0; b < nb; ++b) {
           const char *pc = reinterpret_cast<const char *>(L[b].m);
           if (!A.stage.state || L[b].ml < A.stage_min || (pc >= A.dev_lo[0] && pc < A.dev_hi[0]) ||
               (pc >= A.dev_lo[1] && pc < A.dev_hi[1]))
             continue;
           const int32_t vb = W.f[Lp.bpos[b]];
-          if (b == drv) {
+          if (b == drv && stage_drv) {
             L[b].m = stage_fetch(A.stage, vb, L[b].m, L[b].ml, wfill, wlists, whit, lane);
           } else {
             const unsigned long long st = stage_word(A.stage.state + vb);
@@ -414,12 +516,10 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
         }
         if (lane == 0)
           for (int b = 0; b < nb; ++b) S.pm[b] = L[b].m;
-        walg += 4ull * (L[drv].ml + L[drv].xl);  // the driver is scanned whole
+        walg += stage_drv ? 4ull * (L[drv].ml + L[drv].xl) : 0ull;  // a driver scanned whole (else: per selection)
         const int64_t Bn = (int64_t)S.B;
         const double pD = T.pD;
-        unsigned long long t53 = ~0ull;
-        if (Bn > 0 && pD > 0.0 && pD <= 0.5 && DM((double)Bn, pD) < 10.0 && Bn < T.r0n)
-          t53 = (unsigned long long)floor(DM(T.r0tab[Bn], 9007199254740992.0));
+        const bool fast = Bn > 0 && pD > 0.0 && pD <= 0.5 && DM((double)Bn, pD) < 10.0 && Bn < T.r0n;
         if (lane == 0) {
           S.pos = 0;
           S.ns = 0;
@@ -429,7 +529,12 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
           S.dml = L[drv].ml;
           S.dx = L[drv].x;
           S.dxl = L[drv].xl;
-          S.T53 = t53;
+          S.T53 = fast ? 1ull : ~0ull;
+          S.uj = 0;
+          if (fast) {
+            S.r0 = T.r0tab[Bn];
+            d_skip_table(S.r0, S.pw);
+          }
         }
         __syncwarp();
         continue;
@@ -461,6 +566,59 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
       const int32_t *dm = S.dm, *dx = S.dx;
       const unsigned long long key = S.key, t53 = S.T53;
       const int64_t Bn = (int64_t)S.B;
+      if (t53 != ~0ull) {  // skip sampling: one step of up to 32 selections in the current segment
+        const uint32_t s1 = min(best, (pos / kSkipSeg + 1) * kSkipSeg);
+        const unsigned long long segkey = dchain(key, kSkipTag + pos / kSkipSeg);
+        const uint32_t g = d_skip_gap(S.pw, d_skip_uniform(segkey, S.uj + lane + 1));
+        const uint32_t sel = pos + skip_scan(g, lane) - 1;
+        const bool valid = sel < s1;  // a prefix of the lanes
+        const int nv = __popc(__ballot_sync(FULL, valid));
+        const uint32_t last = __shfl_sync(FULL, sel, 31);
+        bool ok = valid;
+        int32_t v = 0;
+        walg += 4ull * (uint32_t)nv;  // the selected driver elements
+        if (ok) {
+          v = sel < dml ? dm[sel] : dx[sel - dml];
+          for (int s2 = 0; s2 < p; ++s2) ok = ok && W.f[s2] != v;
+          if (ok && Lp.label >= 0) ok = (A.lab ? (int32_t)A.lab[v] : 0) == Lp.label;
+        }
+        if (__any_sync(FULL, ok)) {  // membership in the other backward lists
+          const int drv = S.drv;
+          for (int b = 0; b < nb; ++b) {
+            if (b == drv) continue;
+            const LR Lb = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
+            const int32_t *bm = S.pm[b];
+            walg += 4ull * (Lb.ml + Lb.xl);
+            if (ok) ok = has(bm, Lb.ml, v) || (Lb.xl && has(Lb.x, Lb.xl, v));
+          }
+        }
+        unsigned long long Bc = 0, ck = 0;
+        if (ok) {
+          ck = dchain(key, (unsigned long long)(uint32_t)v);
+          Bc = (unsigned long long)d_binom_pos(ck, Bn, T.pD, S.r0);
+        }
+        const unsigned msk = __ballot_sync(FULL, ok);
+        __syncwarp();
+        if (ok) {
+          const int r = __popc(msk & ((1u << lane) - 1u));
+          S.sv[r] = v;
+          S.sB[r] = Bc;
+          S.skey[r] = ck;
+        }
+        if (lane == 0) {
+          S.ns = __popc(msk);
+          S.si = 0;
+          if (nv == 32 && last + 1 < s1) {
+            S.pos = (int32_t)(last + 1);
+            S.uj += 32;
+          } else {  // the segment is done: the next one starts with a fresh stream
+            S.pos = (int32_t)s1;
+            S.uj = 0;
+          }
+        }
+        __syncwarp();
+        continue;
+      }
       int32_t v[4];
       bool ok[4];
       unsigned long long Bc[4], ck[4];
@@ -476,11 +634,7 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
         if (ok[j] && Lp.label >= 0) ok[j] = (A.lab ? (int32_t)A.lab[v[j]] : 0) == Lp.label;
         Bc[j] = 0;
         ck[j] = 0;
-        if (ok[j]) {
-          ck[j] = dchain(key, (unsigned long long)(uint32_t)v[j]);
-          // in BINV's range a first uniform <= r0 means B' = 0 (binv's loop never runs)
-          ok[j] = t53 == ~0ull || (dmix(ck[j] + 0xD1B54A32D192ED03ULL) >> 11) > t53;
-        }
+        if (ok[j]) ck[j] = dchain(key, (unsigned long long)(uint32_t)v[j]);
       }
 #pragma unroll 1
       for (int j = 0; j < 4; ++j)
