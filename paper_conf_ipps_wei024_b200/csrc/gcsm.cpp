@@ -228,6 +228,7 @@ struct gcsm_ctx {
   uint32_t stage_min = 1;          // shortest list (ints) routed through the arena (GCSM_STAGE_MIN)
   uint32_t walk_stage_epoch = 0;   // this batch's walks stage through the arena too (0 = no)
   int32_t stage_policy = 1;        // smem staging model for device-resident probe lists (GCSM_STAGE_POLICY)
+  int32_t walk_stage = 1;          // staging of skip-sampled walk drivers (GCSM_WALK_STAGE: 0 always, 1 expected >= 1, 2 never)
   // B_comp measurement mode (GCSM_BCOMP=1 at create): bitmap of the vertices whose main list a query's kernels read
   uint32_t *d_touched_bc = nullptr;
   bool bcomp = false;
@@ -434,6 +435,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   if (const char *sm = std::getenv("GCSM_STAGE_MB")) ctx->opt.staging_bytes = std::strtoull(sm, nullptr, 10) << 20;
   if (const char *sm = std::getenv("GCSM_STAGE_MIN")) ctx->stage_min = (uint32_t)std::max(1, std::atoi(sm));
   if (const char *sp = std::getenv("GCSM_STAGE_POLICY")) ctx->stage_policy = std::atoi(sp);
+  if (const char *ws = std::getenv("GCSM_WALK_STAGE")) ctx->walk_stage = std::atoi(ws);
   if (std::getenv("GCSM_BCOMP") && gcsm_set_measure(ctx, GCSM_MEASURE_BCOMP) != GCSM_OK) return bail(GCSM_ENOMEM);
   ctx->grid = match_grid(dev, &ctx->warps_total);
   ctx->ext_grid = ctx->grid;
@@ -910,6 +912,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
     c.stage = StageRef{ctx->d_stage_state, ctx->d_stage_arena, ctx->stage_cap, ctx->d_stage_bump,
                        ctx->walk_stage_epoch};
     c.stage_min = ctx->stage_min;
+    c.walk_stage = ctx->walk_stage;
     c.stage_cnt = sl.d_cnt + CNT_WFILL;  // query 0's block
     c.dev_lo[0] = ctx->cache_valid ? ctx->d_cachebuf[ctx->cache_cur] : nullptr;  // lists cached by the last batch
     c.dev_hi[0] = c.dev_lo[0] ? c.dev_lo[0] + ctx->cache_cap : nullptr;

@@ -667,6 +667,19 @@ __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const
   return w;
 }
 
+// Warp-uniform DFS state of k_extend in shared memory (every lane writes the same values): the partial match, the
+// candidate sets and iterators per level and the list descriptors of the current intersection. Indexed at run time
+// (the query size and plans are runtime data), these arrays lived in local memory and their spills dominated the
+// kernel's DRAM traffic (profiles/ncu_c4_r02_v2.md: 48 GB per prism6 launch for ~1 GB of lists).
+struct WarpDfs {
+  int32_t f[GCSM_MAXK];
+  const int32_t *set[GCSM_MAXK];
+  uint32_t sz[GCSM_MAXK], it[GCSM_MAXK];
+  LRef L[7], Lx[7];
+  int32_t excl[GCSM_MAXK];
+};
+constexpr int kExtSmemBytes = kSmemBytes + kWarps * (int)sizeof(WarpDfs);
+
 // Levels 3..k-1 (DFS): warp per level-2 frontier entry.
 template <bool LIST, int KK>  // KK: compile-time query size (4: the level-3 count only), 0 = any
 __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchArgs A) {
@@ -679,6 +692,11 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   uint32_t *bm = reinterpret_cast<uint32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
   int32_t *sm = reinterpret_cast<int32_t *>(bm) + GCSM_BM_INTS;  // pin area, then transient staging
   constexpr uint32_t kSlice = kSmemInts - GCSM_BM_INTS;
+  WarpDfs &Wd = *reinterpret_cast<WarpDfs *>(reinterpret_cast<char *>(smem_raw) + kSmemBytes +
+                                             (threadIdx.x >> 5) * sizeof(WarpDfs));
+  int32_t *const f = Wd.f;
+  const int32_t **const set = Wd.set;
+  uint32_t *const sz = Wd.sz, *const it = Wd.it;
   const int k = KK ? KK : A.k;
   int32_t *lastbuf = stack + (int64_t)(k > 4 ? k - 4 : 0) * A.dcap;  // LIST: last-level candidates
   int32_t *hbuf = stack + (int64_t)((k > 4 ? k - 4 : 0) + (LIST ? 1 : 0)) * A.dcap;  // hoisted last-level set
@@ -830,12 +848,10 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     const DevPlan &P = A.plans[U.plan];
     const int2 seg = A.useg[ui];
     if (!task) ++x_entries;
-    int32_t f[GCSM_MAXK];
+    __syncwarp();  // every lane is done with the previous entry's state
     f[0] = U.a;
     f[1] = U.b;
     f[2] = f2c[e];
-    const int32_t *set[GCSM_MAXK];
-    uint32_t sz[GCSM_MAXK], it[GCSM_MAXK];
     set[2] = f2c + seg.x;
     sz[2] = (uint32_t)seg.y;
     uint32_t end3 = 0xffffffffu;  // level-3 iteration bound (a task's slice)
@@ -846,7 +862,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     uint32_t hn = 0;
     if (KK == 0 && P.lv[k - 1].hmask && A.hoist) {
       const LevelPlan &Lh = P.lv[k - 1];
-      LRef Lx[7];
+      LRef *const Lx = Wd.Lx;
       int nx = 0, hdrv = 0;
       uint32_t best = 0xffffffffu;
       for (int b = 0; b < Lh.nb; ++b)
@@ -873,7 +889,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     const bool filt = KK == 0 && k >= 5 && P.lv[4].fmask != 0 && A.filter3;
     if (filt) {
       const LevelPlan &L4 = P.lv[4];
-      LRef Lx[7];
+      LRef *const Lx = Wd.Lx;
       int nx = 0, fdrv = 0;
       uint32_t best = 0xffffffffu;
       for (int b = 0; b < L4.nb; ++b)
@@ -933,10 +949,10 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
       if (descend) {
         const int p = lvl + 1;  // compute candidates of position p
         const LevelPlan &Lp = P.lv[p];
-        LRef L[7];
+        LRef *const L = Wd.L;
         int drv = 0;
         int nl = (p == k - 1 && hset) ? 0 : gather_lists(A, Lp, f, L, &drv, acc, lane, pin);
-        int32_t excl[GCSM_MAXK];
+        int32_t *const excl = Wd.excl;
         int nex = 0;
         for (int i = 0; i < Lp.ninj; ++i) excl[nex++] = f[Lp.inj[i]];
         const int32_t *dset = Lp.reuse >= 0 ? set[Lp.reuse] : nullptr;
@@ -1064,7 +1080,10 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
       // choose the next element at the deepest open position (>= 3)
       while (lvl >= 3 && it[lvl] >= (lvl == 3 ? min(end3, it3n) : sz[lvl])) --lvl;
       if (lvl < 3) break;
-      f[lvl] = (lvl == 3 ? it3p : set[lvl])[it[lvl]++];
+      const uint32_t ii = it[lvl];
+      __syncwarp();  // every lane has read the iterator before any lane advances it
+      it[lvl] = ii + 1;
+      f[lvl] = (lvl == 3 ? it3p : set[lvl])[ii];
       descend = true;
     }
     (void)lvl;
@@ -1693,13 +1712,13 @@ cudaError_t upload_plans(DevPlan *dst, const DevPlan *plans, int n, cudaStream_t
 int match_grid(int device, int *warps_total) {
   int sms = 0, occ = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  cudaFuncSetAttribute(k_extend<false, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-  cudaFuncSetAttribute(k_extend<false, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-  cudaFuncSetAttribute(k_extend<true, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  cudaFuncSetAttribute(k_extend<false, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kExtSmemBytes);
+  cudaFuncSetAttribute(k_extend<false, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, kExtSmemBytes);
+  cudaFuncSetAttribute(k_extend<true, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kExtSmemBytes);
   cudaFuncSetAttribute(k_level2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   cudaFuncSetAttribute(k_level2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   cudaFuncSetAttribute(k_last4, cudaFuncAttributeMaxDynamicSharedMemorySize, kL4SmemBytes);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false, 0>, kBlock, kSmemBytes);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<false, 0>, kBlock, kExtSmemBytes);
   int occ2 = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_level2<false>, kBlock, kSmemBytes);
   if (occ2 < occ) occ = occ2;
@@ -1729,10 +1748,10 @@ cudaError_t launch_extend(const MatchArgs &a0, int grid, cudaStream_t s) {
   MatchArgs a = a0;
   a.acc_base = CNT_ACC_EXT;
   if (a.tasks) k_reset_sharing<<<1, 1, 0, s>>>(a.cnt);
-  if (a.listing) k_extend<true, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
+  if (a.listing) k_extend<true, 0><<<grid, kBlock, kExtSmemBytes, s>>>(a);
   else if (a.k == 4 && GCSM_LAST4) k_last4<<<grid, kBlock, kL4SmemBytes, s>>>(a);
-  else if (a.k == 4) k_extend<false, 4><<<grid, kBlock, kSmemBytes, s>>>(a);
-  else k_extend<false, 0><<<grid, kBlock, kSmemBytes, s>>>(a);
+  else if (a.k == 4) k_extend<false, 4><<<grid, kBlock, kExtSmemBytes, s>>>(a);
+  else k_extend<false, 0><<<grid, kBlock, kExtSmemBytes, s>>>(a);
   return cudaGetLastError();
 }
 

@@ -23,7 +23,8 @@ for item in spec.split(","):
         rest, f = rest.split("@")
         frac = float(f)
     env = dict(kv.split(":") for kv in rest.split("+") if kv)
-    saved = {k: os.environ.get(k) for k in ("GCSM_STAGE_MIN", "GCSM_STAGE_MB")}
+    saved = {k: os.environ.get(k) for k in ("GCSM_STAGE_MIN", "GCSM_STAGE_MB", "GCSM_WALK_STAGE", "GCSM_STAGE_POLICY",
+                                            "GCSM_NO_FILTER3", "GCSM_NO_HOIST")}
     for k in saved:
         os.environ.pop(k, None)
     staging = 1 if env.get("GCSM_STAGE_MB") == "0" else 0
@@ -46,6 +47,7 @@ for item in spec.split(","):
         for qi, q in enumerate(queries):
             st = g.query_stats(qi)
             rec = {"var": name, "q": q, "batch": b, "bcomp_mode": meas, "wall_ms": round(wall * 1e3, 1),
+                   "ms_walks": round(st["ms_walks"], 2), "walk_fill_gb": st["walk_fill_bytes"] / 1e9,
                    "create_s": round(create_s, 1), "added": st["added"], "removed": st["removed"],
                    "ms_match": round(st["ms_match"], 2), "ms_extend": round(st["ms_extend"], 2),
                    "ms_copy": round(st["ms_copy"], 2), "frontier": st["frontier"],
