@@ -91,9 +91,9 @@ typedef struct {
   int64_t vertex_capacity; /* ids the graph may grow into: 0 = n (no growth). Insertions may name ids in
                               [n, vertex_capacity): new vertices, each given an empty list with the average
                               degree as capacity; gcsm_add_vertices adds labelled ones */
-  uint64_t staging_bytes;  /* per-GPU HBM arena of the fetch-once staging of zero-copy lists within a batch
-                              (not a cache: emptied every batch): 0 = default (a quarter of the
-                              free HBM when first needed, at most 16 GiB), 1 = off */
+  uint64_t staging_bytes;  /* per-GPU HBM for the fetch-once staging of zero-copy lists within a batch (DESIGN.md
+                              §1d; two arenas, one per in-flight batch; not a cache: emptied every batch):
+                              0 = default (a quarter of the free HBM when first needed, at most 32 GiB), 1 = off */
 } gcsm_options;
 
 /* Per-batch statistics (Table II-style breakdown; hit rate §8d). */

@@ -220,10 +220,14 @@ struct gcsm_ctx {
   bool est_valid = false;          // the device holds a batch's estimator output (gcsm_get_estimates)
   // fetch-once staging of zero-copy lists within a batch (kernels.cu stage_resolve): per-vertex
   // state words, the arena (emptied every batch: a new epoch) and its bump counter
-  unsigned long long *d_stage_state = nullptr;
-  int32_t *d_stage_arena = nullptr;
-  size_t stage_cap = 0;            // ints
-  unsigned long long *d_stage_bump = nullptr;
+  // one arena per in-flight slot: batch t+1's walks (cache step, possibly on its own stream) stage into their slot
+  // while batch t's matching reads the other
+  struct StageSlot {
+    unsigned long long *state = nullptr;
+    int32_t *arena = nullptr;
+    size_t cap = 0;  // ints
+    unsigned long long *bump = nullptr;
+  } stg[2];
   bool stage_failed = false;       // allocation failed once: stay off
   uint32_t stage_min = 1;          // shortest list (ints) routed through the arena (GCSM_STAGE_MIN)
   uint32_t walk_stage_epoch = 0;   // this batch's walks stage through the arena too (0 = no)
@@ -282,7 +286,8 @@ gcsm_ctx::~gcsm_ctx() {
     if (p) cudaFree(p);
   void *dev2[] = {d_hptr, d_touched, d_wcnt, d_woff, d_tids, d_prev_sel, d_bits, d_bytes, d_scan, d_off, d_flag,
                   d_selhist, d_ecursor, d_sel, d_cubtmp, d_eunits, d_r0, d_eitems, d_ef2, d_sfc, d_sidx, d_soff,
-                  d_srec, d_sstage, d_stage_state, d_stage_arena, d_stage_bump, d_touched_bc};
+                  d_srec, d_sstage, d_touched_bc, stg[0].state, stg[0].arena, stg[0].bump, stg[1].state,
+                  stg[1].arena, stg[1].bump};
   for (void *p : dev2)
     if (p) cudaFree(p);
   for (unsigned long long *p : d_levcnt)
@@ -909,8 +914,8 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   for (int qi = 0; qi < nq && qi < GCSM_MAX_QUERIES; ++qi) c.alg_cnt[qi] = sl.d_cnt + (size_t)qi * CNT_N + CNT_WALG;
   sl.walks_timed = est_on;
   if (ctx->walk_stage_epoch && !std::getenv("GCSM_NO_WALK_STAGE")) {  // the walks' zero-copy lists through the arena
-    c.stage = StageRef{ctx->d_stage_state, ctx->d_stage_arena, ctx->stage_cap, ctx->d_stage_bump,
-                       ctx->walk_stage_epoch};
+    const gcsm_ctx::StageSlot &sg = ctx->stg[ctx->batch_seq & 1];
+    c.stage = StageRef{sg.state, sg.arena, sg.cap, sg.bump, ctx->walk_stage_epoch};
     c.stage_min = ctx->stage_min;
     c.walk_stage = ctx->walk_stage;
     c.stage_cnt = sl.d_cnt + CNT_WFILL;  // query 0's block
@@ -1443,40 +1448,44 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     for (gcsm_ctx *p : ctx->peers->members)
       if (p != ctx) CK(cudaStreamWaitEvent(cs, p->slots[ctx->batch_seq & 1].ev_done, 0));
   }
-  // fetch-once staging (k >= 5 extension kernels, and the walks when the cache step shares the context stream):
-  // allocated when first needed; this batch's epoch and an empty arena (the bump counter is reset on the context
-  // stream, after the previous batch's kernels and before this batch's walks / matching)
+  // fetch-once staging (k >= 5 extension kernels and walks): this slot's arena, allocated when first needed; the
+  // batch's epoch and an empty arena, reset on the cache step's stream before its walks (the slot's previous user,
+  // batch t-2, has completed: gcsm_wait_batch collected it)
   const bool staging = kmax >= 5 && !listing && ctx->opt.staging_bytes != 1 && !ctx->stage_failed;
   uint32_t stage_epoch = 0;
+  gcsm_ctx::StageSlot &sg = ctx->stg[ctx->batch_seq & 1];
   if (staging) {
-    if (!ctx->d_stage_arena) {
+    if (!ctx->stg[0].arena) {
       size_t freeb = 0, totalb = 0;
       cudaMemGetInfo(&freeb, &totalb);
-      size_t bytes = ctx->opt.staging_bytes ? ctx->opt.staging_bytes : std::min<size_t>(freeb / 4, (size_t)16 << 30);
-      bytes &= ~(size_t)127;
-      if (bytes < 4096 || cudaMalloc(&ctx->d_stage_arena, bytes) != cudaSuccess ||
-          cudaMalloc(&ctx->d_stage_state, 8 * (size_t)S.ncap) != cudaSuccess ||
-          cudaMalloc(&ctx->d_stage_bump, 8) != cudaSuccess) {
+      size_t bytes = ctx->opt.staging_bytes ? ctx->opt.staging_bytes : std::min<size_t>(freeb / 4, (size_t)32 << 30);
+      bytes = (bytes / 2) & ~(size_t)127;  // per slot
+      bool ok = bytes >= 4096;
+      for (auto &x : ctx->stg)
+        ok = ok && cudaMalloc(&x.arena, bytes) == cudaSuccess &&
+             cudaMalloc(&x.state, 8 * (size_t)S.ncap) == cudaSuccess && cudaMalloc(&x.bump, 8) == cudaSuccess;
+      if (!ok) {
         cudaGetLastError();
-        for (void *p : {(void *)ctx->d_stage_arena, (void *)ctx->d_stage_state, (void *)ctx->d_stage_bump})
-          if (p) cudaFree(p);
-        ctx->d_stage_arena = nullptr;
-        ctx->d_stage_state = nullptr;
-        ctx->d_stage_bump = nullptr;
+        for (auto &x : ctx->stg) {
+          for (void *p : {(void *)x.arena, (void *)x.state, (void *)x.bump})
+            if (p) cudaFree(p);
+          x = gcsm_ctx::StageSlot();
+        }
         ctx->stage_failed = true;
       } else {
-        ctx->stage_cap = bytes / 4;
-        CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.ncap, s));
+        for (auto &x : ctx->stg) {
+          x.cap = bytes / 4;
+          CK(cudaMemsetAsync(x.state, 0, 8 * (size_t)S.ncap, cs));
+        }
       }
     }
-    if (ctx->d_stage_arena) {
+    if (sg.arena) {
       stage_epoch = (uint32_t)(ctx->batch_seq % ((1u << 24) - 1)) + 1;  // 24 bits, never 0
-      if (stage_epoch == 1 && ctx->batch_seq > 0) CK(cudaMemsetAsync(ctx->d_stage_state, 0, 8 * (size_t)S.ncap, s));
-      CK(cudaMemsetAsync(ctx->d_stage_bump, 0, 8, s));
+      if (stage_epoch <= 2 && ctx->batch_seq > 1) CK(cudaMemsetAsync(sg.state, 0, 8 * (size_t)S.ncap, cs));
+      CK(cudaMemsetAsync(sg.bump, 0, 8, cs));
     }
   }
-
-  ctx->walk_stage_epoch = (stage_epoch && ctx->gpu_est && !two_streams) ? stage_epoch : 0;
+  ctx->walk_stage_epoch = (stage_epoch && ctx->gpu_est) ? stage_epoch : 0;
 
   CK(cudaEventRecord(sl.ev_c0, cs));
   if (ctx->batch_seq > 0)  // this batch's descriptors start as the previous batch's (after its cache step)
@@ -1621,10 +1630,10 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.tup_rem_cap = rem_cap;
   A.listing = listing ? 1 : 0;
   if (stage_epoch) {
-    A.stage_state = ctx->d_stage_state;
-    A.stage_arena = ctx->d_stage_arena;
-    A.stage_cap = ctx->stage_cap;
-    A.stage_bump = ctx->d_stage_bump;
+    A.stage_state = sg.state;
+    A.stage_arena = sg.arena;
+    A.stage_cap = sg.cap;
+    A.stage_bump = sg.bump;
     A.stage_epoch = stage_epoch;
     A.stage_min = ctx->stage_min;
   }
