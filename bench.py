@@ -72,6 +72,9 @@ def parse():
     ap.add_argument("--emulate", action="store_true",
                     help="test the N>1 plumbing on one GPU: gloo process group, every rank on cuda:0, shard-local "
                          "counts (no NCCL communicator)")
+    ap.add_argument("--private-store", action="store_true",
+                    help="N > 1: every rank builds its own pinned store (default: ONE node-shared store, rank 0 "
+                         "builds it, the others attach; SURVEY 8e)")
     ap.add_argument("--serial", action="store_true",
                     help="synchronous apply_batch per step (default: pipelined submit/wait, so batch t+1's host "
                          "steps overlap batch t's kernels)")
@@ -208,6 +211,21 @@ def workload_name(w):
             f"{w.meta['n_edges'] / 1e6:.0f}M edges"
             + (f" ({w.meta['planted'][0]} planted {w.meta['planted'][1]}-cliques)" if w.meta['planted'][0] else "")
             + (f", {w.meta['L']} labels" if w.meta['L'] else ""))
+
+
+def mem_status():
+    """This process's memory (GB): private anonymous resident, shared-memory resident, peak resident."""
+    out = {}
+    try:
+        with open("/proc/self/status") as f:
+            for line in f:
+                k, _, v = line.partition(":")
+                if k in ("RssAnon", "RssShmem", "VmHWM"):
+                    out[{"RssAnon": "rss_anon_gb", "RssShmem": "rss_shmem_gb", "VmHWM": "peak_rss_gb"}[k]] = \
+                        int(v.split()[0]) / 2**20
+    except OSError:
+        pass
+    return out
 
 
 def sample_of(ins, dele, s):
@@ -360,21 +378,47 @@ def main():
 
     # the host cores are shared by the ranks of one node
     per_rank = max(1, (os.cpu_count() or 1) // world)
-    os.environ.setdefault("GCSM_GEN_THREADS", str(per_rank))
+    shared_store = world > 1 and not args.private_store
+    # (with a shared store only rank 0 generates the graph, on every core)
+    os.environ.setdefault("GCSM_GEN_THREADS", str(os.cpu_count() if shared_store else per_rank))
+    steps = args.warmup + args.steps
     t0 = time.perf_counter()
-    w = workload(args, world)
+    w = workload(args, world) if (rank == 0 or not shared_store) else None
     gen_s = time.perf_counter() - t0
-    queries = args.queries.split(",") if args.queries else w.queries
-    frac = w.budget_frac if args.budget_frac is None else args.budget_frac
-    budget = int(w.adj_bytes * frac)
     nccl_id = G.distributed_nccl_id() if world > 1 and not args.emulate else None
     # one context per GPU holding every standing query of the config: the store, each batch's normalisation,
     # overlays and merge, and ONE cache under the per-GPU budget are shared (gcsm_add_query)
+    common = dict(device=local, rank=rank, world=world, nccl_id=nccl_id, cache_policy=args.cache_policy,
+                  local_counts=bool(args.emulate and world > 1), host_threads=per_rank if world > 1 else 0)
     t0 = time.perf_counter()
-    g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, device=local, rank=rank, world=world, nccl_id=nccl_id,
-               cache_policy=args.cache_policy, local_counts=bool(args.emulate and world > 1),
-               host_threads=per_rank if world > 1 else 0)
+    if not shared_store:
+        g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, **common)
+    else:
+        # node-shared host store: rank 0 generates the graph and builds ONE pinned store; the other
+        # ranks attach to it by handle and receive only the batches (no graph generation, no replica)
+        import torch.distributed as dist
+        if rank == 0:
+            g = G.Gcsm(w.n, w.row_ptr, w.col, w.labels, store_rank=0, store_world=world, **common)
+            meta = [dict(handle=g.store_handle(), n=w.n, name=w.name, meta=w.meta, queries=w.queries,
+                         budget_frac=w.budget_frac, adj_bytes=w.adj_bytes, edges=int(w.row_ptr[-1]),
+                         batches=[(np.asarray(a, np.int32), np.asarray(b, np.int32))
+                                  for a, b in w.batches[:steps + 1]])]
+            w.col = None  # the graph lives in the shared store now (parity / cpu_baseline run at N = 1 only)
+        else:
+            meta = [None]
+        dist.broadcast_object_list(meta, src=0)
+        m = meta[0]
+        if rank > 0:
+            import types
+            w = types.SimpleNamespace(n=m["n"], name=m["name"], meta=m["meta"], queries=m["queries"],
+                                      budget_frac=m["budget_frac"], adj_bytes=m["adj_bytes"],
+                                      row_ptr=np.array([0, m["edges"]], np.int64), batches=m["batches"])
+            g = G.Gcsm(w.n, None, None, store_rank=rank, store_world=world, store_handle=m["handle"], **common)
+        barrier(world)
     create_s = time.perf_counter() - t0
+    queries = args.queries.split(",") if args.queries else w.queries
+    frac = w.budget_frac if args.budget_frac is None else args.budget_frac
+    budget = int(w.adj_bytes * frac)
     for i, q in enumerate(queries):
         k, qe, ql = gi.query(q)
         if i == 0:
@@ -382,7 +426,6 @@ def main():
         else:
             g.add_query(k, qe, ql, gi.order(q))
     g.set_cache_budget(budget)
-    steps = args.warmup + args.steps
     assert len(w.batches) >= steps + 1, "stream too short"
     batches = [(np.ascontiguousarray(a, dtype=np.int32), np.ascontiguousarray(b, dtype=np.int32))
                for a, b in w.batches[:steps + 1]]
@@ -533,6 +576,16 @@ def main():
                     if bq["bcomp_miss_bytes"] else None,
                     "note": "bytes of the DISTINCT main lists the query's kernels touched (SURVEY 8d lower bound), by "
                             "home, measured on one extra untimed batch (gcsm_set_measure)"}}
+    # per-rank host work and memory (shared store: overlays / merges split by vertex owner, one graph per node)
+    q0 = per_q[queries[0]]
+    me = {"rank": rank, "ms_host_per_batch": sum(q0[x] for x in ("ms_normalize", "ms_estimate", "ms_pack",
+                                                                   "ms_merge")) / K,
+          "ms_normalize": q0["ms_normalize"] / K, "ms_merge": q0["ms_merge"] / K, **mem_status()}
+    ranks_host = [me]
+    if world > 1:
+        import torch.distributed as dist
+        ranks_host = [None] * world
+        dist.all_gather_object(ranks_host, me)
     tot_hit = sum(d["hit_bytes"] + d["delta_bytes"] for d in per_q.values())
     tot_all = sum(d["hit_bytes"] + d["delta_bytes"] + d["miss_bytes"] for d in per_q.values())
     if rank != 0:
@@ -592,6 +645,9 @@ def main():
                           "bcomp_hit_gb": None if bcomp is None else bcomp[q]["bcomp_hit_bytes"] / 1e9,
                           "frontier": d["frontier"] / K} for q, d in per_q.items()},
         "gen_seconds": gen_s, "create_seconds": create_s,
+        "host_store": "node-shared (one pinned store, rank 0 builds, ranks attach)" if shared_store else
+                      ("private per rank" if world > 1 else "private"),
+        "ranks_host": ranks_host,
     }
     print(json.dumps(line), flush=True)
     g.close()

@@ -94,6 +94,18 @@ typedef struct {
   uint64_t staging_bytes;  /* per-GPU HBM for the fetch-once staging of zero-copy lists within a batch (DESIGN.md
                               §1d; two arenas, one per in-flight batch; not a cache: emptied every batch):
                               0 = default (a quarter of the free HBM when first needed, at most 32 GiB), 1 = off */
+  int32_t store_rank, store_world; /* node-shared host store ("one shared shm arena cudaHostRegister'ed
+                              in each process"). store_world = 1 (default): this context owns a private
+                              pinned store. store_world = R in [2, 16]: the R local processes (one GPU each) share ONE
+                              pinned, GPU-mapped store: store_rank 0 creates it from row_ptr / col / labels and returns
+                              its handle from gcsm_store_handle(); ranks 1..R-1 pass that handle in store_handle
+                              (row_ptr / col / labels are then ignored and may be NULL; n must match) after rank 0's
+                              gcsm_create returned. The batch calls become collective over the R ranks (identical
+                              batches, same order): each rank writes the overlays and merges of the updated vertices
+                              it owns (x % R == store_rank) behind process-shared barriers. No id growth
+                              (vertex_capacity must be 0 or n). A rank that fails a batch poisons the others' next
+                              barrier (ESTATE); a barrier waits at most GCSM_SHM_TIMEOUT seconds (default 600). */
+  const char *store_handle; /* NULL on store_rank 0; the creating rank's gcsm_store_handle() string elsewhere */
 } gcsm_options;
 
 /* Per-batch statistics (Table II-style breakdown; hit rate §8d). */
@@ -154,10 +166,19 @@ void gcsm_default_options(gcsm_options *opt);
  * [0, n). labels: n values in [0, 65535], or NULL (unlabelled, R5).
  * The graph is copied into the library's pinned, GPU-mapped host store with
  * 2x capacity per list. opt may be NULL (defaults). EINVAL on any
- * violation (nothing allocated). With world > 1 this is collective (NCCL
- * communicator creation). Per-vertex device arrays are sized for opt->vertex_capacity ids. */
+ * violation (nothing allocated). With world > 1 and an nccl_id the NCCL
+ * communicator is created by the first batch call (collective), so that a
+ * node-shared store's rank 0 can return from gcsm_create and hand its store
+ * handle to the other ranks first. Per-vertex device arrays are sized for
+ * opt->vertex_capacity ids. */
 gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels,
                         const gcsm_options *opt, gcsm_ctx **out);
+
+/* Handle of a node-shared store (gcsm_options.store_world > 1) created by this context (store_rank 0): a
+ * NUL-terminated path (the creating process's memfd under /proc) written to buf[cap]. The other local ranks
+ * pass it as gcsm_options.store_handle while this process is alive. EINVAL for a private store or a buffer
+ * shorter than the handle. */
+gcsm_status gcsm_store_handle(const gcsm_ctx *ctx, char *buf, uint64_t cap);
 
 /* Sets the query pattern: k vertices (2..8), m edges qedges[2m] over [0,k)
  * (undirected, simple, connected), qlabels[k] or NULL (any label), and the

@@ -58,7 +58,10 @@ class Gcsm:
 
     def __init__(self, n, row_ptr, col, labels=None, *, device=-1, rank=0, world=1, nccl_id=None, seed=0x6C53,
                  host_threads=0, cache_policy="estimator", walks_override=0, local_counts=False, symmetry=True,
-                 staging_bytes=0, vertex_capacity=0):
+                 staging_bytes=0, vertex_capacity=0, store_rank=0, store_world=1, store_handle=None):
+        """store_world > 1: a node-shared host store (gcsm.h gcsm_options.store_*): store_rank 0 creates it from
+        the CSR and exposes `store_handle()`; the other local ranks pass that string as store_handle (row_ptr /
+        col / labels may then be None)."""
         lib = _lib.load()
         self._lib = lib
         opt = Options()
@@ -75,18 +78,31 @@ class Gcsm:
         opt.staging_bytes = int(staging_bytes)
         opt.vertex_capacity = int(vertex_capacity)
         opt.flags = (FLAG_LOCAL_COUNTS if local_counts else 0) | (0 if symmetry else FLAG_NO_SYMMETRY)
+        opt.store_rank, opt.store_world = int(store_rank), int(store_world)
+        self._handle_buf = None
+        if store_handle is not None:
+            self._handle_buf = store_handle.encode() if isinstance(store_handle, str) else bytes(store_handle)
+            opt.store_handle = self._handle_buf
         self.n = int(n)
-        self._rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
-        self._col = np.ascontiguousarray(col, dtype=np.int32)
-        lab = _i32(labels)
+        attach = store_handle is not None
+        self._rp = None if attach else np.ascontiguousarray(row_ptr, dtype=np.int64)
+        self._col = None if attach else np.ascontiguousarray(col, dtype=np.int32)
+        lab = None if attach else _i32(labels)
         h = ctypes.c_void_p()
         s = lib.gcsm_create(self.n, _ptr(self._rp), _ptr(self._col), _ptr(lab), ctypes.byref(opt), ctypes.byref(h))
+        self._rp = self._col = None  # copied into the library's store: the caller may free the CSR
         if s:
             raise GcsmError(s, "gcsm_create failed")
         self._h = h
         self.k = None
 
     # ------------------------------------------------------------------ API
+    def store_handle(self) -> str:
+        """The node-shared store's handle (store_rank 0 of a store_world > 1 context)."""
+        buf = ctypes.create_string_buffer(4096)
+        self._check(self._lib.gcsm_store_handle(self._h, buf, len(buf)), "store_handle")
+        return buf.value.decode()
+
     def _check(self, s, what):
         if s:
             msg = self._lib.gcsm_last_error(self._h)

@@ -22,14 +22,15 @@ SYMBOLS = ["gcsm_default_options", "gcsm_create", "gcsm_set_query", "gcsm_set_ca
            "gcsm_nccl_unique_id", "gcsm_get_stream", "gcsm_export_csr", "gcsm_get_estimates", "gcsm_get_cached",
            "gcsm_plan_inspect", "gcsm_query_restrictions", "gcsm_shard",
            "gcsm_measure_host_link", "gcsm_binomial_samples", "gcsm_set_measure",
-           "gcsm_num_vertices", "gcsm_add_vertices", "gcsm_link_peers"]
+           "gcsm_num_vertices", "gcsm_add_vertices", "gcsm_link_peers", "gcsm_store_handle"]
 
 
 class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("nccl_id", ctypes.c_void_p), ("seed", ctypes.c_uint64), ("host_threads", ctypes.c_int32),
                 ("cache_policy", ctypes.c_int32), ("walks_override", ctypes.c_uint64), ("flags", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32), ("vertex_capacity", ctypes.c_int64), ("staging_bytes", ctypes.c_uint64)]
+                ("reserved", ctypes.c_uint32), ("vertex_capacity", ctypes.c_int64), ("staging_bytes", ctypes.c_uint64),
+                ("store_rank", ctypes.c_int32), ("store_world", ctypes.c_int32), ("store_handle", ctypes.c_char_p)]
 
 
 class Stats(ctypes.Structure):
@@ -85,6 +86,7 @@ def load():
         "gcsm_binomial_samples": (st, [U64, I64, ctypes.c_double, I64, P]),
         "gcsm_set_measure": (st, [P, ctypes.c_uint32]),
         "gcsm_num_vertices": (I32, [P]),
+        "gcsm_store_handle": (st, [P, P, U64]),
         "gcsm_link_peers": (st, [P, I32]),
         "gcsm_add_vertices": (st, [P, I32, P, ctypes.POINTER(I32)]),
         "gcsm_query_restrictions": (st, [I32, I32, P, P, P, P, I32, P, ctypes.POINTER(U64)]),

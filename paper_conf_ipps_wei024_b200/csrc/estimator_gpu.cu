@@ -280,6 +280,7 @@ struct WalkArgs {
   uint32_t stage_min;
   unsigned long long *stage_cnt;
   const char *dev_lo[2], *dev_hi[2];
+  int32_t lane_leaf;            // level k-3 nodes one per lane (walk_leaf_parent; GCSM_WALK_LANE=0: warp-wide DFS)
 };
 
 constexpr int kEW = 8;  // warps per block
@@ -425,6 +426,83 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
   }
 }
 
+// A node at level k-3 whose B is in BINV's domain (its expected selections B x len / D are few; C4 prism6: the
+// level-3 nodes) walked by ONE lane: it records B on its next position's backward lists, draws its children by the
+// same skip sampling as the warp-wide step (one segment's gaps drawn one after another with uniforms j = 1, 2, ...
+// of the segment's stream: the same draws), and every surviving child (level k-2, whose children are leaves)
+// records its B' ~ Bin(B, 1/D) conditioned on >= 1 (d_binom_pos, the child's own key). Integer atomics: the sums
+// equal the warp-wide DFS's bit for bit. f[0..cl-1] are the matched positions, v the node's vertex at cl.
+__device__ __noinline__ void walk_leaf_parent(const WalkArgs &A, const DevPlan *P, const int32_t *f, int cl,
+                                              int32_t v, unsigned long long B, unsigned long long key,
+                                              unsigned long long &walg, unsigned long long &whit) {
+  const LevelPlan &Lq = P->lv[cl + 1];
+  const int nb = Lq.nb;
+  auto fat = [&](int p) { return p == cl ? v : f[p]; };
+  for (int b = 0; b < nb; ++b) {
+    const int32_t w = fat(Lq.bpos[b]);
+    atomicAdd(A.levcnt + (size_t)w * A.levels + (cl - 1), B);
+    atomicOr(A.touched + (w >> 5), 1u << (w & 31));
+  }
+  int drv = 0;
+  LR D;
+  uint32_t best = 0xffffffffu;
+  for (int b = 0; b < nb; ++b) {
+    const LR L = view_of(A.vdesc, A.drec, A.dlist, fat(Lq.bpos[b]), Lq.bview[b]);
+    if (L.ml + L.xl < best) {
+      best = L.ml + L.xl;
+      drv = b;
+      D = L;
+    }
+  }
+  if (best == 0) return;
+  // staged copies (this batch's arena) of the main lists, where another reader already fetched them
+  auto staged = [&](int32_t vb, const int32_t *m, uint32_t ml) -> const int32_t * {
+    if (!A.stage.state || ml < A.stage_min) return m;
+    const unsigned long long st = stage_word(A.stage.state + vb);
+    if ((st >> 40) == A.stage.epoch && (st & kStReady) && (st & kStOff) != kStOff) {
+      whit += 4ull * ml;
+      return A.stage.arena + (st & kStOff);
+    }
+    return m;
+  };
+  const int32_t *dm = staged(fat(Lq.bpos[drv]), D.m, D.ml);
+  const double r0 = A.T.r0tab[B];
+  double pw[kSkipLog + 1];
+  d_skip_table(r0, pw);
+  const LevelPlan &Lc = P->lv[cl + 2];  // the children's next position (they record, R17)
+  for (uint32_t s0 = 0; s0 < best; s0 += kSkipSeg) {
+    const uint32_t s1 = min(best, s0 + kSkipSeg);
+    const unsigned long long segkey = dchain(key, kSkipTag + s0 / kSkipSeg);
+    uint32_t pos = s0;
+    for (unsigned long long j = 1;; ++j) {
+      const uint32_t sel = pos + d_skip_gap(pw, d_skip_uniform(segkey, j));
+      if (sel >= s1) break;
+      pos = sel + 1;
+      walg += 4;
+      const int32_t c = sel < D.ml ? dm[sel] : D.x[sel - D.ml];
+      bool ok = c != v;
+      for (int s2 = 0; s2 < cl && ok; ++s2) ok = f[s2] != c;
+      if (ok && Lq.label >= 0) ok = (A.lab ? (int32_t)A.lab[c] : 0) == Lq.label;
+      for (int b = 0; b < nb && ok; ++b) {
+        if (b == drv) continue;
+        const int32_t vb = fat(Lq.bpos[b]);
+        const LR Lb = view_of(A.vdesc, A.drec, A.dlist, vb, Lq.bview[b]);
+        walg += 4ull * (Lb.ml + Lb.xl);
+        ok = has(staged(vb, Lb.m, Lb.ml), Lb.ml, c) || (Lb.xl && has(Lb.x, Lb.xl, c));
+      }
+      if (!ok) continue;
+      const unsigned long long ck = dchain(key, (unsigned long long)(uint32_t)c);
+      const unsigned long long Bc = (unsigned long long)d_binom_pos(ck, (int64_t)B, A.T.pD, r0);
+      for (int b = 0; b < Lc.nb; ++b) {
+        const int p = Lc.bpos[b];
+        const int32_t w = p == cl + 1 ? c : fat(p);
+        atomicAdd(A.levcnt + (size_t)w * A.levels + cl, Bc);
+        atomicOr(A.touched + (w >> 5), 1u << (w & 31));
+      }
+    }
+  }
+}
+
 // Levels >= 2 (phase B, k >= 5): warp per level-2 node, DFS over the rest of its subtree.
 #ifndef GCSM_WALK_MINBLOCKS
 #define GCSM_WALK_MINBLOCKS 3  // resident 256-thread blocks per SM for k_walks (latency hiding of its list reads)
@@ -437,11 +515,18 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
   const unsigned long long n2 = min(*(volatile unsigned long long *)A.f2_count, (unsigned long long)A.f2_cap);
   unsigned long long wfill = 0, wlists = 0, whit = 0;  // fetch-once staging counters
   unsigned long long walg = 0;                         // algorithmic list bytes (driver scans + probes)
+  unsigned long long d_root = 0, d_lane = 0, d_desc = 0, d_step = 0;  // work profile (CNT_WDBG)
   for (;;) {
     unsigned long long u = 0;
     if (lane == 0) u = atomicAdd(A.cursor2, 1ull);
     u = __shfl_sync(FULL, u, 0);
     if (u >= n2) {
+      if (lane == 0 && A.alg_cnt) {
+        atomicAdd(A.alg_cnt + 1, d_root);
+        atomicAdd(A.alg_cnt + 2, d_lane);
+        atomicAdd(A.alg_cnt + 3, d_desc);
+        atomicAdd(A.alg_cnt + 4, d_step);
+      }
       if (lane == 0 && A.stage_cnt && (wfill | wlists | whit)) {
         atomicAdd(A.stage_cnt + 0, wfill);
         atomicAdd(A.stage_cnt + 1, wlists);
@@ -453,6 +538,7 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
     const EstNode2 N = A.f2[u];
     const DevPlan *P = A.plans + N.plan;
     const int k = P->k;
+    ++d_root;
     __syncwarp();
     if (lane == 0) {
       W.f[0] = N.f0;
@@ -544,7 +630,29 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
         continue;
       }
       const int si = S.si, ns = S.ns;
+      if (si == 0 && ns > 0 && level + 1 == k - 3 && A.lane_leaf) {
+        // children at level k-3 in BINV's domain: one lane each (walk_leaf_parent) instead of one warp-wide DFS
+        // descent per child
+        bool fast = true;
+        unsigned long long cB = 0, cK = 0;
+        int32_t cv = 0;
+        if (lane < ns) {
+          cB = S.sB[lane];
+          cK = S.skey[lane];
+          cv = S.sv[lane];
+          fast = cB > 0 && T.pD > 0.0 && T.pD <= 0.5 && DM((double)cB, T.pD) < 10.0 && (int64_t)cB < T.r0n;
+        }
+        if (__all_sync(FULL, fast)) {
+          d_lane += ns;
+          if (lane < ns) walk_leaf_parent(A, P, W.f, level + 1, cv, cB, cK, walg, whit);
+          __syncwarp();
+          if (lane == 0) S.si = ns;
+          __syncwarp();
+          continue;
+        }
+      }
       if (si < ns) {  // descend into the next surviving child
+        ++d_desc;
         __syncwarp();
         if (lane == 0) {
           S.si = si + 1;
@@ -567,6 +675,7 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
         continue;
       }
       const int p = level + 1;
+      ++d_step;
       const int32_t *dm = S.dm, *dx = S.dx;
       const unsigned long long key = S.key, t53 = S.T53;
       const int64_t Bn = (int64_t)S.B;
@@ -1171,6 +1280,7 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.stage_cnt = c.stage_cnt;
       A.alg_cnt = c.alg_cnt[q];
       A.walk_stage = c.walk_stage;
+      A.lane_leaf = c.walk_lane;
       for (int r = 0; r < 2; ++r) {
         A.dev_lo[r] = c.dev_lo[r];
         A.dev_hi[r] = c.dev_hi[r];

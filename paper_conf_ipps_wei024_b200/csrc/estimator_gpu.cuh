@@ -99,6 +99,7 @@ struct CacheStep {
   unsigned long long *alg_cnt[GCSM_MAX_QUERIES] = {};  // per query: algorithmic list bytes of its walks
   StageRef stage{};
   int32_t walk_stage = 1;  // skip-sampled drivers: 0 always staged, 1 when >= 1 selection is expected, 2 never
+  int32_t walk_lane = 1;   // level k-3 nodes in BINV's domain one per lane (walk_leaf_parent)
   uint32_t stage_min = 1;
   unsigned long long *stage_cnt = nullptr;  // fill bytes, lists, hit bytes
   const char *dev_lo[2] = {nullptr, nullptr}, *dev_hi[2] = {nullptr, nullptr};

@@ -155,6 +155,8 @@ struct gcsm_ctx {
   Slot slots[2];
   uint64_t waited = 0;  // batches whose results have been collected
   ncclComm_t comm = nullptr;
+  bool comm_pending = false;       // the communicator is created at the first batch (collective)
+  unsigned char nccl_id[128] = {};
   int grid = 0, warps_total = 0;
   int ext_grid = 0;  // blocks of the extension kernels (GCSM_EXT_RESERVE blocks left for the overlapped cache step)
 
@@ -232,11 +234,15 @@ struct gcsm_ctx {
   uint32_t stage_min = 1;          // shortest list (ints) routed through the arena (GCSM_STAGE_MIN)
   uint32_t walk_stage_epoch = 0;   // this batch's walks stage through the arena too (0 = no)
   int32_t stage_policy = 1;        // smem staging model for device-resident probe lists (GCSM_STAGE_POLICY)
+  int32_t walk_lane = 1;           // GCSM_WALK_LANE=0: level k-3 walk nodes by the warp-wide DFS (A/B)
   int32_t walk_stage = 1;          // staging of skip-sampled walk drivers (GCSM_WALK_STAGE: 0 always, 1 expected >= 1, 2 never)
   // B_comp measurement mode (GCSM_BCOMP=1 at create): bitmap of the vertices whose main list a query's kernels read
   uint32_t *d_touched_bc = nullptr;
   bool bcomp = false;
   std::vector<void *> retired_pinned;  // pinned staging replaced by a larger one (freed at destroy)
+  // shared store: host arrays retired by batch t's merge, recycled once EVERY rank has collected batch t (at the
+  // first barrier of batch t+2: a rank submits t+2 only after waiting for t)
+  std::vector<std::pair<uint64_t, std::vector<std::pair<int32_t *, uint32_t>>>> pending_retired;
 
 
   // cache / batch state
@@ -252,6 +258,7 @@ struct gcsm_ctx {
   gcsm_status fail(gcsm_status s, const std::string &m) {
     err = m;
     if (s == GCSM_EDEVICE || s == GCSM_ENCCL || (in_batch && s != GCSM_EINVAL)) poisoned = true;
+    if (poisoned) store.poison_shared();  // the other ranks of a shared store stop at their next barrier
     return s;
   }
   gcsm_status cuda_fail(cudaError_t e, const char *where) {
@@ -340,6 +347,7 @@ void gcsm_default_options(gcsm_options *o) {
   o->seed = 0x6C53;
   o->host_threads = 0;
   o->cache_policy = GCSM_CACHE_ESTIMATOR;
+  o->store_world = 1;
 }
 
 gcsm_status gcsm_nccl_unique_id(void *out128) {
@@ -360,7 +368,12 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return GCSM_EINVAL;
   if (o.world > 1 && !o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) return GCSM_EINVAL;
   if (o.cache_policy < 0 || o.cache_policy > 2) return GCSM_EINVAL;
-  if (n < 1 || !row_ptr) return GCSM_EINVAL;
+  if (o.store_world < 1) o.store_world = 1;
+  const bool shared = o.store_world > 1;
+  if (shared && (o.store_world > GCSM_MAX_STORE_RANKS || o.store_rank < 0 || o.store_rank >= o.store_world ||
+                 (o.store_rank > 0) != (o.store_handle != nullptr) || (o.vertex_capacity != 0 && o.vertex_capacity != n)))
+    return GCSM_EINVAL;
+  if (n < 1 || (!row_ptr && !(shared && o.store_rank > 0))) return GCSM_EINVAL;
   gcsm_ctx *ctx = new (std::nothrow) gcsm_ctx();
   if (!ctx) return GCSM_ENOMEM;
   ctx->opt = o;
@@ -383,8 +396,13 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
     return GCSM_EINVAL;
   }
   const int32_t ncap = (int32_t)std::max<int64_t>(n, o.vertex_capacity);
-  std::string e = ctx->store.init(n, row_ptr, col, labels, threads, &cuda_err, ncap);
+  std::string e = !shared ? ctx->store.init(n, row_ptr, col, labels, threads, &cuda_err, ncap)
+                  : o.store_rank == 0
+                      ? ctx->store.init_shared(n, row_ptr, col, labels, threads, &cuda_err, o.store_world)
+                      : ctx->store.attach_shared(o.store_handle, n, threads, &cuda_err, o.store_rank, o.store_world);
+  ctx->opt.store_handle = nullptr;  // caller-owned: not kept
   if (!e.empty()) {
+    if (std::getenv("GCSM_TRACE")) std::fprintf(stderr, "[gcsm] create: %s\n", e.c_str());
     delete ctx;
     return cuda_err ? GCSM_EDEVICE : GCSM_EINVAL;
   }
@@ -426,7 +444,7 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
       if (cudaMemcpy(sl.d_vdesc, vd.data(), sizeof(VDesc) * (size_t)ncap, cudaMemcpyHostToDevice) != cudaSuccess)
         return bail(GCSM_EDEVICE);
   }
-  if (labels) {
+  if (!ctx->store.lab.empty()) {
     if (cudaMalloc(&ctx->d_lab, 2 * (size_t)ncap) != cudaSuccess) return bail(GCSM_ENOMEM);
     if (cudaMemcpy(ctx->d_lab, ctx->store.lab.data(), 2 * (size_t)ncap, cudaMemcpyHostToDevice) != cudaSuccess)
       return bail(GCSM_EDEVICE);
@@ -441,17 +459,20 @@ gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, c
   if (const char *sm = std::getenv("GCSM_STAGE_MIN")) ctx->stage_min = (uint32_t)std::max(1, std::atoi(sm));
   if (const char *sp = std::getenv("GCSM_STAGE_POLICY")) ctx->stage_policy = std::atoi(sp);
   if (const char *ws = std::getenv("GCSM_WALK_STAGE")) ctx->walk_stage = std::atoi(ws);
+  if (const char *wl = std::getenv("GCSM_WALK_LANE")) ctx->walk_lane = std::atoi(wl);
   if (std::getenv("GCSM_BCOMP") && gcsm_set_measure(ctx, GCSM_MEASURE_BCOMP) != GCSM_OK) return bail(GCSM_ENOMEM);
   ctx->grid = match_grid(dev, &ctx->warps_total);
   ctx->ext_grid = ctx->grid;
   if (const char *r = std::getenv("GCSM_EXT_RESERVE"))
     if (ctx->overlap) ctx->ext_grid = std::max(1, ctx->grid - std::atoi(r));
   // a communicator whenever an id is given (world 1 included: the single-rank allreduce exercises the same path)
+  // (created at the first batch, which every rank enters collectively: creating it here would block rank 0 of a
+  // node-shared store in ncclCommInitRank before the other ranks could attach to the store it just made)
   if (o.nccl_id && !(o.flags & GCSM_FLAG_LOCAL_COUNTS)) {
-    ncclUniqueId id;
-    std::memcpy(&id, o.nccl_id, sizeof id);
-    if (ncclCommInitRank(&ctx->comm, o.world, id, o.rank) != ncclSuccess) return bail(GCSM_ENCCL);
+    std::memcpy(ctx->nccl_id, o.nccl_id, sizeof ctx->nccl_id);
+    ctx->comm_pending = true;
   }
+  ctx->opt.nccl_id = nullptr;  // caller-owned: copied
   *out = ctx;
   return GCSM_OK;
 }
@@ -493,6 +514,14 @@ gcsm_status gcsm_link_peers(gcsm_ctx *const *ctxs, int32_t n) {
     ctxs[i]->peer_idx = i;
     cudaSetDevice(ctxs[i]->device);
   }
+  return GCSM_OK;
+}
+
+gcsm_status gcsm_store_handle(const gcsm_ctx *ctx, char *buf, uint64_t cap) {
+  if (!ctx || !buf || !ctx->store.shared() || ctx->store.store_rank() != 0) return GCSM_EINVAL;
+  const std::string h = ctx->store.handle();
+  if (cap < h.size() + 1) return GCSM_EINVAL;
+  std::memcpy(buf, h.c_str(), h.size() + 1);
   return GCSM_OK;
 }
 
@@ -913,6 +942,7 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   c.ev_walk = sl.ev_walk.data();
   for (int qi = 0; qi < nq && qi < GCSM_MAX_QUERIES; ++qi) c.alg_cnt[qi] = sl.d_cnt + (size_t)qi * CNT_N + CNT_WALG;
   sl.walks_timed = est_on;
+  c.walk_lane = ctx->walk_lane;
   if (ctx->walk_stage_epoch && !std::getenv("GCSM_NO_WALK_STAGE")) {  // the walks' zero-copy lists through the arena
     const gcsm_ctx::StageSlot &sg = ctx->stg[ctx->batch_seq & 1];
     c.stage = StageRef{sg.state, sg.arena, sg.cap, sg.bump, ctx->walk_stage_epoch};
@@ -971,6 +1001,29 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
 
   // ---- (1) normalise + overlay + units -------------------------------------------------
   Timer t1;
+  if (ctx->comm_pending) {  // every rank's first batch: the count allreduce's communicator
+    ncclUniqueId id;
+    static_assert(sizeof id == sizeof ctx->nccl_id, "ncclUniqueId is 128 bytes");
+    std::memcpy(&id, ctx->nccl_id, sizeof id);
+    if (ncclCommInitRank(&ctx->comm, ctx->opt.world, id, ctx->opt.rank) != ncclSuccess) {
+      ctx->comm = nullptr;
+      return ctx->fail(GCSM_ENCCL, "ncclCommInitRank failed");
+    }
+    ctx->comm_pending = false;
+  }
+  if (S.shared()) {  // node-shared store: every rank enters the batch (and has collected batch t-2)
+    if (!S.barrier()) {
+      ctx->poisoned = true;
+      return ctx->fail(GCSM_ESTATE, S.shared_err);
+    }
+    auto &pr = ctx->pending_retired;
+    size_t keep = 0;
+    for (auto &p : pr) {
+      if (p.first + 2 <= ctx->batch_seq) S.recycle(p.second);
+      else pr[keep++] = std::move(p);
+    }
+    pr.resize(keep);
+  }
   std::string e = S.normalize(n_ins, ins, n_del, del);
   if (!e.empty()) return ctx->fail(GCSM_EINVAL, e);
   ctx->in_batch = true;
@@ -978,8 +1031,14 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
     return ctx->fail(GCSM_ENOMEM, "pinned allocation for new vertices failed");
   tr.mark("normalize");
   bool cuda_err = false;
-  if (!S.build_overlay((int)(ctx->batch_seq & 1), &cuda_err))
+  if (!S.build_overlay((int)(ctx->batch_seq & 1), &cuda_err)) {
+    if (S.shared()) {
+      S.poison_shared();
+      ctx->poisoned = true;
+      return ctx->fail(GCSM_ESTATE, S.shared_err);
+    }
     return ctx->fail(GCSM_EDEVICE, "pinned overlay allocation failed");
+  }
   tr.mark("overlay");
   st.n_ins = S.I.size();
   st.n_del = S.D.size();
@@ -1030,29 +1089,20 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
           cost.push_back(ac[sidx]);
         }
     }
-    if (ctx->opt.world > 1) {
+    {  // this rank's LPT shard (world > 1), heaviest units first (dynamic scheduling tail): one parallel stable
+       // sort by cost serves both
       std::vector<int32_t> rk(units.size());
-      shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data());
-      size_t w = 0;
-      for (size_t i = 0; i < units.size(); ++i)
-        if (rk[i] == ctx->opt.rank) {
-          units[w] = units[i];
-          cost[w] = cost[i];
-          ++w;
+      std::vector<size_t> idx;
+      shard_lpt((int64_t)units.size(), cost.data(), ctx->opt.world, rk.data(), T, &idx);
+      std::vector<Unit> u2;
+      std::vector<uint64_t> c2;
+      u2.reserve(units.size());
+      c2.reserve(units.size());
+      for (size_t i : idx)
+        if (rk[i] == ctx->opt.rank || ctx->opt.world <= 1) {
+          u2.push_back(units[i]);
+          c2.push_back(cost[i]);
         }
-      units.resize(w);
-      cost.resize(w);
-    }
-    {  // heaviest units first (dynamic scheduling tail)
-      std::vector<size_t> idx(units.size());
-      std::iota(idx.begin(), idx.end(), 0);
-      parallel_sort(idx, [&](size_t x, size_t y) { return cost[x] > cost[y]; }, T, /*stable=*/true);
-      std::vector<Unit> u2(units.size());
-      std::vector<uint64_t> c2(units.size());
-      for (size_t i = 0; i < idx.size(); ++i) {
-        u2[i] = units[idx[i]];
-        c2[i] = cost[idx[i]];
-      }
       units.swap(u2);
       cost.swap(c2);
     }
@@ -1793,7 +1843,13 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // ---- (5) reorganise the host lists. P:302 runs it after matching so the kernel reads consistent data: here
   // the merge writes fresh arrays and the ones the in-flight kernels may read are retired, not overwritten.
   Timer t5;
-  if (!S.merge(sl.retired)) return ctx->fail(GCSM_ENOMEM, "pinned allocation for the merged lists failed");
+  if (!S.merge(sl.retired)) {
+    if (S.shared()) {
+      ctx->poisoned = true;
+      return ctx->fail(GCSM_ESTATE, S.shared_err);
+    }
+    return ctx->fail(GCSM_ENOMEM, "pinned allocation for the merged lists failed");
+  }
   tr.mark("merge");
   if (!ctx->gpu_est) {
     parallel_for(T, (int64_t)ctx->prev_cached.size(), [&](int, int64_t lo, int64_t hi) {
@@ -1886,6 +1942,9 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
                    "entries=%llu pruned=%llu l3=%llu l3kept=%llu l4=%llu last_drv=%llu\n",
                    qi, h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_DBG_SPLIT] / 1e9,
                    h[CNT_COPIED] / 1e9, h[CNT_X_ENTRIES], h[CNT_X_PRUNED], h[CNT_X_L3], h[CNT_X_L3F], h[CNT_X_L4], h[CNT_X_LAST]);
+    if (std::getenv("GCSM_TRACE"))
+      std::fprintf(stderr, "[gcsm walks] q=%d roots=%llu lane_nodes=%llu dfs_descents=%llu steps=%llu walg_gb=%.3f\n", qi,
+                   h[CNT_WDBG], h[CNT_WDBG + 1], h[CNT_WDBG + 2], h[CNT_WDBG + 3], h[CNT_WALG] / 1e9);
     if (qi == 0 && (sl.tup_add || sl.tup_rem)) {
       const int k = ctx->qs[0].qp.k;
       const uint64_t na = std::min<uint64_t>(h[CNT_TUP_ADD], sl.add_cap);
@@ -1899,7 +1958,10 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
     st.ms_total = sl.host_ms + tw.ms();
     ctx->qs[qi].stats = st;
   }
-  ctx->store.recycle(sl.retired);  // arrays the batch's kernels could read are free again
+  if (ctx->store.shared())  // other ranks' kernels may still read them: recycled at batch waited+2's first barrier
+    ctx->pending_retired.emplace_back(ctx->waited, std::move(sl.retired)), sl.retired.clear();
+  else
+    ctx->store.recycle(sl.retired);  // arrays the batch's kernels could read are free again
   sl.inflight = false;
   ++ctx->waited;
   if (added) *added = ctx->qs[0].stats.added;

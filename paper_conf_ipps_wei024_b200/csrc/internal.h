@@ -178,6 +178,7 @@ uint64_t rng_chain(uint64_t h, uint64_t x);
 int64_t binomial(uint64_t key, int64_t n, double p);
 
 // ------------------------------------------------------------ sharding
-void shard_lpt(int64_t n, const uint64_t *cost, int world, int32_t *rank_out);
+void shard_lpt(int64_t n, const uint64_t *cost, int world, int32_t *rank_out, int threads = 1,
+               std::vector<size_t> *order_out = nullptr);
 
 }  // namespace gcsm

@@ -52,7 +52,8 @@ enum Counter {
   CNT_WLISTS = 41,
   CNT_WHIT = 42,
   CNT_WALG = 43,   // per query: algorithmic list bytes its walks read (driver scans + membership probes, §8d)
-  CNT_N = 44
+  CNT_WDBG = 44,   // per query, k_walks work profile (GCSM_TRACE): level-2 roots, lane-walked nodes, DFS descents, steps
+  CNT_N = 48
 };
 
 struct MatchArgs {

@@ -239,15 +239,15 @@ std::string build_plan(int k, int m, const int32_t *qedges, const int32_t *qlabe
 
 // Greedy LPT: units by cost descending (ties: lower index first) each go to
 // the least-loaded rank (ties: lower rank). Deterministic on every rank.
-void shard_lpt(int64_t n, const uint64_t *cost, int world, int32_t *rank_out) {
-  if (world <= 1) {
-    for (int64_t i = 0; i < n; ++i) rank_out[i] = 0;
-    return;
-  }
-  std::vector<int64_t> idx(n);
+// The descending order is a parallel stable sort (the same order as a serial one); *order_out (optional) receives
+// it, so a caller can keep its own units heaviest first without sorting again.
+void shard_lpt(int64_t n, const uint64_t *cost, int world, int32_t *rank_out, int threads,
+               std::vector<size_t> *order_out) {
+  std::vector<size_t> idx((size_t)n);
   std::iota(idx.begin(), idx.end(), 0);
-  std::stable_sort(idx.begin(), idx.end(), [&](int64_t x, int64_t y) { return cost[x] > cost[y]; });
-  std::vector<uint64_t> load(world, 0);
+  if (world > 1 || order_out)
+    parallel_sort(idx, [&](size_t x, size_t y) { return cost[x] > cost[y]; }, std::max(1, threads), /*stable=*/true);
+  std::vector<uint64_t> load(std::max(1, world), 0);
   for (int64_t t = 0; t < n; ++t) {
     int best = 0;
     for (int r = 1; r < world; ++r)
@@ -255,6 +255,7 @@ void shard_lpt(int64_t n, const uint64_t *cost, int world, int32_t *rank_out) {
     rank_out[idx[t]] = best;
     load[best] += cost[idx[t]] + 1;
   }
+  if (order_out) order_out->swap(idx);
 }
 
 }  // namespace gcsm

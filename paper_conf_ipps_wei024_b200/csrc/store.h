@@ -29,6 +29,26 @@ struct Chunk {
   size_t size = 0, used = 0;
 };
 
+#define GCSM_MAX_STORE_RANKS 16
+
+// Node-shared store ("one shared shm arena cudaHostRegister'ed in each process"): one memfd mapping at
+// the same virtual address in every local rank, so the list pointers in the shared per-vertex metadata are valid
+// everywhere. Layout: this header (4 KiB), lst / len / cap / lab arrays (ncap each), two overlay areas (one per
+// in-flight batch), the initial lists, then one growth region per rank (the merges of the vertices it owns,
+// x % store_world == store_rank). See DESIGN.md §6.
+struct ShmHeader {
+  uint64_t magic, total_bytes, base_addr;
+  int32_t n, ncap, world, labelled;
+  int32_t leader_pid, fd;
+  uint64_t off_lst, off_len, off_cap, off_lab, off_ovl[2], ovl_bytes, off_lists;
+  uint64_t reg_lo[GCSM_MAX_STORE_RANKS], reg_hi[GCSM_MAX_STORE_RANKS];
+  std::atomic<uint64_t> reg_used[GCSM_MAX_STORE_RANKS];
+  std::atomic<uint32_t> attached;
+  std::atomic<uint32_t> failed;  // a rank poisoned its context: the others' barriers return false
+  alignas(64) std::atomic<uint32_t> bar_count;
+  alignas(64) std::atomic<uint32_t> bar_gen;
+};
+
 class HostStore {
  public:
   ~HostStore();
@@ -37,11 +57,26 @@ class HostStore {
   std::string init(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels, int threads,
                    bool *cuda_err, int32_t ncap = 0);
 
+  // node-shared store: store_rank 0 creates it (init with store_world > 1), the others attach to the handle
+  std::string init_shared(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels, int threads,
+                          bool *cuda_err, int store_world);
+  std::string attach_shared(const char *handle, int32_t n, int threads, bool *cuda_err, int store_rank,
+                            int store_world);
+  std::string handle() const;  // "/proc/<pid>/fd/<fd>" of the leader's memfd ("" for a private store)
+  bool shared() const { return shm_ != nullptr; }
+  int store_rank() const { return srank_; }
+  int store_world() const { return sworld_; }
+  bool owned(int32_t x) const { return !shm_ || x % sworld_ == srank_; }
+  // process-shared barrier of the store's ranks (no-op for a private store); false: timeout or a failed rank
+  bool barrier();
+  void poison_shared();
+  std::string shared_err;  // why the last shared-store operation failed
+
   int32_t n = 0;     // current vertex count (ids [0, n))
   int32_t ncap = 0;  // capacity: every per-vertex array is sized ncap
   int threads = 1;
-  std::vector<int32_t *> lst;   // host address of each list (pinned, mapped)
-  std::vector<uint32_t> len, cap;
+  int32_t **lst = nullptr;   // host address of each list (pinned, mapped); shared metadata with a shared store
+  uint32_t *len = nullptr, *cap = nullptr;
   std::vector<uint16_t> lab;    // empty if unlabelled
   uint32_t maxdeg = 0;
   uint64_t edges2 = 0;          // Σ len
@@ -62,6 +97,8 @@ class HostStore {
   // step ⑤: base(x) <- S(x) ∪ ins(x) for x ∈ U, always into a *fresh* array (a recycled one of the same
   // capacity class, or a doubled one when full) so that a batch whose kernels are still reading
   // the old arrays (pipelined submit) is not disturbed; the old arrays are appended to `retired`.
+  // With a shared store every rank computes the new lengths of all of U, then (after a barrier: every rank is done
+  // reading G_t) merges only the vertices it owns, and a second barrier publishes G_{t+1}.
   bool merge(std::vector<std::pair<int32_t *, uint32_t>> &retired);  // false: pinned allocation failed
   void recycle(std::vector<std::pair<int32_t *, uint32_t>> &retired);  // once their batch has completed
   void clear_batch();
@@ -79,6 +116,13 @@ class HostStore {
   std::vector<uint64_t> deg_hist;          // vertices per degree (exact max degree)
 
  private:
+  std::vector<int32_t *> lst_v_;
+  std::vector<uint32_t> len_v_, cap_v_;
+  ShmHeader *shm_ = nullptr;
+  size_t shm_size_ = 0;
+  int srank_ = 0, sworld_ = 1;
+  double bar_timeout_s_ = 600.0;
+  std::string finish_shared_attach(bool *cuda_err);
   std::vector<Chunk> chunks_;
   Chunk overlay_[2];
   std::map<uint32_t, std::vector<int32_t *>> free_;  // recycled arrays by capacity

@@ -341,7 +341,8 @@ def test_gpu_estimator_unbiased_eq6(G, name):
         assert np.all(row[s_] * M >= N1 * (1 - 1e-12))
 
 
-@pytest.mark.parametrize("name,labelled", [("diamond", False), ("k4", False), ("house5u", False), ("house5", True)])
+@pytest.mark.parametrize("name,labelled", [("diamond", False), ("k4", False), ("house5u", False), ("house5", True),
+                                           ("prism6", False)])
 def test_gpu_walker_equals_host_walker(G, name, labelled):
     """Product-internal: the device walker draws exactly what the host walker draws (R30), batch after batch; the
     two packers select by R23 (GPU path: over the vertices not updated by the batch, R32) — checked against the
@@ -410,6 +411,36 @@ def test_gpu_walker_btrd_range(G, name, M):
     assert np.array_equal(g.cached(), oracle.select_cache(eg, sz, budget & ~15, exclude=updated_vertices(I, D)))
     g.close()
     h.close()
+
+
+@pytest.mark.parametrize("name", ["prism6", "k4tri6", "wheel7"])
+def test_walk_lane_path_equals_warp_dfs(G, name, monkeypatch):
+    """Product-internal: the level k-3 walk nodes walked one per lane (walk_leaf_parent, default) record exactly the
+    sums of the warp-wide DFS (GCSM_WALK_LANE=0) on a C4-shaped planted graph. M is chosen so that level k-3 nodes
+    carry B ~ 2 (M = 2 N1 D^(k-4): B_l ~ M / (N1 D^(l-1))), i.e. they are in BINV's domain AND draw children."""
+    w = gi.make_workload("C4", scale=13, n_edges=60_000, batch=256, n_batches=1)
+    k, qe, ql = gi.query(name)
+    ins, dele = w.batches[0]
+    probe = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0)
+    probe.set_query(k, qe, ql, gi.order(name))
+    probe.apply_batch(ins, dele)
+    st = probe.stats()
+    probe.close()
+    M = 2 * st["n1"] * st["max_degree"] ** (k - 4)
+    out = []
+    for lane in ("1", "0"):
+        monkeypatch.setenv("GCSM_WALK_LANE", lane)
+        g = G.Gcsm(w.n, w.row_ptr, w.col, None, device=0, seed=0xA11, walks_override=M)
+        g.set_query(k, qe, ql, gi.order(name))
+        g.set_cache_budget(w.adj_bytes // 100)
+        cnt = g.apply_batch(ins, dele)
+        _, ids, lev, st = product_estimate(g, w.n, k)
+        out.append((cnt, ids, lev[:, :k - 2], g.cached()))
+        g.close()
+    assert out[0][0] == out[1][0]
+    assert np.array_equal(out[0][1], out[1][1]) and np.array_equal(out[0][2], out[1][2])
+    assert np.array_equal(out[0][3], out[1][3])
+    assert out[0][2][:, k - 3].sum() > 0  # level k-2 records exist: level k-3 nodes drew children
 
 
 def test_degree_policy_cached_set(G):

@@ -162,3 +162,100 @@ def test_libgcsm_world2_gloo():
     for rank, got, mine, _ in res:
         assert got == want
     assert any(any(a or r for a, r in b) for b in res[0][2]) and any(any(a or r for a, r in b) for b in res[1][2])
+
+
+def _shared_worker(rank, world, port, out_q, pipelined):
+    """One rank of an emulated world on cuda:0 over ONE node-shared host store (gcsm_options.store_*): rank 0
+    builds the store from the CSR, the others attach by handle (no CSR of their own); per-rank shard counts are
+    summed over gloo; every rank exports G_{t+1} from the shared store at the end."""
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import gcsm_inputs as gi
+        import oracle
+        import paper_conf_ipps_wei024_b200 as G
+        torch.cuda.set_device(0)
+        w = gi.make_workload("C2", scale=12, n_edges=30_000, batch=256, n_batches=5)
+        queries = ["diamond", "k4", "house5u"]
+        if rank == 0:
+            g = G.Gcsm(w.n, w.row_ptr, w.col, device=0, rank=rank, world=world, local_counts=True,
+                       store_rank=0, store_world=world)
+            h = [g.store_handle()]
+        else:
+            h = [None]
+        dist.broadcast_object_list(h, src=0)
+        if rank > 0:
+            g = G.Gcsm(w.n, None, None, device=0, rank=rank, world=world, local_counts=True,
+                       store_rank=rank, store_world=world, store_handle=h[0])
+        dist.barrier()
+        for i, q in enumerate(queries):
+            k, qe, ql = gi.query(q)
+            (g.set_query if i == 0 else g.add_query)(k, qe, ql)
+        g.set_cache_budget(w.adj_bytes // 10)
+        mine = []
+
+        def collect():
+            g.wait_batch()
+            mine.append([g.query_counts(i) for i in range(len(queries))])
+
+        for b, (ins, dele) in enumerate(w.batches):
+            if pipelined:
+                g.submit_batch(ins, dele)
+                if b >= 1:
+                    collect()
+            else:
+                g.apply_batch(ins, dele)
+                mine.append([g.query_counts(i) for i in range(len(queries))])
+        if pipelined:
+            collect()
+        got = []
+        for c in mine:
+            t = torch.tensor(c, dtype=torch.int64)
+            dist.all_reduce(t)
+            got.append([tuple(x) for x in t.tolist()])
+        rp_f, col_f = g.export_csr()
+        dist.barrier()  # nobody unmaps the store before every rank exported it
+        g.close()
+        want = rp_w = col_w = None
+        if rank == 0:
+            want, rp, col = [], w.row_ptr, w.col
+            for ins, dele in w.batches:
+                want.append([oracle.delta(w.n, rp, col, None, *gi.query(q), ins, dele) for q in queries])
+                I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
+                rp, col = oracle.apply_batch(w.n, rp, col, I, D)
+            rp_w, col_w = rp, col
+        out_q.put((rank, got, mine, want, rp_f, col_f, rp_w, col_w))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world,pipelined", [(2, False), (3, True)])
+def test_shared_store_world_gloo(world, pipelined):
+    """Node-shared host store: R processes on cuda:0, ONE pinned store created by rank 0
+    and attached by the others; each rank writes the overlays / merges of the updated vertices it owns. Shard counts
+    summed over gloo equal the oracle on every batch and query, and every rank exports the oracle's final graph
+    from the shared store (so the owner-partitioned merges composed into G_{t+1})."""
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import __graft_entry__
+    __graft_entry__.build()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_shared_worker, args=(r, world, port, q, pipelined)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=600) for _ in range(world)], key=lambda x: x[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    want, rp_w, col_w = res[0][3], res[0][6], res[0][7]
+    for rank, got, mine, _, rp_f, col_f, _, _ in res:
+        assert got == want
+        assert np.array_equal(rp_f, rp_w) and np.array_equal(col_f, col_w)
+        assert any(any(a or r for a, r in b) for b in mine)
