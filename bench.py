@@ -75,6 +75,8 @@ def parse():
     ap.add_argument("--private-store", action="store_true",
                     help="N > 1: every rank builds its own pinned store (default: ONE node-shared store, rank 0 "
                          "builds it, the others attach; SURVEY 8e)")
+    ap.add_argument("--no-peer-cache", action="store_true",
+                    help="N > 1 with the shared store: do not link the ranks' HBM caches (gcsm_link_store_peers)")
     ap.add_argument("--serial", action="store_true",
                     help="synchronous apply_batch per step (default: pipelined submit/wait, so batch t+1's host "
                          "steps overlap batch t's kernels)")
@@ -426,6 +428,9 @@ def main():
         else:
             g.add_query(k, qe, ql, gi.order(q))
     g.set_cache_budget(budget)
+    peer_linked = shared_store and not args.no_peer_cache and budget > 0
+    if peer_linked:  # NEXT-3 across processes: misses probe the other GPUs' caches over NVLink before PCIe
+        g.link_store_peers()
     assert len(w.batches) >= steps + 1, "stream too short"
     batches = [(np.ascontiguousarray(a, dtype=np.int32), np.ascontiguousarray(b, dtype=np.int32))
                for a, b in w.batches[:steps + 1]]
@@ -502,7 +507,7 @@ def main():
             "ms_allreduce", "ms_merge", "hit_bytes", "miss_bytes", "delta_bytes", "hit_bytes_ext", "miss_bytes_ext",
             "delta_bytes_ext", "host_copied_bytes", "cache_bytes", "cached_vertices", "units", "frontier",
             "h2d_bytes", "d2h_bytes", "kernel_launches", "stage_fill_bytes", "stage_lists", "stage_hit_bytes",
-            "ms_walks", "walk_alg_bytes", "walk_fill_bytes")
+            "ms_walks", "walk_alg_bytes", "walk_fill_bytes", "peer_bytes")
     for step in recs:
         edges += step[0][3]["n_ins"] + step[0][3]["n_del"]
         for q, a, r, st in step:
@@ -641,10 +646,12 @@ def main():
                           "stage_fill_gb": d["stage_fill_bytes"] / K / 1e9,
                           "stage_hit_gb": d["stage_hit_bytes"] / K / 1e9,
                           "ms_walks": d["ms_walks"] / K, "walk_alg_gb": d["walk_alg_bytes"] / K / 1e9,
+                          "peer_gb": d["peer_bytes"] / K / 1e9,
                           "bcomp_miss_gb": None if bcomp is None else bcomp[q]["bcomp_miss_bytes"] / 1e9,
                           "bcomp_hit_gb": None if bcomp is None else bcomp[q]["bcomp_hit_bytes"] / 1e9,
                           "frontier": d["frontier"] / K} for q, d in per_q.items()},
         "gen_seconds": gen_s, "create_seconds": create_s,
+        "peer_cache": "linked (CUDA IPC, gcsm_link_store_peers)" if peer_linked else None,
         "host_store": "node-shared (one pinned store, rank 0 builds, ranks attach)" if shared_store else
                       ("private per rank" if world > 1 else "private"),
         "ranks_host": ranks_host,

@@ -174,6 +174,19 @@ void gcsm_default_options(gcsm_options *opt);
 gcsm_status gcsm_create(int32_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *labels,
                         const gcsm_options *opt, gcsm_ctx **out);
 
+/* Cross-process NVLink peer cache over a node-shared store: collective over the
+ * store's ranks, after gcsm_set_cache_budget and with no batch in flight. Every rank exports its two cache
+ * buffers, its two per-batch descriptor arrays and two interprocess events (CUDA IPC handles in its mailbox of the
+ * shared mapping) and opens every other rank's (peer access enabled lazily). From the next batch on, a list
+ * missing from this rank's cache is looked up in the peers' caches of the same batch (their descriptor array, one
+ * 16-byte read over NVLink per peer) before the staging arena and zero-copy; each batch adds one store barrier
+ * (every rank's cache step of batch t is enqueued), after which the matching waits (device) for the peers' cache
+ * steps. The cache buffers are then fixed: gcsm_set_cache_budget may lower the budget but a larger one is EINVAL.
+ * EINVAL without a shared store or with more than 7 peers; ESTATE before the
+ * budget, with a batch in flight or when already linked; EDEVICE if a handle cannot be opened (the store's other
+ * ranks then fail at their next barrier). */
+gcsm_status gcsm_link_store_peers(gcsm_ctx *ctx);
+
 /* Handle of a node-shared store (gcsm_options.store_world > 1) created by this context (store_rank 0): a
  * NUL-terminated path (the creating process's memfd under /proc) written to buf[cap]. The other local ranks
  * pass it as gcsm_options.store_handle while this process is alive. EINVAL for a private store or a buffer

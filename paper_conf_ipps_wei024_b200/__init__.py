@@ -97,6 +97,11 @@ class Gcsm:
         self.k = None
 
     # ------------------------------------------------------------------ API
+    def link_store_peers(self):
+        """Cross-process peer cache over the node-shared store (collective over the store's ranks; after
+        set_cache_budget): misses probe the other ranks' HBM caches (over NVLink) before zero-copy."""
+        self._check(self._lib.gcsm_link_store_peers(self._h), "link_store_peers")
+
     def store_handle(self) -> str:
         """The node-shared store's handle (store_rank 0 of a store_world > 1 context)."""
         buf = ctypes.create_string_buffer(4096)

@@ -22,7 +22,8 @@ SYMBOLS = ["gcsm_default_options", "gcsm_create", "gcsm_set_query", "gcsm_set_ca
            "gcsm_nccl_unique_id", "gcsm_get_stream", "gcsm_export_csr", "gcsm_get_estimates", "gcsm_get_cached",
            "gcsm_plan_inspect", "gcsm_query_restrictions", "gcsm_shard",
            "gcsm_measure_host_link", "gcsm_binomial_samples", "gcsm_set_measure",
-           "gcsm_num_vertices", "gcsm_add_vertices", "gcsm_link_peers", "gcsm_store_handle"]
+           "gcsm_num_vertices", "gcsm_add_vertices", "gcsm_link_peers", "gcsm_store_handle",
+           "gcsm_link_store_peers"]
 
 
 class Options(ctypes.Structure):
@@ -87,6 +88,7 @@ def load():
         "gcsm_set_measure": (st, [P, ctypes.c_uint32]),
         "gcsm_num_vertices": (I32, [P]),
         "gcsm_store_handle": (st, [P, P, U64]),
+        "gcsm_link_store_peers": (st, [P]),
         "gcsm_link_peers": (st, [P, I32]),
         "gcsm_add_vertices": (st, [P, I32, P, ctypes.POINTER(I32)]),
         "gcsm_query_restrictions": (st, [I32, I32, P, P, P, P, I32, P, ctypes.POINTER(U64)]),

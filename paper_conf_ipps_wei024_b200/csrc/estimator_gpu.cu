@@ -255,6 +255,16 @@ __device__ __forceinline__ bool has(const int32_t *a, uint32_t n, int32_t v) {
   return lo < n && a[lo] == v;
 }
 
+// One record of eq. (3)'s sums: B more reads of vertex w's list at tree level index li (R17). The touched bit is
+// checked through L2 first: the seed vertices of a unit are touched by every node below it, and an atomic to an
+// already-set word is a serialised round trip for nothing.
+__device__ __forceinline__ void rec(unsigned long long *levcnt, int levels, uint32_t *touched, int32_t w, int li,
+                                    unsigned long long B) {
+  atomicAdd(levcnt + (size_t)w * levels + li, B);
+  const uint32_t bit = 1u << (w & 31);
+  if (!(__ldcg(touched + (w >> 5)) & bit)) atomicOr(touched + (w >> 5), bit);
+}
+
 struct WalkArgs {
   const DevPlan *plans;
   const EstUnit *units;
@@ -280,8 +290,42 @@ struct WalkArgs {
   uint32_t stage_min;
   unsigned long long *stage_cnt;
   const char *dev_lo[2], *dev_hi[2];
+  const int32_t *sidx;          // sampled index of the host lists (nullptr: plain binary searches)
+  const uint32_t *soff;
   int32_t lane_leaf;            // level k-3 nodes one per lane (walk_leaf_parent; GCSM_WALK_LANE=0: warp-wide DFS)
 };
+
+// Membership of v in vertex w's main list m[0..ml): a list in the pinned host store is probed through its sampled
+// index in HBM (every 32nd element): a binary search over the samples, then ONE read of the 32-element
+// window that can hold v (8 x 16 B in flight) instead of log2(ml) dependent round trips over PCIe. Lists in device
+// memory (cache, the batch's U lists, the staging arena) are binary-searched in place.
+__device__ __forceinline__ bool probe(const WalkArgs &A, int32_t w, const int32_t *m, uint32_t ml, int32_t v) {
+  const char *pc = reinterpret_cast<const char *>(m);
+  const bool dev = (pc >= A.dev_lo[0] && pc < A.dev_hi[0]) || (pc >= A.dev_lo[1] && pc < A.dev_hi[1]) ||
+                   (A.stage.arena && m >= A.stage.arena && m < A.stage.arena + A.stage.cap);
+  if (dev || !A.sidx || ml < 64) return has(m, ml, v);
+  const uint32_t off = __ldg(A.soff + w);
+  if (off == 0xffffffffu) return has(m, ml, v);
+  const int32_t *smp = A.sidx + off;
+  uint32_t lo = 0, hi = (ml + 31) >> 5;  // first sample > v
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(smp + mid) <= v) lo = mid + 1;
+    else hi = mid;
+  }
+  if (lo == 0) return false;  // v < m[0]
+  const uint32_t base = 32u * (lo - 1), cnt = min(32u, ml - base);
+  const int4 *p4 = reinterpret_cast<const int4 *>(m + base);  // lists are 16-byte aligned, 32-element windows too
+  int4 q[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) q[i] = 4 * i < (int)cnt ? p4[i] : make_int4(INT_MIN, INT_MIN, INT_MIN, INT_MIN);
+  bool hit = false;
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+    hit |= (4 * i + 0 < (int)cnt && q[i].x == v) | (4 * i + 1 < (int)cnt && q[i].y == v) |
+           (4 * i + 2 < (int)cnt && q[i].z == v) | (4 * i + 3 < (int)cnt && q[i].w == v);
+  return hit;
+}
 
 constexpr int kEW = 8;  // warps per block
 struct EstLv {
@@ -299,13 +343,13 @@ struct EstLv {
 };
 struct EstW {
   int32_t f[GCSM_MAXK];
-  EstLv lv[GCSM_MAXK - 1];  // index = tree level 1..k-2
+  EstLv lv[GCSM_MAXK - 3];  // index = tree level - 2 (levels 2..k-2)
 };
 
 // Level 1 (phase A): warp per work item (a unit and kEstItem of its driver elements). The item at index 0 records
 // the level-1 node's reads; children with B' > 0 are recorded directly when they are the last sampled level (k = 4)
 // or appended to the level-2 node list (k >= 5) for k_walks.
-__global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
+__global__ void __launch_bounds__(kEW * 32) k_walks_l1(const __grid_constant__ WalkArgs A) {
   const BinTab T = A.T;
   const int lane = threadIdx.x & 31;
   for (;;) {
@@ -322,8 +366,7 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
     const int32_t f01[2] = {U.a, U.b};
     if (item.y == 0 && lane < nb) {
       const int32_t v = f01[Lp.bpos[lane]];
-      atomicAdd(A.levcnt + (size_t)v * A.levels, U.B);
-      atomicOr(A.touched + (v >> 5), 1u << (v & 31));
+      rec(A.levcnt, A.levels, A.touched, v, 0, U.B);
     }
     if (k <= 3) continue;  // level 1 is the last sampled level
     LR L[7];
@@ -340,16 +383,18 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
     const uint32_t end = min(best, (uint32_t)item.y + (uint32_t)kEstItem);
     const LevelPlan &L3 = P->lv[3];
     // emit one step's children: (k = 4) the reads of the level-2 nodes, (k >= 5) level-2 walk nodes
+    // emit one step's children (level-2 nodes): the reads they share (position 3's lists at the seeds, positions 0
+    // and 1) are recorded once per step with the children's summed B; (k = 4) each child records its own list
+    // (position 2), (k >= 5) the child becomes a root of k_walks, which records that one
     auto emit = [&](bool ok, int32_t v, unsigned long long Bc, unsigned long long ck) {
+      unsigned long long sumB = ok ? Bc : 0ull;
+#pragma unroll
+      for (int o = 16; o; o >>= 1) sumB += __shfl_xor_sync(FULL, sumB, o);
+      if (sumB && lane < L3.nb && L3.bpos[lane] < 2) rec(A.levcnt, A.levels, A.touched, L3.bpos[lane] ? U.b : U.a, 1, sumB);
       if (k == 4) {
-        if (ok) {
-          const int32_t f3[3] = {U.a, U.b, v};
-          for (int b = 0; b < L3.nb; ++b) {
-            const int32_t w = f3[L3.bpos[b]];
-            atomicAdd(A.levcnt + (size_t)w * A.levels + 1, Bc);
-            atomicOr(A.touched + (w >> 5), 1u << (w & 31));
-          }
-        }
+        if (ok)
+          for (int b = 0; b < L3.nb; ++b)
+            if (L3.bpos[b] == 2) rec(A.levcnt, A.levels, A.touched, v, 1, Bc);
       } else {
         const unsigned mask = __ballot_sync(FULL, ok);
         unsigned long long base = 0;
@@ -432,17 +477,17 @@ __global__ void __launch_bounds__(kEW * 32) k_walks_l1(const WalkArgs A) {
 // of the segment's stream: the same draws), and every surviving child (level k-2, whose children are leaves)
 // records its B' ~ Bin(B, 1/D) conditioned on >= 1 (d_binom_pos, the child's own key). Integer atomics: the sums
 // equal the warp-wide DFS's bit for bit. f[0..cl-1] are the matched positions, v the node's vertex at cl.
-__device__ __noinline__ void walk_leaf_parent(const WalkArgs &A, const DevPlan *P, const int32_t *f, int cl,
-                                              int32_t v, unsigned long long B, unsigned long long key,
-                                              unsigned long long &walg, unsigned long long &whit) {
+struct WalkBytes {
+  unsigned long long alg, hit;  // algorithmic list bytes read, bytes served by the staging arena
+};
+__device__ __noinline__ WalkBytes walk_leaf_parent(const WalkArgs &A, const DevPlan *P, const int32_t *f, int cl,
+                                                   int32_t v, unsigned long long B, unsigned long long key) {
+  unsigned long long walg = 0, whit = 0;
   const LevelPlan &Lq = P->lv[cl + 1];
   const int nb = Lq.nb;
   auto fat = [&](int p) { return p == cl ? v : f[p]; };
-  for (int b = 0; b < nb; ++b) {
-    const int32_t w = fat(Lq.bpos[b]);
-    atomicAdd(A.levcnt + (size_t)w * A.levels + (cl - 1), B);
-    atomicOr(A.touched + (w >> 5), 1u << (w & 31));
-  }
+  for (int b = 0; b < nb; ++b)  // its own list (the shared ones at positions < cl: the parent's step)
+    if (Lq.bpos[b] == cl) rec(A.levcnt, A.levels, A.touched, v, cl - 1, B);
   int drv = 0;
   LR D;
   uint32_t best = 0xffffffffu;
@@ -454,7 +499,7 @@ __device__ __noinline__ void walk_leaf_parent(const WalkArgs &A, const DevPlan *
       D = L;
     }
   }
-  if (best == 0) return;
+  if (best == 0) return WalkBytes{walg, whit};
   // staged copies (this batch's arena) of the main lists, where another reader already fetched them
   auto staged = [&](int32_t vb, const int32_t *m, uint32_t ml) -> const int32_t * {
     if (!A.stage.state || ml < A.stage_min) return m;
@@ -470,6 +515,7 @@ __device__ __noinline__ void walk_leaf_parent(const WalkArgs &A, const DevPlan *
   double pw[kSkipLog + 1];
   d_skip_table(r0, pw);
   const LevelPlan &Lc = P->lv[cl + 2];  // the children's next position (they record, R17)
+  unsigned long long sumB = 0;
   for (uint32_t s0 = 0; s0 < best; s0 += kSkipSeg) {
     const uint32_t s1 = min(best, s0 + kSkipSeg);
     const unsigned long long segkey = dchain(key, kSkipTag + s0 / kSkipSeg);
@@ -488,26 +534,38 @@ __device__ __noinline__ void walk_leaf_parent(const WalkArgs &A, const DevPlan *
         const int32_t vb = fat(Lq.bpos[b]);
         const LR Lb = view_of(A.vdesc, A.drec, A.dlist, vb, Lq.bview[b]);
         walg += 4ull * (Lb.ml + Lb.xl);
-        ok = has(staged(vb, Lb.m, Lb.ml), Lb.ml, c) || (Lb.xl && has(Lb.x, Lb.xl, c));
+        ok = probe(A, vb, staged(vb, Lb.m, Lb.ml), Lb.ml, c) || (Lb.xl && has(Lb.x, Lb.xl, c));
       }
       if (!ok) continue;
       const unsigned long long ck = dchain(key, (unsigned long long)(uint32_t)c);
       const unsigned long long Bc = (unsigned long long)d_binom_pos(ck, (int64_t)B, A.T.pD, r0);
-      for (int b = 0; b < Lc.nb; ++b) {
-        const int p = Lc.bpos[b];
-        const int32_t w = p == cl + 1 ? c : fat(p);
-        atomicAdd(A.levcnt + (size_t)w * A.levels + cl, Bc);
-        atomicOr(A.touched + (w >> 5), 1u << (w & 31));
-      }
+      sumB += Bc;
+      for (int b = 0; b < Lc.nb; ++b)
+        if (Lc.bpos[b] == cl + 1) rec(A.levcnt, A.levels, A.touched, c, cl, Bc);
     }
   }
+  if (sumB)  // the children's shared reads (positions <= cl), once
+    for (int b = 0; b < Lc.nb; ++b)
+      if (Lc.bpos[b] <= cl) rec(A.levcnt, A.levels, A.touched, fat(Lc.bpos[b]), cl, sumB);
+  return WalkBytes{walg, whit};
+}
+
+// A step's children (level l+1 nodes, B summed over the warp in sb) read the lists of position l+2 at positions
+// <= l together: one record per list for all of them (their own list, position l+1, each child records itself).
+__device__ __forceinline__ void rec_shared(const WalkArgs &A, const DevPlan *P, const int32_t *f, int l,
+                                           unsigned long long sb, int lane) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) sb += __shfl_xor_sync(FULL, sb, o);
+  if (!sb) return;
+  const LevelPlan &Lc = P->lv[l + 2];
+  if (lane < Lc.nb && Lc.bpos[lane] <= l) rec(A.levcnt, A.levels, A.touched, f[Lc.bpos[lane]], l, sb);
 }
 
 // Levels >= 2 (phase B, k >= 5): warp per level-2 node, DFS over the rest of its subtree.
 #ifndef GCSM_WALK_MINBLOCKS
 #define GCSM_WALK_MINBLOCKS 3  // resident 256-thread blocks per SM for k_walks (latency hiding of its list reads)
 #endif
-__global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const WalkArgs A) {
+__global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const __grid_constant__ WalkArgs A) {
   __shared__ EstW sw[kEW];
   const BinTab T = A.T;
   const int lane = threadIdx.x & 31;
@@ -544,23 +602,20 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
       W.f[0] = N.f0;
       W.f[1] = N.f1;
       W.f[2] = N.f2;
-      W.lv[2].B = N.B;
-      W.lv[2].key = N.key;
+      W.lv[0].B = N.B;
+      W.lv[0].key = N.key;
     }
     __syncwarp();
     int level = 2;
     bool fresh = true;
     while (level >= 2) {
-      EstLv &S = W.lv[level];
+      EstLv &S = W.lv[level - 2];
       const LevelPlan &Lp = P->lv[level + 1];
       const int nb = Lp.nb;
       if (fresh) {  // a node at `level` (positions 0..level matched) reads its next position's backward lists
         fresh = false;
-        if (lane < nb) {
-          const int32_t v = W.f[Lp.bpos[lane]];
-          atomicAdd(A.levcnt + (size_t)v * A.levels + (level - 1), S.B);
-          atomicOr(A.touched + (v >> 5), 1u << (v & 31));
-        }
+        if (lane < nb && Lp.bpos[lane] == level)  // the lists at positions < level: recorded by the parent's step
+          rec(A.levcnt, A.levels, A.touched, W.f[level], level - 1, S.B);
         if (level == k - 2) {  // its children are leaves: they read nothing (R17)
           --level;
           __syncwarp();
@@ -595,7 +650,9 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
             continue;
           const int32_t vb = W.f[Lp.bpos[b]];
           if (b == drv && stage_drv) {
-            L[b].m = stage_fetch(A.stage, vb, L[b].m, L[b].ml, wfill, wlists, whit, lane);
+            const StageRes r = stage_fetch(A.stage, vb, L[b].m, L[b].ml, lane);
+            stage_count(r, L[b].ml, wfill, wlists, whit);
+            L[b].m = r.p;
           } else {
             const unsigned long long st = stage_word(A.stage.state + vb);
             if ((st >> 40) == A.stage.epoch && (st & kStReady) && (st & kStOff) != kStOff) {
@@ -644,7 +701,11 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
         }
         if (__all_sync(FULL, fast)) {
           d_lane += ns;
-          if (lane < ns) walk_leaf_parent(A, P, W.f, level + 1, cv, cB, cK, walg, whit);
+          if (lane < ns) {
+            const WalkBytes wb = walk_leaf_parent(A, P, W.f, level + 1, cv, cB, cK);
+            walg += wb.alg;
+            whit += wb.hit;
+          }
           __syncwarp();
           if (lane == 0) S.si = ns;
           __syncwarp();
@@ -657,8 +718,8 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
         if (lane == 0) {
           S.si = si + 1;
           W.f[level + 1] = S.sv[si];
-          W.lv[level + 1].B = S.sB[si];
-          W.lv[level + 1].key = S.skey[si];
+          W.lv[level - 1].B = S.sB[si];
+          W.lv[level - 1].key = S.skey[si];
         }
         __syncwarp();
         ++level;
@@ -702,7 +763,7 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
             const LR Lb = view_of(A.vdesc, A.drec, A.dlist, W.f[Lp.bpos[b]], Lp.bview[b]);
             const int32_t *bm = S.pm[b];
             walg += 4ull * (Lb.ml + Lb.xl);
-            if (ok) ok = has(bm, Lb.ml, v) || (Lb.xl && has(Lb.x, Lb.xl, v));
+            if (ok) ok = probe(A, W.f[Lp.bpos[b]], bm, Lb.ml, v) || (Lb.xl && has(Lb.x, Lb.xl, v));
           }
         }
         unsigned long long Bc = 0, ck = 0;
@@ -718,6 +779,7 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
           S.sB[r] = Bc;
           S.skey[r] = ck;
         }
+        rec_shared(A, P, W.f, level, ok ? Bc : 0ull, lane);
         if (lane == 0) {
           S.ns = __popc(msk);
           S.si = 0;
@@ -765,7 +827,7 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
           walg += 4ull * (Lb.ml + Lb.xl);  // probed (binary search: an upper bound of the bytes it needs)
 #pragma unroll 1
           for (int j = 0; j < 4; ++j)
-            if (ok[j]) ok[j] = has(bm, Lb.ml, v[j]) || (Lb.xl && has(Lb.x, Lb.xl, v[j]));
+            if (ok[j]) ok[j] = probe(A, W.f[Lp.bpos[b]], bm, Lb.ml, v[j]) || (Lb.xl && has(Lb.x, Lb.xl, v[j]));
         }
       }
       // whole chunks while their survivors fit the 32-entry buffer (chunk 0 always does); the rest is redone
@@ -792,6 +854,13 @@ __global__ void __launch_bounds__(kEW * 32, GCSM_WALK_MINBLOCKS) k_walks(const W
           S.sB[r] = Bc[j];
           S.skey[r] = ck[j];
         }
+      {
+        unsigned long long sb = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          if (j < taken && ok[j]) sb += Bc[j];
+        rec_shared(A, P, W.f, level, sb, lane);
+      }
       if (lane == 0) {
         S.ns = tot;
         S.si = 0;
@@ -1281,6 +1350,8 @@ cudaError_t launch_cache_step(const CacheStep &c, cudaStream_t s, uint64_t *laun
       A.alg_cnt = c.alg_cnt[q];
       A.walk_stage = c.walk_stage;
       A.lane_leaf = c.walk_lane;
+      A.sidx = c.sidx;
+      A.soff = c.soff;
       for (int r = 0; r < 2; ++r) {
         A.dev_lo[r] = c.dev_lo[r];
         A.dev_hi[r] = c.dev_hi[r];

@@ -103,6 +103,8 @@ struct CacheStep {
   uint32_t stage_min = 1;
   unsigned long long *stage_cnt = nullptr;  // fill bytes, lists, hit bytes
   const char *dev_lo[2] = {nullptr, nullptr}, *dev_hi[2] = {nullptr, nullptr};
+  const int32_t *sidx = nullptr;  // sampled index of the host lists (every 32nd element) and per-vertex offsets
+  const uint32_t *soff = nullptr;
 };
 
 size_t cache_step_tmp_bytes(int32_t n);

@@ -83,6 +83,27 @@ struct PeerGroup {
   std::vector<uint64_t> enq;  // per member: batches whose cache step has been enqueued
 };
 
+// Cross-process peer cache over a node-shared store (gcsm_link_store_peers): what each rank publishes in its
+// mailbox of the shared mapping, and what it opened of the others'.
+struct PeerMail {
+  cudaIpcMemHandle_t cache[2], vdesc[2];
+  cudaIpcEventHandle_t ev[2];
+  uint64_t cache_va[2];
+  uint64_t cache_cap;
+  int32_t device, linked;
+  volatile int32_t cache_idx[2];  // per slot: the cache buffer (0 / 1) batch t's kernels read, -1 none
+};
+static_assert(sizeof(PeerMail) <= kShmMailBytes, "mailbox");
+struct StorePeers {
+  int n = 0;
+  int rank[GCSM_MAX_PEERS] = {};
+  void *vdesc[GCSM_MAX_PEERS][2] = {};
+  char *cache_map[GCSM_MAX_PEERS][2] = {};
+  uint64_t cache_va[GCSM_MAX_PEERS][2] = {};
+  uint64_t cache_cap[GCSM_MAX_PEERS] = {};
+  cudaEvent_t ev[GCSM_MAX_PEERS][2] = {};
+};
+
 }  // namespace
 
 struct gcsm_ctx {
@@ -253,6 +274,8 @@ struct gcsm_ctx {
   std::vector<int32_t> degree_order;  // GCSM_CACHE_DEGREE ranking
 
   std::shared_ptr<PeerGroup> peers;  // gcsm_link_peers
+  StorePeers sp;                      // gcsm_link_store_peers (other processes of the node-shared store)
+  cudaEvent_t ev_ipc[2] = {nullptr, nullptr};  // per slot: this batch's cache step is complete (interprocess)
   int peer_idx = -1;
   bool in_batch = false;  // between a successful normalise and the end of submit: failures poison the ctx
   gcsm_status fail(gcsm_status s, const std::string &m) {
@@ -275,6 +298,17 @@ struct gcsm_ctx {
 
 static void peer_leave(gcsm_ctx *ctx);
 
+static void store_peers_close(gcsm_ctx *ctx) {
+  StorePeers &sp = ctx->sp;
+  for (int p = 0; p < sp.n; ++p)
+    for (int j = 0; j < 2; ++j) {
+      if (sp.vdesc[p][j]) cudaIpcCloseMemHandle(sp.vdesc[p][j]);
+      if (sp.cache_map[p][j]) cudaIpcCloseMemHandle(sp.cache_map[p][j]);
+      if (sp.ev[p][j]) cudaEventDestroy(sp.ev[p][j]);
+    }
+  sp = StorePeers();
+}
+
 gcsm_ctx::~gcsm_ctx() {
   peer_leave(this);
   if (stream) cudaStreamSynchronize(stream);
@@ -283,6 +317,9 @@ gcsm_ctx::~gcsm_ctx() {
     for (DevPlan *p : {q.d_plans, q.d_splans})
       if (p) cudaFree(p);
   if (stream3) cudaStreamSynchronize(stream3);
+  store_peers_close(this);  // after this context's kernels (they may read the peers' memory) have finished
+  for (cudaEvent_t e : ev_ipc)
+    if (e) cudaEventDestroy(e);
   void *dev[] = {d_lab, d_scratch, d_red, d_cachebuf[0],
                  d_cachebuf[1], d_gather, d_pidx, d_pval, d_tup, d_hist, d_bsum, d_fresh, d_arena, d_tasks, d_task_ready};
   for (int q = 0; q < GCSM_MAX_QUERIES; ++q) {
@@ -517,6 +554,62 @@ gcsm_status gcsm_link_peers(gcsm_ctx *const *ctxs, int32_t n) {
   return GCSM_OK;
 }
 
+gcsm_status gcsm_link_store_peers(gcsm_ctx *ctx) {
+  if (!ctx) return GCSM_EINVAL;
+  if (ctx->poisoned) return GCSM_ESTATE;
+  HostStore &S = ctx->store;
+  if (!S.shared()) return ctx->fail(GCSM_EINVAL, "gcsm_link_store_peers needs a node-shared store");
+  if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "link with a batch in flight");
+  if (ctx->sp.n) return ctx->fail(GCSM_ESTATE, "already linked");
+  if (!ctx->d_cachebuf[0] || !ctx->d_cachebuf[1]) return ctx->fail(GCSM_ESTATE, "set the cache budget first");
+  if (S.store_world() - 1 > GCSM_MAX_PEERS) return ctx->fail(GCSM_EINVAL, "too many peers");
+  cudaSetDevice(ctx->device);
+  for (cudaEvent_t &e : ctx->ev_ipc)
+    if (!e) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming | cudaEventInterprocess));
+  PeerMail *me = reinterpret_cast<PeerMail *>(S.mailbox(S.store_rank()));
+  std::memset((void *)me, 0, sizeof *me);
+  for (int j = 0; j < 2; ++j) {
+    CK(cudaIpcGetMemHandle(&me->cache[j], ctx->d_cachebuf[j]));
+    CK(cudaIpcGetMemHandle(&me->vdesc[j], ctx->slots[j].d_vdesc));
+    CK(cudaIpcGetEventHandle(&me->ev[j], ctx->ev_ipc[j]));
+    me->cache_va[j] = (uint64_t)(uintptr_t)ctx->d_cachebuf[j];
+    me->cache_idx[j] = -1;
+  }
+  me->cache_cap = ctx->cache_cap;
+  me->device = ctx->device;
+  me->linked = 1;
+  if (!S.barrier()) return ctx->fail(GCSM_ESTATE, S.shared_err);
+  StorePeers sp;
+  bool ok = true;
+  for (int r = 0; r < S.store_world() && ok; ++r) {
+    if (r == S.store_rank()) continue;
+    const PeerMail *pm = reinterpret_cast<const PeerMail *>(S.mailbox(r));
+    if (!pm->linked) {
+      ok = false;
+      break;
+    }
+    const int p = sp.n++;
+    sp.rank[p] = r;
+    sp.cache_cap[p] = pm->cache_cap;
+    for (int j = 0; j < 2 && ok; ++j) {
+      sp.cache_va[p][j] = pm->cache_va[j];
+      ok = cudaIpcOpenMemHandle(&sp.vdesc[p][j], pm->vdesc[j], cudaIpcMemLazyEnablePeerAccess) == cudaSuccess &&
+           cudaIpcOpenMemHandle((void **)&sp.cache_map[p][j], pm->cache[j], cudaIpcMemLazyEnablePeerAccess) ==
+               cudaSuccess &&
+           cudaIpcOpenEventHandle(&sp.ev[p][j], pm->ev[j]) == cudaSuccess;
+    }
+  }
+  ctx->sp = sp;
+  if (!ok) {
+    cudaGetLastError();
+    store_peers_close(ctx);
+    S.poison_shared();
+    return ctx->fail(GCSM_EDEVICE, "opening a peer's IPC handles failed");
+  }
+  if (!S.barrier()) return ctx->fail(GCSM_ESTATE, S.shared_err);
+  return GCSM_OK;
+}
+
 gcsm_status gcsm_store_handle(const gcsm_ctx *ctx, char *buf, uint64_t cap) {
   if (!ctx || !buf || !ctx->store.shared() || ctx->store.store_rank() != 0) return GCSM_EINVAL;
   const std::string h = ctx->store.handle();
@@ -638,6 +731,8 @@ gcsm_status gcsm_set_cache_budget(gcsm_ctx *ctx, uint64_t bytes) {
   if (ctx->poisoned) return GCSM_ESTATE;
   if (ctx->waited != ctx->batch_seq) return ctx->fail(GCSM_ESTATE, "set_cache_budget with a batch in flight");
   bytes &= ~uint64_t(15);
+  if (ctx->sp.n && bytes > ctx->cache_cap)  // the peers hold IPC mappings of the current buffers
+    return ctx->fail(GCSM_EINVAL, "a store-peer-linked cache cannot grow");
   if (bytes > ctx->cache_cap) {
     for (char *&b : ctx->d_cachebuf) {
       if (b) cudaFree(b);
@@ -943,20 +1038,27 @@ static gcsm_status enqueue_gpu_cache(gcsm_ctx *ctx, gcsm_ctx::Slot &sl, cudaStre
   for (int qi = 0; qi < nq && qi < GCSM_MAX_QUERIES; ++qi) c.alg_cnt[qi] = sl.d_cnt + (size_t)qi * CNT_N + CNT_WALG;
   sl.walks_timed = est_on;
   c.walk_lane = ctx->walk_lane;
+  // device-resident lists at walk time (the last batch's cache, the batch's U lists): everything else a descriptor
+  // points to is the pinned host store, whose membership probes may use the sampled index (ctx->d_sidx)
+  c.dev_lo[0] = ctx->cache_valid ? ctx->d_cachebuf[ctx->cache_cur] : nullptr;
+  c.dev_hi[0] = c.dev_lo[0] ? c.dev_lo[0] + ctx->cache_cap : nullptr;
+  c.dev_lo[1] = reinterpret_cast<const char *>(sl.d_ulist);
+  c.dev_hi[1] = reinterpret_cast<const char *>(sl.d_ulist + sl.ulist_n);
+  if (!std::getenv("GCSM_NO_WALK_SIDX")) {
+    c.sidx = ctx->d_sidx;
+    c.soff = ctx->d_soff;
+  }
   if (ctx->walk_stage_epoch && !std::getenv("GCSM_NO_WALK_STAGE")) {  // the walks' zero-copy lists through the arena
     const gcsm_ctx::StageSlot &sg = ctx->stg[ctx->batch_seq & 1];
     c.stage = StageRef{sg.state, sg.arena, sg.cap, sg.bump, ctx->walk_stage_epoch};
     c.stage_min = ctx->stage_min;
     c.walk_stage = ctx->walk_stage;
     c.stage_cnt = sl.d_cnt + CNT_WFILL;  // query 0's block
-    c.dev_lo[0] = ctx->cache_valid ? ctx->d_cachebuf[ctx->cache_cur] : nullptr;  // lists cached by the last batch
-    c.dev_hi[0] = c.dev_lo[0] ? c.dev_lo[0] + ctx->cache_cap : nullptr;
-    c.dev_lo[1] = reinterpret_cast<const char *>(sl.d_ulist);  // the batch's U lists
-    c.dev_hi[1] = reinterpret_cast<const char *>(sl.d_ulist + sl.ulist_n);
   }
   CK(launch_cache_step(c, s, launches));
   ctx->est_valid = est_on;
   CK(cudaEventRecord(sl.ev_c1, s));
+  if (ctx->sp.n) CK(cudaEventRecord(ctx->ev_ipc[ctx->batch_seq & 1], s));  // store peers wait on it
   return GCSM_OK;
 }
 
@@ -1577,6 +1679,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   if (nd) CK(cudaMemcpyAsync(sl.d_dlist, sl.h_dlist, 4 * nd, cudaMemcpyHostToDevice, s));
   if (gnu) CK(cudaMemcpyAsync(sl.d_units, sl.h_units, sizeof(Unit) * (size_t)gnu, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(sl.ev_c1, s));
+  if (ctx->sp.n) CK(cudaEventRecord(ctx->ev_ipc[ctx->batch_seq & 1], s));
   st.h2d_bytes = new_bytes + 8 * gather.size() + 8 * fresh.size() + (sizeof(int64_t) + sizeof(VDesc)) * dirty.size() + sizeof(DRec) * nU +
                  4 * nd + sizeof(Unit) * (size_t)gnu;
   CK(cudaMemsetAsync(sl.d_cnt, 0, sizeof(unsigned long long) * CNT_N * (size_t)nq, s));
@@ -1603,6 +1706,35 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
         CK(cudaStreamWaitEvent(s, p->slots[ctx->batch_seq & 1].ev_c1, 0));
         peer_of[npeer++] = p;
       }
+  }
+
+  // cross-process peers (node-shared store): publish which cache buffer this batch reads, meet every rank (each
+  // has recorded its cache step of batch t), then this context's matching waits (device) for theirs. Slot reuse is
+  // safe: a rank rewrites slot t & 1 (batch t+2) only after the store's entry barrier of t+2, which every rank
+  // passes only after collecting batch t
+  int snpeer = 0;
+  const char *sp_lo[GCSM_MAX_PEERS] = {}, *sp_hi[GCSM_MAX_PEERS] = {}, *sp_map[GCSM_MAX_PEERS] = {};
+  const VDesc *sp_vd[GCSM_MAX_PEERS] = {};
+  if (ctx->sp.n && !ctx->peers) {
+    const int slot = (int)(ctx->batch_seq & 1);
+    PeerMail *me = reinterpret_cast<PeerMail *>(S.mailbox(S.store_rank()));
+    me->cache_idx[slot] = !ctx->d_cache ? -1 : (ctx->d_cache == ctx->d_cachebuf[0] ? 0 : 1);
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    if (!S.barrier()) {
+      ctx->poisoned = true;
+      return ctx->fail(GCSM_ESTATE, S.shared_err);
+    }
+    for (int p = 0; p < ctx->sp.n && npeer + snpeer < GCSM_MAX_PEERS; ++p) {
+      const PeerMail *pm = reinterpret_cast<const PeerMail *>(S.mailbox(ctx->sp.rank[p]));
+      const int ci = pm->cache_idx[slot];
+      if (ci < 0) continue;
+      CK(cudaStreamWaitEvent(s, ctx->sp.ev[p][slot], 0));
+      sp_vd[snpeer] = reinterpret_cast<const VDesc *>(ctx->sp.vdesc[p][slot]);
+      sp_lo[snpeer] = reinterpret_cast<const char *>(ctx->sp.cache_va[p][ci]);
+      sp_hi[snpeer] = sp_lo[snpeer] + ctx->sp.cache_cap[p];
+      sp_map[snpeer] = ctx->sp.cache_map[p][ci];
+      ++snpeer;
+    }
   }
 
   // ---- (4) matching kernels (per query, in registration order, on the context stream) ---------------------
@@ -1691,12 +1823,20 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.stage_policy = ctx->stage_policy;
   A.filter3 = std::getenv("GCSM_NO_FILTER3") ? 0 : 1;
   A.hoist = std::getenv("GCSM_NO_HOIST") ? 0 : 1;
-  A.npeer = npeer;
-  for (int p = 0; p < npeer; ++p) {
+  A.fsplit = std::getenv("GCSM_NO_FSPLIT") ? 0 : 1;
+  A.npeer = npeer + snpeer;
+  for (int p = 0; p < npeer; ++p) {  // same process: the peer's addresses are ours
     const gcsm_ctx::Slot &ps = peer_of[p]->slots[ctx->batch_seq & 1];
     A.peer_vdesc[p] = ps.d_vdesc;
     A.peer_lo[p] = ps.cache_lo;
     A.peer_hi[p] = ps.cache_hi;
+    A.peer_map[p] = ps.cache_lo;
+  }
+  for (int p = 0; p < snpeer; ++p) {  // other processes: their cache addresses are translated into our mapping
+    A.peer_vdesc[npeer + p] = sp_vd[p];
+    A.peer_lo[npeer + p] = sp_lo[p];
+    A.peer_hi[npeer + p] = sp_hi[p];
+    A.peer_map[npeer + p] = sp_map[p];
   }
   if (kmax >= 5 && !listing) {  // level-3 work sharing buffers (64M-int arena, 4M tasks)
     const size_t na = (size_t)64 << 20, nt = (size_t)4 << 20;
@@ -1942,6 +2082,10 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
                    "entries=%llu pruned=%llu l3=%llu l3kept=%llu l4=%llu last_drv=%llu\n",
                    qi, h[CNT_F2], h[CNT_DBG_RUNS], h[CNT_DBG_PINS], h[CNT_DBG_PINBYTES] / 1e9, h[CNT_DBG_SPLIT] / 1e9,
                    h[CNT_COPIED] / 1e9, h[CNT_X_ENTRIES], h[CNT_X_PRUNED], h[CNT_X_L3], h[CNT_X_L3F], h[CNT_X_L4], h[CNT_X_LAST]);
+    if (std::getenv("GCSM_TRACE"))
+      std::fprintf(stderr, "[gcsm ext-time] q=%d warps=%d ph1_mean_ms=%.2f ph1_max_ms=%.2f warp_max_ms=%.2f entry_max_ms=%.3f\n",
+                   qi, ctx->warps_total, h[CNT_XT] / (double)ctx->warps_total / 1.965e6, h[CNT_XT + 1] / 1.965e6,
+                   h[CNT_XT + 2] / 1.965e6, h[CNT_XT + 3] / 1.965e6);
     if (std::getenv("GCSM_TRACE"))
       std::fprintf(stderr, "[gcsm walks] q=%d roots=%llu lane_nodes=%llu dfs_descents=%llu steps=%llu walg_gb=%.3f\n", qi,
                    h[CNT_WDBG], h[CNT_WDBG + 1], h[CNT_WDBG + 2], h[CNT_WDBG + 3], h[CNT_WALG] / 1e9);

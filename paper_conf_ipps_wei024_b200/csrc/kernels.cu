@@ -76,6 +76,16 @@ constexpr int kChunk = GCSM_EXT_CHUNK;  // frontier entries per k_extend work gr
 #define GCSM_TASK_SIZE 2
 #endif
 constexpr uint32_t kSplitMin = GCSM_SPLIT_MIN;  // level-3 sets larger than this are shared as tasks (k >= 5)
+#ifndef GCSM_FSPLIT_MIN
+#define GCSM_FSPLIT_MIN 64
+#endif
+#ifndef GCSM_FTASK_SIZE
+#define GCSM_FTASK_SIZE 32
+#endif
+// level-3 sets larger than kFSplitMin are shared BEFORE the level-3 filter, in slices of kFTaskSize nodes that the
+// takers filter themselves (the filter, one lane per node, is the heavy part of a hub entry)
+constexpr uint32_t kFSplitMin = GCSM_FSPLIT_MIN, kFTaskSize = GCSM_FTASK_SIZE;
+constexpr uint32_t kTaskFilter = 0xffffffffu;  // Task::pad: the slice is unfiltered
 constexpr uint32_t kTaskSize = GCSM_TASK_SIZE;  // level-3 candidates per task
 
 struct LRef {
@@ -86,10 +96,24 @@ struct LRef {
   bool dev;          // main list is in device memory (HBM cache, a staged copy, or shared memory)
 };
 
+// Per-warp accumulators: the counts in registers; the byte statistics (warp-uniform values, updated by lane 0)
+// in a per-warp block of shared memory, so that they cost no registers in the register-bound kernels.
+enum : int { kSHit, kSMiss, kSDelta, kSCopied, kSFill, kSLists, kSSHit, kSPeer, kSN };
 struct Acc {
-  unsigned long long add = 0, rem = 0, hit = 0, miss = 0, delta = 0, copied = 0;
-  unsigned long long sfill = 0, slists = 0, shit = 0;  // fetch-once staging: bytes filled, lists, bytes served
-  unsigned long long peer = 0;                         // bytes read from a linked peer's HBM cache
+  unsigned long long add = 0, rem = 0;
+  unsigned long long *s = nullptr;  // kSN counters (shared memory, this warp's)
+  bool l0 = false;
+  __device__ __forceinline__ void init(unsigned long long *blk, int lane) {
+    s = blk;
+    l0 = lane == 0;
+    __syncwarp();
+    if (l0)
+      for (int i = 0; i < kSN; ++i) s[i] = 0;
+    __syncwarp();
+  }
+  __device__ __forceinline__ void stat(int i, unsigned long long v) {
+    if (l0) s[i] += v;
+  }
 };
 
 // NVLink peer cache (NEXT-3): vertex v's main list in a linked peer's HBM cache for this batch, or nullptr. The
@@ -102,16 +126,22 @@ __device__ __forceinline__ const int32_t *peer_lookup(const MatchArgs &A, int32_
     const char *q = reinterpret_cast<const char *>((unsigned long long)(unsigned)raw.x |
                                                    ((unsigned long long)(unsigned)raw.y << 32));
     if (q >= A.peer_lo[p] && q < A.peer_hi[p] && (uint32_t)raw.z == ml && raw.w == 0)
-      return reinterpret_cast<const int32_t *>(q);
+      return reinterpret_cast<const int32_t *>(A.peer_map[p] + (q - A.peer_lo[p]));
   }
   return nullptr;
 }
 
-__device__ __noinline__ const int32_t *stage_resolve(const MatchArgs &A, int32_t v, const int32_t *hp, uint32_t ml,
-                                                     unsigned long long &sfill, unsigned long long &slists,
-                                                     unsigned long long &shit, int lane) {
+__device__ __forceinline__ const int32_t *stage_resolve(const MatchArgs &A, int32_t v, const int32_t *hp, uint32_t ml,
+                                                        Acc &acc, int lane) {
   const StageRef R{A.stage_state, A.stage_arena, A.stage_cap, A.stage_bump, A.stage_epoch};
-  return stage_fetch(R, v, hp, ml, sfill, slists, shit, lane);
+  const StageRes r = stage_fetch(R, v, hp, ml, lane);
+  if (r.how == kStFilled) {
+    acc.stat(kSFill, 4ull * ml);
+    acc.stat(kSLists, 1);
+  } else if (r.how == kStServed) {
+    acc.stat(kSSHit, 4ull * ml);
+  }
+  return r.p;
 }
 
 __device__ __forceinline__ void mark_touched(const MatchArgs &A, int32_t v) {
@@ -151,10 +181,10 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
   const char *p = reinterpret_cast<const char *>(r.m);
   const bool in_cache = p >= A.cache_lo && p < A.cache_hi, in_ubuf = p >= A.ubuf_lo && p < A.ubuf_hi;
   r.dev = in_cache || in_ubuf;
-  if (in_cache) acc.hit += 4ull * r.ml;
-  else if (in_ubuf) acc.delta += 4ull * r.ml;  // the batch's uploaded stable lists of U (device-resident deltas)
-  else acc.miss += 4ull * r.ml;
-  acc.delta += 4ull * r.xl;
+  if (in_cache) acc.stat(kSHit, 4ull * r.ml);
+  else if (in_ubuf) acc.stat(kSDelta, 4ull * r.ml);  // the batch's uploaded stable lists of U (device-resident deltas)
+  else acc.stat(kSMiss, 4ull * r.ml);
+  acc.stat(kSDelta, 4ull * r.xl);
   if (lane == 0) mark_touched(A, v);
   if (v == pin.v) {  // served from this warp's staged copy
     r.m = pin.p;
@@ -164,11 +194,11 @@ __device__ __forceinline__ LRef list_of(const MatchArgs &A, int32_t v, int view,
     if (q) {
       r.m = q;
       r.dev = true;
-      acc.peer += 4ull * r.ml;
+      acc.stat(kSPeer, 4ull * r.ml);
     }
   }
   if (!r.dev && A.stage_state && r.ml >= A.stage_min) {  // fetched once per batch into HBM
-    r.m = stage_resolve(A, v, r.m, r.ml, acc.sfill, acc.slists, acc.shit, lane);
+    r.m = stage_resolve(A, v, r.m, r.ml, acc, lane);
     r.dev = reinterpret_cast<const char *>(r.m) != p;
   }
   return r;
@@ -264,7 +294,7 @@ __device__ GCSM_COLD void stage_lists(const MatchArgs &A, LRef *L, int nl, int d
     }
     if (!stage) continue;
     const uint32_t n4 = (n + 3) & ~3u;
-    if (!hit) acc.copied += 4ull * n;
+    if (!hit) acc.stat(kSCopied, 4ull * n);
     if (sm_used + n4 <= sm_cap) {
       warp_copy(sm + sm_used, L[p].m, n, lane);
       L[p].m = sm + sm_used;
@@ -480,30 +510,30 @@ __device__ __forceinline__ void emit_tuples(const MatchArgs &A, const DevPlan &P
 }
 
 __device__ __forceinline__ void flush(const MatchArgs &A, const Acc &acc, int lane) {
+  __syncwarp();
   if (lane == 0) {
     if (acc.add) atomicAdd(&A.cnt[CNT_ADDED], acc.add);
     if (acc.rem) atomicAdd(&A.cnt[CNT_REMOVED], acc.rem);
-    if (acc.hit) atomicAdd(&A.cnt[A.acc_base + 0], acc.hit);
-    if (acc.miss) atomicAdd(&A.cnt[A.acc_base + 1], acc.miss);
-    if (acc.delta) atomicAdd(&A.cnt[A.acc_base + 2], acc.delta);
-    if (acc.copied) atomicAdd(&A.cnt[CNT_COPIED], acc.copied);
-    if (acc.sfill) atomicAdd(&A.cnt[CNT_STAGE_FILL], acc.sfill);
-    if (acc.slists) atomicAdd(&A.cnt[CNT_STAGE_LISTS], acc.slists);
-    if (acc.shit) atomicAdd(&A.cnt[CNT_STAGE_HIT], acc.shit);
-    if (acc.peer) atomicAdd(&A.cnt[CNT_PEER], acc.peer);
+    const int dst[kSN] = {A.acc_base + 0, A.acc_base + 1, A.acc_base + 2, CNT_COPIED, CNT_STAGE_FILL,
+                          CNT_STAGE_LISTS, CNT_STAGE_HIT, CNT_PEER};
+#pragma unroll
+    for (int i = 0; i < kSN; ++i)
+      if (acc.s[i]) atomicAdd(&A.cnt[dst[i]], acc.s[i]);
   }
 }
 
 // Level 2 (BFS step): warp per unit.
 template <bool LIST>
-__global__ void __launch_bounds__(kBlock, 4) k_level2(const MatchArgs A) {
+__global__ void __launch_bounds__(kBlock, 4) k_level2(const __grid_constant__ MatchArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int32_t *buf = A.scratch + gw * A.scratch_stride;
   int32_t *gstage = buf + A.scratch_stride - 2 * (int64_t)A.dcap;
   extern __shared__ int4 smem_raw[];
   int32_t *sm = reinterpret_cast<int32_t *>(smem_raw) + (threadIdx.x >> 5) * kSmemInts;
+  __shared__ unsigned long long s_stats[kWarps][kSN];
   Acc acc;
+  acc.init(s_stats[threadIdx.x >> 5], lane);
   for (;;) {
     unsigned long long u = 0;
     if (lane == 0) u = atomicAdd(&A.cnt[CNT_CURSOR0], 1ull);
@@ -581,14 +611,19 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
 }
 
 // Level-3 filter (LevelPlan::fmask): position 4's candidates for a level-3 node x3 lie in
-// F ∩ view(N(x3)), where F (sorted, label-filtered) is the intersection of position 4's lists fixed for the whole
+// F ∩ view(N(x3)), where F = F[0..nF1) ∪ F2[0..nF-nF1) (two sorted runs, label-filtered) is the intersection of position 4's lists fixed for the whole
 // level-2 entry. Lane i tests node i: does its own list meet F? Nodes that cannot (almost all of them on C4) are
 // dropped from the level-3 set before the warp-wide DFS visits them; the test ignores injectivity and symmetry
 // ranges, so it only ever keeps too much (exact). Survivors go to out (may be set3 itself: compaction in place);
 // returns their number.
+// The byte counters go out through facc[6] (hit, miss, delta, staged, peer, filled) and fl[1] (lists filled): the
+// warp's shared DFS record, so that the caller's Acc is never address-taken.
 __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const int32_t *set3, uint32_t n3,
-                                               int32_t *out, const int32_t *F, uint32_t nF1, uint32_t nF, Acc &acc,
-                                               int lane) {
+                                               int32_t *out, const int32_t *F, const int32_t *F2, uint32_t nF1,
+                                               uint32_t nF, unsigned long long *stats, int lane) {
+  Acc acc;  // statistics only: the caller's warp block
+  acc.s = stats;
+  acc.l0 = lane == 0;
   uint32_t w = 0;
   unsigned long long hb = 0, mb = 0, db = 0, sb = 0, pb = 0;  // per-lane algorithmic bytes: hit, miss, delta, staged, peer
   for (uint32_t base = 0; base < n3; base += 32) {
@@ -639,19 +674,20 @@ __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const
       const int32_t vl = __shfl_sync(kFull, v, l);
       const unsigned long long hp = __shfl_sync(kFull, (unsigned long long)m, l);
       const uint32_t mll = __shfl_sync(kFull, ml, l);
-      const int32_t *q = stage_resolve(A, vl, reinterpret_cast<const int32_t *>(hp), mll, acc.sfill, acc.slists,
-                                       acc.shit, lane);
+      const int32_t *q = stage_resolve(A, vl, reinterpret_cast<const int32_t *>(hp), mll, acc, lane);
       if (lane == l) m = q;
     }
     bool hit = false;
     if (act) {
       if (ml + xl <= nF) {  // stream the node's list, probe F (its two sorted runs)
-        const int32_t *F2 = F + nF1;
         const uint32_t nF2 = nF - nF1;
         for (uint32_t j = 0; j < ml && !hit; ++j) hit = bsearch_has(F, nF1, m[j]) || (nF2 && bsearch_has(F2, nF2, m[j]));
         for (uint32_t j = 0; j < xl && !hit; ++j) hit = bsearch_has(F, nF1, x[j]) || (nF2 && bsearch_has(F2, nF2, x[j]));
       } else {  // stream F, probe the node's list
-        for (uint32_t j = 0; j < nF && !hit; ++j) hit = bsearch_has(m, ml, F[j]) || (xl && bsearch_has(x, xl, F[j]));
+        for (uint32_t j = 0; j < nF && !hit; ++j) {
+          const int32_t fj = j < nF1 ? F[j] : F2[j - nF1];
+          hit = bsearch_has(m, ml, fj) || (xl && bsearch_has(x, xl, fj));
+        }
       }
     }
     const unsigned hm = __ballot_sync(kFull, hit);
@@ -659,11 +695,12 @@ __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const
     w += __popc(hm);
     __syncwarp();
   }
-  acc.hit += warp_sum64(hb);
-  acc.miss += warp_sum64(mb);
-  acc.delta += warp_sum64(db);
-  acc.shit += warp_sum64(sb);
-  acc.peer += warp_sum64(pb);
+  acc.stat(kSHit, warp_sum64(hb));
+  acc.stat(kSMiss, warp_sum64(mb));
+  acc.stat(kSDelta, warp_sum64(db));
+  acc.stat(kSSHit, warp_sum64(sb));
+  acc.stat(kSPeer, warp_sum64(pb));
+  __syncwarp();
   return w;
 }
 
@@ -677,12 +714,13 @@ struct WarpDfs {
   uint32_t sz[GCSM_MAXK], it[GCSM_MAXK];
   LRef L[7], Lx[7];
   int32_t excl[GCSM_MAXK];
+  unsigned long long stats[kSN];  // this warp's byte statistics (Acc)
 };
 constexpr int kExtSmemBytes = kSmemBytes + kWarps * (int)sizeof(WarpDfs);
 
 // Levels 3..k-1 (DFS): warp per level-2 frontier entry.
 template <bool LIST, int KK>  // KK: compile-time query size (4: the level-3 count only), 0 = any
-__global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchArgs A) {
+__global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_constant__ MatchArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int32_t *stack = A.scratch + gw * A.scratch_stride;  // buffer for position p: stack + (p - 3) * dcap
@@ -709,12 +747,15 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const int64_t chunk = max((int64_t)1, min((int64_t)kChunk, n_f2 / (4 * warps)));
   Acc acc;
+  acc.init(Wd.stats, lane);
   Pinned pin;
   unsigned long long x_entries = 0, x_pruned = 0, x_l3 = 0, x_l4 = 0, x_last = 0, x_l3f = 0;  // work profile
   uint32_t pin_sm = 0;  // ints of the shared slice held by the pinned x2 list
   int64_t ci = 0, c_end = 0, c_start = 0;
   bool producing = true;  // phase 1: walk the (grouped) frontier; phase 2 (k >= 5): take shared level-3 tasks
   const bool sharing = KK == 0 && !LIST && k >= 5 && A.tasks != nullptr;
+  const long long t_start = clock64();
+  long long t_ph1 = 0, t_entry = 0, t_emax = 0;  // timing profile (CNT_XT)
   for (;;) {
     int64_t e;
     bool task = false;
@@ -729,6 +770,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           atomicAdd(&A.cnt[CNT_PRODUCERS], (unsigned long long)(c_end - c_start));
         }
         if ((int64_t)c0 >= n_f2) {
+          t_ph1 = clock64() - t_start;
           if (!sharing) break;
           producing = false;
           pin.v = -1;
@@ -769,7 +811,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           }
         }
         if (miss && A.stage_state && ml >= A.stage_min) {  // the run's x2 list, fetched once per batch
-          const int32_t *sp = stage_resolve(A, x2, mp, ml, acc.sfill, acc.slists, acc.shit, lane);
+          const int32_t *sp = stage_resolve(A, x2, mp, ml, acc, lane);
           if (sp != mp) {
             mp = sp;
             miss = false;
@@ -781,14 +823,14 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
         pin.bm_v = -1;
         if (run >= 2 && ml >= 32 && ml4 <= GCSM_PIN_SMEM_MAX) {  // fits the shared slice: pin hits and misses
           warp_copy(sm, mp, ml, lane);
-          if (miss) acc.copied += 4ull * ml;
+          if (miss) acc.stat(kSCopied, 4ull * ml);
           __syncwarp();
           pin.v = x2;
           pin.p = sm;
           pin_sm = ml4;
         } else if (run >= 2 && ml >= 32 && miss && ml <= (uint32_t)A.dcap) {
           warp_copy(pstage, mp, ml, lane);
-          acc.copied += 4ull * ml;
+          acc.stat(kSCopied, 4ull * ml);
           __syncwarp();
           pin.v = x2;
           pin.p = pstage;
@@ -835,13 +877,19 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
       // never from a possibly stale L1 line
       {
         const unsigned long long *src = reinterpret_cast<const unsigned long long *>(&A.tasks[h]);
-        unsigned long long w[4];
+        unsigned long long w[7];
 #pragma unroll
-        for (int i = 0; i < 4; ++i) w[i] = __ldcg(src + i);
+        for (int i = 0; i < 7; ++i) w[i] = __ldcg(src + i);
         memcpy(&tk, w, sizeof(Task));
       }
+      if (tk.lo >= tk.hi) continue;  // an empty placeholder (its producer kept the work)
       e = tk.e;
       task = true;
+    }
+    {
+      const long long now = clock64();
+      if (t_entry) t_emax = max(t_emax, now - t_entry);
+      t_entry = now;
     }
     const int32_t ui = f2u[e];
     const Unit U = A.units[ui];
@@ -860,7 +908,13 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     // hoisted last-level set (LevelPlan::hmask): ∩ of the last position's lists fixed at level 2, label-filtered
     const int32_t *hset = nullptr;
     uint32_t hn = 0;
-    if (KK == 0 && P.lv[k - 1].hmask && A.hoist) {
+    if (task && tk.xoff != ~0ull) {  // H and F as the producer computed them (L2 reads: written in this launch)
+      hn = tk.hn;
+      for (uint32_t i = lane; i < hn; i += 32) hbuf[i] = __ldcg(A.arena + tk.xoff + i);
+      for (uint32_t i = lane; i < tk.nF; i += 32) fbuf[i] = __ldcg(A.arena + tk.xoff + hn + i);
+      __syncwarp();
+      if (KK == 0 && P.lv[k - 1].hmask && A.hoist) hset = hbuf;
+    } else if (KK == 0 && P.lv[k - 1].hmask && A.hoist) {
       const LevelPlan &Lh = P.lv[k - 1];
       LRef *const Lx = Wd.Lx;
       int nx = 0, hdrv = 0;
@@ -875,19 +929,28 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           }
           ++nx;
         }
-      hn = warp_isect<true>(A, nullptr, 0, Lx, nx, hdrv, nullptr, 0, Lh.label, hbuf, lane);
-      __syncwarp();
-      hset = hbuf;
+      if (nx == 1 && Lh.label < 0 && Lx[0].dev && Lx[0].xl == 0) {  // one device-resident run: referenced
+        hset = Lx[0].m;
+        hn = Lx[0].ml;
+      } else {
+        hn = warp_isect<true>(A, nullptr, 0, Lx, nx, hdrv, nullptr, 0, Lh.label, hbuf, lane);
+        __syncwarp();
+        hset = hbuf;
+      }
       if (hn == 0) {  // no candidate for the last position anywhere below this entry
         ++x_pruned;
         continue;
       }
     }
     // level-3 filter set F (LevelPlan::fmask): ∩ of position 4's lists fixed for this entry, label-filtered
-    uint32_t nF = 0, nF1 = 0;  // F = fset[0..nF1) ∪ fset[nF1..nF), two sorted runs
-    const int32_t *fset = fbuf;
+    uint32_t nF = 0, nF1 = 0;  // F = fset[0..nF1) ∪ fset2[0..nF-nF1), two sorted runs
+    const int32_t *fset = fbuf, *fset2 = fbuf;
     const bool filt = KK == 0 && k >= 5 && P.lv[4].fmask != 0 && A.filter3;
-    if (filt) {
+    if (filt && task && tk.xoff != ~0ull) {
+      nF1 = tk.nF1;
+      nF = tk.nF;
+      fset2 = fbuf + nF1;
+    } else if (filt) {
       const LevelPlan &L4 = P.lv[4];
       LRef *const Lx = Wd.Lx;
       int nx = 0, fdrv = 0;
@@ -905,16 +968,24 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
       // F as two sorted runs: survivors of the driver's main run, then of its delta run (an updated vertex's
       // view is main ∪ delta, each sorted, not sorted together); the filter binary-searches each run
       const LRef dfull = Lx[fdrv];
+      if (nx == 1 && L4.label < 0 && dfull.dev) {  // F is one device-resident view: referenced, not copied
+        fset = dfull.m;
+        nF1 = dfull.ml;
+        fset2 = dfull.x;
+        nF = dfull.ml + dfull.xl;
+      } else {
       Lx[fdrv].xl = 0;
       nF1 = warp_isect<true>(A, nullptr, 0, Lx, nx, fdrv, nullptr, 0, L4.label, fbuf, lane);
       __syncwarp();
       nF = nF1;
+      fset2 = fbuf + nF1;
       if (dfull.xl) {
         Lx[fdrv].m = dfull.x;
         Lx[fdrv].ml = dfull.xl;
         Lx[fdrv].dev = true;
         nF += warp_isect<true>(A, nullptr, 0, Lx, nx, fdrv, nullptr, 0, L4.label, fbuf + nF1, lane);
         __syncwarp();
+      }
       }
       if (nF == 0) {  // no position-4 candidate for any level-3 node of this entry
         ++x_pruned;
@@ -927,7 +998,24 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
     uint32_t it3n = 0;
     bool reuse3 = false;
     for (int q = 4; q < k; ++q) reuse3 |= P.lv[q].reuse == 3;
-    if (task) {
+    if (task && tk.pad == kTaskFilter) {
+      // an unfiltered slice: copy it (or the whole set when a later position reuses it), filter it here
+      int32_t *own = stack;
+      const uint32_t lo = reuse3 ? 0 : tk.lo, cnt = reuse3 ? tk.n : tk.hi - tk.lo;
+      for (uint32_t i = lane; i < cnt; i += 32) own[i] = __ldcg(A.arena + tk.off + lo + i);
+      __syncwarp();
+      const int32_t *slice = reuse3 ? own + tk.lo : own;
+      it3n = filter_level3(A, P.lv[4].bview[P.lv[4].f3], slice, tk.hi - tk.lo, ibuf, fset, fset2, nF1, nF, acc.s, lane);
+      x_l3f += it3n;
+      it3p = ibuf;
+      __syncwarp();
+      set[3] = own;
+      sz[3] = cnt;
+      it[3] = 0;
+      end3 = it3n;
+      lvl = 3;
+      descend = false;
+    } else if (task) {
       int32_t *own = stack;  // this warp's level-3 buffer: a private, L1-safe copy of the shared set
       for (uint32_t i = lane; i < tk.n; i += 32) own[i] = __ldcg(A.arena + tk.off + i);
       it3p = own;
@@ -1012,10 +1100,11 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
             it3p = out;
             it3n = sz[3];
           }
-          if (p == 3 && filt && sz[3]) {  // keep only the level-3 nodes whose own list meets F
+          const bool unf = p == 3 && filt && sharing && A.fsplit && sz[3] > kFSplitMin;  // shared unfiltered
+          if (p == 3 && filt && sz[3] && !unf) {  // keep only the level-3 nodes whose own list meets F
             __syncwarp();
             int32_t *dst = reuse3 ? ibuf : out;
-            it3n = filter_level3(A, P.lv[4].bview[P.lv[4].f3], out, sz[3], dst, fset, nF1, nF, acc, lane);
+            it3n = filter_level3(A, P.lv[4].bview[P.lv[4].f3], out, sz[3], dst, fset, fset2, nF1, nF, acc.s, lane);
             it3p = dst;
             if (!reuse3) sz[3] = it3n;
             x_l3f += it3n;
@@ -1025,30 +1114,41 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
           it[p] = 0;
           lvl = p;
           descend = false;
-          if (p == 3 && sharing && it3n > kSplitMin) {
+          if (p == 3 && sharing && (unf || it3n > kSplitMin)) {
             // share this level-3 set: copy it (and a separate iteration list) to the arena and publish slices of the
-            // iteration list as tasks
-            const bool sep = it3p != out;
-            const uint32_t n3 = sz[3], ni = it3n, nt = (ni + kTaskSize - 1) / kTaskSize;
+            // iteration list as tasks (unf: slices of the unfiltered set, each filtered by its taker)
+            const bool sep = !unf && it3p != out;
+            const uint32_t tsz = unf ? kFTaskSize : kTaskSize;
+            const uint32_t n3 = sz[3], ni = it3n, nt = (ni + tsz - 1) / tsz;
+            const uint32_t nH = hset ? hn : 0, nFx = filt ? nF : 0;  // the entry's H and F go with the set
+            const unsigned long long need = (unsigned long long)n3 + (sep ? ni : 0) + nH + nFx;
             unsigned long long off = 0, t0 = 0;
             if (lane == 0) {
-              off = atomicAdd(&A.cnt[CNT_ARENA], (unsigned long long)(n3 + (sep ? ni : 0)));
+              off = atomicAdd(&A.cnt[CNT_ARENA], need);
               t0 = atomicAdd(&A.cnt[CNT_TAIL], (unsigned long long)nt);
             }
             off = __shfl_sync(kFull, off, 0);
             t0 = __shfl_sync(kFull, t0, 0);
-            if (off + n3 + (sep ? ni : 0) <= A.arena_cap && t0 + nt <= A.task_cap) {
+            const unsigned long long xoff = off + n3 + (sep ? ni : 0);
+            if (off + need <= A.arena_cap && t0 + nt <= A.task_cap) {
               for (uint32_t i = lane; i < n3; i += 32) A.arena[off + i] = out[i];
               if (sep)
                 for (uint32_t i = lane; i < ni; i += 32) A.arena[off + n3 + i] = it3p[i];
+              for (uint32_t i = lane; i < nH; i += 32) A.arena[xoff + i] = hset[i];
+              for (uint32_t i = lane; i < nFx; i += 32) A.arena[xoff + nH + i] = i < nF1 ? fset[i] : fset2[i - nF1];
               for (uint32_t t = lane; t < nt; t += 32) {
                 Task q;
                 q.e = e;
                 q.off = off;
                 q.n = n3;
-                q.lo = t * kTaskSize;
-                q.hi = min(ni, (t + 1) * kTaskSize);
-                q.pad = sep ? ni + 1 : 0;
+                q.lo = t * tsz;
+                q.hi = min(ni, (t + 1) * tsz);
+                q.pad = unf ? kTaskFilter : (sep ? ni + 1 : 0);
+                q.xoff = xoff;
+                q.hn = nH;
+                q.nF1 = filt ? nF1 : 0;
+                q.nF = nFx;
+                q.pad2 = 0;
                 A.tasks[t0 + t] = q;
               }
               __threadfence();
@@ -1066,6 +1166,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
                   q.n = 0;
                   q.lo = q.hi = 0;
                   q.pad = 0;
+                  q.xoff = ~0ull;
+                  q.hn = q.nF1 = q.nF = q.pad2 = 0;
                   A.tasks[t0 + t] = q;
                 }
               }
@@ -1090,6 +1192,12 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const MatchAr
   }
   flush(A, acc, lane);
   if (lane == 0) {
+    const long long t_all = clock64() - t_start;
+    if (!t_ph1) t_ph1 = t_all;
+    atomicAdd(&A.cnt[CNT_XT + 0], (unsigned long long)t_ph1);
+    atomicMax(&A.cnt[CNT_XT + 1], (unsigned long long)t_ph1);
+    atomicMax(&A.cnt[CNT_XT + 2], (unsigned long long)t_all);
+    atomicMax(&A.cnt[CNT_XT + 3], (unsigned long long)t_emax);
     atomicAdd(&A.cnt[CNT_X_ENTRIES], x_entries);
     atomicAdd(&A.cnt[CNT_X_PRUNED], x_pruned);
     atomicAdd(&A.cnt[CNT_X_L3], x_l3);
@@ -1192,21 +1300,21 @@ __device__ __forceinline__ LR lr_make(const MatchArgs &A, const int4 r, int xl, 
   const char *c = reinterpret_cast<const char *>(l.m);
   const bool in_ubuf = c >= A.ubuf_lo && c < A.ubuf_hi;
   l.dev = is_hit(A, l.m);
-  if (in_ubuf) acc.delta += 4ull * l.ml;
-  else if (l.dev) acc.hit += 4ull * l.ml;
-  else acc.miss += 4ull * l.ml;
-  acc.delta += 4ull * l.xl;
+  if (in_ubuf) acc.stat(kSDelta, 4ull * l.ml);
+  else if (l.dev) acc.stat(kSHit, 4ull * l.ml);
+  else acc.stat(kSMiss, 4ull * l.ml);
+  acc.stat(kSDelta, 4ull * l.xl);
   return l;
 }
 
 // bulk-copy a zero-copy list when the staging rule of stage_lists says so (drv: always), into the free part of
 // the warp's shared slice, else its HBM staging buffer (out of line: rare, and its copy loop is register-hungry)
-__device__ __noinline__ void stage_slow(LR &L, bool drv, uint32_t d, int32_t *&sm, uint32_t &sm_left, int32_t *&g,
-                                        uint32_t &g_left, int lane, unsigned long long &copied) {
+__device__ __noinline__ uint32_t stage_slow(LR &L, bool drv, uint32_t d, int32_t *&sm, uint32_t &sm_left,
+                                            int32_t *&g, uint32_t &g_left, int lane) {  // returns the bytes copied
   const uint32_t n = L.ml;
   if (!drv) {
     const uint32_t lg = 32u - __clz(n);
-    if (4ull * n > 32ull * d * (lg > 4 ? lg - 3 : 1)) return;
+    if (4ull * n > 32ull * d * (lg > 4 ? lg - 3 : 1)) return 0;
   }
   // a trimmed run starts anywhere: copy from its 16-byte granule (lists are allocated in granules)
   const uint32_t mis = (uint32_t)((reinterpret_cast<uintptr_t>(L.m) >> 2) & 3u);
@@ -1221,19 +1329,19 @@ __device__ __noinline__ void stage_slow(LR &L, bool drv, uint32_t d, int32_t *&s
     g += n4;
     g_left -= n4;
   } else {
-    return;
+    return 0;
   }
   warp_copy(dst, L.m - mis, cn, lane);
   __syncwarp();
-  copied += 4ull * cn;
   L.m = dst + mis;
   L.dev = true;
+  return 4u * cn;
 }
 
 __device__ __forceinline__ void stage_one(LR &L, bool drv, uint32_t d, int32_t *&sm, uint32_t &sm_left,
                                           int32_t *&g, uint32_t &g_left, int lane, Acc &acc) {
   if (L.dev || L.ml < 32) return;
-  stage_slow(L, drv, d, sm, sm_left, g, g_left, lane, acc.copied);
+  acc.stat(kSCopied, stage_slow(L, drv, d, sm, sm_left, g, g_left, lane));
 }
 
 __device__ __noinline__ void copy_list(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
@@ -1286,7 +1394,7 @@ __device__ __forceinline__ bool l4_range(unsigned pk, int32_t a, int32_t b, int3
 constexpr int kL4Meta = 32 * 4;  // int4 per warp: 32 entries x 4
 constexpr int kL4SmemBytes = kSmemBytes + kWarps * kL4Meta * 16 + GCSM_MAXPLANS * 16;
 
-__global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const MatchArgs A) {
+__global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const __grid_constant__ MatchArgs A) {
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   extern __shared__ int4 smem_raw[];
@@ -1304,7 +1412,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
   // work grab: up to GCSM_L4_GRAB entries (rounds of 32), fewer when the frontier would leave warps idle. A run of
   // entries sharing x2 is cut only at grab boundaries, where its zero-copy list is fetched again.
   const int64_t chunk = max((int64_t)1, min((int64_t)GCSM_L4_GRAB, n_f2 / (8 * warps)));
+  __shared__ unsigned long long s_stats[kWarps][kSN];
   Acc acc;
+  acc.init(s_stats[wib], lane);
   unsigned long long d_runs = 0, d_pinb = 0, d_pins = 0, d_split = 0;
   for (;;) {
     unsigned long long g0 = 0;
@@ -1426,13 +1536,13 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
         }
         if (run >= 2 && pin_len >= 32 && cn4 <= GCSM_PIN_SMEM_MAX) {
           copy_list(sm, mp + (lb - mis), cn, lane);
-          if (!pin_hit) acc.copied += 4ull * cn;
+          if (!pin_hit) acc.stat(kSCopied, 4ull * cn);
           pin_p = sm + mis;
           pin_dev = true;
           pin_sm = cn4;
         } else if (run >= 2 && pin_len >= 32 && !pin_hit) {
           copy_list(pstage, mp + (lb - mis), cn, lane);
-          acc.copied += 4ull * cn;
+          acc.stat(kSCopied, 4ull * cn);
           pin_p = pstage + mis;
           pin_dev = true;
         }
@@ -1470,10 +1580,10 @@ __global__ void __launch_bounds__(kBlock, GCSM_L4_MINBLOCKS) k_last4(const Match
           Lc.x = A.dlist + (vw == VIEW_NEW ? xrec.x : xrec.z);
           Lc.xl = (uint32_t)(vw == VIEW_NEW ? xrec.y : xrec.w);
         }
-        if (pin_hit && !pin_peer) acc.hit += 4ull * (uint32_t)xraw.z;  // algorithmic: the whole list
-        else acc.miss += 4ull * (uint32_t)xraw.z;
-        if (pin_peer) acc.peer += 4ull * (uint32_t)xraw.z;
-        acc.delta += 4ull * Lc.xl;
+        if (pin_hit && !pin_peer) acc.stat(kSHit, 4ull * (uint32_t)xraw.z);  // algorithmic: the whole list
+        else acc.stat(kSMiss, 4ull * (uint32_t)xraw.z);
+        if (pin_peer) acc.stat(kSPeer, 4ull * (uint32_t)xraw.z);
+        acc.stat(kSDelta, 4ull * Lc.xl);
       }
       const LR first = (need & 1u) ? La : ((need & 2u) ? Lb : Lc);
       const LR second = (need & 1u) ? ((need & 2u) ? Lb : Lc) : Lc;

@@ -53,7 +53,8 @@ enum Counter {
   CNT_WHIT = 42,
   CNT_WALG = 43,   // per query: algorithmic list bytes its walks read (driver scans + membership probes, §8d)
   CNT_WDBG = 44,   // per query, k_walks work profile (GCSM_TRACE): level-2 roots, lane-walked nodes, DFS descents, steps
-  CNT_N = 48
+  CNT_XT = 48,     // k_extend timing profile (cycles): sum and max of the warps' frontier phase, max warp, max entry
+  CNT_N = 52
 };
 
 struct MatchArgs {
@@ -92,6 +93,7 @@ struct MatchArgs {
   struct Task *tasks;
   int32_t *task_ready;
   uint32_t task_cap;
+  int32_t fsplit;           // k >= 5: share large level-3 sets before the level-3 filter (GCSM_NO_FSPLIT=1: after)
   int32_t task_gen;         // ready-flag value of this launch (no per-launch clearing)
   // fetch-once staging of zero-copy lists within a batch: per vertex state word (epoch << 40 | ready << 39 |
   // offset), the batch arena and its bump counter; nullptr = off
@@ -109,7 +111,8 @@ struct MatchArgs {
   // batch; a zero-copy miss whose list a peer holds in HBM is read from there (peer / NVLink) instead
   int32_t npeer;
   const VDesc *peer_vdesc[GCSM_MAX_PEERS];
-  const char *peer_lo[GCSM_MAX_PEERS], *peer_hi[GCSM_MAX_PEERS];
+  const char *peer_lo[GCSM_MAX_PEERS], *peer_hi[GCSM_MAX_PEERS];  // the peer's cache range (its addresses)
+  const char *peer_map[GCSM_MAX_PEERS];  // where that range is mapped here (= peer_lo within one process)
 };
 
 struct Task {
@@ -118,7 +121,11 @@ struct Task {
   uint32_t n;       // set size
   uint32_t lo, hi;  // the slice of positions this task iterates
   uint32_t pad;
+  uint64_t xoff;    // the entry's hoisted last-level set H then its level-3 filter set F, in the arena (computed once
+                    // by the producer: a taker copies them instead of intersecting the entry's lists again)
+  uint32_t hn, nF1, nF, pad2;
 };
+static_assert(sizeof(Task) == 56, "Task is read as 7 x 8 bytes");
 
 // plans live in a per-context device buffer (contexts may run concurrently)
 cudaError_t upload_plans(DevPlan *dst, const DevPlan *plans, int n, cudaStream_t s);

@@ -57,9 +57,25 @@ __device__ __forceinline__ unsigned long long stage_word(const unsigned long lon
   return v;
 }
 
-__device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v, const int32_t *hp, uint32_t ml,
-                                                   unsigned long long &sfill, unsigned long long &slists,
-                                                   unsigned long long &shit, int lane) {
+// Outcome of a fetch-once lookup: where the list is read from and how (kStZc: zero-copy, no room this batch;
+// kStServed: an arena copy made by someone else; kStFilled: this warp copied it). Returned by value so that the
+// callers' byte counters stay in registers (a reference argument of an out-of-line call would pin them to local
+// memory).
+enum : uint32_t { kStZc = 0, kStServed = 1, kStFilled = 2 };
+struct StageRes {
+  const int32_t *p;
+  uint32_t how;
+};
+__device__ __forceinline__ void stage_count(const StageRes &r, uint32_t ml, unsigned long long &sfill,
+                                            unsigned long long &slists, unsigned long long &shit) {
+  if (r.how == kStFilled) {
+    sfill += 4ull * ml;
+    slists += 1;
+  } else if (r.how == kStServed) {
+    shit += 4ull * ml;
+  }
+}
+__device__ __noinline__ StageRes stage_fetch(const StageRef &A, int32_t v, const int32_t *hp, uint32_t ml, int lane) {
   const unsigned long long ep = (unsigned long long)A.epoch << 40;
   unsigned long long res = 0;
   int claimed = 0;
@@ -105,14 +121,11 @@ __device__ __noinline__ const int32_t *stage_fetch(const StageRef &A, int32_t v,
     __syncwarp();
     __threadfence();  // release: the copy before the state word
     if (lane == 0) atomicExch(A.state + v, ep | kStReady | res);
-    sfill += 4ull * ml;
-    slists += 1;
-    return dst;
+    return StageRes{dst, kStFilled};
   }
   __syncwarp();
-  if (res == kStOff) return hp;
-  shit += 4ull * ml;
-  return A.arena + res;
+  if (res == kStOff) return StageRes{hp, kStZc};
+  return StageRes{A.arena + res, kStServed};
 }
 
 }  // namespace

@@ -209,7 +209,8 @@ std::string HostStore::init_shared(int32_t n_, const int64_t *rp, const int32_t 
   hd.off_lst = off; off = align_up(off + 8ull * n, 4096);
   hd.off_len = off; off = align_up(off + 4ull * n, 4096);
   hd.off_cap = off; off = align_up(off + 4ull * n, 4096);
-  hd.off_lab = off; off = align_up(off + (labels ? 2ull * n : 0), pg);
+  hd.off_lab = off; off = align_up(off + (labels ? 2ull * n : 0), 4096);
+  hd.off_mail = off; off = align_up(off + kShmMailBytes * (uint64_t)store_world, pg);
   for (int sl = 0; sl < 2; ++sl) { hd.off_ovl[sl] = off; off += ovl_b; }
   hd.ovl_bytes = ovl_b;
   hd.off_lists = off; off = align_up(off + lists_b, pg);
@@ -241,6 +242,7 @@ std::string HostStore::init_shared(int32_t n_, const int64_t *rp, const int32_t 
   h.leader_pid = (int32_t)getpid();
   h.fd = fd;  // kept open for the leader's lifetime: the other ranks open /proc/<pid>/fd/<fd>
   h.off_lst = hd.off_lst; h.off_len = hd.off_len; h.off_cap = hd.off_cap; h.off_lab = hd.off_lab;
+  h.off_mail = hd.off_mail;
   h.off_ovl[0] = hd.off_ovl[0]; h.off_ovl[1] = hd.off_ovl[1]; h.ovl_bytes = ovl_b; h.off_lists = hd.off_lists;
   for (int r = 0; r < store_world; ++r) {
     h.reg_lo[r] = hd.reg_lo[r];

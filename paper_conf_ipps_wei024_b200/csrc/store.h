@@ -30,6 +30,7 @@ struct Chunk {
 };
 
 #define GCSM_MAX_STORE_RANKS 16
+constexpr uint64_t kShmMailBytes = 4096;
 
 // Node-shared store ("one shared shm arena cudaHostRegister'ed in each process"): one memfd mapping at
 // the same virtual address in every local rank, so the list pointers in the shared per-vertex metadata are valid
@@ -41,6 +42,7 @@ struct ShmHeader {
   int32_t n, ncap, world, labelled;
   int32_t leader_pid, fd;
   uint64_t off_lst, off_len, off_cap, off_lab, off_ovl[2], ovl_bytes, off_lists;
+  uint64_t off_mail;  // per-rank mailboxes (kShmMailBytes each): the peer-cache IPC handles and per-batch state
   uint64_t reg_lo[GCSM_MAX_STORE_RANKS], reg_hi[GCSM_MAX_STORE_RANKS];
   std::atomic<uint64_t> reg_used[GCSM_MAX_STORE_RANKS];
   std::atomic<uint32_t> attached;
@@ -67,6 +69,9 @@ class HostStore {
   int store_rank() const { return srank_; }
   int store_world() const { return sworld_; }
   bool owned(int32_t x) const { return !shm_ || x % sworld_ == srank_; }
+  void *mailbox(int rank) const {  // rank's kShmMailBytes-byte mailbox in the shared mapping (shared store only)
+    return shm_ ? (char *)shm_ + shm_->off_mail + (uint64_t)rank * kShmMailBytes : nullptr;
+  }
   // process-shared barrier of the store's ranks (no-op for a private store); false: timeout or a failed rank
   bool barrier();
   void poison_shared();

@@ -413,7 +413,7 @@ def test_gpu_walker_btrd_range(G, name, M):
     h.close()
 
 
-@pytest.mark.parametrize("name", ["prism6", "k4tri6", "wheel7"])
+@pytest.mark.parametrize("name", ["house5u", "prism6", "k4tri6", "wheel7"])
 def test_walk_lane_path_equals_warp_dfs(G, name, monkeypatch):
     """Product-internal: the level k-3 walk nodes walked one per lane (walk_leaf_parent, default) record exactly the
     sums of the warp-wide DFS (GCSM_WALK_LANE=0) on a C4-shaped planted graph. M is chosen so that level k-3 nodes

@@ -164,7 +164,7 @@ def test_libgcsm_world2_gloo():
     assert any(any(a or r for a, r in b) for b in res[0][2]) and any(any(a or r for a, r in b) for b in res[1][2])
 
 
-def _shared_worker(rank, world, port, out_q, pipelined):
+def _shared_worker(rank, world, port, out_q, pipelined, link=False):
     """One rank of an emulated world on cuda:0 over ONE node-shared host store (gcsm_options.store_*): rank 0
     builds the store from the CSR, the others attach by handle (no CSR of their own); per-rank shard counts are
     summed over gloo; every rank exports G_{t+1} from the shared store at the end."""
@@ -196,11 +196,14 @@ def _shared_worker(rank, world, port, out_q, pipelined):
             k, qe, ql = gi.query(q)
             (g.set_query if i == 0 else g.add_query)(k, qe, ql)
         g.set_cache_budget(w.adj_bytes // 10)
-        mine = []
+        if link:
+            g.link_store_peers()
+        mine, peer = [], []
 
         def collect():
             g.wait_batch()
             mine.append([g.query_counts(i) for i in range(len(queries))])
+            peer.append(sum(g.query_stats(i)["peer_bytes"] for i in range(len(queries))))
 
         for b, (ins, dele) in enumerate(w.batches):
             if pipelined:
@@ -210,6 +213,7 @@ def _shared_worker(rank, world, port, out_q, pipelined):
             else:
                 g.apply_batch(ins, dele)
                 mine.append([g.query_counts(i) for i in range(len(queries))])
+                peer.append(sum(g.query_stats(i)["peer_bytes"] for i in range(len(queries))))
         if pipelined:
             collect()
         got = []
@@ -228,18 +232,21 @@ def _shared_worker(rank, world, port, out_q, pipelined):
                 I, D, _ = oracle.normalize_batch(w.n, rp, col, ins, dele)
                 rp, col = oracle.apply_batch(w.n, rp, col, I, D)
             rp_w, col_w = rp, col
-        out_q.put((rank, got, mine, want, rp_f, col_f, rp_w, col_w))
+        out_q.put((rank, got, mine, want, rp_f, col_f, rp_w, col_w, sum(peer)))
     finally:
         dist.destroy_process_group()
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("world,pipelined", [(2, False), (3, True)])
-def test_shared_store_world_gloo(world, pipelined):
+@pytest.mark.parametrize("world,pipelined,link", [(2, False, False), (3, True, False), (2, True, True),
+                                                  (3, False, True)])
+def test_shared_store_world_gloo(world, pipelined, link):
     """Node-shared host store: R processes on cuda:0, ONE pinned store created by rank 0
     and attached by the others; each rank writes the overlays / merges of the updated vertices it owns. Shard counts
     summed over gloo equal the oracle on every batch and query, and every rank exports the oracle's final graph
-    from the shared store (so the owner-partitioned merges composed into G_{t+1})."""
+    from the shared store (so the owner-partitioned merges composed into G_{t+1}). With `link` the ranks also read
+    each other's HBM caches through CUDA IPC (gcsm_link_store_peers, NEXT-3 across processes): counts unchanged and
+    some list bytes served by a peer."""
     if not torch.cuda.is_available():
         pytest.skip("needs a GPU")
     import __graft_entry__
@@ -247,7 +254,7 @@ def test_shared_store_world_gloo(world, pipelined):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_shared_worker, args=(r, world, port, q, pipelined)) for r in range(world)]
+    procs = [ctx.Process(target=_shared_worker, args=(r, world, port, q, pipelined, link)) for r in range(world)]
     for p in procs:
         p.start()
     res = sorted([q.get(timeout=600) for _ in range(world)], key=lambda x: x[0])
@@ -255,7 +262,9 @@ def test_shared_store_world_gloo(world, pipelined):
         p.join(timeout=60)
         assert p.exitcode == 0
     want, rp_w, col_w = res[0][3], res[0][6], res[0][7]
-    for rank, got, mine, _, rp_f, col_f, _, _ in res:
+    for rank, got, mine, _, rp_f, col_f, _, _, _ in res:
         assert got == want
         assert np.array_equal(rp_f, rp_w) and np.array_equal(col_f, col_w)
         assert any(any(a or r for a, r in b) for b in mine)
+    peer_bytes = sum(x[8] for x in res)
+    assert (peer_bytes > 0) if link else (peer_bytes == 0)
