@@ -1824,6 +1824,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   A.filter3 = std::getenv("GCSM_NO_FILTER3") ? 0 : 1;
   A.hoist = std::getenv("GCSM_NO_HOIST") ? 0 : 1;
   A.fsplit = std::getenv("GCSM_NO_FSPLIT") ? 0 : 1;
+  A.merge2 = std::getenv("GCSM_MERGE2") ? 1 : 0;  // measured no faster on C3 / C4 (profiles/ab9_r02.txt)
   A.npeer = npeer + snpeer;
   for (int p = 0; p < npeer; ++p) {  // same process: the peer's addresses are ours
     const gcsm_ctx::Slot &ps = peer_of[p]->slots[ctx->batch_seq & 1];
@@ -2086,6 +2087,10 @@ static gcsm_status wait_impl(gcsm_ctx *ctx, uint64_t *added, uint64_t *removed) 
       std::fprintf(stderr, "[gcsm ext-time] q=%d warps=%d ph1_mean_ms=%.2f ph1_max_ms=%.2f warp_max_ms=%.2f entry_max_ms=%.3f\n",
                    qi, ctx->warps_total, h[CNT_XT] / (double)ctx->warps_total / 1.965e6, h[CNT_XT + 1] / 1.965e6,
                    h[CNT_XT + 2] / 1.965e6, h[CNT_XT + 3] / 1.965e6);
+    if (std::getenv("GCSM_TRACE"))
+      std::fprintf(stderr, "[gcsm ext-phase] q=%d max_ms hoist=%.3f F=%.3f l3set=%.3f filter=%.3f rest=%.3f\n", qi,
+                   h[CNT_XT + 4] / 1.965e6, h[CNT_XT + 5] / 1.965e6, h[CNT_XT + 6] / 1.965e6, h[CNT_XT + 7] / 1.965e6,
+                   h[CNT_XT + 8] / 1.965e6);
     if (std::getenv("GCSM_TRACE"))
       std::fprintf(stderr, "[gcsm walks] q=%d roots=%llu lane_nodes=%llu dfs_descents=%llu steps=%llu walg_gb=%.3f\n", qi,
                    h[CNT_WDBG], h[CNT_WDBG + 1], h[CNT_WDBG + 2], h[CNT_WDBG + 3], h[CNT_WALG] / 1e9);

@@ -218,6 +218,79 @@ __device__ __forceinline__ bool contains(const LRef &L, int32_t v) {
   return bsearch_has(L.m, L.ml, v) || (L.xl != 0 && bsearch_has(L.x, L.xl, v));
 }
 
+__device__ __forceinline__ uint32_t lb_idx(const int32_t *a, uint32_t n, int32_t v) {  // first i with a[i] >= v
+  uint32_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (a[mid] < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// Two-list intersection by merge path (both lists device-resident, single sorted runs): the warp splits the merged
+// sequence a ∪ b into 32 diagonal ranges (co-rank search) and each lane merges its own, O((na + nb) / 32) steps
+// instead of ceil(na / 32) rounds of log2(nb)-step binary searches — what a hub entry needs when its lists have
+// comparable lengths (C4: one warp intersecting two lists of 10^4-10^5 elements took up to 20 ms by binary search).
+// MATERIALIZE: a count pass, an exclusive warp scan of the lanes' counts, and a writing pass keep the output
+// sorted. Same survivors as warp_isect (range, exclusions, label).
+template <bool MATERIALIZE>
+__device__ GCSM_COLD uint32_t merge_isect(const MatchArgs &A, const int32_t *a, uint32_t na, const int32_t *b,
+                                          uint32_t nb, const int32_t *excl, int nexcl, int label, int32_t *out,
+                                          int lane, int32_t vlo, int32_t vhi) {
+  if (vlo != INT_MIN) {
+    const uint32_t ua = lb_idx(a, na, vlo + 1), ub = lb_idx(b, nb, vlo + 1);
+    a += ua;
+    na -= ua;
+    b += ub;
+    nb -= ub;
+  }
+  if (vhi != INT_MAX) {
+    na = lb_idx(a, na, vhi);
+    nb = lb_idx(b, nb, vhi);
+  }
+  const uint32_t T = na + nb;
+  const uint32_t d0 = (uint32_t)(((uint64_t)T * (uint32_t)lane) >> 5);
+  const uint32_t d1 = (uint32_t)(((uint64_t)T * (uint32_t)(lane + 1)) >> 5);
+  uint32_t lo = d0 > nb ? d0 - nb : 0, hi = d0 < na ? d0 : na;
+  while (lo < hi) {
+    const uint32_t i = (lo + hi) >> 1;
+    if (a[i] <= b[d0 - i - 1]) lo = i + 1;
+    else hi = i;
+  }
+  const uint32_t i0 = lo, j0 = d0 - lo;
+  auto pass = [&](bool write, uint32_t base) -> uint32_t {
+    uint32_t i = i0, j = j0, c = 0;
+    while (i + j < d1) {
+      const int32_t ai = i < na ? a[i] : INT_MAX;
+      const int32_t bj = j < nb ? b[j] : INT_MAX;
+      const bool le = ai <= bj, ge = ai >= bj;
+      if (le && ge) {
+        bool ok = true;
+        for (int e = 0; e < nexcl; ++e) ok = ok && ai != excl[e];
+        if (ok && label >= 0) ok = A.lab[ai] == (uint16_t)label;
+        if (ok) {
+          if (write) out[base + c] = ai;
+          ++c;
+        }
+      }
+      i += le;
+      j += ge;
+    }
+    return c;
+  };
+  const uint32_t c = pass(false, 0);
+  uint32_t incl = c;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFull, incl, o);
+    if (lane >= o) incl += y;
+  }
+  const uint32_t total = __shfl_sync(kFull, incl, 31);
+  if (MATERIALIZE && total) pass(true, incl - c);
+  return total;
+}
+
 // Warp-cooperative intersection. Driver: the device set dset[0..dn) if dset
 // != nullptr (code motion; then every L[] is a probe), else L[drv] (main then
 // delta segment; L[drv] is not probed). A driver element v survives if it is
@@ -228,6 +301,15 @@ template <bool MATERIALIZE>
 __device__ GCSM_COLD uint32_t warp_isect(const MatchArgs &A, const int32_t *dset, uint32_t dn, const LRef *L,
                                                int nl, int drv, const int32_t *excl, int nexcl, int label,
                                                int32_t *out, int lane, int32_t vlo = INT_MIN, int32_t vhi = INT_MAX) {
+  if (!dset && nl == 2 && A.merge2 && L[0].dev && L[1].dev && L[0].xl == 0 && L[1].xl == 0 && L[0].ml && L[1].ml) {
+    // two single-run device-resident lists: merge path when cheaper than lane-parallel binary searches
+    const uint32_t d = L[drv].ml, big = L[1 - drv].ml;
+    const uint32_t lg = 31u - __clz(big | 1u);
+    const uint64_t bs_cost = (uint64_t)((d + 31) >> 5) * (7 * lg + 12);
+    const uint64_t mg_cost = (MATERIALIZE ? 2ull : 1ull) * (7ull * ((d + big + 31) >> 5)) + 10ull * lg + 40;
+    if (mg_cost < bs_cost)
+      return merge_isect<MATERIALIZE>(A, L[0].m, L[0].ml, L[1].m, L[1].ml, excl, nexcl, label, out, lane, vlo, vhi);
+  }
   const int32_t *s0, *s1;
   uint32_t n0, n1;
   if (dset) {
@@ -756,6 +838,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
   const bool sharing = KK == 0 && !LIST && k >= 5 && A.tasks != nullptr;
   const long long t_start = clock64();
   long long t_ph1 = 0, t_entry = 0, t_emax = 0;  // timing profile (CNT_XT)
+  long long tp[5] = {0, 0, 0, 0, 0}, tpm[5] = {0, 0, 0, 0, 0};  // this entry's phases / the warp's maxima:
+                                                                  // hoist, F, level-3 set, filter, rest
   for (;;) {
     int64_t e;
     bool task = false;
@@ -888,7 +972,18 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
     }
     {
       const long long now = clock64();
-      if (t_entry) t_emax = max(t_emax, now - t_entry);
+      if (t_entry) {
+        t_emax = max(t_emax, now - t_entry);
+        long long rest = now - t_entry;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          tpm[i] = max(tpm[i], tp[i]);
+          rest -= tp[i];
+        }
+        tpm[4] = max(tpm[4], rest);
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) tp[i] = 0;
       t_entry = now;
     }
     const int32_t ui = f2u[e];
@@ -933,9 +1028,11 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
         hset = Lx[0].m;
         hn = Lx[0].ml;
       } else {
+        const long long t0 = clock64();
         hn = warp_isect<true>(A, nullptr, 0, Lx, nx, hdrv, nullptr, 0, Lh.label, hbuf, lane);
         __syncwarp();
         hset = hbuf;
+        tp[0] += clock64() - t0;
       }
       if (hn == 0) {  // no candidate for the last position anywhere below this entry
         ++x_pruned;
@@ -975,6 +1072,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
         nF = dfull.ml + dfull.xl;
       } else {
       Lx[fdrv].xl = 0;
+      const long long t0 = clock64();
       nF1 = warp_isect<true>(A, nullptr, 0, Lx, nx, fdrv, nullptr, 0, L4.label, fbuf, lane);
       __syncwarp();
       nF = nF1;
@@ -986,6 +1084,7 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
         nF += warp_isect<true>(A, nullptr, 0, Lx, nx, fdrv, nullptr, 0, L4.label, fbuf + nF1, lane);
         __syncwarp();
       }
+      tp[1] += clock64() - t0;
       }
       if (nF == 0) {  // no position-4 candidate for any level-3 node of this entry
         ++x_pruned;
@@ -1005,7 +1104,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
       for (uint32_t i = lane; i < cnt; i += 32) own[i] = __ldcg(A.arena + tk.off + lo + i);
       __syncwarp();
       const int32_t *slice = reuse3 ? own + tk.lo : own;
+      const long long tf = clock64();
       it3n = filter_level3(A, P.lv[4].bview[P.lv[4].f3], slice, tk.hi - tk.lo, ibuf, fset, fset2, nF1, nF, acc.s, lane);
+      tp[3] += clock64() - tf;
       x_l3f += it3n;
       it3p = ibuf;
       __syncwarp();
@@ -1093,7 +1194,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
           descend = false;
         } else {
           int32_t *out = stack + (int64_t)(p - 3) * A.dcap;
+          const long long t3 = clock64();
           sz[p] = warp_isect<true>(A, dset, dn, L, nl, drv, excl, nex, Lp.label, out, lane, vlo, vhi);
+          if (p == 3) tp[2] += clock64() - t3;
           if (p == 3) x_l3 += sz[p];
           else if (p == 4) x_l4 += sz[p];
           if (p == 3) {
@@ -1104,7 +1207,9 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
           if (p == 3 && filt && sz[3] && !unf) {  // keep only the level-3 nodes whose own list meets F
             __syncwarp();
             int32_t *dst = reuse3 ? ibuf : out;
+            const long long tf = clock64();
             it3n = filter_level3(A, P.lv[4].bview[P.lv[4].f3], out, sz[3], dst, fset, fset2, nF1, nF, acc.s, lane);
+            tp[3] += clock64() - tf;
             it3p = dst;
             if (!reuse3) sz[3] = it3n;
             x_l3f += it3n;
@@ -1198,6 +1303,8 @@ __global__ void __launch_bounds__(kBlock, GCSM_MINBLOCKS) k_extend(const __grid_
     atomicMax(&A.cnt[CNT_XT + 1], (unsigned long long)t_ph1);
     atomicMax(&A.cnt[CNT_XT + 2], (unsigned long long)t_all);
     atomicMax(&A.cnt[CNT_XT + 3], (unsigned long long)t_emax);
+#pragma unroll
+    for (int i = 0; i < 5; ++i) atomicMax(&A.cnt[CNT_XT + 4 + i], (unsigned long long)tpm[i]);
     atomicAdd(&A.cnt[CNT_X_ENTRIES], x_entries);
     atomicAdd(&A.cnt[CNT_X_PRUNED], x_pruned);
     atomicAdd(&A.cnt[CNT_X_L3], x_l3);

@@ -53,8 +53,9 @@ enum Counter {
   CNT_WHIT = 42,
   CNT_WALG = 43,   // per query: algorithmic list bytes its walks read (driver scans + membership probes, §8d)
   CNT_WDBG = 44,   // per query, k_walks work profile (GCSM_TRACE): level-2 roots, lane-walked nodes, DFS descents, steps
-  CNT_XT = 48,     // k_extend timing profile (cycles): sum and max of the warps' frontier phase, max warp, max entry
-  CNT_N = 52
+  CNT_XT = 48,     // k_extend timing profile (cycles): sum and max of the warps' frontier phase, max warp, max entry,
+                   // then the largest single-entry time of each phase (hoist, F, level-3 set, filter, rest)
+  CNT_N = 57
 };
 
 struct MatchArgs {
@@ -93,7 +94,9 @@ struct MatchArgs {
   struct Task *tasks;
   int32_t *task_ready;
   uint32_t task_cap;
-  int32_t fsplit;           // k >= 5: share large level-3 sets before the level-3 filter (GCSM_NO_FSPLIT=1: after)
+  int32_t fsplit;
+  int32_t merge2;           // two-list materialising intersections by merge path when cheaper (GCSM_MERGE2=1; off:
+                            // measured no faster, profiles/ab9_r02.txt)           // k >= 5: share large level-3 sets before the level-3 filter (GCSM_NO_FSPLIT=1: after)
   int32_t task_gen;         // ready-flag value of this launch (no per-launch clearing)
   // fetch-once staging of zero-copy lists within a batch: per vertex state word (epoch << 40 | ready << 39 |
   // offset), the batch arena and its bump counter; nullptr = off
