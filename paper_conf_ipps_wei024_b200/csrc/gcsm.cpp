@@ -190,7 +190,8 @@ struct gcsm_ctx {
   // copy) runs here while batch t's extension kernels run on `stream` (GCSM_NO_OVERLAP=1 at create: on `stream`)
   cudaStream_t stream3 = nullptr;
   bool overlap = false;
-  int overlap_kmax = 5;  // largest query size whose batches overlap the cache step (GCSM_OVERLAP_KMAX)
+  int overlap_kmax = 8;  // largest query size whose batches overlap the cache step (GCSM_OVERLAP_KMAX; C4 A/B:
+                         // 100.4-100.8 ms per step with the overlap, 101.3-103.0 without, profiles/ab10_r02.txt)
   uint32_t *d_hist = nullptr;                         // n counters + scan
   uint32_t *d_bsum = nullptr;
   int32_t *d_scratch = nullptr; size_t scratch_cap = 0;
@@ -1582,7 +1583,7 @@ static gcsm_status submit_impl(gcsm_ctx *ctx, int64_t n_ins, const int32_t *ins,
   // the cache step's stream: with overlap it runs beside the previous batch's matching (it writes only this slot's
   // descriptors, delta records, units and counters and the other cache buffer; the previous use of this slot was
   // batch t-2, already collected by gcsm_wait_batch)
-  // (not with a query larger than overlap_kmax, default 5: a 6-vertex query's level->=2 walks read zero-copy lists
+  // (not with a query larger than overlap_kmax, default 8 since the late round-2 kernels; it was 5 while a 6-vertex query's level->=2 walks read zero-copy lists
   // and contend for the host link with the extension kernels they would run beside; GCSM_OVERLAP_KMAX
   // at create moves the limit)
   // Invariant of the overlapped step: k_sidx_update (in the cache step of t+1) rewrites the sampled index of batch

@@ -86,6 +86,10 @@ constexpr uint32_t kSplitMin = GCSM_SPLIT_MIN;  // level-3 sets larger than this
 // takers filter themselves (the filter, one lane per node, is the heavy part of a hub entry)
 constexpr uint32_t kFSplitMin = GCSM_FSPLIT_MIN, kFTaskSize = GCSM_FTASK_SIZE;
 constexpr uint32_t kTaskFilter = 0xffffffffu;  // Task::pad: the slice is unfiltered
+#ifndef GCSM_FILT_LANE
+#define GCSM_FILT_LANE 128
+#endif
+constexpr uint32_t kFiltLane = GCSM_FILT_LANE;  // level-3 filter: larger per-node tests run warp-wide
 constexpr uint32_t kTaskSize = GCSM_TASK_SIZE;  // level-3 candidates per task
 
 struct LRef {
@@ -692,6 +696,32 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
   return x;
 }
 
+// Do the sorted runs a[0..na) and b[0..nb) share an element? Merge path over the warp (co-rank split, each lane
+// merges its diagonal range): O((na + nb) / 32) steps, for two long device-resident runs whose lane-parallel
+// binary-search test would take min(na, nb) / 32 rounds of log2 steps (the level-3 filter of a C4 hub node).
+__device__ __forceinline__ bool merge_meet(const int32_t *a, uint32_t na, const int32_t *b, uint32_t nb, int lane) {
+  const uint32_t T = na + nb;
+  const uint32_t d0 = (uint32_t)(((uint64_t)T * (uint32_t)lane) >> 5);
+  const uint32_t d1 = (uint32_t)(((uint64_t)T * (uint32_t)(lane + 1)) >> 5);
+  uint32_t lo = d0 > nb ? d0 - nb : 0, hi = d0 < na ? d0 : na;
+  while (lo < hi) {
+    const uint32_t i = (lo + hi) >> 1;
+    if (a[i] <= b[d0 - i - 1]) lo = i + 1;
+    else hi = i;
+  }
+  uint32_t i = lo, j = d0 - lo;
+  bool hit = false;
+  // one step past the range as well: an equal pair split across two lanes' ranges is seen by the earlier lane
+  while (i + j <= d1 && !hit) {
+    const int32_t ai = i < na ? a[i] : INT_MAX;
+    const int32_t bj = j < nb ? b[j] : INT_MAX;
+    if (ai == bj && ai != INT_MAX) hit = true;
+    i += ai <= bj;
+    j += ai >= bj;
+  }
+  return __any_sync(kFull, hit);
+}
+
 // Level-3 filter (LevelPlan::fmask): position 4's candidates for a level-3 node x3 lie in
 // F ∩ view(N(x3)), where F = F[0..nF1) ∪ F2[0..nF-nF1) (two sorted runs, label-filtered) is the intersection of position 4's lists fixed for the whole
 // level-2 entry. Lane i tests node i: does its own list meet F? Nodes that cannot (almost all of them on C4) are
@@ -760,9 +790,12 @@ __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const
       if (lane == l) m = q;
     }
     bool hit = false;
-    if (act) {
+    const uint32_t nF2 = nF - nF1;
+    // a node whose test streams more than kFiltLane elements is tested by the whole warp below (one lane alone took
+    // up to 20 ms on a C4 hub node: profiles/c4_trace_r02_v7.txt)
+    const bool big = act && min(ml + xl, nF) > kFiltLane;
+    if (act && !big) {
       if (ml + xl <= nF) {  // stream the node's list, probe F (its two sorted runs)
-        const uint32_t nF2 = nF - nF1;
         for (uint32_t j = 0; j < ml && !hit; ++j) hit = bsearch_has(F, nF1, m[j]) || (nF2 && bsearch_has(F2, nF2, m[j]));
         for (uint32_t j = 0; j < xl && !hit; ++j) hit = bsearch_has(F, nF1, x[j]) || (nF2 && bsearch_has(F2, nF2, x[j]));
       } else {  // stream F, probe the node's list
@@ -771,6 +804,53 @@ __device__ __noinline__ uint32_t filter_level3(const MatchArgs &A, int vw, const
           hit = bsearch_has(m, ml, fj) || (xl && bsearch_has(x, xl, fj));
         }
       }
+    }
+    for (unsigned bgm = __ballot_sync(kFull, big); bgm; bgm &= bgm - 1) {  // warp-wide tests, early exit on a hit
+      const int l = __ffs(bgm) - 1;
+      const int32_t *bm_ = reinterpret_cast<const int32_t *>(__shfl_sync(kFull, (unsigned long long)m, l));
+      const int32_t *bx = reinterpret_cast<const int32_t *>(__shfl_sync(kFull, (unsigned long long)x, l));
+      const uint32_t bml = __shfl_sync(kFull, ml, l), bxl = __shfl_sync(kFull, xl, l);
+      bool found = false;
+      const char *pc = reinterpret_cast<const char *>(bm_);
+      const bool bdev = (pc >= A.cache_lo && pc < A.cache_hi) || (pc >= A.ubuf_lo && pc < A.ubuf_hi) ||
+                        (A.stage_arena && bm_ >= A.stage_arena && bm_ < A.stage_arena + A.stage_cap) ||
+                        (pc >= reinterpret_cast<const char *>(A.scratch) &&
+                         pc < reinterpret_cast<const char *>(A.scratch_end)) || __isShared(bm_);
+      if (bdev && nF1 && bml && (uint64_t)nF1 + bml < 8ull * min(nF1, bml)) {
+        // two long runs: merge path for main x main, lane-parallel probes for the short delta runs
+        found = merge_meet(F, nF1, bm_, bml, lane);
+        for (uint32_t j0 = 0; j0 < bxl && !found; j0 += 32) {
+          const uint32_t j = j0 + lane;
+          const bool h = j < bxl && (bsearch_has(F, nF1, bx[j]) || (nF2 && bsearch_has(F2, nF2, bx[j])));
+          found = __any_sync(kFull, h);
+        }
+        for (uint32_t j0 = 0; j0 < nF2 && !found; j0 += 32) {
+          const uint32_t j = j0 + lane;
+          const bool h = j < nF2 && bsearch_has(bm_, bml, F2[j]);
+          found = __any_sync(kFull, h);
+        }
+      } else if (bml + bxl <= nF) {
+        for (uint32_t j0 = 0; j0 < bml + bxl && !found; j0 += 32) {
+          const uint32_t j = j0 + lane;
+          bool h = false;
+          if (j < bml + bxl) {
+            const int32_t u = j < bml ? bm_[j] : bx[j - bml];
+            h = bsearch_has(F, nF1, u) || (nF2 && bsearch_has(F2, nF2, u));
+          }
+          found = __any_sync(kFull, h);
+        }
+      } else {
+        for (uint32_t j0 = 0; j0 < nF && !found; j0 += 32) {
+          const uint32_t j = j0 + lane;
+          bool h = false;
+          if (j < nF) {
+            const int32_t fj = j < nF1 ? F[j] : F2[j - nF1];
+            h = bsearch_has(bm_, bml, fj) || (bxl && bsearch_has(bx, bxl, fj));
+          }
+          found = __any_sync(kFull, h);
+        }
+      }
+      if (lane == l) hit = found;
     }
     const unsigned hm = __ballot_sync(kFull, hit);
     if (hit) out[w + __popc(hm & ((1u << lane) - 1u))] = v;

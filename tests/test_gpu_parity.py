@@ -240,6 +240,39 @@ def test_c4_shaped_planted(G, name):
     assert got == want
 
 
+@pytest.mark.parametrize("overlap", ["8", "5"])
+def test_c4_shaped_pipelined_multi_query(G, overlap, monkeypatch):
+    """The bench's C4 layout on a C4-shaped graph: ONE context holding prism6 + K4+2tri6 + K6, pipelined
+    submit / wait, 1 % budget; with the cache step of batch t+1 beside the matching of batch t (GCSM_OVERLAP_KMAX=8,
+    the default) and without (5). Every query's counts equal the oracle's on every batch, and the final graph too."""
+    monkeypatch.setenv("GCSM_OVERLAP_KMAX", overlap)
+    w = gi.make_workload("C4", scale=13, n_edges=60_000, batch=256, n_batches=4)
+    names = ["prism6", "k4tri6", "k6"]
+    want = {q: oracle_run(w.n, w.row_ptr, w.col, None, q, w.batches)[0] for q in names}
+    g = G.Gcsm(w.n, w.row_ptr, w.col, device=0)
+    for i, q in enumerate(names):
+        k, qe, ql = gi.query(q)
+        (g.set_query if i == 0 else g.add_query)(k, qe, ql, gi.order(q))
+    g.set_cache_budget(w.adj_bytes // 100)
+    got = {q: [] for q in names}
+
+    def collect():
+        g.wait_batch()
+        for i, q in enumerate(names):
+            got[q].append(g.query_counts(i))
+
+    g.submit_batch(*w.batches[0])
+    for b in w.batches[1:]:
+        g.submit_batch(*b)
+        collect()
+    collect()
+    assert got == want
+    _, (rp1, col1) = oracle_run(w.n, w.row_ptr, w.col, None, "edge", w.batches)
+    rp2, col2 = g.export_csr()
+    assert np.array_equal(rp1, rp2) and np.array_equal(col1, col2)
+    g.close()
+
+
 @pytest.mark.parametrize("r", [1, 2, 3])
 def test_star_closed_form_at_scale(G, r):
     """SURVEY §8c degree closed form for K_{1,r}: added = Σ_U P(d',r) - P(s,r), removed = Σ_U P(d,r) - P(s,r)."""
