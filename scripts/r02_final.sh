@@ -14,3 +14,9 @@ timeout 1200 /usr/local/cuda/bin/ncu --metrics gpu__time_duration.sum --clock-co
 NB=2 QUERIES=prism6 timeout 1500 /usr/local/cuda/bin/ncu --set full --import-source on --clock-control none --kernel-name-base function \
   -k regex:"^(k_extend|k_walks)$" --launch-skip 2 --launch-count 2 -f -o $o/ncu_c4_prism6_final \
   python scripts/c4_ncu.py > $o/final_ncu_full.log 2>&1; echo "exit $?" >> $o/final_ncu_full.log
+out=$o/final_ab_merge2.txt; : > $out
+for v in def merge2 def merge2; do
+  mg=""; [ $v == merge2 ] && mg=1
+  env ${mg:+GCSM_MERGE2=1} timeout 900 python bench.py --quick --steps 8 --warmup 3 --parity-edges 0 2>>$o/final_ab_merge2.err | tail -1 | \
+    python -c "import sys,json; d=json.loads(sys.stdin.read()); print('$v', round(d['value']), round(d['ms_per_step'],2), {q: (round(x['ms_extend'],2), round(x['ms_walks'],2)) for q,x in d['per_query'].items()})" >> $out
+done
