@@ -40,6 +40,31 @@ __device__ __forceinline__ void warp_copy(int32_t *dst, const int32_t *src, uint
   }
 }
 
+#ifndef GCSM_STAGE_DEEP
+#define GCSM_STAGE_DEEP 0
+#endif
+// The arena fill's copy (out of line, in stage_fetch): GCSM_STAGE_DEEP = 1 keeps 8 x 16 B per lane in flight (4 KB
+// per warp) for hub lists crossing PCIe.
+__device__ __forceinline__ void warp_copy_fill(int32_t *dst, const int32_t *src, uint32_t n, int lane) {
+#if GCSM_STAGE_DEEP
+  __syncwarp();
+  const uint32_t n4 = (n + 3) >> 2;
+  const int4 *s4 = reinterpret_cast<const int4 *>(src);
+  int4 *d4 = reinterpret_cast<int4 *>(dst);
+  for (uint32_t base = 0; base < n4; base += 256) {
+    int4 v[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (base + lane + 32 * k < n4) v[k] = s4[base + lane + 32 * k];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (base + lane + 32 * k < n4) d4[base + lane + 32 * k] = v[k];
+  }
+#else
+  warp_copy(dst, src, n, lane);
+#endif
+}
+
 // ---- fetch-once staging of zero-copy lists within a batch -------------------------------------
 // The first warp of the batch that needs vertex v's zero-copy main list claims it (CAS of its state word from an
 // older epoch to "loading"), copies it over PCIe into the batch arena (bump-allocated, 128-byte granules so that
@@ -117,7 +142,7 @@ __device__ __noinline__ StageRes stage_fetch(const StageRef &A, int32_t v, const
   res = __shfl_sync(0xffffffffu, res, 0);
   if (claimed) {
     int32_t *dst = A.arena + res;
-    warp_copy(dst, hp, ml, lane);
+    warp_copy_fill(dst, hp, ml, lane);
     __syncwarp();
     __threadfence();  // release: the copy before the state word
     if (lane == 0) atomicExch(A.state + v, ep | kStReady | res);
